@@ -1,0 +1,215 @@
+/*
+ * cualign_bp.h -- C ABI of the B200-native NetAlignBP + matching engine.
+ *
+ * Method: cuAlign (Xiang, Khan, Ferdous, Aravind, Halappanavar, SC-W 2023),
+ * /root/reference/PAPER.md.  The engine runs the data-parallel hot path of
+ * the paper's Alg. 2 on one B200 (sm_100a):
+ *
+ *   init     a1  canonical L (A-side rows, B-side incidence)
+ *            a2  overlap matrix S (Alg. 3) + its square layout PAPER.md:66, :181, :185-197
+ *   iterate  a3  F = bound_{0,beta}[beta S + S^p'], d = alpha w + F e   (Alg. 2 l.9-10, :162-163)
+ *            a4  y^c = d - othermaxcol(z^p), z^c = d - othermaxrow(y^p) (l.11-12, :164-165, :203)
+ *            a5  S^c = diag(y^c + z^c - d) S - F                        (l.13, :166)
+ *            a6  damping with gamma^p                                   (l.14-16, :167-169)
+ *   round    a7  1/2-approx. locally-dominant matching on y^c and z^c  (l.17-20, :170-173, :207-209)
+ *            a8  evaluate alpha*w(M) + beta*x'Sx/2, keep the best      (l.21-24, :174-177, Eq. 1 :64-72)
+ *
+ * Readings of the paper where it is silent or garbled are listed in DESIGN.md
+ * (Z1-Z27); the ones that change results are selectable through flags.
+ *
+ * Conventions (all functions):
+ *   - Every function returns a cualign_status and never throws; on error a
+ *     human-readable message is available from cualign_last_error()
+ *     (thread-local, valid until the next call on the same thread).
+ *   - Inputs are borrowed for the duration of the call and copied; outputs are
+ *     written to caller-owned buffers; the handle owns all device memory it
+ *     allocates until cualign_bp_free().
+ *   - Pointers are HOST pointers unless CUALIGN_FLAG_DEVICE_PTRS is set in
+ *     cualign_params.flags, in which case the graph / edge arrays given to
+ *     cualign_bp_init are device pointers on params.device.  State / output
+ *     buffers of the get/set functions are always host pointers.
+ *   - cualign_bp_iterate() is asynchronous on params.stream; CUDA errors
+ *     surface at the next synchronising call.  cualign_bp_round() with a
+ *     non-NULL info, every get_* function and cualign_bp_free() synchronise.
+ *   - One handle per host thread; distinct handles are independent.
+ *   - Sizes are int64; vertex ids and edge ids are int32 (m < 2^31), S row
+ *     pointers int64 (nnz(S) may exceed 2^31).
+ */
+#ifndef CUALIGN_BP_H
+#define CUALIGN_BP_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct cualign_bp cualign_bp; /* opaque handle; owns all device state */
+
+typedef enum {
+    CUALIGN_OK = 0,
+    CUALIGN_EINVAL = -1, /* invalid argument / malformed input (message says which) */
+    CUALIGN_ENOMEM = -2, /* device allocation failed */
+    CUALIGN_ECUDA = -3,  /* a CUDA runtime call failed */
+    CUALIGN_ENCCL = -4,  /* an NCCL call failed (sharded handles) */
+    CUALIGN_ESTATE = -5  /* call not valid in the handle's current state */
+} cualign_status;
+
+/* flags (cualign_params.flags) */
+#define CUALIGN_FLAG_DEVICE_PTRS      0x01u /* init arrays are device pointers */
+#define CUALIGN_FLAG_EXACT            0x02u /* oracle-order fp64 sums: row sums of F in ascending f
+                                               from 0.0, matching weight summed in ascending edge id
+                                               (bitwise reproduces the oracle; slow on hub rows) */
+#define CUALIGN_FLAG_OTHERMAX_LITERAL 0x04u /* reading Z4 literal: om(e) = max_{f!=e} v_f (no 0);
+                                               default max-plus: om(e) = max(0, max_{f!=e} v_f) */
+#define CUALIGN_FLAG_ROUND_DAMPED     0x08u /* reading Z5 variant: round y^p, z^p instead of y^c, z^c */
+#define CUALIGN_FLAG_TIMING           0x10u /* record CUDA events around every kernel (diagnostics) */
+
+/* Undirected simple graph: symmetric CSR, row i lists the
+ * neighbours of i strictly increasing, no self loops (reading Z14).
+ * rowptr has n+1 entries, rowptr[0] = 0; col has rowptr[n] entries. */
+typedef struct {
+    int32_t n;
+    const int64_t *rowptr;
+    const int32_t *col;
+} cualign_graph;
+
+/* Candidate bipartite graph L = (V_A u V_B, E_L, w):
+ * m edges (a[k], b[k]) with 0 <= a < n_A, 0 <= b < n_B, strictly increasing in
+ * (a, b) lexicographic order -- the canonical edge id of (a[k], b[k]) is k --
+ * and finite weights w[k]. */
+typedef struct {
+    int64_t m;
+    const int32_t *a;
+    const int32_t *b;
+    const double *w;
+} cualign_edges;
+
+typedef struct {
+    double alpha;     /* >= 0, weight of the matching term of Eq. 1 */
+    double beta;      /* >= 0, weight of the overlap term of Eq. 1 */
+    double gamma;     /* damping base, 0 < gamma <= 1; iteration p damps with
+                         g = gamma^p, h = 1 - g computed on the host in fp64 (Z2) */
+    uint32_t flags;   /* CUALIGN_FLAG_* */
+    int32_t device;   /* CUDA device ordinal */
+    void *stream;     /* cudaStream_t to run on (e.g. torch.cuda.current_stream());
+                         NULL = the handle creates its own non-blocking stream */
+    int32_t rank;     /* reserved for sharded handles; must be 0 */
+    int32_t world;    /* reserved for sharded handles; must be 1 (or 0 = 1) */
+    const void *nccl_unique_id; /* reserved; must be NULL */
+} cualign_params;
+
+/* Result of one rounding step (Alg. 2 l.17-24). */
+typedef struct {
+    int32_t iter;        /* BP iteration p the rounded messages belong to */
+    int32_t source;      /* 0 = M_y chosen, 1 = M_z (M_y wins ties, reading Z8) */
+    int32_t improved;    /* 1 if score > bestScore (strict) and best was replaced */
+    int32_t best_iter;   /* iteration of the best matching so far (0 = none) */
+    int32_t card_y, card_z;       /* |M_y|, |M_z| */
+    double score_y, score_z;      /* alpha*w(M) + beta*overlap(M) */
+    double weight_y, weight_z;    /* sum of the original w over M (reading Z9) */
+    double score;                 /* max(score_y, score_z) */
+    double best_score;            /* bestScore after this round (starts at 0) */
+    int64_t overlap_y, overlap_z; /* x'Sx/2: squares {e,f} with both e, f in M */
+    int32_t rounds_y, rounds_z;   /* pointer rounds the matchings took */
+} cualign_round_info;
+
+/* Sizes of an initialised handle. */
+typedef struct {
+    int32_t n_a, n_b;
+    int64_t m;          /* |E_L| */
+    int64_t s;          /* nnz(S) = 2 * squares */
+    int64_t squares;    /* s / 2 (reading Z18) */
+    int64_t max_row;    /* longest S row */
+    int32_t p;          /* iterations done */
+    int32_t fixed_point_bits; /* fraction bits of the fast-mode F-sum accumulator */
+    int64_t device_bytes;     /* device memory held by the handle */
+} cualign_sizes;
+
+/* Diagnostics: per-kernel-class event timing (needs CUALIGN_FLAG_TIMING) and
+ * launch counts since the last reset. */
+#define CUALIGN_NUM_KERNEL_CLASSES 8
+typedef struct {
+    int64_t launches;                              /* all kernels launched by the handle */
+    int64_t class_launches[CUALIGN_NUM_KERNEL_CLASSES];
+    double class_ms[CUALIGN_NUM_KERNEL_CLASSES];   /* summed event time */
+} cualign_stats;
+/* kernel classes */
+#define CUALIGN_K_TOP2    0 /* a4: per-vertex top-2 of y^p (A rows) and z^p (B columns) */
+#define CUALIGN_K_EDGE    1 /* a3 tail + a4 + a6 on vectors: d, y^c, z^c, u, damping of y, z */
+#define CUALIGN_K_SQUARE  2 /* a3 + a5 + a6 on S values: the square pass (dominant kernel) */
+#define CUALIGN_K_ROWSUM  3 /* exact mode: sequential row sums of F */
+#define CUALIGN_K_MATCH   4 /* a7 + a8: matching on y^c and z^c, evaluate, best */
+#define CUALIGN_K_INIT    5 /* a1 + a2: validation, L layouts, S build */
+#define CUALIGN_K_STATE   6 /* get/set state gathers and scatters */
+#define CUALIGN_K_OTHER   7
+
+/* a1 + a2: validate, copy A, B, L to the device, build L's A-side rows and
+ * B-side incidence, build S (Alg. 3) and its square layout, zero the BP state
+ * (Alg. 2 l.1-7).  n_A = A->n, n_B = B->n (reading Z15:
+ * n_A != n_B allowed).  Validation failures return CUALIGN_EINVAL with a
+ * message: out-of-range ids, unsorted or duplicate L edges, asymmetric graphs,
+ * self loops, unsorted rows, non-finite w, alpha < 0, beta < 0,
+ * gamma outside (0, 1].  On failure *out is set to NULL. */
+cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B,
+                               const cualign_edges *L, const cualign_params *params,
+                               cualign_bp **out);
+
+/* a3-a6: run n_steps iterations of Alg. 2 lines 9-16,
+ * p += n_steps.  Asynchronous on the handle's stream.  n_steps >= 0. */
+cualign_status cualign_bp_iterate(cualign_bp *h, int32_t n_steps);
+
+/* a7-a8: Alg. 2 lines 17-24 on the current y^c, z^c: two matchings, evaluate,
+ * select, best update -- all on the device.  info == NULL: fully asynchronous
+ * (best is tracked on the device); otherwise synchronises and fills *info. */
+cualign_status cualign_bp_round(cualign_bp *h, cualign_round_info *info);
+
+/* Best matching so far: mate_a[a] = canonical id of the L edge matched at A
+ * vertex a, or -1 (host buffer of n_A int32; may be NULL).  info receives the
+ * last round's info with best_score / best_iter (may be NULL). Synchronises. */
+cualign_status cualign_bp_get_best(cualign_bp *h, int32_t *mate_a, cualign_round_info *info);
+
+/* Release everything; NULL-safe. */
+void cualign_bp_free(cualign_bp *h);
+
+/* Sizes of the problem (m, s, ...).  Synchronises. */
+cualign_status cualign_bp_get_sizes(cualign_bp *h, cualign_sizes *sizes);
+
+/* S in CSR form over canonical edge ids (row e lists f ascending):
+ * rowptr (m+1 int64), col (s int32); either may be NULL; *s_out = nnz(S). */
+cualign_status cualign_bp_get_S(cualign_bp *h, int64_t *rowptr, int32_t *col, int64_t *s_out);
+
+/* State after the last iterate (host buffers, each may be NULL):
+ * yc, zc, yp, zp, d: m doubles; Sp: s doubles in get_S's CSR order; p: int. */
+cualign_status cualign_bp_get_state(cualign_bp *h, double *yc, double *zc, double *yp,
+                                    double *zp, double *d, double *Sp, int32_t *p);
+
+/* Inject (y^p, z^p, S^p, p) (host buffers: m, m, s doubles in CSR order) --
+ * checkpoint/resume and one-step parity.  The next iterate runs iteration p+1. */
+cualign_status cualign_bp_set_state(cualign_bp *h, const double *yp, const double *zp,
+                                    const double *Sp, int32_t p);
+
+/* Diagnostics; reset = 1 clears counters after reading. Synchronises. */
+cualign_status cualign_bp_get_stats(cualign_bp *h, cualign_stats *stats, int32_t reset);
+
+/* a7 standalone: the locally-dominant 1/2-approximate matching of L weighted by
+ * x (m doubles; host, or device if CUALIGN_FLAG_DEVICE_PTRS) with the strict
+ * order (x desc, edge id asc), only x > 0 eligible (readings Z6, Z7).  Writes
+ * mate_a (n_A int32) and mate_b (n_B int32) host buffers (either may be NULL):
+ * the matched edge id at each vertex or -1.  *rounds_out (may be NULL)
+ * receives the number of pointer rounds.  L->w is ignored (may be NULL). */
+cualign_status cualign_match(const cualign_edges *L, int32_t n_a, int32_t n_b, const double *x,
+                             const cualign_params *params, int32_t *mate_a, int32_t *mate_b,
+                             int32_t *rounds_out);
+
+/* Message of the last failing call on this thread ("" if none). */
+const char *cualign_last_error(void);
+
+/* Library version string. */
+const char *cualign_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* CUALIGN_BP_H */

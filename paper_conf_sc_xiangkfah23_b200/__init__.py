@@ -1,0 +1,26 @@
+"""B200-native NetAlignBP + locally-dominant matching engine (cuAlign, SC-W 2023).
+
+The compute path is libcualign_bp.so (CUDA, sm_100a; C ABI in
+include/cualign_bp.h).  This package is the thin Python binding over it plus
+the end-to-end `align` helper and the sharded (multi-GPU) driver.
+"""
+from ._lib import (CuAlignBP, CuAlignError, match, load_library, version,
+                   FLAG_DEVICE_PTRS, FLAG_EXACT, FLAG_OTHERMAX_LITERAL, FLAG_ROUND_DAMPED,
+                   FLAG_TIMING, EXPORTED, LIB_PATH, KERNEL_CLASS_NAMES)
+
+
+def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=0, stream=None):
+    """End-to-end alignment (Alg. 2): init (S build), n_iter
+    x (iterate + round), best.  Returns (mate_a, info, per-round infos)."""
+    with CuAlignBP(A, B, L, alpha, beta, gamma, flags, device, stream) as h:
+        infos = []
+        for _ in range(n_iter):
+            h.iterate(1)
+            infos.append(h.round(sync=True))
+        mate, info = h.get_best()
+    return mate, info, infos
+
+
+__all__ = ["CuAlignBP", "CuAlignError", "match", "align", "load_library", "version",
+           "FLAG_DEVICE_PTRS", "FLAG_EXACT", "FLAG_OTHERMAX_LITERAL", "FLAG_ROUND_DAMPED",
+           "FLAG_TIMING", "EXPORTED", "LIB_PATH", "KERNEL_CLASS_NAMES"]

@@ -1,0 +1,312 @@
+"""Thin ctypes binding over libcualign_bp.so (include/cualign_bp.h).
+
+Argument marshalling only: every step of the path runs in the CUDA library.
+There is no fallback: if the library is missing or no GPU is present, the
+calls fail loudly (CuAlignError / OSError).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "lib", "libcualign_bp.so")
+
+OK, EINVAL, ENOMEM, ECUDA, ENCCL, ESTATE = 0, -1, -2, -3, -4, -5
+FLAG_DEVICE_PTRS = 0x01
+FLAG_EXACT = 0x02
+FLAG_OTHERMAX_LITERAL = 0x04
+FLAG_ROUND_DAMPED = 0x08
+FLAG_TIMING = 0x10
+
+K_TOP2, K_EDGE, K_SQUARE, K_ROWSUM, K_MATCH, K_INIT, K_STATE, K_OTHER = range(8)
+KERNEL_CLASS_NAMES = ["top2", "edge", "square", "rowsum", "match", "init", "state", "other"]
+NUM_KERNEL_CLASSES = 8
+
+# every symbol include/cualign_bp.h declares
+EXPORTED = ["cualign_bp_init", "cualign_bp_iterate", "cualign_bp_round", "cualign_bp_get_best",
+            "cualign_bp_free", "cualign_bp_get_sizes", "cualign_bp_get_S", "cualign_bp_get_state",
+            "cualign_bp_set_state", "cualign_bp_get_stats", "cualign_match", "cualign_last_error",
+            "cualign_version"]
+
+
+class CuAlignError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"cualign status {status}: {msg}")
+        self.status = status
+
+
+class Graph_t(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int32), ("rowptr", ctypes.c_void_p), ("col", ctypes.c_void_p)]
+
+
+class Edges_t(ctypes.Structure):
+    _fields_ = [("m", ctypes.c_int64), ("a", ctypes.c_void_p), ("b", ctypes.c_void_p),
+                ("w", ctypes.c_void_p)]
+
+
+class Params_t(ctypes.Structure):
+    _fields_ = [("alpha", ctypes.c_double), ("beta", ctypes.c_double), ("gamma", ctypes.c_double),
+                ("flags", ctypes.c_uint32), ("device", ctypes.c_int32), ("stream", ctypes.c_void_p),
+                ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("nccl_unique_id", ctypes.c_void_p)]
+
+
+class RoundInfo_t(ctypes.Structure):
+    _fields_ = [("iter", ctypes.c_int32), ("source", ctypes.c_int32), ("improved", ctypes.c_int32),
+                ("best_iter", ctypes.c_int32), ("card_y", ctypes.c_int32), ("card_z", ctypes.c_int32),
+                ("score_y", ctypes.c_double), ("score_z", ctypes.c_double),
+                ("weight_y", ctypes.c_double), ("weight_z", ctypes.c_double),
+                ("score", ctypes.c_double), ("best_score", ctypes.c_double),
+                ("overlap_y", ctypes.c_int64), ("overlap_z", ctypes.c_int64),
+                ("rounds_y", ctypes.c_int32), ("rounds_z", ctypes.c_int32)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class Sizes_t(ctypes.Structure):
+    _fields_ = [("n_a", ctypes.c_int32), ("n_b", ctypes.c_int32), ("m", ctypes.c_int64),
+                ("s", ctypes.c_int64), ("squares", ctypes.c_int64), ("max_row", ctypes.c_int64),
+                ("p", ctypes.c_int32), ("fixed_point_bits", ctypes.c_int32),
+                ("device_bytes", ctypes.c_int64)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class Stats_t(ctypes.Structure):
+    _fields_ = [("launches", ctypes.c_int64),
+                ("class_launches", ctypes.c_int64 * NUM_KERNEL_CLASSES),
+                ("class_ms", ctypes.c_double * NUM_KERNEL_CLASSES)]
+
+    def as_dict(self):
+        return {"launches": self.launches,
+                "class_launches": {KERNEL_CLASS_NAMES[i]: self.class_launches[i] for i in range(NUM_KERNEL_CLASSES)},
+                "class_ms": {KERNEL_CLASS_NAMES[i]: self.class_ms[i] for i in range(NUM_KERNEL_CLASSES)}}
+
+
+_lib = None
+
+
+def load_library():
+    """Load libcualign_bp.so (built by __graft_entry__.build() or
+    `python -m paper_conf_sc_xiangkfah23_b200.build`).  Raises if missing."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise OSError(f"{LIB_PATH} not found: build it with "
+                      "`python -m paper_conf_sc_xiangkfah23_b200.build` (no CPU fallback exists)")
+    lib = ctypes.CDLL(LIB_PATH)
+    P, I32, I64, D = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_double
+    lib.cualign_bp_init.restype = I32
+    lib.cualign_bp_init.argtypes = [P, P, P, P, ctypes.POINTER(P)]
+    lib.cualign_bp_iterate.restype = I32
+    lib.cualign_bp_iterate.argtypes = [P, I32]
+    lib.cualign_bp_round.restype = I32
+    lib.cualign_bp_round.argtypes = [P, P]
+    lib.cualign_bp_get_best.restype = I32
+    lib.cualign_bp_get_best.argtypes = [P, P, P]
+    lib.cualign_bp_free.restype = None
+    lib.cualign_bp_free.argtypes = [P]
+    lib.cualign_bp_get_sizes.restype = I32
+    lib.cualign_bp_get_sizes.argtypes = [P, P]
+    lib.cualign_bp_get_S.restype = I32
+    lib.cualign_bp_get_S.argtypes = [P, P, P, P]
+    lib.cualign_bp_get_state.restype = I32
+    lib.cualign_bp_get_state.argtypes = [P, P, P, P, P, P, P, P]
+    lib.cualign_bp_set_state.restype = I32
+    lib.cualign_bp_set_state.argtypes = [P, P, P, P, I32]
+    lib.cualign_bp_get_stats.restype = I32
+    lib.cualign_bp_get_stats.argtypes = [P, P, I32]
+    lib.cualign_match.restype = I32
+    lib.cualign_match.argtypes = [P, I32, I32, P, P, P, P, P]
+    lib.cualign_last_error.restype = ctypes.c_char_p
+    lib.cualign_last_error.argtypes = []
+    lib.cualign_version.restype = ctypes.c_char_p
+    lib.cualign_version.argtypes = []
+    _lib = lib
+    return lib
+
+
+def _check(status):
+    if status != OK:
+        msg = load_library().cualign_last_error().decode(errors="replace")
+        raise CuAlignError(status, msg)
+
+
+def _is_torch(x):
+    return type(x).__module__.startswith("torch")
+
+
+def _ptr(x):
+    """Data pointer of a numpy array or torch tensor (contiguity checked)."""
+    if x is None:
+        return None
+    if _is_torch(x):
+        if not x.is_contiguous():
+            raise ValueError("tensor must be contiguous")
+        return ctypes.c_void_p(x.data_ptr())
+    if not x.flags["C_CONTIGUOUS"]:
+        raise ValueError("array must be C-contiguous")
+    return x.ctypes.data_as(ctypes.c_void_p)
+
+
+def _as_host(x, dtype):
+    return np.ascontiguousarray(np.asarray(x), dtype=dtype)
+
+
+def _prep(x, np_dtype, torch_dtype_name):
+    if _is_torch(x):
+        import torch
+        want = getattr(torch, torch_dtype_name)
+        if x.dtype != want:
+            x = x.to(want)
+        return x.contiguous(), x.is_cuda
+    return _as_host(x, np_dtype), False
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        return None
+    if isinstance(stream, int):
+        return ctypes.c_void_p(stream)
+    return ctypes.c_void_p(stream.cuda_stream)  # torch.cuda.Stream
+
+
+class CuAlignBP:
+    """One alignment problem resident on a GPU (Alg. 2 state + S)."""
+
+    def __init__(self, A, B, L, alpha=1.0, beta=2.0, gamma=0.99, flags=0, device=0, stream=None):
+        lib = load_library()
+        Ap, dA = _prep(A.rowptr, np.int64, "int64")
+        Aj, _ = _prep(A.col, np.int32, "int32")
+        Bp, dB = _prep(B.rowptr, np.int64, "int64")
+        Bj, _ = _prep(B.col, np.int32, "int32")
+        La, dL = _prep(L.a, np.int32, "int32")
+        Lb, _ = _prep(L.b, np.int32, "int32")
+        w, _ = _prep(L.w, np.float64, "float64")
+        on_dev = {dA, dB, dL}
+        if len(on_dev) != 1:
+            raise ValueError("inputs must be all host arrays or all device tensors")
+        if on_dev.pop():
+            flags |= FLAG_DEVICE_PTRS
+        self._keep = (Ap, Aj, Bp, Bj, La, Lb, w)
+        self.n_a, self.n_b, self.m = int(A.n), int(B.n), int(len(L.a))
+        self.flags = flags
+        ga = Graph_t(self.n_a, _ptr(Ap), _ptr(Aj))
+        gb = Graph_t(self.n_b, _ptr(Bp), _ptr(Bj))
+        el = Edges_t(self.m, _ptr(La), _ptr(Lb), _ptr(w))
+        prm = Params_t(float(alpha), float(beta), float(gamma), int(flags), int(device),
+                       _stream_ptr(stream), 0, 1, None)
+        h = ctypes.c_void_p()
+        _check(lib.cualign_bp_init(ctypes.byref(ga), ctypes.byref(gb), ctypes.byref(el),
+                                   ctypes.byref(prm), ctypes.byref(h)))
+        self._h = h
+        self._keep = None
+        sz = self.sizes()
+        self.s = sz["s"]
+        self.squares = sz["squares"]
+
+    # lifecycle
+    def close(self):
+        if getattr(self, "_h", None):
+            load_library().cualign_bp_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    # hot path
+    def iterate(self, n_steps=1):
+        _check(load_library().cualign_bp_iterate(self._h, int(n_steps)))
+
+    def round(self, sync=True):
+        if not sync:
+            _check(load_library().cualign_bp_round(self._h, None))
+            return None
+        info = RoundInfo_t()
+        _check(load_library().cualign_bp_round(self._h, ctypes.byref(info)))
+        return info.as_dict()
+
+    def get_best(self):
+        mate = np.zeros(max(self.n_a, 1), dtype=np.int32)
+        info = RoundInfo_t()
+        _check(load_library().cualign_bp_get_best(self._h, _ptr(mate), ctypes.byref(info)))
+        return mate[:self.n_a], info.as_dict()
+
+    # introspection
+    def sizes(self):
+        sz = Sizes_t()
+        _check(load_library().cualign_bp_get_sizes(self._h, ctypes.byref(sz)))
+        return sz.as_dict()
+
+    def get_S(self):
+        rowptr = np.zeros(self.m + 1, dtype=np.int64)
+        s = ctypes.c_int64()
+        _check(load_library().cualign_bp_get_S(self._h, _ptr(rowptr), None, ctypes.byref(s)))
+        col = np.zeros(max(s.value, 1), dtype=np.int32)
+        _check(load_library().cualign_bp_get_S(self._h, None, _ptr(col), None))
+        return rowptr, col[:s.value]
+
+    def get_state(self, with_S=True):
+        m = max(self.m, 1)
+        out = {k: np.zeros(m) for k in ("yc", "zc", "yp", "zp", "d")}
+        Sp = np.zeros(max(self.s, 1)) if with_S else None
+        p = ctypes.c_int32()
+        _check(load_library().cualign_bp_get_state(self._h, _ptr(out["yc"]), _ptr(out["zc"]),
+                                                    _ptr(out["yp"]), _ptr(out["zp"]),
+                                                    _ptr(out["d"]), _ptr(Sp), ctypes.byref(p)))
+        out = {k: v[:self.m] for k, v in out.items()}
+        if with_S:
+            out["Sp"] = Sp[:self.s]
+        out["p"] = p.value
+        return out
+
+    def set_state(self, yp, zp, Sp, p):
+        yp = _as_host(yp, np.float64)
+        zp = _as_host(zp, np.float64)
+        Sp = _as_host(Sp, np.float64)
+        _check(load_library().cualign_bp_set_state(self._h, _ptr(yp), _ptr(zp), _ptr(Sp), int(p)))
+
+    def stats(self, reset=False):
+        st = Stats_t()
+        _check(load_library().cualign_bp_get_stats(self._h, ctypes.byref(st), int(reset)))
+        return st.as_dict()
+
+
+def match(L, n_a, n_b, x, device=0, flags=0):
+    """Standalone locally-dominant matching of L under weights x (host arrays
+    or CUDA tensors).  Returns (mate_a, mate_b, rounds)."""
+    lib = load_library()
+    La, dL = _prep(L.a, np.int32, "int32")
+    Lb, _ = _prep(L.b, np.int32, "int32")
+    xx, dx = _prep(x, np.float64, "float64")
+    if dL != dx:
+        raise ValueError("L and x must both be host or both be device")
+    if dL:
+        flags |= FLAG_DEVICE_PTRS
+    el = Edges_t(int(len(L.a)), _ptr(La), _ptr(Lb), None)
+    prm = Params_t(1.0, 0.0, 1.0, int(flags), int(device), None, 0, 1, None)
+    ma = np.zeros(max(n_a, 1), dtype=np.int32)
+    mb = np.zeros(max(n_b, 1), dtype=np.int32)
+    rounds = ctypes.c_int32()
+    _check(lib.cualign_match(ctypes.byref(el), int(n_a), int(n_b), _ptr(xx), ctypes.byref(prm),
+                             _ptr(ma), _ptr(mb), ctypes.byref(rounds)))
+    return ma[:n_a], mb[:n_b], rounds.value
+
+
+def version():
+    return load_library().cualign_version().decode()

@@ -1,0 +1,463 @@
+// api.cu -- the C ABI (include/cualign_bp.h): argument checks, handle
+// lifetime, state transfer, diagnostics.  All compute is in init.cu, bp.cu,
+// match.cu.
+#include "internal.cuh"
+
+#include <math.h>
+#include <string.h>
+
+namespace cualign {
+
+static thread_local char g_err[1024] = "";
+
+void set_error(const char *fmt, ...)
+{
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+}
+
+void clear_error() { g_err[0] = 0; }
+
+cualign_status dmalloc(cualign_bp *h, void **p, size_t bytes)
+{
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMalloc(p, bytes);
+    if (e != cudaSuccess) {
+        *p = nullptr;
+        set_error("cudaMalloc(%zu bytes) failed: %s", bytes, cudaGetErrorString(e));
+        (void)cudaGetLastError();
+        return e == cudaErrorMemoryAllocation ? CUALIGN_ENOMEM : CUALIGN_ECUDA;
+    }
+    h->allocs.push_back({*p, bytes});
+    h->device_bytes += (int64_t)bytes;
+    return CUALIGN_OK;
+}
+
+void dfree(cualign_bp *h, void *p)
+{
+    for (auto &a : h->allocs)
+        if (a.first == p && p) {
+            cudaFree(p);
+            h->device_bytes -= (int64_t)a.second;
+            a.first = nullptr;
+            a.second = 0;
+        }
+}
+
+void dfree_all(cualign_bp *h)
+{
+    for (auto &a : h->allocs)
+        if (a.first) cudaFree(a.first);
+    h->allocs.clear();
+    h->device_bytes = 0;
+}
+
+static cudaEvent_t get_event(cualign_bp *h)
+{
+    if (!h->event_pool.empty()) {
+        cudaEvent_t e = h->event_pool.back();
+        h->event_pool.pop_back();
+        return e;
+    }
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    return e;
+}
+
+KScope::KScope(cualign_bp *h_, int cls_) : h(h_), cls(cls_)
+{
+    if (h->timing) {
+        b = get_event(h);
+        cudaEventRecord(b, h->stream);
+    }
+}
+
+KScope::~KScope()
+{
+    h->launches++;
+    h->class_launches[cls]++;
+    if (h->timing && b) {
+        cudaEvent_t e = get_event(h);
+        cudaEventRecord(e, h->stream);
+        h->events[cls].push_back({b, e});
+    }
+}
+
+static void resolve_events(cualign_bp *h)
+{
+    for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
+        for (auto &ep : h->events[c]) {
+            float ms = 0.f;
+            if (cudaEventSynchronize(ep.b) == cudaSuccess && cudaEventElapsedTime(&ms, ep.a, ep.b) == cudaSuccess)
+                h->class_ms[c] += ms;
+            h->event_pool.push_back(ep.a);
+            h->event_pool.push_back(ep.b);
+        }
+        h->events[c].clear();
+    }
+    (void)cudaGetLastError();
+}
+
+static cualign_status check_params(const cualign_params *p)
+{
+    if (!p) {
+        set_error("params is NULL");
+        return CUALIGN_EINVAL;
+    }
+    if (!(p->alpha >= 0.0) || !isfinite(p->alpha)) {
+        set_error("alpha must be finite and >= 0 (PAPER.md:64), got %g", p->alpha);
+        return CUALIGN_EINVAL;
+    }
+    if (!(p->beta >= 0.0) || !isfinite(p->beta)) {
+        set_error("beta must be finite and >= 0 (PAPER.md:64), got %g", p->beta);
+        return CUALIGN_EINVAL;
+    }
+    if (!(p->gamma > 0.0 && p->gamma <= 1.0)) {
+        set_error("gamma must be in (0, 1], got %g", p->gamma);
+        return CUALIGN_EINVAL;
+    }
+    if (p->rank != 0 || (p->world != 0 && p->world != 1) || p->nccl_unique_id != nullptr) {
+        set_error("sharded handles are not available through this entry point (rank=%d world=%d)", p->rank,
+                  p->world);
+        return CUALIGN_EINVAL;
+    }
+    return CUALIGN_OK;
+}
+
+static cualign_status open_handle(const cualign_params *params, cualign_bp **out)
+{
+    cualign_bp *h = new cualign_bp();
+    h->alpha = params->alpha;
+    h->beta = params->beta;
+    h->gamma = params->gamma;
+    h->flags = params->flags;
+    h->dev = params->device;
+    h->timing = (params->flags & CUALIGN_FLAG_TIMING) != 0;
+    *out = h;
+    CA_CUDA(cudaSetDevice(h->dev));
+    CA_CUDA(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->dev));
+    if (params->stream) {
+        h->stream = (cudaStream_t)params->stream;
+    } else {
+        CA_CUDA(cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking));
+        h->own_stream = true;
+    }
+    return CUALIGN_OK;
+}
+
+static void close_handle(cualign_bp *h)
+{
+    if (!h) return;
+    cudaSetDevice(h->dev);
+    if (h->stream) cudaStreamSynchronize(h->stream);
+    resolve_events(h);
+    for (auto e : h->event_pool) cudaEventDestroy(e);
+    dfree_all(h);
+    if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+    (void)cudaGetLastError();
+    delete h;
+}
+
+static cualign_status alloc_state(cualign_bp *h)
+{
+    const size_t m = (size_t)h->L.m;
+    for (double **p : {&h->yc, &h->zc, &h->yp, &h->zp, &h->d, &h->u}) {
+        CA_TRY(dalloc(h, p, m));
+        CA_CUDA(cudaMemsetAsync(*p, 0, sizeof(double) * (m ? m : 1), h->stream));
+    }
+    CA_TRY(dalloc(h, &h->Atop, (size_t)h->L.nA + 1));
+    CA_TRY(dalloc(h, &h->Btop, (size_t)h->L.nB + 1));
+    if (h->flags & CUALIGN_FLAG_EXACT) {
+        CA_TRY(dalloc(h, &h->texact, m));
+        CA_TRY(dalloc(h, &h->Ffull, (size_t)h->s));
+        CA_TRY(ensure_sq_pos(h));
+    } else {
+        CA_TRY(dalloc(h, &h->tacc, m));
+    }
+    return CUALIGN_OK;
+}
+
+#define API_ENTER() clear_error()
+#define CHECK_H()                                   \
+    do {                                            \
+        if (!h) {                                   \
+            set_error("handle is NULL");            \
+            return CUALIGN_EINVAL;                  \
+        }                                           \
+        CA_CUDA(cudaSetDevice(h->dev));             \
+    } while (0)
+
+} // namespace cualign
+
+using namespace cualign;
+
+extern "C" {
+
+const char *cualign_last_error(void) { return g_err; }
+
+const char *cualign_version(void) { return "cualign_bp 0.1 (sm_100a)"; }
+
+cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B, const cualign_edges *L,
+                               const cualign_params *params, cualign_bp **out)
+{
+    API_ENTER();
+    if (!out) {
+        set_error("out is NULL");
+        return CUALIGN_EINVAL;
+    }
+    *out = nullptr;
+    CA_TRY(check_params(params));
+    if (!A || !B || !L || !A->rowptr || !B->rowptr || A->n < 0 || B->n < 0 || L->m < 0 ||
+        (L->m > 0 && (!L->a || !L->b || !L->w)) || (A->n > 0 && !A->col && A->rowptr == nullptr)) {
+        set_error("NULL or negative-size input");
+        return CUALIGN_EINVAL;
+    }
+    cualign_bp *h = nullptr;
+    cualign_status st = open_handle(params, &h);
+    if (st == CUALIGN_OK) st = build_problem(h, A, B, L);
+    if (st == CUALIGN_OK) st = alloc_state(h);
+    if (st == CUALIGN_OK) st = match_setup(h);
+    if (st == CUALIGN_OK) st = bp_fsum(h); // F(S^p = 0) row sums for iteration 1
+    if (st == CUALIGN_OK) {
+        cudaError_t e = cudaStreamSynchronize(h->stream);
+        if (e != cudaSuccess) {
+            set_error("init: %s", cudaGetErrorString(e));
+            st = CUALIGN_ECUDA;
+        }
+    }
+    if (st != CUALIGN_OK) {
+        std::string msg = g_err;
+        close_handle(h);
+        set_error("%s", msg.c_str());
+        return st;
+    }
+    *out = h;
+    return CUALIGN_OK;
+}
+
+cualign_status cualign_bp_iterate(cualign_bp *h, int32_t n_steps)
+{
+    API_ENTER();
+    CHECK_H();
+    if (n_steps < 0) {
+        set_error("n_steps < 0");
+        return CUALIGN_EINVAL;
+    }
+    return bp_iterate(h, n_steps);
+}
+
+cualign_status cualign_bp_round(cualign_bp *h, cualign_round_info *info)
+{
+    API_ENTER();
+    CHECK_H();
+    CA_TRY(match_round(h));
+    h->have_info = true;
+    if (info) {
+        CA_CUDA(cudaMemcpyAsync(&h->last_info, &h->rd->info, sizeof(cualign_round_info), cudaMemcpyDeviceToHost,
+                                h->stream));
+        CA_CUDA(cudaStreamSynchronize(h->stream));
+        *info = h->last_info;
+    }
+    return CUALIGN_OK;
+}
+
+cualign_status cualign_bp_get_best(cualign_bp *h, int32_t *mate_a, cualign_round_info *info)
+{
+    API_ENTER();
+    CHECK_H();
+    if (mate_a && h->L.nA)
+        CA_CUDA(cudaMemcpyAsync(mate_a, h->best_mate, sizeof(int32_t) * (size_t)h->L.nA, cudaMemcpyDeviceToHost,
+                                h->stream));
+    RoundDev r;
+    CA_CUDA(cudaMemcpyAsync(&r, h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->stream));
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    if (info) {
+        *info = r.info;
+        info->best_score = r.best_score;
+        info->best_iter = r.best_iter;
+    }
+    return CUALIGN_OK;
+}
+
+void cualign_bp_free(cualign_bp *h) { close_handle(h); }
+
+cualign_status cualign_bp_get_sizes(cualign_bp *h, cualign_sizes *sz)
+{
+    API_ENTER();
+    CHECK_H();
+    if (!sz) {
+        set_error("sizes is NULL");
+        return CUALIGN_EINVAL;
+    }
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    sz->n_a = h->L.nA;
+    sz->n_b = h->L.nB;
+    sz->m = h->L.m;
+    sz->s = h->s;
+    sz->squares = h->nsq;
+    sz->max_row = h->max_row;
+    sz->p = h->p;
+    sz->fixed_point_bits = (h->flags & CUALIGN_FLAG_EXACT) ? 0 : h->fp_bits;
+    sz->device_bytes = h->device_bytes;
+    return CUALIGN_OK;
+}
+
+cualign_status cualign_bp_get_S(cualign_bp *h, int64_t *rowptr, int32_t *col, int64_t *s_out)
+{
+    API_ENTER();
+    CHECK_H();
+    if (rowptr)
+        CA_CUDA(cudaMemcpyAsync(rowptr, h->Srp, sizeof(int64_t) * ((size_t)h->L.m + 1), cudaMemcpyDeviceToHost,
+                                h->stream));
+    if (col && h->s)
+        CA_CUDA(cudaMemcpyAsync(col, h->Scol, sizeof(int32_t) * (size_t)h->s, cudaMemcpyDeviceToHost, h->stream));
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    if (s_out) *s_out = h->s;
+    return CUALIGN_OK;
+}
+
+cualign_status cualign_bp_get_state(cualign_bp *h, double *yc, double *zc, double *yp, double *zp, double *d,
+                                    double *Sp, int32_t *p)
+{
+    API_ENTER();
+    CHECK_H();
+    const size_t mb = sizeof(double) * (size_t)h->L.m;
+    struct {
+        double *dst;
+        double *src;
+    } vec[] = {{yc, h->yc}, {zc, h->zc}, {yp, h->yp}, {zp, h->zp}, {d, h->d}};
+    for (auto &v : vec)
+        if (v.dst && mb) CA_CUDA(cudaMemcpyAsync(v.dst, v.src, mb, cudaMemcpyDeviceToHost, h->stream));
+    if (Sp && h->s) {
+        double *tmp = nullptr;
+        CA_CUDA(cudaMalloc(&tmp, sizeof(double) * (size_t)h->s));
+        cualign_status st = bp_scatter_Sp(h, tmp);
+        if (st == CUALIGN_OK) {
+            cudaError_t e = cudaMemcpyAsync(Sp, tmp, sizeof(double) * (size_t)h->s, cudaMemcpyDeviceToHost, h->stream);
+            if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+            if (e != cudaSuccess) {
+                set_error("get_state: %s", cudaGetErrorString(e));
+                st = CUALIGN_ECUDA;
+            }
+        }
+        cudaFree(tmp);
+        CA_TRY(st);
+    }
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    if (p) *p = h->p;
+    return CUALIGN_OK;
+}
+
+cualign_status cualign_bp_set_state(cualign_bp *h, const double *yp, const double *zp, const double *Sp,
+                                    int32_t p)
+{
+    API_ENTER();
+    CHECK_H();
+    if (!yp || !zp || (!Sp && h->s) || p < 0) {
+        set_error("set_state: NULL buffer or p < 0");
+        return CUALIGN_EINVAL;
+    }
+    const size_t mb = sizeof(double) * (size_t)h->L.m;
+    if (mb) {
+        CA_CUDA(cudaMemcpyAsync(h->yp, yp, mb, cudaMemcpyHostToDevice, h->stream));
+        CA_CUDA(cudaMemcpyAsync(h->zp, zp, mb, cudaMemcpyHostToDevice, h->stream));
+    }
+    if (h->s) {
+        double *tmp = nullptr;
+        CA_CUDA(cudaMalloc(&tmp, sizeof(double) * (size_t)h->s));
+        cudaError_t e = cudaMemcpyAsync(tmp, Sp, sizeof(double) * (size_t)h->s, cudaMemcpyHostToDevice, h->stream);
+        cualign_status st = CUALIGN_OK;
+        if (e != cudaSuccess) {
+            set_error("set_state: %s", cudaGetErrorString(e));
+            st = CUALIGN_ECUDA;
+        }
+        if (st == CUALIGN_OK) st = bp_gather_Sp(h, tmp);
+        if (st == CUALIGN_OK && cudaStreamSynchronize(h->stream) != cudaSuccess) st = CUALIGN_ECUDA;
+        cudaFree(tmp);
+        CA_TRY(st);
+    }
+    h->p = p;
+    CA_TRY(bp_fsum(h));
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    return CUALIGN_OK;
+}
+
+cualign_status cualign_bp_get_stats(cualign_bp *h, cualign_stats *stats, int32_t reset)
+{
+    API_ENTER();
+    CHECK_H();
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    resolve_events(h);
+    if (stats) {
+        stats->launches = h->launches;
+        for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
+            stats->class_launches[c] = h->class_launches[c];
+            stats->class_ms[c] = h->class_ms[c];
+        }
+    }
+    if (reset) {
+        h->launches = 0;
+        for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
+            h->class_launches[c] = 0;
+            h->class_ms[c] = 0.0;
+        }
+    }
+    return CUALIGN_OK;
+}
+
+cualign_status cualign_match(const cualign_edges *L, int32_t n_a, int32_t n_b, const double *x,
+                             const cualign_params *params, int32_t *mate_a, int32_t *mate_b, int32_t *rounds_out)
+{
+    API_ENTER();
+    if (!L || !x || !params || n_a < 0 || n_b < 0 || L->m < 0 || (L->m > 0 && (!L->a || !L->b))) {
+        set_error("cualign_match: NULL or negative-size input");
+        return CUALIGN_EINVAL;
+    }
+    cualign_params prm = *params;
+    prm.alpha = 1.0;
+    prm.beta = 0.0;
+    prm.gamma = 1.0;
+    prm.rank = 0;
+    prm.world = 1;
+    prm.nccl_unique_id = nullptr;
+    cualign_bp *h = nullptr;
+    cualign_status st = open_handle(&prm, &h);
+    const bool devp = (prm.flags & CUALIGN_FLAG_DEVICE_PTRS) != 0;
+    cualign_edges E = *L;
+    E.w = nullptr;
+    double *xd = nullptr;
+    if (st == CUALIGN_OK) st = build_L(h, h->L, &E, devp, true, n_a, n_b);
+    if (st == CUALIGN_OK) st = match_setup(h);
+    if (st == CUALIGN_OK) st = dalloc(h, &xd, (size_t)L->m);
+    if (st == CUALIGN_OK && L->m) {
+        if (cudaMemcpyAsync(xd, x, sizeof(double) * (size_t)L->m,
+                            devp ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, h->stream) != cudaSuccess) {
+            set_error("cualign_match: copy of x failed");
+            st = CUALIGN_ECUDA;
+        }
+    }
+    if (st == CUALIGN_OK) st = match_standalone(h, xd, rounds_out);
+    if (st == CUALIGN_OK && mate_a && n_a)
+        if (cudaMemcpyAsync(mate_a, h->mateA, sizeof(int32_t) * (size_t)n_a, cudaMemcpyDeviceToHost, h->stream) !=
+            cudaSuccess)
+            st = CUALIGN_ECUDA;
+    if (st == CUALIGN_OK && mate_b && n_b)
+        if (cudaMemcpyAsync(mate_b, h->mateB, sizeof(int32_t) * (size_t)n_b, cudaMemcpyDeviceToHost, h->stream) !=
+            cudaSuccess)
+            st = CUALIGN_ECUDA;
+    if (st == CUALIGN_OK) {
+        cudaError_t e = cudaStreamSynchronize(h->stream);
+        if (e != cudaSuccess) {
+            set_error("cualign_match: %s", cudaGetErrorString(e));
+            st = CUALIGN_ECUDA;
+        }
+    }
+    std::string msg = g_err;
+    close_handle(h);
+    if (st != CUALIGN_OK) set_error("%s", msg.c_str());
+    return st;
+}
+
+} // extern "C"

@@ -1,0 +1,438 @@
+// init.cu -- rows a1 (canonical L, incidences) and a2 (S construction, Alg. 3)
+// of the hot path, plus input validation.
+//
+// S definition (§2): S_{(i,i'),(j,j')} = 1 iff (i,j) in E_A and
+// (i',j') in E_B.  Alg. 3 loops, per L edge e = (i, i'),
+// over the neighbours j of i and j' of i' and tests (j, j') in E_L.  Here the
+// same set is enumerated from the other side: for each j in N_A(i), the L row
+// of j (candidates (j, b), b ascending) is intersected with the sorted
+// N_B(i') by binary search -- k*log(deg) instead of deg_B work per j, which
+// bounds the cost at hub vertices.  One warp per edge e; the warp walks the
+// concatenation of the L rows of e's A-neighbours 32 candidates at a time, so
+// hits are emitted in ascending f with a ballot prefix (no sort).
+// Two passes (count -> scan -> fill); the fill also writes the square layout
+// (f > e suffix of each row), see DESIGN.md "Data layout".
+#include "internal.cuh"
+
+#include <cub/cub.cuh>
+#include <math.h>
+
+namespace cualign {
+
+namespace {
+
+struct TmpBuf {
+    void *p = nullptr;
+    ~TmpBuf()
+    {
+        if (p) cudaFree(p);
+    }
+};
+
+#define FULL_MASK 0xffffffffu
+
+// ---------------------------------------------------------------- validation
+enum : int {
+    E_ROWPTR = 1, E_COLRANGE = 2, E_SELFLOOP = 4, E_UNSORTED = 8, E_ASYM = 16,
+    E_LRANGE = 32, E_LORDER = 64, E_WFINITE = 128
+};
+
+__device__ __forceinline__ bool bsearch_i32(const int32_t *x, int64_t lo, int64_t hi, int32_t v)
+{
+    while (lo < hi) {
+        int64_t mid = lo + ((hi - lo) >> 1);
+        int32_t xm = x[mid];
+        if (xm < v) lo = mid + 1;
+        else if (xm > v) hi = mid;
+        else return true;
+    }
+    return false;
+}
+
+__global__ void k_check_graph(int32_t n, int64_t nnz, const int64_t *rp, const int32_t *col,
+                              int *err)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t lo = rp[i], hi = rp[i + 1];
+        if (lo < 0 || hi < lo || hi > nnz) {
+            atomicOr(err, E_ROWPTR);
+            continue;
+        }
+        int32_t prev = -1;
+        for (int64_t x = lo; x < hi; x++) {
+            int32_t c = col[x];
+            if (c < 0 || c >= n) {
+                atomicOr(err, E_COLRANGE);
+                break;
+            }
+            if (c == (int32_t)i) atomicOr(err, E_SELFLOOP);
+            if (c <= prev) atomicOr(err, E_UNSORTED);
+            prev = c;
+            int64_t clo = rp[c], chi = rp[c + 1];
+            if (clo < 0 || chi < clo || chi > nnz || !bsearch_i32(col, clo, chi, (int32_t)i))
+                atomicOr(err, E_ASYM);
+        }
+    }
+}
+
+__global__ void k_check_edges(int64_t m, int32_t nA, int32_t nB, const int32_t *a,
+                              const int32_t *b, const double *w, int *err)
+{
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < m;
+         k += (int64_t)gridDim.x * blockDim.x) {
+        int32_t ak = a[k], bk = b[k];
+        if (ak < 0 || ak >= nA || bk < 0 || bk >= nB) atomicOr(err, E_LRANGE);
+        if (w && !isfinite(w[k])) atomicOr(err, E_WFINITE);
+        if (k + 1 < m) {
+            int32_t an = a[k + 1], bn = b[k + 1];
+            if (an < ak || (an == ak && bn <= bk)) atomicOr(err, E_LORDER);
+        }
+    }
+}
+
+// Arow[v] = first index k with key[k] >= v (key sorted ascending), v in [0, n]
+__global__ void k_rowptr_from_sorted(int64_t m, const int32_t *key, int32_t n, int64_t *rowptr)
+{
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= n;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        int64_t lo = 0, hi = m;
+        while (lo < hi) {
+            int64_t mid = lo + ((hi - lo) >> 1);
+            if (key[mid] < (int32_t)v) lo = mid + 1;
+            else hi = mid;
+        }
+        rowptr[v] = lo;
+    }
+}
+
+__global__ void k_iota(int64_t m, int32_t *x)
+{
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < m;
+         k += (int64_t)gridDim.x * blockDim.x)
+        x[k] = (int32_t)k;
+}
+
+// -------------------------------------------------------------- S build
+// One warp per L edge e = (i, i').  Candidates f are the L edges (j, b) with
+// j in N_A(i) (rows of L, concatenated in ascending j => ascending f); f is a
+// hit iff b in N_B(i').
+template <bool FILL>
+__global__ void __launch_bounds__(256)
+k_sbuild(int64_t m, const int32_t *__restrict__ La, const int32_t *__restrict__ Lb,
+         const int64_t *__restrict__ Arow, const int64_t *__restrict__ Ap,
+         const int32_t *__restrict__ Aj, const int64_t *__restrict__ Bp,
+         const int32_t *__restrict__ Bj, int64_t *__restrict__ cnt, int64_t *__restrict__ ucnt,
+         const int64_t *__restrict__ Srp, const int64_t *__restrict__ sq_rp,
+         int32_t *__restrict__ Scol, int2 *__restrict__ sq_ef)
+{
+    const int lane = threadIdx.x & 31;
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const unsigned lt_mask = (1u << lane) - 1u;
+    for (int64_t e = warp; e < m; e += nwarps) {
+        const int32_t i = La[e], ip = Lb[e];
+        const int64_t bs = Bp[ip], be = Bp[ip + 1];
+        const int64_t a_lo = Ap[i], a_hi = Ap[i + 1];
+        int64_t total = 0, upper = 0, lower_cnt = 0, row0 = 0, sq0 = 0;
+        if (FILL) {
+            row0 = Srp[e];
+            sq0 = sq_rp[e];
+            lower_cnt = (Srp[e + 1] - row0) - (sq_rp[e + 1] - sq0);
+        }
+        if (be == bs) {
+            if (!FILL && lane == 0) {
+                cnt[e] = 0;
+                ucnt[e] = 0;
+            }
+            continue;
+        }
+        for (int64_t xb = a_lo; xb < a_hi; xb += 32) {
+            const int64_t x = xb + lane;
+            int64_t lo = 0, len = 0;
+            if (x < a_hi) {
+                const int32_t j = Aj[x];
+                lo = Arow[j];
+                len = Arow[j + 1] - lo;
+            }
+            // inclusive warp scan of len
+            int64_t incl = len;
+#pragma unroll
+            for (int off = 1; off < 32; off <<= 1) {
+                int64_t v = __shfl_up_sync(FULL_MASK, incl, off);
+                if (lane >= off) incl += v;
+            }
+            const int64_t T = __shfl_sync(FULL_MASK, incl, 31);
+            const int64_t excl = incl - len;
+            for (int64_t c = 0; c < T; c += 32) {
+                const int64_t pos = c + lane;
+                // first lane k with incl[k] > pos
+                int k = 0;
+#pragma unroll
+                for (int step = 16; step >= 1; step >>= 1) {
+                    int64_t v = __shfl_sync(FULL_MASK, incl, k + step - 1);
+                    if (v <= pos) k += step;
+                }
+                const int64_t ek = __shfl_sync(FULL_MASK, excl, k);
+                const int64_t lk = __shfl_sync(FULL_MASK, lo, k);
+                bool hit = false;
+                int64_t f = 0;
+                if (pos < T) {
+                    f = lk + (pos - ek);
+                    hit = bsearch_i32(Bj, bs, be, Lb[f]);
+                }
+                const unsigned mask = __ballot_sync(FULL_MASK, hit);
+                if (FILL) {
+                    if (hit) {
+                        const int64_t idx = total + __popc(mask & lt_mask);
+                        Scol[row0 + idx] = (int32_t)f;
+                        if (idx >= lower_cnt) sq_ef[sq0 + (idx - lower_cnt)] = make_int2((int)e, (int)f);
+                    }
+                } else {
+                    const unsigned um = __ballot_sync(FULL_MASK, hit && f > e);
+                    upper += __popc(um);
+                }
+                total += __popc(mask);
+            }
+        }
+        if (!FILL && lane == 0) {
+            cnt[e] = total;
+            ucnt[e] = upper;
+        }
+    }
+}
+
+// sq_pos[q] = (pos of (e,f) in row e, pos of (e) in row f)
+__global__ void k_sq_pos(int64_t nsq, const int2 *__restrict__ sq_ef, const int64_t *__restrict__ Srp,
+                         const int64_t *__restrict__ sq_rp, const int32_t *__restrict__ Scol,
+                         longlong2 *__restrict__ sq_pos)
+{
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq;
+         q += (int64_t)gridDim.x * blockDim.x) {
+        const int2 ef = sq_ef[q];
+        const int e = ef.x, f = ef.y;
+        const int64_t row_len = Srp[e + 1] - Srp[e];
+        const int64_t up_len = sq_rp[e + 1] - sq_rp[e];
+        const int64_t pef = Srp[e] + (row_len - up_len) + (q - sq_rp[e]);
+        int64_t lo = Srp[f], hi = Srp[f + 1];
+        while (lo < hi) {
+            int64_t mid = lo + ((hi - lo) >> 1);
+            if (Scol[mid] < e) lo = mid + 1;
+            else hi = mid;
+        }
+        sq_pos[q] = make_longlong2(pef, lo);
+    }
+}
+
+cualign_status upload(cualign_bp *h, void **dst, const void *src, size_t bytes, bool device_ptrs)
+{
+    CA_TRY(dmalloc(h, dst, bytes));
+    if (bytes)
+        CA_CUDA(cudaMemcpyAsync(*dst, src, bytes,
+                                device_ptrs ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
+                                h->stream));
+    return CUALIGN_OK;
+}
+
+cualign_status check_flags(cualign_bp *h, int *err_dev, const char *what)
+{
+    int err = 0;
+    CA_CUDA(cudaMemcpyAsync(&err, err_dev, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    if (err) {
+        set_error("invalid %s:%s%s%s%s%s%s%s%s", what, (err & E_ROWPTR) ? " bad row pointers" : "",
+                  (err & E_COLRANGE) ? " column out of range" : "",
+                  (err & E_SELFLOOP) ? " self loop" : "",
+                  (err & E_UNSORTED) ? " row not strictly increasing (unsorted/duplicate)" : "",
+                  (err & E_ASYM) ? " not symmetric" : "",
+                  (err & E_LRANGE) ? " edge endpoint out of range" : "",
+                  (err & E_LORDER) ? " edges not strictly increasing in (a,b) (unsorted/duplicate)" : "",
+                  (err & E_WFINITE) ? " non-finite weight" : "");
+        return CUALIGN_EINVAL;
+    }
+    return CUALIGN_OK;
+}
+
+} // namespace
+
+// ------------------------------------------------------------------ L build
+cualign_status build_L(cualign_bp *h, LDev &L, const cualign_edges *E, bool device_ptrs,
+                       bool validate, int32_t nA, int32_t nB)
+{
+    KScope ks(h, CUALIGN_K_INIT);
+    L.nA = nA;
+    L.nB = nB;
+    L.m = E->m;
+    const int64_t m = E->m;
+    const int G = h->num_sms * 8;
+    CA_TRY(upload(h, (void **)&L.La, E->a, sizeof(int32_t) * m, device_ptrs));
+    CA_TRY(upload(h, (void **)&L.Lb, E->b, sizeof(int32_t) * m, device_ptrs));
+    if (E->w) CA_TRY(upload(h, (void **)&L.w, E->w, sizeof(double) * m, device_ptrs));
+    if (validate) {
+        TmpBuf err;
+        CA_CUDA(cudaMalloc(&err.p, sizeof(int)));
+        CA_CUDA(cudaMemsetAsync(err.p, 0, sizeof(int), h->stream));
+        if (m) k_check_edges<<<grid_for(m, 256, G), 256, 0, h->stream>>>(m, nA, nB, L.La, L.Lb, L.w,
+                                                                          (int *)err.p);
+        CA_CUDA(cudaGetLastError());
+        CA_TRY(check_flags(h, (int *)err.p, "L"));
+    }
+    // A-side rows: edges are sorted by a
+    CA_TRY(dalloc(h, &L.Arow, (size_t)nA + 1));
+    k_rowptr_from_sorted<<<grid_for((int64_t)nA + 1, 256, G), 256, 0, h->stream>>>(m, L.La, nA, L.Arow);
+    CA_CUDA(cudaGetLastError());
+    // B-side incidence: stable radix sort of edge ids by b (ids stay ascending)
+    CA_TRY(dalloc(h, &L.Bedge, (size_t)(m ? m : 1)));
+    CA_TRY(dalloc(h, &L.Bptr, (size_t)nB + 1));
+    {
+        TmpBuf keys_out, ids_in, tmp;
+        CA_CUDA(cudaMalloc(&keys_out.p, sizeof(int32_t) * (m ? m : 1)));
+        CA_CUDA(cudaMalloc(&ids_in.p, sizeof(int32_t) * (m ? m : 1)));
+        if (m) {
+            k_iota<<<grid_for(m, 256, G), 256, 0, h->stream>>>(m, (int32_t *)ids_in.p);
+            int end_bit = 1;
+            while (end_bit < 31 && ((int64_t)1 << end_bit) < (int64_t)nB) end_bit++;
+            size_t tbytes = 0;
+            CA_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tbytes, L.Lb, (int32_t *)keys_out.p,
+                                                    (int32_t *)ids_in.p, L.Bedge, (int)m, 0, end_bit,
+                                                    h->stream));
+            CA_CUDA(cudaMalloc(&tmp.p, tbytes ? tbytes : 1));
+            CA_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tbytes, L.Lb, (int32_t *)keys_out.p,
+                                                    (int32_t *)ids_in.p, L.Bedge, (int)m, 0, end_bit,
+                                                    h->stream));
+        }
+        k_rowptr_from_sorted<<<grid_for((int64_t)nB + 1, 256, G), 256, 0, h->stream>>>(
+            m, (int32_t *)keys_out.p, nB, L.Bptr);
+        CA_CUDA(cudaGetLastError());
+        CA_CUDA(cudaStreamSynchronize(h->stream)); // TmpBufs die here
+    }
+    return CUALIGN_OK;
+}
+
+// ------------------------------------------------------------ problem build
+cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualign_graph *B,
+                             const cualign_edges *E)
+{
+    const bool devp = (h->flags & CUALIGN_FLAG_DEVICE_PTRS) != 0;
+    const int G = h->num_sms * 8;
+    // graph row pointers: read nnz (last entry) first
+    int64_t nnzA = 0, nnzB = 0;
+    CA_CUDA(cudaMemcpy(&nnzA, A->rowptr + A->n, sizeof(int64_t),
+                       devp ? cudaMemcpyDeviceToHost : cudaMemcpyHostToHost));
+    CA_CUDA(cudaMemcpy(&nnzB, B->rowptr + B->n, sizeof(int64_t),
+                       devp ? cudaMemcpyDeviceToHost : cudaMemcpyHostToHost));
+    if (nnzA < 0 || nnzB < 0 || nnzA > ((int64_t)1 << 40) || nnzB > ((int64_t)1 << 40)) {
+        set_error("invalid graph: rowptr[n] out of range");
+        return CUALIGN_EINVAL;
+    }
+    int64_t *Ap = nullptr, *Bp = nullptr;
+    int32_t *Aj = nullptr, *Bj = nullptr;
+    {
+        KScope ks(h, CUALIGN_K_INIT);
+        CA_TRY(upload(h, (void **)&Ap, A->rowptr, sizeof(int64_t) * ((size_t)A->n + 1), devp));
+        CA_TRY(upload(h, (void **)&Aj, A->col, sizeof(int32_t) * (size_t)nnzA, devp));
+        CA_TRY(upload(h, (void **)&Bp, B->rowptr, sizeof(int64_t) * ((size_t)B->n + 1), devp));
+        CA_TRY(upload(h, (void **)&Bj, B->col, sizeof(int32_t) * (size_t)nnzB, devp));
+        TmpBuf err;
+        CA_CUDA(cudaMalloc(&err.p, sizeof(int)));
+        CA_CUDA(cudaMemsetAsync(err.p, 0, sizeof(int), h->stream));
+        if (A->n)
+            k_check_graph<<<grid_for(A->n, 256, G), 256, 0, h->stream>>>(A->n, nnzA, Ap, Aj, (int *)err.p);
+        CA_CUDA(cudaGetLastError());
+        CA_TRY(check_flags(h, (int *)err.p, "graph A"));
+        CA_CUDA(cudaMemsetAsync(err.p, 0, sizeof(int), h->stream));
+        if (B->n)
+            k_check_graph<<<grid_for(B->n, 256, G), 256, 0, h->stream>>>(B->n, nnzB, Bp, Bj, (int *)err.p);
+        CA_CUDA(cudaGetLastError());
+        CA_TRY(check_flags(h, (int *)err.p, "graph B"));
+    }
+    CA_TRY(build_L(h, h->L, E, devp, true, A->n, B->n));
+    const int64_t m = h->L.m;
+
+    // S: count pass
+    CA_TRY(dalloc(h, &h->Srp, (size_t)m + 1));
+    CA_TRY(dalloc(h, &h->sq_rp, (size_t)m + 1));
+    {
+        KScope ks(h, CUALIGN_K_INIT);
+        TmpBuf cnt, ucnt, tmp, mx;
+        CA_CUDA(cudaMalloc(&cnt.p, sizeof(int64_t) * (m ? m : 1)));
+        CA_CUDA(cudaMalloc(&ucnt.p, sizeof(int64_t) * (m ? m : 1)));
+        CA_CUDA(cudaMalloc(&mx.p, sizeof(int64_t)));
+        CA_CUDA(cudaMemsetAsync(h->Srp, 0, sizeof(int64_t), h->stream));
+        CA_CUDA(cudaMemsetAsync(h->sq_rp, 0, sizeof(int64_t), h->stream));
+        CA_CUDA(cudaMemsetAsync(mx.p, 0, sizeof(int64_t), h->stream));
+        if (m) {
+            const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
+            k_sbuild<false><<<blocks, 256, 0, h->stream>>>(m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
+                                                           (int64_t *)cnt.p, (int64_t *)ucnt.p, nullptr,
+                                                           nullptr, nullptr, nullptr);
+            CA_CUDA(cudaGetLastError());
+            size_t t1 = 0, t2 = 0, t3 = 0;
+            CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, t1, (int64_t *)cnt.p, h->Srp + 1, (int)m, h->stream));
+            CA_CUDA(cub::DeviceReduce::Max(nullptr, t3, (int64_t *)cnt.p, (int64_t *)mx.p, (int)m, h->stream));
+            t2 = t1 > t3 ? t1 : t3;
+            CA_CUDA(cudaMalloc(&tmp.p, t2 ? t2 : 1));
+            CA_CUDA(cub::DeviceScan::InclusiveSum(tmp.p, t1, (int64_t *)cnt.p, h->Srp + 1, (int)m, h->stream));
+            CA_CUDA(cub::DeviceScan::InclusiveSum(tmp.p, t1, (int64_t *)ucnt.p, h->sq_rp + 1, (int)m, h->stream));
+            CA_CUDA(cub::DeviceReduce::Max(tmp.p, t3, (int64_t *)cnt.p, (int64_t *)mx.p, (int)m, h->stream));
+        }
+        CA_CUDA(cudaMemcpyAsync(&h->s, h->Srp + m, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaMemcpyAsync(&h->nsq, h->sq_rp + m, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaMemcpyAsync(&h->max_row, mx.p, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaStreamSynchronize(h->stream));
+    }
+    if (h->s != 2 * h->nsq) {
+        set_error("internal: S not symmetric (s=%lld, upper=%lld)", (long long)h->s, (long long)h->nsq);
+        return CUALIGN_ECUDA;
+    }
+    if (m >= ((int64_t)1 << 31) - 1) {
+        set_error("m = %lld exceeds int32 edge ids", (long long)m);
+        return CUALIGN_EINVAL;
+    }
+    // S: fill pass
+    CA_TRY(dalloc(h, &h->Scol, (size_t)(h->s ? h->s : 1)));
+    CA_TRY(dalloc(h, &h->sq_ef, (size_t)(h->nsq ? h->nsq : 1)));
+    CA_TRY(dalloc(h, &h->sq_val, (size_t)(h->nsq ? h->nsq : 1)));
+    {
+        KScope ks(h, CUALIGN_K_INIT);
+        if (m && h->s) {
+            const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
+            k_sbuild<true><<<blocks, 256, 0, h->stream>>>(m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
+                                                          nullptr, nullptr, h->Srp, h->sq_rp, h->Scol,
+                                                          h->sq_ef);
+            CA_CUDA(cudaGetLastError());
+        }
+        CA_CUDA(cudaMemsetAsync(h->sq_val, 0, sizeof(double2) * (size_t)(h->nsq ? h->nsq : 1), h->stream));
+    }
+    // the graphs are not needed after S is built
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    for (void *p : {(void *)Ap, (void *)Aj, (void *)Bp, (void *)Bj}) dfree(h, p);
+    // fixed-point scale for the F row sums: beta * max_row * 2^bits < 2^62
+    {
+        double bound = h->beta * (double)h->max_row;
+        int bits = 52;
+        if (bound > 0) {
+            int ex = 0;
+            frexp(bound, &ex); // bound < 2^ex
+            bits = 61 - ex;
+            if (bits > 1000) bits = 1000;
+        }
+        h->fp_bits = bits;
+        h->fp_scale = ldexp(1.0, bits);
+        h->fp_inv = ldexp(1.0, -bits);
+    }
+    return CUALIGN_OK;
+}
+
+cualign_status ensure_sq_pos(cualign_bp *h)
+{
+    if (h->sq_pos || h->nsq == 0) return CUALIGN_OK;
+    KScope ks(h, CUALIGN_K_INIT);
+    CA_TRY(dalloc(h, &h->sq_pos, (size_t)h->nsq));
+    k_sq_pos<<<grid_for(h->nsq, 256, h->num_sms * 16), 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->Srp,
+                                                                            h->sq_rp, h->Scol, h->sq_pos);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
+} // namespace cualign

@@ -1,0 +1,174 @@
+// internal.cuh -- shared internals of libcualign_bp (CUDA, sm_100a).
+// Not part of the ABI; the ABI is include/cualign_bp.h.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <stdarg.h>
+#include <string>
+#include <vector>
+
+#include "../../include/cualign_bp.h"
+
+namespace cualign {
+
+// ------------------------------------------------------------------ errors
+void set_error(const char *fmt, ...);
+void clear_error();
+
+#define CA_CUDA(call)                                                              \
+    do {                                                                           \
+        cudaError_t _e = (call);                                                   \
+        if (_e != cudaSuccess) {                                                   \
+            ::cualign::set_error("%s:%d: %s: %s", __FILE__, __LINE__, #call,       \
+                                 cudaGetErrorString(_e));                          \
+            return _e == cudaErrorMemoryAllocation ? CUALIGN_ENOMEM : CUALIGN_ECUDA; \
+        }                                                                          \
+    } while (0)
+
+#define CA_TRY(call)                                  \
+    do {                                              \
+        cualign_status _s = (call);                   \
+        if (_s != CUALIGN_OK) return _s;              \
+    } while (0)
+
+// ------------------------------------------------------------- L structure
+// Device layout of the candidate graph L (row a1 of SURVEY §8):
+//   La, Lb, w   canonical (a, b)-sorted edge list (edge id = index)
+//   Arow        A-side rows: edges of A vertex a are Arow[a] .. Arow[a+1]-1
+//   Bptr/Bedge  B-side incidence: Bedge[Bptr[b] .. Bptr[b+1]-1] = edge ids
+//               of B vertex b, ascending
+struct LDev {
+    int32_t nA = 0, nB = 0;
+    int64_t m = 0;
+    int32_t *La = nullptr, *Lb = nullptr;
+    double *w = nullptr;
+    int64_t *Arow = nullptr, *Bptr = nullptr;
+    int32_t *Bedge = nullptr;
+};
+
+// Device-side round bookkeeping (persistent across rounds: best).
+struct RoundDev {
+    unsigned int flag[2][2];      // [round parity][instance]: a match happened
+    int rounds[2];
+    unsigned long long overlap[2];
+    unsigned long long card[2];
+    double weight[2];
+    double best_score;
+    int best_iter;
+    int improved;
+    int source;
+    int pad;
+    cualign_round_info info;
+};
+
+struct EventPair {
+    cudaEvent_t a, b;
+};
+
+} // namespace cualign
+
+struct cualign_bp {
+    int dev = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    double alpha = 0, beta = 0, gamma = 1;
+    uint32_t flags = 0;
+    int num_sms = 148;
+
+    cualign::LDev L;
+
+    // S: full CSR over edge ids, and the square layout
+    int64_t s = 0, nsq = 0, max_row = 0;
+    int64_t *Srp = nullptr;      // m+1
+    int32_t *Scol = nullptr;     // s
+    int64_t *sq_rp = nullptr;    // m+1: squares {e<f} of row e are sq_rp[e]..sq_rp[e+1]-1
+    int2 *sq_ef = nullptr;       // nsq: (e, f), e < f, sorted by (e, f)
+    double2 *sq_val = nullptr;   // nsq: (S^p_ef, S^p_fe)
+    longlong2 *sq_pos = nullptr; // nsq: (pos(e,f), pos(f,e)) in the CSR; built lazily
+
+    // fixed-point accumulator of the F row sums (fast mode)
+    int fp_bits = 0;
+    double fp_scale = 1.0, fp_inv = 1.0;
+
+    // per-edge state (Alg. 2 l.5, :158); d^p is never used (reading Z16)
+    double *yc = nullptr, *zc = nullptr, *yp = nullptr, *zp = nullptr;
+    double *d = nullptr, *u = nullptr;
+    unsigned long long *tacc = nullptr; // fast mode: sum_f F_ef in fixed point
+    double *texact = nullptr;           // exact mode: sum_f F_ef, oracle order
+    double *Ffull = nullptr;            // exact mode: F in CSR order
+    double2 *Atop = nullptr, *Btop = nullptr; // per-vertex (max1, max2)
+    int32_t p = 0;
+
+    // matching (two instances: y and z)
+    int32_t *candA = nullptr, *candB = nullptr, *mateA = nullptr, *mateB = nullptr;
+    int32_t *best_mate = nullptr;
+    double *partial_w = nullptr;
+    int match_grid = 0, match_block = 256;
+    cualign::RoundDev *rd = nullptr;
+    cualign_round_info last_info{};
+    bool have_info = false;
+
+    // diagnostics
+    bool timing = false;
+    int64_t launches = 0;
+    int64_t class_launches[CUALIGN_NUM_KERNEL_CLASSES] = {};
+    std::vector<cualign::EventPair> events[CUALIGN_NUM_KERNEL_CLASSES];
+    std::vector<cudaEvent_t> event_pool;
+    double class_ms[CUALIGN_NUM_KERNEL_CLASSES] = {};
+
+    std::vector<std::pair<void *, size_t>> allocs;
+    int64_t device_bytes = 0;
+};
+
+namespace cualign {
+
+// --------------------------------------------------------------- memory
+cualign_status dmalloc(cualign_bp *h, void **p, size_t bytes);
+template <class T>
+inline cualign_status dalloc(cualign_bp *h, T **p, size_t n)
+{
+    return dmalloc(h, reinterpret_cast<void **>(p), n * sizeof(T));
+}
+void dfree(cualign_bp *h, void *p);
+void dfree_all(cualign_bp *h);
+
+// ------------------------------------------------------- launch accounting
+struct KScope {
+    cualign_bp *h;
+    int cls;
+    cudaEvent_t b = nullptr;
+    KScope(cualign_bp *h_, int cls_);
+    ~KScope();
+};
+
+// ------------------------------------------------------------ subsystems
+// init.cu
+cualign_status build_L(cualign_bp *h, LDev &L, const cualign_edges *E, bool device_ptrs,
+                       bool validate, int32_t nA, int32_t nB);
+cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualign_graph *B,
+                             const cualign_edges *E);
+cualign_status ensure_sq_pos(cualign_bp *h);
+
+// bp.cu
+cualign_status bp_fsum(cualign_bp *h);                 // t <- sum_f F(S^p) (init / set_state)
+cualign_status bp_iterate(cualign_bp *h, int32_t n);   // Alg. 2 l.9-16, n times
+cualign_status bp_scatter_Sp(cualign_bp *h, double *Sfull_dev);        // squares -> CSR
+cualign_status bp_gather_Sp(cualign_bp *h, const double *Sfull_dev);   // CSR -> squares
+
+// match.cu
+cualign_status match_setup(cualign_bp *h);
+cualign_status match_round(cualign_bp *h);  // a7 + a8 on the device
+cualign_status match_standalone(cualign_bp *h, const double *x_dev, int32_t *rounds);
+
+// helpers
+inline int grid_for(int64_t n, int block, int max_blocks)
+{
+    int64_t g = (n + block - 1) / block;
+    if (g < 1) g = 1;
+    if (g > max_blocks) g = max_blocks;
+    return (int)g;
+}
+
+} // namespace cualign

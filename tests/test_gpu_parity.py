@@ -1,0 +1,374 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, element by
+element, on the same seeded inputs.
+
+Bars (BASELINE.json:north_star):
+  * S (row pointers, columns): bit-exact.
+  * fp64 messages y^c, z^c, y^p, z^p, d, S^p: |gpu - oracle|_inf <= 1e-9 *
+    max(|oracle|_inf, 1) every iteration (fast mode); bit-exact in
+    CUALIGN_FLAG_EXACT mode and in the integer regime (P6).
+  * matchings and integer overlap counts: bit-exact given identical messages.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from oracle import Oracle, gamma_power
+from synth import make_config, random_candidates, complete_candidates
+from tests.util import tiny_instance, graph_from_edges, load_golden, golden_instance
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-9
+
+
+@pytest.fixture(scope="module")
+def ca():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_sc_xiangkfah23_b200 as ca
+    ca.load_library()
+    return ca
+
+
+def rel_err(got, want):
+    scale = max(float(np.max(np.abs(want))) if want.size else 0.0, 1.0)
+    return float(np.max(np.abs(got - want))) / scale if want.size else 0.0
+
+
+def assert_state_close(g, o, tol=TOL, keys=("d", "yc", "zc", "yp", "zp", "Sp"), where=""):
+    for k in keys:
+        e = rel_err(g[k], o[k])
+        assert e <= tol, f"{where} {k}: rel err {e:.3e} > {tol}"
+
+
+def assert_state_equal(g, o, keys=("d", "yc", "zc", "yp", "zp", "Sp"), where=""):
+    for k in keys:
+        bad = np.nonzero(g[k] != o[k])[0]
+        assert bad.size == 0, f"{where} {k}: {bad.size} differ, first {bad[:5]} {g[k][bad[:3]]} vs {o[k][bad[:3]]}"
+
+
+INSTANCES = {
+    "T": lambda: make_config("T"),
+    "P10": lambda: make_config("P", scale=0.1),
+    "O005": lambda: make_config("O", scale=0.005),
+}
+
+
+# ---------------------------------------------------------------- a2: S build
+@pytest.mark.parametrize("name", ["T", "P10", "O005"])
+def test_S_bit_exact(ca, name):
+    inst = INSTANCES[name]()
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma) as h:
+        rp, col = h.get_S()
+        orp, ocol, _ = o.get_S()
+        assert np.array_equal(rp, orp)
+        assert np.array_equal(col, ocol)
+        sz = h.sizes()
+        assert sz["s"] == o.s and sz["squares"] * 2 == o.s
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_S_bit_exact_tiny_and_ragged(ca, seed):
+    A, B, L, _ = tiny_instance(seed, n=9, n_edges=14, k=1 + seed % 5, n_b=5 + seed)
+    o = Oracle(A, B, L, 1.0, 2.0)
+    with ca.CuAlignBP(A, B, L, 1.0, 2.0, 0.9) as h:
+        rp, col = h.get_S()
+        orp, ocol, _ = o.get_S()
+        assert np.array_equal(rp, orp) and np.array_equal(col, ocol)
+
+
+def test_S_hub_rows_longer_than_a_warp(ca):
+    """A star centre with 100 neighbours in A and B and complete-ish L: rows of
+    S much longer than 32 and neighbour lists spanning many warp chunks."""
+    n = 101
+    edges = [(0, j) for j in range(1, n)] + [(j, j + 1) for j in range(1, n - 1)]
+    A = graph_from_edges(n, edges)
+    B = graph_from_edges(n, edges)
+    rng = np.random.default_rng(3)
+    L = random_candidates(n, n, 40, rng, truth=np.arange(n))
+    o = Oracle(A, B, L, 1.0, 2.0)
+    with ca.CuAlignBP(A, B, L, 1.0, 2.0, 0.9) as h:
+        rp, col = h.get_S()
+        orp, ocol, _ = o.get_S()
+        assert np.array_equal(rp, orp) and np.array_equal(col, ocol)
+        assert np.max(np.diff(rp)) > 64
+
+
+# ------------------------------------------------------- a3-a6: BP iteration
+def _run_both(ca, inst, n_iter, flags=0, gamma=None, alpha=None, beta=None, check=None):
+    alpha = inst.alpha if alpha is None else alpha
+    beta = inst.beta if beta is None else beta
+    gamma = inst.gamma if gamma is None else gamma
+    oflags = (oracle.OTHERMAX_LITERAL if flags & ca.FLAG_OTHERMAX_LITERAL else 0) | \
+             (oracle.ROUND_DAMPED if flags & ca.FLAG_ROUND_DAMPED else 0)
+    o = Oracle(inst.A, inst.B, inst.L, alpha, beta, oflags)
+    h = ca.CuAlignBP(inst.A, inst.B, inst.L, alpha, beta, gamma, flags)
+    for p in range(1, n_iter + 1):
+        o.step_gamma(gamma)
+        h.iterate(1)
+        check(p, h.get_state(), o.get_state(), o, h)
+    return o, h
+
+
+@pytest.mark.parametrize("name,n_iter", [("T", 20), ("P10", 30), ("O005", 10)])
+def test_fast_mode_trajectory_within_1e9(ca, name, n_iter):
+    inst = INSTANCES[name]()
+
+    def check(p, g, o, *_):
+        assert_state_close(g, o, where=f"{name} p={p}")
+
+    o, h = _run_both(ca, inst, n_iter, check=check)
+    h.close()
+
+
+@pytest.mark.parametrize("name,n_iter", [("T", 20), ("P10", 15)])
+@pytest.mark.parametrize("literal", [False, True])
+def test_exact_mode_trajectory_bitwise(ca, name, n_iter, literal):
+    inst = INSTANCES[name]()
+    flags = ca.FLAG_EXACT | (ca.FLAG_OTHERMAX_LITERAL if literal else 0)
+
+    def check(p, g, o, *_):
+        assert_state_equal(g, o, where=f"{name} p={p}")
+
+    o, h = _run_both(ca, inst, n_iter, flags=flags, check=check)
+    h.close()
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_integer_regime_fast_mode_bitwise(ca, seed):
+    """P6: gamma = 1, integer alpha, beta, w: all values are integers, exact in
+    any summation order -> the fast path equals the oracle bit for bit."""
+    inst = make_config("T", seed=77 + seed)
+    inst.L.w[:] = np.random.default_rng(seed).integers(1, 5, size=inst.L.m).astype(np.float64)
+
+    def check(p, g, o, oo, hh):
+        assert_state_equal(g, o, where=f"p={p}")
+        ri = hh.round()
+        ro = oo.round()
+        for k in ("card_y", "card_z", "overlap_y", "overlap_z", "source", "improved", "best_iter"):
+            assert ri[k] == ro[k], (p, k, ri[k], ro[k])
+        for k in ("score_y", "score_z", "weight_y", "weight_z", "best_score"):
+            assert ri[k] == ro[k], (p, k)
+
+    o, h = _run_both(ca, inst, 12, gamma=1.0, alpha=2.0, beta=3.0, check=check)
+    mate_g, _ = h.get_best()
+    mate_o, _, _ = o.get_best()
+    assert np.array_equal(mate_g, mate_o)
+    h.close()
+
+
+@pytest.mark.parametrize("name", ["P10", "O005"])
+def test_one_step_parity_from_injected_state(ca, name):
+    """set_state a random (y^p, z^p, S^p) into both, one iteration, compare."""
+    inst = INSTANCES[name]()
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    rng = np.random.default_rng(11)
+    m, s = o.m, o.s
+    yp, zp = rng.normal(size=m) * 3, rng.normal(size=m) * 3
+    Sp = rng.normal(size=s) * 2
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma) as h:
+        for p in (7, 40):
+            o.set_state(yp, zp, Sp, p)
+            h.set_state(yp, zp, Sp, p)
+            o.step_gamma(inst.gamma)
+            h.iterate(1)
+            g, oo = h.get_state(), o.get_state()
+            assert_state_close(g, oo, tol=1e-12, where=f"p={p}")
+            assert g["p"] == oo["p"] == p + 1
+
+
+def test_get_state_roundtrip(ca):
+    inst = make_config("T")
+    rng = np.random.default_rng(5)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L) as h:
+        Sp = rng.normal(size=h.s)
+        yp, zp = rng.normal(size=h.m), rng.normal(size=h.m)
+        h.set_state(yp, zp, Sp, 3)
+        g = h.get_state()
+        assert np.array_equal(g["Sp"], Sp) and np.array_equal(g["yp"], yp) and g["p"] == 3
+
+
+# ------------------------------------------------------------ a7: matching
+@pytest.mark.parametrize("seed", range(12))
+@pytest.mark.parametrize("weights", ["ties", "ties_signed", "uniform"])
+def test_matching_bit_exact_vs_greedy(ca, seed, weights):
+    rng = np.random.default_rng(seed)
+    n_a, n_b = int(rng.integers(5, 300)), int(rng.integers(5, 300))
+    L = random_candidates(n_a, n_b, int(rng.integers(1, 12)), rng, weights=weights)
+    o = Oracle(graph_from_edges(n_a, []), graph_from_edges(n_b, []), L, 1.0, 0.0)
+    want, _ = o.greedy(L.w)
+    ma, mb, rounds = ca.match(L, n_a, n_b, L.w)
+    assert np.array_equal(ma, want)
+    # mate_b consistent with mate_a
+    for a in range(n_a):
+        if ma[a] >= 0:
+            assert mb[L.b[ma[a]]] == ma[a]
+    assert np.sum(mb >= 0) == np.sum(ma >= 0)
+
+
+def test_matching_large_random(ca):
+    rng = np.random.default_rng(0)
+    n_a, n_b = 20000, 15000
+    L = random_candidates(n_a, n_b, 12, rng, weights="uniform")
+    o = Oracle(graph_from_edges(n_a, []), graph_from_edges(n_b, []), L, 1.0, 0.0)
+    for x in (L.w, np.round(L.w * 4) / 4):  # generic and massively tied weights
+        want, _ = o.greedy(x)
+        ma, _, rounds = ca.match(L, n_a, n_b, x)
+        assert np.array_equal(ma, want)
+
+
+def test_matching_empty_and_degenerate(ca):
+    L = random_candidates(4, 4, 2, np.random.default_rng(1))
+    ma, mb, _ = ca.match(L, 4, 4, -np.ones(L.m))   # nothing eligible
+    assert np.all(ma == -1) and np.all(mb == -1)
+    from synth import Candidates
+    E = Candidates(3, 3, np.zeros(0, np.int32), np.zeros(0, np.int32), np.zeros(0))
+    ma, mb, _ = ca.match(E, 3, 3, np.zeros(0))
+    assert np.all(ma == -1)
+
+
+# ------------------------------------------------ a7 + a8: round and best
+@pytest.mark.parametrize("name,n_iter", [("T", 20), ("P10", 20)])
+def test_round_matches_oracle(ca, name, n_iter):
+    """Rounding on the GPU's own messages vs oracle rounding on the SAME
+    messages (state injected), so matchings must be bit-exact."""
+    inst = INSTANCES[name]()
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma) as h:
+        for p in range(1, n_iter + 1):
+            h.iterate(1)
+            r = h.round()
+            g = h.get_state()
+            my, cy = o.greedy(g["yc"])
+            mz, cz = o.greedy(g["zc"])
+            ey, ez = o.evaluate(my), o.evaluate(mz)
+            assert r["card_y"] == cy and r["card_z"] == cz
+            assert r["overlap_y"] == ey["overlap"] and r["overlap_z"] == ez["overlap"]
+            assert abs(r["weight_y"] - ey["weight"]) <= 1e-12 * max(1, ey["weight"])
+            assert abs(r["score_z"] - ez["score"]) <= 1e-12 * max(1, ez["score"])
+            assert r["iter"] == p
+
+
+@pytest.mark.parametrize("name", ["T", "P10"])
+def test_end_to_end_align_exact_mode(ca, name):
+    inst = INSTANCES[name]()
+    n_iter = 20
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    oinfos = o.align(n_iter, inst.gamma)
+    mate, info, infos = ca.align(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma,
+                                 n_iter=n_iter, flags=ca.FLAG_EXACT)
+    for gi, oi in zip(infos, oinfos):
+        for k in ("card_y", "card_z", "overlap_y", "overlap_z", "source", "improved", "best_iter",
+                  "score_y", "score_z", "weight_y", "weight_z", "best_score"):
+            assert gi[k] == oi[k], (gi["iter"], k, gi[k], oi[k])
+    omate, obest, oit = o.get_best()
+    assert np.array_equal(mate, omate) and info["best_score"] == obest and info["best_iter"] == oit
+
+
+def test_end_to_end_align_fast_mode(ca):
+    inst = make_config("T")
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    oinfos = o.align(inst.n_iter, inst.gamma)
+    mate, info, infos = ca.align(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma,
+                                 n_iter=inst.n_iter)
+    omate, obest, oit = o.get_best()
+    assert abs(info["best_score"] - obest) <= 1e-9 * max(1.0, abs(obest))
+    if not np.array_equal(mate, omate):  # only a near-tie may flip the choice
+        gaps = [abs(oi["score_y"] - oi["score_z"]) for oi in oinfos]
+        assert min(gaps) < 1e-9 * max(1.0, abs(obest))
+
+
+# ------------------------------------------------------------ golden W1/W2
+def test_W1_on_gpu(ca):
+    from fractions import Fraction
+    g = load_golden("W1.json")
+    A, B, L = golden_instance(g)
+    with ca.CuAlignBP(A, B, L, g["alpha"], g["beta"], float(Fraction(g["gamma"]))) as h:
+        rp, col = h.get_S()
+        for it in g["iterations"]:
+            h.iterate(1)
+            st = h.get_state()
+            for key in ("d", "yc", "zc", "yp", "zp"):
+                assert list(st[key]) == [float(Fraction(x)) for x in it[key]], (it["p"], key)
+            vals = []
+            for e, f in g["S_pairs"]:
+                row = list(col[rp[e]:rp[e + 1]])
+                vals.append(st["Sp"][rp[e] + row.index(f)])
+            assert vals == [float(Fraction(x)) for x in it["Sp"]]
+            r = h.round()
+            assert r["score"] == 3.5 and r["overlap_y"] == 1
+        _, info = h.get_best()
+        assert info["best_score"] == 3.5 and info["best_iter"] == 1
+
+
+@pytest.mark.parametrize("literal", [False, True])
+def test_W2_on_gpu(ca, literal):
+    g = load_golden("W2.json")
+    A, B, L = golden_instance(g)
+    flags = ca.FLAG_OTHERMAX_LITERAL if literal else 0
+    with ca.CuAlignBP(A, B, L, g["alpha"], g["beta"], 1.0, flags) as h:
+        for it in g["literal" if literal else "maxplus"]:
+            h.iterate(1)
+            st = h.get_state()
+            assert list(st["yc"]) == [float(x) for x in it["yc"]]
+            assert list(st["zc"]) == [float(x) for x in it["zc"]]
+            h.round()
+        _, info = h.get_best()
+        assert info["best_score"] == 5 and info["best_iter"] == 1
+
+
+# --------------------------------------------------------------- edge cases
+def test_empty_L_and_edgeless_graphs(ca):
+    from synth import Candidates
+    A = graph_from_edges(3, [])
+    B = graph_from_edges(4, [])
+    E = Candidates(3, 4, np.zeros(0, np.int32), np.zeros(0, np.int32), np.zeros(0))
+    with ca.CuAlignBP(A, B, E) as h:
+        h.iterate(3)
+        r = h.round()
+        assert r["card_y"] == 0 and r["score"] == 0.0
+        assert h.sizes()["s"] == 0
+
+
+def test_n_a_differs_from_n_b(ca):
+    inst = make_config("O", scale=0.002)
+    assert inst.A.n != inst.B.n
+    o = Oracle(inst.A, inst.B, inst.L, 1.0, 2.0)
+    oinfos = o.align(5, 0.99)
+    mate, info, infos = ca.align(inst.A, inst.B, inst.L, 1.0, 2.0, 0.99, n_iter=5, flags=ca.FLAG_EXACT)
+    assert info["best_score"] == o.get_best()[1]
+
+
+@pytest.mark.parametrize("bad", ["unsorted", "duplicate", "range", "asym", "selfloop", "nan", "alpha", "gamma"])
+def test_validation_rejects_bad_inputs(ca, bad):
+    inst = make_config("T", scale=0.2)
+    A, B, L = inst.A, inst.B, inst.L
+    kw = dict(alpha=1.0, beta=2.0, gamma=0.9)
+    import copy
+    L2 = copy.deepcopy(L)
+    A2 = copy.deepcopy(A)
+    if bad == "unsorted":
+        L2.a, L2.b = L2.a[::-1].copy(), L2.b[::-1].copy()
+    elif bad == "duplicate":
+        L2.a[1], L2.b[1] = L2.a[0], L2.b[0]
+    elif bad == "range":
+        L2.b[-1] = B.n + 5
+    elif bad == "asym":
+        A2.col = A2.col.copy()
+        i = int(np.argmax(np.diff(A2.rowptr) > 1))
+        A2.col[A2.rowptr[i]] = (A2.col[A2.rowptr[i]] + 1) % A2.n  # breaks symmetry/order somewhere
+    elif bad == "selfloop":
+        A2.col = A2.col.copy()
+        A2.col[A2.rowptr[0]] = 0
+    elif bad == "nan":
+        L2.w = L2.w.copy()
+        L2.w[3] = np.nan
+    elif bad == "alpha":
+        kw["alpha"] = -1.0
+    elif bad == "gamma":
+        kw["gamma"] = 1.5
+    with pytest.raises(ca.CuAlignError) as ei:
+        ca.CuAlignBP(A2, B, L2, **kw)
+    assert ei.value.status == -1
