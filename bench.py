@@ -1,0 +1,396 @@
+#!/usr/bin/env python
+"""Benchmark of the NetAlignBP + matching hot path (BASELINE.json:metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+A "step" is one pass of the per-iteration hot path of Alg. 2:
+BP update a3-a6 (iterate) + rounding a7-a8 (two matchings, evaluate, best) on
+config O (BASELINE.json:configs[2], ontology-shaped, ~5e6 L edges, ~1e8 nnz(S)),
+with S (a2) and the L layouts (a1) built once before timing (they are
+"executed only once").  `value` = steps per second =
+BP iterations/s; squares/s and the end-to-end align time (init + 100
+iterations + best, host buffers, through the C ABI) are reported beside it.
+
+Prints ONE JSON line on rank 0.  See DESIGN.md "Measurement".
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import platform
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import numpy as np
+
+METRIC = "BP iterations/sec and squares/sec; end-to-end align time at 1/2/4/8 B200"
+UNIT = "iterations/s"
+# algorithmic bytes: (2*sigma + 4) per nonzero of S, (9*sigma + 8) per L edge
+SIGMA = 8
+BYTES_PER_NZ = 2 * SIGMA + 4
+BYTES_PER_EDGE = 9 * SIGMA + 8
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def read_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as fh:
+            pk = json.load(fh)
+        return float(pk["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons via NVML while the timed region runs."""
+
+    def __init__(self, device_index=0, period_s=0.005):
+        self.samples = []
+        self.reasons = set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nv = pynvml
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+            self._ok = True
+        except Exception as e:  # pragma: no cover
+            log("clock sampler unavailable:", e)
+        self.period = period_s
+        self._t = None
+
+    def _names(self, mask):
+        nv = self._nv
+        table = {
+            "gpu_idle": getattr(nv, "nvmlClocksEventReasonGpuIdle", 0x1),
+            "applications_clocks_setting": getattr(nv, "nvmlClocksEventReasonApplicationsClocksSetting", 0x2),
+            "sw_power_cap": getattr(nv, "nvmlClocksEventReasonSwPowerCap", 0x4),
+            "hw_slowdown": getattr(nv, "nvmlClocksEventReasonHwSlowdown", 0x8),
+            "sync_boost": getattr(nv, "nvmlClocksEventReasonSyncBoost", 0x10),
+            "sw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonSwThermalSlowdown", 0x20),
+            "hw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonHwThermalSlowdown", 0x40),
+            "hw_power_brake_slowdown": getattr(nv, "nvmlClocksEventReasonHwPowerBrakeSlowdown", 0x80),
+        }
+        return [k for k, v in table.items() if mask & v]
+
+    def _run(self):
+        nv = self._nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM))
+                try:
+                    mask = nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+                except AttributeError:
+                    mask = nv.nvmlDeviceGetCurrentClocksThrottleReasons(self._h)
+                for r in self._names(mask):
+                    if r != "gpu_idle":
+                        self.reasons.add(r)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def start(self):
+        if self._ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+
+    def stop(self):
+        if self._t:
+            self._stop.set()
+            self._t.join()
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": float(statistics.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def dist_setup(args):
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch.distributed as dist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        backend = "gloo" if args.impl == "reference" else "nccl"
+        if backend == "nccl":
+            import torch
+            torch.cuda.set_device(local)
+        dist.init_process_group(backend=backend)
+    return rank, world, local
+
+
+def barrier(world):
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def max_over_ranks(x, world, device=None):
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def oracle_rate(scale, n_iter, full_work):
+    """Oracle (single thread, fp64) on config O generated at `scale`: create +
+    n_iter x (step + round).  Returns (iterations/s extrapolated to the full
+    workload linearly in s + m, detail dict)."""
+    import oracle
+    from oracle import Oracle
+    from synth import make_config
+    inst = make_config("O", scale=scale)
+    t0 = time.perf_counter()
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    t1 = time.perf_counter()
+    for _ in range(n_iter):
+        o.step_gamma(inst.gamma)
+        o.round()
+    t2 = time.perf_counter()
+    per_iter = (t2 - t1) / n_iter
+    work = o.s + o.m
+    rate_sample = 1.0 / per_iter
+    rate_full = rate_sample * work / full_work
+    return rate_full, dict(scale=scale, m=o.m, s=o.s, iters=n_iter, create_s=t1 - t0,
+                           per_iter_s=per_iter, rate_sample=rate_sample)
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the oracle as it stands on the host cores (no
+    reference implementation exists)."""
+    if rank != 0:
+        return
+    from synth import O_full_work
+    full_m, full_s = O_full_work()
+    full_work = full_m + full_s
+    import oracle
+    from oracle import Oracle
+    from synth import make_config
+    scale = args.ref_scale
+    inst = make_config("O", scale=scale)
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    for _ in range(args.warmup):
+        o.step_gamma(inst.gamma)
+        o.round()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        o.step_gamma(inst.gamma)
+        o.round()
+    dt = time.perf_counter() - t0
+    rate_sample = args.steps / dt
+    value = rate_sample * (o.s + o.m) / full_work
+    sample = (f"config O generator at scale {scale} (m={o.m}, s={o.s}); {args.steps} steps of "
+              f"oracle step+round, single thread; rate extrapolated linearly in (s+m) to full O "
+              f"(m={full_m}, s={full_s})")
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000.0 / value,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": "O: ontology-shaped pair (BASELINE.json configs[2])", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=300)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="O")
+    ap.add_argument("--scale", type=float, default=1.0)
+    ap.add_argument("--e2e-iters", type=int, default=100)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-scale", type=float, default=0.2)
+    ap.add_argument("--ref-scale", type=float, default=0.05)
+    ap.add_argument("--exact", action="store_true", help="CUALIGN_FLAG_EXACT (oracle-order sums)")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        ap.error("--warmup must be >= 3")
+    rank, world, local = dist_setup(args)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        barrier(world)
+        return
+
+    import torch
+    import paper_conf_sc_xiangkfah23_b200 as ca
+    from synth import make_config
+
+    dev = local
+    torch.cuda.set_device(dev)
+    t_gen = time.perf_counter()
+    inst = make_config(args.config, scale=args.scale, seed=None)
+    t_gen = time.perf_counter() - t_gen
+    log(f"[rank {rank}] generated {args.config} (scale {args.scale}) in {t_gen:.1f}s: "
+        f"n_A={inst.A.n} n_B={inst.B.n} m={inst.L.m}")
+    stream = torch.cuda.current_stream()
+    flags = ca.FLAG_TIMING | (ca.FLAG_EXACT if args.exact else 0)
+
+    # ---------------------------------------------------------------- init
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    h = ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags=flags,
+                     device=dev, stream=stream)
+    torch.cuda.synchronize()
+    init_s = time.perf_counter() - t0
+    sz = h.sizes()
+    m, s, squares = sz["m"], sz["s"], sz["squares"]
+    log(f"[rank {rank}] init {init_s:.3f}s s={s} squares={squares} max_row={sz['max_row']} "
+        f"fp_bits={sz['fixed_point_bits']} device_bytes={sz['device_bytes']/1e9:.2f}GB")
+
+    # ------------------------------------------------------------- warmup
+    for _ in range(args.warmup):
+        h.iterate(1)
+        h.round(sync=False)
+    torch.cuda.synchronize()
+    h.stats(reset=True)
+    barrier(world)
+
+    # --------------------------------------------------------- timed region
+    sampler = ClockSampler(dev)
+    sampler.start()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    barrier(world)
+    ev0.record(stream)
+    for _ in range(args.steps):
+        h.iterate(1)
+        h.round(sync=False)
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    barrier(world)
+    clocks = sampler.stop()
+    elapsed_ms = ev0.elapsed_time(ev1)
+    elapsed_ms = max_over_ranks(elapsed_ms, world, device=f"cuda:{dev}")
+    st = h.stats(reset=True)
+    _, info = h.get_best()
+
+    steps_total = args.steps * world
+    value = steps_total / (elapsed_ms / 1e3)
+    ms_per_step = elapsed_ms / args.steps
+    cls_ms = st["class_ms"]
+    cls_n = st["class_launches"]
+    sq_ms = cls_ms["square"] / max(cls_n["square"], 1)
+    bp_ms = (cls_ms["top2"] + cls_ms["edge"] + cls_ms["square"] + cls_ms["rowsum"]) / args.steps
+    round_ms = cls_ms["match"] / max(cls_n["match"], 1)
+    peak, peak_src = read_peaks()
+    sq_bytes = BYTES_PER_NZ * s                    # algorithmic bytes of one square-pass launch
+    sq_gbs = sq_bytes / (sq_ms * 1e-3) / 1e9 if sq_ms > 0 else 0.0
+    it_bytes = BYTES_PER_NZ * s + BYTES_PER_EDGE * m
+    it_gbs = it_bytes / (bp_ms * 1e-3) / 1e9 if bp_ms > 0 else 0.0
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "square_traffic.json")
+    if os.path.exists(tpath):
+        try:
+            with open(tpath) as fh:
+                tj = json.load(fh)
+            if tj.get("s") == s:
+                traffic = tj.get("dram_bytes_per_launch")
+        except Exception:
+            pass
+
+    # ------------------------------------------------------------------ e2e
+    e2e = None
+    align_time_s = None
+    if not args.no_e2e:
+        # pinned host buffers, the public API (C ABI), H2D of all inputs and
+        # D2H of every round's info and of the best matching inside the region
+        def pin(x):
+            return torch.from_numpy(np.ascontiguousarray(x)).pin_memory()
+
+        class G:  # graph with pinned arrays
+            pass
+
+        GA, GB, GL = G(), G(), G()
+        GA.n, GA.rowptr, GA.col = inst.A.n, pin(inst.A.rowptr), pin(inst.A.col)
+        GB.n, GB.rowptr, GB.col = inst.B.n, pin(inst.B.rowptr), pin(inst.B.col)
+        GL.a, GL.b, GL.w = pin(inst.L.a), pin(inst.L.b), pin(inst.L.w)
+        h2d = sum(int(t.numel() * t.element_size()) for t in
+                  (GA.rowptr, GA.col, GB.rowptr, GB.col, GL.a, GL.b, GL.w))
+        del h
+        torch.cuda.empty_cache()
+        torch.cuda.synchronize()
+        barrier(world)
+        t0 = time.perf_counter()
+        mate, binfo, infos = ca.align(GA, GB, GL, inst.alpha, inst.beta, inst.gamma,
+                                      n_iter=args.e2e_iters, device=dev, stream=stream)
+        torch.cuda.synchronize()
+        align_time_s = max_over_ranks(time.perf_counter() - t0, world, device=f"cuda:{dev}")
+        import ctypes
+        d2h = args.e2e_iters * 112 + 4 * inst.A.n
+        e2e = {"value": args.e2e_iters * world / align_time_s, "unit": UNIT,
+               "h2d_bytes_per_step": h2d / args.e2e_iters, "d2h_bytes_per_step": d2h / args.e2e_iters,
+               "align_time_s": align_time_s, "iters": args.e2e_iters,
+               "best_score": binfo["best_score"], "best_iter": binfo["best_iter"]}
+    else:
+        del h
+
+    # --------------------------------------------------------- cpu baseline
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and args.config == "O":
+        try:
+            rate, det = oracle_rate(args.cpu_scale, 3, m + s)
+            cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
+                   "sample": (f"config O generator at scale {det['scale']} (m={det['m']}, s={det['s']}), "
+                              f"oracle create + {det['iters']} x (step + round) single-threaded fp64 "
+                              f"({det['per_iter_s']:.3f} s/iteration); extrapolated linearly in s+m to "
+                              f"full O (m={m}, s={s})"),
+                   "host": platform.processor() or platform.machine(), "nproc": os.cpu_count()}
+        except Exception as e:  # pragma: no cover
+            cpu = {"value": None, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": f"failed: {e}"}
+
+    if rank != 0:
+        return
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{args.config}: " + inst.meta["desc"], "scale": args.scale,
+                   "n_a": inst.A.n, "n_b": inst.B.n, "m": m, "s": s, "squares": squares,
+                   "alpha": inst.alpha, "beta": inst.beta, "gamma": inst.gamma,
+                   "parallelism": "replicas" if world > 1 else "single",
+                   "l2": "inputs larger than L2 (square layout %.2f GB vs 126 MB L2)" % (24 * squares / 1e9),
+                   "mode": "exact" if args.exact else "fast"},
+        "squares_per_s": squares * steps_total / (elapsed_ms / 1e3),
+        "bp_iters_per_s": 1e3 / bp_ms if bp_ms > 0 else None,
+        "round_ms": round_ms, "bp_ms": bp_ms, "init_s": init_s,
+        "roofline": {"bound": "hbm", "kernel": "k_square (a3+a5+a6 square pass)",
+                     "achieved": sq_gbs, "peak": peak, "unit": "GB/s", "frac": sq_gbs / peak,
+                     "traffic": traffic, "alg_bytes_per_launch": sq_bytes,
+                     "launch_ms": sq_ms, "peak_source": peak_src},
+        "iteration_roofline": {"achieved": it_gbs, "frac": it_gbs / peak, "alg_bytes": it_bytes,
+                               "bp_ms": bp_ms},
+        "kernel_ms_per_step": {k: v / args.steps for k, v in cls_ms.items() if v},
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": st["launches"],
+        "clocks": clocks,
+        "best_score": info["best_score"],
+    }
+    print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()

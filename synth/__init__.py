@@ -7,11 +7,11 @@ bipartite graphs L with the shapes of the paper's workloads
 Both the oracle (`oracle/`) and the CUDA path consume its arrays; neither
 imports the other.
 """
-from .graphs import (Graph, Candidates, csr_from_pairs, er_graph, chung_lu_graph,
+from .graphs import (Graph, Candidates, csr_from_pairs, er_graph, chung_lu_graph, small_world_power_law,
                      rmat_graph, permuted_noisy_copy, induced_subgraph,
                      knn_candidates, proxy_candidates, complete_candidates,
                      random_candidates)
-from .configs import CONFIGS, make_config, Instance
+from .configs import CONFIGS, make_config, Instance, O_full_work
 
 __all__ = ["Graph", "Candidates", "csr_from_pairs", "er_graph", "chung_lu_graph",
            "rmat_graph", "permuted_noisy_copy", "induced_subgraph", "knn_candidates",

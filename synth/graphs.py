@@ -363,3 +363,27 @@ def proxy_candidates(gb: Graph, anchor: np.ndarray, k: float, lam: float,
         b_out = np.concatenate([b_out, np.asarray(extra_b, dtype=np.int64)])
     w = _uniform01_open_low(rng, a_out.shape[0])
     return _finish_candidates(n_a, n_b, a_out, b_out, w)
+
+
+def small_world_power_law(n: int, h: int, n_random: int, tau: float,
+                          rng: np.random.Generator, max_deg_frac: float = 0.01) -> Graph:
+    """Clustered power-law graph: a ring lattice (each vertex joined to its h
+    nearest ring neighbours on each side: high clustering, like the local
+    structure of ontology / PPI networks) plus a Chung-Lu power-law layer of
+    n_random edges (hubs).  Vertices are relabelled randomly."""
+    base = np.arange(n, dtype=np.int64)
+    us, vs = [], []
+    for d in range(1, h + 1):
+        us.append(base)
+        vs.append((base + d) % n)
+    ring_u = np.concatenate(us) if us else np.zeros(0, dtype=np.int64)
+    ring_v = np.concatenate(vs) if vs else np.zeros(0, dtype=np.int64)
+    if n_random > 0:
+        cl = chung_lu_graph(n, n_random, tau, rng, max_deg_frac=max_deg_frac)
+        cu, cv = cl.edge_pairs()
+    else:
+        cu = cv = np.zeros(0, dtype=np.int64)
+    relabel = rng.permutation(n).astype(np.int64)
+    u = relabel[np.concatenate([ring_u, cu])]
+    v = relabel[np.concatenate([ring_v, cv])]
+    return csr_from_pairs(n, u, v)
