@@ -223,6 +223,7 @@ def main():
     ap.add_argument("--cpu-scale", type=float, default=0.2)
     ap.add_argument("--ref-scale", type=float, default=0.05)
     ap.add_argument("--exact", action="store_true", help="CUALIGN_FLAG_EXACT (oracle-order sums)")
+    ap.add_argument("--match-rounds", action="store_true", help="pointer-round matching schedule")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
@@ -244,7 +245,8 @@ def main():
     log(f"[rank {rank}] generated {args.config} (scale {args.scale}) in {t_gen:.1f}s: "
         f"n_A={inst.A.n} n_B={inst.B.n} m={inst.L.m}")
     stream = torch.cuda.current_stream()
-    flags = ca.FLAG_TIMING | (ca.FLAG_EXACT if args.exact else 0)
+    flags = ca.FLAG_TIMING | (ca.FLAG_EXACT if args.exact else 0) | \
+        (ca.FLAG_MATCH_ROUNDS if args.match_rounds else 0)
 
     # ---------------------------------------------------------------- init
     torch.cuda.synchronize()
@@ -388,6 +390,9 @@ def main():
         "gpu_launches": st["launches"],
         "clocks": clocks,
         "best_score": info["best_score"],
+        "last_round": {k: info[k] for k in ("iter", "card_y", "card_z", "overlap_y", "overlap_z",
+                                            "rounds_y", "rounds_z", "score")},
+        "match_schedule": "rounds" if args.match_rounds else "suitor",
     }
     print(json.dumps(line), flush=True)
 

@@ -64,6 +64,8 @@ typedef enum {
                                                default max-plus: om(e) = max(0, max_{f!=e} v_f) */
 #define CUALIGN_FLAG_ROUND_DAMPED     0x08u /* reading Z5 variant: round y^p, z^p instead of y^c, z^c */
 #define CUALIGN_FLAG_TIMING           0x10u /* record CUDA events around every kernel (diagnostics) */
+#define CUALIGN_FLAG_MATCH_ROUNDS     0x20u /* a7 schedule: synchronous pointer rounds (paper's Phase 1/2)
+                                               instead of the default Suitor proposals; same matching */
 
 /* Undirected simple graph: symmetric CSR, row i lists the
  * neighbours of i strictly increasing, no self loops (reading Z14).
@@ -111,7 +113,8 @@ typedef struct {
     double score;                 /* max(score_y, score_z) */
     double best_score;            /* bestScore after this round (starts at 0) */
     int64_t overlap_y, overlap_z; /* x'Sx/2: squares {e,f} with both e, f in M */
-    int32_t rounds_y, rounds_z;   /* pointer rounds the matchings took */
+    int32_t rounds_y, rounds_z;   /* matching work: successful proposals (Suitor schedule) or
+                                     pointer rounds (CUALIGN_FLAG_MATCH_ROUNDS) */
 } cualign_round_info;
 
 /* Sizes of an initialised handle. */
@@ -197,7 +200,8 @@ cualign_status cualign_bp_get_stats(cualign_bp *h, cualign_stats *stats, int32_t
  * order (x desc, edge id asc), only x > 0 eligible (readings Z6, Z7).  Writes
  * mate_a (n_A int32) and mate_b (n_B int32) host buffers (either may be NULL):
  * the matched edge id at each vertex or -1.  *rounds_out (may be NULL)
- * receives the number of pointer rounds.  L->w is ignored (may be NULL). */
+ * receives the matching work (see cualign_round_info.rounds_y).  L->w is
+ * ignored (may be NULL). */
 cualign_status cualign_match(const cualign_edges *L, int32_t n_a, int32_t n_b, const double *x,
                              const cualign_params *params, int32_t *mate_a, int32_t *mate_b,
                              int32_t *rounds_out);

@@ -6,7 +6,7 @@ the end-to-end `align` helper and the sharded (multi-GPU) driver.
 """
 from ._lib import (CuAlignBP, CuAlignError, match, load_library, version,
                    FLAG_DEVICE_PTRS, FLAG_EXACT, FLAG_OTHERMAX_LITERAL, FLAG_ROUND_DAMPED,
-                   FLAG_TIMING, EXPORTED, LIB_PATH, KERNEL_CLASS_NAMES)
+                   FLAG_TIMING, FLAG_MATCH_ROUNDS, EXPORTED, LIB_PATH, KERNEL_CLASS_NAMES)
 
 
 def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=0, stream=None):
@@ -23,4 +23,4 @@ def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=
 
 __all__ = ["CuAlignBP", "CuAlignError", "match", "align", "load_library", "version",
            "FLAG_DEVICE_PTRS", "FLAG_EXACT", "FLAG_OTHERMAX_LITERAL", "FLAG_ROUND_DAMPED",
-           "FLAG_TIMING", "EXPORTED", "LIB_PATH", "KERNEL_CLASS_NAMES"]
+           "FLAG_TIMING", "FLAG_MATCH_ROUNDS", "EXPORTED", "LIB_PATH", "KERNEL_CLASS_NAMES"]

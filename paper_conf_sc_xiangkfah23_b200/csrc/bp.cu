@@ -300,13 +300,13 @@ cualign_status bp_iterate(cualign_bp *h, int32_t n)
                 KScope ks(h, CUALIGN_K_TOP2);
                 const int64_t N = (int64_t)h->L.nA + h->L.nB;
                 const int64_t threads = (N + (32 / TOP2_G) - 1) / (32 / TOP2_G) * 32;
-                k_top2<<<grid_for(threads, 256, h->num_sms * 8), 256, 0, h->stream>>>(
+                k_top2<<<grid_for(threads, 256, 1 << 30), 256, 0, h->stream>>>(
                     h->L.nA, h->L.nB, h->L.Arow, h->L.Bptr, h->L.Bedge, h->yp, h->zp, h->Atop, h->Btop);
                 CA_CUDA(cudaGetLastError());
             }
             {
                 KScope ks(h, CUALIGN_K_EDGE);
-                const int grid = grid_for(m, 256, h->num_sms * 8);
+                const int grid = grid_for(m, 256, 1 << 30);
 #define EDGE_ARGS                                                                                    \
     m, h->L.La, h->L.Lb, h->L.w, h->alpha, g, hh, h->fp_inv, h->tacc, h->texact, h->Atop, h->Btop, \
         h->yp, h->zp, h->yc, h->zc, h->d, h->u

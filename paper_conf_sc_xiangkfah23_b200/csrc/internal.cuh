@@ -105,7 +105,8 @@ struct cualign_bp {
     int32_t *candA = nullptr, *candB = nullptr, *mateA = nullptr, *mateB = nullptr;
     int32_t *best_mate = nullptr;
     double *partial_w = nullptr;
-    int match_grid = 0, match_block = 256;
+    int match_grid = 0, match_block = 256, eval_grid = 1;
+    unsigned long long *match_work = nullptr; // proposals (suitor) or rounds, per instance
     cualign::RoundDev *rd = nullptr;
     cualign_round_info last_info{};
     bool have_info = false;

@@ -1,24 +1,29 @@
 // match.cu -- rows a7 (rounding by 1/2-approximate matching) and a8
 // (evaluate + best) of the hot path: Alg. 2 lines 17-24.
 //
-// Matching: the locally-dominant algorithm (Preis [24]) as
-// synchronous pointer rounds inside ONE persistent cooperative kernel that
-// matches y^c and z^c at the same time (two independent instances):
-//   init  every vertex (A and B side) points at its heaviest eligible
-//         neighbour under the strict order (x desc, edge id asc) (readings
-//         Z6, Z7) -- Phase 1's "candidate mate";
-//   M     an A vertex whose candidate's B endpoint points back is matched
-//         (a locally dominant edge); no atomics: a B vertex has exactly one
-//         candidate, so at most one A vertex can claim it;
-//   R     unmatched vertices whose candidate endpoint got matched re-point
-//         (Phase 2's "those neighbors will have to find new candidates");
-//   repeat until a round matches nothing.  grid.sync() separates phases, so
-//   the paper's Q_C / Q_N queues are not needed.  Under a strict total order
-//   the result is exactly the greedy matching (pin P9), so it is bit-exact
-//   against the oracle for identical message vectors.
-// Evaluate: weight(M) over the original w (Z9), overlap(M) = x'Sx/2 counted
-// on the square layout (each square {e<f} stored once at e), score = alpha w
-// + beta overlap (Eq. 1, :64-72), M_y wins ties, best on a strict > (Z8).
+// The paper rounds with the locally-dominant algorithm (
+// Preis [24], Halappanavar [10]).  Under a strict total order of the edges --
+// (x desc, edge id asc), readings Z6/Z7 -- every locally-dominant schedule
+// produces the same matching: the greedy one (pin P9).  Two schedules are
+// implemented; both are bit-exact against the oracle's sort-greedy:
+//
+//  * SUITOR (default).  Every vertex of V_A u V_B proposes to its heaviest
+//    eligible neighbour whose current suitor is lighter; a CAS on the
+//    neighbour's suitor slot (an edge id) installs the proposal and the
+//    displaced suitor -- now owned by the same thread -- proposes again
+//    (Manne & Halappanavar's Suitor algorithm, a lock-free form of the
+//    locally-dominant rule).  One kernel, no grid-wide barriers; the matched
+//    edges are the mutual suitor pairs.  y^c and z^c are matched in the same
+//    launch (two instances).
+//  * POINTER ROUNDS (CUALIGN_FLAG_MATCH_ROUNDS).  The paper's Phase 1 / Phase 2
+//    as synchronous rounds in one persistent cooperative kernel: every vertex
+//    points at its best eligible unmatched neighbour, mutual pointers match,
+//    vertices whose target got matched re-point; grid.sync() between phases
+//    replaces the Q_C / Q_N queues.  Kept for comparison (ablation).
+//
+// Evaluate: weight(M) over the original w (Z9), overlap(M) = x'Sx/2 counted on
+// the square layout (each square {e<f} stored once, at e), score = alpha*w +
+// beta*overlap (Eq. 1, :64-72); M_y wins ties; best on a strict > (Z8).
 #include "internal.cuh"
 
 #include <cooperative_groups.h>
@@ -36,18 +41,11 @@ struct MatchParams {
     const int32_t *La, *Lb;
     const int64_t *Arow, *Bptr;
     const int32_t *Bedge;
-    const double *x[2];
-    int32_t *candA, *candB, *mateA, *mateB;
+    const double *x0, *x1;
+    int32_t *candA, *candB; // SUITOR: suitor slots (edge id of the proposer's edge)
+    int32_t *mateA, *mateB;
     RoundDev *rd;
-    // evaluate
-    int evaluate, exact;
-    const double *w;
-    const int64_t *sq_rp;
-    const int2 *sq_ef;
-    double alpha, beta;
-    double *partial_w;
-    int32_t *best_mate;
-    int32_t p;
+    unsigned long long *work; // per instance: proposals (suitor) / rounds
 };
 
 __device__ __forceinline__ bool better(double xa, int ea, double xb, int eb)
@@ -55,9 +53,71 @@ __device__ __forceinline__ bool better(double xa, int ea, double xb, int eb)
     return eb < 0 || xa > xb || (xa == xb && ea < eb);
 }
 
+__device__ __forceinline__ const double *xk(const MatchParams &P, int k) { return k ? P.x1 : P.x0; }
+
+// ------------------------------------------------------------------ Suitor
+// Slot v in [0, ninst*(nA+nB)): instance k, vertex r (A vertex if r < nA).
+// suitor slots: candA[k*nA + a] = edge by which a B vertex proposes to a,
+//               candB[k*nB + b] = edge by which an A vertex proposes to b.
+__global__ void __launch_bounds__(128) k_suitor(MatchParams P)
+{
+    const int64_t nA = P.nA, nB = P.nB, NV = nA + nB;
+    const int64_t slot = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (slot >= P.ninst * NV) return;
+    const int k = (int)(slot / NV);
+    int64_t r = slot - k * NV;
+    const double *__restrict__ x = xk(P, k);
+    int32_t *sA = P.candA + k * nA;
+    int32_t *sB = P.candB + k * nB;
+    bool sideA = r < nA;
+    int cur = sideA ? (int)r : (int)(r - nA);
+    unsigned long long proposals = 0;
+    while (true) {
+        // heaviest eligible neighbour of `cur` whose suitor is lighter
+        int best = -1;
+        double bx = 0.0;
+        if (sideA) {
+            const int64_t hi = P.Arow[cur + 1];
+            for (int64_t e = P.Arow[cur]; e < hi; e++) {
+                const double xe = __ldg(x + e);
+                if (!(xe > 0.0)) continue;
+                if (!better(xe, (int)e, bx, best)) continue;
+                const int s = *(volatile int32_t *)(sB + __ldg(P.Lb + e));
+                if (s >= 0 && !better(xe, (int)e, __ldg(x + s), s)) continue;
+                best = (int)e;
+                bx = xe;
+            }
+        } else {
+            const int64_t hi = P.Bptr[cur + 1];
+            for (int64_t j = P.Bptr[cur]; j < hi; j++) {
+                const int e = __ldg(P.Bedge + j);
+                const double xe = __ldg(x + e);
+                if (!(xe > 0.0)) continue;
+                if (!better(xe, e, bx, best)) continue;
+                const int s = *(volatile int32_t *)(sA + __ldg(P.La + e));
+                if (s >= 0 && !better(xe, e, __ldg(x + s), s)) continue;
+                best = e;
+                bx = xe;
+            }
+        }
+        if (best < 0) break;
+        int32_t *slotp = sideA ? (sB + __ldg(P.Lb + best)) : (sA + __ldg(P.La + best));
+        const int s = *(volatile int32_t *)slotp;
+        if (s >= 0 && !better(bx, best, __ldg(x + s), s)) continue; // lost a race: rescan
+        const int old = atomicCAS(slotp, s, best);
+        if (old != s) continue;                                     // lost a race: rescan
+        proposals++;
+        if (s < 0) break;
+        // the displaced suitor (other end of edge s, same side as cur) proposes again
+        cur = sideA ? __ldg(P.La + s) : __ldg(P.Lb + s);
+    }
+    if (proposals) atomicAdd(P.work + k, proposals);
+}
+
+// ---------------------------------------------------------- pointer rounds
 __device__ int cand_A(const MatchParams &P, int k, int a)
 {
-    const double *x = P.x[k];
+    const double *x = xk(P, k);
     const int32_t *mB = P.mateB + (int64_t)k * P.nB;
     int best = -1;
     double bx = 0.0;
@@ -76,7 +136,7 @@ __device__ int cand_A(const MatchParams &P, int k, int a)
 
 __device__ int cand_B(const MatchParams &P, int k, int b)
 {
-    const double *x = P.x[k];
+    const double *x = xk(P, k);
     const int32_t *mA = P.mateA + (int64_t)k * P.nA;
     int best = -1;
     double bx = 0.0;
@@ -94,45 +154,16 @@ __device__ int cand_B(const MatchParams &P, int k, int b)
     return best;
 }
 
-template <class T>
-__device__ T block_sum(T v, T *smem)
-{
-    // deterministic tree: warp shuffles, then warp 0 over the warp sums
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-#pragma unroll
-    for (int off = 16; off >= 1; off >>= 1) v += __shfl_down_sync(0xffffffffu, v, off);
-    __syncthreads();
-    if (lane == 0) smem[wid] = v;
-    __syncthreads();
-    const int nw = (blockDim.x + 31) >> 5;
-    T r = 0;
-    if (wid == 0) {
-        r = (lane < nw) ? smem[lane] : (T)0;
-#pragma unroll
-        for (int off = 16; off >= 1; off >>= 1) r += __shfl_down_sync(0xffffffffu, r, off);
-    }
-    return r; // valid in thread 0
-}
-
-__global__ void __launch_bounds__(256) k_match(MatchParams P)
+__global__ void __launch_bounds__(256) k_pointer_rounds(MatchParams P)
 {
     cg::grid_group grid = cg::this_grid();
-    __shared__ double sd[32];
-    __shared__ unsigned long long su[32];
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
     const int64_t nA = P.nA, nB = P.nB;
     const int64_t NV = nA + nB;
     RoundDev *rd = P.rd;
-
     if (tid == 0) {
-        for (int k = 0; k < 2; k++) {
-            rd->flag[0][k] = rd->flag[1][k] = 0;
-            rd->rounds[k] = 0;
-            rd->overlap[k] = 0;
-            rd->card[k] = 0;
-            rd->weight[k] = 0.0;
-        }
+        for (int k = 0; k < 2; k++) rd->flag[0][k] = rd->flag[1][k] = 0;
     }
     for (int64_t v = tid; v < P.ninst * NV; v += nthr) {
         const int k = (int)(v / NV);
@@ -141,7 +172,6 @@ __global__ void __launch_bounds__(256) k_match(MatchParams P)
         else P.mateB[k * nB + (r - nA)] = -1;
     }
     grid.sync();
-    // Phase 1: candidate mates among all (unmatched) vertices
     for (int64_t v = tid; v < P.ninst * NV; v += nthr) {
         const int k = (int)(v / NV);
         const int64_t r = v - k * NV;
@@ -151,7 +181,6 @@ __global__ void __launch_bounds__(256) k_match(MatchParams P)
     grid.sync();
     for (int round = 0; round < P.max_rounds; round++) {
         const int par = round & 1;
-        // M: locally dominant edges
         for (int64_t v = tid; v < P.ninst * nA; v += nthr) {
             const int k = (int)(v / nA);
             const int64_t a = v - k * nA;
@@ -172,10 +201,9 @@ __global__ void __launch_bounds__(256) k_match(MatchParams P)
         if (tid == 0) {
             rd->flag[par ^ 1][0] = 0u;
             rd->flag[par ^ 1][1] = 0u;
-            rd->rounds[0] += (int)f0;
-            rd->rounds[1] += (int)f1;
+            P.work[0] += f0;
+            P.work[1] += f1;
         }
-        // R: re-point vertices whose candidate endpoint was just matched
         for (int64_t v = tid; v < P.ninst * NV; v += nthr) {
             const int k = (int)(v / NV);
             const int64_t r = v - k * NV;
@@ -194,14 +222,77 @@ __global__ void __launch_bounds__(256) k_match(MatchParams P)
         }
         grid.sync();
     }
-    if (!P.evaluate) return;
+}
 
-    // a8: evaluate both matchings
-    for (int k = 0; k < P.ninst; k++) {
+// ------------------------------------------------------- mates from suitors
+__global__ void k_suitor_to_mates(int64_t nA, int64_t nB, int ninst, const int32_t *__restrict__ La,
+                                  const int32_t *__restrict__ Lb, const int32_t *__restrict__ sA,
+                                  const int32_t *__restrict__ sB, int32_t *__restrict__ mateA,
+                                  int32_t *__restrict__ mateB)
+{
+    const int64_t NV = nA + nB;
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * NV;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        const int k = (int)(v / NV);
+        const int64_t r = v - k * NV;
+        if (r < nA) {
+            int e = sA[k * nA + r];
+            if (e >= 0 && sB[k * nB + Lb[e]] != e) e = -1;
+            mateA[k * nA + r] = e;
+        } else {
+            const int64_t b = r - nA;
+            int e = sB[k * nB + b];
+            if (e >= 0 && sA[k * nA + La[e]] != e) e = -1;
+            mateB[k * nB + b] = e;
+        }
+    }
+}
+
+// ---------------------------------------------------------------- evaluate
+template <class T>
+__device__ T block_sum(T v, T *smem)
+{
+    // deterministic tree: warp shuffles, then warp 0 over the warp sums
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+    for (int off = 16; off >= 1; off >>= 1) v += __shfl_down_sync(0xffffffffu, v, off);
+    __syncthreads();
+    if (lane == 0) smem[wid] = v;
+    __syncthreads();
+    const int nw = (blockDim.x + 31) >> 5;
+    T r = 0;
+    if (wid == 0) {
+        r = (lane < nw) ? smem[lane] : (T)0;
+#pragma unroll
+        for (int off = 16; off >= 1; off >>= 1) r += __shfl_down_sync(0xffffffffu, r, off);
+    }
+    return r; // valid in thread 0
+}
+
+struct EvalParams {
+    int64_t nA;
+    const int32_t *La;
+    const double *w;
+    const int64_t *sq_rp;
+    const int2 *sq_ef;
+    const int32_t *mateA; // 2 instances, final
+    double *partial_w;    // [2][gridDim]
+    RoundDev *rd;
+};
+
+// weight partial sums per block (fixed partition: deterministic), overlap and
+// cardinality as integer atomics (exact)
+__global__ void __launch_bounds__(256) k_eval(EvalParams P)
+{
+    __shared__ double sd[32];
+    __shared__ unsigned long long su[32];
+    const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+    for (int k = 0; k < 2; k++) {
+        const int32_t *mA = P.mateA + (int64_t)k * P.nA;
         double wsum = 0.0;
         unsigned long long ov = 0, card = 0;
-        const int32_t *mA = P.mateA + (int64_t)k * nA;
-        for (int64_t a = tid; a < nA; a += nthr) {
+        for (int64_t a = tid; a < P.nA; a += nthr) {
             const int e = mA[a];
             if (e < 0) continue;
             wsum += P.w[e];
@@ -215,77 +306,73 @@ __global__ void __launch_bounds__(256) k_match(MatchParams P)
         const double bw = block_sum<double>(wsum, sd);
         if (threadIdx.x == 0) P.partial_w[k * gridDim.x + blockIdx.x] = bw;
         const unsigned long long bo = block_sum<unsigned long long>(ov, su);
-        if (threadIdx.x == 0 && bo) atomicAdd(&rd->overlap[k], bo);
+        if (threadIdx.x == 0 && bo) atomicAdd(&P.rd->overlap[k], bo);
         const unsigned long long bc = block_sum<unsigned long long>(card, su);
-        if (threadIdx.x == 0 && bc) atomicAdd(&rd->card[k], bc);
-    }
-    grid.sync();
-    if (blockIdx.x == 0) {
-        double wk[2] = {0.0, 0.0};
-        for (int k = 0; k < P.ninst; k++) {
-            if (P.exact) {
-                // oracle order: ascending edge id == ascending A vertex
-                if (threadIdx.x == 0) {
-                    double s = 0.0;
-                    const int32_t *mA = P.mateA + (int64_t)k * nA;
-                    for (int64_t a = 0; a < nA; a++)
-                        if (mA[a] >= 0) s = s + P.w[mA[a]];
-                    wk[k] = s;
-                }
-            } else {
-                double s = 0.0;
-                for (int i = threadIdx.x; i < (int)gridDim.x; i += blockDim.x) s += P.partial_w[k * gridDim.x + i];
-                s = block_sum<double>(s, sd);
-                if (threadIdx.x == 0) wk[k] = s;
-            }
-        }
-        if (threadIdx.x == 0) {
-            cualign_round_info &I = rd->info;
-            const unsigned long long ov0 = *(volatile unsigned long long *)&rd->overlap[0];
-            const unsigned long long ov1 = *(volatile unsigned long long *)&rd->overlap[1];
-            const unsigned long long c0 = *(volatile unsigned long long *)&rd->card[0];
-            const unsigned long long c1 = *(volatile unsigned long long *)&rd->card[1];
-            I.iter = P.p;
-            I.weight_y = wk[0];
-            I.weight_z = wk[1];
-            I.overlap_y = (int64_t)ov0;
-            I.overlap_z = (int64_t)ov1;
-            I.card_y = (int32_t)c0;
-            I.card_z = (int32_t)c1;
-            I.score_y = P.alpha * wk[0] + P.beta * (double)(int64_t)ov0;
-            I.score_z = P.alpha * wk[1] + P.beta * (double)(int64_t)ov1;
-            I.rounds_y = rd->rounds[0];
-            I.rounds_z = rd->rounds[1];
-            const int src = (I.score_y >= I.score_z) ? 0 : 1;
-            I.source = src;
-            I.score = src ? I.score_z : I.score_y;
-            I.improved = 0;
-            if (I.score > rd->best_score) {
-                rd->best_score = I.score;
-                rd->best_iter = P.p;
-                I.improved = 1;
-            }
-            I.best_score = rd->best_score;
-            I.best_iter = rd->best_iter;
-            rd->improved = I.improved;
-            rd->source = src;
-        }
-    }
-    grid.sync();
-    if (*(volatile int *)&rd->improved) {
-        const int src = *(volatile int *)&rd->source;
-        const int32_t *mA = P.mateA + (int64_t)src * nA;
-        for (int64_t a = tid; a < nA; a += nthr) P.best_mate[a] = mA[a];
+        if (threadIdx.x == 0 && bc) atomicAdd(&P.rd->card[k], bc);
     }
 }
 
-cualign_status launch_match(cualign_bp *h, MatchParams &P)
+// one block: finish the sums, score, select, best (Alg. 2 l.21-24)
+__global__ void __launch_bounds__(256)
+k_round_final(EvalParams P, int nblocks, int exact, double alpha, double beta, int32_t p,
+              const unsigned long long *work)
 {
-    KScope ks(h, CUALIGN_K_MATCH);
-    void *args[] = {&P};
-    CA_CUDA(cudaLaunchCooperativeKernel((void *)k_match, dim3(h->match_grid), dim3(h->match_block), args, 0,
-                                        h->stream));
-    return CUALIGN_OK;
+    __shared__ double sd[32];
+    double wk[2] = {0.0, 0.0};
+    for (int k = 0; k < 2; k++) {
+        if (exact) {
+            // oracle order: ascending edge id == ascending A vertex
+            if (threadIdx.x == 0) {
+                double s = 0.0;
+                const int32_t *mA = P.mateA + (int64_t)k * P.nA;
+                for (int64_t a = 0; a < P.nA; a++)
+                    if (mA[a] >= 0) s = s + P.w[mA[a]];
+                wk[k] = s;
+            }
+        } else {
+            double s = 0.0;
+            for (int i = threadIdx.x; i < nblocks; i += blockDim.x) s += P.partial_w[k * nblocks + i];
+            s = block_sum<double>(s, sd);
+            if (threadIdx.x == 0) wk[k] = s;
+        }
+    }
+    if (threadIdx.x != 0) return;
+    RoundDev *rd = P.rd;
+    cualign_round_info &I = rd->info;
+    const long long ov0 = (long long)rd->overlap[0], ov1 = (long long)rd->overlap[1];
+    I.iter = p;
+    I.weight_y = wk[0];
+    I.weight_z = wk[1];
+    I.overlap_y = ov0;
+    I.overlap_z = ov1;
+    I.card_y = (int32_t)rd->card[0];
+    I.card_z = (int32_t)rd->card[1];
+    I.score_y = alpha * wk[0] + beta * (double)ov0;
+    I.score_z = alpha * wk[1] + beta * (double)ov1;
+    I.rounds_y = (int32_t)work[0];
+    I.rounds_z = (int32_t)work[1];
+    const int src = (I.score_y >= I.score_z) ? 0 : 1;
+    I.source = src;
+    I.score = src ? I.score_z : I.score_y;
+    I.improved = 0;
+    if (I.score > rd->best_score) {
+        rd->best_score = I.score;
+        rd->best_iter = p;
+        I.improved = 1;
+    }
+    I.best_score = rd->best_score;
+    I.best_iter = rd->best_iter;
+    rd->improved = I.improved;
+    rd->source = src;
+}
+
+__global__ void k_copy_best(int64_t nA, const int32_t *__restrict__ mateA, const RoundDev *__restrict__ rd,
+                            int32_t *__restrict__ best_mate)
+{
+    if (!rd->improved) return;
+    const int32_t *src = mateA + (int64_t)rd->source * nA;
+    for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < nA; a += (int64_t)gridDim.x * blockDim.x)
+        best_mate[a] = src[a];
 }
 
 MatchParams base_params(cualign_bp *h)
@@ -293,7 +380,8 @@ MatchParams base_params(cualign_bp *h)
     MatchParams P{};
     P.nA = h->L.nA;
     P.nB = h->L.nB;
-    P.max_rounds = (int)((int64_t)h->L.nA + h->L.nB + 4 > (1 << 30) ? (1 << 30) : (int64_t)h->L.nA + h->L.nB + 4);
+    const int64_t mr = (int64_t)h->L.nA + h->L.nB + 4;
+    P.max_rounds = (int)(mr > (1 << 30) ? (1 << 30) : mr);
     P.La = h->L.La;
     P.Lb = h->L.Lb;
     P.Arow = h->L.Arow;
@@ -304,7 +392,37 @@ MatchParams base_params(cualign_bp *h)
     P.mateA = h->mateA;
     P.mateB = h->mateB;
     P.rd = h->rd;
+    P.work = h->match_work;
     return P;
+}
+
+// run the matching of ninst instances; leaves mateA / mateB final
+cualign_status run_matching(cualign_bp *h, MatchParams &P)
+{
+    const int64_t nA = h->L.nA, nB = h->L.nB;
+    CA_CUDA(cudaMemsetAsync(h->match_work, 0, 2 * sizeof(unsigned long long), h->stream));
+    if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) {
+        KScope ks(h, CUALIGN_K_MATCH);
+        void *args[] = {&P};
+        CA_CUDA(cudaLaunchCooperativeKernel((void *)k_pointer_rounds, dim3(h->match_grid), dim3(256), args, 0,
+                                            h->stream));
+        return CUALIGN_OK;
+    }
+    CA_CUDA(cudaMemsetAsync(h->candA, 0xff, sizeof(int32_t) * (size_t)(2 * nA + 1), h->stream));
+    CA_CUDA(cudaMemsetAsync(h->candB, 0xff, sizeof(int32_t) * (size_t)(2 * nB + 1), h->stream));
+    const int64_t slots = P.ninst * (nA + nB);
+    if (slots > 0) {
+        KScope ks(h, CUALIGN_K_MATCH);
+        k_suitor<<<grid_for(slots, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        CA_CUDA(cudaGetLastError());
+    }
+    {
+        KScope ks(h, CUALIGN_K_MATCH);
+        k_suitor_to_mates<<<grid_for(slots, 256, h->num_sms * 8), 256, 0, h->stream>>>(
+            nA, nB, P.ninst, P.La, P.Lb, P.candA, P.candB, P.mateA, P.mateB);
+        CA_CUDA(cudaGetLastError());
+    }
+    return CUALIGN_OK;
 }
 
 } // namespace
@@ -318,15 +436,19 @@ cualign_status match_setup(cualign_bp *h)
     CA_TRY(dalloc(h, &h->mateB, 2 * nB + 1));
     CA_TRY(dalloc(h, &h->best_mate, nA + 1));
     CA_TRY(dalloc(h, &h->rd, 1));
+    CA_TRY(dalloc(h, &h->match_work, 2));
     CA_CUDA(cudaMemsetAsync(h->rd, 0, sizeof(RoundDev), h->stream));
+    CA_CUDA(cudaMemsetAsync(h->mateA, 0xff, sizeof(int32_t) * (2 * nA + 1), h->stream));
+    CA_CUDA(cudaMemsetAsync(h->mateB, 0xff, sizeof(int32_t) * (2 * nB + 1), h->stream));
     CA_CUDA(cudaMemsetAsync(h->best_mate, 0xff, sizeof(int32_t) * (nA + 1), h->stream));
     int occ = 0;
-    CA_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_match, h->match_block, 0));
+    CA_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pointer_rounds, 256, 0));
     if (occ < 1) occ = 1;
-    int64_t want = ((int64_t)2 * (nA + nB) + h->match_block - 1) / h->match_block;
+    int64_t want = ((int64_t)2 * (nA + nB) + 255) / 256;
     int64_t cap = (int64_t)occ * h->num_sms;
     h->match_grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
-    CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * h->match_grid));
+    h->eval_grid = grid_for((int64_t)nA, 256, h->num_sms * 4);
+    CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * h->eval_grid));
     return CUALIGN_OK;
 }
 
@@ -335,34 +457,52 @@ cualign_status match_round(cualign_bp *h)
     MatchParams P = base_params(h);
     const bool damped = (h->flags & CUALIGN_FLAG_ROUND_DAMPED) != 0;
     P.ninst = 2;
-    P.x[0] = damped ? h->yp : h->yc;
-    P.x[1] = damped ? h->zp : h->zc;
-    P.evaluate = 1;
-    P.exact = (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0;
-    P.w = h->L.w;
-    P.sq_rp = h->sq_rp;
-    P.sq_ef = h->sq_ef;
-    P.alpha = h->alpha;
-    P.beta = h->beta;
-    P.partial_w = h->partial_w;
-    P.best_mate = h->best_mate;
-    P.p = h->p;
-    return launch_match(h, P);
+    P.x0 = damped ? h->yp : h->yc;
+    P.x1 = damped ? h->zp : h->zc;
+    CA_TRY(run_matching(h, P));
+    EvalParams E{};
+    E.nA = h->L.nA;
+    E.La = h->L.La;
+    E.w = h->L.w;
+    E.sq_rp = h->sq_rp;
+    E.sq_ef = h->sq_ef;
+    E.mateA = h->mateA;
+    E.partial_w = h->partial_w;
+    E.rd = h->rd;
+    // overlap / card accumulators (the rest of rd persists: best)
+    CA_CUDA(cudaMemsetAsync(&h->rd->overlap[0], 0, 4 * sizeof(unsigned long long), h->stream));
+    {
+        KScope ks(h, CUALIGN_K_MATCH);
+        k_eval<<<h->eval_grid, 256, 0, h->stream>>>(E);
+        CA_CUDA(cudaGetLastError());
+    }
+    {
+        KScope ks(h, CUALIGN_K_MATCH);
+        k_round_final<<<1, 256, 0, h->stream>>>(E, h->eval_grid, (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha,
+                                                h->beta, h->p, h->match_work);
+        CA_CUDA(cudaGetLastError());
+    }
+    {
+        KScope ks(h, CUALIGN_K_MATCH);
+        k_copy_best<<<grid_for(h->L.nA, 256, h->num_sms * 4), 256, 0, h->stream>>>(h->L.nA, h->mateA, h->rd,
+                                                                                  h->best_mate);
+        CA_CUDA(cudaGetLastError());
+    }
+    return CUALIGN_OK;
 }
 
 cualign_status match_standalone(cualign_bp *h, const double *x_dev, int32_t *rounds)
 {
     MatchParams P = base_params(h);
     P.ninst = 1;
-    P.x[0] = x_dev;
-    P.x[1] = x_dev;
-    P.evaluate = 0;
-    CA_TRY(launch_match(h, P));
+    P.x0 = x_dev;
+    P.x1 = x_dev;
+    CA_TRY(run_matching(h, P));
     if (rounds) {
-        RoundDev r;
-        CA_CUDA(cudaMemcpyAsync(&r, h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->stream));
+        unsigned long long w[2] = {0, 0};
+        CA_CUDA(cudaMemcpyAsync(w, h->match_work, sizeof(w), cudaMemcpyDeviceToHost, h->stream));
         CA_CUDA(cudaStreamSynchronize(h->stream));
-        *rounds = r.rounds[0];
+        *rounds = (int32_t)w[0];
     }
     return CUALIGN_OK;
 }

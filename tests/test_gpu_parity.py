@@ -193,13 +193,15 @@ def test_get_state_roundtrip(ca):
 # ------------------------------------------------------------ a7: matching
 @pytest.mark.parametrize("seed", range(12))
 @pytest.mark.parametrize("weights", ["ties", "ties_signed", "uniform"])
-def test_matching_bit_exact_vs_greedy(ca, seed, weights):
+@pytest.mark.parametrize("schedule", ["suitor", "rounds"])
+def test_matching_bit_exact_vs_greedy(ca, seed, weights, schedule):
     rng = np.random.default_rng(seed)
     n_a, n_b = int(rng.integers(5, 300)), int(rng.integers(5, 300))
     L = random_candidates(n_a, n_b, int(rng.integers(1, 12)), rng, weights=weights)
     o = Oracle(graph_from_edges(n_a, []), graph_from_edges(n_b, []), L, 1.0, 0.0)
     want, _ = o.greedy(L.w)
-    ma, mb, rounds = ca.match(L, n_a, n_b, L.w)
+    flags = ca.FLAG_MATCH_ROUNDS if schedule == "rounds" else 0
+    ma, mb, rounds = ca.match(L, n_a, n_b, L.w, flags=flags)
     assert np.array_equal(ma, want)
     # mate_b consistent with mate_a
     for a in range(n_a):
@@ -208,15 +210,34 @@ def test_matching_bit_exact_vs_greedy(ca, seed, weights):
     assert np.sum(mb >= 0) == np.sum(ma >= 0)
 
 
-def test_matching_large_random(ca):
+@pytest.mark.parametrize("schedule", ["suitor", "rounds"])
+def test_matching_large_random(ca, schedule):
     rng = np.random.default_rng(0)
     n_a, n_b = 20000, 15000
     L = random_candidates(n_a, n_b, 12, rng, weights="uniform")
     o = Oracle(graph_from_edges(n_a, []), graph_from_edges(n_b, []), L, 1.0, 0.0)
+    flags = ca.FLAG_MATCH_ROUNDS if schedule == "rounds" else 0
     for x in (L.w, np.round(L.w * 4) / 4):  # generic and massively tied weights
         want, _ = o.greedy(x)
-        ma, _, rounds = ca.match(L, n_a, n_b, x)
+        ma, _, rounds = ca.match(L, n_a, n_b, x, flags=flags)
         assert np.array_equal(ma, want)
+
+
+def test_round_schedules_agree_on_config(ca):
+    """Suitor and pointer-round schedules give the same matchings and scores."""
+    inst = make_config("O", scale=0.01)
+    res = []
+    for flags in (0, ca.FLAG_MATCH_ROUNDS):
+        with ca.CuAlignBP(inst.A, inst.B, inst.L, flags=flags) as h:
+            infos = []
+            for _ in range(5):
+                h.iterate(1)
+                infos.append(h.round())
+            res.append((infos, h.get_best()[0]))
+    for a, b in zip(res[0][0], res[1][0]):
+        for k in ("card_y", "card_z", "overlap_y", "overlap_z", "score_y", "score_z", "best_score"):
+            assert a[k] == b[k], k
+    assert np.array_equal(res[0][1], res[1][1])
 
 
 def test_matching_empty_and_degenerate(ca):
