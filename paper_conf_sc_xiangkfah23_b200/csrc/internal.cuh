@@ -107,6 +107,8 @@ struct cualign_bp {
     double *partial_w = nullptr;
     int match_grid = 0, match_block = 256, eval_grid = 1;
     unsigned long long *match_work = nullptr; // proposals (suitor) or rounds, per instance
+    bool propose_from_b = false;              // suitor: proposing side (smaller max degree)
+    int64_t max_deg_a = 0, max_deg_b = 0;     // max degree of A / B vertices in L
     cualign::RoundDev *rd = nullptr;
     cualign_round_info last_info{};
     bool have_info = false;

@@ -7,14 +7,13 @@
 // produces the same matching: the greedy one (pin P9).  Two schedules are
 // implemented; both are bit-exact against the oracle's sort-greedy:
 //
-//  * SUITOR (default).  Every vertex of V_A u V_B proposes to its heaviest
+//  * SUITOR (default).  Every vertex of one side proposes to its heaviest
 //    eligible neighbour whose current suitor is lighter; a CAS on the
 //    neighbour's suitor slot (an edge id) installs the proposal and the
 //    displaced suitor -- now owned by the same thread -- proposes again
-//    (Manne & Halappanavar's Suitor algorithm, a lock-free form of the
-//    locally-dominant rule).  One kernel, no grid-wide barriers; the matched
-//    edges are the mutual suitor pairs.  y^c and z^c are matched in the same
-//    launch (two instances).
+//    (the Suitor algorithm of Manne & Halappanavar, a lock-free form of the
+//    locally-dominant rule, here one-sided: see k_suitor).  One kernel, no
+//    grid-wide barriers.  y^c and z^c are matched in the same launch.
 //  * POINTER ROUNDS (CUALIGN_FLAG_MATCH_ROUNDS).  The paper's Phase 1 / Phase 2
 //    as synchronous rounds in one persistent cooperative kernel: every vertex
 //    points at its best eligible unmatched neighbour, mutual pointers match,
@@ -43,6 +42,7 @@ struct MatchParams {
     const int32_t *Bedge;
     const double *x0, *x1;
     int32_t *candA, *candB; // SUITOR: suitor slots (edge id of the proposer's edge)
+    int propose_from_b;     // SUITOR: proposing side
     int32_t *mateA, *mateB;
     RoundDev *rd;
     unsigned long long *work; // per instance: proposals (suitor) / rounds
@@ -56,60 +56,55 @@ __device__ __forceinline__ bool better(double xa, int ea, double xb, int eb)
 __device__ __forceinline__ const double *xk(const MatchParams &P, int k) { return k ? P.x1 : P.x0; }
 
 // ------------------------------------------------------------------ Suitor
-// Slot v in [0, ninst*(nA+nB)): instance k, vertex r (A vertex if r < nA).
-// suitor slots: candA[k*nA + a] = edge by which a B vertex proposes to a,
-//               candB[k*nB + b] = edge by which an A vertex proposes to b.
+// One-sided proposals.  In a bipartite graph whose preferences come from ONE
+// global strict ranking of the edges (x desc, id asc), the stable matching is
+// unique and equals the greedy matching; deferred acceptance from either side
+// (each proposer repeatedly proposes to its best neighbour whose current
+// suitor is worse, displacing it) reaches it in any order -- the Suitor
+// algorithm restricted to one side.  The proposing side is the one with the
+// smaller maximum degree (on the paper's workloads: the k candidates of each A
+// vertex), so no thread ever scans a hub's list.
+// Slot v in [0, ninst*nP): instance k, proposer r.  suitor[k*nT + t] = edge
+// by which the current suitor proposes to target t (-1 = none).
 __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
 {
-    const int64_t nA = P.nA, nB = P.nB, NV = nA + nB;
+    const bool fromB = P.propose_from_b != 0;
+    const int64_t nP = fromB ? P.nB : P.nA;
+    const int64_t nT = fromB ? P.nA : P.nB;
     const int64_t slot = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (slot >= P.ninst * NV) return;
-    const int k = (int)(slot / NV);
-    int64_t r = slot - k * NV;
+    if (slot >= P.ninst * nP) return;
+    const int k = (int)(slot / nP);
+    int cur = (int)(slot - k * nP);
     const double *__restrict__ x = xk(P, k);
-    int32_t *sA = P.candA + k * nA;
-    int32_t *sB = P.candB + k * nB;
-    bool sideA = r < nA;
-    int cur = sideA ? (int)r : (int)(r - nA);
+    int32_t *sT = (fromB ? P.candA : P.candB) + k * nT;
+    const int64_t *__restrict__ rp = fromB ? P.Bptr : P.Arow;
+    const int32_t *__restrict__ tgt = fromB ? P.La : P.Lb;   // target vertex of an edge
+    const int32_t *__restrict__ own = fromB ? P.Lb : P.La;   // proposer vertex of an edge
     unsigned long long proposals = 0;
     while (true) {
         // heaviest eligible neighbour of `cur` whose suitor is lighter
         int best = -1;
         double bx = 0.0;
-        if (sideA) {
-            const int64_t hi = P.Arow[cur + 1];
-            for (int64_t e = P.Arow[cur]; e < hi; e++) {
-                const double xe = __ldg(x + e);
-                if (!(xe > 0.0)) continue;
-                if (!better(xe, (int)e, bx, best)) continue;
-                const int s = *(volatile int32_t *)(sB + __ldg(P.Lb + e));
-                if (s >= 0 && !better(xe, (int)e, __ldg(x + s), s)) continue;
-                best = (int)e;
-                bx = xe;
-            }
-        } else {
-            const int64_t hi = P.Bptr[cur + 1];
-            for (int64_t j = P.Bptr[cur]; j < hi; j++) {
-                const int e = __ldg(P.Bedge + j);
-                const double xe = __ldg(x + e);
-                if (!(xe > 0.0)) continue;
-                if (!better(xe, e, bx, best)) continue;
-                const int s = *(volatile int32_t *)(sA + __ldg(P.La + e));
-                if (s >= 0 && !better(xe, e, __ldg(x + s), s)) continue;
-                best = e;
-                bx = xe;
-            }
+        const int64_t hi = rp[cur + 1];
+        for (int64_t j = rp[cur]; j < hi; j++) {
+            const int e = fromB ? __ldg(P.Bedge + j) : (int)j;
+            const double xe = __ldg(x + e);
+            if (!(xe > 0.0)) continue;
+            if (!better(xe, e, bx, best)) continue;
+            const int s = *(volatile int32_t *)(sT + __ldg(tgt + e));
+            if (s >= 0 && !better(xe, e, __ldg(x + s), s)) continue;
+            best = e;
+            bx = xe;
         }
         if (best < 0) break;
-        int32_t *slotp = sideA ? (sB + __ldg(P.Lb + best)) : (sA + __ldg(P.La + best));
+        int32_t *slotp = sT + __ldg(tgt + best);
         const int s = *(volatile int32_t *)slotp;
         if (s >= 0 && !better(bx, best, __ldg(x + s), s)) continue; // lost a race: rescan
         const int old = atomicCAS(slotp, s, best);
         if (old != s) continue;                                     // lost a race: rescan
         proposals++;
         if (s < 0) break;
-        // the displaced suitor (other end of edge s, same side as cur) proposes again
-        cur = sideA ? __ldg(P.La + s) : __ldg(P.Lb + s);
+        cur = __ldg(own + s); // the displaced proposer proposes again
     }
     if (proposals) atomicAdd(P.work + k, proposals);
 }
@@ -225,26 +220,17 @@ __global__ void __launch_bounds__(256) k_pointer_rounds(MatchParams P)
 }
 
 // ------------------------------------------------------- mates from suitors
-__global__ void k_suitor_to_mates(int64_t nA, int64_t nB, int ninst, const int32_t *__restrict__ La,
-                                  const int32_t *__restrict__ Lb, const int32_t *__restrict__ sA,
-                                  const int32_t *__restrict__ sB, int32_t *__restrict__ mateA,
-                                  int32_t *__restrict__ mateB)
+// the final suitor of each target is its mate (mateX arrays pre-set to -1)
+__global__ void k_suitor_to_mates(int64_t nT, int ninst, const int32_t *__restrict__ own,
+                                  const int32_t *__restrict__ sT, int32_t *__restrict__ mateT,
+                                  int32_t *__restrict__ mateP, int64_t nP)
 {
-    const int64_t NV = nA + nB;
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * NV;
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * nT;
          v += (int64_t)gridDim.x * blockDim.x) {
-        const int k = (int)(v / NV);
-        const int64_t r = v - k * NV;
-        if (r < nA) {
-            int e = sA[k * nA + r];
-            if (e >= 0 && sB[k * nB + Lb[e]] != e) e = -1;
-            mateA[k * nA + r] = e;
-        } else {
-            const int64_t b = r - nA;
-            int e = sB[k * nB + b];
-            if (e >= 0 && sA[k * nA + La[e]] != e) e = -1;
-            mateB[k * nB + b] = e;
-        }
+        const int k = (int)(v / nT);
+        const int e = sT[v];
+        mateT[v] = e;
+        if (e >= 0) mateP[k * nP + own[e]] = e;
     }
 }
 
@@ -281,24 +267,28 @@ struct EvalParams {
 };
 
 // weight partial sums per block (fixed partition: deterministic), overlap and
-// cardinality as integer atomics (exact)
+// cardinality as integer atomics (exact).  One warp per A vertex: the lanes
+// stride over the matched edge's square row (rows reach thousands of squares).
 __global__ void __launch_bounds__(256) k_eval(EvalParams P)
 {
     __shared__ double sd[32];
     __shared__ unsigned long long su[32];
-    const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+    const int lane = threadIdx.x & 31;
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int k = 0; k < 2; k++) {
         const int32_t *mA = P.mateA + (int64_t)k * P.nA;
         double wsum = 0.0;
         unsigned long long ov = 0, card = 0;
-        for (int64_t a = tid; a < P.nA; a += nthr) {
+        for (int64_t a = warp; a < P.nA; a += nwarps) {
             const int e = mA[a];
             if (e < 0) continue;
-            wsum += P.w[e];
-            card++;
+            if (lane == 0) {
+                wsum += P.w[e];
+                card++;
+            }
             const int64_t hi = P.sq_rp[e + 1];
-            for (int64_t q = P.sq_rp[e]; q < hi; q++) {
+            for (int64_t q = P.sq_rp[e] + lane; q < hi; q += 32) {
                 const int f = P.sq_ef[q].y;
                 if (mA[P.La[f]] == f) ov++;
             }
@@ -375,6 +365,24 @@ __global__ void k_copy_best(int64_t nA, const int32_t *__restrict__ mateA, const
         best_mate[a] = src[a];
 }
 
+__global__ void k_maxdeg(int64_t nA, const int64_t *__restrict__ Arow, int64_t nB,
+                         const int64_t *__restrict__ Bptr, unsigned long long *out)
+{
+    unsigned long long ma = 0, mb = 0;
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < nA + nB;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        if (v < nA) {
+            const unsigned long long d = (unsigned long long)(Arow[v + 1] - Arow[v]);
+            ma = d > ma ? d : ma;
+        } else {
+            const unsigned long long d = (unsigned long long)(Bptr[v - nA + 1] - Bptr[v - nA]);
+            mb = d > mb ? d : mb;
+        }
+    }
+    if (ma) atomicMax(out, ma);
+    if (mb) atomicMax(out + 1, mb);
+}
+
 MatchParams base_params(cualign_bp *h)
 {
     MatchParams P{};
@@ -408,18 +416,23 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
                                             h->stream));
         return CUALIGN_OK;
     }
-    CA_CUDA(cudaMemsetAsync(h->candA, 0xff, sizeof(int32_t) * (size_t)(2 * nA + 1), h->stream));
-    CA_CUDA(cudaMemsetAsync(h->candB, 0xff, sizeof(int32_t) * (size_t)(2 * nB + 1), h->stream));
-    const int64_t slots = P.ninst * (nA + nB);
+    const bool fromB = h->propose_from_b;
+    P.propose_from_b = fromB ? 1 : 0;
+    const int64_t nP = fromB ? nB : nA, nT = fromB ? nA : nB;
+    int32_t *sT = fromB ? h->candA : h->candB;
+    CA_CUDA(cudaMemsetAsync(sT, 0xff, sizeof(int32_t) * (size_t)(2 * nT + 1), h->stream));
+    CA_CUDA(cudaMemsetAsync(fromB ? h->mateB : h->mateA, 0xff, sizeof(int32_t) * (size_t)(2 * nP + 1),
+                            h->stream));
+    const int64_t slots = P.ninst * nP;
     if (slots > 0) {
         KScope ks(h, CUALIGN_K_MATCH);
         k_suitor<<<grid_for(slots, 128, 1 << 30), 128, 0, h->stream>>>(P);
         CA_CUDA(cudaGetLastError());
     }
-    {
+    if (P.ninst * nT > 0) {
         KScope ks(h, CUALIGN_K_MATCH);
-        k_suitor_to_mates<<<grid_for(slots, 256, h->num_sms * 8), 256, 0, h->stream>>>(
-            nA, nB, P.ninst, P.La, P.Lb, P.candA, P.candB, P.mateA, P.mateB);
+        k_suitor_to_mates<<<grid_for(P.ninst * nT, 256, h->num_sms * 8), 256, 0, h->stream>>>(
+            nT, P.ninst, fromB ? P.Lb : P.La, sT, fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP);
         CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;
@@ -441,13 +454,26 @@ cualign_status match_setup(cualign_bp *h)
     CA_CUDA(cudaMemsetAsync(h->mateA, 0xff, sizeof(int32_t) * (2 * nA + 1), h->stream));
     CA_CUDA(cudaMemsetAsync(h->mateB, 0xff, sizeof(int32_t) * (2 * nB + 1), h->stream));
     CA_CUDA(cudaMemsetAsync(h->best_mate, 0xff, sizeof(int32_t) * (nA + 1), h->stream));
+    {
+        KScope ks(h, CUALIGN_K_INIT);
+        unsigned long long md[2] = {0, 0};
+        CA_CUDA(cudaMemsetAsync(h->match_work, 0, 2 * sizeof(unsigned long long), h->stream));
+        k_maxdeg<<<grid_for((int64_t)(nA + nB), 256, h->num_sms * 8), 256, 0, h->stream>>>(
+            (int64_t)nA, h->L.Arow, (int64_t)nB, h->L.Bptr, h->match_work);
+        CA_CUDA(cudaGetLastError());
+        CA_CUDA(cudaMemcpyAsync(md, h->match_work, sizeof(md), cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaStreamSynchronize(h->stream));
+        h->max_deg_a = (int64_t)md[0];
+        h->max_deg_b = (int64_t)md[1];
+        h->propose_from_b = h->max_deg_b < h->max_deg_a;
+    }
     int occ = 0;
     CA_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pointer_rounds, 256, 0));
     if (occ < 1) occ = 1;
     int64_t want = ((int64_t)2 * (nA + nB) + 255) / 256;
     int64_t cap = (int64_t)occ * h->num_sms;
     h->match_grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
-    h->eval_grid = grid_for((int64_t)nA, 256, h->num_sms * 4);
+    h->eval_grid = grid_for((int64_t)nA * 32, 256, h->num_sms * 8);
     CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * h->eval_grid));
     return CUALIGN_OK;
 }

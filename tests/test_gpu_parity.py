@@ -223,6 +223,22 @@ def test_matching_large_random(ca, schedule):
         assert np.array_equal(ma, want)
 
 
+@pytest.mark.parametrize("seed", range(6))
+def test_matching_b_side_proposals(ca, seed):
+    """Wide A rows, thin B columns: the Suitor schedule proposes from B."""
+    rng = np.random.default_rng(40 + seed)
+    n_a, n_b = 12, 400
+    for weights in ("ties", "uniform"):
+        L = random_candidates(n_a, n_b, 60, rng, weights=weights)
+        o = Oracle(graph_from_edges(n_a, []), graph_from_edges(n_b, []), L, 1.0, 0.0)
+        want, _ = o.greedy(L.w)
+        ma, mb, _ = ca.match(L, n_a, n_b, L.w)
+        assert np.array_equal(ma, want)
+        for b in range(n_b):
+            if mb[b] >= 0:
+                assert ma[L.a[mb[b]]] == mb[b]
+
+
 def test_round_schedules_agree_on_config(ca):
     """Suitor and pointer-round schedules give the same matchings and scores."""
     inst = make_config("O", scale=0.01)
