@@ -167,8 +167,7 @@ static cualign_status alloc_state(cualign_bp *h)
         CA_TRY(dalloc(h, p, m));
         CA_CUDA(cudaMemsetAsync(*p, 0, sizeof(double) * (m ? m : 1), h->stream));
     }
-    CA_TRY(dalloc(h, &h->Atop, (size_t)h->L.nA + 1));
-    CA_TRY(dalloc(h, &h->Btop, (size_t)h->L.nB + 1));
+    CA_TRY(bp_setup(h));
     if (h->flags & CUALIGN_FLAG_EXACT) {
         CA_TRY(dalloc(h, &h->texact, m));
         CA_TRY(dalloc(h, &h->Ffull, (size_t)h->s));

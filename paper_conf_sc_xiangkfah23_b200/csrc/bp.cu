@@ -26,15 +26,17 @@
 // "Row sums"); CUALIGN_FLAG_EXACT sums in the oracle's order instead.
 #include "internal.cuh"
 
+#include <cooperative_groups.h>
+#include <cub/cub.cuh>
 #include <math.h>
+
+namespace cg = cooperative_groups;
 
 namespace cualign {
 
 namespace {
 
 #define FULL_MASK 0xffffffffu
-
-constexpr int TOP2_G = 8; // lanes per vertex in k_top2
 
 __device__ __forceinline__ void top2_push(double &m1, double &m2, double v)
 {
@@ -74,74 +76,161 @@ __device__ __forceinline__ double clamp_beta(double x, double beta)
     return v;
 }
 
-__global__ void __launch_bounds__(256)
-k_top2(int32_t nA, int32_t nB, const int64_t *__restrict__ Arow, const int64_t *__restrict__ Bptr,
-       const int32_t *__restrict__ Bedge, const double *__restrict__ yp, const double *__restrict__ zp,
-       double2 *__restrict__ Atop, double2 *__restrict__ Btop)
+// B-side top-2 (othermaxcol input), load-balanced: the B incidence lists are
+// cut into chunks of at most B_CHUNK entries (built once, bp_setup); one
+// G-lane tile per chunk gathers z^p through the incidence and reduces.  Hub
+// columns (thousands of L edges) become many independent chunks; consumers
+// merge a column's chunk results (almost always one).
+constexpr int B_CHUNK = 32;
+constexpr int TB_G = 8, TB_U = B_CHUNK / TB_G;
+
+template <int G, class Tile>
+__device__ __forceinline__ void tile_top2(Tile &tile, double &m1, double &m2)
 {
-    constexpr int VPW = 32 / TOP2_G;
-    const int lane = threadIdx.x & 31;
-    const int sub = lane % TOP2_G;
-    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int64_t N = (int64_t)nA + nB;
-    for (int64_t base = warp * VPW; base < N; base += nwarps * VPW) {
-        const int64_t v = base + lane / TOP2_G;
-        double m1 = -INFINITY, m2 = -INFINITY;
-        if (v < nA) {
-            const int64_t lo = Arow[v], hi = Arow[v + 1];
-            for (int64_t x = lo + sub; x < hi; x += TOP2_G) top2_push(m1, m2, yp[x]);
-        } else if (v < N) {
-            const int64_t b = v - nA;
-            const int64_t lo = Bptr[b], hi = Bptr[b + 1];
-            for (int64_t x = lo + sub; x < hi; x += TOP2_G) top2_push(m1, m2, zp[Bedge[x]]);
-        }
 #pragma unroll
-        for (int off = TOP2_G / 2; off >= 1; off >>= 1) {
-            const double b1 = __shfl_xor_sync(FULL_MASK, m1, off);
-            const double b2 = __shfl_xor_sync(FULL_MASK, m2, off);
-            top2_merge(m1, m2, b1, b2);
+    for (int off = G / 2; off >= 1; off >>= 1) {
+        const double b1 = tile.shfl_xor(m1, off);
+        const double b2 = tile.shfl_xor(m2, off);
+        top2_merge(m1, m2, b1, b2);
+    }
+}
+
+__global__ void __launch_bounds__(256)
+k_top2B(int64_t nchunks, const int32_t *__restrict__ chunk_b, const int64_t *__restrict__ Bcp,
+        const int64_t *__restrict__ Bptr, const int32_t *__restrict__ Bedge, const double *__restrict__ zp,
+        double2 *__restrict__ Bct)
+{
+    auto tile = cg::tiled_partition<TB_G>(cg::this_thread_block());
+    const int lane = tile.thread_rank();
+    const int64_t t0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / TB_G;
+    const int64_t nt = ((int64_t)gridDim.x * blockDim.x) / TB_G;
+    for (int64_t c = t0; c < nchunks; c += nt) {
+        const int b = chunk_b[c];
+        const int64_t start = Bptr[b] + (c - Bcp[b]) * B_CHUNK;
+        const int64_t end = min(start + (int64_t)B_CHUNK, Bptr[b + 1]);
+        int eidx[TB_U];
+#pragma unroll
+        for (int j = 0; j < TB_U; j++) {
+            const int64_t idx = start + lane + j * TB_G;
+            eidx[j] = idx < end ? __ldg(Bedge + idx) : -1;
         }
-        if (sub == 0) {
-            if (v < nA) Atop[v] = make_double2(m1, m2);
-            else if (v < N) Btop[v - nA] = make_double2(m1, m2);
+        double m1 = -INFINITY, m2 = -INFINITY;
+#pragma unroll
+        for (int j = 0; j < TB_U; j++)
+            if (eidx[j] >= 0) top2_push(m1, m2, zp[eidx[j]]);
+        tile_top2<TB_G>(tile, m1, m2);
+        if (lane == 0) Bct[c] = make_double2(m1, m2);
+    }
+}
+
+__device__ __forceinline__ double2 col_top2(int b, const int64_t *__restrict__ Bcp, const double2 *__restrict__ Bct)
+{
+    const int64_t c0 = Bcp[b], c1 = Bcp[b + 1];
+    double2 t = Bct[c0];
+    for (int64_t c = c0 + 1; c < c1; c++) {
+        const double2 o = Bct[c];
+        top2_merge(t.x, t.y, o.x, o.y);
+    }
+    return t;
+}
+
+struct RowArgs {
+    int64_t nA;
+    const int64_t *Arow;
+    const int32_t *Lb;
+    const double *w;
+    double alpha, g, hh, fp_inv;
+    unsigned long long *tacc;
+    const double *texact;
+    const int64_t *Bcp;
+    const double2 *Bct;
+    double *yp, *zp, *yc, *zc, *d, *u;
+};
+
+// the per-edge part of lines 10-15 for edge e, given its row's (max1, max2)
+template <bool EXACT, bool LITERAL>
+__device__ __forceinline__ void edge_update(const RowArgs &R, int64_t e, double ype, double zpe, double we,
+                                            double t, int b, double2 atop)
+{
+    const double de = R.alpha * we + t;                                   // line 10
+    const double omc = othermax<LITERAL>(zpe, col_top2(b, R.Bcp, R.Bct)); // line 11
+    const double omr = othermax<LITERAL>(ype, atop);                     // line 12
+    const double yce = de - omc;
+    const double zce = de - omr;
+    const double ue = (yce + zce) - de;                                   // line 13 diagonal
+    R.yp[e] = R.g * yce + R.hh * ype;                                     // line 14
+    R.zp[e] = R.g * zce + R.hh * zpe;                                     // line 15
+    R.yc[e] = yce;
+    R.zc[e] = zce;
+    R.d[e] = de;
+    R.u[e] = ue;
+}
+
+template <bool EXACT>
+__device__ __forceinline__ double take_t(const RowArgs &R, int64_t e)
+{
+    if (EXACT) return R.texact[e];
+    const unsigned long long T = R.tacc[e];
+    R.tacc[e] = 0ull; // ready for this iteration's k_square accumulation
+    return __ull2double_rn(T) * R.fp_inv;
+}
+
+// One G-lane tile per A vertex (its L row is contiguous): top-2 of y^p over the
+// row in registers (othermaxrow), then every edge of the row is updated.
+// Rows of up to G*U edges are loaded once into registers.
+template <int G, int U, bool EXACT, bool LITERAL>
+__global__ void __launch_bounds__(256) k_rowA(RowArgs R)
+{
+    auto tile = cg::tiled_partition<G>(cg::this_thread_block());
+    const int lane = tile.thread_rank();
+    const int64_t t0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
+    const int64_t nt = ((int64_t)gridDim.x * blockDim.x) / G;
+    for (int64_t a = t0; a < R.nA; a += nt) {
+        const int64_t lo = R.Arow[a], hi = R.Arow[a + 1];
+        if (hi - lo <= G * U) {
+            double ype[U], zpe[U], we[U];
+            int lb[U];
+            double m1 = -INFINITY, m2 = -INFINITY;
+#pragma unroll
+            for (int j = 0; j < U; j++) {
+                const int64_t e = lo + lane + j * G;
+                if (e < hi) {
+                    ype[j] = R.yp[e];
+                    zpe[j] = R.zp[e];
+                    we[j] = R.w[e];
+                    lb[j] = R.Lb[e];
+                    top2_push(m1, m2, ype[j]);
+                }
+            }
+            tile_top2<G>(tile, m1, m2);
+            const double2 atop = make_double2(m1, m2);
+#pragma unroll
+            for (int j = 0; j < U; j++) {
+                const int64_t e = lo + lane + j * G;
+                if (e < hi) edge_update<EXACT, LITERAL>(R, e, ype[j], zpe[j], we[j], take_t<EXACT>(R, e), lb[j], atop);
+            }
+        } else {
+            double m1 = -INFINITY, m2 = -INFINITY;
+            for (int64_t e = lo + lane; e < hi; e += G) top2_push(m1, m2, R.yp[e]);
+            tile_top2<G>(tile, m1, m2);
+            tile.sync(); // every lane has read its old y^p before any is overwritten
+            const double2 atop = make_double2(m1, m2);
+            for (int64_t e = lo + lane; e < hi; e += G)
+                edge_update<EXACT, LITERAL>(R, e, R.yp[e], R.zp[e], R.w[e], take_t<EXACT>(R, e), R.Lb[e], atop);
         }
     }
 }
 
-template <bool EXACT, bool LITERAL>
-__global__ void __launch_bounds__(256)
-k_edge(int64_t m, const int32_t *__restrict__ La, const int32_t *__restrict__ Lb,
-       const double *__restrict__ w, double alpha, double g, double hh, double fp_inv,
-       unsigned long long *__restrict__ tacc, const double *__restrict__ texact,
-       const double2 *__restrict__ Atop, const double2 *__restrict__ Btop, double *__restrict__ yp,
-       double *__restrict__ zp, double *__restrict__ yc, double *__restrict__ zc,
-       double *__restrict__ d, double *__restrict__ u)
+__global__ void k_chunk_count(int64_t nB, const int64_t *__restrict__ Bptr, int64_t *__restrict__ cnt)
 {
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m;
-         e += (int64_t)gridDim.x * blockDim.x) {
-        double t;
-        if (EXACT) {
-            t = texact[e];
-        } else {
-            const unsigned long long T = tacc[e];
-            tacc[e] = 0ull; // ready for this iteration's k_square accumulation
-            t = __ull2double_rn(T) * fp_inv;
-        }
-        const double de = alpha * w[e] + t;                       // line 10
-        const double ype = yp[e], zpe = zp[e];
-        const double omc = othermax<LITERAL>(zpe, Btop[Lb[e]]);   // line 11
-        const double omr = othermax<LITERAL>(ype, Atop[La[e]]);   // line 12
-        const double yce = de - omc;
-        const double zce = de - omr;
-        const double ue = (yce + zce) - de;                       // line 13 diagonal
-        yp[e] = g * yce + hh * ype;                               // line 14
-        zp[e] = g * zce + hh * zpe;                               // line 15
-        yc[e] = yce;
-        zc[e] = zce;
-        d[e] = de;
-        u[e] = ue;
-    }
+    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nB; b += (int64_t)gridDim.x * blockDim.x)
+        cnt[b] = (Bptr[b + 1] - Bptr[b] + B_CHUNK - 1) / B_CHUNK;
+}
+
+__global__ void k_chunk_fill(int64_t nB, const int64_t *__restrict__ Bcp, int32_t *__restrict__ chunk_b)
+{
+    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nB; b += (int64_t)gridDim.x * blockDim.x)
+        for (int64_t c = Bcp[b]; c < Bcp[b + 1]; c++) chunk_b[c] = (int32_t)b;
 }
 
 // segmented (by sorted key) warp sum, then one atomic per segment
@@ -279,6 +368,34 @@ cualign_status launch_square(cualign_bp *h, bool update, double g, double hh)
 
 } // namespace
 
+cualign_status bp_setup(cualign_bp *h)
+{
+    // B-side chunks for k_top2B
+    KScope ks(h, CUALIGN_K_INIT);
+    const int64_t nB = h->L.nB;
+    CA_TRY(dalloc(h, &h->Bcp, (size_t)nB + 1));
+    CA_CUDA(cudaMemsetAsync(h->Bcp, 0, sizeof(int64_t), h->stream));
+    if (nB > 0) {
+        int64_t *cnt = nullptr;
+        void *tmp = nullptr;
+        size_t tb = 0;
+        CA_CUDA(cudaMalloc(&cnt, sizeof(int64_t) * (size_t)nB));
+        k_chunk_count<<<grid_for(nB, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB, h->L.Bptr, cnt);
+        CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, cnt, h->Bcp + 1, (int)nB, h->stream));
+        CA_CUDA(cudaMalloc(&tmp, tb ? tb : 1));
+        CA_CUDA(cub::DeviceScan::InclusiveSum(tmp, tb, cnt, h->Bcp + 1, (int)nB, h->stream));
+        CA_CUDA(cudaMemcpyAsync(&h->nchunks, h->Bcp + nB, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaStreamSynchronize(h->stream));
+        cudaFree(cnt);
+        cudaFree(tmp);
+    }
+    CA_TRY(dalloc(h, &h->chunk_b, (size_t)h->nchunks + 1));
+    CA_TRY(dalloc(h, &h->Bct, (size_t)h->nchunks + 1));
+    if (nB > 0) k_chunk_fill<<<grid_for(nB, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB, h->Bcp, h->chunk_b);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
 cualign_status bp_fsum(cualign_bp *h)
 {
     if (!(h->flags & CUALIGN_FLAG_EXACT))
@@ -296,25 +413,22 @@ cualign_status bp_iterate(cualign_bp *h, int32_t n)
         const double g = pow(h->gamma, (double)p); // reading Z2: host fp64 gamma^p
         const double hh = 1.0 - g;
         if (m > 0) {
-            {
+            if (h->nchunks > 0) {
                 KScope ks(h, CUALIGN_K_TOP2);
-                const int64_t N = (int64_t)h->L.nA + h->L.nB;
-                const int64_t threads = (N + (32 / TOP2_G) - 1) / (32 / TOP2_G) * 32;
-                k_top2<<<grid_for(threads, 256, 1 << 30), 256, 0, h->stream>>>(
-                    h->L.nA, h->L.nB, h->L.Arow, h->L.Bptr, h->L.Bedge, h->yp, h->zp, h->Atop, h->Btop);
+                k_top2B<<<grid_for(h->nchunks * TB_G, 256, 1 << 30), 256, 0, h->stream>>>(
+                    h->nchunks, h->chunk_b, h->Bcp, h->L.Bptr, h->L.Bedge, h->zp, h->Bct);
                 CA_CUDA(cudaGetLastError());
             }
             {
                 KScope ks(h, CUALIGN_K_EDGE);
-                const int grid = grid_for(m, 256, 1 << 30);
-#define EDGE_ARGS                                                                                    \
-    m, h->L.La, h->L.Lb, h->L.w, h->alpha, g, hh, h->fp_inv, h->tacc, h->texact, h->Atop, h->Btop, \
-        h->yp, h->zp, h->yc, h->zc, h->d, h->u
-                if (exact && literal) k_edge<true, true><<<grid, 256, 0, h->stream>>>(EDGE_ARGS);
-                else if (exact) k_edge<true, false><<<grid, 256, 0, h->stream>>>(EDGE_ARGS);
-                else if (literal) k_edge<false, true><<<grid, 256, 0, h->stream>>>(EDGE_ARGS);
-                else k_edge<false, false><<<grid, 256, 0, h->stream>>>(EDGE_ARGS);
-#undef EDGE_ARGS
+                RowArgs R{(int64_t)h->L.nA, h->L.Arow, h->L.Lb, h->L.w, h->alpha, g, hh, h->fp_inv, h->tacc,
+                          h->texact, h->Bcp, h->Bct, h->yp, h->zp, h->yc, h->zc, h->d, h->u};
+                constexpr int G = 8, U = 3;
+                const int grid = grid_for((int64_t)h->L.nA * G, 256, 1 << 30);
+                if (exact && literal) k_rowA<G, U, true, true><<<grid, 256, 0, h->stream>>>(R);
+                else if (exact) k_rowA<G, U, true, false><<<grid, 256, 0, h->stream>>>(R);
+                else if (literal) k_rowA<G, U, false, true><<<grid, 256, 0, h->stream>>>(R);
+                else k_rowA<G, U, false, false><<<grid, 256, 0, h->stream>>>(R);
                 CA_CUDA(cudaGetLastError());
             }
             CA_TRY(launch_square(h, true, g, hh));

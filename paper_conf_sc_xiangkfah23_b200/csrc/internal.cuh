@@ -98,7 +98,10 @@ struct cualign_bp {
     unsigned long long *tacc = nullptr; // fast mode: sum_f F_ef in fixed point
     double *texact = nullptr;           // exact mode: sum_f F_ef, oracle order
     double *Ffull = nullptr;            // exact mode: F in CSR order
-    double2 *Atop = nullptr, *Btop = nullptr; // per-vertex (max1, max2)
+    int64_t nchunks = 0;                // B incidence chunks (k_top2B load balance)
+    int64_t *Bcp = nullptr;             // nB+1: chunks of B vertex b are Bcp[b]..Bcp[b+1]-1
+    int32_t *chunk_b = nullptr;         // nchunks: owning B vertex
+    double2 *Bct = nullptr;             // nchunks: (max1, max2) of z^p over the chunk
     int32_t p = 0;
 
     // matching (two instances: y and z)
@@ -155,6 +158,7 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
 cualign_status ensure_sq_pos(cualign_bp *h);
 
 // bp.cu
+cualign_status bp_setup(cualign_bp *h);                // B chunks
 cualign_status bp_fsum(cualign_bp *h);                 // t <- sum_f F(S^p) (init / set_state)
 cualign_status bp_iterate(cualign_bp *h, int32_t n);   // Alg. 2 l.9-16, n times
 cualign_status bp_scatter_Sp(cualign_bp *h, double *Sfull_dev);        // squares -> CSR

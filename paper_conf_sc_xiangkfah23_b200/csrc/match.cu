@@ -66,13 +66,19 @@ __device__ __forceinline__ const double *xk(const MatchParams &P, int k) { retur
 // vertex), so no thread ever scans a hub's list.
 // Slot v in [0, ninst*nP): instance k, proposer r.  suitor[k*nT + t] = edge
 // by which the current suitor proposes to target t (-1 = none).
+// One G-lane tile per proposer: the lanes scan the proposer's list together
+// (G edges per step, independent loads), a tile argmax picks the heaviest
+// eligible target, lane 0 attempts the CAS and the outcome is broadcast.
+template <int G>
 __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
 {
+    auto tile = cg::tiled_partition<G>(cg::this_thread_block());
+    const int lane = tile.thread_rank();
     const bool fromB = P.propose_from_b != 0;
     const int64_t nP = fromB ? P.nB : P.nA;
     const int64_t nT = fromB ? P.nA : P.nB;
-    const int64_t slot = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (slot >= P.ninst * nP) return;
+    const int64_t slot = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
+    if (slot >= P.ninst * nP) return; // tile-uniform
     const int k = (int)(slot / nP);
     int cur = (int)(slot - k * nP);
     const double *__restrict__ x = xk(P, k);
@@ -86,7 +92,7 @@ __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
         int best = -1;
         double bx = 0.0;
         const int64_t hi = rp[cur + 1];
-        for (int64_t j = rp[cur]; j < hi; j++) {
+        for (int64_t j = rp[cur] + lane; j < hi; j += G) {
             const int e = fromB ? __ldg(P.Bedge + j) : (int)j;
             const double xe = __ldg(x + e);
             if (!(xe > 0.0)) continue;
@@ -96,17 +102,38 @@ __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
             best = e;
             bx = xe;
         }
-        if (best < 0) break;
-        int32_t *slotp = sT + __ldg(tgt + best);
-        const int s = *(volatile int32_t *)slotp;
-        if (s >= 0 && !better(bx, best, __ldg(x + s), s)) continue; // lost a race: rescan
-        const int old = atomicCAS(slotp, s, best);
-        if (old != s) continue;                                     // lost a race: rescan
-        proposals++;
-        if (s < 0) break;
-        cur = __ldg(own + s); // the displaced proposer proposes again
+#pragma unroll
+        for (int off = G / 2; off >= 1; off >>= 1) {
+            const double ox = tile.shfl_xor(bx, off);
+            const int oe = tile.shfl_xor(best, off);
+            if (oe >= 0 && better(ox, oe, bx, best)) {
+                bx = ox;
+                best = oe;
+            }
+        }
+        if (best < 0) break; // tile-uniform after the all-reduce
+        int code = 0;        // 0 retry, 1 done, 2 displaced
+        int next = cur;
+        if (lane == 0) {
+            int32_t *slotp = sT + __ldg(tgt + best);
+            const int s = *(volatile int32_t *)slotp;
+            if (s < 0 || better(bx, best, __ldg(x + s), s)) {
+                if (atomicCAS(slotp, s, best) == s) {
+                    proposals++;
+                    if (s < 0) {
+                        code = 1;
+                    } else {
+                        code = 2;
+                        next = __ldg(own + s); // the displaced proposer proposes again
+                    }
+                }
+            }
+        }
+        code = tile.shfl(code, 0);
+        if (code == 1) break;
+        if (code == 2) cur = tile.shfl(next, 0);
     }
-    if (proposals) atomicAdd(P.work + k, proposals);
+    if (lane == 0 && proposals) atomicAdd(P.work + k, proposals);
 }
 
 // ---------------------------------------------------------- pointer rounds
@@ -273,9 +300,10 @@ __global__ void __launch_bounds__(256) k_eval(EvalParams P)
 {
     __shared__ double sd[32];
     __shared__ unsigned long long su[32];
-    const int lane = threadIdx.x & 31;
-    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    constexpr int G = 8;
+    const int lane = threadIdx.x & (G - 1);
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) / G;
     for (int k = 0; k < 2; k++) {
         const int32_t *mA = P.mateA + (int64_t)k * P.nA;
         double wsum = 0.0;
@@ -288,7 +316,7 @@ __global__ void __launch_bounds__(256) k_eval(EvalParams P)
                 card++;
             }
             const int64_t hi = P.sq_rp[e + 1];
-            for (int64_t q = P.sq_rp[e] + lane; q < hi; q += 32) {
+            for (int64_t q = P.sq_rp[e] + lane; q < hi; q += G) {
                 const int f = P.sq_ef[q].y;
                 if (mA[P.La[f]] == f) ov++;
             }
@@ -426,7 +454,9 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     const int64_t slots = P.ninst * nP;
     if (slots > 0) {
         KScope ks(h, CUALIGN_K_MATCH);
-        k_suitor<<<grid_for(slots, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        const int64_t dmax = fromB ? h->max_deg_b : h->max_deg_a;
+        if (dmax > 64) k_suitor<32><<<grid_for(slots * 32, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else k_suitor<8><<<grid_for(slots * 8, 128, 1 << 30), 128, 0, h->stream>>>(P);
         CA_CUDA(cudaGetLastError());
     }
     if (P.ninst * nT > 0) {
@@ -473,7 +503,7 @@ cualign_status match_setup(cualign_bp *h)
     int64_t want = ((int64_t)2 * (nA + nB) + 255) / 256;
     int64_t cap = (int64_t)occ * h->num_sms;
     h->match_grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
-    h->eval_grid = grid_for((int64_t)nA * 32, 256, h->num_sms * 8);
+    h->eval_grid = grid_for((int64_t)nA * 8, 256, h->num_sms * 8);
     CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * h->eval_grid));
     return CUALIGN_OK;
 }
