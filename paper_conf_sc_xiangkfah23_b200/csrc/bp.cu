@@ -1,12 +1,15 @@
 // bp.cu -- rows a3-a6 of the hot path: one NetAlignBP iteration,
 // Alg. 2 lines 9-16, as three kernels:
 //
-//   k_top2    per-vertex (max1, max2) of y^p over A rows of L and of z^p over
-//             B columns (the "othermaxrow/othermaxcol" reductions, :164-165,
-//             defined at :203)
+//   k_top2    per-vertex (max1, max2) of y^p over the A rows of L and of z^p
+//             over the B columns -- the inputs of othermaxrow / othermaxcol
+//             (:164-165, defined at :203).  8-lane tiles; B columns are cut
+//             into chunks of <= 32 entries so hub columns spread over many
+//             tiles (the last tile of a column merges its chunks).
 //   k_edge    per edge: d = alpha w + sum_f F_ef (line 10), y^c = d - omc(z^p),
 //             z^c = d - omr(y^p) (lines 11-12), u = y^c + z^c - d (the diagonal
-//             of line 13), damping of y, z (lines 14-15)
+//             of line 13), damping of y, z (lines 14-15).  Flat and coalesced,
+//             EPT edges per thread with all loads issued up front.
 //   k_square  per unordered square {e < f}: the pair (S^p_ef, S^p_fe) is read
 //             once, F_ef = clamp(beta + S^p_fe), F_fe = clamp(beta + S^p_ef)
 //             (line 9), S^c = u - F (line 13), damping (line 16), and the
@@ -58,6 +61,17 @@ __device__ __forceinline__ void top2_merge(double &m1, double &m2, double b1, do
     m2 = r2;
 }
 
+template <int G, class Tile>
+__device__ __forceinline__ void tile_top2(Tile &tile, double &m1, double &m2)
+{
+#pragma unroll
+    for (int off = G / 2; off >= 1; off >>= 1) {
+        const double b1 = tile.shfl_xor(m1, off);
+        const double b2 = tile.shfl_xor(m2, off);
+        top2_merge(m1, m2, b1, b2);
+    }
+}
+
 // om(e) from the (max1, max2) of e's row/column (reading Z4)
 template <bool LITERAL>
 __device__ __forceinline__ double othermax(double v, double2 t)
@@ -76,161 +90,130 @@ __device__ __forceinline__ double clamp_beta(double x, double beta)
     return v;
 }
 
-// B-side top-2 (othermaxcol input), load-balanced: the B incidence lists are
-// cut into chunks of at most B_CHUNK entries (built once, bp_setup); one
-// G-lane tile per chunk gathers z^p through the incidence and reduces.  Hub
-// columns (thousands of L edges) become many independent chunks; consumers
-// merge a column's chunk results (almost always one).
 constexpr int B_CHUNK = 32;
-constexpr int TB_G = 8, TB_U = B_CHUNK / TB_G;
+constexpr int TG = 8;                 // lanes per tile in k_top2
+constexpr int TB_U = B_CHUNK / TG;    // gathers per lane per chunk
 
-template <int G, class Tile>
-__device__ __forceinline__ void tile_top2(Tile &tile, double &m1, double &m2)
-{
-#pragma unroll
-    for (int off = G / 2; off >= 1; off >>= 1) {
-        const double b1 = tile.shfl_xor(m1, off);
-        const double b2 = tile.shfl_xor(m2, off);
-        top2_merge(m1, m2, b1, b2);
-    }
-}
-
-__global__ void __launch_bounds__(256)
-k_top2B(int64_t nchunks, const int32_t *__restrict__ chunk_b, const int64_t *__restrict__ Bcp,
-        const int64_t *__restrict__ Bptr, const int32_t *__restrict__ Bedge, const double *__restrict__ zp,
-        double2 *__restrict__ Bct)
-{
-    auto tile = cg::tiled_partition<TB_G>(cg::this_thread_block());
-    const int lane = tile.thread_rank();
-    const int64_t t0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / TB_G;
-    const int64_t nt = ((int64_t)gridDim.x * blockDim.x) / TB_G;
-    for (int64_t c = t0; c < nchunks; c += nt) {
-        const int b = chunk_b[c];
-        const int64_t start = Bptr[b] + (c - Bcp[b]) * B_CHUNK;
-        const int64_t end = min(start + (int64_t)B_CHUNK, Bptr[b + 1]);
-        int eidx[TB_U];
-#pragma unroll
-        for (int j = 0; j < TB_U; j++) {
-            const int64_t idx = start + lane + j * TB_G;
-            eidx[j] = idx < end ? __ldg(Bedge + idx) : -1;
-        }
-        double m1 = -INFINITY, m2 = -INFINITY;
-#pragma unroll
-        for (int j = 0; j < TB_U; j++)
-            if (eidx[j] >= 0) top2_push(m1, m2, zp[eidx[j]]);
-        tile_top2<TB_G>(tile, m1, m2);
-        if (lane == 0) Bct[c] = make_double2(m1, m2);
-    }
-}
-
-__device__ __forceinline__ double2 col_top2(int b, const int64_t *__restrict__ Bcp, const double2 *__restrict__ Bct)
-{
-    const int64_t c0 = Bcp[b], c1 = Bcp[b + 1];
-    double2 t = Bct[c0];
-    for (int64_t c = c0 + 1; c < c1; c++) {
-        const double2 o = Bct[c];
-        top2_merge(t.x, t.y, o.x, o.y);
-    }
-    return t;
-}
-
-struct RowArgs {
-    int64_t nA;
+struct Top2Args {
+    int64_t nA, nchunks;
     const int64_t *Arow;
-    const int32_t *Lb;
+    const int32_t *chunk_b;
+    const int64_t *Bcp, *Bptr;
+    const int32_t *Bedge;
+    const double *yp, *zp;
+    double2 *Atop, *Btop, *Bct;
+    unsigned int *Bcnt;
+};
+
+__global__ void __launch_bounds__(256) k_top2(Top2Args T)
+{
+    auto tile = cg::tiled_partition<TG>(cg::this_thread_block());
+    const int lane = tile.thread_rank();
+    const int64_t t0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / TG;
+    const int64_t nt = ((int64_t)gridDim.x * blockDim.x) / TG;
+    for (int64_t t = t0; t < T.nA + T.nchunks; t += nt) {
+        double m1 = -INFINITY, m2 = -INFINITY;
+        if (t < T.nA) {
+            // A row: contiguous edges
+            const int64_t lo = T.Arow[t], hi = T.Arow[t + 1];
+            for (int64_t e = lo + lane; e < hi; e += TG) top2_push(m1, m2, T.yp[e]);
+            tile_top2<TG>(tile, m1, m2);
+            if (lane == 0) T.Atop[t] = make_double2(m1, m2);
+        } else {
+            // B chunk: gather z^p through the incidence
+            const int64_t c = t - T.nA;
+            const int b = T.chunk_b[c];
+            const int64_t c0 = T.Bcp[b], c1 = T.Bcp[b + 1];
+            const int64_t start = T.Bptr[b] + (c - c0) * B_CHUNK;
+            const int64_t end = min(start + (int64_t)B_CHUNK, T.Bptr[b + 1]);
+            int eidx[TB_U];
+#pragma unroll
+            for (int j = 0; j < TB_U; j++) {
+                const int64_t idx = start + lane + j * TG;
+                eidx[j] = idx < end ? __ldg(T.Bedge + idx) : -1;
+            }
+#pragma unroll
+            for (int j = 0; j < TB_U; j++)
+                if (eidx[j] >= 0) top2_push(m1, m2, T.zp[eidx[j]]);
+            tile_top2<TG>(tile, m1, m2);
+            if (lane == 0) {
+                if (c1 - c0 == 1) {
+                    T.Btop[b] = make_double2(m1, m2);
+                } else {
+                    // hub column: the last chunk to finish merges all chunks
+                    T.Bct[c] = make_double2(m1, m2);
+                    __threadfence();
+                    const unsigned int prev = atomicAdd(T.Bcnt + b, 1u);
+                    if (prev == (unsigned int)(c1 - c0 - 1)) {
+                        __threadfence();
+                        double r1 = -INFINITY, r2 = -INFINITY;
+                        for (int64_t cc = c0; cc < c1; cc++) {
+                            const double2 o = __ldcg(T.Bct + cc);
+                            top2_merge(r1, r2, o.x, o.y);
+                        }
+                        T.Btop[b] = make_double2(r1, r2);
+                        T.Bcnt[b] = 0u; // ready for the next iteration
+                    }
+                }
+            }
+        }
+    }
+}
+
+struct EdgeArgs {
+    int64_t m;
+    const int32_t *La, *Lb;
     const double *w;
     double alpha, g, hh, fp_inv;
     unsigned long long *tacc;
     const double *texact;
-    const int64_t *Bcp;
-    const double2 *Bct;
+    const double2 *Atop, *Btop;
     double *yp, *zp, *yc, *zc, *d, *u;
 };
 
-// the per-edge part of lines 10-15 for edge e, given its row's (max1, max2)
-template <bool EXACT, bool LITERAL>
-__device__ __forceinline__ void edge_update(const RowArgs &R, int64_t e, double ype, double zpe, double we,
-                                            double t, int b, double2 atop)
+template <int EPT, bool EXACT, bool LITERAL>
+__global__ void __launch_bounds__(256) k_edge(EdgeArgs R)
 {
-    const double de = R.alpha * we + t;                                   // line 10
-    const double omc = othermax<LITERAL>(zpe, col_top2(b, R.Bcp, R.Bct)); // line 11
-    const double omr = othermax<LITERAL>(ype, atop);                     // line 12
-    const double yce = de - omc;
-    const double zce = de - omr;
-    const double ue = (yce + zce) - de;                                   // line 13 diagonal
-    R.yp[e] = R.g * yce + R.hh * ype;                                     // line 14
-    R.zp[e] = R.g * zce + R.hh * zpe;                                     // line 15
-    R.yc[e] = yce;
-    R.zc[e] = zce;
-    R.d[e] = de;
-    R.u[e] = ue;
-}
-
-template <bool EXACT>
-__device__ __forceinline__ double take_t(const RowArgs &R, int64_t e)
-{
-    if (EXACT) return R.texact[e];
-    const unsigned long long T = R.tacc[e];
-    R.tacc[e] = 0ull; // ready for this iteration's k_square accumulation
-    return __ull2double_rn(T) * R.fp_inv;
-}
-
-// One G-lane tile per A vertex (its L row is contiguous): top-2 of y^p over the
-// row in registers (othermaxrow), then every edge of the row is updated.
-// Rows of up to G*U edges are loaded once into registers.
-template <int G, int U, bool EXACT, bool LITERAL>
-__global__ void __launch_bounds__(256) k_rowA(RowArgs R)
-{
-    auto tile = cg::tiled_partition<G>(cg::this_thread_block());
-    const int lane = tile.thread_rank();
-    const int64_t t0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
-    const int64_t nt = ((int64_t)gridDim.x * blockDim.x) / G;
-    for (int64_t a = t0; a < R.nA; a += nt) {
-        const int64_t lo = R.Arow[a], hi = R.Arow[a + 1];
-        if (hi - lo <= G * U) {
-            double ype[U], zpe[U], we[U];
-            int lb[U];
-            double m1 = -INFINITY, m2 = -INFINITY;
+    const int64_t base = (int64_t)blockIdx.x * blockDim.x * EPT + threadIdx.x;
+    int64_t e[EPT];
+    int a[EPT], b[EPT];
+    double we[EPT], ype[EPT], zpe[EPT], t[EPT];
 #pragma unroll
-            for (int j = 0; j < U; j++) {
-                const int64_t e = lo + lane + j * G;
-                if (e < hi) {
-                    ype[j] = R.yp[e];
-                    zpe[j] = R.zp[e];
-                    we[j] = R.w[e];
-                    lb[j] = R.Lb[e];
-                    top2_push(m1, m2, ype[j]);
-                }
+    for (int j = 0; j < EPT; j++) {
+        e[j] = base + (int64_t)j * blockDim.x;
+        if (e[j] < R.m) {
+            a[j] = __ldg(R.La + e[j]);
+            b[j] = __ldg(R.Lb + e[j]);
+            we[j] = __ldg(R.w + e[j]);
+            ype[j] = R.yp[e[j]];
+            zpe[j] = R.zp[e[j]];
+            if (EXACT) {
+                t[j] = R.texact[e[j]];
+            } else {
+                const unsigned long long T = R.tacc[e[j]];
+                t[j] = __ull2double_rn(T) * R.fp_inv;
             }
-            tile_top2<G>(tile, m1, m2);
-            const double2 atop = make_double2(m1, m2);
-#pragma unroll
-            for (int j = 0; j < U; j++) {
-                const int64_t e = lo + lane + j * G;
-                if (e < hi) edge_update<EXACT, LITERAL>(R, e, ype[j], zpe[j], we[j], take_t<EXACT>(R, e), lb[j], atop);
-            }
-        } else {
-            double m1 = -INFINITY, m2 = -INFINITY;
-            for (int64_t e = lo + lane; e < hi; e += G) top2_push(m1, m2, R.yp[e]);
-            tile_top2<G>(tile, m1, m2);
-            tile.sync(); // every lane has read its old y^p before any is overwritten
-            const double2 atop = make_double2(m1, m2);
-            for (int64_t e = lo + lane; e < hi; e += G)
-                edge_update<EXACT, LITERAL>(R, e, R.yp[e], R.zp[e], R.w[e], take_t<EXACT>(R, e), R.Lb[e], atop);
         }
     }
-}
-
-__global__ void k_chunk_count(int64_t nB, const int64_t *__restrict__ Bptr, int64_t *__restrict__ cnt)
-{
-    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nB; b += (int64_t)gridDim.x * blockDim.x)
-        cnt[b] = (Bptr[b + 1] - Bptr[b] + B_CHUNK - 1) / B_CHUNK;
-}
-
-__global__ void k_chunk_fill(int64_t nB, const int64_t *__restrict__ Bcp, int32_t *__restrict__ chunk_b)
-{
-    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nB; b += (int64_t)gridDim.x * blockDim.x)
-        for (int64_t c = Bcp[b]; c < Bcp[b + 1]; c++) chunk_b[c] = (int32_t)b;
+#pragma unroll
+    for (int j = 0; j < EPT; j++) {
+        if (e[j] >= R.m) continue;
+        const double2 at = __ldg(R.Atop + a[j]);
+        const double2 bt = __ldg(R.Btop + b[j]);
+        const double de = R.alpha * we[j] + t[j];          // line 10
+        const double omc = othermax<LITERAL>(zpe[j], bt);  // line 11
+        const double omr = othermax<LITERAL>(ype[j], at);  // line 12
+        const double yce = de - omc;
+        const double zce = de - omr;
+        const double ue = (yce + zce) - de;                // line 13 diagonal
+        R.yp[e[j]] = R.g * yce + R.hh * ype[j];            // line 14
+        R.zp[e[j]] = R.g * zce + R.hh * zpe[j];            // line 15
+        R.yc[e[j]] = yce;
+        R.zc[e[j]] = zce;
+        R.d[e[j]] = de;
+        R.u[e[j]] = ue;
+        if (!EXACT) R.tacc[e[j]] = 0ull; // ready for this iteration's k_square
+    }
 }
 
 // segmented (by sorted key) warp sum, then one atomic per segment
@@ -248,8 +231,8 @@ __device__ __forceinline__ void seg_atomic_add(unsigned long long v, int key, in
     if (head && key >= 0 && v) atomicAdd(dst + key, v);
 }
 
-// MODE: UPDATE = apply lines 9, 13, 16 to the pair; otherwise only (re)compute
-// the F row sums of the current S^p (init, set_state).
+// UPDATE = apply lines 9, 13, 16 to the pair; otherwise only (re)compute the
+// F row sums of the current S^p (init, set_state).
 template <bool UPDATE, bool EXACT>
 __global__ void __launch_bounds__(256)
 k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_val,
@@ -328,6 +311,18 @@ __global__ void k_gather_Sp(int64_t nsq, double2 *__restrict__ sq_val, const lon
     }
 }
 
+__global__ void k_chunk_count(int64_t nB, const int64_t *__restrict__ Bptr, int64_t *__restrict__ cnt)
+{
+    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nB; b += (int64_t)gridDim.x * blockDim.x)
+        cnt[b] = (Bptr[b + 1] - Bptr[b] + B_CHUNK - 1) / B_CHUNK;
+}
+
+__global__ void k_chunk_fill(int64_t nB, const int64_t *__restrict__ Bcp, int32_t *__restrict__ chunk_b)
+{
+    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nB; b += (int64_t)gridDim.x * blockDim.x)
+        for (int64_t c = Bcp[b]; c < Bcp[b + 1]; c++) chunk_b[c] = (int32_t)b;
+}
+
 int square_grid(cualign_bp *h)
 {
     // persistent-style grid: 8 resident 256-thread CTAs per SM
@@ -340,21 +335,12 @@ cualign_status launch_square(cualign_bp *h, bool update, double g, double hh)
     if (h->nsq > 0) {
         KScope ks(h, CUALIGN_K_SQUARE);
         const int grid = square_grid(h);
-        if (update) {
-            if (exact)
-                k_square<true, true><<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, g, hh,
-                                                                  h->fp_scale, h->tacc, h->sq_pos, h->Ffull);
-            else
-                k_square<true, false><<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, g,
-                                                                   hh, h->fp_scale, h->tacc, h->sq_pos, h->Ffull);
-        } else {
-            if (exact)
-                k_square<false, true><<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, g,
-                                                                   hh, h->fp_scale, h->tacc, h->sq_pos, h->Ffull);
-            else
-                k_square<false, false><<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, g,
-                                                                    hh, h->fp_scale, h->tacc, h->sq_pos, h->Ffull);
-        }
+#define SQ_ARGS h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, g, hh, h->fp_scale, h->tacc, h->sq_pos, h->Ffull
+        if (update && exact) k_square<true, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+        else if (update) k_square<true, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+        else if (exact) k_square<false, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+        else k_square<false, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+#undef SQ_ARGS
         CA_CUDA(cudaGetLastError());
     }
     if (exact) {
@@ -370,9 +356,13 @@ cualign_status launch_square(cualign_bp *h, bool update, double g, double hh)
 
 cualign_status bp_setup(cualign_bp *h)
 {
-    // B-side chunks for k_top2B
     KScope ks(h, CUALIGN_K_INIT);
-    const int64_t nB = h->L.nB;
+    const int64_t nA = h->L.nA, nB = h->L.nB;
+    CA_TRY(dalloc(h, &h->Atop, (size_t)nA + 1));
+    CA_TRY(dalloc(h, &h->Btop, (size_t)nB + 1));
+    CA_TRY(dalloc(h, &h->Bcnt, (size_t)nB + 1));
+    CA_CUDA(cudaMemsetAsync(h->Bcnt, 0, sizeof(unsigned int) * ((size_t)nB + 1), h->stream));
+    // B-side chunks for k_top2
     CA_TRY(dalloc(h, &h->Bcp, (size_t)nB + 1));
     CA_CUDA(cudaMemsetAsync(h->Bcp, 0, sizeof(int64_t), h->stream));
     if (nB > 0) {
@@ -413,22 +403,23 @@ cualign_status bp_iterate(cualign_bp *h, int32_t n)
         const double g = pow(h->gamma, (double)p); // reading Z2: host fp64 gamma^p
         const double hh = 1.0 - g;
         if (m > 0) {
-            if (h->nchunks > 0) {
+            {
                 KScope ks(h, CUALIGN_K_TOP2);
-                k_top2B<<<grid_for(h->nchunks * TB_G, 256, 1 << 30), 256, 0, h->stream>>>(
-                    h->nchunks, h->chunk_b, h->Bcp, h->L.Bptr, h->L.Bedge, h->zp, h->Bct);
+                Top2Args T{(int64_t)h->L.nA, h->nchunks, h->L.Arow, h->chunk_b, h->Bcp, h->L.Bptr, h->L.Bedge,
+                           h->yp, h->zp, h->Atop, h->Btop, h->Bct, h->Bcnt};
+                k_top2<<<grid_for((T.nA + T.nchunks) * TG, 256, 1 << 30), 256, 0, h->stream>>>(T);
                 CA_CUDA(cudaGetLastError());
             }
             {
                 KScope ks(h, CUALIGN_K_EDGE);
-                RowArgs R{(int64_t)h->L.nA, h->L.Arow, h->L.Lb, h->L.w, h->alpha, g, hh, h->fp_inv, h->tacc,
-                          h->texact, h->Bcp, h->Bct, h->yp, h->zp, h->yc, h->zc, h->d, h->u};
-                constexpr int G = 8, U = 3;
-                const int grid = grid_for((int64_t)h->L.nA * G, 256, 1 << 30);
-                if (exact && literal) k_rowA<G, U, true, true><<<grid, 256, 0, h->stream>>>(R);
-                else if (exact) k_rowA<G, U, true, false><<<grid, 256, 0, h->stream>>>(R);
-                else if (literal) k_rowA<G, U, false, true><<<grid, 256, 0, h->stream>>>(R);
-                else k_rowA<G, U, false, false><<<grid, 256, 0, h->stream>>>(R);
+                EdgeArgs R{m, h->L.La, h->L.Lb, h->L.w, h->alpha, g, hh, h->fp_inv, h->tacc, h->texact,
+                           h->Atop, h->Btop, h->yp, h->zp, h->yc, h->zc, h->d, h->u};
+                constexpr int EPT = 4;
+                const int grid = grid_for((m + EPT - 1) / EPT, 256, 1 << 30);
+                if (exact && literal) k_edge<EPT, true, true><<<grid, 256, 0, h->stream>>>(R);
+                else if (exact) k_edge<EPT, true, false><<<grid, 256, 0, h->stream>>>(R);
+                else if (literal) k_edge<EPT, false, true><<<grid, 256, 0, h->stream>>>(R);
+                else k_edge<EPT, false, false><<<grid, 256, 0, h->stream>>>(R);
                 CA_CUDA(cudaGetLastError());
             }
             CA_TRY(launch_square(h, true, g, hh));

@@ -102,6 +102,8 @@ struct cualign_bp {
     int64_t *Bcp = nullptr;             // nB+1: chunks of B vertex b are Bcp[b]..Bcp[b+1]-1
     int32_t *chunk_b = nullptr;         // nchunks: owning B vertex
     double2 *Bct = nullptr;             // nchunks: (max1, max2) of z^p over the chunk
+    unsigned int *Bcnt = nullptr;       // nB: chunks finished (hub columns' last-arriver merge)
+    double2 *Atop = nullptr, *Btop = nullptr; // per-vertex (max1, max2) of y^p / z^p
     int32_t p = 0;
 
     // matching (two instances: y and z)
@@ -111,6 +113,7 @@ struct cualign_bp {
     int match_grid = 0, match_block = 256, eval_grid = 1;
     unsigned long long *match_work = nullptr; // proposals (suitor) or rounds, per instance
     bool propose_from_b = false;              // suitor: proposing side (smaller max degree)
+    uint8_t *mflag = nullptr;                 // [2][m]: edge in M_y / M_z (evaluate)
     int64_t max_deg_a = 0, max_deg_b = 0;     // max degree of A / B vertices in L
     cualign::RoundDev *rd = nullptr;
     cualign_round_info last_info{};

@@ -248,16 +248,31 @@ __global__ void __launch_bounds__(256) k_pointer_rounds(MatchParams P)
 
 // ------------------------------------------------------- mates from suitors
 // the final suitor of each target is its mate (mateX arrays pre-set to -1)
+// and every matched edge is flagged in mflag (pre-cleared) for the evaluation
 __global__ void k_suitor_to_mates(int64_t nT, int ninst, const int32_t *__restrict__ own,
                                   const int32_t *__restrict__ sT, int32_t *__restrict__ mateT,
-                                  int32_t *__restrict__ mateP, int64_t nP)
+                                  int32_t *__restrict__ mateP, int64_t nP, uint8_t *__restrict__ mflag, int64_t m)
 {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * nT;
          v += (int64_t)gridDim.x * blockDim.x) {
         const int k = (int)(v / nT);
         const int e = sT[v];
         mateT[v] = e;
-        if (e >= 0) mateP[k * nP + own[e]] = e;
+        if (e >= 0) {
+            mateP[k * nP + own[e]] = e;
+            mflag[k * m + e] = 1;
+        }
+    }
+}
+
+// pointer-round schedule: flag the matched edges from mate_A
+__global__ void k_mark(int64_t nA, int ninst, const int32_t *__restrict__ mateA, uint8_t *__restrict__ mflag,
+                       int64_t m)
+{
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * nA;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        const int e = mateA[v];
+        if (e >= 0) mflag[(v / nA) * m + e] = 1;
     }
 }
 
@@ -289,6 +304,8 @@ struct EvalParams {
     const int64_t *sq_rp;
     const int2 *sq_ef;
     const int32_t *mateA; // 2 instances, final
+    const uint8_t *mflag; // [2][m]: edge matched
+    int64_t m;
     double *partial_w;    // [2][gridDim]
     RoundDev *rd;
 };
@@ -318,7 +335,7 @@ __global__ void __launch_bounds__(256) k_eval(EvalParams P)
             const int64_t hi = P.sq_rp[e + 1];
             for (int64_t q = P.sq_rp[e] + lane; q < hi; q += G) {
                 const int f = P.sq_ef[q].y;
-                if (mA[P.La[f]] == f) ov++;
+                if (P.mflag[k * P.m + f]) ov++;
             }
         }
         const double bw = block_sum<double>(wsum, sd);
@@ -435,13 +452,19 @@ MatchParams base_params(cualign_bp *h)
 // run the matching of ninst instances; leaves mateA / mateB final
 cualign_status run_matching(cualign_bp *h, MatchParams &P)
 {
-    const int64_t nA = h->L.nA, nB = h->L.nB;
+    const int64_t nA = h->L.nA, nB = h->L.nB, m = h->L.m;
     CA_CUDA(cudaMemsetAsync(h->match_work, 0, 2 * sizeof(unsigned long long), h->stream));
+    CA_CUDA(cudaMemsetAsync(h->mflag, 0, (size_t)(2 * m + 1), h->stream));
     if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) {
+        {
+            KScope ks(h, CUALIGN_K_MATCH);
+            void *args[] = {&P};
+            CA_CUDA(cudaLaunchCooperativeKernel((void *)k_pointer_rounds, dim3(h->match_grid), dim3(256), args, 0,
+                                                h->stream));
+        }
         KScope ks(h, CUALIGN_K_MATCH);
-        void *args[] = {&P};
-        CA_CUDA(cudaLaunchCooperativeKernel((void *)k_pointer_rounds, dim3(h->match_grid), dim3(256), args, 0,
-                                            h->stream));
+        k_mark<<<grid_for(P.ninst * nA, 256, h->num_sms * 8), 256, 0, h->stream>>>(nA, P.ninst, P.mateA, h->mflag, m);
+        CA_CUDA(cudaGetLastError());
         return CUALIGN_OK;
     }
     const bool fromB = h->propose_from_b;
@@ -462,7 +485,8 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     if (P.ninst * nT > 0) {
         KScope ks(h, CUALIGN_K_MATCH);
         k_suitor_to_mates<<<grid_for(P.ninst * nT, 256, h->num_sms * 8), 256, 0, h->stream>>>(
-            nT, P.ninst, fromB ? P.Lb : P.La, sT, fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP);
+            nT, P.ninst, fromB ? P.Lb : P.La, sT, fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP,
+            h->mflag, m);
         CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;
@@ -480,6 +504,7 @@ cualign_status match_setup(cualign_bp *h)
     CA_TRY(dalloc(h, &h->best_mate, nA + 1));
     CA_TRY(dalloc(h, &h->rd, 1));
     CA_TRY(dalloc(h, &h->match_work, 2));
+    CA_TRY(dalloc(h, &h->mflag, (size_t)(2 * h->L.m + 1)));
     CA_CUDA(cudaMemsetAsync(h->rd, 0, sizeof(RoundDev), h->stream));
     CA_CUDA(cudaMemsetAsync(h->mateA, 0xff, sizeof(int32_t) * (2 * nA + 1), h->stream));
     CA_CUDA(cudaMemsetAsync(h->mateB, 0xff, sizeof(int32_t) * (2 * nB + 1), h->stream));
@@ -523,6 +548,8 @@ cualign_status match_round(cualign_bp *h)
     E.sq_rp = h->sq_rp;
     E.sq_ef = h->sq_ef;
     E.mateA = h->mateA;
+    E.mflag = h->mflag;
+    E.m = h->L.m;
     E.partial_w = h->partial_w;
     E.rd = h->rd;
     // overlap / card accumulators (the rest of rd persists: best)
