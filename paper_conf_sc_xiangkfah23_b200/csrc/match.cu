@@ -87,20 +87,39 @@ __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
     const int32_t *__restrict__ tgt = fromB ? P.La : P.Lb;   // target vertex of an edge
     const int32_t *__restrict__ own = fromB ? P.Lb : P.La;   // proposer vertex of an edge
     unsigned long long proposals = 0;
+    constexpr int U = 3; // edges per lane per pass: loads of a pass are issued together
     while (true) {
         // heaviest eligible neighbour of `cur` whose suitor is lighter
         int best = -1;
         double bx = 0.0;
         const int64_t hi = rp[cur + 1];
-        for (int64_t j = rp[cur] + lane; j < hi; j += G) {
-            const int e = fromB ? __ldg(P.Bedge + j) : (int)j;
-            const double xe = __ldg(x + e);
-            if (!(xe > 0.0)) continue;
-            if (!better(xe, e, bx, best)) continue;
-            const int s = *(volatile int32_t *)(sT + __ldg(tgt + e));
-            if (s >= 0 && !better(xe, e, __ldg(x + s), s)) continue;
-            best = e;
-            bx = xe;
+        for (int64_t j0 = rp[cur] + lane; j0 < hi; j0 += G * U) {
+            int ee[U], tt[U], ss[U];
+            double xx[U], xs[U];
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                const int64_t j = j0 + u * G;
+                ee[u] = -1;
+                if (j < hi) {
+                    const int e = fromB ? __ldg(P.Bedge + j) : (int)j;
+                    xx[u] = __ldg(x + e);
+                    tt[u] = __ldg(tgt + e);
+                    ee[u] = (xx[u] > 0.0) ? e : -1; // only x > 0 is eligible (Z6)
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < U; u++) ss[u] = ee[u] >= 0 ? *(volatile int32_t *)(sT + tt[u]) : -1;
+#pragma unroll
+            for (int u = 0; u < U; u++) xs[u] = ss[u] >= 0 ? __ldg(x + ss[u]) : 0.0;
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                if (ee[u] < 0) continue;
+                if (ss[u] >= 0 && !better(xx[u], ee[u], xs[u], ss[u])) continue;
+                if (better(xx[u], ee[u], bx, best)) {
+                    best = ee[u];
+                    bx = xx[u];
+                }
+            }
         }
 #pragma unroll
         for (int off = G / 2; off >= 1; off >>= 1) {
