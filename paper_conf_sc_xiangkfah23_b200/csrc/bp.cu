@@ -240,40 +240,67 @@ k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_v
          unsigned long long *__restrict__ tacc, const longlong2 *__restrict__ sq_pos,
          double *__restrict__ Ffull)
 {
+    // SQ_U warp-rows of 32 squares per pass: all streaming loads of a pass are
+    // issued before any use (memory-level parallelism); the square arrays are
+    // streamed with evict-first hints (__ldcs / __stcs) so that the per-edge u
+    // and the accumulator tacc stay resident in L2.
+    constexpr int SQ_U = 2;
     const int lane = threadIdx.x & 31;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t base = warp * 32; base < nsq; base += nwarps * 32) {
-        const int64_t q = base + lane;
-        int key = -1 - lane;
-        unsigned long long Tef = 0ull;
-        if (q < nsq) {
-            const int2 ef = sq_ef[q];
-            double2 v = sq_val[q]; // (S^p_ef, S^p_fe)
-            if (UPDATE) {
-                const double Fef = clamp_beta(beta + v.y, beta);    // line 9
-                const double Ffe = clamp_beta(beta + v.x, beta);
-                const double Scef = u[ef.x] - Fef;                  // line 13
-                const double Scfe = u[ef.y] - Ffe;
-                v.x = g * Scef + hh * v.x;                          // line 16
-                v.y = g * Scfe + hh * v.y;
-                sq_val[q] = v;
-            }
-            // F of the next iteration (line 9 at p+1) from the new pair
-            const double Nef = clamp_beta(beta + v.y, beta);
-            const double Nfe = clamp_beta(beta + v.x, beta);
-            if (EXACT) {
-                const longlong2 pos = sq_pos[q];
-                Ffull[pos.x] = Nef;
-                Ffull[pos.y] = Nfe;
-            } else {
-                const unsigned long long Tfe = __double2ull_rn(Nfe * fp_scale);
-                if (Tfe) atomicAdd(tacc + ef.y, Tfe);
-                Tef = __double2ull_rn(Nef * fp_scale);
-                key = ef.x;
+    for (int64_t base = warp * 32 * SQ_U; base < nsq; base += nwarps * 32 * SQ_U) {
+        int2 ef[SQ_U];
+        double2 v[SQ_U];
+        double ue[SQ_U], uf[SQ_U];
+#pragma unroll
+        for (int j = 0; j < SQ_U; j++) {
+            const int64_t q = base + j * 32 + lane;
+            if (q < nsq) {
+                ef[j] = __ldcs(sq_ef + q);
+                v[j] = __ldcs(sq_val + q); // (S^p_ef, S^p_fe)
             }
         }
-        if (!EXACT) seg_atomic_add(Tef, key, lane, tacc);
+        if (UPDATE) {
+#pragma unroll
+            for (int j = 0; j < SQ_U; j++) {
+                const int64_t q = base + j * 32 + lane;
+                if (q < nsq) {
+                    ue[j] = __ldg(u + ef[j].x);
+                    uf[j] = __ldg(u + ef[j].y);
+                }
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < SQ_U; j++) {
+            const int64_t q = base + j * 32 + lane;
+            int key = -1 - lane;
+            unsigned long long Tef = 0ull;
+            if (q < nsq) {
+                if (UPDATE) {
+                    const double Fef = clamp_beta(beta + v[j].y, beta);    // line 9
+                    const double Ffe = clamp_beta(beta + v[j].x, beta);
+                    const double Scef = ue[j] - Fef;                       // line 13
+                    const double Scfe = uf[j] - Ffe;
+                    v[j].x = g * Scef + hh * v[j].x;                       // line 16
+                    v[j].y = g * Scfe + hh * v[j].y;
+                    __stcs(sq_val + q, v[j]);
+                }
+                // F of the next iteration (line 9 at p+1) from the new pair
+                const double Nef = clamp_beta(beta + v[j].y, beta);
+                const double Nfe = clamp_beta(beta + v[j].x, beta);
+                if (EXACT) {
+                    const longlong2 pos = sq_pos[q];
+                    Ffull[pos.x] = Nef;
+                    Ffull[pos.y] = Nfe;
+                } else {
+                    const unsigned long long Tfe = __double2ull_rn(Nfe * fp_scale);
+                    if (Tfe) atomicAdd(tacc + ef[j].y, Tfe);
+                    Tef = __double2ull_rn(Nef * fp_scale);
+                    key = ef[j].x;
+                }
+            }
+            if (!EXACT) seg_atomic_add(Tef, key, lane, tacc);
+        }
     }
 }
 

@@ -135,9 +135,12 @@ __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
         int next = cur;
         if (lane == 0) {
             int32_t *slotp = sT + __ldg(tgt + best);
-            const int s = *(volatile int32_t *)slotp;
-            if (s < 0 || better(bx, best, __ldg(x + s), s)) {
-                if (atomicCAS(slotp, s, best) == s) {
+            int s = *(volatile int32_t *)slotp;
+            // CAS loop: retry directly while our edge still beats the occupant,
+            // rescan the list only when it does not
+            while (s < 0 || better(bx, best, __ldg(x + s), s)) {
+                const int old = atomicCAS(slotp, s, best);
+                if (old == s) {
                     proposals++;
                     if (s < 0) {
                         code = 1;
@@ -145,7 +148,9 @@ __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
                         code = 2;
                         next = __ldg(own + s); // the displaced proposer proposes again
                     }
+                    break;
                 }
+                s = old;
             }
         }
         code = tile.shfl(code, 0);
