@@ -224,6 +224,7 @@ def main():
     ap.add_argument("--ref-scale", type=float, default=0.05)
     ap.add_argument("--exact", action="store_true", help="CUALIGN_FLAG_EXACT (oracle-order sums)")
     ap.add_argument("--match-rounds", action="store_true", help="pointer-round matching schedule")
+    ap.add_argument("--prof-steps", type=int, default=20, help="steps of the per-kernel timing pass")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
@@ -245,8 +246,7 @@ def main():
     log(f"[rank {rank}] generated {args.config} (scale {args.scale}) in {t_gen:.1f}s: "
         f"n_A={inst.A.n} n_B={inst.B.n} m={inst.L.m}")
     stream = torch.cuda.current_stream()
-    flags = ca.FLAG_TIMING | (ca.FLAG_EXACT if args.exact else 0) | \
-        (ca.FLAG_MATCH_ROUNDS if args.match_rounds else 0)
+    flags = (ca.FLAG_EXACT if args.exact else 0) | (ca.FLAG_MATCH_ROUNDS if args.match_rounds else 0)
 
     # ---------------------------------------------------------------- init
     torch.cuda.synchronize()
@@ -261,9 +261,8 @@ def main():
         f"fp_bits={sz['fixed_point_bits']} device_bytes={sz['device_bytes']/1e9:.2f}GB")
 
     # ------------------------------------------------------------- warmup
-    for _ in range(args.warmup):
-        h.iterate(1)
-        h.round(sync=False)
+    # (each step = iterate(1) + round, replayed from the library's CUDA graph)
+    h.run(args.warmup)
     torch.cuda.synchronize()
     h.stats(reset=True)
     barrier(world)
@@ -276,9 +275,7 @@ def main():
     torch.cuda.synchronize()
     barrier(world)
     ev0.record(stream)
-    for _ in range(args.steps):
-        h.iterate(1)
-        h.round(sync=False)
+    h.run(args.steps)
     ev1.record(stream)
     torch.cuda.synchronize()
     barrier(world)
@@ -288,14 +285,23 @@ def main():
     st = h.stats(reset=True)
     _, info = h.get_best()
 
+    # ----------------------------------------------- per-kernel timing pass
+    # event-record nodes inside the captured step graph, read after each replay
+    prof_steps = max(1, min(args.prof_steps, args.steps))
+    h.set_timing(True)
+    h.run(prof_steps)
+    h.set_timing(False)
+    torch.cuda.synchronize()
+    pst = h.stats(reset=True)
+
     steps_total = args.steps * world
     value = steps_total / (elapsed_ms / 1e3)
     ms_per_step = elapsed_ms / args.steps
-    cls_ms = st["class_ms"]
-    cls_n = st["class_launches"]
+    cls_ms = pst["class_ms"]
+    cls_n = pst["class_launches"]
     sq_ms = cls_ms["square"] / max(cls_n["square"], 1)
-    bp_ms = (cls_ms["top2"] + cls_ms["edge"] + cls_ms["square"] + cls_ms["rowsum"]) / args.steps
-    round_ms = cls_ms["match"] / max(cls_n["match"], 1)
+    bp_ms = (cls_ms["top2"] + cls_ms["edge"] + cls_ms["square"] + cls_ms["rowsum"] + cls_ms["other"]) / prof_steps
+    round_ms = cls_ms["match"] / prof_steps
     peak, peak_src = read_peaks()
     sq_bytes = BYTES_PER_NZ * s                    # algorithmic bytes of one square-pass launch
     sq_gbs = sq_bytes / (sq_ms * 1e-3) / 1e9 if sq_ms > 0 else 0.0
@@ -384,7 +390,9 @@ def main():
                      "launch_ms": sq_ms, "peak_source": peak_src},
         "iteration_roofline": {"achieved": it_gbs, "frac": it_gbs / peak, "alg_bytes": it_bytes,
                                "bp_ms": bp_ms},
-        "kernel_ms_per_step": {k: v / args.steps for k, v in cls_ms.items() if v},
+        "kernel_ms_per_step": {k: v / prof_steps for k, v in cls_ms.items() if v},
+        "kernel_timing": (f"CUDA event-record nodes around each kernel inside the captured step "
+                          f"graph, {prof_steps} steps after the timed region"),
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": st["launches"],

@@ -167,6 +167,18 @@ cualign_status cualign_bp_iterate(cualign_bp *h, int32_t n_steps);
  * (best is tracked on the device); otherwise synchronises and fills *info. */
 cualign_status cualign_bp_round(cualign_bp *h, cualign_round_info *info);
 
+/* a3-a8 repeated: n_steps x (iterate(1), then round if with_round != 0),
+ * replayed from a CUDA graph of one step captured on first use (no host work
+ * per kernel; g = gamma^p is read by the kernels from a host-computed table,
+ * reading Z2).  Same results as the equivalent sequence of iterate/round
+ * calls.  Asynchronous on params.stream; read results with get_best. */
+cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t with_round);
+
+/* Diagnostics: enable (1) / disable (0) per-kernel event timing (as
+ * CUALIGN_FLAG_TIMING).  Graph replays with timing on synchronise after each
+ * step to read the per-kernel events; results via cualign_bp_get_stats. */
+cualign_status cualign_bp_set_timing(cualign_bp *h, int32_t on);
+
 /* Best matching so far: mate_a[a] = canonical id of the L edge matched at A
  * vertex a, or -1 (host buffer of n_A int32; may be NULL).  info receives the
  * last round's info with best_score / best_iter (may be NULL). Synchronises. */

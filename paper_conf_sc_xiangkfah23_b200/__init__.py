@@ -15,8 +15,8 @@ def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=
     with CuAlignBP(A, B, L, alpha, beta, gamma, flags, device, stream) as h:
         infos = []
         for _ in range(n_iter):
-            h.iterate(1)
-            infos.append(h.round(sync=True))
+            h.run(1)                                      # graph replay of iterate + round
+            infos.append(h.get_best(with_mate=False)[1])  # the step's result to the host
         mate, info = h.get_best()
     return mate, info, infos
 

@@ -27,7 +27,8 @@ KERNEL_CLASS_NAMES = ["top2", "edge", "square", "rowsum", "match", "init", "stat
 NUM_KERNEL_CLASSES = 8
 
 # every symbol include/cualign_bp.h declares
-EXPORTED = ["cualign_bp_init", "cualign_bp_iterate", "cualign_bp_round", "cualign_bp_get_best",
+EXPORTED = ["cualign_bp_init", "cualign_bp_iterate", "cualign_bp_round", "cualign_bp_run",
+            "cualign_bp_set_timing", "cualign_bp_get_best",
             "cualign_bp_free", "cualign_bp_get_sizes", "cualign_bp_get_S", "cualign_bp_get_state",
             "cualign_bp_set_state", "cualign_bp_get_stats", "cualign_match", "cualign_last_error",
             "cualign_version"]
@@ -109,6 +110,10 @@ def load_library():
     lib.cualign_bp_iterate.argtypes = [P, I32]
     lib.cualign_bp_round.restype = I32
     lib.cualign_bp_round.argtypes = [P, P]
+    lib.cualign_bp_run.restype = I32
+    lib.cualign_bp_run.argtypes = [P, I32, I32]
+    lib.cualign_bp_set_timing.restype = I32
+    lib.cualign_bp_set_timing.argtypes = [P, I32]
     lib.cualign_bp_get_best.restype = I32
     lib.cualign_bp_get_best.argtypes = [P, P, P]
     lib.cualign_bp_free.restype = None
@@ -234,6 +239,13 @@ class CuAlignBP:
     def iterate(self, n_steps=1):
         _check(load_library().cualign_bp_iterate(self._h, int(n_steps)))
 
+    def run(self, n_steps=1, with_round=True):
+        """n_steps x (iterate(1) [+ round]) replayed from a CUDA graph (async)."""
+        _check(load_library().cualign_bp_run(self._h, int(n_steps), 1 if with_round else 0))
+
+    def set_timing(self, on=True):
+        _check(load_library().cualign_bp_set_timing(self._h, 1 if on else 0))
+
     def round(self, sync=True):
         if not sync:
             _check(load_library().cualign_bp_round(self._h, None))
@@ -242,11 +254,11 @@ class CuAlignBP:
         _check(load_library().cualign_bp_round(self._h, ctypes.byref(info)))
         return info.as_dict()
 
-    def get_best(self):
-        mate = np.zeros(max(self.n_a, 1), dtype=np.int32)
+    def get_best(self, with_mate=True):
+        mate = np.zeros(max(self.n_a, 1), dtype=np.int32) if with_mate else None
         info = RoundInfo_t()
         _check(load_library().cualign_bp_get_best(self._h, _ptr(mate), ctypes.byref(info)))
-        return mate[:self.n_a], info.as_dict()
+        return (mate[:self.n_a] if with_mate else None), info.as_dict()
 
     # introspection
     def sizes(self):

@@ -66,11 +66,14 @@ static cudaEvent_t get_event(cualign_bp *h)
     return e;
 }
 
+// While a graph is being captured, timing events become event-record nodes
+// (cudaEventRecordExternal) owned by the graph; they are read after each replay.
 KScope::KScope(cualign_bp *h_, int cls_) : h(h_), cls(cls_)
 {
     if (h->timing) {
         b = get_event(h);
-        cudaEventRecord(b, h->stream);
+        if (h->capturing) cudaEventRecordWithFlags(b, h->stream, cudaEventRecordExternal);
+        else cudaEventRecord(b, h->stream);
     }
 }
 
@@ -80,9 +83,108 @@ KScope::~KScope()
     h->class_launches[cls]++;
     if (h->timing && b) {
         cudaEvent_t e = get_event(h);
-        cudaEventRecord(e, h->stream);
-        h->events[cls].push_back({b, e});
+        if (h->capturing) {
+            cudaEventRecordWithFlags(e, h->stream, cudaEventRecordExternal);
+            h->graph_events[1].push_back({cls, {b, e}});
+        } else {
+            cudaEventRecord(e, h->stream);
+            h->events[cls].push_back({b, e});
+        }
     }
+}
+
+void invalidate_graphs(cualign_bp *h)
+{
+    for (int t = 0; t < 2; t++)
+        for (int r = 0; r < 2; r++)
+            if (h->graph[t][r]) {
+                cudaGraphExecDestroy(h->graph[t][r]);
+                h->graph[t][r] = nullptr;
+            }
+    for (auto &pe : h->graph_events[1]) {
+        h->event_pool.push_back(pe.second.a);
+        h->event_pool.push_back(pe.second.b);
+    }
+    h->graph_events[1].clear();
+}
+
+// Capture one step (iterate(1) [+ round]) on the handle's capture stream.
+static cualign_status capture_step(cualign_bp *h, int timed, int with_round)
+{
+    const int32_t p_save = h->p;
+    const int64_t l0 = h->launches;
+    int64_t c0[CUALIGN_NUM_KERNEL_CLASSES];
+    for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) c0[c] = h->class_launches[c];
+    const bool timing_save = h->timing;
+    cudaStream_t user = h->stream;
+    h->timing = timed != 0;
+    h->stream = h->gstream;
+    h->capturing = true;
+    cualign_status st = CUALIGN_OK;
+    cudaError_t e = cudaStreamBeginCapture(h->gstream, cudaStreamCaptureModeThreadLocal);
+    if (e == cudaSuccess) {
+        st = bp_iterate(h, 1);
+        if (st == CUALIGN_OK && with_round) st = match_round(h);
+        cudaGraph_t g = nullptr;
+        cudaError_t e2 = cudaStreamEndCapture(h->gstream, &g);
+        if (st == CUALIGN_OK && e2 != cudaSuccess) {
+            set_error("graph capture: %s", cudaGetErrorString(e2));
+            st = CUALIGN_ECUDA;
+        }
+        if (st == CUALIGN_OK) {
+            e2 = cudaGraphInstantiate(&h->graph[timed][with_round], g, 0);
+            if (e2 != cudaSuccess) {
+                set_error("graph instantiate: %s", cudaGetErrorString(e2));
+                st = CUALIGN_ECUDA;
+            }
+        }
+        if (g) cudaGraphDestroy(g);
+    } else {
+        set_error("graph capture: %s", cudaGetErrorString(e));
+        st = CUALIGN_ECUDA;
+    }
+    h->capturing = false;
+    h->stream = user;
+    h->timing = timing_save;
+    h->p = p_save;
+    h->graph_launches[timed][with_round] = h->launches - l0;
+    for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
+        h->graph_class_launches[timed][with_round][c] = h->class_launches[c] - c0[c];
+        h->class_launches[c] = c0[c];
+    }
+    h->launches = l0;
+    (void)cudaGetLastError();
+    return st;
+}
+
+// n steps through the captured graph; the user stream and the capture stream
+// are ordered with events, so the caller's stream semantics are preserved.
+static cualign_status run_graph(cualign_bp *h, int32_t n, int with_round)
+{
+    const int timed = h->timing ? 1 : 0;
+    CA_TRY(ensure_gh(h, (int64_t)h->p + n + 1));
+    if (!h->graph[timed][with_round]) CA_TRY(capture_step(h, timed, with_round));
+    cudaGraphExec_t ge = h->graph[timed][with_round];
+    CA_CUDA(cudaEventRecord(h->sync_ev[0], h->stream));
+    CA_CUDA(cudaStreamWaitEvent(h->gstream, h->sync_ev[0], 0));
+    for (int32_t k = 0; k < n; k++) {
+        CA_CUDA(cudaGraphLaunch(ge, h->gstream));
+        h->p += 1;
+        h->launches += h->graph_launches[timed][with_round];
+        for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++)
+            h->class_launches[c] += h->graph_class_launches[timed][with_round][c];
+        if (timed) {
+            CA_CUDA(cudaStreamSynchronize(h->gstream));
+            for (auto &pe : h->graph_events[1]) {
+                float ms = 0.f;
+                if (cudaEventElapsedTime(&ms, pe.second.a, pe.second.b) == cudaSuccess) h->class_ms[pe.first] += ms;
+            }
+        }
+    }
+    if (with_round) h->have_info = true;
+    CA_CUDA(cudaEventRecord(h->sync_ev[1], h->gstream));
+    CA_CUDA(cudaStreamWaitEvent(h->stream, h->sync_ev[1], 0));
+    return CUALIGN_OK;
 }
 
 static void resolve_events(cualign_bp *h)
@@ -144,6 +246,9 @@ static cualign_status open_handle(const cualign_params *params, cualign_bp **out
         CA_CUDA(cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking));
         h->own_stream = true;
     }
+    CA_CUDA(cudaStreamCreateWithFlags(&h->gstream, cudaStreamNonBlocking));
+    CA_CUDA(cudaEventCreateWithFlags(&h->sync_ev[0], cudaEventDisableTiming));
+    CA_CUDA(cudaEventCreateWithFlags(&h->sync_ev[1], cudaEventDisableTiming));
     return CUALIGN_OK;
 }
 
@@ -152,10 +257,15 @@ static void close_handle(cualign_bp *h)
     if (!h) return;
     cudaSetDevice(h->dev);
     if (h->stream) cudaStreamSynchronize(h->stream);
+    if (h->gstream) cudaStreamSynchronize(h->gstream);
     resolve_events(h);
+    invalidate_graphs(h);
     for (auto e : h->event_pool) cudaEventDestroy(e);
+    for (auto e : h->sync_ev)
+        if (e) cudaEventDestroy(e);
     dfree_all(h);
     if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+    if (h->gstream) cudaStreamDestroy(h->gstream);
     (void)cudaGetLastError();
     delete h;
 }
@@ -168,6 +278,9 @@ static cualign_status alloc_state(cualign_bp *h)
         CA_CUDA(cudaMemsetAsync(*p, 0, sizeof(double) * (m ? m : 1), h->stream));
     }
     CA_TRY(bp_setup(h));
+    CA_TRY(dalloc(h, &h->p_dev, 1));
+    CA_CUDA(cudaMemsetAsync(h->p_dev, 0, sizeof(int), h->stream));
+    CA_TRY(ensure_gh(h, 1));
     if (h->flags & CUALIGN_FLAG_EXACT) {
         CA_TRY(dalloc(h, &h->texact, m));
         CA_TRY(dalloc(h, &h->Ffull, (size_t)h->s));
@@ -245,6 +358,26 @@ cualign_status cualign_bp_iterate(cualign_bp *h, int32_t n_steps)
         return CUALIGN_EINVAL;
     }
     return bp_iterate(h, n_steps);
+}
+
+cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t with_round)
+{
+    API_ENTER();
+    CHECK_H();
+    if (n_steps < 0) {
+        set_error("n_steps < 0");
+        return CUALIGN_EINVAL;
+    }
+    if (n_steps == 0) return CUALIGN_OK;
+    return run_graph(h, n_steps, with_round ? 1 : 0);
+}
+
+cualign_status cualign_bp_set_timing(cualign_bp *h, int32_t on)
+{
+    API_ENTER();
+    CHECK_H();
+    h->timing = on != 0;
+    return CUALIGN_OK;
 }
 
 cualign_status cualign_bp_round(cualign_bp *h, cualign_round_info *info)
@@ -378,6 +511,8 @@ cualign_status cualign_bp_set_state(cualign_bp *h, const double *yp, const doubl
         CA_TRY(st);
     }
     h->p = p;
+    CA_TRY(ensure_gh(h, (int64_t)p + 1));
+    CA_CUDA(cudaMemcpyAsync(h->p_dev, &h->p, sizeof(int), cudaMemcpyHostToDevice, h->stream));
     CA_TRY(bp_fsum(h));
     CA_CUDA(cudaStreamSynchronize(h->stream));
     return CUALIGN_OK;

@@ -164,7 +164,9 @@ struct EdgeArgs {
     int64_t m;
     const int32_t *La, *Lb;
     const double *w;
-    double alpha, g, hh, fp_inv;
+    double alpha, fp_inv;
+    const double2 *gh;   // gh[p] = (gamma^p, 1 - gamma^p), host-computed (reading Z2)
+    const int *p_dev;    // iterations done; this iteration is p_dev + 1
     unsigned long long *tacc;
     const double *texact;
     const double2 *Atop, *Btop;
@@ -175,6 +177,8 @@ template <int EPT, bool EXACT, bool LITERAL>
 __global__ void __launch_bounds__(256) k_edge(EdgeArgs R)
 {
     const int64_t base = (int64_t)blockIdx.x * blockDim.x * EPT + threadIdx.x;
+    const double2 ghp = R.gh[*R.p_dev + 1];
+    const double g = ghp.x, hh = ghp.y;
     int64_t e[EPT];
     int a[EPT], b[EPT];
     double we[EPT], ype[EPT], zpe[EPT], t[EPT];
@@ -206,8 +210,8 @@ __global__ void __launch_bounds__(256) k_edge(EdgeArgs R)
         const double yce = de - omc;
         const double zce = de - omr;
         const double ue = (yce + zce) - de;                // line 13 diagonal
-        R.yp[e[j]] = R.g * yce + R.hh * ype[j];            // line 14
-        R.zp[e[j]] = R.g * zce + R.hh * zpe[j];            // line 15
+        R.yp[e[j]] = g * yce + hh * ype[j];                // line 14
+        R.zp[e[j]] = g * zce + hh * zpe[j];                // line 15
         R.yc[e[j]] = yce;
         R.zc[e[j]] = zce;
         R.d[e[j]] = de;
@@ -236,7 +240,8 @@ __device__ __forceinline__ void seg_atomic_add(unsigned long long v, int key, in
 template <bool UPDATE, bool EXACT>
 __global__ void __launch_bounds__(256)
 k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_val,
-         const double *__restrict__ u, double beta, double g, double hh, double fp_scale,
+         const double *__restrict__ u, double beta, const double2 *__restrict__ gh,
+         const int *__restrict__ p_dev, double fp_scale,
          unsigned long long *__restrict__ tacc, const longlong2 *__restrict__ sq_pos,
          double *__restrict__ Ffull)
 {
@@ -245,6 +250,12 @@ k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_v
     // streamed with evict-first hints (__ldcs / __stcs) so that the per-edge u
     // and the accumulator tacc stay resident in L2.
     constexpr int SQ_U = 2;
+    double g = 0.0, hh = 1.0;
+    if (UPDATE) {
+        const double2 ghp = gh[*p_dev + 1];
+        g = ghp.x;
+        hh = ghp.y;
+    }
     const int lane = threadIdx.x & 31;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -356,13 +367,15 @@ int square_grid(cualign_bp *h)
     return grid_for(h->nsq, 256, h->num_sms * 8);
 }
 
-cualign_status launch_square(cualign_bp *h, bool update, double g, double hh)
+__global__ void k_advance(int *p_dev) { *p_dev += 1; }
+
+cualign_status launch_square(cualign_bp *h, bool update)
 {
     const bool exact = (h->flags & CUALIGN_FLAG_EXACT) != 0;
     if (h->nsq > 0) {
         KScope ks(h, CUALIGN_K_SQUARE);
         const int grid = square_grid(h);
-#define SQ_ARGS h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, g, hh, h->fp_scale, h->tacc, h->sq_pos, h->Ffull
+#define SQ_ARGS h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, h->gh_dev, h->p_dev, h->fp_scale, h->tacc, h->sq_pos, h->Ffull
         if (update && exact) k_square<true, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
         else if (update) k_square<true, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
         else if (exact) k_square<false, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
@@ -380,6 +393,32 @@ cualign_status launch_square(cualign_bp *h, bool update, double g, double hh)
 }
 
 } // namespace
+
+// gh[p] = (gamma^p, 1 - gamma^p) for p = 0..cap-1, computed on the host in
+// fp64 exactly as the oracle does (reading Z2) and read by the kernels at
+// gh[p_dev + 1], so an iteration can be replayed from a CUDA graph.
+cualign_status ensure_gh(cualign_bp *h, int64_t pmax)
+{
+    if (pmax < h->gh_cap) return CUALIGN_OK;
+    int64_t cap = h->gh_cap ? h->gh_cap : 65536;
+    while (cap <= pmax) cap *= 2;
+    std::vector<double2> tab((size_t)cap);
+    for (int64_t p = 0; p < cap; p++) {
+        const double g = pow(h->gamma, (double)p);
+        tab[(size_t)p] = make_double2(g, 1.0 - g);
+    }
+    double2 *nd = nullptr;
+    CA_TRY(dalloc(h, &nd, (size_t)cap));
+    CA_CUDA(cudaMemcpy(nd, tab.data(), sizeof(double2) * (size_t)cap, cudaMemcpyHostToDevice));
+    if (h->gh_dev) {
+        CA_CUDA(cudaStreamSynchronize(h->stream));
+        dfree(h, h->gh_dev);
+    }
+    h->gh_dev = nd;
+    h->gh_cap = cap;
+    invalidate_graphs(h); // captured kernels hold the old table pointer
+    return CUALIGN_OK;
+}
 
 cualign_status bp_setup(cualign_bp *h)
 {
@@ -417,7 +456,7 @@ cualign_status bp_fsum(cualign_bp *h)
 {
     if (!(h->flags & CUALIGN_FLAG_EXACT))
         CA_CUDA(cudaMemsetAsync(h->tacc, 0, sizeof(unsigned long long) * (size_t)(h->L.m ? h->L.m : 1), h->stream));
-    return launch_square(h, false, 0.0, 1.0);
+    return launch_square(h, false);
 }
 
 cualign_status bp_iterate(cualign_bp *h, int32_t n)
@@ -425,10 +464,9 @@ cualign_status bp_iterate(cualign_bp *h, int32_t n)
     const bool exact = (h->flags & CUALIGN_FLAG_EXACT) != 0;
     const bool literal = (h->flags & CUALIGN_FLAG_OTHERMAX_LITERAL) != 0;
     const int64_t m = h->L.m;
+    if (!h->capturing) CA_TRY(ensure_gh(h, h->p + n));
     for (int32_t k = 0; k < n; k++) {
         const int32_t p = h->p + 1;
-        const double g = pow(h->gamma, (double)p); // reading Z2: host fp64 gamma^p
-        const double hh = 1.0 - g;
         if (m > 0) {
             {
                 KScope ks(h, CUALIGN_K_TOP2);
@@ -439,7 +477,7 @@ cualign_status bp_iterate(cualign_bp *h, int32_t n)
             }
             {
                 KScope ks(h, CUALIGN_K_EDGE);
-                EdgeArgs R{m, h->L.La, h->L.Lb, h->L.w, h->alpha, g, hh, h->fp_inv, h->tacc, h->texact,
+                EdgeArgs R{m, h->L.La, h->L.Lb, h->L.w, h->alpha, h->fp_inv, h->gh_dev, h->p_dev, h->tacc, h->texact,
                            h->Atop, h->Btop, h->yp, h->zp, h->yc, h->zc, h->d, h->u};
                 constexpr int EPT = 4;
                 const int grid = grid_for((m + EPT - 1) / EPT, 256, 1 << 30);
@@ -449,7 +487,12 @@ cualign_status bp_iterate(cualign_bp *h, int32_t n)
                 else k_edge<EPT, false, false><<<grid, 256, 0, h->stream>>>(R);
                 CA_CUDA(cudaGetLastError());
             }
-            CA_TRY(launch_square(h, true, g, hh));
+            CA_TRY(launch_square(h, true));
+        }
+        {
+            KScope ks(h, CUALIGN_K_OTHER);
+            k_advance<<<1, 1, 0, h->stream>>>(h->p_dev);
+            CA_CUDA(cudaGetLastError());
         }
         h->p = p;
     }

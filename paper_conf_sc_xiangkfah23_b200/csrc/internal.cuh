@@ -104,7 +104,19 @@ struct cualign_bp {
     double2 *Bct = nullptr;             // nchunks: (max1, max2) of z^p over the chunk
     unsigned int *Bcnt = nullptr;       // nB: chunks finished (hub columns' last-arriver merge)
     double2 *Atop = nullptr, *Btop = nullptr; // per-vertex (max1, max2) of y^p / z^p
-    int32_t p = 0;
+    int32_t p = 0;                      // host mirror of the iteration count
+    int *p_dev = nullptr;               // device iteration count (kernels read p_dev + 1)
+    double2 *gh_dev = nullptr;          // gh[p] = (gamma^p, 1 - gamma^p)
+    int64_t gh_cap = 0;
+
+    // CUDA graphs of one step (iterate(1) [+ round]); [0] = no round, [1] = with round
+    cudaStream_t gstream = nullptr;     // capture / replay stream (never the legacy stream)
+    cudaEvent_t sync_ev[2] = {nullptr, nullptr};
+    bool capturing = false;
+    cudaGraphExec_t graph[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}}; // [timed][round]
+    int64_t graph_launches[2][2] = {{0, 0}, {0, 0}};                        // kernels per replay
+    int64_t graph_class_launches[2][2][CUALIGN_NUM_KERNEL_CLASSES] = {};
+    std::vector<std::pair<int, cualign::EventPair>> graph_events[2];        // timed graphs' events
 
     // matching (two instances: y and z)
     int32_t *candA = nullptr, *candB = nullptr, *mateA = nullptr, *mateB = nullptr;
@@ -160,7 +172,11 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
                              const cualign_edges *E);
 cualign_status ensure_sq_pos(cualign_bp *h);
 
+// api.cu
+void invalidate_graphs(cualign_bp *h);
+
 // bp.cu
+cualign_status ensure_gh(cualign_bp *h, int64_t pmax); // gamma^p table covers p <= pmax
 cualign_status bp_setup(cualign_bp *h);                // B chunks
 cualign_status bp_fsum(cualign_bp *h);                 // t <- sum_f F(S^p) (init / set_state)
 cualign_status bp_iterate(cualign_bp *h, int32_t n);   // Alg. 2 l.9-16, n times

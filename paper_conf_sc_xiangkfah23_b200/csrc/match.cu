@@ -46,6 +46,7 @@ struct MatchParams {
     int32_t *mateA, *mateB;
     RoundDev *rd;
     unsigned long long *work; // per instance: proposals (suitor) / rounds
+    unsigned long long *dbg;  // optional diagnostics (CUALIGN_MATCH_DEBUG)
 };
 
 __device__ __forceinline__ bool better(double xa, int ea, double xb, int eb)
@@ -86,9 +87,10 @@ __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
     const int64_t *__restrict__ rp = fromB ? P.Bptr : P.Arow;
     const int32_t *__restrict__ tgt = fromB ? P.La : P.Lb;   // target vertex of an edge
     const int32_t *__restrict__ own = fromB ? P.Lb : P.La;   // proposer vertex of an edge
-    unsigned long long proposals = 0;
+    unsigned long long proposals = 0, scans = 0;
     constexpr int U = 3; // edges per lane per pass: loads of a pass are issued together
     while (true) {
+        scans++;
         // heaviest eligible neighbour of `cur` whose suitor is lighter
         int best = -1;
         double bx = 0.0;
@@ -158,6 +160,13 @@ __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
         if (code == 2) cur = tile.shfl(next, 0);
     }
     if (lane == 0 && proposals) atomicAdd(P.work + k, proposals);
+    if (P.dbg && lane == 0) {
+        atomicMax(P.dbg + 0, scans);
+        atomicAdd(P.dbg + 1, scans);
+        if (scans > 8) atomicAdd(P.dbg + 2, 1ull);
+        if (scans > 64) atomicAdd(P.dbg + 3, 1ull);
+        atomicMax(P.dbg + 4, proposals);
+    }
 }
 
 // ---------------------------------------------------------- pointer rounds
@@ -373,7 +382,7 @@ __global__ void __launch_bounds__(256) k_eval(EvalParams P)
 
 // one block: finish the sums, score, select, best (Alg. 2 l.21-24)
 __global__ void __launch_bounds__(256)
-k_round_final(EvalParams P, int nblocks, int exact, double alpha, double beta, int32_t p,
+k_round_final(EvalParams P, int nblocks, int exact, double alpha, double beta, const int *p_dev,
               const unsigned long long *work)
 {
     __shared__ double sd[32];
@@ -399,6 +408,7 @@ k_round_final(EvalParams P, int nblocks, int exact, double alpha, double beta, i
     RoundDev *rd = P.rd;
     cualign_round_info &I = rd->info;
     const long long ov0 = (long long)rd->overlap[0], ov1 = (long long)rd->overlap[1];
+    const int32_t p = *p_dev;
     I.iter = p;
     I.weight_y = wk[0];
     I.weight_z = wk[1];
@@ -482,9 +492,17 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) {
         {
             KScope ks(h, CUALIGN_K_MATCH);
-            void *args[] = {&P};
-            CA_CUDA(cudaLaunchCooperativeKernel((void *)k_pointer_rounds, dim3(h->match_grid), dim3(256), args, 0,
-                                                h->stream));
+            // cooperative launch through cudaLaunchKernelEx: capturable into a graph
+            cudaLaunchConfig_t cfg{};
+            cfg.gridDim = dim3(h->match_grid);
+            cfg.blockDim = dim3(256);
+            cfg.stream = h->stream;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeCooperative;
+            attr[0].val.cooperative = 1;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            CA_CUDA(cudaLaunchKernelEx(&cfg, k_pointer_rounds, P));
         }
         KScope ks(h, CUALIGN_K_MATCH);
         k_mark<<<grid_for(P.ninst * nA, 256, h->num_sms * 8), 256, 0, h->stream>>>(nA, P.ninst, P.mateA, h->mflag, m);
@@ -499,12 +517,33 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     CA_CUDA(cudaMemsetAsync(fromB ? h->mateB : h->mateA, 0xff, sizeof(int32_t) * (size_t)(2 * nP + 1),
                             h->stream));
     const int64_t slots = P.ninst * nP;
+    static const bool dbg_env = getenv("CUALIGN_MATCH_DEBUG") != nullptr;
+    const bool dbg = dbg_env && !h->capturing;
+    unsigned long long *dbuf = nullptr;
+    if (dbg) {
+        CA_CUDA(cudaMalloc(&dbuf, 8 * sizeof(unsigned long long)));
+        CA_CUDA(cudaMemsetAsync(dbuf, 0, 8 * sizeof(unsigned long long), h->stream));
+        P.dbg = dbuf;
+    }
     if (slots > 0) {
         KScope ks(h, CUALIGN_K_MATCH);
         const int64_t dmax = fromB ? h->max_deg_b : h->max_deg_a;
-        if (dmax > 64) k_suitor<32><<<grid_for(slots * 32, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        static const int genv = getenv("CUALIGN_SUITOR_G") ? atoi(getenv("CUALIGN_SUITOR_G")) : 0;
+        const int G = genv ? genv : (dmax > 64 ? 32 : 8);
+        if (G == 32) k_suitor<32><<<grid_for(slots * 32, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else if (G == 16) k_suitor<16><<<grid_for(slots * 16, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else if (G == 4) k_suitor<4><<<grid_for(slots * 4, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else if (G == 1) k_suitor<1><<<grid_for(slots, 128, 1 << 30), 128, 0, h->stream>>>(P);
         else k_suitor<8><<<grid_for(slots * 8, 128, 1 << 30), 128, 0, h->stream>>>(P);
         CA_CUDA(cudaGetLastError());
+    }
+    if (dbg) {
+        unsigned long long d[8];
+        CA_CUDA(cudaMemcpyAsync(d, dbuf, sizeof(d), cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaStreamSynchronize(h->stream));
+        fprintf(stderr, "[suitor] tiles=%lld max_scans=%llu total_scans=%llu tiles>8=%llu tiles>64=%llu max_props=%llu\n",
+                (long long)slots, d[0], d[1], d[2], d[3], d[4]);
+        cudaFree(dbuf);
     }
     if (P.ninst * nT > 0) {
         KScope ks(h, CUALIGN_K_MATCH);
@@ -586,7 +625,7 @@ cualign_status match_round(cualign_bp *h)
     {
         KScope ks(h, CUALIGN_K_MATCH);
         k_round_final<<<1, 256, 0, h->stream>>>(E, h->eval_grid, (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha,
-                                                h->beta, h->p, h->match_work);
+                                                h->beta, h->p_dev, h->match_work);
         CA_CUDA(cudaGetLastError());
     }
     {

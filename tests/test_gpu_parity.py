@@ -317,6 +317,48 @@ def test_end_to_end_align_fast_mode(ca):
         assert min(gaps) < 1e-9 * max(1.0, abs(obest))
 
 
+@pytest.mark.parametrize("flags_name", ["fast", "exact", "rounds"])
+def test_graph_run_equals_step_by_step(ca, flags_name):
+    """cualign_bp_run (CUDA-graph replay of iterate+round) gives bit-identical
+    state, round infos and best matching to the eager call sequence."""
+    inst = INSTANCES["P10"]()
+    flags = {"fast": 0, "exact": ca.FLAG_EXACT, "rounds": ca.FLAG_MATCH_ROUNDS}[flags_name]
+    n = 12
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, flags=flags) as h1, \
+            ca.CuAlignBP(inst.A, inst.B, inst.L, flags=flags) as h2:
+        for _ in range(n):
+            h1.iterate(1)
+            h1.round(sync=False)
+        h2.run(5)
+        h2.set_timing(True)
+        h2.run(4)               # timed graph variant
+        h2.set_timing(False)
+        h2.run(n - 9)
+        s1, s2 = h1.get_state(), h2.get_state()
+        assert_state_equal(s2, s1)
+        assert s1["p"] == s2["p"] == n
+        m1, i1 = h1.get_best()
+        m2, i2 = h2.get_best()
+        assert np.array_equal(m1, m2)
+        for k in ("iter", "best_score", "best_iter", "score_y", "score_z", "overlap_y", "card_z"):
+            assert i1[k] == i2[k], k
+        st = h2.stats()
+        assert st["class_ms"]["square"] > 0 and st["class_launches"]["square"] >= n
+
+
+def test_graph_run_matches_oracle_exact(ca):
+    inst = make_config("T")
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    oinfos = o.align(inst.n_iter, inst.gamma)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, ca.FLAG_EXACT) as h:
+        h.run(inst.n_iter)
+        mate, info = h.get_best()
+        assert_state_equal(h.get_state(), o.get_state())
+    omate, obest, oit = o.get_best()
+    assert np.array_equal(mate, omate) and info["best_score"] == obest and info["best_iter"] == oit
+    assert info["iter"] == inst.n_iter and info["score"] == oinfos[-1]["score"]
+
+
 # ------------------------------------------------------------ golden W1/W2
 def test_W1_on_gpu(ca):
     from fractions import Fraction
