@@ -245,7 +245,11 @@ def main():
     t_gen = time.perf_counter() - t_gen
     log(f"[rank {rank}] generated {args.config} (scale {args.scale}) in {t_gen:.1f}s: "
         f"n_A={inst.A.n} n_B={inst.B.n} m={inst.L.m}")
-    stream = torch.cuda.current_stream()
+    # a dedicated stream: the library launches on it and the timing events are
+    # recorded on it (torch's default stream is the legacy stream, which does
+    # not order against the library's non-blocking streams)
+    stream = torch.cuda.Stream(device=dev)
+    torch.cuda.set_stream(stream)
     flags = (ca.FLAG_EXACT if args.exact else 0) | (ca.FLAG_MATCH_ROUNDS if args.match_rounds else 0)
 
     # ---------------------------------------------------------------- init

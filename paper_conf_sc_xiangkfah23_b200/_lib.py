@@ -178,9 +178,10 @@ def _prep(x, np_dtype, torch_dtype_name):
 def _stream_ptr(stream):
     if stream is None:
         return None
-    if isinstance(stream, int):
-        return ctypes.c_void_p(stream)
-    return ctypes.c_void_p(stream.cuda_stream)  # torch.cuda.Stream
+    handle = stream if isinstance(stream, int) else stream.cuda_stream  # torch.cuda.Stream
+    # handle 0 is the legacy default stream: pass cudaStreamLegacy (0x1) so the
+    # library runs on it instead of creating a private stream
+    return ctypes.c_void_p(handle if handle else 1)
 
 
 class CuAlignBP:
