@@ -237,7 +237,7 @@ __device__ __forceinline__ void seg_atomic_add(unsigned long long v, int key, in
 
 // UPDATE = apply lines 9, 13, 16 to the pair; otherwise only (re)compute the
 // F row sums of the current S^p (init, set_state).
-template <bool UPDATE, bool EXACT>
+template <bool UPDATE, bool EXACT, int SQ_U = 2, bool HINTS = true>
 __global__ void __launch_bounds__(256)
 k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_val,
          const double *__restrict__ u, double beta, const double2 *__restrict__ gh,
@@ -249,7 +249,7 @@ k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_v
     // issued before any use (memory-level parallelism); the square arrays are
     // streamed with evict-first hints (__ldcs / __stcs) so that the per-edge u
     // and the accumulator tacc stay resident in L2.
-    constexpr int SQ_U = 2;
+    // SQ_U, HINTS: template parameters (variants measured in profiles/)
     double g = 0.0, hh = 1.0;
     if (UPDATE) {
         const double2 ghp = gh[*p_dev + 1];
@@ -267,8 +267,8 @@ k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_v
         for (int j = 0; j < SQ_U; j++) {
             const int64_t q = base + j * 32 + lane;
             if (q < nsq) {
-                ef[j] = __ldcs(sq_ef + q);
-                v[j] = __ldcs(sq_val + q); // (S^p_ef, S^p_fe)
+                ef[j] = (HINTS ? __ldcs(sq_ef + q) : sq_ef[q]);
+                v[j] = (HINTS ? __ldcs(sq_val + q) : sq_val[q]); // (S^p_ef, S^p_fe)
             }
         }
         if (UPDATE) {
@@ -294,7 +294,7 @@ k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_v
                     const double Scfe = uf[j] - Ffe;
                     v[j].x = g * Scef + hh * v[j].x;                       // line 16
                     v[j].y = g * Scfe + hh * v[j].y;
-                    __stcs(sq_val + q, v[j]);
+                    if (HINTS) __stcs(sq_val + q, v[j]); else sq_val[q] = v[j];
                 }
                 // F of the next iteration (line 9 at p+1) from the new pair
                 const double Nef = clamp_beta(beta + v[j].y, beta);
@@ -377,7 +377,14 @@ cualign_status launch_square(cualign_bp *h, bool update)
         const int grid = square_grid(h);
 #define SQ_ARGS h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, h->gh_dev, h->p_dev, h->fp_scale, h->tacc, h->sq_pos, h->Ffull
         if (update && exact) k_square<true, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
-        else if (update) k_square<true, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+        else if (update) {
+            static const int var = getenv("CUALIGN_SQ_VARIANT") ? atoi(getenv("CUALIGN_SQ_VARIANT")) : 3;
+            if (var == 0) k_square<true, false, 1, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+            else if (var == 1) k_square<true, false, 1, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+            else if (var == 2) k_square<true, false, 2, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+            else if (var == 4) k_square<true, false, 4, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+            else k_square<true, false, 2, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+        }
         else if (exact) k_square<false, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
         else k_square<false, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
 #undef SQ_ARGS

@@ -70,16 +70,36 @@ __device__ __forceinline__ const double *xk(const MatchParams &P, int k) { retur
 // One G-lane tile per proposer: the lanes scan the proposer's list together
 // (G edges per step, independent loads), a tile argmax picks the heaviest
 // eligible target, lane 0 attempts the CAS and the outcome is broadcast.
+constexpr int WORK_SPREAD = 64, WORK_STRIDE = 16; // counter slots, 128 B apart
+
+template <int G, class Tile>
+__device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
+                                            int64_t nT, int64_t slot, unsigned long long *s_props);
+
 template <int G>
 __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
 {
+    __shared__ unsigned long long s_props[2];
+    if (threadIdx.x < 2) s_props[threadIdx.x] = 0;
+    __syncthreads();
     auto tile = cg::tiled_partition<G>(cg::this_thread_block());
     const int lane = tile.thread_rank();
     const bool fromB = P.propose_from_b != 0;
     const int64_t nP = fromB ? P.nB : P.nA;
     const int64_t nT = fromB ? P.nA : P.nB;
     const int64_t slot = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
-    if (slot >= P.ninst * nP) return; // tile-uniform
+    if (slot < P.ninst * nP) suitor_tile<G>(P, tile, lane, fromB, nP, nT, slot, s_props);
+    // the proposal counters: block-aggregated, spread over WORK_SPREAD slots
+    // (a single global address would serialise ~10^5 atomics in one L2 slice)
+    __syncthreads();
+    if (threadIdx.x < 2 && s_props[threadIdx.x])
+        atomicAdd(P.work + (blockIdx.x % WORK_SPREAD) * WORK_STRIDE + threadIdx.x, s_props[threadIdx.x]);
+}
+
+template <int G, class Tile>
+__device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
+                                            int64_t nT, int64_t slot, unsigned long long *s_props)
+{
     const int k = (int)(slot / nP);
     int cur = (int)(slot - k * nP);
     const double *__restrict__ x = xk(P, k);
@@ -159,7 +179,7 @@ __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
         if (code == 1) break;
         if (code == 2) cur = tile.shfl(next, 0);
     }
-    if (lane == 0 && proposals) atomicAdd(P.work + k, proposals);
+    if (lane == 0 && proposals) atomicAdd_block(s_props + k, proposals);
     if (P.dbg && lane == 0) {
         atomicMax(P.dbg + 0, scans);
         atomicAdd(P.dbg + 1, scans);
@@ -418,8 +438,13 @@ k_round_final(EvalParams P, int nblocks, int exact, double alpha, double beta, c
     I.card_z = (int32_t)rd->card[1];
     I.score_y = alpha * wk[0] + beta * (double)ov0;
     I.score_z = alpha * wk[1] + beta * (double)ov1;
-    I.rounds_y = (int32_t)work[0];
-    I.rounds_z = (int32_t)work[1];
+    unsigned long long w0 = 0, w1 = 0;
+    for (int i = 0; i < WORK_SPREAD; i++) {
+        w0 += work[i * WORK_STRIDE];
+        w1 += work[i * WORK_STRIDE + 1];
+    }
+    I.rounds_y = (int32_t)w0;
+    I.rounds_z = (int32_t)w1;
     const int src = (I.score_y >= I.score_z) ? 0 : 1;
     I.source = src;
     I.score = src ? I.score_z : I.score_y;
@@ -487,7 +512,7 @@ MatchParams base_params(cualign_bp *h)
 cualign_status run_matching(cualign_bp *h, MatchParams &P)
 {
     const int64_t nA = h->L.nA, nB = h->L.nB, m = h->L.m;
-    CA_CUDA(cudaMemsetAsync(h->match_work, 0, 2 * sizeof(unsigned long long), h->stream));
+    CA_CUDA(cudaMemsetAsync(h->match_work, 0, WORK_SPREAD * WORK_STRIDE * sizeof(unsigned long long), h->stream));
     CA_CUDA(cudaMemsetAsync(h->mflag, 0, (size_t)(2 * m + 1), h->stream));
     if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) {
         {
@@ -566,7 +591,7 @@ cualign_status match_setup(cualign_bp *h)
     CA_TRY(dalloc(h, &h->mateB, 2 * nB + 1));
     CA_TRY(dalloc(h, &h->best_mate, nA + 1));
     CA_TRY(dalloc(h, &h->rd, 1));
-    CA_TRY(dalloc(h, &h->match_work, 2));
+    CA_TRY(dalloc(h, &h->match_work, WORK_SPREAD * WORK_STRIDE));
     CA_TRY(dalloc(h, &h->mflag, (size_t)(2 * h->L.m + 1)));
     CA_CUDA(cudaMemsetAsync(h->rd, 0, sizeof(RoundDev), h->stream));
     CA_CUDA(cudaMemsetAsync(h->mateA, 0xff, sizeof(int32_t) * (2 * nA + 1), h->stream));
@@ -645,10 +670,13 @@ cualign_status match_standalone(cualign_bp *h, const double *x_dev, int32_t *rou
     P.x1 = x_dev;
     CA_TRY(run_matching(h, P));
     if (rounds) {
-        unsigned long long w[2] = {0, 0};
-        CA_CUDA(cudaMemcpyAsync(w, h->match_work, sizeof(w), cudaMemcpyDeviceToHost, h->stream));
+        std::vector<unsigned long long> w(WORK_SPREAD * WORK_STRIDE);
+        CA_CUDA(cudaMemcpyAsync(w.data(), h->match_work, sizeof(unsigned long long) * w.size(),
+                                cudaMemcpyDeviceToHost, h->stream));
         CA_CUDA(cudaStreamSynchronize(h->stream));
-        *rounds = (int32_t)w[0];
+        unsigned long long s = 0;
+        for (int i = 0; i < WORK_SPREAD; i++) s += w[(size_t)i * WORK_STRIDE];
+        *rounds = (int32_t)s;
     }
     return CUALIGN_OK;
 }
