@@ -237,7 +237,7 @@ __device__ __forceinline__ void seg_atomic_add(unsigned long long v, int key, in
 
 // UPDATE = apply lines 9, 13, 16 to the pair; otherwise only (re)compute the
 // F row sums of the current S^p (init, set_state).
-template <bool UPDATE, bool EXACT, int SQ_U = 2, bool HINTS = true>
+template <bool UPDATE, bool EXACT, int SQ_U = 2, bool HINTS = true, bool NOATOM = false>
 __global__ void __launch_bounds__(256)
 k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_val,
          const double *__restrict__ u, double beta, const double2 *__restrict__ gh,
@@ -305,12 +305,12 @@ k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_v
                     Ffull[pos.y] = Nfe;
                 } else {
                     const unsigned long long Tfe = __double2ull_rn(Nfe * fp_scale);
-                    if (Tfe) atomicAdd(tacc + ef[j].y, Tfe);
+                    if (Tfe && !NOATOM) atomicAdd(tacc + ef[j].y, Tfe);
                     Tef = __double2ull_rn(Nef * fp_scale);
                     key = ef[j].x;
                 }
             }
-            if (!EXACT) seg_atomic_add(Tef, key, lane, tacc);
+            if (!EXACT && !NOATOM) seg_atomic_add(Tef, key, lane, tacc);
         }
     }
 }
@@ -361,33 +361,43 @@ __global__ void k_chunk_fill(int64_t nB, const int64_t *__restrict__ Bcp, int32_
         for (int64_t c = Bcp[b]; c < Bcp[b + 1]; c++) chunk_b[c] = (int32_t)b;
 }
 
-int square_grid(cualign_bp *h)
+// Grid-stride kernels run as exactly one wave: (resident CTAs per SM) x SMs,
+// capped by the work (a 1.6-wave grid left 40% of the SMs idle in the tail).
+int one_wave_grid(cualign_bp *h, const void *fn, int block, int64_t items, int64_t items_per_block)
 {
-    // persistent-style grid: 8 resident 256-thread CTAs per SM
-    return grid_for(h->nsq, 256, h->num_sms * 8);
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, block, 0) != cudaSuccess || occ < 1) occ = 1;
+    (void)cudaGetLastError();
+    return grid_for((items + items_per_block - 1) / items_per_block, 1, occ * h->num_sms);
 }
 
 __global__ void k_advance(int *p_dev) { *p_dev += 1; }
+
+template <bool UPDATE, bool EXACT, int SQ_U, bool HINTS, bool NOATOM = false>
+void square_launch(cualign_bp *h)
+{
+    auto fn = k_square<UPDATE, EXACT, SQ_U, HINTS, NOATOM>;
+    const int grid = one_wave_grid(h, (const void *)fn, 256, h->nsq, 256 * SQ_U);
+    fn<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, h->gh_dev, h->p_dev, h->fp_scale,
+                                    h->tacc, h->sq_pos, h->Ffull);
+}
 
 cualign_status launch_square(cualign_bp *h, bool update)
 {
     const bool exact = (h->flags & CUALIGN_FLAG_EXACT) != 0;
     if (h->nsq > 0) {
         KScope ks(h, CUALIGN_K_SQUARE);
-        const int grid = square_grid(h);
-#define SQ_ARGS h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, h->gh_dev, h->p_dev, h->fp_scale, h->tacc, h->sq_pos, h->Ffull
-        if (update && exact) k_square<true, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
+        if (update && exact) square_launch<true, true, 2, true>(h);
         else if (update) {
             static const int var = getenv("CUALIGN_SQ_VARIANT") ? atoi(getenv("CUALIGN_SQ_VARIANT")) : 3;
-            if (var == 0) k_square<true, false, 1, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
-            else if (var == 1) k_square<true, false, 1, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
-            else if (var == 2) k_square<true, false, 2, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
-            else if (var == 4) k_square<true, false, 4, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
-            else k_square<true, false, 2, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
-        }
-        else if (exact) k_square<false, true><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
-        else k_square<false, false><<<grid, 256, 0, h->stream>>>(SQ_ARGS);
-#undef SQ_ARGS
+            if (var == 0) square_launch<true, false, 1, false>(h);
+            else if (var == 1) square_launch<true, false, 1, true>(h);
+            else if (var == 2) square_launch<true, false, 2, false>(h);
+            else if (var == 4) square_launch<true, false, 4, false>(h);
+            else if (var == 5) square_launch<true, false, 2, true, true>(h); // timing probe only: no F sums
+            else square_launch<true, false, 2, true>(h);
+        } else if (exact) square_launch<false, true, 2, true>(h);
+        else square_launch<false, false, 2, true>(h);
         CA_CUDA(cudaGetLastError());
     }
     if (exact) {
