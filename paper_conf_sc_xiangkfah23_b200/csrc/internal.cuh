@@ -59,7 +59,7 @@ struct RoundDev {
     int best_iter;
     int improved;
     int source;
-    int pad;
+    unsigned int done;            // k_eval blocks finished (last-block final reduction)
     cualign_round_info info;
 };
 

@@ -72,33 +72,25 @@ __device__ __forceinline__ const double *xk(const MatchParams &P, int k) { retur
 // eligible target, lane 0 attempts the CAS and the outcome is broadcast.
 constexpr int WORK_SPREAD = 64, WORK_STRIDE = 16; // counter slots, 128 B apart
 
-template <int G, class Tile>
+template <int G, int U, class Tile>
 __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
-                                            int64_t nT, int64_t slot, unsigned long long *s_props);
+                                            int64_t nT, int64_t slot);
 
-template <int G>
+template <int G, int U>
 __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
 {
-    __shared__ unsigned long long s_props[2];
-    if (threadIdx.x < 2) s_props[threadIdx.x] = 0;
-    __syncthreads();
     auto tile = cg::tiled_partition<G>(cg::this_thread_block());
     const int lane = tile.thread_rank();
     const bool fromB = P.propose_from_b != 0;
     const int64_t nP = fromB ? P.nB : P.nA;
     const int64_t nT = fromB ? P.nA : P.nB;
     const int64_t slot = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
-    if (slot < P.ninst * nP) suitor_tile<G>(P, tile, lane, fromB, nP, nT, slot, s_props);
-    // the proposal counters: block-aggregated, spread over WORK_SPREAD slots
-    // (a single global address would serialise ~10^5 atomics in one L2 slice)
-    __syncthreads();
-    if (threadIdx.x < 2 && s_props[threadIdx.x])
-        atomicAdd(P.work + (blockIdx.x % WORK_SPREAD) * WORK_STRIDE + threadIdx.x, s_props[threadIdx.x]);
+    if (slot < P.ninst * nP) suitor_tile<G, U>(P, tile, lane, fromB, nP, nT, slot);
 }
 
-template <int G, class Tile>
+template <int G, int U, class Tile>
 __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
-                                            int64_t nT, int64_t slot, unsigned long long *s_props)
+                                            int64_t nT, int64_t slot)
 {
     const int k = (int)(slot / nP);
     int cur = (int)(slot - k * nP);
@@ -108,22 +100,23 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
     const int32_t *__restrict__ tgt = fromB ? P.La : P.Lb;   // target vertex of an edge
     const int32_t *__restrict__ own = fromB ? P.Lb : P.La;   // proposer vertex of an edge
     unsigned long long proposals = 0, scans = 0;
-    constexpr int U = 3; // edges per lane per pass: loads of a pass are issued together
+    // U edges per lane per pass: the loads of a pass are issued together;
+    // positions in L's arrays are < m < 2^31, so 32-bit index math
     while (true) {
         scans++;
         // heaviest eligible neighbour of `cur` whose suitor is lighter
         int best = -1;
         double bx = 0.0;
-        const int64_t hi = rp[cur + 1];
-        for (int64_t j0 = rp[cur] + lane; j0 < hi; j0 += G * U) {
+        const int hi = (int)rp[cur + 1];
+        for (int j0 = (int)rp[cur] + lane; j0 < hi; j0 += G * U) {
             int ee[U], tt[U], ss[U];
             double xx[U], xs[U];
 #pragma unroll
             for (int u = 0; u < U; u++) {
-                const int64_t j = j0 + u * G;
+                const int j = j0 + u * G;
                 ee[u] = -1;
                 if (j < hi) {
-                    const int e = fromB ? __ldg(P.Bedge + j) : (int)j;
+                    const int e = fromB ? __ldg(P.Bedge + j) : j;
                     xx[u] = __ldg(x + e);
                     tt[u] = __ldg(tgt + e);
                     ee[u] = (xx[u] > 0.0) ? e : -1; // only x > 0 is eligible (Z6)
@@ -179,7 +172,9 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
         if (code == 1) break;
         if (code == 2) cur = tile.shfl(next, 0);
     }
-    if (lane == 0 && proposals) atomicAdd_block(s_props + k, proposals);
+    // proposal counters spread over WORK_SPREAD slots (one global address
+    // would serialise ~10^5 atomics in one L2 slice)
+    if (lane == 0 && proposals) atomicAdd(P.work + (slot % WORK_SPREAD) * WORK_STRIDE + k, proposals);
     if (P.dbg && lane == 0) {
         atomicMax(P.dbg + 0, scans);
         atomicAdd(P.dbg + 1, scans);
@@ -363,49 +358,11 @@ struct EvalParams {
     RoundDev *rd;
 };
 
-// weight partial sums per block (fixed partition: deterministic), overlap and
-// cardinality as integer atomics (exact).  One warp per A vertex: the lanes
-// stride over the matched edge's square row (rows reach thousands of squares).
-__global__ void __launch_bounds__(256) k_eval(EvalParams P)
+// One block (the last one of k_eval to finish): finish the sums, score, select,
+// best (Alg. 2 l.21-24).
+__device__ void round_final_block(const EvalParams &P, int nblocks, int exact, double alpha, double beta,
+                                  const int *p_dev, const unsigned long long *work, double *sd)
 {
-    __shared__ double sd[32];
-    __shared__ unsigned long long su[32];
-    constexpr int G = 8;
-    const int lane = threadIdx.x & (G - 1);
-    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) / G;
-    for (int k = 0; k < 2; k++) {
-        const int32_t *mA = P.mateA + (int64_t)k * P.nA;
-        double wsum = 0.0;
-        unsigned long long ov = 0, card = 0;
-        for (int64_t a = warp; a < P.nA; a += nwarps) {
-            const int e = mA[a];
-            if (e < 0) continue;
-            if (lane == 0) {
-                wsum += P.w[e];
-                card++;
-            }
-            const int64_t hi = P.sq_rp[e + 1];
-            for (int64_t q = P.sq_rp[e] + lane; q < hi; q += G) {
-                const int f = P.sq_ef[q].y;
-                if (P.mflag[k * P.m + f]) ov++;
-            }
-        }
-        const double bw = block_sum<double>(wsum, sd);
-        if (threadIdx.x == 0) P.partial_w[k * gridDim.x + blockIdx.x] = bw;
-        const unsigned long long bo = block_sum<unsigned long long>(ov, su);
-        if (threadIdx.x == 0 && bo) atomicAdd(&P.rd->overlap[k], bo);
-        const unsigned long long bc = block_sum<unsigned long long>(card, su);
-        if (threadIdx.x == 0 && bc) atomicAdd(&P.rd->card[k], bc);
-    }
-}
-
-// one block: finish the sums, score, select, best (Alg. 2 l.21-24)
-__global__ void __launch_bounds__(256)
-k_round_final(EvalParams P, int nblocks, int exact, double alpha, double beta, const int *p_dev,
-              const unsigned long long *work)
-{
-    __shared__ double sd[32];
     double wk[2] = {0.0, 0.0};
     for (int k = 0; k < 2; k++) {
         if (exact) {
@@ -419,7 +376,7 @@ k_round_final(EvalParams P, int nblocks, int exact, double alpha, double beta, c
             }
         } else {
             double s = 0.0;
-            for (int i = threadIdx.x; i < nblocks; i += blockDim.x) s += P.partial_w[k * nblocks + i];
+            for (int i = threadIdx.x; i < nblocks; i += blockDim.x) s += __ldcg(P.partial_w + k * nblocks + i);
             s = block_sum<double>(s, sd);
             if (threadIdx.x == 0) wk[k] = s;
         }
@@ -427,15 +384,16 @@ k_round_final(EvalParams P, int nblocks, int exact, double alpha, double beta, c
     if (threadIdx.x != 0) return;
     RoundDev *rd = P.rd;
     cualign_round_info &I = rd->info;
-    const long long ov0 = (long long)rd->overlap[0], ov1 = (long long)rd->overlap[1];
+    const long long ov0 = (long long)*(volatile unsigned long long *)&rd->overlap[0];
+    const long long ov1 = (long long)*(volatile unsigned long long *)&rd->overlap[1];
     const int32_t p = *p_dev;
     I.iter = p;
     I.weight_y = wk[0];
     I.weight_z = wk[1];
     I.overlap_y = ov0;
     I.overlap_z = ov1;
-    I.card_y = (int32_t)rd->card[0];
-    I.card_z = (int32_t)rd->card[1];
+    I.card_y = (int32_t)*(volatile unsigned long long *)&rd->card[0];
+    I.card_z = (int32_t)*(volatile unsigned long long *)&rd->card[1];
     I.score_y = alpha * wk[0] + beta * (double)ov0;
     I.score_z = alpha * wk[1] + beta * (double)ov1;
     unsigned long long w0 = 0, w1 = 0;
@@ -458,6 +416,57 @@ k_round_final(EvalParams P, int nblocks, int exact, double alpha, double beta, c
     I.best_iter = rd->best_iter;
     rd->improved = I.improved;
     rd->source = src;
+}
+
+// Evaluate both matchings: weight partial sums per block (fixed partition:
+// deterministic), overlap and cardinality as integer atomics (exact).  A
+// 4-lane tile per A vertex handles M_y and M_z; the lanes stride over the
+// matched edge's square row (rows reach thousands of squares).  The last block
+// to finish runs the final reduction (no separate launch).
+__global__ void __launch_bounds__(256)
+k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, const unsigned long long *work)
+{
+    __shared__ double sd[32];
+    __shared__ unsigned long long su[32];
+    __shared__ bool last;
+    constexpr int G = 4;
+    const int lane = threadIdx.x & (G - 1);
+    const int64_t t0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
+    const int64_t nt = ((int64_t)gridDim.x * blockDim.x) / G;
+    double wsum[2] = {0.0, 0.0};
+    unsigned long long ov[2] = {0, 0}, card[2] = {0, 0};
+    for (int64_t a = t0; a < P.nA; a += nt) {
+        const int es[2] = {P.mateA[a], P.mateA[P.nA + a]};
+#pragma unroll
+        for (int k = 0; k < 2; k++) {
+            const int e = es[k];
+            if (e < 0) continue;
+            if (lane == 0) {
+                wsum[k] += P.w[e];
+                card[k]++;
+            }
+            const int64_t hi = P.sq_rp[e + 1];
+            for (int64_t q = P.sq_rp[e] + lane; q < hi; q += G)
+                if (P.mflag[k * P.m + P.sq_ef[q].y]) ov[k]++;
+        }
+    }
+    for (int k = 0; k < 2; k++) {
+        const double bw = block_sum<double>(wsum[k], sd);
+        if (threadIdx.x == 0) P.partial_w[k * gridDim.x + blockIdx.x] = bw;
+        const unsigned long long bo = block_sum<unsigned long long>(ov[k], su);
+        if (threadIdx.x == 0 && bo) atomicAdd(&P.rd->overlap[k], bo);
+        const unsigned long long bc = block_sum<unsigned long long>(card[k], su);
+        if (threadIdx.x == 0 && bc) atomicAdd(&P.rd->card[k], bc);
+    }
+    if (threadIdx.x == 0) {
+        __threadfence();
+        last = atomicAdd(&P.rd->done, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    round_final_block(P, gridDim.x, exact, alpha, beta, p_dev, work, sd);
+    if (threadIdx.x == 0) P.rd->done = 0u;
 }
 
 __global__ void k_copy_best(int64_t nA, const int32_t *__restrict__ mateA, const RoundDev *__restrict__ rd,
@@ -554,12 +563,14 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
         KScope ks(h, CUALIGN_K_MATCH);
         const int64_t dmax = fromB ? h->max_deg_b : h->max_deg_a;
         static const int genv = getenv("CUALIGN_SUITOR_G") ? atoi(getenv("CUALIGN_SUITOR_G")) : 0;
-        const int G = genv ? genv : (dmax > 64 ? 32 : 8);
-        if (G == 32) k_suitor<32><<<grid_for(slots * 32, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else if (G == 16) k_suitor<16><<<grid_for(slots * 16, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else if (G == 4) k_suitor<4><<<grid_for(slots * 4, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else if (G == 1) k_suitor<1><<<grid_for(slots, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else k_suitor<8><<<grid_for(slots * 8, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        // tile width: G lanes x U edges cover a typical proposer list in one pass
+        const int G = genv ? genv : (dmax > 64 ? 32 : (dmax > 24 ? 16 : (dmax > 20 ? 8 : 4)));
+        if (G == 32) k_suitor<32, 2><<<grid_for(slots * 32, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else if (G == 16) k_suitor<16, 2><<<grid_for(slots * 16, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else if (G == 4) k_suitor<4, 5><<<grid_for(slots * 4, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else if (G == 2) k_suitor<2, 9><<<grid_for(slots * 2, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else if (G == 1) k_suitor<1, 8><<<grid_for(slots, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else k_suitor<8, 3><<<grid_for(slots * 8, 128, 1 << 30), 128, 0, h->stream>>>(P);
         CA_CUDA(cudaGetLastError());
     }
     if (dbg) {
@@ -616,7 +627,7 @@ cualign_status match_setup(cualign_bp *h)
     int64_t want = ((int64_t)2 * (nA + nB) + 255) / 256;
     int64_t cap = (int64_t)occ * h->num_sms;
     h->match_grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
-    h->eval_grid = grid_for((int64_t)nA * 8, 256, h->num_sms * 8);
+    h->eval_grid = grid_for((int64_t)nA * 4, 256, h->num_sms * 8);
     CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * h->eval_grid));
     return CUALIGN_OK;
 }
@@ -644,13 +655,8 @@ cualign_status match_round(cualign_bp *h)
     CA_CUDA(cudaMemsetAsync(&h->rd->overlap[0], 0, 4 * sizeof(unsigned long long), h->stream));
     {
         KScope ks(h, CUALIGN_K_MATCH);
-        k_eval<<<h->eval_grid, 256, 0, h->stream>>>(E);
-        CA_CUDA(cudaGetLastError());
-    }
-    {
-        KScope ks(h, CUALIGN_K_MATCH);
-        k_round_final<<<1, 256, 0, h->stream>>>(E, h->eval_grid, (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha,
-                                                h->beta, h->p_dev, h->match_work);
+        k_eval<<<h->eval_grid, 256, 0, h->stream>>>(E, (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha, h->beta,
+                                                    h->p_dev, h->match_work);
         CA_CUDA(cudaGetLastError());
     }
     {
