@@ -131,7 +131,7 @@ typedef struct {
 
 /* Diagnostics: per-kernel-class event timing (needs CUALIGN_FLAG_TIMING) and
  * launch counts since the last reset. */
-#define CUALIGN_NUM_KERNEL_CLASSES 8
+#define CUALIGN_NUM_KERNEL_CLASSES 10
 typedef struct {
     int64_t launches;                              /* all kernels launched by the handle */
     int64_t class_launches[CUALIGN_NUM_KERNEL_CLASSES];
@@ -145,7 +145,9 @@ typedef struct {
 #define CUALIGN_K_MATCH   4 /* a7 + a8: matching on y^c and z^c, evaluate, best */
 #define CUALIGN_K_INIT    5 /* a1 + a2: validation, L layouts, S build */
 #define CUALIGN_K_STATE   6 /* get/set state gathers and scatters */
-#define CUALIGN_K_OTHER   7
+#define CUALIGN_K_OTHER   7 /* iteration counter advance */
+#define CUALIGN_K_EVAL    8 /* a8: evaluate M_y, M_z + final score / select / best reduction */
+#define CUALIGN_K_MATCHAUX 9 /* a7 bookkeeping: mates from suitors, best-matching copy */
 
 /* a1 + a2: validate, copy A, B, L to the device, build L's A-side rows and
  * B-side incidence, build S (Alg. 3) and its square layout, zero the BP state

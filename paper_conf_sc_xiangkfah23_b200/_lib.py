@@ -22,9 +22,10 @@ FLAG_ROUND_DAMPED = 0x08
 FLAG_TIMING = 0x10
 FLAG_MATCH_ROUNDS = 0x20
 
-K_TOP2, K_EDGE, K_SQUARE, K_ROWSUM, K_MATCH, K_INIT, K_STATE, K_OTHER = range(8)
-KERNEL_CLASS_NAMES = ["top2", "edge", "square", "rowsum", "match", "init", "state", "other"]
-NUM_KERNEL_CLASSES = 8
+K_TOP2, K_EDGE, K_SQUARE, K_ROWSUM, K_MATCH, K_INIT, K_STATE, K_OTHER, K_EVAL, K_MATCHAUX = range(10)
+KERNEL_CLASS_NAMES = ["top2", "edge", "square", "rowsum", "match", "init", "state", "other", "eval",
+                      "matchaux"]
+NUM_KERNEL_CLASSES = 10
 
 # every symbol include/cualign_bp.h declares
 EXPORTED = ["cualign_bp_init", "cualign_bp_iterate", "cualign_bp_round", "cualign_bp_run",

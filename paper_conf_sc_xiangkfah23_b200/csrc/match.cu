@@ -538,7 +538,7 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
             cfg.numAttrs = 1;
             CA_CUDA(cudaLaunchKernelEx(&cfg, k_pointer_rounds, P));
         }
-        KScope ks(h, CUALIGN_K_MATCH);
+        KScope ks(h, CUALIGN_K_MATCHAUX);
         k_mark<<<grid_for(P.ninst * nA, 256, h->num_sms * 8), 256, 0, h->stream>>>(nA, P.ninst, P.mateA, h->mflag, m);
         CA_CUDA(cudaGetLastError());
         return CUALIGN_OK;
@@ -582,7 +582,7 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
         cudaFree(dbuf);
     }
     if (P.ninst * nT > 0) {
-        KScope ks(h, CUALIGN_K_MATCH);
+        KScope ks(h, CUALIGN_K_MATCHAUX);
         k_suitor_to_mates<<<grid_for(P.ninst * nT, 256, h->num_sms * 8), 256, 0, h->stream>>>(
             nT, P.ninst, fromB ? P.Lb : P.La, sT, fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP,
             h->mflag, m);
@@ -654,13 +654,13 @@ cualign_status match_round(cualign_bp *h)
     // overlap / card accumulators (the rest of rd persists: best)
     CA_CUDA(cudaMemsetAsync(&h->rd->overlap[0], 0, 4 * sizeof(unsigned long long), h->stream));
     {
-        KScope ks(h, CUALIGN_K_MATCH);
+        KScope ks(h, CUALIGN_K_EVAL);
         k_eval<<<h->eval_grid, 256, 0, h->stream>>>(E, (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha, h->beta,
                                                     h->p_dev, h->match_work);
         CA_CUDA(cudaGetLastError());
     }
     {
-        KScope ks(h, CUALIGN_K_MATCH);
+        KScope ks(h, CUALIGN_K_MATCHAUX);
         k_copy_best<<<grid_for(h->L.nA, 256, h->num_sms * 4), 256, 0, h->stream>>>(h->L.nA, h->mateA, h->rd,
                                                                                   h->best_mate);
         CA_CUDA(cudaGetLastError());
