@@ -169,12 +169,15 @@ cualign_status cualign_bp_iterate(cualign_bp *h, int32_t n_steps);
  * (best is tracked on the device); otherwise synchronises and fills *info. */
 cualign_status cualign_bp_round(cualign_bp *h, cualign_round_info *info);
 
-/* a3-a8 repeated: n_steps x (iterate(1), then round if with_round != 0),
- * replayed from a CUDA graph of one step captured on first use (no host work
- * per kernel; g = gamma^p is read by the kernels from a host-computed table,
- * reading Z2).  Same results as the equivalent sequence of iterate/round
- * calls.  Asynchronous on params.stream; read results with get_best. */
-cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t with_round);
+/* a3-a8 repeated: n_steps x (iterate(1) if what & CUALIGN_RUN_ITERATE, then
+ * round if what & CUALIGN_RUN_ROUND), replayed from a CUDA graph of one step
+ * captured on first use (no host work per kernel; g = gamma^p is read by the
+ * kernels from a host-computed table, reading Z2).  Same results as the
+ * equivalent sequence of iterate/round calls.  Asynchronous on params.stream;
+ * read results with get_best.  what must be 1, 2 or 3. */
+#define CUALIGN_RUN_ITERATE 1
+#define CUALIGN_RUN_ROUND   2
+cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t what);
 
 /* Diagnostics: enable (1) / disable (0) per-kernel event timing (as
  * CUALIGN_FLAG_TIMING).  Graph replays with timing on synchronise after each

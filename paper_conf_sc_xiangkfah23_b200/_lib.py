@@ -241,9 +241,10 @@ class CuAlignBP:
     def iterate(self, n_steps=1):
         _check(load_library().cualign_bp_iterate(self._h, int(n_steps)))
 
-    def run(self, n_steps=1, with_round=True):
+    def run(self, n_steps=1, with_round=True, iterate=True):
         """n_steps x (iterate(1) [+ round]) replayed from a CUDA graph (async)."""
-        _check(load_library().cualign_bp_run(self._h, int(n_steps), 1 if with_round else 0))
+        what = (1 if iterate else 0) | (2 if with_round else 0)
+        _check(load_library().cualign_bp_run(self._h, int(n_steps), what))
 
     def set_timing(self, on=True):
         _check(load_library().cualign_bp_set_timing(self._h, 1 if on else 0))

@@ -85,7 +85,7 @@ KScope::~KScope()
         cudaEvent_t e = get_event(h);
         if (h->capturing) {
             cudaEventRecordWithFlags(e, h->stream, cudaEventRecordExternal);
-            h->graph_events[1].push_back({cls, {b, e}});
+            h->graph_events[h->capture_what].push_back({cls, {b, e}});
         } else {
             cudaEventRecord(e, h->stream);
             h->events[cls].push_back({b, e});
@@ -96,20 +96,23 @@ KScope::~KScope()
 void invalidate_graphs(cualign_bp *h)
 {
     for (int t = 0; t < 2; t++)
-        for (int r = 0; r < 2; r++)
+        for (int r = 0; r < 4; r++)
             if (h->graph[t][r]) {
                 cudaGraphExecDestroy(h->graph[t][r]);
                 h->graph[t][r] = nullptr;
             }
-    for (auto &pe : h->graph_events[1]) {
-        h->event_pool.push_back(pe.second.a);
-        h->event_pool.push_back(pe.second.b);
+    for (int r = 0; r < 4; r++) {
+        for (auto &pe : h->graph_events[r]) {
+            h->event_pool.push_back(pe.second.a);
+            h->event_pool.push_back(pe.second.b);
+        }
+        h->graph_events[r].clear();
     }
-    h->graph_events[1].clear();
 }
 
 // Capture one step (iterate(1) [+ round]) on the handle's capture stream.
-static cualign_status capture_step(cualign_bp *h, int timed, int with_round)
+// what: bit 0 = iterate(1), bit 1 = round (CUALIGN_RUN_*)
+static cualign_status capture_step(cualign_bp *h, int timed, int what)
 {
     const int32_t p_save = h->p;
     const int64_t l0 = h->launches;
@@ -120,11 +123,12 @@ static cualign_status capture_step(cualign_bp *h, int timed, int with_round)
     h->timing = timed != 0;
     h->stream = h->gstream;
     h->capturing = true;
+    h->capture_what = what;
     cualign_status st = CUALIGN_OK;
     cudaError_t e = cudaStreamBeginCapture(h->gstream, cudaStreamCaptureModeThreadLocal);
     if (e == cudaSuccess) {
-        st = bp_iterate(h, 1);
-        if (st == CUALIGN_OK && with_round) st = match_round(h);
+        if (what & CUALIGN_RUN_ITERATE) st = bp_iterate(h, 1);
+        if (st == CUALIGN_OK && (what & CUALIGN_RUN_ROUND)) st = match_round(h);
         cudaGraph_t g = nullptr;
         cudaError_t e2 = cudaStreamEndCapture(h->gstream, &g);
         if (st == CUALIGN_OK && e2 != cudaSuccess) {
@@ -132,7 +136,7 @@ static cualign_status capture_step(cualign_bp *h, int timed, int with_round)
             st = CUALIGN_ECUDA;
         }
         if (st == CUALIGN_OK) {
-            e2 = cudaGraphInstantiate(&h->graph[timed][with_round], g, 0);
+            e2 = cudaGraphInstantiate(&h->graph[timed][what], g, 0);
             if (e2 != cudaSuccess) {
                 set_error("graph instantiate: %s", cudaGetErrorString(e2));
                 st = CUALIGN_ECUDA;
@@ -147,9 +151,9 @@ static cualign_status capture_step(cualign_bp *h, int timed, int with_round)
     h->stream = user;
     h->timing = timing_save;
     h->p = p_save;
-    h->graph_launches[timed][with_round] = h->launches - l0;
+    h->graph_launches[timed][what] = h->launches - l0;
     for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
-        h->graph_class_launches[timed][with_round][c] = h->class_launches[c] - c0[c];
+        h->graph_class_launches[timed][what][c] = h->class_launches[c] - c0[c];
         h->class_launches[c] = c0[c];
     }
     h->launches = l0;
@@ -159,29 +163,29 @@ static cualign_status capture_step(cualign_bp *h, int timed, int with_round)
 
 // n steps through the captured graph; the user stream and the capture stream
 // are ordered with events, so the caller's stream semantics are preserved.
-static cualign_status run_graph(cualign_bp *h, int32_t n, int with_round)
+static cualign_status run_graph(cualign_bp *h, int32_t n, int what)
 {
     const int timed = h->timing ? 1 : 0;
     CA_TRY(ensure_gh(h, (int64_t)h->p + n + 1));
-    if (!h->graph[timed][with_round]) CA_TRY(capture_step(h, timed, with_round));
-    cudaGraphExec_t ge = h->graph[timed][with_round];
+    if (!h->graph[timed][what]) CA_TRY(capture_step(h, timed, what));
+    cudaGraphExec_t ge = h->graph[timed][what];
     CA_CUDA(cudaEventRecord(h->sync_ev[0], h->stream));
     CA_CUDA(cudaStreamWaitEvent(h->gstream, h->sync_ev[0], 0));
     for (int32_t k = 0; k < n; k++) {
         CA_CUDA(cudaGraphLaunch(ge, h->gstream));
-        h->p += 1;
-        h->launches += h->graph_launches[timed][with_round];
+        if (what & CUALIGN_RUN_ITERATE) h->p += 1;
+        h->launches += h->graph_launches[timed][what];
         for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++)
-            h->class_launches[c] += h->graph_class_launches[timed][with_round][c];
+            h->class_launches[c] += h->graph_class_launches[timed][what][c];
         if (timed) {
             CA_CUDA(cudaStreamSynchronize(h->gstream));
-            for (auto &pe : h->graph_events[1]) {
+            for (auto &pe : h->graph_events[what]) {
                 float ms = 0.f;
                 if (cudaEventElapsedTime(&ms, pe.second.a, pe.second.b) == cudaSuccess) h->class_ms[pe.first] += ms;
             }
         }
     }
-    if (with_round) h->have_info = true;
+    if (what & CUALIGN_RUN_ROUND) h->have_info = true;
     CA_CUDA(cudaEventRecord(h->sync_ev[1], h->gstream));
     CA_CUDA(cudaStreamWaitEvent(h->stream, h->sync_ev[1], 0));
     return CUALIGN_OK;
@@ -360,7 +364,7 @@ cualign_status cualign_bp_iterate(cualign_bp *h, int32_t n_steps)
     return bp_iterate(h, n_steps);
 }
 
-cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t with_round)
+cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t what)
 {
     API_ENTER();
     CHECK_H();
@@ -369,7 +373,11 @@ cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t with_round
         return CUALIGN_EINVAL;
     }
     if (n_steps == 0) return CUALIGN_OK;
-    return run_graph(h, n_steps, with_round ? 1 : 0);
+    if (what < 1 || what > 3) {
+        set_error("run: what must be CUALIGN_RUN_ITERATE, CUALIGN_RUN_ROUND or both");
+        return CUALIGN_EINVAL;
+    }
+    return run_graph(h, n_steps, what);
 }
 
 cualign_status cualign_bp_set_timing(cualign_bp *h, int32_t on)

@@ -113,10 +113,11 @@ struct cualign_bp {
     cudaStream_t gstream = nullptr;     // capture / replay stream (never the legacy stream)
     cudaEvent_t sync_ev[2] = {nullptr, nullptr};
     bool capturing = false;
-    cudaGraphExec_t graph[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}}; // [timed][round]
-    int64_t graph_launches[2][2] = {{0, 0}, {0, 0}};                        // kernels per replay
-    int64_t graph_class_launches[2][2][CUALIGN_NUM_KERNEL_CLASSES] = {};
-    std::vector<std::pair<int, cualign::EventPair>> graph_events[2];        // timed graphs' events
+    int capture_what = 0;
+    cudaGraphExec_t graph[2][4] = {};                       // [timed][what = CUALIGN_RUN_* bits]
+    int64_t graph_launches[2][4] = {};                      // kernels per replay
+    int64_t graph_class_launches[2][4][CUALIGN_NUM_KERNEL_CLASSES] = {};
+    std::vector<std::pair<int, cualign::EventPair>> graph_events[4]; // timed graphs' event nodes
 
     // matching (two instances: y and z)
     int32_t *candA = nullptr, *candB = nullptr, *mateA = nullptr, *mateB = nullptr;

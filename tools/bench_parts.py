@@ -30,11 +30,9 @@ def main():
     h.run(args.pre)
     torch.cuda.synchronize()
     h.stats(reset=True)
-    # rounds only, at the fixed state: event-timed eager launches with the
-    # queue kept full by a pre-enqueued iteration-free sequence
+    # rounds only, at the fixed state (graph replays, event nodes per kernel)
     h.set_timing(True)
-    for _ in range(args.n):
-        h.round(sync=False)
+    h.run(args.n, with_round=True, iterate=False)
     torch.cuda.synchronize()
     r = h.stats(reset=True)
     h.run(args.n, with_round=False)
