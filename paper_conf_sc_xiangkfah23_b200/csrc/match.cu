@@ -26,6 +26,7 @@
 #include "internal.cuh"
 
 #include <cooperative_groups.h>
+#include <cub/cub.cuh>
 
 namespace cg = cooperative_groups;
 
@@ -325,6 +326,30 @@ __global__ void k_mark(int64_t nA, int ninst, const int32_t *__restrict__ mateA,
 }
 
 // ---------------------------------------------------------------- evaluate
+constexpr int64_t LONG_ROW = 32; // square rows longer than this are chunked for evaluate
+
+__global__ void k_longrow_count(int64_t m, const int64_t *__restrict__ sq_rp, int64_t *__restrict__ cnt)
+{
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t len = sq_rp[e + 1] - sq_rp[e];
+        cnt[e] = len > LONG_ROW ? (len + LONG_ROW - 1) / LONG_ROW : 0;
+    }
+}
+
+__global__ void k_longrow_fill(int64_t m, const int64_t *__restrict__ sq_rp, const int64_t *__restrict__ start,
+                               int32_t *__restrict__ lc_e, int64_t *__restrict__ lc_q)
+{
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t len = sq_rp[e + 1] - sq_rp[e];
+        if (len <= LONG_ROW) continue;
+        int64_t c = start[e];
+        for (int64_t q = sq_rp[e]; q < sq_rp[e + 1]; q += LONG_ROW, c++) {
+            lc_e[c] = (int32_t)e;
+            lc_q[c] = q;
+        }
+    }
+}
+
 template <class T>
 __device__ T block_sum(T v, T *smem)
 {
@@ -354,6 +379,9 @@ struct EvalParams {
     const int32_t *mateA; // 2 instances, final
     const uint8_t *mflag; // [2][m]: edge matched
     int64_t m;
+    int64_t nlc;          // chunks of the long square rows
+    const int32_t *lc_e;  // chunk -> row (edge)
+    const int64_t *lc_q;  // chunk -> first square
     double *partial_w;    // [2][gridDim]
     RoundDev *rd;
 };
@@ -435,6 +463,8 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, con
     const int64_t nt = ((int64_t)gridDim.x * blockDim.x) / G;
     double wsum[2] = {0.0, 0.0};
     unsigned long long ov[2] = {0, 0}, card[2] = {0, 0};
+    // part 1: one tile per A vertex (rows longer than LONG_ROW squares are
+    // skipped here and counted in part 2)
     for (int64_t a = t0; a < P.nA; a += nt) {
         const int es[2] = {P.mateA[a], P.mateA[P.nA + a]};
 #pragma unroll
@@ -445,8 +475,22 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, con
                 wsum[k] += P.w[e];
                 card[k]++;
             }
-            const int64_t hi = P.sq_rp[e + 1];
-            for (int64_t q = P.sq_rp[e] + lane; q < hi; q += G)
+            const int64_t lo = P.sq_rp[e], hi = P.sq_rp[e + 1];
+            if (hi - lo > LONG_ROW) continue;
+            for (int64_t q = lo + lane; q < hi; q += G)
+                if (P.mflag[k * P.m + P.sq_ef[q].y]) ov[k]++;
+        }
+    }
+    // part 2: the long rows, cut once (at setup) into chunks of LONG_ROW
+    // squares, one tile per chunk: the work of hub rows is spread evenly
+    for (int64_t c = t0; c < P.nlc; c += nt) {
+        const int e = P.lc_e[c];
+        const int64_t q0 = P.lc_q[c];
+        const int64_t hi = min(q0 + (int64_t)LONG_ROW, P.sq_rp[e + 1]);
+#pragma unroll
+        for (int k = 0; k < 2; k++) {
+            if (!P.mflag[k * P.m + e]) continue;
+            for (int64_t q = q0 + lane; q < hi; q += G)
                 if (P.mflag[k * P.m + P.sq_ef[q].y]) ov[k]++;
         }
     }
@@ -621,6 +665,36 @@ cualign_status match_setup(cualign_bp *h)
         h->max_deg_b = (int64_t)md[1];
         h->propose_from_b = h->max_deg_b < h->max_deg_a;
     }
+    // long square rows, chunked for a balanced evaluate (static: S is fixed)
+    if (h->sq_rp && h->L.m > 0) {
+        KScope ks(h, CUALIGN_K_INIT);
+        const int64_t m = h->L.m;
+        int64_t *cnt = nullptr, *start = nullptr;
+        void *tmp = nullptr;
+        size_t tb = 0;
+        CA_CUDA(cudaMalloc(&cnt, sizeof(int64_t) * (size_t)m));
+        CA_CUDA(cudaMalloc(&start, sizeof(int64_t) * (size_t)m));
+        k_longrow_count<<<grid_for(m, 256, h->num_sms * 8), 256, 0, h->stream>>>(m, h->sq_rp, cnt);
+        CA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, start, (int)m, h->stream));
+        CA_CUDA(cudaMalloc(&tmp, tb ? tb : 1));
+        CA_CUDA(cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, start, (int)m, h->stream));
+        int64_t last[2] = {0, 0};
+        CA_CUDA(cudaMemcpyAsync(&last[0], start + m - 1, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaMemcpyAsync(&last[1], cnt + m - 1, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaStreamSynchronize(h->stream));
+        h->nlc = last[0] + last[1];
+        cualign_status st = dalloc(h, &h->lc_e, (size_t)h->nlc + 1);
+        if (st == CUALIGN_OK) st = dalloc(h, &h->lc_q, (size_t)h->nlc + 1);
+        if (st == CUALIGN_OK && h->nlc)
+            k_longrow_fill<<<grid_for(m, 256, h->num_sms * 8), 256, 0, h->stream>>>(m, h->sq_rp, start, h->lc_e,
+                                                                                   h->lc_q);
+        cudaStreamSynchronize(h->stream);
+        cudaFree(cnt);
+        cudaFree(start);
+        cudaFree(tmp);
+        CA_TRY(st);
+        CA_CUDA(cudaGetLastError());
+    }
     int occ = 0;
     CA_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pointer_rounds, 256, 0));
     if (occ < 1) occ = 1;
@@ -649,6 +723,9 @@ cualign_status match_round(cualign_bp *h)
     E.mateA = h->mateA;
     E.mflag = h->mflag;
     E.m = h->L.m;
+    E.nlc = h->nlc;
+    E.lc_e = h->lc_e;
+    E.lc_q = h->lc_q;
     E.partial_w = h->partial_w;
     E.rd = h->rd;
     // overlap / card accumulators (the rest of rd persists: best)
