@@ -406,7 +406,12 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
     }
     // the graphs are not needed after S is built
     CA_CUDA(cudaStreamSynchronize(h->stream));
-    for (void *p : {(void *)Ap, (void *)Aj, (void *)Bp, (void *)Bj}) dfree(h, p);
+    // the graphs stay resident: evaluate counts overlapped edges on them
+    h->Ap = Ap;
+    h->Aj = Aj;
+    h->Bp = Bp;
+    h->Bj = Bj;
+    h->nA_edges_dir = nnzA;
     // fixed-point scale for the F row sums: beta * max_row * 2^bits < 2^62
     {
         double bound = h->beta * (double)h->max_row;

@@ -126,10 +126,11 @@ struct cualign_bp {
     int match_grid = 0, match_block = 256, eval_grid = 1;
     unsigned long long *match_work = nullptr; // proposals (suitor) or rounds, per instance
     bool propose_from_b = false;              // suitor: proposing side (smaller max degree)
-    uint8_t *mflag = nullptr;                 // [2][m]: edge in M_y / M_z (evaluate)
-    int64_t nlc = 0;                          // long square rows cut into chunks (evaluate balance)
-    int32_t *lc_e = nullptr;
-    int64_t *lc_q = nullptr;
+    // graphs A and B (CSR), kept for evaluate: overlap = #A edges {i,j} with
+    // (M(i), M(j)) in E_B
+    int64_t *Ap = nullptr, *Bp = nullptr;
+    int32_t *Aj = nullptr, *Bj = nullptr;
+    int64_t nA_edges_dir = 0;
     int64_t max_deg_a = 0, max_deg_b = 0;     // max degree of A / B vertices in L
     cualign::RoundDev *rd = nullptr;
     cualign_round_info last_info{};

@@ -10,7 +10,7 @@
 //  * SUITOR (default).  Every vertex of one side proposes to its heaviest
 //    eligible neighbour whose current suitor is lighter; a CAS on the
 //    neighbour's suitor slot (an edge id) installs the proposal and the
-//    displaced suitor -- now owned by the same thread -- proposes again
+//    displaced suitor -- now owned by the same thread tile -- proposes again
 //    (the Suitor algorithm of Manne & Halappanavar, a lock-free form of the
 //    locally-dominant rule, here one-sided: see k_suitor).  One kernel, no
 //    grid-wide barriers.  y^c and z^c are matched in the same launch.
@@ -20,13 +20,14 @@
 //    vertices whose target got matched re-point; grid.sync() between phases
 //    replaces the Q_C / Q_N queues.  Kept for comparison (ablation).
 //
-// Evaluate: weight(M) over the original w (Z9), overlap(M) = x'Sx/2 counted on
-// the square layout (each square {e<f} stored once, at e), score = alpha*w +
-// beta*overlap (Eq. 1, :64-72); M_y wins ties; best on a strict > (Z8).
+// Evaluate (Eq. 1): weight(M) over the original w (Z9);
+// overlap(M) counted straight from the paper's definition: the
+// A edges {i, j} whose images (M(i), M(j)) are a B edge -- equal to x'Sx/2
+// (pin P11), but it reads the 20 MB graph CSRs instead of scattered S rows;
+// score = alpha*w + beta*overlap; M_y wins ties; best on a strict > (Z8).
 #include "internal.cuh"
 
 #include <cooperative_groups.h>
-#include <cub/cub.cuh>
 
 namespace cg = cooperative_groups;
 
@@ -46,9 +47,11 @@ struct MatchParams {
     int propose_from_b;     // SUITOR: proposing side
     int32_t *mateA, *mateB;
     RoundDev *rd;
-    unsigned long long *work; // per instance: proposals (suitor) / rounds
+    unsigned long long *work; // proposals (suitor) / rounds, spread counters
     unsigned long long *dbg;  // optional diagnostics (CUALIGN_MATCH_DEBUG)
 };
+
+constexpr int WORK_SPREAD = 64, WORK_STRIDE = 16; // counter slots, 128 B apart
 
 __device__ __forceinline__ bool better(double xa, int ea, double xb, int eb)
 {
@@ -65,30 +68,13 @@ __device__ __forceinline__ const double *xk(const MatchParams &P, int k) { retur
 // suitor is worse, displacing it) reaches it in any order -- the Suitor
 // algorithm restricted to one side.  The proposing side is the one with the
 // smaller maximum degree (on the paper's workloads: the k candidates of each A
-// vertex), so no thread ever scans a hub's list.
+// vertex), so no tile ever scans a hub's list.
 // Slot v in [0, ninst*nP): instance k, proposer r.  suitor[k*nT + t] = edge
 // by which the current suitor proposes to target t (-1 = none).
 // One G-lane tile per proposer: the lanes scan the proposer's list together
-// (G edges per step, independent loads), a tile argmax picks the heaviest
-// eligible target, lane 0 attempts the CAS and the outcome is broadcast.
-constexpr int WORK_SPREAD = 64, WORK_STRIDE = 16; // counter slots, 128 B apart
-
-template <int G, int U, class Tile>
-__device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
-                                            int64_t nT, int64_t slot);
-
-template <int G, int U>
-__global__ void __launch_bounds__(128) k_suitor(MatchParams P)
-{
-    auto tile = cg::tiled_partition<G>(cg::this_thread_block());
-    const int lane = tile.thread_rank();
-    const bool fromB = P.propose_from_b != 0;
-    const int64_t nP = fromB ? P.nB : P.nA;
-    const int64_t nT = fromB ? P.nA : P.nB;
-    const int64_t slot = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
-    if (slot < P.ninst * nP) suitor_tile<G, U>(P, tile, lane, fromB, nP, nT, slot);
-}
-
+// (G x U edges per pass, the loads of a pass issued together), a tile argmax
+// picks the heaviest eligible target, lane 0 attempts the CAS and the outcome
+// is broadcast.
 template <int G, int U, class Tile>
 __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
                                             int64_t nT, int64_t slot)
@@ -101,14 +87,12 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
     const int32_t *__restrict__ tgt = fromB ? P.La : P.Lb;   // target vertex of an edge
     const int32_t *__restrict__ own = fromB ? P.Lb : P.La;   // proposer vertex of an edge
     unsigned long long proposals = 0, scans = 0;
-    // U edges per lane per pass: the loads of a pass are issued together;
-    // positions in L's arrays are < m < 2^31, so 32-bit index math
     while (true) {
         scans++;
         // heaviest eligible neighbour of `cur` whose suitor is lighter
         int best = -1;
         double bx = 0.0;
-        const int hi = (int)rp[cur + 1];
+        const int hi = (int)rp[cur + 1]; // positions < m < 2^31: 32-bit index math
         for (int j0 = (int)rp[cur] + lane; j0 < hi; j0 += G * U) {
             int ee[U], tt[U], ss[U];
             double xx[U], xs[U];
@@ -147,7 +131,7 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
             }
         }
         if (best < 0) break; // tile-uniform after the all-reduce
-        int code = 0;        // 0 retry, 1 done, 2 displaced
+        int code = 0;        // 0 rescan, 1 done, 2 displaced
         int next = cur;
         if (lane == 0) {
             int32_t *slotp = sT + __ldg(tgt + best);
@@ -182,6 +166,32 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
         if (scans > 8) atomicAdd(P.dbg + 2, 1ull);
         if (scans > 64) atomicAdd(P.dbg + 3, 1ull);
         atomicMax(P.dbg + 4, proposals);
+    }
+}
+
+template <int G, int U>
+__global__ void __launch_bounds__(128) k_suitor(MatchParams P)
+{
+    auto tile = cg::tiled_partition<G>(cg::this_thread_block());
+    const int lane = tile.thread_rank();
+    const bool fromB = P.propose_from_b != 0;
+    const int64_t nP = fromB ? P.nB : P.nA;
+    const int64_t nT = fromB ? P.nA : P.nB;
+    const int64_t slot = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
+    if (slot < P.ninst * nP) suitor_tile<G, U>(P, tile, lane, fromB, nP, nT, slot);
+}
+
+// the final suitor of each target is its mate (mate arrays pre-set to -1)
+__global__ void k_suitor_to_mates(int64_t nT, int ninst, const int32_t *__restrict__ own,
+                                  const int32_t *__restrict__ sT, int32_t *__restrict__ mateT,
+                                  int32_t *__restrict__ mateP, int64_t nP)
+{
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * nT;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        const int k = (int)(v / nT);
+        const int e = sT[v];
+        mateT[v] = e;
+        if (e >= 0) mateP[k * nP + own[e]] = e;
     }
 }
 
@@ -295,61 +305,7 @@ __global__ void __launch_bounds__(256) k_pointer_rounds(MatchParams P)
     }
 }
 
-// ------------------------------------------------------- mates from suitors
-// the final suitor of each target is its mate (mateX arrays pre-set to -1)
-// and every matched edge is flagged in mflag (pre-cleared) for the evaluation
-__global__ void k_suitor_to_mates(int64_t nT, int ninst, const int32_t *__restrict__ own,
-                                  const int32_t *__restrict__ sT, int32_t *__restrict__ mateT,
-                                  int32_t *__restrict__ mateP, int64_t nP, uint8_t *__restrict__ mflag, int64_t m)
-{
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * nT;
-         v += (int64_t)gridDim.x * blockDim.x) {
-        const int k = (int)(v / nT);
-        const int e = sT[v];
-        mateT[v] = e;
-        if (e >= 0) {
-            mateP[k * nP + own[e]] = e;
-            mflag[k * m + e] = 1;
-        }
-    }
-}
-
-// pointer-round schedule: flag the matched edges from mate_A
-__global__ void k_mark(int64_t nA, int ninst, const int32_t *__restrict__ mateA, uint8_t *__restrict__ mflag,
-                       int64_t m)
-{
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * nA;
-         v += (int64_t)gridDim.x * blockDim.x) {
-        const int e = mateA[v];
-        if (e >= 0) mflag[(v / nA) * m + e] = 1;
-    }
-}
-
 // ---------------------------------------------------------------- evaluate
-constexpr int64_t LONG_ROW = 32; // square rows longer than this are chunked for evaluate
-
-__global__ void k_longrow_count(int64_t m, const int64_t *__restrict__ sq_rp, int64_t *__restrict__ cnt)
-{
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t len = sq_rp[e + 1] - sq_rp[e];
-        cnt[e] = len > LONG_ROW ? (len + LONG_ROW - 1) / LONG_ROW : 0;
-    }
-}
-
-__global__ void k_longrow_fill(int64_t m, const int64_t *__restrict__ sq_rp, const int64_t *__restrict__ start,
-                               int32_t *__restrict__ lc_e, int64_t *__restrict__ lc_q)
-{
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t len = sq_rp[e + 1] - sq_rp[e];
-        if (len <= LONG_ROW) continue;
-        int64_t c = start[e];
-        for (int64_t q = sq_rp[e]; q < sq_rp[e + 1]; q += LONG_ROW, c++) {
-            lc_e[c] = (int32_t)e;
-            lc_q[c] = q;
-        }
-    }
-}
-
 template <class T>
 __device__ T block_sum(T v, T *smem)
 {
@@ -370,18 +326,25 @@ __device__ T block_sum(T v, T *smem)
     return r; // valid in thread 0
 }
 
+__device__ __forceinline__ bool bsearch_i32(const int32_t *x, int64_t lo, int64_t hi, int32_t v)
+{
+    while (lo < hi) {
+        const int64_t mid = lo + ((hi - lo) >> 1);
+        const int32_t xm = __ldg(x + mid);
+        if (xm < v) lo = mid + 1;
+        else if (xm > v) hi = mid;
+        else return true;
+    }
+    return false;
+}
+
 struct EvalParams {
     int64_t nA;
-    const int32_t *La;
+    const int32_t *Lb;
     const double *w;
-    const int64_t *sq_rp;
-    const int2 *sq_ef;
     const int32_t *mateA; // 2 instances, final
-    const uint8_t *mflag; // [2][m]: edge matched
-    int64_t m;
-    int64_t nlc;          // chunks of the long square rows
-    const int32_t *lc_e;  // chunk -> row (edge)
-    const int64_t *lc_q;  // chunk -> first square
+    const int64_t *Ap, *Bp;
+    const int32_t *Aj, *Bj;
     double *partial_w;    // [2][gridDim]
     RoundDev *rd;
 };
@@ -446,11 +409,12 @@ __device__ void round_final_block(const EvalParams &P, int nblocks, int exact, d
     rd->source = src;
 }
 
-// Evaluate both matchings: weight partial sums per block (fixed partition:
-// deterministic), overlap and cardinality as integer atomics (exact).  A
-// 4-lane tile per A vertex handles M_y and M_z; the lanes stride over the
-// matched edge's square row (rows reach thousands of squares).  The last block
-// to finish runs the final reduction (no separate launch).
+// Evaluate M_y and M_z: a 4-lane tile per A vertex i.  weight: partial sums
+// per block over a fixed partition (deterministic); cardinality and overlap:
+// integer atomics (exact).  Overlap by PAPER.md:60: for each A edge {i, j}
+// (j > i, so once), count it when both ends are matched and (M(i), M(j)) is
+// an edge of B (binary search in B's sorted row of M(i)).  The last block to
+// finish runs the final reduction (no separate launch).
 __global__ void __launch_bounds__(256)
 k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, const unsigned long long *work)
 {
@@ -463,35 +427,31 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, con
     const int64_t nt = ((int64_t)gridDim.x * blockDim.x) / G;
     double wsum[2] = {0.0, 0.0};
     unsigned long long ov[2] = {0, 0}, card[2] = {0, 0};
-    // part 1: one tile per A vertex (rows longer than LONG_ROW squares are
-    // skipped here and counted in part 2)
-    for (int64_t a = t0; a < P.nA; a += nt) {
-        const int es[2] = {P.mateA[a], P.mateA[P.nA + a]};
-#pragma unroll
-        for (int k = 0; k < 2; k++) {
-            const int e = es[k];
-            if (e < 0) continue;
-            if (lane == 0) {
-                wsum[k] += P.w[e];
-                card[k]++;
+    for (int64_t i = t0; i < P.nA; i += nt) {
+        const int e0 = P.mateA[i], e1 = P.mateA[P.nA + i];
+        if (e0 < 0 && e1 < 0) continue;
+        const int mb0 = e0 >= 0 ? __ldg(P.Lb + e0) : -1; // M_y(i) in V_B
+        const int mb1 = e1 >= 0 ? __ldg(P.Lb + e1) : -1; // M_z(i)
+        if (lane == 0) {
+            if (e0 >= 0) {
+                wsum[0] += P.w[e0];
+                card[0]++;
             }
-            const int64_t lo = P.sq_rp[e], hi = P.sq_rp[e + 1];
-            if (hi - lo > LONG_ROW) continue;
-            for (int64_t q = lo + lane; q < hi; q += G)
-                if (P.mflag[k * P.m + P.sq_ef[q].y]) ov[k]++;
+            if (e1 >= 0) {
+                wsum[1] += P.w[e1];
+                card[1]++;
+            }
         }
-    }
-    // part 2: the long rows, cut once (at setup) into chunks of LONG_ROW
-    // squares, one tile per chunk: the work of hub rows is spread evenly
-    for (int64_t c = t0; c < P.nlc; c += nt) {
-        const int e = P.lc_e[c];
-        const int64_t q0 = P.lc_q[c];
-        const int64_t hi = min(q0 + (int64_t)LONG_ROW, P.sq_rp[e + 1]);
-#pragma unroll
-        for (int k = 0; k < 2; k++) {
-            if (!P.mflag[k * P.m + e]) continue;
-            for (int64_t q = q0 + lane; q < hi; q += G)
-                if (P.mflag[k * P.m + P.sq_ef[q].y]) ov[k]++;
+        const int64_t b0lo = mb0 >= 0 ? P.Bp[mb0] : 0, b0hi = mb0 >= 0 ? P.Bp[mb0 + 1] : 0;
+        const int64_t b1lo = mb1 >= 0 ? P.Bp[mb1] : 0, b1hi = mb1 >= 0 ? P.Bp[mb1 + 1] : 0;
+        const int64_t hi = P.Ap[i + 1];
+        for (int64_t x = P.Ap[i] + lane; x < hi; x += G) {
+            const int j = __ldg(P.Aj + x);
+            if (j <= i) continue;
+            const int f0 = mb0 >= 0 ? P.mateA[j] : -1;
+            const int f1 = mb1 >= 0 ? P.mateA[P.nA + j] : -1;
+            if (f0 >= 0 && bsearch_i32(P.Bj, b0lo, b0hi, __ldg(P.Lb + f0))) ov[0]++;
+            if (f1 >= 0 && bsearch_i32(P.Bj, b1lo, b1hi, __ldg(P.Lb + f1))) ov[1]++;
         }
     }
     for (int k = 0; k < 2; k++) {
@@ -536,8 +496,18 @@ __global__ void k_maxdeg(int64_t nA, const int64_t *__restrict__ Arow, int64_t n
             mb = d > mb ? d : mb;
         }
     }
-    if (ma) atomicMax(out, ma);
-    if (mb) atomicMax(out + 1, mb);
+    // warp max first: one atomic per warp
+#pragma unroll
+    for (int off = 16; off >= 1; off >>= 1) {
+        const unsigned long long oa = __shfl_xor_sync(0xffffffffu, ma, off);
+        const unsigned long long ob = __shfl_xor_sync(0xffffffffu, mb, off);
+        ma = oa > ma ? oa : ma;
+        mb = ob > mb ? ob : mb;
+    }
+    if ((threadIdx.x & 31) == 0) {
+        if (ma) atomicMax(out, ma);
+        if (mb) atomicMax(out + 1, mb);
+    }
 }
 
 MatchParams base_params(cualign_bp *h)
@@ -564,27 +534,21 @@ MatchParams base_params(cualign_bp *h)
 // run the matching of ninst instances; leaves mateA / mateB final
 cualign_status run_matching(cualign_bp *h, MatchParams &P)
 {
-    const int64_t nA = h->L.nA, nB = h->L.nB, m = h->L.m;
+    const int64_t nA = h->L.nA, nB = h->L.nB;
     CA_CUDA(cudaMemsetAsync(h->match_work, 0, WORK_SPREAD * WORK_STRIDE * sizeof(unsigned long long), h->stream));
-    CA_CUDA(cudaMemsetAsync(h->mflag, 0, (size_t)(2 * m + 1), h->stream));
     if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) {
-        {
-            KScope ks(h, CUALIGN_K_MATCH);
-            // cooperative launch through cudaLaunchKernelEx: capturable into a graph
-            cudaLaunchConfig_t cfg{};
-            cfg.gridDim = dim3(h->match_grid);
-            cfg.blockDim = dim3(256);
-            cfg.stream = h->stream;
-            cudaLaunchAttribute attr[1];
-            attr[0].id = cudaLaunchAttributeCooperative;
-            attr[0].val.cooperative = 1;
-            cfg.attrs = attr;
-            cfg.numAttrs = 1;
-            CA_CUDA(cudaLaunchKernelEx(&cfg, k_pointer_rounds, P));
-        }
-        KScope ks(h, CUALIGN_K_MATCHAUX);
-        k_mark<<<grid_for(P.ninst * nA, 256, h->num_sms * 8), 256, 0, h->stream>>>(nA, P.ninst, P.mateA, h->mflag, m);
-        CA_CUDA(cudaGetLastError());
+        KScope ks(h, CUALIGN_K_MATCH);
+        // cooperative launch through cudaLaunchKernelEx: capturable into a graph
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3(h->match_grid);
+        cfg.blockDim = dim3(256);
+        cfg.stream = h->stream;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeCooperative;
+        attr[0].val.cooperative = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        CA_CUDA(cudaLaunchKernelEx(&cfg, k_pointer_rounds, P));
         return CUALIGN_OK;
     }
     const bool fromB = h->propose_from_b;
@@ -611,10 +575,10 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
         const int G = genv ? genv : (dmax > 64 ? 32 : (dmax > 24 ? 16 : (dmax > 20 ? 8 : 4)));
         if (G == 32) k_suitor<32, 2><<<grid_for(slots * 32, 128, 1 << 30), 128, 0, h->stream>>>(P);
         else if (G == 16) k_suitor<16, 2><<<grid_for(slots * 16, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else if (G == 4) k_suitor<4, 5><<<grid_for(slots * 4, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else if (G == 8) k_suitor<8, 3><<<grid_for(slots * 8, 128, 1 << 30), 128, 0, h->stream>>>(P);
         else if (G == 2) k_suitor<2, 9><<<grid_for(slots * 2, 128, 1 << 30), 128, 0, h->stream>>>(P);
         else if (G == 1) k_suitor<1, 8><<<grid_for(slots, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else k_suitor<8, 3><<<grid_for(slots * 8, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else k_suitor<4, 5><<<grid_for(slots * 4, 128, 1 << 30), 128, 0, h->stream>>>(P);
         CA_CUDA(cudaGetLastError());
     }
     if (dbg) {
@@ -628,8 +592,7 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     if (P.ninst * nT > 0) {
         KScope ks(h, CUALIGN_K_MATCHAUX);
         k_suitor_to_mates<<<grid_for(P.ninst * nT, 256, h->num_sms * 8), 256, 0, h->stream>>>(
-            nT, P.ninst, fromB ? P.Lb : P.La, sT, fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP,
-            h->mflag, m);
+            nT, P.ninst, fromB ? P.Lb : P.La, sT, fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP);
         CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;
@@ -647,7 +610,6 @@ cualign_status match_setup(cualign_bp *h)
     CA_TRY(dalloc(h, &h->best_mate, nA + 1));
     CA_TRY(dalloc(h, &h->rd, 1));
     CA_TRY(dalloc(h, &h->match_work, WORK_SPREAD * WORK_STRIDE));
-    CA_TRY(dalloc(h, &h->mflag, (size_t)(2 * h->L.m + 1)));
     CA_CUDA(cudaMemsetAsync(h->rd, 0, sizeof(RoundDev), h->stream));
     CA_CUDA(cudaMemsetAsync(h->mateA, 0xff, sizeof(int32_t) * (2 * nA + 1), h->stream));
     CA_CUDA(cudaMemsetAsync(h->mateB, 0xff, sizeof(int32_t) * (2 * nB + 1), h->stream));
@@ -664,36 +626,6 @@ cualign_status match_setup(cualign_bp *h)
         h->max_deg_a = (int64_t)md[0];
         h->max_deg_b = (int64_t)md[1];
         h->propose_from_b = h->max_deg_b < h->max_deg_a;
-    }
-    // long square rows, chunked for a balanced evaluate (static: S is fixed)
-    if (h->sq_rp && h->L.m > 0) {
-        KScope ks(h, CUALIGN_K_INIT);
-        const int64_t m = h->L.m;
-        int64_t *cnt = nullptr, *start = nullptr;
-        void *tmp = nullptr;
-        size_t tb = 0;
-        CA_CUDA(cudaMalloc(&cnt, sizeof(int64_t) * (size_t)m));
-        CA_CUDA(cudaMalloc(&start, sizeof(int64_t) * (size_t)m));
-        k_longrow_count<<<grid_for(m, 256, h->num_sms * 8), 256, 0, h->stream>>>(m, h->sq_rp, cnt);
-        CA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, start, (int)m, h->stream));
-        CA_CUDA(cudaMalloc(&tmp, tb ? tb : 1));
-        CA_CUDA(cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, start, (int)m, h->stream));
-        int64_t last[2] = {0, 0};
-        CA_CUDA(cudaMemcpyAsync(&last[0], start + m - 1, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
-        CA_CUDA(cudaMemcpyAsync(&last[1], cnt + m - 1, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
-        CA_CUDA(cudaStreamSynchronize(h->stream));
-        h->nlc = last[0] + last[1];
-        cualign_status st = dalloc(h, &h->lc_e, (size_t)h->nlc + 1);
-        if (st == CUALIGN_OK) st = dalloc(h, &h->lc_q, (size_t)h->nlc + 1);
-        if (st == CUALIGN_OK && h->nlc)
-            k_longrow_fill<<<grid_for(m, 256, h->num_sms * 8), 256, 0, h->stream>>>(m, h->sq_rp, start, h->lc_e,
-                                                                                   h->lc_q);
-        cudaStreamSynchronize(h->stream);
-        cudaFree(cnt);
-        cudaFree(start);
-        cudaFree(tmp);
-        CA_TRY(st);
-        CA_CUDA(cudaGetLastError());
     }
     int occ = 0;
     CA_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pointer_rounds, 256, 0));
@@ -716,16 +648,13 @@ cualign_status match_round(cualign_bp *h)
     CA_TRY(run_matching(h, P));
     EvalParams E{};
     E.nA = h->L.nA;
-    E.La = h->L.La;
+    E.Lb = h->L.Lb;
     E.w = h->L.w;
-    E.sq_rp = h->sq_rp;
-    E.sq_ef = h->sq_ef;
     E.mateA = h->mateA;
-    E.mflag = h->mflag;
-    E.m = h->L.m;
-    E.nlc = h->nlc;
-    E.lc_e = h->lc_e;
-    E.lc_q = h->lc_q;
+    E.Ap = h->Ap;
+    E.Aj = h->Aj;
+    E.Bp = h->Bp;
+    E.Bj = h->Bj;
     E.partial_w = h->partial_w;
     E.rd = h->rd;
     // overlap / card accumulators (the rest of rd persists: best)
