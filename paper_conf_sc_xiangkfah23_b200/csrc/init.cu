@@ -224,6 +224,32 @@ __global__ void k_sq_pos(int64_t nsq, const int2 *__restrict__ sq_ef, const int6
     }
 }
 
+// undirected A edges as (i, j) pairs with i < j: the suffix of each sorted row
+__global__ void k_upper_count(int64_t n, const int64_t *__restrict__ rp, const int32_t *__restrict__ col,
+                              int64_t *__restrict__ cnt)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t lo = rp[i], hi = rp[i + 1];
+        const int64_t end = hi;
+        while (lo < hi) { // first position with col > i
+            const int64_t mid = lo + ((hi - lo) >> 1);
+            if (col[mid] <= (int32_t)i) lo = mid + 1;
+            else hi = mid;
+        }
+        cnt[i] = end - lo;
+    }
+}
+
+__global__ void k_upper_fill(int64_t n, const int64_t *__restrict__ rp, const int32_t *__restrict__ col,
+                             const int64_t *__restrict__ start, int2 *__restrict__ pairs)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t o = start[i];
+        for (int64_t x = rp[i]; x < rp[i + 1]; x++)
+            if (col[x] > (int32_t)i) pairs[o++] = make_int2((int)i, col[x]);
+    }
+}
+
 cualign_status upload(cualign_bp *h, void **dst, const void *src, size_t bytes, bool device_ptrs)
 {
     CA_TRY(dmalloc(h, dst, bytes));
@@ -406,12 +432,43 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
     }
     // the graphs are not needed after S is built
     CA_CUDA(cudaStreamSynchronize(h->stream));
-    // the graphs stay resident: evaluate counts overlapped edges on them
-    h->Ap = Ap;
-    h->Aj = Aj;
+    // Evaluate counts overlapped edges by the definition: it
+    // keeps B's CSR and the undirected A edges as a flat (i < j) pair list --
+    // one pair per thread, no per-vertex imbalance at hubs.
     h->Bp = Bp;
     h->Bj = Bj;
-    h->nA_edges_dir = nnzA;
+    {
+        KScope ks(h, CUALIGN_K_INIT);
+        const int64_t nA = A->n;
+        int64_t *cnt = nullptr, *start = nullptr;
+        void *tmp = nullptr;
+        size_t tb = 0;
+        h->nApairs = 0;
+        if (nA > 0) {
+            CA_CUDA(cudaMalloc(&cnt, sizeof(int64_t) * (size_t)nA));
+            CA_CUDA(cudaMalloc(&start, sizeof(int64_t) * (size_t)nA));
+            k_upper_count<<<grid_for(nA, 256, G), 256, 0, h->stream>>>(nA, Ap, Aj, cnt);
+            CA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, start, (int)nA, h->stream));
+            CA_CUDA(cudaMalloc(&tmp, tb ? tb : 1));
+            CA_CUDA(cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, start, (int)nA, h->stream));
+            int64_t last[2];
+            CA_CUDA(cudaMemcpyAsync(&last[0], start + nA - 1, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+            CA_CUDA(cudaMemcpyAsync(&last[1], cnt + nA - 1, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+            CA_CUDA(cudaStreamSynchronize(h->stream));
+            h->nApairs = last[0] + last[1];
+        }
+        cualign_status st = dalloc(h, &h->Apairs, (size_t)h->nApairs + 1);
+        if (st == CUALIGN_OK && h->nApairs)
+            k_upper_fill<<<grid_for(nA, 256, G), 256, 0, h->stream>>>(nA, Ap, Aj, start, h->Apairs);
+        cudaStreamSynchronize(h->stream);
+        if (cnt) cudaFree(cnt);
+        if (start) cudaFree(start);
+        if (tmp) cudaFree(tmp);
+        CA_TRY(st);
+        CA_CUDA(cudaGetLastError());
+    }
+    dfree(h, Ap);
+    dfree(h, Aj);
     // fixed-point scale for the F row sums: beta * max_row * 2^bits < 2^62
     {
         double bound = h->beta * (double)h->max_row;

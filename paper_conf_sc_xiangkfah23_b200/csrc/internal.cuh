@@ -128,9 +128,10 @@ struct cualign_bp {
     bool propose_from_b = false;              // suitor: proposing side (smaller max degree)
     // graphs A and B (CSR), kept for evaluate: overlap = #A edges {i,j} with
     // (M(i), M(j)) in E_B
-    int64_t *Ap = nullptr, *Bp = nullptr;
-    int32_t *Aj = nullptr, *Bj = nullptr;
-    int64_t nA_edges_dir = 0;
+    int64_t *Bp = nullptr;
+    int32_t *Bj = nullptr;
+    int2 *Apairs = nullptr;  // undirected A edges (i, j), i < j
+    int64_t nApairs = 0;
     int64_t max_deg_a = 0, max_deg_b = 0;     // max degree of A / B vertices in L
     cualign::RoundDev *rd = nullptr;
     cualign_round_info last_info{};

@@ -343,8 +343,10 @@ struct EvalParams {
     const int32_t *Lb;
     const double *w;
     const int32_t *mateA; // 2 instances, final
-    const int64_t *Ap, *Bp;
-    const int32_t *Aj, *Bj;
+    const int64_t *Bp;
+    const int32_t *Bj;
+    const int2 *pairs;    // undirected A edges (i < j)
+    int64_t npairs;
     double *partial_w;    // [2][gridDim]
     RoundDev *rd;
 };
@@ -409,49 +411,42 @@ __device__ void round_final_block(const EvalParams &P, int nblocks, int exact, d
     rd->source = src;
 }
 
-// Evaluate M_y and M_z: a 4-lane tile per A vertex i.  weight: partial sums
-// per block over a fixed partition (deterministic); cardinality and overlap:
-// integer atomics (exact).  Overlap by PAPER.md:60: for each A edge {i, j}
-// (j > i, so once), count it when both ends are matched and (M(i), M(j)) is
-// an edge of B (binary search in B's sorted row of M(i)).  The last block to
-// finish runs the final reduction (no separate launch).
+// Evaluate M_y and M_z.  weight: partial sums per block over a fixed
+// partition of the A vertices (deterministic); cardinality and overlap:
+// integer atomics (exact).  Overlap by PAPER.md:60: one thread per undirected
+// A edge {i, j}; it counts when both ends are matched and (M(i), M(j)) is an
+// edge of B (binary search in B's sorted row of M(i)) -- balanced whatever the
+// degree of i.  The last block to finish runs the final reduction.
 __global__ void __launch_bounds__(256)
 k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, const unsigned long long *work)
 {
     __shared__ double sd[32];
     __shared__ unsigned long long su[32];
     __shared__ bool last;
-    constexpr int G = 4;
-    const int lane = threadIdx.x & (G - 1);
-    const int64_t t0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
-    const int64_t nt = ((int64_t)gridDim.x * blockDim.x) / G;
+    const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
     double wsum[2] = {0.0, 0.0};
     unsigned long long ov[2] = {0, 0}, card[2] = {0, 0};
-    for (int64_t i = t0; i < P.nA; i += nt) {
+    for (int64_t i = tid; i < P.nA; i += nthr) {
         const int e0 = P.mateA[i], e1 = P.mateA[P.nA + i];
-        if (e0 < 0 && e1 < 0) continue;
-        const int mb0 = e0 >= 0 ? __ldg(P.Lb + e0) : -1; // M_y(i) in V_B
-        const int mb1 = e1 >= 0 ? __ldg(P.Lb + e1) : -1; // M_z(i)
-        if (lane == 0) {
-            if (e0 >= 0) {
-                wsum[0] += P.w[e0];
-                card[0]++;
-            }
-            if (e1 >= 0) {
-                wsum[1] += P.w[e1];
-                card[1]++;
-            }
+        if (e0 >= 0) {
+            wsum[0] += P.w[e0];
+            card[0]++;
         }
-        const int64_t b0lo = mb0 >= 0 ? P.Bp[mb0] : 0, b0hi = mb0 >= 0 ? P.Bp[mb0 + 1] : 0;
-        const int64_t b1lo = mb1 >= 0 ? P.Bp[mb1] : 0, b1hi = mb1 >= 0 ? P.Bp[mb1 + 1] : 0;
-        const int64_t hi = P.Ap[i + 1];
-        for (int64_t x = P.Ap[i] + lane; x < hi; x += G) {
-            const int j = __ldg(P.Aj + x);
-            if (j <= i) continue;
-            const int f0 = mb0 >= 0 ? P.mateA[j] : -1;
-            const int f1 = mb1 >= 0 ? P.mateA[P.nA + j] : -1;
-            if (f0 >= 0 && bsearch_i32(P.Bj, b0lo, b0hi, __ldg(P.Lb + f0))) ov[0]++;
-            if (f1 >= 0 && bsearch_i32(P.Bj, b1lo, b1hi, __ldg(P.Lb + f1))) ov[1]++;
+        if (e1 >= 0) {
+            wsum[1] += P.w[e1];
+            card[1]++;
+        }
+    }
+    for (int64_t q = tid; q < P.npairs; q += nthr) {
+        const int2 ij = __ldg(P.pairs + q);
+#pragma unroll
+        for (int k = 0; k < 2; k++) {
+            const int ei = P.mateA[k * P.nA + ij.x];
+            const int ej = P.mateA[k * P.nA + ij.y];
+            if (ei < 0 || ej < 0) continue;
+            const int mi = __ldg(P.Lb + ei), mj = __ldg(P.Lb + ej); // M(i), M(j) in V_B
+            if (bsearch_i32(P.Bj, P.Bp[mi], P.Bp[mi + 1], mj)) ov[k]++;
         }
     }
     for (int k = 0; k < 2; k++) {
@@ -633,7 +628,7 @@ cualign_status match_setup(cualign_bp *h)
     int64_t want = ((int64_t)2 * (nA + nB) + 255) / 256;
     int64_t cap = (int64_t)occ * h->num_sms;
     h->match_grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
-    h->eval_grid = grid_for((int64_t)nA * 4, 256, h->num_sms * 8);
+    h->eval_grid = grid_for(h->nApairs > (int64_t)nA ? h->nApairs : (int64_t)nA, 256, h->num_sms * 8);
     CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * h->eval_grid));
     return CUALIGN_OK;
 }
@@ -651,10 +646,10 @@ cualign_status match_round(cualign_bp *h)
     E.Lb = h->L.Lb;
     E.w = h->L.w;
     E.mateA = h->mateA;
-    E.Ap = h->Ap;
-    E.Aj = h->Aj;
     E.Bp = h->Bp;
     E.Bj = h->Bj;
+    E.pairs = h->Apairs;
+    E.npairs = h->nApairs;
     E.partial_w = h->partial_w;
     E.rd = h->rd;
     // overlap / card accumulators (the rest of rd persists: best)
