@@ -127,8 +127,29 @@ static cualign_status capture_step(cualign_bp *h, int timed, int what)
     cualign_status st = CUALIGN_OK;
     cudaError_t e = cudaStreamBeginCapture(h->gstream, cudaStreamCaptureModeThreadLocal);
     if (e == cudaSuccess) {
-        if (what & CUALIGN_RUN_ITERATE) st = bp_iterate(h, 1);
-        if (st == CUALIGN_OK && (what & CUALIGN_RUN_ROUND)) st = match_round(h);
+        if (what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND)) {
+            // the rounding of iteration p reads only y^c, z^c (or y^p, z^p),
+            // w and L -- final after the first half -- and the square pass
+            // touches none of them: fork the rounding onto a side branch so
+            // the latency-bound matching overlaps the bandwidth-bound pass.
+            st = bp_iterate_front(h);
+            if (st == CUALIGN_OK && cudaEventRecord(h->fork_ev[0], h->gstream) != cudaSuccess) st = CUALIGN_ECUDA;
+            if (st == CUALIGN_OK && cudaStreamWaitEvent(h->gstream2, h->fork_ev[0], 0) != cudaSuccess)
+                st = CUALIGN_ECUDA;
+            if (st == CUALIGN_OK) {
+                h->stream = h->gstream2;
+                st = match_round(h);
+                h->stream = h->gstream;
+            }
+            if (st == CUALIGN_OK) st = bp_iterate_back(h);
+            if (st == CUALIGN_OK && cudaEventRecord(h->fork_ev[1], h->gstream2) != cudaSuccess) st = CUALIGN_ECUDA;
+            if (st == CUALIGN_OK && cudaStreamWaitEvent(h->gstream, h->fork_ev[1], 0) != cudaSuccess)
+                st = CUALIGN_ECUDA;
+            if (st == CUALIGN_OK) h->p += 1;
+        } else {
+            if (what & CUALIGN_RUN_ITERATE) st = bp_iterate(h, 1);
+            if (st == CUALIGN_OK && (what & CUALIGN_RUN_ROUND)) st = match_round(h);
+        }
         cudaGraph_t g = nullptr;
         cudaError_t e2 = cudaStreamEndCapture(h->gstream, &g);
         if (st == CUALIGN_OK && e2 != cudaSuccess) {
@@ -251,8 +272,11 @@ static cualign_status open_handle(const cualign_params *params, cualign_bp **out
         h->own_stream = true;
     }
     CA_CUDA(cudaStreamCreateWithFlags(&h->gstream, cudaStreamNonBlocking));
-    CA_CUDA(cudaEventCreateWithFlags(&h->sync_ev[0], cudaEventDisableTiming));
-    CA_CUDA(cudaEventCreateWithFlags(&h->sync_ev[1], cudaEventDisableTiming));
+    CA_CUDA(cudaStreamCreateWithFlags(&h->gstream2, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; i++) {
+        CA_CUDA(cudaEventCreateWithFlags(&h->sync_ev[i], cudaEventDisableTiming));
+        CA_CUDA(cudaEventCreateWithFlags(&h->fork_ev[i], cudaEventDisableTiming));
+    }
     return CUALIGN_OK;
 }
 
@@ -267,9 +291,12 @@ static void close_handle(cualign_bp *h)
     for (auto e : h->event_pool) cudaEventDestroy(e);
     for (auto e : h->sync_ev)
         if (e) cudaEventDestroy(e);
+    for (auto e : h->fork_ev)
+        if (e) cudaEventDestroy(e);
     dfree_all(h);
     if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
     if (h->gstream) cudaStreamDestroy(h->gstream);
+    if (h->gstream2) cudaStreamDestroy(h->gstream2);
     (void)cudaGetLastError();
     delete h;
 }

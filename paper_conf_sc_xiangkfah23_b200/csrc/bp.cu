@@ -177,7 +177,7 @@ template <int EPT, bool EXACT, bool LITERAL>
 __global__ void __launch_bounds__(256) k_edge(EdgeArgs R)
 {
     const int64_t base = (int64_t)blockIdx.x * blockDim.x * EPT + threadIdx.x;
-    const double2 ghp = R.gh[*R.p_dev + 1];
+    const double2 ghp = R.gh[*R.p_dev];
     const double g = ghp.x, hh = ghp.y;
     int64_t e[EPT];
     int a[EPT], b[EPT];
@@ -252,7 +252,7 @@ k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_v
     // SQ_U, HINTS: template parameters (variants measured in profiles/)
     double g = 0.0, hh = 1.0;
     if (UPDATE) {
-        const double2 ghp = gh[*p_dev + 1];
+        const double2 ghp = gh[*p_dev];
         g = ghp.x;
         hh = ghp.y;
     }
@@ -476,42 +476,58 @@ cualign_status bp_fsum(cualign_bp *h)
     return launch_square(h, false);
 }
 
-cualign_status bp_iterate(cualign_bp *h, int32_t n)
+// First half of an iteration: the device counter advances to this iteration
+// p (kernels read gh[p]), then lines 9-12 and 14-15 on the vectors (top-2,
+// k_edge).  y^c, z^c of iteration p are final after this half, so the
+// rounding of p may run concurrently with the second half.
+cualign_status bp_iterate_front(cualign_bp *h)
 {
     const bool exact = (h->flags & CUALIGN_FLAG_EXACT) != 0;
     const bool literal = (h->flags & CUALIGN_FLAG_OTHERMAX_LITERAL) != 0;
     const int64_t m = h->L.m;
-    if (!h->capturing) CA_TRY(ensure_gh(h, h->p + n));
-    for (int32_t k = 0; k < n; k++) {
-        const int32_t p = h->p + 1;
-        if (m > 0) {
-            {
-                KScope ks(h, CUALIGN_K_TOP2);
-                Top2Args T{(int64_t)h->L.nA, h->nchunks, h->L.Arow, h->chunk_b, h->Bcp, h->L.Bptr, h->L.Bedge,
-                           h->yp, h->zp, h->Atop, h->Btop, h->Bct, h->Bcnt};
-                k_top2<<<grid_for((T.nA + T.nchunks) * TG, 256, 1 << 30), 256, 0, h->stream>>>(T);
-                CA_CUDA(cudaGetLastError());
-            }
-            {
-                KScope ks(h, CUALIGN_K_EDGE);
-                EdgeArgs R{m, h->L.La, h->L.Lb, h->L.w, h->alpha, h->fp_inv, h->gh_dev, h->p_dev, h->tacc, h->texact,
-                           h->Atop, h->Btop, h->yp, h->zp, h->yc, h->zc, h->d, h->u};
-                constexpr int EPT = 4;
-                const int grid = grid_for((m + EPT - 1) / EPT, 256, 1 << 30);
-                if (exact && literal) k_edge<EPT, true, true><<<grid, 256, 0, h->stream>>>(R);
-                else if (exact) k_edge<EPT, true, false><<<grid, 256, 0, h->stream>>>(R);
-                else if (literal) k_edge<EPT, false, true><<<grid, 256, 0, h->stream>>>(R);
-                else k_edge<EPT, false, false><<<grid, 256, 0, h->stream>>>(R);
-                CA_CUDA(cudaGetLastError());
-            }
-            CA_TRY(launch_square(h, true));
-        }
+    {
+        KScope ks(h, CUALIGN_K_OTHER);
+        k_advance<<<1, 1, 0, h->stream>>>(h->p_dev);
+        CA_CUDA(cudaGetLastError());
+    }
+    if (m > 0) {
         {
-            KScope ks(h, CUALIGN_K_OTHER);
-            k_advance<<<1, 1, 0, h->stream>>>(h->p_dev);
+            KScope ks(h, CUALIGN_K_TOP2);
+            Top2Args T{(int64_t)h->L.nA, h->nchunks, h->L.Arow, h->chunk_b, h->Bcp, h->L.Bptr, h->L.Bedge,
+                       h->yp, h->zp, h->Atop, h->Btop, h->Bct, h->Bcnt};
+            k_top2<<<grid_for((T.nA + T.nchunks) * TG, 256, 1 << 30), 256, 0, h->stream>>>(T);
             CA_CUDA(cudaGetLastError());
         }
-        h->p = p;
+        {
+            KScope ks(h, CUALIGN_K_EDGE);
+            EdgeArgs R{m, h->L.La, h->L.Lb, h->L.w, h->alpha, h->fp_inv, h->gh_dev, h->p_dev, h->tacc, h->texact,
+                       h->Atop, h->Btop, h->yp, h->zp, h->yc, h->zc, h->d, h->u};
+            constexpr int EPT = 4;
+            const int grid = grid_for((m + EPT - 1) / EPT, 256, 1 << 30);
+            if (exact && literal) k_edge<EPT, true, true><<<grid, 256, 0, h->stream>>>(R);
+            else if (exact) k_edge<EPT, true, false><<<grid, 256, 0, h->stream>>>(R);
+            else if (literal) k_edge<EPT, false, true><<<grid, 256, 0, h->stream>>>(R);
+            else k_edge<EPT, false, false><<<grid, 256, 0, h->stream>>>(R);
+            CA_CUDA(cudaGetLastError());
+        }
+    }
+    return CUALIGN_OK;
+}
+
+// Second half: lines 9, 13, 16 on the S values (the square pass).
+cualign_status bp_iterate_back(cualign_bp *h)
+{
+    if (h->L.m > 0) CA_TRY(launch_square(h, true));
+    return CUALIGN_OK;
+}
+
+cualign_status bp_iterate(cualign_bp *h, int32_t n)
+{
+    if (!h->capturing) CA_TRY(ensure_gh(h, h->p + n));
+    for (int32_t k = 0; k < n; k++) {
+        CA_TRY(bp_iterate_front(h));
+        CA_TRY(bp_iterate_back(h));
+        h->p += 1;
     }
     return CUALIGN_OK;
 }

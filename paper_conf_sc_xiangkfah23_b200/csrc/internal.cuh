@@ -111,7 +111,9 @@ struct cualign_bp {
 
     // CUDA graphs of one step (iterate(1) [+ round]); [0] = no round, [1] = with round
     cudaStream_t gstream = nullptr;     // capture / replay stream (never the legacy stream)
+    cudaStream_t gstream2 = nullptr;    // capture side branch: rounding overlapped with the square pass
     cudaEvent_t sync_ev[2] = {nullptr, nullptr};
+    cudaEvent_t fork_ev[2] = {nullptr, nullptr};
     bool capturing = false;
     int capture_what = 0;
     cudaGraphExec_t graph[2][4] = {};                       // [timed][what = CUALIGN_RUN_* bits]
@@ -186,6 +188,8 @@ cualign_status ensure_gh(cualign_bp *h, int64_t pmax); // gamma^p table covers p
 cualign_status bp_setup(cualign_bp *h);                // B chunks
 cualign_status bp_fsum(cualign_bp *h);                 // t <- sum_f F(S^p) (init / set_state)
 cualign_status bp_iterate(cualign_bp *h, int32_t n);   // Alg. 2 l.9-16, n times
+cualign_status bp_iterate_front(cualign_bp *h);        // advance p, top-2, k_edge
+cualign_status bp_iterate_back(cualign_bp *h);         // square pass
 cualign_status bp_scatter_Sp(cualign_bp *h, double *Sfull_dev);        // squares -> CSR
 cualign_status bp_gather_Sp(cualign_bp *h, const double *Sfull_dev);   // CSR -> squares
 
