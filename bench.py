@@ -305,7 +305,7 @@ def main():
     cls_n = pst["class_launches"]
     sq_ms = cls_ms["square"] / max(cls_n["square"], 1)
     bp_ms = (cls_ms["top2"] + cls_ms["edge"] + cls_ms["square"] + cls_ms["rowsum"] + cls_ms["other"]) / prof_steps
-    round_ms = cls_ms["match"] / prof_steps
+    round_ms = (cls_ms["match"] + cls_ms["eval"] + cls_ms["matchaux"]) / prof_steps
     peak, peak_src = read_peaks()
     sq_bytes = BYTES_PER_NZ * s                    # algorithmic bytes of one square-pass launch
     sq_gbs = sq_bytes / (sq_ms * 1e-3) / 1e9 if sq_ms > 0 else 0.0

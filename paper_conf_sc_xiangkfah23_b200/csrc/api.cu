@@ -272,7 +272,13 @@ static cualign_status open_handle(const cualign_params *params, cualign_bp **out
         h->own_stream = true;
     }
     CA_CUDA(cudaStreamCreateWithFlags(&h->gstream, cudaStreamNonBlocking));
-    CA_CUDA(cudaStreamCreateWithFlags(&h->gstream2, cudaStreamNonBlocking));
+    {
+        // the rounding branch gets the higher priority: its latency-bound
+        // kernels are scheduled first when square-pass CTAs retire
+        int lo = 0, hi = 0;
+        CA_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+        CA_CUDA(cudaStreamCreateWithPriority(&h->gstream2, cudaStreamNonBlocking, hi));
+    }
     for (int i = 0; i < 2; i++) {
         CA_CUDA(cudaEventCreateWithFlags(&h->sync_ev[i], cudaEventDisableTiming));
         CA_CUDA(cudaEventCreateWithFlags(&h->fork_ev[i], cudaEventDisableTiming));

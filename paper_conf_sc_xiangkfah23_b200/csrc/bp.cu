@@ -377,7 +377,11 @@ template <bool UPDATE, bool EXACT, int SQ_U, bool HINTS, bool NOATOM = false>
 void square_launch(cualign_bp *h)
 {
     auto fn = k_square<UPDATE, EXACT, SQ_U, HINTS, NOATOM>;
-    const int grid = one_wave_grid(h, (const void *)fn, 256, h->nsq, 256 * SQ_U);
+    int grid = one_wave_grid(h, (const void *)fn, 256, h->nsq, 256 * SQ_U);
+    // leave room for the concurrent rounding branch (graph step): a fraction
+    // of the resident CTAs still saturates HBM
+    static const double frac = getenv("CUALIGN_SQ_FRAC") ? atof(getenv("CUALIGN_SQ_FRAC")) : 1.0;
+    if (frac > 0.0 && frac < 1.0) grid = (int)(grid * frac) > 0 ? (int)(grid * frac) : 1;
     fn<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, h->gh_dev, h->p_dev, h->fp_scale,
                                     h->tacc, h->sq_pos, h->Ffull);
 }
