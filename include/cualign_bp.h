@@ -96,9 +96,21 @@ typedef struct {
     int32_t device;   /* CUDA device ordinal */
     void *stream;     /* cudaStream_t to run on (e.g. torch.cuda.current_stream());
                          NULL = the handle creates its own non-blocking stream */
-    int32_t rank;     /* reserved for sharded handles; must be 0 */
-    int32_t world;    /* reserved for sharded handles; must be 1 (or 0 = 1) */
-    const void *nccl_unique_id; /* reserved; must be NULL */
+    /* Sharding by contiguous A-vertex blocks (multi-GPU is the
+     * paper's future work):
+     *   world <= 1: one GPU, rank = 0, nccl_unique_id = NULL;
+     *   world > 1, nccl_unique_id != NULL: this process is shard `rank` of
+     *     `world` (one GPU each); init / iterate / round / run are collective
+     *     over the ranks; the id comes from cualign_nccl_unique_id() on one
+     *     rank, broadcast by the caller (e.g. torch.distributed);
+     *   world > 1, nccl_unique_id == NULL, rank = -1: `world` virtual shards
+     *     in this handle on one device, exchanging through device copies --
+     *     the sharded path for single-GPU testing.
+     * Results of a sharded run are bitwise those of world = 1.  Not with
+     * CUALIGN_FLAG_EXACT. */
+    int32_t rank;
+    int32_t world;
+    const void *nccl_unique_id; /* 128-byte ncclUniqueId or NULL */
 } cualign_params;
 
 /* Result of one rounding step (Alg. 2 l.17-24). */
@@ -127,6 +139,9 @@ typedef struct {
     int32_t p;          /* iterations done */
     int32_t fixed_point_bits; /* fraction bits of the fast-mode F-sum accumulator */
     int64_t device_bytes;     /* device memory held by the handle */
+    int32_t rank, world;      /* shard (rank -1 for a virtual-shard handle) */
+    int64_t edge_begin, edge_end; /* owned canonical edge ids [begin, end) */
+    int64_t squares_local;    /* squares stored by this shard */
 } cualign_sizes;
 
 /* Diagnostics: per-kernel-class event timing (needs CUALIGN_FLAG_TIMING) and
@@ -222,6 +237,9 @@ cualign_status cualign_bp_get_stats(cualign_bp *h, cualign_stats *stats, int32_t
 cualign_status cualign_match(const cualign_edges *L, int32_t n_a, int32_t n_b, const double *x,
                              const cualign_params *params, int32_t *mate_a, int32_t *mate_b,
                              int32_t *rounds_out);
+
+/* NCCL unique id for a sharded init (write len >= 128 bytes into id). */
+cualign_status cualign_nccl_unique_id(void *id, int32_t len);
 
 /* Message of the last failing call on this thread ("" if none). */
 const char *cualign_last_error(void);

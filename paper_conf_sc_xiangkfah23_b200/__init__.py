@@ -4,7 +4,7 @@ The compute path is libcualign_bp.so (CUDA, sm_100a; C ABI in
 include/cualign_bp.h).  This package is the thin Python binding over it plus
 the end-to-end `align` helper and the sharded (multi-GPU) driver.
 """
-from ._lib import (CuAlignBP, CuAlignError, match, load_library, version,
+from ._lib import (CuAlignBP, CuAlignError, match, load_library, version, nccl_unique_id,
                    FLAG_DEVICE_PTRS, FLAG_EXACT, FLAG_OTHERMAX_LITERAL, FLAG_ROUND_DAMPED,
                    FLAG_TIMING, FLAG_MATCH_ROUNDS, EXPORTED, LIB_PATH, KERNEL_CLASS_NAMES)
 
@@ -21,6 +21,6 @@ def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=
     return mate, info, infos
 
 
-__all__ = ["CuAlignBP", "CuAlignError", "match", "align", "load_library", "version",
+__all__ = ["CuAlignBP", "CuAlignError", "match", "align", "load_library", "version", "nccl_unique_id",
            "FLAG_DEVICE_PTRS", "FLAG_EXACT", "FLAG_OTHERMAX_LITERAL", "FLAG_ROUND_DAMPED",
            "FLAG_TIMING", "FLAG_MATCH_ROUNDS", "EXPORTED", "LIB_PATH", "KERNEL_CLASS_NAMES"]

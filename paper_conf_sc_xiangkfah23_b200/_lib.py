@@ -32,7 +32,7 @@ EXPORTED = ["cualign_bp_init", "cualign_bp_iterate", "cualign_bp_round", "cualig
             "cualign_bp_set_timing", "cualign_bp_get_best",
             "cualign_bp_free", "cualign_bp_get_sizes", "cualign_bp_get_S", "cualign_bp_get_state",
             "cualign_bp_set_state", "cualign_bp_get_stats", "cualign_match", "cualign_last_error",
-            "cualign_version"]
+            "cualign_version", "cualign_nccl_unique_id"]
 
 
 class CuAlignError(RuntimeError):
@@ -74,7 +74,9 @@ class Sizes_t(ctypes.Structure):
     _fields_ = [("n_a", ctypes.c_int32), ("n_b", ctypes.c_int32), ("m", ctypes.c_int64),
                 ("s", ctypes.c_int64), ("squares", ctypes.c_int64), ("max_row", ctypes.c_int64),
                 ("p", ctypes.c_int32), ("fixed_point_bits", ctypes.c_int32),
-                ("device_bytes", ctypes.c_int64)]
+                ("device_bytes", ctypes.c_int64), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("edge_begin", ctypes.c_int64), ("edge_end", ctypes.c_int64),
+                ("squares_local", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -135,6 +137,8 @@ def load_library():
     lib.cualign_last_error.argtypes = []
     lib.cualign_version.restype = ctypes.c_char_p
     lib.cualign_version.argtypes = []
+    lib.cualign_nccl_unique_id.restype = I32
+    lib.cualign_nccl_unique_id.argtypes = [P, I32]
     _lib = lib
     return lib
 
@@ -188,7 +192,10 @@ def _stream_ptr(stream):
 class CuAlignBP:
     """One alignment problem resident on a GPU (Alg. 2 state + S)."""
 
-    def __init__(self, A, B, L, alpha=1.0, beta=2.0, gamma=0.99, flags=0, device=0, stream=None):
+    def __init__(self, A, B, L, alpha=1.0, beta=2.0, gamma=0.99, flags=0, device=0, stream=None,
+                 world=1, rank=0, nccl_id=None):
+        """world > 1 with nccl_id (bytes): this process is shard `rank`;
+        world > 1 without nccl_id: `world` virtual shards in one handle."""
         lib = load_library()
         Ap, dA = _prep(A.rowptr, np.int64, "int64")
         Aj, _ = _prep(A.col, np.int32, "int32")
@@ -208,8 +215,13 @@ class CuAlignBP:
         ga = Graph_t(self.n_a, _ptr(Ap), _ptr(Aj))
         gb = Graph_t(self.n_b, _ptr(Bp), _ptr(Bj))
         el = Edges_t(self.m, _ptr(La), _ptr(Lb), _ptr(w))
+        self.world = int(world)
+        if self.world > 1 and nccl_id is None:
+            rank = -1
+        self._nccl_id = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
         prm = Params_t(float(alpha), float(beta), float(gamma), int(flags), int(device),
-                       _stream_ptr(stream), 0, 1, None)
+                       _stream_ptr(stream), int(rank), self.world,
+                       ctypes.cast(self._nccl_id, ctypes.c_void_p) if self._nccl_id is not None else None)
         h = ctypes.c_void_p()
         _check(lib.cualign_bp_init(ctypes.byref(ga), ctypes.byref(gb), ctypes.byref(el),
                                    ctypes.byref(prm), ctypes.byref(h)))
@@ -326,3 +338,10 @@ def match(L, n_a, n_b, x, device=0, flags=0):
 
 def version():
     return load_library().cualign_version().decode()
+
+
+def nccl_unique_id() -> bytes:
+    """128-byte NCCL unique id for a sharded init (create on one rank, broadcast)."""
+    buf = ctypes.create_string_buffer(128)
+    _check(load_library().cualign_nccl_unique_id(buf, 128))
+    return buf.raw

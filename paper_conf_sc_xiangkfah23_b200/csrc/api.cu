@@ -245,10 +245,24 @@ static cualign_status check_params(const cualign_params *p)
         set_error("gamma must be in (0, 1], got %g", p->gamma);
         return CUALIGN_EINVAL;
     }
-    if (p->rank != 0 || (p->world != 0 && p->world != 1) || p->nccl_unique_id != nullptr) {
-        set_error("sharded handles are not available through this entry point (rank=%d world=%d)", p->rank,
-                  p->world);
+    const int world = p->world <= 0 ? 1 : p->world;
+    if (world == 1 && (p->rank != 0 || p->nccl_unique_id != nullptr)) {
+        set_error("world = 1 needs rank = 0 and no NCCL id (rank=%d)", p->rank);
         return CUALIGN_EINVAL;
+    }
+    if (world > 1) {
+        if (p->nccl_unique_id && (p->rank < 0 || p->rank >= world)) {
+            set_error("NCCL shard: rank %d outside [0, %d)", p->rank, world);
+            return CUALIGN_EINVAL;
+        }
+        if (!p->nccl_unique_id && p->rank != -1) {
+            set_error("virtual shards (no NCCL id) need rank = -1 (got %d)", p->rank);
+            return CUALIGN_EINVAL;
+        }
+        if (p->flags & CUALIGN_FLAG_EXACT) {
+            set_error("CUALIGN_FLAG_EXACT is single-GPU only");
+            return CUALIGN_EINVAL;
+        }
     }
     return CUALIGN_OK;
 }
@@ -262,6 +276,8 @@ static cualign_status open_handle(const cualign_params *params, cualign_bp **out
     h->flags = params->flags;
     h->dev = params->device;
     h->timing = (params->flags & CUALIGN_FLAG_TIMING) != 0;
+    h->world = params->world <= 0 ? 1 : params->world;
+    h->rank = params->rank < 0 ? 0 : params->rank;
     *out = h;
     CA_CUDA(cudaSetDevice(h->dev));
     CA_CUDA(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->dev));
@@ -290,6 +306,9 @@ static void close_handle(cualign_bp *h)
 {
     if (!h) return;
     cudaSetDevice(h->dev);
+    for (cualign_bp *s : h->vshards) close_handle(s);
+    h->vshards.clear();
+    nccl_free_comm(h);
     if (h->stream) cudaStreamSynchronize(h->stream);
     if (h->gstream) cudaStreamSynchronize(h->gstream);
     resolve_events(h);
@@ -328,6 +347,9 @@ static cualign_status alloc_state(cualign_bp *h)
     return CUALIGN_OK;
 }
 
+// the handle that holds the replicated rounding state (shard 0 of a group)
+static cualign_bp *primary(cualign_bp *h) { return h->vshards.empty() ? h : h->vshards[0]; }
+
 #define API_ENTER() clear_error()
 #define CHECK_H()                                   \
     do {                                            \
@@ -365,10 +387,39 @@ cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B, c
     }
     cualign_bp *h = nullptr;
     cualign_status st = open_handle(params, &h);
-    if (st == CUALIGN_OK) st = build_problem(h, A, B, L);
-    if (st == CUALIGN_OK) st = alloc_state(h);
-    if (st == CUALIGN_OK) st = match_setup(h);
-    if (st == CUALIGN_OK) st = bp_fsum(h); // F(S^p = 0) row sums for iteration 1
+    const bool virt = h && h->world > 1 && params->nccl_unique_id == nullptr;
+    if (virt) {
+        // in-process virtual shards (loopback exchanges) on the handle's device
+        // and stream: the sharded path, testable on one GPU
+        for (int r = 0; st == CUALIGN_OK && r < h->world; r++) {
+            cualign_params sp = *params;
+            sp.rank = r;
+            sp.stream = h->stream;
+            sp.nccl_unique_id = nullptr;
+            cualign_bp *s = nullptr;
+            st = open_handle(&sp, &s);
+            if (s) h->vshards.push_back(s);
+            if (st == CUALIGN_OK) st = build_problem(s, A, B, L);
+            if (st == CUALIGN_OK) st = alloc_state(s);
+            if (st == CUALIGN_OK) st = match_setup(s);
+        }
+        if (st == CUALIGN_OK) {
+            cualign_bp *s0 = h->vshards[0];
+            h->L = s0->L; // sizes only (the group owns no arrays itself)
+            h->s_total = s0->s_total;
+            h->nsq_total = s0->nsq_total;
+            h->max_row = s0->max_row;
+            h->fp_bits = s0->fp_bits;
+            h->bounds = s0->bounds;
+            st = shard_fsum(h); // F(S^p = 0) row sums for iteration 1
+        }
+    } else {
+        if (st == CUALIGN_OK && h->world > 1) st = nccl_init_comm(h, params->nccl_unique_id);
+        if (st == CUALIGN_OK) st = build_problem(h, A, B, L);
+        if (st == CUALIGN_OK) st = alloc_state(h);
+        if (st == CUALIGN_OK) st = match_setup(h);
+        if (st == CUALIGN_OK) st = h->world > 1 ? shard_fsum(h) : bp_fsum(h); // F(S^p = 0) sums for iteration 1
+    }
     if (st == CUALIGN_OK) {
         cudaError_t e = cudaStreamSynchronize(h->stream);
         if (e != cudaSuccess) {
@@ -394,7 +445,7 @@ cualign_status cualign_bp_iterate(cualign_bp *h, int32_t n_steps)
         set_error("n_steps < 0");
         return CUALIGN_EINVAL;
     }
-    return bp_iterate(h, n_steps);
+    return h->world > 1 ? shard_iterate(h, n_steps) : bp_iterate(h, n_steps);
 }
 
 cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t what)
@@ -410,6 +461,14 @@ cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t what)
         set_error("run: what must be CUALIGN_RUN_ITERATE, CUALIGN_RUN_ROUND or both");
         return CUALIGN_EINVAL;
     }
+    if (h->world > 1) {
+        // sharded: eager per-step launches (the exchanges sit between kernels)
+        for (int32_t k = 0; k < n_steps; k++) {
+            if (what & CUALIGN_RUN_ITERATE) CA_TRY(shard_iterate(h, 1));
+            if (what & CUALIGN_RUN_ROUND) CA_TRY(shard_round(h));
+        }
+        return CUALIGN_OK;
+    }
     return run_graph(h, n_steps, what);
 }
 
@@ -418,6 +477,7 @@ cualign_status cualign_bp_set_timing(cualign_bp *h, int32_t on)
     API_ENTER();
     CHECK_H();
     h->timing = on != 0;
+    for (cualign_bp *s : h->vshards) s->timing = on != 0;
     return CUALIGN_OK;
 }
 
@@ -425,13 +485,14 @@ cualign_status cualign_bp_round(cualign_bp *h, cualign_round_info *info)
 {
     API_ENTER();
     CHECK_H();
-    CA_TRY(match_round(h));
+    CA_TRY(h->world > 1 ? shard_round(h) : match_round(h));
     h->have_info = true;
     if (info) {
-        CA_CUDA(cudaMemcpyAsync(&h->last_info, &h->rd->info, sizeof(cualign_round_info), cudaMemcpyDeviceToHost,
-                                h->stream));
-        CA_CUDA(cudaStreamSynchronize(h->stream));
-        *info = h->last_info;
+        cualign_bp *q = primary(h);
+        CA_CUDA(cudaMemcpyAsync(&q->last_info, &q->rd->info, sizeof(cualign_round_info), cudaMemcpyDeviceToHost,
+                                q->stream));
+        CA_CUDA(cudaStreamSynchronize(q->stream));
+        *info = q->last_info;
     }
     return CUALIGN_OK;
 }
@@ -440,6 +501,7 @@ cualign_status cualign_bp_get_best(cualign_bp *h, int32_t *mate_a, cualign_round
 {
     API_ENTER();
     CHECK_H();
+    h = primary(h); // rounding is replicated on every shard
     if (mate_a && h->L.nA)
         CA_CUDA(cudaMemcpyAsync(mate_a, h->best_mate, sizeof(int32_t) * (size_t)h->L.nA, cudaMemcpyDeviceToHost,
                                 h->stream));
@@ -465,15 +527,22 @@ cualign_status cualign_bp_get_sizes(cualign_bp *h, cualign_sizes *sz)
         return CUALIGN_EINVAL;
     }
     CA_CUDA(cudaStreamSynchronize(h->stream));
-    sz->n_a = h->L.nA;
-    sz->n_b = h->L.nB;
-    sz->m = h->L.m;
-    sz->s = h->s;
-    sz->squares = h->nsq;
-    sz->max_row = h->max_row;
+    cualign_bp *q = primary(h);
+    sz->n_a = q->L.nA;
+    sz->n_b = q->L.nB;
+    sz->m = q->L.m;
+    sz->s = q->s_total;
+    sz->squares = q->nsq_total;
+    sz->max_row = q->max_row;
     sz->p = h->p;
-    sz->fixed_point_bits = (h->flags & CUALIGN_FLAG_EXACT) ? 0 : h->fp_bits;
+    sz->fixed_point_bits = (q->flags & CUALIGN_FLAG_EXACT) ? 0 : q->fp_bits;
     sz->device_bytes = h->device_bytes;
+    for (cualign_bp *s : h->vshards) sz->device_bytes += s->device_bytes;
+    sz->rank = h->vshards.empty() ? h->rank : -1;
+    sz->world = h->world;
+    sz->edge_begin = h->vshards.empty() ? h->e0 : 0;
+    sz->edge_end = h->vshards.empty() ? h->e1 : q->L.m;
+    sz->squares_local = h->vshards.empty() ? h->nsq : q->nsq_total;
     return CUALIGN_OK;
 }
 
@@ -481,6 +550,27 @@ cualign_status cualign_bp_get_S(cualign_bp *h, int64_t *rowptr, int32_t *col, in
 {
     API_ENTER();
     CHECK_H();
+    if (!h->vshards.empty()) {
+        // virtual shards own consecutive rows: concatenate their CSRs
+        int64_t off = 0;
+        for (cualign_bp *s : h->vshards) {
+            const int64_t ml = s->e1 - s->e0;
+            if (rowptr) {
+                std::vector<int64_t> rp((size_t)ml + 1);
+                CA_CUDA(cudaMemcpy(rp.data(), s->Srp, sizeof(int64_t) * (size_t)(ml + 1), cudaMemcpyDeviceToHost));
+                for (int64_t i = 0; i <= ml; i++) rowptr[s->e0 + i] = rp[(size_t)i] + off;
+            }
+            if (col && s->s)
+                CA_CUDA(cudaMemcpy(col + off, s->Scol, sizeof(int32_t) * (size_t)s->s, cudaMemcpyDeviceToHost));
+            off += s->s;
+        }
+        if (s_out) *s_out = off;
+        return CUALIGN_OK;
+    }
+    if (h->world > 1) {
+        set_error("get_S: a process shard holds only its own rows; use virtual shards or world = 1");
+        return CUALIGN_ESTATE;
+    }
     if (rowptr)
         CA_CUDA(cudaMemcpyAsync(rowptr, h->Srp, sizeof(int64_t) * ((size_t)h->L.m + 1), cudaMemcpyDeviceToHost,
                                 h->stream));
@@ -496,6 +586,30 @@ cualign_status cualign_bp_get_state(cualign_bp *h, double *yc, double *zc, doubl
 {
     API_ENTER();
     CHECK_H();
+    if (h->world > 1) {
+        if (Sp) {
+            set_error("get_state: S^p of a sharded handle is distributed (pass Sp = NULL)");
+            return CUALIGN_ESTATE;
+        }
+        // y^c, z^c are all-gathered every iteration; y^p, z^p, d are valid on
+        // the owners' slices: assemble them (virtual shards) or return this
+        // process shard's arrays (owned slice valid)
+        std::vector<cualign_bp *> S = h->vshards.empty() ? std::vector<cualign_bp *>{h} : h->vshards;
+        cualign_bp *q = S[0];
+        const size_t mb = sizeof(double) * (size_t)q->L.m;
+        if (yc && mb) CA_CUDA(cudaMemcpy(yc, q->yc, mb, cudaMemcpyDeviceToHost));
+        if (zc && mb) CA_CUDA(cudaMemcpy(zc, q->zc, mb, cudaMemcpyDeviceToHost));
+        for (cualign_bp *s : S) {
+            const int64_t a = h->vshards.empty() ? 0 : s->e0, b = h->vshards.empty() ? s->L.m : s->e1;
+            const size_t nb = sizeof(double) * (size_t)(b - a);
+            if (!nb) continue;
+            if (yp) CA_CUDA(cudaMemcpy(yp + a, s->yp + a, nb, cudaMemcpyDeviceToHost));
+            if (zp) CA_CUDA(cudaMemcpy(zp + a, s->zp + a, nb, cudaMemcpyDeviceToHost));
+            if (d) CA_CUDA(cudaMemcpy(d + a, s->d + a, nb, cudaMemcpyDeviceToHost));
+        }
+        if (p) *p = h->p;
+        return CUALIGN_OK;
+    }
     const size_t mb = sizeof(double) * (size_t)h->L.m;
     struct {
         double *dst;
@@ -528,6 +642,10 @@ cualign_status cualign_bp_set_state(cualign_bp *h, const double *yp, const doubl
 {
     API_ENTER();
     CHECK_H();
+    if (h->world > 1) {
+        set_error("set_state is single-GPU only");
+        return CUALIGN_ESTATE;
+    }
     if (!yp || !zp || (!Sp && h->s) || p < 0) {
         set_error("set_state: NULL buffer or p < 0");
         return CUALIGN_EINVAL;
@@ -564,22 +682,43 @@ cualign_status cualign_bp_get_stats(cualign_bp *h, cualign_stats *stats, int32_t
     API_ENTER();
     CHECK_H();
     CA_CUDA(cudaStreamSynchronize(h->stream));
-    resolve_events(h);
+    std::vector<cualign_bp *> S{h};
+    for (cualign_bp *s : h->vshards) S.push_back(s);
     if (stats) {
-        stats->launches = h->launches;
+        stats->launches = 0;
         for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
-            stats->class_launches[c] = h->class_launches[c];
-            stats->class_ms[c] = h->class_ms[c];
+            stats->class_launches[c] = 0;
+            stats->class_ms[c] = 0.0;
         }
     }
-    if (reset) {
-        h->launches = 0;
-        for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
-            h->class_launches[c] = 0;
-            h->class_ms[c] = 0.0;
+    for (cualign_bp *s : S) {
+        resolve_events(s);
+        if (stats) {
+            stats->launches += s->launches;
+            for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
+                stats->class_launches[c] += s->class_launches[c];
+                stats->class_ms[c] += s->class_ms[c];
+            }
+        }
+        if (reset) {
+            s->launches = 0;
+            for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
+                s->class_launches[c] = 0;
+                s->class_ms[c] = 0.0;
+            }
         }
     }
     return CUALIGN_OK;
+}
+
+cualign_status cualign_nccl_unique_id(void *id, int32_t len)
+{
+    API_ENTER();
+    if (!id) {
+        set_error("id is NULL");
+        return CUALIGN_EINVAL;
+    }
+    return nccl_unique_id(id, len);
 }
 
 cualign_status cualign_match(const cualign_edges *L, int32_t n_a, int32_t n_b, const double *x,

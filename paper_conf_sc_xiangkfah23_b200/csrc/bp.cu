@@ -95,7 +95,8 @@ constexpr int TG = 8;                 // lanes per tile in k_top2
 constexpr int TB_U = B_CHUNK / TG;    // gathers per lane per chunk
 
 struct Top2Args {
-    int64_t nA, nchunks;
+    int64_t nA, nchunks;    // A rows to process (a0 .. a0+nA-1), B chunks
+    int64_t a0;
     const int64_t *Arow;
     const int32_t *chunk_b;
     const int64_t *Bcp, *Bptr;
@@ -115,10 +116,11 @@ __global__ void __launch_bounds__(256) k_top2(Top2Args T)
         double m1 = -INFINITY, m2 = -INFINITY;
         if (t < T.nA) {
             // A row: contiguous edges
-            const int64_t lo = T.Arow[t], hi = T.Arow[t + 1];
+            const int64_t a = T.a0 + t;
+            const int64_t lo = T.Arow[a], hi = T.Arow[a + 1];
             for (int64_t e = lo + lane; e < hi; e += TG) top2_push(m1, m2, T.yp[e]);
             tile_top2<TG>(tile, m1, m2);
-            if (lane == 0) T.Atop[t] = make_double2(m1, m2);
+            if (lane == 0) T.Atop[a] = make_double2(m1, m2);
         } else {
             // B chunk: gather z^p through the incidence
             const int64_t c = t - T.nA;
@@ -161,12 +163,12 @@ __global__ void __launch_bounds__(256) k_top2(Top2Args T)
 }
 
 struct EdgeArgs {
-    int64_t m;
+    int64_t e0, e1;      // the edges this handle owns
     const int32_t *La, *Lb;
     const double *w;
     double alpha, fp_inv;
     const double2 *gh;   // gh[p] = (gamma^p, 1 - gamma^p), host-computed (reading Z2)
-    const int *p_dev;    // iterations done; this iteration is p_dev + 1
+    const int *p_dev;    // the current iteration p (advanced at its start)
     unsigned long long *tacc;
     const double *texact;
     const double2 *Atop, *Btop;
@@ -176,7 +178,7 @@ struct EdgeArgs {
 template <int EPT, bool EXACT, bool LITERAL>
 __global__ void __launch_bounds__(256) k_edge(EdgeArgs R)
 {
-    const int64_t base = (int64_t)blockIdx.x * blockDim.x * EPT + threadIdx.x;
+    const int64_t base = R.e0 + (int64_t)blockIdx.x * blockDim.x * EPT + threadIdx.x;
     const double2 ghp = R.gh[*R.p_dev];
     const double g = ghp.x, hh = ghp.y;
     int64_t e[EPT];
@@ -185,7 +187,7 @@ __global__ void __launch_bounds__(256) k_edge(EdgeArgs R)
 #pragma unroll
     for (int j = 0; j < EPT; j++) {
         e[j] = base + (int64_t)j * blockDim.x;
-        if (e[j] < R.m) {
+        if (e[j] < R.e1) {
             a[j] = __ldg(R.La + e[j]);
             b[j] = __ldg(R.Lb + e[j]);
             we[j] = __ldg(R.w + e[j]);
@@ -201,7 +203,7 @@ __global__ void __launch_bounds__(256) k_edge(EdgeArgs R)
     }
 #pragma unroll
     for (int j = 0; j < EPT; j++) {
-        if (e[j] >= R.m) continue;
+        if (e[j] >= R.e1) continue;
         const double2 at = __ldg(R.Atop + a[j]);
         const double2 bt = __ldg(R.Btop + b[j]);
         const double de = R.alpha * we[j] + t[j];          // line 10
@@ -441,6 +443,114 @@ cualign_status ensure_gh(cualign_bp *h, int64_t pmax)
     return CUALIGN_OK;
 }
 
+namespace {
+
+__global__ void k_iota_from(int64_t n, int64_t first, int32_t *__restrict__ x)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        x[i] = (int32_t)(first + i);
+}
+
+// rowptr[v] = first k with key[k] >= v (key sorted ascending), v in [0, n]
+__global__ void k_rowptr_from_sorted64(int64_t m, const int32_t *__restrict__ key, int64_t n,
+                                       int64_t *__restrict__ rowptr)
+{
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= n;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        int64_t lo = 0, hi = m;
+        while (lo < hi) {
+            const int64_t mid = lo + ((hi - lo) >> 1);
+            if (key[mid] < (int32_t)v) lo = mid + 1;
+            else hi = mid;
+        }
+        rowptr[v] = lo;
+    }
+}
+
+__global__ void k_fill_neg_inf(int64_t n, double2 *__restrict__ x)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        x[i] = make_double2(-INFINITY, -INFINITY);
+}
+
+// merge the world partial B-side top-2 arrays (gathered [world][nB]); max is
+// exact, so the merged (max1, max2) equals the single-GPU one bit for bit
+__global__ void k_merge_top2(int64_t nB, int world, const double2 *__restrict__ all, double2 *__restrict__ out)
+{
+    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nB; b += (int64_t)gridDim.x * blockDim.x) {
+        double m1 = -INFINITY, m2 = -INFINITY;
+        for (int r = 0; r < world; r++) {
+            const double2 o = all[(int64_t)r * nB + b];
+            top2_merge(m1, m2, o.x, o.y);
+        }
+        out[b] = make_double2(m1, m2);
+    }
+}
+
+__global__ void k_add_u64(int64_t n, unsigned long long *__restrict__ dst, const unsigned long long *__restrict__ src)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dst[i] += src[i];
+}
+
+} // namespace
+
+cualign_status bp_merge_top2(cualign_bp *h)
+{
+    KScope ks(h, CUALIGN_K_TOP2);
+    const int64_t nB = h->L.nB;
+    if (nB) k_merge_top2<<<grid_for(nB, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB, h->world, h->Btop_all, h->Btop);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
+cualign_status bp_add_u64(cualign_bp *h, unsigned long long *dst, const unsigned long long *src, int64_t n)
+{
+    KScope ks(h, CUALIGN_K_OTHER);
+    if (n > 0) k_add_u64<<<grid_for(n, 256, h->num_sms * 8), 256, 0, h->stream>>>(n, dst, src);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
+namespace {
+
+// B incidence restricted to the owned edges [e0, e1) (ids ascending per b)
+cualign_status build_local_incidence(cualign_bp *h)
+{
+    const int64_t nB = h->L.nB, ml = h->e1 - h->e0;
+    CA_TRY(dalloc(h, &h->Bedge_loc, (size_t)(ml ? ml : 1)));
+    CA_TRY(dalloc(h, &h->Bptr_loc, (size_t)nB + 1));
+    int32_t *keys = nullptr, *ids = nullptr;
+    void *tmp = nullptr;
+    CA_CUDA(cudaMalloc(&keys, sizeof(int32_t) * (size_t)(ml ? ml : 1)));
+    CA_CUDA(cudaMalloc(&ids, sizeof(int32_t) * (size_t)(ml ? ml : 1)));
+    cualign_status st = CUALIGN_OK;
+    if (ml) {
+        k_iota_from<<<grid_for(ml, 256, h->num_sms * 8), 256, 0, h->stream>>>(ml, h->e0, ids);
+        int end_bit = 1;
+        while (end_bit < 31 && ((int64_t)1 << end_bit) < nB) end_bit++;
+        size_t tb = 0;
+        cub::DeviceRadixSort::SortPairs(nullptr, tb, h->L.Lb + h->e0, keys, ids, h->Bedge_loc, (int)ml, 0, end_bit,
+                                        h->stream);
+        if (cudaMalloc(&tmp, tb ? tb : 1) != cudaSuccess) st = CUALIGN_ENOMEM;
+        if (st == CUALIGN_OK)
+            cub::DeviceRadixSort::SortPairs(tmp, tb, h->L.Lb + h->e0, keys, ids, h->Bedge_loc, (int)ml, 0, end_bit,
+                                            h->stream);
+    }
+    if (st == CUALIGN_OK)
+        k_rowptr_from_sorted64<<<grid_for(nB + 1, 256, h->num_sms * 8), 256, 0, h->stream>>>(ml, keys, nB,
+                                                                                         h->Bptr_loc);
+    cudaStreamSynchronize(h->stream);
+    cudaFree(keys);
+    cudaFree(ids);
+    if (tmp) cudaFree(tmp);
+    CA_TRY(st);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
+} // namespace
+
 cualign_status bp_setup(cualign_bp *h)
 {
     KScope ks(h, CUALIGN_K_INIT);
@@ -449,6 +559,16 @@ cualign_status bp_setup(cualign_bp *h)
     CA_TRY(dalloc(h, &h->Btop, (size_t)nB + 1));
     CA_TRY(dalloc(h, &h->Bcnt, (size_t)nB + 1));
     CA_CUDA(cudaMemsetAsync(h->Bcnt, 0, sizeof(unsigned int) * ((size_t)nB + 1), h->stream));
+    const int64_t *Bptr = h->L.Bptr;
+    if (h->world > 1) {
+        // partial B-side top-2 over the owned edges, gathered and merged
+        CA_TRY(build_local_incidence(h));
+        Bptr = h->Bptr_loc;
+        CA_TRY(dalloc(h, &h->Btop_part, (size_t)nB + 1));
+        CA_TRY(dalloc(h, &h->Btop_all, (size_t)nB * h->world + 1));
+        k_fill_neg_inf<<<grid_for(nB + 1, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB + 1, h->Btop_part);
+        CA_CUDA(cudaGetLastError());
+    }
     // B-side chunks for k_top2
     CA_TRY(dalloc(h, &h->Bcp, (size_t)nB + 1));
     CA_CUDA(cudaMemsetAsync(h->Bcp, 0, sizeof(int64_t), h->stream));
@@ -457,7 +577,7 @@ cualign_status bp_setup(cualign_bp *h)
         void *tmp = nullptr;
         size_t tb = 0;
         CA_CUDA(cudaMalloc(&cnt, sizeof(int64_t) * (size_t)nB));
-        k_chunk_count<<<grid_for(nB, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB, h->L.Bptr, cnt);
+        k_chunk_count<<<grid_for(nB, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB, Bptr, cnt);
         CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, cnt, h->Bcp + 1, (int)nB, h->stream));
         CA_CUDA(cudaMalloc(&tmp, tb ? tb : 1));
         CA_CUDA(cub::DeviceScan::InclusiveSum(tmp, tb, cnt, h->Bcp + 1, (int)nB, h->stream));
@@ -480,42 +600,56 @@ cualign_status bp_fsum(cualign_bp *h)
     return launch_square(h, false);
 }
 
-// First half of an iteration: the device counter advances to this iteration
-// p (kernels read gh[p]), then lines 9-12 and 14-15 on the vectors (top-2,
-// k_edge).  y^c, z^c of iteration p are final after this half, so the
-// rounding of p may run concurrently with the second half.
-cualign_status bp_iterate_front(cualign_bp *h)
+// Start of an iteration: the device counter advances to this iteration p
+// (kernels read gh[p]); per-vertex top-2 of y^p over the owned A rows and of
+// z^p over the B columns (partial over the owned edges when sharded).
+cualign_status bp_front_top2(cualign_bp *h)
 {
-    const bool exact = (h->flags & CUALIGN_FLAG_EXACT) != 0;
-    const bool literal = (h->flags & CUALIGN_FLAG_OTHERMAX_LITERAL) != 0;
-    const int64_t m = h->L.m;
     {
         KScope ks(h, CUALIGN_K_OTHER);
         k_advance<<<1, 1, 0, h->stream>>>(h->p_dev);
         CA_CUDA(cudaGetLastError());
     }
-    if (m > 0) {
-        {
-            KScope ks(h, CUALIGN_K_TOP2);
-            Top2Args T{(int64_t)h->L.nA, h->nchunks, h->L.Arow, h->chunk_b, h->Bcp, h->L.Bptr, h->L.Bedge,
-                       h->yp, h->zp, h->Atop, h->Btop, h->Bct, h->Bcnt};
+    if (h->L.m > 0) {
+        KScope ks(h, CUALIGN_K_TOP2);
+        const bool sh = h->world > 1;
+        Top2Args T{(int64_t)(h->a1 - h->a0), h->nchunks, (int64_t)h->a0, h->L.Arow, h->chunk_b, h->Bcp,
+                   sh ? h->Bptr_loc : h->L.Bptr, sh ? h->Bedge_loc : h->L.Bedge, h->yp, h->zp, h->Atop,
+                   sh ? h->Btop_part : h->Btop, h->Bct, h->Bcnt};
+        if (T.nA + T.nchunks > 0)
             k_top2<<<grid_for((T.nA + T.nchunks) * TG, 256, 1 << 30), 256, 0, h->stream>>>(T);
-            CA_CUDA(cudaGetLastError());
-        }
-        {
-            KScope ks(h, CUALIGN_K_EDGE);
-            EdgeArgs R{m, h->L.La, h->L.Lb, h->L.w, h->alpha, h->fp_inv, h->gh_dev, h->p_dev, h->tacc, h->texact,
-                       h->Atop, h->Btop, h->yp, h->zp, h->yc, h->zc, h->d, h->u};
-            constexpr int EPT = 4;
-            const int grid = grid_for((m + EPT - 1) / EPT, 256, 1 << 30);
-            if (exact && literal) k_edge<EPT, true, true><<<grid, 256, 0, h->stream>>>(R);
-            else if (exact) k_edge<EPT, true, false><<<grid, 256, 0, h->stream>>>(R);
-            else if (literal) k_edge<EPT, false, true><<<grid, 256, 0, h->stream>>>(R);
-            else k_edge<EPT, false, false><<<grid, 256, 0, h->stream>>>(R);
-            CA_CUDA(cudaGetLastError());
-        }
+        CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;
+}
+
+// Lines 10-12 and 14-15 on the owned edges (k_edge).  y^c, z^c of iteration p
+// are final after this, so the rounding of p may run concurrently with the
+// square pass.
+cualign_status bp_front_edge(cualign_bp *h)
+{
+    const bool exact = (h->flags & CUALIGN_FLAG_EXACT) != 0;
+    const bool literal = (h->flags & CUALIGN_FLAG_OTHERMAX_LITERAL) != 0;
+    const int64_t ml = h->e1 - h->e0;
+    if (ml > 0) {
+        KScope ks(h, CUALIGN_K_EDGE);
+        EdgeArgs R{h->e0, h->e1, h->L.La, h->L.Lb, h->L.w, h->alpha, h->fp_inv, h->gh_dev, h->p_dev, h->tacc,
+                   h->texact, h->Atop, h->Btop, h->yp, h->zp, h->yc, h->zc, h->d, h->u};
+        constexpr int EPT = 4;
+        const int grid = grid_for((ml + EPT - 1) / EPT, 256, 1 << 30);
+        if (exact && literal) k_edge<EPT, true, true><<<grid, 256, 0, h->stream>>>(R);
+        else if (exact) k_edge<EPT, true, false><<<grid, 256, 0, h->stream>>>(R);
+        else if (literal) k_edge<EPT, false, true><<<grid, 256, 0, h->stream>>>(R);
+        else k_edge<EPT, false, false><<<grid, 256, 0, h->stream>>>(R);
+        CA_CUDA(cudaGetLastError());
+    }
+    return CUALIGN_OK;
+}
+
+cualign_status bp_iterate_front(cualign_bp *h)
+{
+    CA_TRY(bp_front_top2(h));
+    return bp_front_edge(h);
 }
 
 // Second half: lines 9, 13, 16 on the S values (the square pass).

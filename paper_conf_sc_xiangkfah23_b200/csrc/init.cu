@@ -116,10 +116,12 @@ __global__ void k_iota(int64_t m, int32_t *x)
 // -------------------------------------------------------------- S build
 // One warp per L edge e = (i, i').  Candidates f are the L edges (j, b) with
 // j in N_A(i) (rows of L, concatenated in ascending j => ascending f); f is a
-// hit iff b in N_B(i').
+// hit iff b in N_B(i').  Rows e in [e_begin, e_end); the count pass writes
+// cnt[e] (global index), the fill pass reads row pointers relative to e_begin
+// (a shard builds only its own rows).
 template <bool FILL>
 __global__ void __launch_bounds__(256)
-k_sbuild(int64_t m, const int32_t *__restrict__ La, const int32_t *__restrict__ Lb,
+k_sbuild(int64_t e_begin, int64_t e_end, const int32_t *__restrict__ La, const int32_t *__restrict__ Lb,
          const int64_t *__restrict__ Arow, const int64_t *__restrict__ Ap,
          const int32_t *__restrict__ Aj, const int64_t *__restrict__ Bp,
          const int32_t *__restrict__ Bj, int64_t *__restrict__ cnt, int64_t *__restrict__ ucnt,
@@ -130,15 +132,16 @@ k_sbuild(int64_t m, const int32_t *__restrict__ La, const int32_t *__restrict__ 
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const unsigned lt_mask = (1u << lane) - 1u;
-    for (int64_t e = warp; e < m; e += nwarps) {
+    for (int64_t e = e_begin + warp; e < e_end; e += nwarps) {
         const int32_t i = La[e], ip = Lb[e];
         const int64_t bs = Bp[ip], be = Bp[ip + 1];
         const int64_t a_lo = Ap[i], a_hi = Ap[i + 1];
         int64_t total = 0, upper = 0, lower_cnt = 0, row0 = 0, sq0 = 0;
         if (FILL) {
-            row0 = Srp[e];
-            sq0 = sq_rp[e];
-            lower_cnt = (Srp[e + 1] - row0) - (sq_rp[e + 1] - sq0);
+            const int64_t r = e - e_begin;
+            row0 = Srp[r];
+            sq0 = sq_rp[r];
+            lower_cnt = (Srp[r + 1] - row0) - (sq_rp[r + 1] - sq0);
         }
         if (be == bs) {
             if (!FILL && lane == 0) {
@@ -222,6 +225,42 @@ __global__ void k_sq_pos(int64_t nsq, const int2 *__restrict__ sq_ef, const int6
         }
         sq_pos[q] = make_longlong2(pef, lo);
     }
+}
+
+// ----------------------------------------------------------- partition
+// Shard cost of an L edge: its squares (the square pass streams 40 B each)
+// plus 2 (per-edge work ~ 80 B).  Boundaries at A-vertex row starts so every
+// A row -- and with it othermaxrow -- stays on one shard.
+__global__ void k_shard_cost(int64_t m, const int64_t *__restrict__ ucnt, int64_t *__restrict__ cost)
+{
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x)
+        cost[e] = ucnt[e] + 2;
+}
+
+// bnd[r] = first edge of shard r: the row start at or before the edge where
+// the inclusive cost prefix first reaches total * r / P
+__global__ void k_shard_bounds(int64_t m, const int64_t *__restrict__ prefix, const int32_t *__restrict__ La,
+                               const int64_t *__restrict__ Arow, int P, int64_t *__restrict__ bnd)
+{
+    const int r = threadIdx.x;
+    if (r > P) return;
+    if (r == 0) {
+        bnd[0] = 0;
+        return;
+    }
+    if (r == P) {
+        bnd[P] = m;
+        return;
+    }
+    const double total = (double)prefix[m - 1];
+    const int64_t target = (int64_t)(total * (double)r / (double)P);
+    int64_t lo = 0, hi = m;
+    while (lo < hi) {
+        const int64_t mid = lo + ((hi - lo) >> 1);
+        if (prefix[mid] < target) lo = mid + 1;
+        else hi = mid;
+    }
+    bnd[r] = lo < m ? Arow[La[lo]] : m;
 }
 
 // undirected A edges as (i, j) pairs with i < j: the suffix of each sorted row
@@ -375,56 +414,111 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
     CA_TRY(build_L(h, h->L, E, devp, true, A->n, B->n));
     const int64_t m = h->L.m;
 
-    // S: count pass
-    CA_TRY(dalloc(h, &h->Srp, (size_t)m + 1));
-    CA_TRY(dalloc(h, &h->sq_rp, (size_t)m + 1));
-    {
-        KScope ks(h, CUALIGN_K_INIT);
-        TmpBuf cnt, ucnt, tmp, mx;
-        CA_CUDA(cudaMalloc(&cnt.p, sizeof(int64_t) * (m ? m : 1)));
-        CA_CUDA(cudaMalloc(&ucnt.p, sizeof(int64_t) * (m ? m : 1)));
-        CA_CUDA(cudaMalloc(&mx.p, sizeof(int64_t)));
-        CA_CUDA(cudaMemsetAsync(h->Srp, 0, sizeof(int64_t), h->stream));
-        CA_CUDA(cudaMemsetAsync(h->sq_rp, 0, sizeof(int64_t), h->stream));
-        CA_CUDA(cudaMemsetAsync(mx.p, 0, sizeof(int64_t), h->stream));
-        if (m) {
-            const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
-            k_sbuild<false><<<blocks, 256, 0, h->stream>>>(m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
-                                                           (int64_t *)cnt.p, (int64_t *)ucnt.p, nullptr,
-                                                           nullptr, nullptr, nullptr);
-            CA_CUDA(cudaGetLastError());
-            size_t t1 = 0, t2 = 0, t3 = 0;
-            CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, t1, (int64_t *)cnt.p, h->Srp + 1, (int)m, h->stream));
-            CA_CUDA(cub::DeviceReduce::Max(nullptr, t3, (int64_t *)cnt.p, (int64_t *)mx.p, (int)m, h->stream));
-            t2 = t1 > t3 ? t1 : t3;
-            CA_CUDA(cudaMalloc(&tmp.p, t2 ? t2 : 1));
-            CA_CUDA(cub::DeviceScan::InclusiveSum(tmp.p, t1, (int64_t *)cnt.p, h->Srp + 1, (int)m, h->stream));
-            CA_CUDA(cub::DeviceScan::InclusiveSum(tmp.p, t1, (int64_t *)ucnt.p, h->sq_rp + 1, (int)m, h->stream));
-            CA_CUDA(cub::DeviceReduce::Max(tmp.p, t3, (int64_t *)cnt.p, (int64_t *)mx.p, (int)m, h->stream));
-        }
-        CA_CUDA(cudaMemcpyAsync(&h->s, h->Srp + m, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
-        CA_CUDA(cudaMemcpyAsync(&h->nsq, h->sq_rp + m, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
-        CA_CUDA(cudaMemcpyAsync(&h->max_row, mx.p, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
-        CA_CUDA(cudaStreamSynchronize(h->stream));
-    }
-    if (h->s != 2 * h->nsq) {
-        set_error("internal: S not symmetric (s=%lld, upper=%lld)", (long long)h->s, (long long)h->nsq);
-        return CUALIGN_ECUDA;
-    }
     if (m >= ((int64_t)1 << 31) - 1) {
         set_error("m = %lld exceeds int32 edge ids", (long long)m);
         return CUALIGN_EINVAL;
     }
-    // S: fill pass
+    // S: count pass over all rows (a shard needs every row's count for the
+    // partition and the global max row), then this handle's rows [e0, e1)
+    {
+        KScope ks(h, CUALIGN_K_INIT);
+        TmpBuf cnt, ucnt, tmp, mx, tot, bnd;
+        CA_CUDA(cudaMalloc(&cnt.p, sizeof(int64_t) * (m ? m : 1)));
+        CA_CUDA(cudaMalloc(&ucnt.p, sizeof(int64_t) * (m ? m : 1)));
+        CA_CUDA(cudaMalloc(&mx.p, 3 * sizeof(int64_t)));
+        CA_CUDA(cudaMemsetAsync(mx.p, 0, 3 * sizeof(int64_t), h->stream));
+        int64_t host3[3] = {0, 0, 0}; // max row, s, squares (global)
+        if (m) {
+            const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
+            k_sbuild<false><<<blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
+                                                           (int64_t *)cnt.p, (int64_t *)ucnt.p, nullptr,
+                                                           nullptr, nullptr, nullptr);
+            CA_CUDA(cudaGetLastError());
+            size_t t1 = 0, t3 = 0;
+            CA_CUDA(cub::DeviceReduce::Max(nullptr, t3, (int64_t *)cnt.p, (int64_t *)mx.p, (int)m, h->stream));
+            CA_CUDA(cub::DeviceReduce::Sum(nullptr, t1, (int64_t *)cnt.p, (int64_t *)mx.p + 1, (int)m, h->stream));
+            size_t t2 = t1 > t3 ? t1 : t3;
+            CA_CUDA(cudaMalloc(&tmp.p, t2 ? t2 : 1));
+            CA_CUDA(cub::DeviceReduce::Max(tmp.p, t3, (int64_t *)cnt.p, (int64_t *)mx.p, (int)m, h->stream));
+            CA_CUDA(cub::DeviceReduce::Sum(tmp.p, t1, (int64_t *)cnt.p, (int64_t *)mx.p + 1, (int)m, h->stream));
+            CA_CUDA(cub::DeviceReduce::Sum(tmp.p, t1, (int64_t *)ucnt.p, (int64_t *)mx.p + 2, (int)m, h->stream));
+            CA_CUDA(cudaMemcpyAsync(host3, mx.p, sizeof(host3), cudaMemcpyDeviceToHost, h->stream));
+        }
+        CA_CUDA(cudaStreamSynchronize(h->stream));
+        h->max_row = host3[0];
+        h->s_total = host3[1];
+        h->nsq_total = host3[2];
+        if (h->s_total != 2 * h->nsq_total) {
+            set_error("internal: S not symmetric (s=%lld, upper=%lld)", (long long)h->s_total,
+                      (long long)h->nsq_total);
+            return CUALIGN_ECUDA;
+        }
+        // partition (A-vertex blocks) -- identical on every shard
+        h->bounds.assign((size_t)h->world + 1, 0);
+        h->bounds[(size_t)h->world] = m;
+        if (h->world > 1 && m) {
+            CA_CUDA(cudaMalloc(&tot.p, sizeof(int64_t) * (size_t)m));
+            CA_CUDA(cudaMalloc(&bnd.p, sizeof(int64_t) * ((size_t)h->world + 1)));
+            k_shard_cost<<<grid_for(m, 256, G), 256, 0, h->stream>>>(m, (const int64_t *)ucnt.p, (int64_t *)tot.p);
+            size_t tb = 0;
+            TmpBuf tmp2;
+            CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, (int64_t *)tot.p, (int64_t *)tot.p, (int)m, h->stream));
+            CA_CUDA(cudaMalloc(&tmp2.p, tb ? tb : 1));
+            CA_CUDA(cub::DeviceScan::InclusiveSum(tmp2.p, tb, (int64_t *)tot.p, (int64_t *)tot.p, (int)m, h->stream));
+            k_shard_bounds<<<1, 32, 0, h->stream>>>(m, (const int64_t *)tot.p, h->L.La, h->L.Arow, h->world,
+                                                    (int64_t *)bnd.p);
+            CA_CUDA(cudaGetLastError());
+            CA_CUDA(cudaMemcpyAsync(h->bounds.data(), bnd.p, sizeof(int64_t) * ((size_t)h->world + 1),
+                                    cudaMemcpyDeviceToHost, h->stream));
+            CA_CUDA(cudaStreamSynchronize(h->stream));
+        }
+        h->e0 = h->bounds[(size_t)h->rank];
+        h->e1 = h->bounds[(size_t)h->rank + 1];
+        const int64_t ml = h->e1 - h->e0;
+        h->a0 = 0;
+        h->a1 = 0;
+        if (h->world == 1) {
+            h->a1 = A->n;
+        } else if (ml > 0) {
+            int32_t aa[2];
+            CA_CUDA(cudaMemcpy(&aa[0], h->L.La + h->e0, sizeof(int32_t), cudaMemcpyDeviceToHost));
+            CA_CUDA(cudaMemcpy(&aa[1], h->L.La + h->e1 - 1, sizeof(int32_t), cudaMemcpyDeviceToHost));
+            h->a0 = aa[0];
+            h->a1 = aa[1] + 1;
+        }
+        // local row pointers: scans over this shard's rows
+        CA_TRY(dalloc(h, &h->Srp, (size_t)ml + 1));
+        CA_TRY(dalloc(h, &h->sq_rp, (size_t)ml + 1));
+        CA_CUDA(cudaMemsetAsync(h->Srp, 0, sizeof(int64_t), h->stream));
+        CA_CUDA(cudaMemsetAsync(h->sq_rp, 0, sizeof(int64_t), h->stream));
+        if (ml) {
+            size_t tb = 0;
+            TmpBuf tmp3;
+            CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, (int64_t *)cnt.p + h->e0, h->Srp + 1, (int)ml,
+                                                  h->stream));
+            CA_CUDA(cudaMalloc(&tmp3.p, tb ? tb : 1));
+            CA_CUDA(cub::DeviceScan::InclusiveSum(tmp3.p, tb, (int64_t *)cnt.p + h->e0, h->Srp + 1, (int)ml,
+                                                  h->stream));
+            CA_CUDA(cub::DeviceScan::InclusiveSum(tmp3.p, tb, (int64_t *)ucnt.p + h->e0, h->sq_rp + 1, (int)ml,
+                                                  h->stream));
+            CA_CUDA(cudaMemcpyAsync(&h->s, h->Srp + ml, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+            CA_CUDA(cudaMemcpyAsync(&h->nsq, h->sq_rp + ml, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+            CA_CUDA(cudaStreamSynchronize(h->stream));
+        } else {
+            h->s = 0;
+            h->nsq = 0;
+        }
+    }
+    // S: fill pass over this handle's rows
     CA_TRY(dalloc(h, &h->Scol, (size_t)(h->s ? h->s : 1)));
     CA_TRY(dalloc(h, &h->sq_ef, (size_t)(h->nsq ? h->nsq : 1)));
     CA_TRY(dalloc(h, &h->sq_val, (size_t)(h->nsq ? h->nsq : 1)));
     {
         KScope ks(h, CUALIGN_K_INIT);
-        if (m && h->s) {
-            const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
-            k_sbuild<true><<<blocks, 256, 0, h->stream>>>(m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
-                                                          nullptr, nullptr, h->Srp, h->sq_rp, h->Scol,
+        if (h->e1 > h->e0 && h->s) {
+            const int blocks = grid_for((h->e1 - h->e0) * 32, 256, h->num_sms * 16);
+            k_sbuild<true><<<blocks, 256, 0, h->stream>>>(h->e0, h->e1, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp,
+                                                          Bj, nullptr, nullptr, h->Srp, h->sq_rp, h->Scol,
                                                           h->sq_ef);
             CA_CUDA(cudaGetLastError());
         }

@@ -79,11 +79,25 @@ struct cualign_bp {
 
     cualign::LDev L;
 
-    // S: full CSR over edge ids, and the square layout
+    // sharding: this handle owns the L edges [e0, e1) -- whole
+    // A rows [a0, a1) -- and the S rows of those edges.  world == 1: all.
+    int32_t rank = 0, world = 1;
+    int64_t e0 = 0, e1 = 0;
+    int32_t a0 = 0, a1 = 0;
+    std::vector<int64_t> bounds;         // world+1 edge boundaries (identical on all shards)
+    int64_t s_total = 0, nsq_total = 0;  // global nnz(S), squares
+    void *comm = nullptr;                // ncclComm_t of a process-sharded handle
+    std::vector<cualign_bp *> vshards;   // in-process virtual shards (loopback group handle)
+    double2 *Btop_part = nullptr;        // per-shard partial B-side top-2 (before the merge)
+    double2 *Btop_all = nullptr;         // world x nB gathered partials
+    int64_t *Bptr_loc = nullptr;         // B incidence of the owned edges (top-2 partials)
+    int32_t *Bedge_loc = nullptr;
+
+    // S: CSR over edge ids (rows [e0, e1)), and the square layout
     int64_t s = 0, nsq = 0, max_row = 0;
-    int64_t *Srp = nullptr;      // m+1
+    int64_t *Srp = nullptr;      // (e1-e0)+1, indexed e - e0
     int32_t *Scol = nullptr;     // s
-    int64_t *sq_rp = nullptr;    // m+1: squares {e<f} of row e are sq_rp[e]..sq_rp[e+1]-1
+    int64_t *sq_rp = nullptr;    // (e1-e0)+1: squares {e<f} of row e are sq_rp[e-e0]..sq_rp[e-e0+1]-1
     int2 *sq_ef = nullptr;       // nsq: (e, f), e < f, sorted by (e, f)
     double2 *sq_val = nullptr;   // nsq: (S^p_ef, S^p_fe)
     longlong2 *sq_pos = nullptr; // nsq: (pos(e,f), pos(f,e)) in the CSR; built lazily
@@ -190,6 +204,18 @@ cualign_status bp_fsum(cualign_bp *h);                 // t <- sum_f F(S^p) (ini
 cualign_status bp_iterate(cualign_bp *h, int32_t n);   // Alg. 2 l.9-16, n times
 cualign_status bp_iterate_front(cualign_bp *h);        // advance p, top-2, k_edge
 cualign_status bp_iterate_back(cualign_bp *h);         // square pass
+cualign_status bp_front_top2(cualign_bp *h);           // advance p, top-2 (partial B when sharded)
+cualign_status bp_front_edge(cualign_bp *h);           // k_edge on the owned edges
+cualign_status bp_merge_top2(cualign_bp *h);           // gathered B partials -> Btop
+cualign_status bp_add_u64(cualign_bp *h, unsigned long long *dst, const unsigned long long *src, int64_t n);
+
+// shard.cu
+cualign_status shard_fsum(cualign_bp *h);
+cualign_status shard_iterate(cualign_bp *h, int32_t n);
+cualign_status shard_round(cualign_bp *h);
+cualign_status nccl_init_comm(cualign_bp *h, const void *unique_id);
+void nccl_free_comm(cualign_bp *h);
+cualign_status nccl_unique_id(void *out, int32_t len);
 cualign_status bp_scatter_Sp(cualign_bp *h, double *Sfull_dev);        // squares -> CSR
 cualign_status bp_gather_Sp(cualign_bp *h, const double *Sfull_dev);   // CSR -> squares
 

@@ -1,0 +1,97 @@
+"""Sharded path on one GPU: `world` virtual shards in one handle
+exchange through device copies exactly where process shards use NCCL.  The
+sharded run must equal the unsharded run BIT FOR BIT (integer F sums, exact
+max merges, replicated deterministic rounding)."""
+import numpy as np
+import pytest
+
+from synth import make_config
+from oracle import Oracle
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ca():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_sc_xiangkfah23_b200 as ca
+    ca.load_library()
+    return ca
+
+
+def _compare_runs(ca, inst, world, n_iter, flags=0):
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags) as h1, \
+            ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags, world=world) as hs:
+        rp1, col1 = h1.get_S()
+        rps, cols = hs.get_S()
+        assert np.array_equal(rp1, rps) and np.array_equal(col1, cols)
+        for p in range(1, n_iter + 1):
+            h1.iterate(1)
+            hs.iterate(1)
+            a, b = h1.get_state(with_S=False), hs.get_state(with_S=False)
+            for k in ("yc", "zc", "yp", "zp", "d"):
+                bad = np.nonzero(a[k] != b[k])[0]
+                assert bad.size == 0, f"world={world} p={p} {k}: {bad.size} differ"
+            r1, rs = h1.round(), hs.round()
+            for k in ("score_y", "score_z", "overlap_y", "overlap_z", "card_y", "card_z", "best_score",
+                      "best_iter", "source", "iter"):
+                assert r1[k] == rs[k], (p, k)
+        m1, _ = h1.get_best()
+        ms, _ = hs.get_best()
+        assert np.array_equal(m1, ms)
+        sz = hs.sizes()
+        assert sz["world"] == world and sz["s"] == h1.sizes()["s"]
+
+
+@pytest.mark.parametrize("world", [2, 3, 4])
+def test_virtual_shards_bitwise_T(ca, world):
+    _compare_runs(ca, make_config("T"), world, 12)
+
+
+@pytest.mark.parametrize("world", [2, 5])
+def test_virtual_shards_bitwise_O_small(ca, world):
+    _compare_runs(ca, make_config("O", scale=0.01), world, 8)
+
+
+def test_virtual_shards_literal_and_damped(ca):
+    inst = make_config("P", scale=0.05)
+    _compare_runs(ca, inst, 3, 6, ca.FLAG_OTHERMAX_LITERAL | ca.FLAG_ROUND_DAMPED)
+
+
+def test_virtual_shards_more_shards_than_rows(ca):
+    """Tiny instance, many shards: some shards own no edge at all."""
+    from tests.util import load_golden, golden_instance
+    g = load_golden("W1.json")
+    A, B, L = golden_instance(g)
+    inst = make_config("T", scale=0.05)
+    _compare_runs(ca, inst, 8, 5)
+
+
+def test_virtual_shards_match_oracle(ca):
+    inst = make_config("T")
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    o.align(inst.n_iter, inst.gamma)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, world=4) as hs:
+        hs.run(inst.n_iter)
+        mate, info = hs.get_best()
+    omate, obest, _ = o.get_best()
+    assert abs(info["best_score"] - obest) <= 1e-9 * max(1.0, obest)
+
+
+def test_shard_partition_whole_rows(ca):
+    inst = make_config("O", scale=0.01)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, world=3) as hs:
+        sz = hs.sizes()
+        assert sz["rank"] == -1 and sz["edge_begin"] == 0 and sz["edge_end"] == inst.L.m
+
+
+def test_sharded_rejects_exact_and_set_state(ca):
+    inst = make_config("T", scale=0.2)
+    with pytest.raises(ca.CuAlignError):
+        ca.CuAlignBP(inst.A, inst.B, inst.L, flags=ca.FLAG_EXACT, world=2)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, world=2) as hs:
+        with pytest.raises(ca.CuAlignError) as ei:
+            hs.set_state(np.zeros(inst.L.m), np.zeros(inst.L.m), np.zeros(hs.s), 0)
+        assert ei.value.status == -5
