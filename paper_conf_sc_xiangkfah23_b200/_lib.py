@@ -216,6 +216,8 @@ class CuAlignBP:
         gb = Graph_t(self.n_b, _ptr(Bp), _ptr(Bj))
         el = Edges_t(self.m, _ptr(La), _ptr(Lb), _ptr(w))
         self.world = int(world)
+        if nccl_id is not None:
+            import torch  # noqa: F401  -- load torch's NCCL before the library dlopens one
         if self.world > 1 and nccl_id is None:
             rank = -1
         self._nccl_id = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
@@ -342,6 +344,7 @@ def version():
 
 def nccl_unique_id() -> bytes:
     """128-byte NCCL unique id for a sharded init (create on one rank, broadcast)."""
+    import torch  # noqa: F401  -- torch's NCCL must be the one loaded (the library dlopens libnccl.so.2)
     buf = ctypes.create_string_buffer(128)
     _check(load_library().cualign_nccl_unique_id(buf, 128))
     return buf.raw

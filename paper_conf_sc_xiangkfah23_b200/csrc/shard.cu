@@ -21,17 +21,64 @@
 // against the unsharded one on a single GPU.
 #include "internal.cuh"
 
+#include <dlfcn.h>
 #include <nccl.h>
 
 namespace cualign {
 
 namespace {
 
+// NCCL is resolved at run time (dlopen "libnccl.so.2"): a process that already
+// loaded torch gets torch's NCCL, and loading this library never pins an NCCL
+// version that torch would then fail to bind against.
+struct NcclApi {
+    bool tried = false, ok = false;
+    ncclResult_t (*GetUniqueId)(ncclUniqueId *) = nullptr;
+    ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*AllGather)(const void *, void *, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*Broadcast)(const void *, void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*Reduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, int, ncclComm_t,
+                           cudaStream_t) = nullptr;
+    ncclResult_t (*GroupStart)() = nullptr;
+    ncclResult_t (*GroupEnd)() = nullptr;
+    const char *(*GetErrorString)(ncclResult_t) = nullptr;
+};
+
+NcclApi &nccl()
+{
+    static NcclApi api;
+    if (!api.tried) {
+        api.tried = true;
+        void *lib = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!lib) lib = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+        if (lib) {
+            api.GetUniqueId = (decltype(api.GetUniqueId))dlsym(lib, "ncclGetUniqueId");
+            api.CommInitRank = (decltype(api.CommInitRank))dlsym(lib, "ncclCommInitRank");
+            api.CommDestroy = (decltype(api.CommDestroy))dlsym(lib, "ncclCommDestroy");
+            api.AllGather = (decltype(api.AllGather))dlsym(lib, "ncclAllGather");
+            api.Broadcast = (decltype(api.Broadcast))dlsym(lib, "ncclBroadcast");
+            api.Reduce = (decltype(api.Reduce))dlsym(lib, "ncclReduce");
+            api.GroupStart = (decltype(api.GroupStart))dlsym(lib, "ncclGroupStart");
+            api.GroupEnd = (decltype(api.GroupEnd))dlsym(lib, "ncclGroupEnd");
+            api.GetErrorString = (decltype(api.GetErrorString))dlsym(lib, "ncclGetErrorString");
+            api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.AllGather && api.Broadcast &&
+                     api.Reduce && api.GroupStart && api.GroupEnd && api.GetErrorString;
+        }
+    }
+    return api;
+}
+
 #define CA_NCCL(call)                                                                          \
     do {                                                                                       \
-        ncclResult_t _r = (call);                                                              \
+        if (!nccl().ok) {                                                                      \
+            ::cualign::set_error("NCCL (libnccl.so.2) could not be loaded");                  \
+            return CUALIGN_ENCCL;                                                              \
+        }                                                                                      \
+        ncclResult_t _r = nccl().call;                                                         \
         if (_r != ncclSuccess) {                                                               \
-            ::cualign::set_error("%s:%d: %s: %s", __FILE__, __LINE__, #call, ncclGetErrorString(_r)); \
+            ::cualign::set_error("%s:%d: nccl%s: %s", __FILE__, __LINE__, #call,               \
+                                 nccl().GetErrorString(_r));                                   \
             return CUALIGN_ENCCL;                                                              \
         }                                                                                      \
     } while (0)
@@ -96,7 +143,7 @@ struct Nccl : Exchange {
     {
         cualign_bp *h = S[0];
         const int64_t nB = h->L.nB;
-        CA_NCCL(ncclAllGather(h->Btop_part, h->Btop_all, (size_t)(2 * nB), ncclFloat64, (ncclComm_t)h->comm,
+        CA_NCCL(AllGather(h->Btop_part, h->Btop_all, (size_t)(2 * nB), ncclFloat64, (ncclComm_t)h->comm,
                               h->stream));
         return bp_merge_top2(h);
     }
@@ -105,26 +152,26 @@ struct Nccl : Exchange {
         // all-gather-v: one in-place broadcast per owner, grouped
         cualign_bp *h = S[0];
         double *buf = h->*field;
-        CA_NCCL(ncclGroupStart());
+        CA_NCCL(GroupStart());
         for (int r = 0; r < h->world; r++) {
             const int64_t off = h->bounds[(size_t)r], n = h->bounds[(size_t)r + 1] - off;
-            if (n) CA_NCCL(ncclBroadcast(buf + off, buf + off, (size_t)n, ncclFloat64, r, (ncclComm_t)h->comm, h->stream));
+            if (n) CA_NCCL(Broadcast(buf + off, buf + off, (size_t)n, ncclFloat64, r, (ncclComm_t)h->comm, h->stream));
         }
-        CA_NCCL(ncclGroupEnd());
+        CA_NCCL(GroupEnd());
         return CUALIGN_OK;
     }
     cualign_status reduce_t(std::vector<cualign_bp *> &S) override
     {
         // reduce-scatter-v: one in-place reduce per owner, grouped
         cualign_bp *h = S[0];
-        CA_NCCL(ncclGroupStart());
+        CA_NCCL(GroupStart());
         for (int r = 0; r < h->world; r++) {
             const int64_t off = h->bounds[(size_t)r], n = h->bounds[(size_t)r + 1] - off;
             if (n)
-                CA_NCCL(ncclReduce(h->tacc + off, h->tacc + off, (size_t)n, ncclUint64, ncclSum, r,
+                CA_NCCL(Reduce(h->tacc + off, h->tacc + off, (size_t)n, ncclUint64, ncclSum, r,
                                    (ncclComm_t)h->comm, h->stream));
         }
-        CA_NCCL(ncclGroupEnd());
+        CA_NCCL(GroupEnd());
         return zero_unowned(h);
     }
 };
@@ -188,7 +235,7 @@ cualign_status nccl_init_comm(cualign_bp *h, const void *unique_id)
     ncclUniqueId id;
     memcpy(&id, unique_id, sizeof(id));
     ncclComm_t c = nullptr;
-    CA_NCCL(ncclCommInitRank(&c, h->world, id, h->rank));
+    CA_NCCL(CommInitRank(&c, h->world, id, h->rank));
     h->comm = c;
     return CUALIGN_OK;
 }
@@ -196,7 +243,7 @@ cualign_status nccl_init_comm(cualign_bp *h, const void *unique_id)
 void nccl_free_comm(cualign_bp *h)
 {
     if (h->comm) {
-        ncclCommDestroy((ncclComm_t)h->comm);
+        if (nccl().ok) nccl().CommDestroy((ncclComm_t)h->comm);
         h->comm = nullptr;
     }
 }
@@ -208,7 +255,7 @@ cualign_status nccl_unique_id(void *out, int32_t len)
         return CUALIGN_EINVAL;
     }
     ncclUniqueId id;
-    CA_NCCL(ncclGetUniqueId(&id));
+    CA_NCCL(GetUniqueId(&id));
     memcpy(out, &id, sizeof(id));
     return CUALIGN_OK;
 }
