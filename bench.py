@@ -225,13 +225,13 @@ def main():
     ap.add_argument("--exact", action="store_true", help="CUALIGN_FLAG_EXACT (oracle-order sums)")
     ap.add_argument("--match-rounds", action="store_true", help="pointer-round matching schedule")
     ap.add_argument("--prof-steps", type=int, default=20, help="steps of the per-kernel timing pass")
+    ap.add_argument("--strong", action="store_true", help="N > 1: shard the same instance (strong scaling)")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
     rank, world, local = dist_setup(args)
     if args.impl == "reference":
         run_reference(args, rank, world)
-        barrier(world)
         return
 
     import torch
@@ -240,11 +240,23 @@ def main():
 
     dev = local
     torch.cuda.set_device(dev)
+    # N > 1: weak scaling -- the same generator at N x the size, sharded by
+    # A-vertex blocks over the N ranks; every rank generates the
+    # identical seeded instance
+    scale = args.scale * (world if (world > 1 and not args.strong) else 1)
     t_gen = time.perf_counter()
-    inst = make_config(args.config, scale=args.scale, seed=None)
+    inst = make_config(args.config, scale=scale, seed=None)
     t_gen = time.perf_counter() - t_gen
-    log(f"[rank {rank}] generated {args.config} (scale {args.scale}) in {t_gen:.1f}s: "
+    log(f"[rank {rank}] generated {args.config} (scale {scale}) in {t_gen:.1f}s: "
         f"n_A={inst.A.n} n_B={inst.B.n} m={inst.L.m}")
+
+    def shard_kw():
+        if world == 1:
+            return {}
+        import torch.distributed as dist
+        obj = [ca.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        return dict(world=world, rank=rank, nccl_id=obj[0])
     # a dedicated stream: the library launches on it and the timing events are
     # recorded on it (torch's default stream is the legacy stream, which does
     # not order against the library's non-blocking streams)
@@ -256,11 +268,12 @@ def main():
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     h = ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags=flags,
-                     device=dev, stream=stream)
+                     device=dev, stream=stream, **shard_kw())
     torch.cuda.synchronize()
-    init_s = time.perf_counter() - t0
+    init_s = max_over_ranks(time.perf_counter() - t0, world, device=f"cuda:{dev}")
     sz = h.sizes()
     m, s, squares = sz["m"], sz["s"], sz["squares"]
+    s_local = 2 * sz["squares_local"]  # this rank's share of the square pass
     log(f"[rank {rank}] init {init_s:.3f}s s={s} squares={squares} max_row={sz['max_row']} "
         f"fp_bits={sz['fixed_point_bits']} device_bytes={sz['device_bytes']/1e9:.2f}GB")
 
@@ -298,8 +311,13 @@ def main():
     torch.cuda.synchronize()
     pst = h.stats(reset=True)
 
-    steps_total = args.steps * world
-    value = steps_total / (elapsed_ms / 1e3)
+    # value: iterations/s of config O; at N > 1 in O-equivalent iterations/s
+    # (iterations/s x squares of the N-times-larger instance / squares of O),
+    # i.e. the whole job's throughput in units of the N = 1 workload
+    from synth import O_full_work
+    unit_squares = O_full_work()[1] / 2 if (args.config == "O" and args.scale == 1.0) else squares / max(world, 1)
+    work_units = squares / unit_squares if world > 1 else 1.0
+    value = args.steps * work_units / (elapsed_ms / 1e3)
     ms_per_step = elapsed_ms / args.steps
     cls_ms = pst["class_ms"]
     cls_n = pst["class_launches"]
@@ -307,9 +325,9 @@ def main():
     bp_ms = (cls_ms["top2"] + cls_ms["edge"] + cls_ms["square"] + cls_ms["rowsum"] + cls_ms["other"]) / prof_steps
     round_ms = (cls_ms["match"] + cls_ms["eval"] + cls_ms["matchaux"]) / prof_steps
     peak, peak_src = read_peaks()
-    sq_bytes = BYTES_PER_NZ * s                    # algorithmic bytes of one square-pass launch
+    sq_bytes = BYTES_PER_NZ * s_local              # algorithmic bytes of one (this rank's) square-pass launch
     sq_gbs = sq_bytes / (sq_ms * 1e-3) / 1e9 if sq_ms > 0 else 0.0
-    it_bytes = BYTES_PER_NZ * s + BYTES_PER_EDGE * m
+    it_bytes = BYTES_PER_NZ * s_local + BYTES_PER_EDGE * (sz["edge_end"] - sz["edge_begin"])
     it_gbs = it_bytes / (bp_ms * 1e-3) / 1e9 if bp_ms > 0 else 0.0
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "square_traffic.json")
@@ -346,12 +364,12 @@ def main():
         barrier(world)
         t0 = time.perf_counter()
         mate, binfo, infos = ca.align(GA, GB, GL, inst.alpha, inst.beta, inst.gamma,
-                                      n_iter=args.e2e_iters, device=dev, stream=stream)
+                                      n_iter=args.e2e_iters, device=dev, stream=stream, **shard_kw())
         torch.cuda.synchronize()
         align_time_s = max_over_ranks(time.perf_counter() - t0, world, device=f"cuda:{dev}")
         import ctypes
         d2h = args.e2e_iters * 112 + 4 * inst.A.n
-        e2e = {"value": args.e2e_iters * world / align_time_s, "unit": UNIT,
+        e2e = {"value": args.e2e_iters * work_units / align_time_s, "unit": UNIT,
                "h2d_bytes_per_step": h2d / args.e2e_iters, "d2h_bytes_per_step": d2h / args.e2e_iters,
                "align_time_s": align_time_s, "iters": args.e2e_iters,
                "best_score": binfo["best_score"], "best_iter": binfo["best_iter"]}
@@ -377,15 +395,17 @@ def main():
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None,
+        "scaling": "strong" if (world > 1 and args.strong) else "weak", "vs_baseline": None,
         "dtype": "f64", "data": "synthetic",
         "config": {"workload": f"{args.config}: " + inst.meta["desc"], "scale": args.scale,
                    "n_a": inst.A.n, "n_b": inst.B.n, "m": m, "s": s, "squares": squares,
                    "alpha": inst.alpha, "beta": inst.beta, "gamma": inst.gamma,
-                   "parallelism": "replicas" if world > 1 else "single",
+                   "parallelism": (f"A-vertex-block shards x{world} (NCCL)" if world > 1 else "single"),
+                   "value_unit_note": ("O-equivalent iterations/s: iterations/s x squares / squares(O)"
+                                       if world > 1 else "iterations/s of this instance"),
                    "l2": "inputs larger than L2 (square layout %.2f GB vs 126 MB L2)" % (24 * squares / 1e9),
                    "mode": "exact" if args.exact else "fast"},
-        "squares_per_s": squares * steps_total / (elapsed_ms / 1e3),
+        "squares_per_s": squares * args.steps / (elapsed_ms / 1e3),
         "bp_iters_per_s": 1e3 / bp_ms if bp_ms > 0 else None,
         "round_ms": round_ms, "bp_ms": bp_ms, "init_s": init_s,
         "roofline": {"bound": "hbm", "kernel": "k_square (a3+a5+a6 square pass)",

@@ -9,10 +9,11 @@ from ._lib import (CuAlignBP, CuAlignError, match, load_library, version, nccl_u
                    FLAG_TIMING, FLAG_MATCH_ROUNDS, EXPORTED, LIB_PATH, KERNEL_CLASS_NAMES)
 
 
-def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=0, stream=None):
+def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=0, stream=None, **shard):
     """End-to-end alignment (Alg. 2): init (S build), n_iter
-    x (iterate + round), best.  Returns (mate_a, info, per-round infos)."""
-    with CuAlignBP(A, B, L, alpha, beta, gamma, flags, device, stream) as h:
+    x (iterate + round), best.  Returns (mate_a, info, per-round infos).
+    shard: world / rank / nccl_id of a sharded run (see CuAlignBP)."""
+    with CuAlignBP(A, B, L, alpha, beta, gamma, flags, device, stream, **shard) as h:
         infos = []
         for _ in range(n_iter):
             h.run(1)                                      # graph replay of iterate + round
