@@ -4,6 +4,8 @@ The compute path is libcualign_bp.so (CUDA, sm_100a; C ABI in
 include/cualign_bp.h).  This package is the thin Python binding over it plus
 the end-to-end `align` helper and the sharded (multi-GPU) driver.
 """
+import time
+
 from ._lib import (CuAlignBP, CuAlignError, match, load_library, version, nccl_unique_id,
                    FLAG_DEVICE_PTRS, FLAG_EXACT, FLAG_OTHERMAX_LITERAL, FLAG_ROUND_DAMPED,
                    FLAG_TIMING, FLAG_MATCH_ROUNDS, EXPORTED, LIB_PATH, KERNEL_CLASS_NAMES)
@@ -19,6 +21,7 @@ def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=
             h.run(1)                                      # graph replay of iterate + round
             infos.append(h.get_best(with_mate=False)[1])  # the step's result to the host
         mate, info = h.get_best()
+        info["t_result"] = time.perf_counter()            # result on the host (before teardown)
     return mate, info, infos
 
 

@@ -20,10 +20,27 @@ void set_error(const char *fmt, ...)
 
 void clear_error() { g_err[0] = 0; }
 
+// Device memory comes from the device's stream-ordered pool with an unlimited
+// release threshold: freed blocks stay cached in the process, so a new handle
+// (a new alignment) reuses them instead of paying cudaMalloc / cudaFree.
+static void keep_pool(int dev)
+{
+    static bool done[64] = {};
+    if (dev < 0 || dev >= 64 || done[dev]) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    (void)cudaGetLastError();
+    done[dev] = true;
+}
+
 cualign_status dmalloc(cualign_bp *h, void **p, size_t bytes)
 {
     if (bytes == 0) bytes = 16;
-    cudaError_t e = cudaMalloc(p, bytes);
+    keep_pool(h->dev);
+    cudaError_t e = cudaMallocAsync(p, bytes, h->stream);
     if (e != cudaSuccess) {
         *p = nullptr;
         set_error("cudaMalloc(%zu bytes) failed: %s", bytes, cudaGetErrorString(e));
@@ -39,7 +56,7 @@ void dfree(cualign_bp *h, void *p)
 {
     for (auto &a : h->allocs)
         if (a.first == p && p) {
-            cudaFree(p);
+            cudaFreeAsync(p, h->stream);
             h->device_bytes -= (int64_t)a.second;
             a.first = nullptr;
             a.second = 0;
@@ -49,7 +66,8 @@ void dfree(cualign_bp *h, void *p)
 void dfree_all(cualign_bp *h)
 {
     for (auto &a : h->allocs)
-        if (a.first) cudaFree(a.first);
+        if (a.first) cudaFreeAsync(a.first, h->stream);
+    cudaStreamSynchronize(h->stream);
     h->allocs.clear();
     h->device_bytes = 0;
 }
