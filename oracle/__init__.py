@@ -79,6 +79,8 @@ def _load():
         lib.orc_round.argtypes = [P, ctypes.POINTER(RoundInfo), P, P]
         lib.orc_get_best.argtypes = [P, P, P, P]
         lib.orc_align.argtypes = [P, ctypes.c_int32, ctypes.c_double, ctypes.POINTER(RoundInfo)]
+        lib.orc_create_light.restype = P
+        lib.orc_create_light.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_int64, P, P, P]
         _lib = lib
     return _lib
 
@@ -191,6 +193,34 @@ class Oracle:
         infos = (RoundInfo * max(n_iter, 1))()
         _load().orc_align(self._h, int(n_iter), float(gamma), infos)
         return [infos[k].as_dict() for k in range(n_iter)]
+
+
+class LightOracle:
+    """L only (no S): the greedy matching of full-size instances."""
+
+    def __init__(self, L):
+        lib = _load()
+        self._keep = [np.ascontiguousarray(L.a, dtype=np.int32), np.ascontiguousarray(L.b, dtype=np.int32),
+                      np.ascontiguousarray(L.w, dtype=np.float64)]
+        self.n_a, self.n_b, self.m = int(L.n_a), int(L.n_b), int(len(L.a))
+        self._h = lib.orc_create_light(self.n_a, self.n_b, self.m, *[_ptr(x) for x in self._keep])
+
+    def greedy(self, x):
+        x = np.ascontiguousarray(x, dtype=np.float64)
+        mate = np.zeros(max(self.n_a, 1), dtype=np.int32)
+        card = _load().orc_greedy(self._h, _ptr(x), _ptr(mate))
+        return mate[:self.n_a], int(card)
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _load().orc_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 def gamma_power(gamma: float, p: int) -> float:
