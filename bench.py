@@ -223,6 +223,7 @@ def main():
     ap.add_argument("--cpu-scale", type=float, default=0.2)
     ap.add_argument("--ref-scale", type=float, default=0.05)
     ap.add_argument("--exact", action="store_true", help="CUALIGN_FLAG_EXACT (oracle-order sums)")
+    ap.add_argument("--fp32", action="store_true", help="CUALIGN_FLAG_FP32_S (S^p stored in fp32, NEXT-3)")
     ap.add_argument("--match-rounds", action="store_true", help="pointer-round matching schedule")
     ap.add_argument("--prof-steps", type=int, default=20, help="steps of the per-kernel timing pass")
     ap.add_argument("--strong", action="store_true", help="N > 1: shard the same instance (strong scaling)")
@@ -262,7 +263,9 @@ def main():
     # not order against the library's non-blocking streams)
     stream = torch.cuda.Stream(device=dev)
     torch.cuda.set_stream(stream)
-    flags = (ca.FLAG_EXACT if args.exact else 0) | (ca.FLAG_MATCH_ROUNDS if args.match_rounds else 0)
+    flags = (ca.FLAG_EXACT if args.exact else 0) | (ca.FLAG_MATCH_ROUNDS if args.match_rounds else 0) | \
+        (ca.FLAG_FP32_S if args.fp32 else 0)
+    bytes_per_nz = (2 * 4 + 4) if args.fp32 else BYTES_PER_NZ  # S^p pair stored as 2 x fp32
 
     # ---------------------------------------------------------------- init
     torch.cuda.synchronize()
@@ -325,9 +328,9 @@ def main():
     bp_ms = (cls_ms["top2"] + cls_ms["edge"] + cls_ms["square"] + cls_ms["rowsum"] + cls_ms["other"]) / prof_steps
     round_ms = (cls_ms["match"] + cls_ms["eval"] + cls_ms["matchaux"]) / prof_steps
     peak, peak_src = read_peaks()
-    sq_bytes = BYTES_PER_NZ * s_local              # algorithmic bytes of one (this rank's) square-pass launch
+    sq_bytes = bytes_per_nz * s_local              # algorithmic bytes of one (this rank's) square-pass launch
     sq_gbs = sq_bytes / (sq_ms * 1e-3) / 1e9 if sq_ms > 0 else 0.0
-    it_bytes = BYTES_PER_NZ * s_local + BYTES_PER_EDGE * (sz["edge_end"] - sz["edge_begin"])
+    it_bytes = bytes_per_nz * s_local + BYTES_PER_EDGE * (sz["edge_end"] - sz["edge_begin"])
     it_gbs = it_bytes / (bp_ms * 1e-3) / 1e9 if bp_ms > 0 else 0.0
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "square_traffic.json")
@@ -335,7 +338,7 @@ def main():
         try:
             with open(tpath) as fh:
                 tj = json.load(fh)
-            if tj.get("s") == s:
+            if tj.get("s") == s and bool(tj.get("fp32", False)) == bool(args.fp32):
                 traffic = tj.get("dram_bytes_per_launch")
         except Exception:
             pass
@@ -364,7 +367,7 @@ def main():
         barrier(world)
         t0 = time.perf_counter()
         mate, binfo, infos = ca.align(GA, GB, GL, inst.alpha, inst.beta, inst.gamma,
-                                      n_iter=args.e2e_iters, device=dev, stream=stream, **shard_kw())
+                                      n_iter=args.e2e_iters, flags=flags, device=dev, stream=stream, **shard_kw())
         torch.cuda.synchronize()
         t_done = time.perf_counter()
         # end-to-end = inputs on the host -> best matching on the host; the
@@ -407,7 +410,7 @@ def main():
                    "value_unit_note": ("O-equivalent iterations/s: iterations/s x squares / squares(O)"
                                        if world > 1 else "iterations/s of this instance"),
                    "l2": "inputs larger than L2 (square layout %.2f GB vs 126 MB L2)" % (24 * squares / 1e9),
-                   "mode": "exact" if args.exact else "fast"},
+                   "mode": ("exact" if args.exact else "fast") + ("+fp32S" if args.fp32 else "")},
         "squares_per_s": squares * args.steps / (elapsed_ms / 1e3),
         "bp_iters_per_s": 1e3 / bp_ms if bp_ms > 0 else None,
         "round_ms": round_ms, "bp_ms": bp_ms, "init_s": init_s,

@@ -66,6 +66,11 @@ typedef enum {
 #define CUALIGN_FLAG_TIMING           0x10u /* record CUDA events around every kernel (diagnostics) */
 #define CUALIGN_FLAG_MATCH_ROUNDS     0x20u /* a7 schedule: synchronous pointer rounds (paper's Phase 1/2)
                                                instead of the default Suitor proposals; same matching */
+#define CUALIGN_FLAG_FP32_S           0x40u /* NEXT-3: store the square messages S^p (the dominant HBM
+                                               stream, 16 -> 8 B per square) in fp32; all arithmetic
+                                               stays fp64, S^p is rounded to fp32 on store.  Not an
+                                               oracle reading: parity is to a tolerance (DESIGN.md
+                                               "fp32 S^p"), not bitwise.  Rejected with EXACT. */
 
 /* Undirected simple graph: symmetric CSR, row i lists the
  * neighbours of i strictly increasing, no self loops (reading Z14).

@@ -8,7 +8,7 @@ import time
 
 from ._lib import (CuAlignBP, CuAlignError, match, load_library, version, nccl_unique_id,
                    FLAG_DEVICE_PTRS, FLAG_EXACT, FLAG_OTHERMAX_LITERAL, FLAG_ROUND_DAMPED,
-                   FLAG_TIMING, FLAG_MATCH_ROUNDS, EXPORTED, LIB_PATH, KERNEL_CLASS_NAMES)
+                   FLAG_TIMING, FLAG_MATCH_ROUNDS, FLAG_FP32_S, EXPORTED, LIB_PATH, KERNEL_CLASS_NAMES)
 
 
 def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=0, stream=None, **shard):
@@ -27,4 +27,4 @@ def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=
 
 __all__ = ["CuAlignBP", "CuAlignError", "match", "align", "load_library", "version", "nccl_unique_id",
            "FLAG_DEVICE_PTRS", "FLAG_EXACT", "FLAG_OTHERMAX_LITERAL", "FLAG_ROUND_DAMPED",
-           "FLAG_TIMING", "FLAG_MATCH_ROUNDS", "EXPORTED", "LIB_PATH", "KERNEL_CLASS_NAMES"]
+           "FLAG_TIMING", "FLAG_MATCH_ROUNDS", "FLAG_FP32_S", "EXPORTED", "LIB_PATH", "KERNEL_CLASS_NAMES"]

@@ -21,6 +21,7 @@ FLAG_OTHERMAX_LITERAL = 0x04
 FLAG_ROUND_DAMPED = 0x08
 FLAG_TIMING = 0x10
 FLAG_MATCH_ROUNDS = 0x20
+FLAG_FP32_S = 0x40
 
 K_TOP2, K_EDGE, K_SQUARE, K_ROWSUM, K_MATCH, K_INIT, K_STATE, K_OTHER, K_EVAL, K_MATCHAUX = range(10)
 KERNEL_CLASS_NAMES = ["top2", "edge", "square", "rowsum", "match", "init", "state", "other", "eval",

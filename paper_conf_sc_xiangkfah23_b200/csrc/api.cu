@@ -263,6 +263,10 @@ static cualign_status check_params(const cualign_params *p)
         set_error("gamma must be in (0, 1], got %g", p->gamma);
         return CUALIGN_EINVAL;
     }
+    if ((p->flags & CUALIGN_FLAG_FP32_S) && (p->flags & CUALIGN_FLAG_EXACT)) {
+        set_error("CUALIGN_FLAG_FP32_S and CUALIGN_FLAG_EXACT are exclusive");
+        return CUALIGN_EINVAL;
+    }
     const int world = p->world <= 0 ? 1 : p->world;
     if (world == 1 && (p->rank != 0 || p->nccl_unique_id != nullptr)) {
         set_error("world = 1 needs rank = 0 and no NCCL id (rank=%d)", p->rank);

@@ -239,9 +239,40 @@ __device__ __forceinline__ void seg_atomic_add(unsigned long long v, int key, in
 
 // UPDATE = apply lines 9, 13, 16 to the pair; otherwise only (re)compute the
 // F row sums of the current S^p (init, set_state).
-template <bool UPDATE, bool EXACT, int SQ_U = 2, bool HINTS = true, bool NOATOM = false>
+// S^p pair storage: fp64 (double2, default) or fp32 (float2, CUALIGN_FLAG_FP32_S,
+// NEXT-3).  Arithmetic is fp64 either way; the fp32 mode rounds the stored
+// state once per update and the next iteration's F is taken from the rounded
+// (stored) value, so the F sums always describe the state that persists.
+template <bool HINTS>
+__device__ __forceinline__ double2 load_pair(const double2 *p)
+{
+    return HINTS ? __ldcs(p) : *p;
+}
+template <bool HINTS>
+__device__ __forceinline__ double2 load_pair(const float2 *p)
+{
+    const float2 f = HINTS ? __ldcs(p) : *p;
+    return make_double2((double)f.x, (double)f.y);
+}
+template <bool HINTS>
+__device__ __forceinline__ double2 store_pair(double2 *p, double2 v)
+{
+    if (HINTS) __stcs(p, v);
+    else *p = v;
+    return v;
+}
+template <bool HINTS>
+__device__ __forceinline__ double2 store_pair(float2 *p, double2 v)
+{
+    const float2 f = make_float2((float)v.x, (float)v.y); // round to nearest
+    if (HINTS) __stcs(p, f);
+    else *p = f;
+    return make_double2((double)f.x, (double)f.y);
+}
+
+template <bool UPDATE, bool EXACT, int SQ_U = 2, bool HINTS = true, bool NOATOM = false, class V = double2>
 __global__ void __launch_bounds__(256)
-k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_val,
+k_square(int64_t nsq, const int2 *__restrict__ sq_ef, V *__restrict__ sq_val,
          const double *__restrict__ u, double beta, const double2 *__restrict__ gh,
          const int *__restrict__ p_dev, double fp_scale,
          unsigned long long *__restrict__ tacc, const longlong2 *__restrict__ sq_pos,
@@ -270,7 +301,7 @@ k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_v
             const int64_t q = base + j * 32 + lane;
             if (q < nsq) {
                 ef[j] = (HINTS ? __ldcs(sq_ef + q) : sq_ef[q]);
-                v[j] = (HINTS ? __ldcs(sq_val + q) : sq_val[q]); // (S^p_ef, S^p_fe)
+                v[j] = load_pair<HINTS>(sq_val + q); // (S^p_ef, S^p_fe)
             }
         }
         if (UPDATE) {
@@ -296,7 +327,7 @@ k_square(int64_t nsq, const int2 *__restrict__ sq_ef, double2 *__restrict__ sq_v
                     const double Scfe = uf[j] - Ffe;
                     v[j].x = g * Scef + hh * v[j].x;                       // line 16
                     v[j].y = g * Scfe + hh * v[j].y;
-                    if (HINTS) __stcs(sq_val + q, v[j]); else sq_val[q] = v[j];
+                    v[j] = store_pair<HINTS>(sq_val + q, v[j]);
                 }
                 // F of the next iteration (line 9 at p+1) from the new pair
                 const double Nef = clamp_beta(beta + v[j].y, beta);
@@ -329,25 +360,27 @@ __global__ void k_rowsum(int64_t m, const int64_t *__restrict__ Srp, const doubl
     }
 }
 
-__global__ void k_scatter_Sp(int64_t nsq, const double2 *__restrict__ sq_val,
-                             const longlong2 *__restrict__ sq_pos, double *__restrict__ Sfull)
+template <class V>
+__global__ void k_scatter_Sp(int64_t nsq, const V *__restrict__ sq_val, const longlong2 *__restrict__ sq_pos,
+                             double *__restrict__ Sfull)
 {
     for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq;
          q += (int64_t)gridDim.x * blockDim.x) {
         const longlong2 pos = sq_pos[q];
-        const double2 v = sq_val[q];
+        const double2 v = load_pair<false>(sq_val + q);
         Sfull[pos.x] = v.x;
         Sfull[pos.y] = v.y;
     }
 }
 
-__global__ void k_gather_Sp(int64_t nsq, double2 *__restrict__ sq_val, const longlong2 *__restrict__ sq_pos,
+template <class V>
+__global__ void k_gather_Sp(int64_t nsq, V *__restrict__ sq_val, const longlong2 *__restrict__ sq_pos,
                             const double *__restrict__ Sfull)
 {
     for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq;
          q += (int64_t)gridDim.x * blockDim.x) {
         const longlong2 pos = sq_pos[q];
-        sq_val[q] = make_double2(Sfull[pos.x], Sfull[pos.y]);
+        store_pair<false>(sq_val + q, make_double2(Sfull[pos.x], Sfull[pos.y]));
     }
 }
 
@@ -375,17 +408,24 @@ int one_wave_grid(cualign_bp *h, const void *fn, int block, int64_t items, int64
 
 __global__ void k_advance(int *p_dev) { *p_dev += 1; }
 
-template <bool UPDATE, bool EXACT, int SQ_U, bool HINTS, bool NOATOM = false>
-void square_launch(cualign_bp *h)
+template <bool UPDATE, bool EXACT, int SQ_U, bool HINTS, bool NOATOM, class V>
+void square_launch_v(cualign_bp *h, V *vals)
 {
-    auto fn = k_square<UPDATE, EXACT, SQ_U, HINTS, NOATOM>;
+    auto fn = k_square<UPDATE, EXACT, SQ_U, HINTS, NOATOM, V>;
     int grid = one_wave_grid(h, (const void *)fn, 256, h->nsq, 256 * SQ_U);
     // leave room for the concurrent rounding branch (graph step): a fraction
     // of the resident CTAs still saturates HBM
     static const double frac = getenv("CUALIGN_SQ_FRAC") ? atof(getenv("CUALIGN_SQ_FRAC")) : 1.0;
     if (frac > 0.0 && frac < 1.0) grid = (int)(grid * frac) > 0 ? (int)(grid * frac) : 1;
-    fn<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->sq_val, h->u, h->beta, h->gh_dev, h->p_dev, h->fp_scale,
-                                    h->tacc, h->sq_pos, h->Ffull);
+    fn<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, vals, h->u, h->beta, h->gh_dev, h->p_dev, h->fp_scale, h->tacc,
+                                    h->sq_pos, h->Ffull);
+}
+
+template <bool UPDATE, bool EXACT, int SQ_U, bool HINTS, bool NOATOM = false>
+void square_launch(cualign_bp *h)
+{
+    if (h->sq_val32) square_launch_v<UPDATE, EXACT, SQ_U, HINTS, NOATOM>(h, h->sq_val32);
+    else square_launch_v<UPDATE, EXACT, SQ_U, HINTS, NOATOM>(h, h->sq_val);
 }
 
 cualign_status launch_square(cualign_bp *h, bool update)
@@ -674,9 +714,11 @@ cualign_status bp_scatter_Sp(cualign_bp *h, double *Sfull_dev)
 {
     CA_TRY(ensure_sq_pos(h));
     KScope ks(h, CUALIGN_K_STATE);
-    if (h->nsq)
-        k_scatter_Sp<<<grid_for(h->nsq, 256, h->num_sms * 8), 256, 0, h->stream>>>(h->nsq, h->sq_val, h->sq_pos,
-                                                                                  Sfull_dev);
+    const int grid = grid_for(h->nsq, 256, h->num_sms * 8);
+    if (h->nsq && h->sq_val32)
+        k_scatter_Sp<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_val32, h->sq_pos, Sfull_dev);
+    else if (h->nsq)
+        k_scatter_Sp<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_val, h->sq_pos, Sfull_dev);
     CA_CUDA(cudaGetLastError());
     return CUALIGN_OK;
 }
@@ -685,9 +727,11 @@ cualign_status bp_gather_Sp(cualign_bp *h, const double *Sfull_dev)
 {
     CA_TRY(ensure_sq_pos(h));
     KScope ks(h, CUALIGN_K_STATE);
-    if (h->nsq)
-        k_gather_Sp<<<grid_for(h->nsq, 256, h->num_sms * 8), 256, 0, h->stream>>>(h->nsq, h->sq_val, h->sq_pos,
-                                                                                 Sfull_dev);
+    const int grid = grid_for(h->nsq, 256, h->num_sms * 8);
+    if (h->nsq && h->sq_val32)
+        k_gather_Sp<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_val32, h->sq_pos, Sfull_dev);
+    else if (h->nsq)
+        k_gather_Sp<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_val, h->sq_pos, Sfull_dev);
     CA_CUDA(cudaGetLastError());
     return CUALIGN_OK;
 }

@@ -100,6 +100,7 @@ struct cualign_bp {
     int64_t *sq_rp = nullptr;    // (e1-e0)+1: squares {e<f} of row e are sq_rp[e-e0]..sq_rp[e-e0+1]-1
     int2 *sq_ef = nullptr;       // nsq: (e, f), e < f, sorted by (e, f)
     double2 *sq_val = nullptr;   // nsq: (S^p_ef, S^p_fe)
+    float2 *sq_val32 = nullptr;  // same, CUALIGN_FLAG_FP32_S storage (sq_val unused then)
     longlong2 *sq_pos = nullptr; // nsq: (pos(e,f), pos(f,e)) in the CSR; built lazily
 
     // fixed-point accumulator of the F row sums (fast mode)
