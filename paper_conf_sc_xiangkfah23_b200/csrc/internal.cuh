@@ -138,6 +138,7 @@ struct cualign_bp {
 
     // matching (two instances: y and z)
     int32_t *candA = nullptr, *candB = nullptr, *mateA = nullptr, *mateB = nullptr;
+    unsigned long long *suit = nullptr; // Suitor slots, 2 instances x max(nA, nB)
     int32_t *best_mate = nullptr;
     double *partial_w = nullptr;
     int match_grid = 0, match_block = 256, eval_grid = 1;

@@ -43,7 +43,8 @@ struct MatchParams {
     const int64_t *Arow, *Bptr;
     const int32_t *Bedge;
     const double *x0, *x1;
-    int32_t *candA, *candB; // SUITOR: suitor slots (edge id of the proposer's edge)
+    int32_t *candA, *candB; // POINTER ROUNDS: candidate pointers
+    unsigned long long *suit; // SUITOR: suitor slots of the targets (packed, see suitor_key)
     int propose_from_b;     // SUITOR: proposing side
     int32_t *mateA, *mateB;
     RoundDev *rd;
@@ -75,6 +76,29 @@ __device__ __forceinline__ const double *xk(const MatchParams &P, int k) { retur
 // (G x U edges per pass, the loads of a pass issued together), a tile argmax
 // picks the heaviest eligible target, lane 0 attempts the CAS and the outcome
 // is broadcast.
+//
+// Suitor slot (u64): 0 = empty, else (key(x) << 32) | e, key(x) = the bits of
+// fp32(x) rounded toward -inf, plus 1 (x > 0 only, so the key is monotone
+// non-decreasing in x and never 0).  Different keys order two proposals
+// without loading the occupant's weight; equal keys (weights within an fp32
+// ulp) fall back to the exact fp64 comparison, so the order is exactly
+// (x desc, id asc).
+__device__ __forceinline__ uint32_t suitor_key(double x)
+{
+    return __float_as_uint(__double2float_rd(x)) + 1u;
+}
+
+// does the proposal (xe, e) with key ke beat the occupant slot s?
+__device__ __forceinline__ bool beats(const double *__restrict__ x, double xe, int e, uint32_t ke,
+                                      unsigned long long s)
+{
+    if (s == 0ull) return true;
+    const uint32_t ks = (uint32_t)(s >> 32);
+    if (ke != ks) return ke > ks;
+    const int es = (int)(uint32_t)s;
+    return better(xe, e, __ldg(x + es), es);
+}
+
 template <int G, int U, class Tile>
 __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
                                             int64_t nT, int64_t slot)
@@ -82,11 +106,14 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
     const int k = (int)(slot / nP);
     int cur = (int)(slot - k * nP);
     const double *__restrict__ x = xk(P, k);
-    int32_t *sT = (fromB ? P.candA : P.candB) + k * nT;
+    unsigned long long *sT = P.suit + k * nT;
     const int64_t *__restrict__ rp = fromB ? P.Bptr : P.Arow;
     const int32_t *__restrict__ tgt = fromB ? P.La : P.Lb;   // target vertex of an edge
     const int32_t *__restrict__ own = fromB ? P.Lb : P.La;   // proposer vertex of an edge
     unsigned long long proposals = 0, scans = 0;
+    // the first scan of a proposer skips the suitor filter (its best target
+    // is tried directly; a better occupant sends it back to a filtered scan)
+    bool filter = false;
     while (true) {
         scans++;
         // heaviest eligible neighbour of `cur` whose suitor is lighter
@@ -94,8 +121,9 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
         double bx = 0.0;
         const int hi = (int)rp[cur + 1]; // positions < m < 2^31: 32-bit index math
         for (int j0 = (int)rp[cur] + lane; j0 < hi; j0 += G * U) {
-            int ee[U], tt[U], ss[U];
-            double xx[U], xs[U];
+            int ee[U], tt[U];
+            double xx[U];
+            unsigned long long ss[U];
 #pragma unroll
             for (int u = 0; u < U; u++) {
                 const int j = j0 + u * G;
@@ -107,20 +135,21 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
                     ee[u] = (xx[u] > 0.0) ? e : -1; // only x > 0 is eligible (Z6)
                 }
             }
+            if (filter) {
 #pragma unroll
-            for (int u = 0; u < U; u++) ss[u] = ee[u] >= 0 ? *(volatile int32_t *)(sT + tt[u]) : -1;
-#pragma unroll
-            for (int u = 0; u < U; u++) xs[u] = ss[u] >= 0 ? __ldg(x + ss[u]) : 0.0;
+                for (int u = 0; u < U; u++) ss[u] = ee[u] >= 0 ? *(volatile unsigned long long *)(sT + tt[u]) : 0ull;
+            }
 #pragma unroll
             for (int u = 0; u < U; u++) {
                 if (ee[u] < 0) continue;
-                if (ss[u] >= 0 && !better(xx[u], ee[u], xs[u], ss[u])) continue;
+                if (filter && !beats(x, xx[u], ee[u], suitor_key(xx[u]), ss[u])) continue;
                 if (better(xx[u], ee[u], bx, best)) {
                     best = ee[u];
                     bx = xx[u];
                 }
             }
         }
+        filter = true;
 #pragma unroll
         for (int off = G / 2; off >= 1; off >>= 1) {
             const double ox = tile.shfl_xor(bx, off);
@@ -134,19 +163,21 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
         int code = 0;        // 0 rescan, 1 done, 2 displaced
         int next = cur;
         if (lane == 0) {
-            int32_t *slotp = sT + __ldg(tgt + best);
-            int s = *(volatile int32_t *)slotp;
+            unsigned long long *slotp = sT + __ldg(tgt + best);
+            const uint32_t kb = suitor_key(bx);
+            const unsigned long long mine = ((unsigned long long)kb << 32) | (uint32_t)best;
+            unsigned long long s = *(volatile unsigned long long *)slotp;
             // CAS loop: retry directly while our edge still beats the occupant,
             // rescan the list only when it does not
-            while (s < 0 || better(bx, best, __ldg(x + s), s)) {
-                const int old = atomicCAS(slotp, s, best);
+            while (beats(x, bx, best, kb, s)) {
+                const unsigned long long old = atomicCAS(slotp, s, mine);
                 if (old == s) {
                     proposals++;
-                    if (s < 0) {
+                    if (s == 0ull) {
                         code = 1;
                     } else {
                         code = 2;
-                        next = __ldg(own + s); // the displaced proposer proposes again
+                        next = __ldg(own + (int)(uint32_t)s); // the displaced proposer proposes again
                     }
                     break;
                 }
@@ -183,13 +214,14 @@ __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
 
 // the final suitor of each target is its mate (mate arrays pre-set to -1)
 __global__ void k_suitor_to_mates(int64_t nT, int ninst, const int32_t *__restrict__ own,
-                                  const int32_t *__restrict__ sT, int32_t *__restrict__ mateT,
+                                  const unsigned long long *__restrict__ sT, int32_t *__restrict__ mateT,
                                   int32_t *__restrict__ mateP, int64_t nP)
 {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * nT;
          v += (int64_t)gridDim.x * blockDim.x) {
         const int k = (int)(v / nT);
-        const int e = sT[v];
+        const unsigned long long s = sT[v];
+        const int e = s ? (int)(uint32_t)s : -1;
         mateT[v] = e;
         if (e >= 0) mateP[k * nP + own[e]] = e;
     }
@@ -519,6 +551,7 @@ MatchParams base_params(cualign_bp *h)
     P.Bedge = h->L.Bedge;
     P.candA = h->candA;
     P.candB = h->candB;
+    P.suit = h->suit;
     P.mateA = h->mateA;
     P.mateB = h->mateB;
     P.rd = h->rd;
@@ -549,8 +582,7 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     const bool fromB = h->propose_from_b;
     P.propose_from_b = fromB ? 1 : 0;
     const int64_t nP = fromB ? nB : nA, nT = fromB ? nA : nB;
-    int32_t *sT = fromB ? h->candA : h->candB;
-    CA_CUDA(cudaMemsetAsync(sT, 0xff, sizeof(int32_t) * (size_t)(2 * nT + 1), h->stream));
+    CA_CUDA(cudaMemsetAsync(h->suit, 0, sizeof(unsigned long long) * (size_t)(2 * nT + 1), h->stream));
     CA_CUDA(cudaMemsetAsync(fromB ? h->mateB : h->mateA, 0xff, sizeof(int32_t) * (size_t)(2 * nP + 1),
                             h->stream));
     const int64_t slots = P.ninst * nP;
@@ -587,7 +619,7 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     if (P.ninst * nT > 0) {
         KScope ks(h, CUALIGN_K_MATCHAUX);
         k_suitor_to_mates<<<grid_for(P.ninst * nT, 256, h->num_sms * 8), 256, 0, h->stream>>>(
-            nT, P.ninst, fromB ? P.Lb : P.La, sT, fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP);
+            nT, P.ninst, fromB ? P.Lb : P.La, h->suit, fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP);
         CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;
@@ -600,6 +632,7 @@ cualign_status match_setup(cualign_bp *h)
     const size_t nA = (size_t)h->L.nA, nB = (size_t)h->L.nB;
     CA_TRY(dalloc(h, &h->candA, 2 * nA + 1));
     CA_TRY(dalloc(h, &h->candB, 2 * nB + 1));
+    CA_TRY(dalloc(h, &h->suit, 2 * (nA > nB ? nA : nB) + 1));
     CA_TRY(dalloc(h, &h->mateA, 2 * nA + 1));
     CA_TRY(dalloc(h, &h->mateB, 2 * nB + 1));
     CA_TRY(dalloc(h, &h->best_mate, nA + 1));
