@@ -348,6 +348,157 @@ k_square(int64_t nsq, const int2 *__restrict__ sq_ef, V *__restrict__ sq_val,
     }
 }
 
+// ------------------------------------------------ TMA-pipelined square pass
+// Same per-square arithmetic as k_square<UPDATE=true, EXACT=false>, but the
+// two streams (sq_ef, sq_val) are moved by the bulk-copy engine
+// (cp.async.bulk, 1-D TMA) into a ring of shared-memory stages, so the
+// streaming reads no longer wait behind the dependent u gathers in the
+// consumer warps' scoreboard: one producer lane keeps SQT_STAGES chunks in
+// flight per CTA, the consumer warps copy a stage to registers, release it
+// (mbarrier arrive) and only then gather u and issue the F-sum atomics.
+// The streams carry an evict-first L2 policy (u and tacc stay resident).
+constexpr int SQT_CHUNK = 512;            // squares per stage
+constexpr int SQT_STAGES = 4;
+constexpr int SQT_CWARPS = 8;             // consumer warps; + 1 producer warp
+constexpr int SQT_PER_THREAD = SQT_CHUNK / (SQT_CWARPS * 32);
+
+__device__ __forceinline__ uint32_t smem_addr(const void *p)
+{
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar)
+{
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
+{
+    asm volatile("{\n\t.reg .pred p;\n"
+                 "MBAR_WAIT_%=:\n\t"
+                 "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+                 "@!p bra MBAR_WAIT_%=;\n}\n" ::"r"(smem_addr(bar)),
+                 "r"(parity)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_load(void *dst, const void *src, uint32_t bytes, uint64_t *bar,
+                                          uint64_t policy)
+{
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+                 " [%0], [%1], %2, [%3], %4;" ::"r"(smem_addr(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_addr(bar)), "l"(policy)
+                 : "memory");
+}
+
+template <class V>
+__global__ void __launch_bounds__((SQT_CWARPS + 1) * 32)
+k_square_tma(int64_t nsq, const int2 *__restrict__ sq_ef, V *__restrict__ sq_val,
+             const double *__restrict__ u, double beta, const double2 *__restrict__ gh,
+             const int *__restrict__ p_dev, double fp_scale, unsigned long long *__restrict__ tacc)
+{
+    // dynamic shared memory: [full | empty barriers (128 B)] [ef stages] [value stages]
+    extern __shared__ __align__(128) unsigned char sq_smem[];
+    uint64_t *full = reinterpret_cast<uint64_t *>(sq_smem);
+    uint64_t *empty = full + SQT_STAGES;
+    int2 (*s_ef)[SQT_CHUNK] = reinterpret_cast<int2 (*)[SQT_CHUNK]>(sq_smem + 128);
+    V (*s_val)[SQT_CHUNK] = reinterpret_cast<V (*)[SQT_CHUNK]>(sq_smem + 128 + sizeof(int2) * SQT_STAGES * SQT_CHUNK);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t nchunks = (nsq + SQT_CHUNK - 1) / SQT_CHUNK;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < SQT_STAGES; s++) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], SQT_CWARPS);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (warp == SQT_CWARPS) {
+        // producer: one lane issues the bulk copies of this CTA's chunks
+        if (lane == 0) {
+            uint64_t policy;
+            asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(policy));
+            int i = 0;
+            for (int64_t c = blockIdx.x; c < nchunks; c += gridDim.x, i++) {
+                const int s = i % SQT_STAGES;
+                if (i >= SQT_STAGES) mbar_wait(&empty[s], (uint32_t)((i / SQT_STAGES) - 1) & 1u);
+                const int64_t q0 = c * SQT_CHUNK;
+                const int n = (int)((nsq - q0) < SQT_CHUNK ? (nsq - q0) : SQT_CHUNK);
+                // 16-byte multiples (the arrays carry 2 elements of padding)
+                const uint32_t b_ef = (uint32_t)((n * sizeof(int2) + 15) & ~(size_t)15);
+                const uint32_t b_val = (uint32_t)((n * sizeof(V) + 15) & ~(size_t)15);
+                mbar_expect_tx(&full[s], b_ef + b_val);
+                bulk_load(&s_ef[s][0], sq_ef + q0, b_ef, &full[s], policy);
+                bulk_load(&s_val[s][0], sq_val + q0, b_val, &full[s], policy);
+            }
+        }
+        return;
+    }
+    const double2 ghp = gh[*p_dev];
+    const double g = ghp.x, hh = ghp.y;
+    const int tid = threadIdx.x; // consumer thread 0 .. SQT_CWARPS*32-1
+    int i = 0;
+    for (int64_t c = blockIdx.x; c < nchunks; c += gridDim.x, i++) {
+        const int s = i % SQT_STAGES;
+        mbar_wait(&full[s], (uint32_t)(i / SQT_STAGES) & 1u);
+        const int64_t q0 = c * SQT_CHUNK;
+        const int n = (int)((nsq - q0) < SQT_CHUNK ? (nsq - q0) : SQT_CHUNK);
+        int2 ef[SQT_PER_THREAD];
+        double2 v[SQT_PER_THREAD];
+#pragma unroll
+        for (int j = 0; j < SQT_PER_THREAD; j++) {
+            const int r = j * (SQT_CWARPS * 32) + tid; // a warp covers 32 consecutive squares
+            if (r < n) {
+                ef[j] = s_ef[s][r];
+                v[j] = load_pair<false>(&s_val[s][r]);
+            }
+        }
+        // order this warp's generic-proxy reads of the stage before the
+        // async-proxy (bulk copy) writes that refill it -- without the fence
+        // a refill can land before the LDS has read the stage (measured)
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[s]); // stage may be refilled
+        double ue[SQT_PER_THREAD], uf[SQT_PER_THREAD];
+#pragma unroll
+        for (int j = 0; j < SQT_PER_THREAD; j++) {
+            const int r = j * (SQT_CWARPS * 32) + tid;
+            if (r < n) {
+                ue[j] = __ldg(u + ef[j].x);
+                uf[j] = __ldg(u + ef[j].y);
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < SQT_PER_THREAD; j++) {
+            const int r = j * (SQT_CWARPS * 32) + tid;
+            int key = -1 - lane;
+            unsigned long long Tef = 0ull;
+            if (r < n) {
+                const double Fef = clamp_beta(beta + v[j].y, beta);    // line 9
+                const double Ffe = clamp_beta(beta + v[j].x, beta);
+                const double Scef = ue[j] - Fef;                       // line 13
+                const double Scfe = uf[j] - Ffe;
+                v[j].x = g * Scef + hh * v[j].x;                       // line 16
+                v[j].y = g * Scfe + hh * v[j].y;
+                v[j] = store_pair<true>(sq_val + q0 + r, v[j]);
+                const double Nef = clamp_beta(beta + v[j].y, beta);   // line 9 at p+1
+                const double Nfe = clamp_beta(beta + v[j].x, beta);
+                const unsigned long long Tfe = __double2ull_rn(Nfe * fp_scale);
+                if (Tfe) atomicAdd(tacc + ef[j].y, Tfe);
+                Tef = __double2ull_rn(Nef * fp_scale);
+                key = ef[j].x;
+            }
+            seg_atomic_add(Tef, key, lane, tacc);
+        }
+    }
+}
+
 // exact mode: t_e = sum of F over row e in ascending f starting from 0.0
 __global__ void k_rowsum(int64_t m, const int64_t *__restrict__ Srp, const double *__restrict__ Ffull,
                          double *__restrict__ texact)
@@ -421,6 +572,38 @@ void square_launch_v(cualign_bp *h, V *vals)
                                     h->sq_pos, h->Ffull);
 }
 
+template <class V>
+constexpr size_t square_tma_smem()
+{
+    return 128 + (sizeof(int2) + sizeof(V)) * SQT_STAGES * SQT_CHUNK;
+}
+
+template <class V>
+void square_tma_launch_v(cualign_bp *h, V *vals)
+{
+    auto fn = k_square_tma<V>;
+    constexpr size_t smem = square_tma_smem<V>();
+    static bool attr_set = false; // per process and V: the attribute is a property of the function
+    if (!attr_set) {
+        cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        attr_set = true;
+    }
+    const int block = (SQT_CWARPS + 1) * 32;
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, block, smem) != cudaSuccess || occ < 1) occ = 1;
+    (void)cudaGetLastError();
+    const int64_t nchunks = (h->nsq + SQT_CHUNK - 1) / SQT_CHUNK;
+    const int grid = grid_for(nchunks, 1, (int64_t)occ * h->num_sms);
+    fn<<<grid, block, smem, h->stream>>>(h->nsq, h->sq_ef, vals, h->u, h->beta, h->gh_dev, h->p_dev, h->fp_scale,
+                                         h->tacc);
+}
+
+void square_tma_launch(cualign_bp *h)
+{
+    if (h->sq_val32) square_tma_launch_v(h, h->sq_val32);
+    else square_tma_launch_v(h, h->sq_val);
+}
+
 template <bool UPDATE, bool EXACT, int SQ_U, bool HINTS, bool NOATOM = false>
 void square_launch(cualign_bp *h)
 {
@@ -435,8 +618,9 @@ cualign_status launch_square(cualign_bp *h, bool update)
         KScope ks(h, CUALIGN_K_SQUARE);
         if (update && exact) square_launch<true, true, 2, true>(h);
         else if (update) {
-            static const int var = getenv("CUALIGN_SQ_VARIANT") ? atoi(getenv("CUALIGN_SQ_VARIANT")) : 3;
-            if (var == 0) square_launch<true, false, 1, false>(h);
+            static const int var = getenv("CUALIGN_SQ_VARIANT") ? atoi(getenv("CUALIGN_SQ_VARIANT")) : 6;
+            if (var == 6) square_tma_launch(h);
+            else if (var == 0) square_launch<true, false, 1, false>(h);
             else if (var == 1) square_launch<true, false, 1, true>(h);
             else if (var == 2) square_launch<true, false, 2, false>(h);
             else if (var == 4) square_launch<true, false, 4, false>(h);

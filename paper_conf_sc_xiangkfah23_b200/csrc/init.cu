@@ -511,10 +511,10 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
     }
     // S: fill pass over this handle's rows
     CA_TRY(dalloc(h, &h->Scol, (size_t)(h->s ? h->s : 1)));
-    CA_TRY(dalloc(h, &h->sq_ef, (size_t)(h->nsq ? h->nsq : 1)));
+    CA_TRY(dalloc(h, &h->sq_ef, (size_t)h->nsq + 2)); // +2: 16-byte bulk-copy tails
     const bool fp32 = (h->flags & CUALIGN_FLAG_FP32_S) != 0;
-    if (fp32) CA_TRY(dalloc(h, &h->sq_val32, (size_t)(h->nsq ? h->nsq : 1)));
-    else CA_TRY(dalloc(h, &h->sq_val, (size_t)(h->nsq ? h->nsq : 1)));
+    if (fp32) CA_TRY(dalloc(h, &h->sq_val32, (size_t)h->nsq + 2));
+    else CA_TRY(dalloc(h, &h->sq_val, (size_t)h->nsq + 2));
     {
         KScope ks(h, CUALIGN_K_INIT);
         if (h->e1 > h->e0 && h->s) {
@@ -524,8 +524,8 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
                                                           h->sq_ef);
             CA_CUDA(cudaGetLastError());
         }
-        if (fp32) CA_CUDA(cudaMemsetAsync(h->sq_val32, 0, sizeof(float2) * (size_t)(h->nsq ? h->nsq : 1), h->stream));
-        else CA_CUDA(cudaMemsetAsync(h->sq_val, 0, sizeof(double2) * (size_t)(h->nsq ? h->nsq : 1), h->stream));
+        if (fp32) CA_CUDA(cudaMemsetAsync(h->sq_val32, 0, sizeof(float2) * ((size_t)h->nsq + 2), h->stream));
+        else CA_CUDA(cudaMemsetAsync(h->sq_val, 0, sizeof(double2) * ((size_t)h->nsq + 2), h->stream));
     }
     // the graphs are not needed after S is built
     CA_CUDA(cudaStreamSynchronize(h->stream));
