@@ -243,6 +243,41 @@ cualign_status cualign_match(const cualign_edges *L, int32_t n_a, int32_t n_b, c
                              const cualign_params *params, int32_t *mate_a, int32_t *mate_b,
                              int32_t *rounds_out);
 
+/* NEXT-4 quality harness: scores of an alignment of A to B against the
+ * network-alignment quality measures the paper uses (PAPER.md:327-333,
+ * "NCV-GS^3 ... normalized by the sizes of the networks", defined in its
+ * refs [18, 20]):
+ *   conserved = A edges {i, j} with {M(i), M(j)} in E_B  (= overlap, :60)
+ *   induced   = B edges with both ends in M(V_A)
+ *   NC   = correct / truth_total          (node correctness vs the ground truth P, :327)
+ *   EC   = conserved / |E_A|              (edge correctness)
+ *   ICS  = conserved / induced            (induced conserved structure)
+ *   S3   = conserved / (|E_A| + induced - conserved)   (symmetric substructure score)
+ *   NCV  = 2 aligned / (|V_A| + |V_B|)    (node coverage)
+ *   GS3  = S3 (one-to-one alignment)
+ *   NCV-GS3 = sqrt(NCV * GS3)
+ * A ratio with a zero denominator is 0. */
+typedef struct {
+    int64_t n_a, n_b;         /* |V_A|, |V_B| */
+    int64_t edges_a, edges_b; /* undirected edge counts */
+    int64_t aligned;          /* A vertices with an image */
+    int64_t truth_total;      /* A vertices with a true image (0 without truth) */
+    int64_t correct;          /* A vertices mapped to their true image */
+    int64_t conserved;
+    int64_t induced;
+    double nc, ec, ics, s3, ncv, gs3, ncv_gs3;
+} cualign_quality;
+
+/* Evaluate the alignment map_ab (n_A int32: B vertex of each A vertex, -1 =
+ * unaligned; must be injective) against A, B (validated like
+ * cualign_bp_init) and the optional ground truth (n_A int32, -1 = none; NULL
+ * = no truth).  Pointers are host pointers unless CUALIGN_FLAG_DEVICE_PTRS;
+ * params supplies flags / device / stream only.  EINVAL on a map entry out
+ * of range or two A vertices mapped to one B vertex. */
+cualign_status cualign_quality_eval(const cualign_graph *A, const cualign_graph *B, const int32_t *map_ab,
+                                    const int32_t *truth, const cualign_params *params,
+                                    cualign_quality *out);
+
 /* NCCL unique id for a sharded init (write len >= 128 bytes into id). */
 cualign_status cualign_nccl_unique_id(void *id, int32_t len);
 

@@ -33,7 +33,7 @@ EXPORTED = ["cualign_bp_init", "cualign_bp_iterate", "cualign_bp_round", "cualig
             "cualign_bp_set_timing", "cualign_bp_get_best",
             "cualign_bp_free", "cualign_bp_get_sizes", "cualign_bp_get_S", "cualign_bp_get_state",
             "cualign_bp_set_state", "cualign_bp_get_stats", "cualign_match", "cualign_last_error",
-            "cualign_version", "cualign_nccl_unique_id"]
+            "cualign_version", "cualign_nccl_unique_id", "cualign_quality_eval"]
 
 
 class CuAlignError(RuntimeError):
@@ -134,6 +134,8 @@ def load_library():
     lib.cualign_bp_get_stats.argtypes = [P, P, I32]
     lib.cualign_match.restype = I32
     lib.cualign_match.argtypes = [P, I32, I32, P, P, P, P, P]
+    lib.cualign_quality_eval.restype = I32
+    lib.cualign_quality_eval.argtypes = [P, P, P, P, P, P]
     lib.cualign_last_error.restype = ctypes.c_char_p
     lib.cualign_last_error.argtypes = []
     lib.cualign_version.restype = ctypes.c_char_p
@@ -337,6 +339,46 @@ def match(L, n_a, n_b, x, device=0, flags=0):
     _check(lib.cualign_match(ctypes.byref(el), int(n_a), int(n_b), _ptr(xx), ctypes.byref(prm),
                              _ptr(ma), _ptr(mb), ctypes.byref(rounds)))
     return ma[:n_a], mb[:n_b], rounds.value
+
+
+class Quality_t(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_int64) for k in ("n_a", "n_b", "edges_a", "edges_b", "aligned", "truth_total",
+                                              "correct", "conserved", "induced")] + \
+               [(k, ctypes.c_double) for k in ("nc", "ec", "ics", "s3", "ncv", "gs3", "ncv_gs3")]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+def alignment_map(mate_a, L):
+    """B vertex of each A vertex from a matching given as L edge ids (-1 = none)."""
+    mate_a = np.asarray(mate_a)
+    lb = np.asarray(L.b, dtype=np.int32)
+    return np.where(mate_a >= 0, lb[np.maximum(mate_a, 0)], -1).astype(np.int32)
+
+
+def quality(A, B, map_ab, truth=None, device=0, flags=0):
+    """NEXT-4 quality scores of the alignment map_ab (B vertex per A vertex,
+    -1 = unaligned) against A, B and the optional ground truth (see
+    cualign_quality_eval).  Returns a dict."""
+    lib = load_library()
+    Ap, dA = _prep(A.rowptr, np.int64, "int64")
+    Aj, _ = _prep(A.col, np.int32, "int32")
+    Bp, dB = _prep(B.rowptr, np.int64, "int64")
+    Bj, _ = _prep(B.col, np.int32, "int32")
+    mp, dm = _prep(map_ab, np.int32, "int32")
+    tr, dt = (None, dm) if truth is None else _prep(truth, np.int32, "int32")
+    if len({dA, dB, dm, dt}) != 1:
+        raise ValueError("inputs must be all host arrays or all device tensors")
+    if dA:
+        flags |= FLAG_DEVICE_PTRS
+    ga = Graph_t(int(A.n), _ptr(Ap), _ptr(Aj))
+    gb = Graph_t(int(B.n), _ptr(Bp), _ptr(Bj))
+    prm = Params_t(1.0, 0.0, 1.0, int(flags), int(device), None, 0, 1, None)
+    q = Quality_t()
+    _check(lib.cualign_quality_eval(ctypes.byref(ga), ctypes.byref(gb), _ptr(mp), _ptr(tr), ctypes.byref(prm),
+                                    ctypes.byref(q)))
+    return q.as_dict()
 
 
 def version():

@@ -796,4 +796,29 @@ cualign_status cualign_match(const cualign_edges *L, int32_t n_a, int32_t n_b, c
     return st;
 }
 
+cualign_status cualign_quality_eval(const cualign_graph *A, const cualign_graph *B, const int32_t *map_ab,
+                                    const int32_t *truth, const cualign_params *params, cualign_quality *out)
+{
+    API_ENTER();
+    if (!A || !B || !params || !out || (A->n > 0 && !map_ab)) {
+        set_error("cualign_quality_eval: NULL input");
+        return CUALIGN_EINVAL;
+    }
+    cualign_params prm = *params;
+    prm.alpha = 1.0;
+    prm.beta = 0.0;
+    prm.gamma = 1.0;
+    prm.rank = 0;
+    prm.world = 1;
+    prm.nccl_unique_id = nullptr;
+    prm.flags &= (CUALIGN_FLAG_DEVICE_PTRS | CUALIGN_FLAG_TIMING);
+    cualign_bp *h = nullptr;
+    cualign_status st = open_handle(&prm, &h);
+    if (st == CUALIGN_OK) st = quality_eval(h, A, B, map_ab, truth, out);
+    std::string msg = g_err;
+    close_handle(h);
+    if (st != CUALIGN_OK) set_error("%s", msg.c_str());
+    return st;
+}
+
 } // extern "C"

@@ -374,43 +374,48 @@ cualign_status build_L(cualign_bp *h, LDev &L, const cualign_edges *E, bool devi
     return CUALIGN_OK;
 }
 
+// ------------------------------------------------------------ graph upload
+cualign_status upload_graph(cualign_bp *h, const cualign_graph *g, const char *what, int64_t **rp, int32_t **col,
+                            int64_t *nnz_out)
+{
+    const bool devp = (h->flags & CUALIGN_FLAG_DEVICE_PTRS) != 0;
+    if (!g || g->n < 0 || !g->rowptr || (g->n > 0 && !g->col)) {
+        set_error("invalid %s: NULL pointer or negative n", what);
+        return CUALIGN_EINVAL;
+    }
+    // row pointers: read nnz (last entry) first
+    int64_t nnz = 0;
+    CA_CUDA(cudaMemcpy(&nnz, g->rowptr + g->n, sizeof(int64_t), devp ? cudaMemcpyDeviceToHost : cudaMemcpyHostToHost));
+    if (nnz < 0 || nnz > ((int64_t)1 << 40)) {
+        set_error("invalid %s: rowptr[n] out of range", what);
+        return CUALIGN_EINVAL;
+    }
+    KScope ks(h, CUALIGN_K_INIT);
+    CA_TRY(upload(h, (void **)rp, g->rowptr, sizeof(int64_t) * ((size_t)g->n + 1), devp));
+    CA_TRY(upload(h, (void **)col, g->col, sizeof(int32_t) * (size_t)nnz, devp));
+    TmpBuf err;
+    CA_CUDA(cudaMalloc(&err.p, sizeof(int)));
+    CA_CUDA(cudaMemsetAsync(err.p, 0, sizeof(int), h->stream));
+    if (g->n)
+        k_check_graph<<<grid_for(g->n, 256, h->num_sms * 8), 256, 0, h->stream>>>(g->n, nnz, *rp, *col,
+                                                                                   (int *)err.p);
+    CA_CUDA(cudaGetLastError());
+    CA_TRY(check_flags(h, (int *)err.p, what));
+    *nnz_out = nnz;
+    return CUALIGN_OK;
+}
+
 // ------------------------------------------------------------ problem build
 cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualign_graph *B,
                              const cualign_edges *E)
 {
     const bool devp = (h->flags & CUALIGN_FLAG_DEVICE_PTRS) != 0;
     const int G = h->num_sms * 8;
-    // graph row pointers: read nnz (last entry) first
     int64_t nnzA = 0, nnzB = 0;
-    CA_CUDA(cudaMemcpy(&nnzA, A->rowptr + A->n, sizeof(int64_t),
-                       devp ? cudaMemcpyDeviceToHost : cudaMemcpyHostToHost));
-    CA_CUDA(cudaMemcpy(&nnzB, B->rowptr + B->n, sizeof(int64_t),
-                       devp ? cudaMemcpyDeviceToHost : cudaMemcpyHostToHost));
-    if (nnzA < 0 || nnzB < 0 || nnzA > ((int64_t)1 << 40) || nnzB > ((int64_t)1 << 40)) {
-        set_error("invalid graph: rowptr[n] out of range");
-        return CUALIGN_EINVAL;
-    }
     int64_t *Ap = nullptr, *Bp = nullptr;
     int32_t *Aj = nullptr, *Bj = nullptr;
-    {
-        KScope ks(h, CUALIGN_K_INIT);
-        CA_TRY(upload(h, (void **)&Ap, A->rowptr, sizeof(int64_t) * ((size_t)A->n + 1), devp));
-        CA_TRY(upload(h, (void **)&Aj, A->col, sizeof(int32_t) * (size_t)nnzA, devp));
-        CA_TRY(upload(h, (void **)&Bp, B->rowptr, sizeof(int64_t) * ((size_t)B->n + 1), devp));
-        CA_TRY(upload(h, (void **)&Bj, B->col, sizeof(int32_t) * (size_t)nnzB, devp));
-        TmpBuf err;
-        CA_CUDA(cudaMalloc(&err.p, sizeof(int)));
-        CA_CUDA(cudaMemsetAsync(err.p, 0, sizeof(int), h->stream));
-        if (A->n)
-            k_check_graph<<<grid_for(A->n, 256, G), 256, 0, h->stream>>>(A->n, nnzA, Ap, Aj, (int *)err.p);
-        CA_CUDA(cudaGetLastError());
-        CA_TRY(check_flags(h, (int *)err.p, "graph A"));
-        CA_CUDA(cudaMemsetAsync(err.p, 0, sizeof(int), h->stream));
-        if (B->n)
-            k_check_graph<<<grid_for(B->n, 256, G), 256, 0, h->stream>>>(B->n, nnzB, Bp, Bj, (int *)err.p);
-        CA_CUDA(cudaGetLastError());
-        CA_TRY(check_flags(h, (int *)err.p, "graph B"));
-    }
+    CA_TRY(upload_graph(h, A, "graph A", &Ap, &Aj, &nnzA));
+    CA_TRY(upload_graph(h, B, "graph B", &Bp, &Bj, &nnzB));
     CA_TRY(build_L(h, h->L, E, devp, true, A->n, B->n));
     const int64_t m = h->L.m;
 

@@ -192,6 +192,8 @@ struct KScope {
 // init.cu
 cualign_status build_L(cualign_bp *h, LDev &L, const cualign_edges *E, bool device_ptrs,
                        bool validate, int32_t nA, int32_t nB);
+cualign_status upload_graph(cualign_bp *h, const cualign_graph *g, const char *what, int64_t **rp, int32_t **col,
+                            int64_t *nnz_out); // copy + validate (Z14); device CSR owned by h
 cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualign_graph *B,
                              const cualign_edges *E);
 cualign_status ensure_sq_pos(cualign_bp *h);
@@ -222,6 +224,8 @@ cualign_status bp_scatter_Sp(cualign_bp *h, double *Sfull_dev);        // square
 cualign_status bp_gather_Sp(cualign_bp *h, const double *Sfull_dev);   // CSR -> squares
 
 // match.cu
+cualign_status quality_eval(cualign_bp *h, const cualign_graph *A, const cualign_graph *B, const int32_t *map_ab,
+                            const int32_t *truth, cualign_quality *out); // NEXT-4 (quality.cu)
 cualign_status match_setup(cualign_bp *h);
 cualign_status match_round(cualign_bp *h);  // a7 + a8 on the device
 cualign_status match_standalone(cualign_bp *h, const double *x_dev, int32_t *rounds);
