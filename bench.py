@@ -379,6 +379,14 @@ def main():
                "h2d_bytes_per_step": h2d / args.e2e_iters, "d2h_bytes_per_step": d2h / args.e2e_iters,
                "align_time_s": align_time_s, "teardown_s": teardown_s, "iters": args.e2e_iters,
                "best_score": binfo["best_score"], "best_iter": binfo["best_iter"]}
+        if rank == 0:
+            # NEXT-4: quality of the best alignment against the generator's ground truth
+            try:
+                qd = ca.quality(inst.A, inst.B, ca.alignment_map(mate, inst.L),
+                                np.asarray(inst.truth, dtype=np.int32), device=dev)
+                e2e["quality"] = {k: qd[k] for k in ("nc", "ec", "ics", "s3", "ncv", "ncv_gs3")}
+            except Exception as ex:  # pragma: no cover
+                e2e["quality"] = {"error": str(ex)}
     else:
         del h
 

@@ -147,6 +147,8 @@ typedef struct {
     int32_t rank, world;      /* shard (rank -1 for a virtual-shard handle) */
     int64_t edge_begin, edge_end; /* owned canonical edge ids [begin, end) */
     int64_t squares_local;    /* squares stored by this shard */
+    int32_t merge_rounds;     /* sharded rounding (NEXT-1): merge rounds of the last round() (0 if unsharded) */
+    int32_t reserved;
 } cualign_sizes;
 
 /* Diagnostics: per-kernel-class event timing (needs CUALIGN_FLAG_TIMING) and
@@ -220,7 +222,11 @@ cualign_status cualign_bp_get_sizes(cualign_bp *h, cualign_sizes *sizes);
 cualign_status cualign_bp_get_S(cualign_bp *h, int64_t *rowptr, int32_t *col, int64_t *s_out);
 
 /* State after the last iterate (host buffers, each may be NULL):
- * yc, zc, yp, zp, d: m doubles; Sp: s doubles in get_S's CSR order; p: int. */
+ * yc, zc, yp, zp, d: m doubles; Sp: s doubles in get_S's CSR order; p: int.
+ * Sharded handles: Sp must be NULL; a virtual-shard handle assembles the
+ * owners' slices, a process shard returns arrays whose owned slice
+ * [edge_begin, edge_end) is valid (rounding is sharded too, NEXT-1, so the
+ * messages are never all-gathered). */
 cualign_status cualign_bp_get_state(cualign_bp *h, double *yc, double *zc, double *yp,
                                     double *zp, double *d, double *Sp, int32_t *p);
 

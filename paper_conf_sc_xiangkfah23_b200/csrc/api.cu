@@ -565,6 +565,7 @@ cualign_status cualign_bp_get_sizes(cualign_bp *h, cualign_sizes *sz)
     sz->edge_begin = h->vshards.empty() ? h->e0 : 0;
     sz->edge_end = h->vshards.empty() ? h->e1 : q->L.m;
     sz->squares_local = h->vshards.empty() ? h->nsq : q->nsq_total;
+    sz->merge_rounds = q->dist_rounds;
     return CUALIGN_OK;
 }
 
@@ -613,18 +614,17 @@ cualign_status cualign_bp_get_state(cualign_bp *h, double *yc, double *zc, doubl
             set_error("get_state: S^p of a sharded handle is distributed (pass Sp = NULL)");
             return CUALIGN_ESTATE;
         }
-        // y^c, z^c are all-gathered every iteration; y^p, z^p, d are valid on
-        // the owners' slices: assemble them (virtual shards) or return this
-        // process shard's arrays (owned slice valid)
+        // every per-edge vector is valid on its owner's slice: assemble the
+        // slices (virtual shards) or return this process shard's arrays (its
+        // owned slice [edge_begin, edge_end) valid)
         std::vector<cualign_bp *> S = h->vshards.empty() ? std::vector<cualign_bp *>{h} : h->vshards;
-        cualign_bp *q = S[0];
-        const size_t mb = sizeof(double) * (size_t)q->L.m;
-        if (yc && mb) CA_CUDA(cudaMemcpy(yc, q->yc, mb, cudaMemcpyDeviceToHost));
-        if (zc && mb) CA_CUDA(cudaMemcpy(zc, q->zc, mb, cudaMemcpyDeviceToHost));
+        CA_CUDA(cudaStreamSynchronize(S[0]->stream));
         for (cualign_bp *s : S) {
             const int64_t a = h->vshards.empty() ? 0 : s->e0, b = h->vshards.empty() ? s->L.m : s->e1;
             const size_t nb = sizeof(double) * (size_t)(b - a);
             if (!nb) continue;
+            if (yc) CA_CUDA(cudaMemcpy(yc + a, s->yc + a, nb, cudaMemcpyDeviceToHost));
+            if (zc) CA_CUDA(cudaMemcpy(zc + a, s->zc + a, nb, cudaMemcpyDeviceToHost));
             if (yp) CA_CUDA(cudaMemcpy(yp + a, s->yp + a, nb, cudaMemcpyDeviceToHost));
             if (zp) CA_CUDA(cudaMemcpy(zp + a, s->zp + a, nb, cudaMemcpyDeviceToHost));
             if (d) CA_CUDA(cudaMemcpy(d + a, s->d + a, nb, cudaMemcpyDeviceToHost));

@@ -139,6 +139,10 @@ struct cualign_bp {
     // matching (two instances: y and z)
     int32_t *candA = nullptr, *candB = nullptr, *mateA = nullptr, *mateB = nullptr;
     unsigned long long *suit = nullptr; // Suitor slots, 2 instances x max(nA, nB)
+    // sharded rounding (NEXT-1): replicated global suitors per (instance, B vertex)
+    unsigned long long *dist_gx = nullptr, *dist_wxl = nullptr, *dist_wxg = nullptr, *dist_cnt = nullptr;
+    int32_t *dist_gi = nullptr, *dist_wid = nullptr, *dist_hold = nullptr, *dist_act = nullptr;
+    int dist_rounds = 0; // merge rounds of the last sharded rounding
     int32_t *best_mate = nullptr;
     double *partial_w = nullptr;
     int match_grid = 0, match_block = 256, eval_grid = 1;
@@ -228,6 +232,15 @@ cualign_status quality_eval(cualign_bp *h, const cualign_graph *A, const cualign
                             const int32_t *truth, cualign_quality *out); // NEXT-4 (quality.cu)
 cualign_status match_setup(cualign_bp *h);
 cualign_status match_round(cualign_bp *h);  // a7 + a8 on the device
+cualign_status match_evaluate(cualign_bp *h); // a8 on mateA / mateB
+// sharded rounding (NEXT-1), driven by shard_round: begin, then rounds of
+// local -> all-reduce MAX(dist_wxg) -> cand -> all-reduce MIN(dist_wid) ->
+// update -> all-reduce SUM(dist_cnt) until the count is 0, then finish
+cualign_status dist_match_begin(cualign_bp *h);
+cualign_status dist_match_local(cualign_bp *h);
+cualign_status dist_match_cand(cualign_bp *h);
+cualign_status dist_match_update(cualign_bp *h);
+cualign_status dist_match_finish(cualign_bp *h);
 cualign_status match_standalone(cualign_bp *h, const double *x_dev, int32_t *rounds);
 
 // helpers

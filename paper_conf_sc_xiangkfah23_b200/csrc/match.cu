@@ -27,6 +27,7 @@
 // score = alpha*w + beta*overlap; M_y wins ties; best on a strict > (Z8).
 #include "internal.cuh"
 
+#include <climits>
 #include <cooperative_groups.h>
 
 namespace cg = cooperative_groups;
@@ -50,6 +51,13 @@ struct MatchParams {
     RoundDev *rd;
     unsigned long long *work; // proposals (suitor) / rounds, spread counters
     unsigned long long *dbg;  // optional diagnostics (CUALIGN_MATCH_DEBUG)
+    // DIST (sharded rounding, NEXT-1): the proposers are this shard's A rows
+    // [p0, p0 + nPl) with edges [e0, e1); every target slot starts a round
+    // from the global suitor (gx = fp64 bits of its weight, gi = its edge)
+    int32_t p0, nPl, e0, e1;
+    const unsigned long long *gx;
+    const int32_t *gi;
+    const int32_t *act; // active flag per (instance, local proposer)
 };
 
 constexpr int WORK_SPREAD = 64, WORK_STRIDE = 16; // counter slots, 128 B apart
@@ -88,23 +96,34 @@ __device__ __forceinline__ uint32_t suitor_key(double x)
     return __float_as_uint(__double2float_rd(x)) + 1u;
 }
 
-// does the proposal (xe, e) with key ke beat the occupant slot s?
-__device__ __forceinline__ bool beats(const double *__restrict__ x, double xe, int e, uint32_t ke,
-                                      unsigned long long s)
+// does the proposal (xe, e) with key ke beat the occupant slot s of target t?
+// The occupant's exact weight (needed only on equal keys) is x[es] for an
+// edge of this process; in DIST mode an occupant from another shard can only
+// be the round's initial global suitor, whose weight is gx[t].
+template <bool DIST>
+__device__ __forceinline__ bool beats(const MatchParams &P, const double *__restrict__ x, int k, int64_t nT, int t,
+                                      double xe, int e, uint32_t ke, unsigned long long s)
 {
     if (s == 0ull) return true;
     const uint32_t ks = (uint32_t)(s >> 32);
     if (ke != ks) return ke > ks;
     const int es = (int)(uint32_t)s;
-    return better(xe, e, __ldg(x + es), es);
+    double xs;
+    if (DIST && es == P.gi[k * nT + t]) xs = __longlong_as_double((long long)P.gx[k * nT + t]);
+    else xs = __ldg(x + es);
+    return better(xe, e, xs, es);
 }
 
-template <int G, int U, class Tile>
+template <int G, int U, bool DIST, class Tile>
 __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
                                             int64_t nT, int64_t slot)
 {
     const int k = (int)(slot / nP);
     int cur = (int)(slot - k * nP);
+    if (DIST) {
+        if (!P.act[slot]) return; // settled (or exhausted) in an earlier round
+        cur += P.p0;
+    }
     const double *__restrict__ x = xk(P, k);
     unsigned long long *sT = P.suit + k * nT;
     const int64_t *__restrict__ rp = fromB ? P.Bptr : P.Arow;
@@ -142,7 +161,7 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
 #pragma unroll
             for (int u = 0; u < U; u++) {
                 if (ee[u] < 0) continue;
-                if (filter && !beats(x, xx[u], ee[u], suitor_key(xx[u]), ss[u])) continue;
+                if (filter && !beats<DIST>(P, x, k, nT, tt[u], xx[u], ee[u], suitor_key(xx[u]), ss[u])) continue;
                 if (better(xx[u], ee[u], bx, best)) {
                     best = ee[u];
                     bx = xx[u];
@@ -163,21 +182,23 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
         int code = 0;        // 0 rescan, 1 done, 2 displaced
         int next = cur;
         if (lane == 0) {
-            unsigned long long *slotp = sT + __ldg(tgt + best);
+            const int tb = __ldg(tgt + best);
+            unsigned long long *slotp = sT + tb;
             const uint32_t kb = suitor_key(bx);
             const unsigned long long mine = ((unsigned long long)kb << 32) | (uint32_t)best;
             unsigned long long s = *(volatile unsigned long long *)slotp;
             // CAS loop: retry directly while our edge still beats the occupant,
             // rescan the list only when it does not
-            while (beats(x, bx, best, kb, s)) {
+            while (beats<DIST>(P, x, k, nT, tb, bx, best, kb, s)) {
                 const unsigned long long old = atomicCAS(slotp, s, mine);
                 if (old == s) {
                     proposals++;
-                    if (s == 0ull) {
-                        code = 1;
+                    const int es = (int)(uint32_t)s;
+                    if (s == 0ull || (DIST && (es < P.e0 || es >= P.e1))) {
+                        code = 1; // free slot, or another shard's suitor (its owner re-proposes)
                     } else {
                         code = 2;
-                        next = __ldg(own + (int)(uint32_t)s); // the displaced proposer proposes again
+                        next = __ldg(own + es); // the displaced proposer proposes again
                     }
                     break;
                 }
@@ -200,16 +221,108 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
     }
 }
 
-template <int G, int U>
+template <int G, int U, bool DIST = false>
 __global__ void __launch_bounds__(128) k_suitor(MatchParams P)
 {
     auto tile = cg::tiled_partition<G>(cg::this_thread_block());
     const int lane = tile.thread_rank();
-    const bool fromB = P.propose_from_b != 0;
-    const int64_t nP = fromB ? P.nB : P.nA;
+    const bool fromB = !DIST && P.propose_from_b != 0;
+    const int64_t nP = DIST ? P.nPl : (fromB ? P.nB : P.nA);
     const int64_t nT = fromB ? P.nA : P.nB;
     const int64_t slot = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G;
-    if (slot < P.ninst * nP) suitor_tile<G, U>(P, tile, lane, fromB, nP, nT, slot);
+    if (slot < P.ninst * nP) suitor_tile<G, U, DIST>(P, tile, lane, fromB, nP, nT, slot);
+}
+
+// ------------------------------------------------- DIST round helper kernels
+// slots of a round start from the global suitors
+__global__ void k_dist_init_slots(int64_t n, const unsigned long long *__restrict__ gx, const int32_t *__restrict__ gi,
+                                  unsigned long long *__restrict__ sT)
+{
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const int e = gi[v];
+        sT[v] = e < 0 ? 0ull
+                      : ((unsigned long long)suitor_key(__longlong_as_double((long long)gx[v])) << 32) | (uint32_t)e;
+    }
+}
+
+// local winner per target -> (weight bits, edge) for the global merge; x > 0
+// for every suitor, so the fp64 bits order like the weights
+__global__ void k_dist_pack(int64_t nB, const unsigned long long *__restrict__ sT, const unsigned long long *__restrict__ gx,
+                            const int32_t *__restrict__ gi, const double *__restrict__ x0, const double *__restrict__ x1,
+                            unsigned long long *__restrict__ wxl, unsigned long long *__restrict__ wxg,
+                            int32_t *__restrict__ wid)
+{
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < 2 * nB; v += (int64_t)gridDim.x * blockDim.x) {
+        const unsigned long long s = sT[v];
+        unsigned long long bits = 0ull;
+        int32_t e = INT_MAX;
+        if (s) {
+            e = (int32_t)(uint32_t)s;
+            bits = (e == gi[v]) ? gx[v] : (unsigned long long)__double_as_longlong((v < nB ? x0 : x1)[e]);
+        }
+        wxl[v] = bits;
+        wxg[v] = bits;
+        wid[v] = e;
+    }
+}
+
+// among the shards whose winner has the global max weight, the lowest edge id wins (Z7)
+__global__ void k_dist_cand(int64_t n, const unsigned long long *__restrict__ wxl, const unsigned long long *__restrict__ wxg,
+                            int32_t *__restrict__ wid)
+{
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        if (!(wxl[v] != 0ull && wxl[v] == wxg[v])) wid[v] = INT_MAX;
+}
+
+// new global suitors; which local proposers hold a local slot
+__global__ void k_dist_update(int64_t nB, const unsigned long long *__restrict__ wxg, const int32_t *__restrict__ wid,
+                              unsigned long long *__restrict__ gx, int32_t *__restrict__ gi,
+                              const unsigned long long *__restrict__ sT, const int32_t *__restrict__ La, int32_t e0,
+                              int32_t e1, int32_t p0, int32_t nPl, int32_t *__restrict__ hold)
+{
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < 2 * nB; v += (int64_t)gridDim.x * blockDim.x) {
+        gx[v] = wxg[v];
+        gi[v] = wid[v] == INT_MAX ? -1 : wid[v];
+        const unsigned long long s = sT[v];
+        if (s) {
+            const int e = (int)(uint32_t)s;
+            if (e >= e0 && e < e1) hold[(v < nB ? 0 : nPl) + (La[e] - p0)] = e;
+        }
+    }
+}
+
+// a local proposer is active next round iff it holds a slot locally that is
+// not the global suitor (displaced by another shard); count the active ones
+__global__ void k_dist_active(int32_t nPl, int64_t nB, const int32_t *__restrict__ hold,
+                              const int32_t *__restrict__ gi, const int32_t *__restrict__ Lb,
+                              int32_t *__restrict__ act, unsigned long long *__restrict__ cnt)
+{
+    unsigned long long c = 0;
+    for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < 2 * (int64_t)nPl;
+         j += (int64_t)gridDim.x * blockDim.x) {
+        const int e = hold[j];
+        const int k = j < nPl ? 0 : 1;
+        const int a = (e >= 0 && gi[k * nB + Lb[e]] != e) ? 1 : 0;
+        act[j] = a;
+        c += a;
+    }
+    for (int off = 16; off >= 1; off >>= 1) c += __shfl_down_sync(0xffffffffu, c, off);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(cnt, c);
+}
+
+__global__ void k_dist_mates(int64_t nB, int64_t nA, const int32_t *__restrict__ gi, const int32_t *__restrict__ La,
+                             int32_t *__restrict__ mateA, int32_t *__restrict__ mateB)
+{
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < 2 * nB; v += (int64_t)gridDim.x * blockDim.x) {
+        const int e = gi[v];
+        mateB[v] = e;
+        if (e >= 0) mateA[(v < nB ? 0 : nA) + La[e]] = e;
+    }
+}
+
+__global__ void k_fill_i32(int64_t n, int32_t *__restrict__ x, int32_t v)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) x[i] = v;
 }
 
 // the final suitor of each target is its mate (mate arrays pre-set to -1)
@@ -674,6 +787,124 @@ cualign_status match_round(cualign_bp *h)
     P.x0 = damped ? h->yp : h->yc;
     P.x1 = damped ? h->zp : h->zc;
     CA_TRY(run_matching(h, P));
+    return match_evaluate(h);
+}
+
+// ------------------------------------------------ sharded rounding (NEXT-1)
+// Deferred acceptance in rounds across shards.  Every
+// shard proposes only from its own A rows (so it needs y^c, z^c only on its
+// own edges -- no all-gather of the messages); the targets' suitors are kept
+// replicated as (weight bits, edge id) per B vertex.  A round: each shard runs
+// the Suitor kernel for its active proposers against slots initialised with
+// the global suitors (local displacement chains resolve inside the round),
+// then the local winners are merged: all-reduce MAX of the weight bits, then
+// all-reduce MIN of the edge id among the shards holding that weight (lowest
+// index wins, Z7).  A proposer whose slot went to another shard is active in
+// the next round; rounds end when no shard has an active proposer.  The
+// stable matching under one strict edge order is unique, so the result is the
+// single-GPU (greedy) matching bit for bit; evaluation is then replicated.
+static MatchParams dist_params(cualign_bp *h)
+{
+    MatchParams P = base_params(h);
+    const bool damped = (h->flags & CUALIGN_FLAG_ROUND_DAMPED) != 0;
+    P.ninst = 2;
+    P.x0 = damped ? h->yp : h->yc;
+    P.x1 = damped ? h->zp : h->zc;
+    P.propose_from_b = 0;
+    P.p0 = h->a0;
+    P.nPl = h->a1 - h->a0;
+    P.e0 = (int32_t)h->e0;
+    P.e1 = (int32_t)h->e1;
+    P.gx = h->dist_gx;
+    P.gi = h->dist_gi;
+    P.act = h->dist_act;
+    return P;
+}
+
+cualign_status dist_match_begin(cualign_bp *h)
+{
+    const size_t nB = (size_t)h->L.nB, nPl = (size_t)(h->a1 - h->a0);
+    if (!h->dist_gx) {
+        CA_TRY(dalloc(h, &h->dist_gx, 2 * nB + 1));
+        CA_TRY(dalloc(h, &h->dist_wxl, 2 * nB + 1));
+        CA_TRY(dalloc(h, &h->dist_wxg, 2 * nB + 1));
+        CA_TRY(dalloc(h, &h->dist_gi, 2 * nB + 1));
+        CA_TRY(dalloc(h, &h->dist_wid, 2 * nB + 1));
+        CA_TRY(dalloc(h, &h->dist_hold, 2 * nPl + 1));
+        CA_TRY(dalloc(h, &h->dist_act, 2 * nPl + 1));
+        CA_TRY(dalloc(h, &h->dist_cnt, 1));
+    }
+    const int G = h->num_sms * 8;
+    CA_CUDA(cudaMemsetAsync(h->match_work, 0, WORK_SPREAD * WORK_STRIDE * sizeof(unsigned long long), h->stream));
+    CA_CUDA(cudaMemsetAsync(h->dist_gx, 0, sizeof(unsigned long long) * (2 * nB + 1), h->stream));
+    k_fill_i32<<<grid_for((int64_t)(2 * nB + 1), 256, G), 256, 0, h->stream>>>((int64_t)(2 * nB + 1), h->dist_gi, -1);
+    k_fill_i32<<<grid_for((int64_t)(2 * nPl + 1), 256, G), 256, 0, h->stream>>>((int64_t)(2 * nPl + 1), h->dist_act, 1);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
+cualign_status dist_match_local(cualign_bp *h)
+{
+    MatchParams P = dist_params(h);
+    const int64_t nB = h->L.nB, slots = 2 * (int64_t)P.nPl;
+    const int G = h->num_sms * 8;
+    KScope ks(h, CUALIGN_K_MATCH);
+    k_dist_init_slots<<<grid_for(2 * nB, 256, G), 256, 0, h->stream>>>(2 * nB, h->dist_gx, h->dist_gi, h->suit);
+    if (slots > 0) {
+        const int64_t dmax = h->max_deg_a;
+        if (dmax > 64) k_suitor<32, 2, true><<<grid_for(slots * 32, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else if (dmax > 24) k_suitor<16, 2, true><<<grid_for(slots * 16, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else if (dmax > 20) k_suitor<8, 3, true><<<grid_for(slots * 8, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else k_suitor<4, 5, true><<<grid_for(slots * 4, 128, 1 << 30), 128, 0, h->stream>>>(P);
+    }
+    k_dist_pack<<<grid_for(2 * nB, 256, G), 256, 0, h->stream>>>(nB, h->suit, h->dist_gx, h->dist_gi, P.x0, P.x1,
+                                                                 h->dist_wxl, h->dist_wxg, h->dist_wid);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
+cualign_status dist_match_cand(cualign_bp *h)
+{
+    const int64_t n = 2 * (int64_t)h->L.nB;
+    k_dist_cand<<<grid_for(n, 256, h->num_sms * 8), 256, 0, h->stream>>>(n, h->dist_wxl, h->dist_wxg, h->dist_wid);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
+cualign_status dist_match_update(cualign_bp *h)
+{
+    const int64_t nB = h->L.nB;
+    const int32_t nPl = h->a1 - h->a0;
+    const int G = h->num_sms * 8;
+    k_fill_i32<<<grid_for(2 * (int64_t)nPl + 1, 256, G), 256, 0, h->stream>>>(2 * (int64_t)nPl + 1, h->dist_hold, -1);
+    k_dist_update<<<grid_for(2 * nB, 256, G), 256, 0, h->stream>>>(nB, h->dist_wxg, h->dist_wid, h->dist_gx,
+                                                                   h->dist_gi, h->suit, h->L.La, (int32_t)h->e0,
+                                                                   (int32_t)h->e1, h->a0, nPl, h->dist_hold);
+    CA_CUDA(cudaMemsetAsync(h->dist_cnt, 0, sizeof(unsigned long long), h->stream));
+    if (nPl > 0)
+        k_dist_active<<<grid_for(2 * (int64_t)nPl, 256, G), 256, 0, h->stream>>>(nPl, nB, h->dist_hold, h->dist_gi,
+                                                                                 h->L.Lb, h->dist_act, h->dist_cnt);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
+cualign_status dist_match_finish(cualign_bp *h)
+{
+    const int64_t nA = h->L.nA, nB = h->L.nB;
+    CA_CUDA(cudaMemsetAsync(h->mateA, 0xff, sizeof(int32_t) * (size_t)(2 * nA + 1), h->stream));
+    {
+        KScope ks(h, CUALIGN_K_MATCHAUX);
+        if (nB)
+            k_dist_mates<<<grid_for(2 * nB, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB, nA, h->dist_gi, h->L.La,
+                                                                                       h->mateA, h->mateB);
+        CA_CUDA(cudaGetLastError());
+    }
+    return match_evaluate(h);
+}
+
+// a8 (evaluate + best) of the matchings in mateA / mateB
+cualign_status match_evaluate(cualign_bp *h)
+{
     EvalParams E{};
     E.nA = h->L.nA;
     E.Lb = h->L.Lb;

@@ -7,13 +7,14 @@
 // entries of y^p, z^p, d.  Per iteration the exchanges are:
 //   1. B-side top-2: every shard reduces its owned edges per B vertex; the
 //      partials are all-gathered and merged (max is exact).
-//   2. u, y^c, z^c: each shard's owned slice is all-gathered (the square pass
-//      needs u_f of any f; rounding needs the full y^c, z^c).
+//   2. u: each shard's owned slice is all-gathered (the square pass needs
+//      u_f of any f).
 //   3. F row sums: each shard accumulates fixed-point partial sums for every
 //      edge; the slices are reduce-scattered to their owners.  Integer sums
 //      are associative, so the result is bitwise the single-GPU one.
-//   Rounding (a7, a8) is replicated on every shard (identical inputs, same
-//   deterministic kernels).
+//   Rounding (a7) is sharded (NEXT-1, see match.cu dist_match_*): proposals
+//   from the owned A rows, per-round all-reduces of the B-side suitors; the
+//   final matching and its evaluation (a8) are then replicated.
 // Two transports implement the exchanges: NCCL between processes (one shard
 // per GPU, communicator from a unique id broadcast by torch.distributed), and
 // an in-process loopback that holds several virtual shards on one device
@@ -40,6 +41,8 @@ struct NcclApi {
     ncclResult_t (*Broadcast)(const void *, void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
     ncclResult_t (*Reduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, int, ncclComm_t,
                            cudaStream_t) = nullptr;
+    ncclResult_t (*AllReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                              cudaStream_t) = nullptr;
     ncclResult_t (*GroupStart)() = nullptr;
     ncclResult_t (*GroupEnd)() = nullptr;
     const char *(*GetErrorString)(ncclResult_t) = nullptr;
@@ -59,11 +62,12 @@ NcclApi &nccl()
             api.AllGather = (decltype(api.AllGather))dlsym(lib, "ncclAllGather");
             api.Broadcast = (decltype(api.Broadcast))dlsym(lib, "ncclBroadcast");
             api.Reduce = (decltype(api.Reduce))dlsym(lib, "ncclReduce");
+            api.AllReduce = (decltype(api.AllReduce))dlsym(lib, "ncclAllReduce");
             api.GroupStart = (decltype(api.GroupStart))dlsym(lib, "ncclGroupStart");
             api.GroupEnd = (decltype(api.GroupEnd))dlsym(lib, "ncclGroupEnd");
             api.GetErrorString = (decltype(api.GetErrorString))dlsym(lib, "ncclGetErrorString");
             api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.AllGather && api.Broadcast &&
-                     api.Reduce && api.GroupStart && api.GroupEnd && api.GetErrorString;
+                     api.Reduce && api.AllReduce && api.GroupStart && api.GroupEnd && api.GetErrorString;
         }
     }
     return api;
@@ -83,12 +87,35 @@ NcclApi &nccl()
         }                                                                                      \
     } while (0)
 
+enum RedOp { RED_MAX_U64, RED_MIN_I32, RED_SUM_U64 };
+
 struct Exchange {
     virtual ~Exchange() {}
     virtual cualign_status top2(std::vector<cualign_bp *> &S) = 0;
     virtual cualign_status allgather(std::vector<cualign_bp *> &S, double *cualign_bp::*field) = 0;
     virtual cualign_status reduce_t(std::vector<cualign_bp *> &S) = 0;
+    // in-place all-reduce of an array of n entries held by every shard
+    virtual cualign_status allreduce(std::vector<cualign_bp *> &S, void *(*field)(cualign_bp *), int64_t n,
+                                     RedOp op) = 0;
 };
+
+__global__ void k_red_max_u64(int64_t n, unsigned long long *dst, const unsigned long long *src)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        if (src[i] > dst[i]) dst[i] = src[i];
+}
+__global__ void k_red_min_i32(int64_t n, int32_t *dst, const int32_t *src)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        if (src[i] < dst[i]) dst[i] = src[i];
+}
+__global__ void k_red_sum_u64(int64_t n, unsigned long long *dst, const unsigned long long *src)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dst[i] += src[i];
+}
+
+size_t red_size(RedOp op) { return op == RED_MIN_I32 ? sizeof(int32_t) : sizeof(unsigned long long); }
 
 cualign_status zero_unowned(cualign_bp *q)
 {
@@ -135,6 +162,27 @@ struct Loopback : Exchange {
         for (cualign_bp *q : S) CA_TRY(zero_unowned(q));
         return CUALIGN_OK;
     }
+    cualign_status allreduce(std::vector<cualign_bp *> &S, void *(*field)(cualign_bp *), int64_t n,
+                             RedOp op) override
+    {
+        // fold every shard into shard 0 (fixed order), then copy back
+        cualign_bp *h = S[0];
+        void *dst = field(h);
+        const int grid = grid_for(n, 256, h->num_sms * 8);
+        for (size_t r = 1; r < S.size() && n; r++) {
+            const void *src = field(S[r]);
+            if (op == RED_MAX_U64)
+                k_red_max_u64<<<grid, 256, 0, h->stream>>>(n, (unsigned long long *)dst, (const unsigned long long *)src);
+            else if (op == RED_MIN_I32)
+                k_red_min_i32<<<grid, 256, 0, h->stream>>>(n, (int32_t *)dst, (const int32_t *)src);
+            else
+                k_red_sum_u64<<<grid, 256, 0, h->stream>>>(n, (unsigned long long *)dst, (const unsigned long long *)src);
+            CA_CUDA(cudaGetLastError());
+        }
+        for (size_t r = 1; r < S.size() && n; r++)
+            CA_CUDA(cudaMemcpyAsync(field(S[r]), dst, red_size(op) * (size_t)n, cudaMemcpyDeviceToDevice, h->stream));
+        return CUALIGN_OK;
+    }
 };
 
 // -------------------------------------------------------------------- NCCL
@@ -174,6 +222,17 @@ struct Nccl : Exchange {
         CA_NCCL(GroupEnd());
         return zero_unowned(h);
     }
+    cualign_status allreduce(std::vector<cualign_bp *> &S, void *(*field)(cualign_bp *), int64_t n,
+                             RedOp op) override
+    {
+        cualign_bp *h = S[0];
+        void *buf = field(h);
+        if (!n) return CUALIGN_OK;
+        const ncclDataType_t t = op == RED_MIN_I32 ? ncclInt32 : ncclUint64;
+        const ncclRedOp_t o = op == RED_MAX_U64 ? ncclMax : (op == RED_MIN_I32 ? ncclMin : ncclSum);
+        CA_NCCL(AllReduce(buf, buf, (size_t)n, t, o, (ncclComm_t)h->comm, h->stream));
+        return CUALIGN_OK;
+    }
 };
 
 Exchange *exchange_for(cualign_bp *h, std::vector<cualign_bp *> &S)
@@ -202,19 +261,12 @@ cualign_status shard_iterate(cualign_bp *h, int32_t n)
 {
     std::vector<cualign_bp *> S;
     Exchange *X = exchange_for(h, S);
-    const bool damped = (S[0]->flags & CUALIGN_FLAG_ROUND_DAMPED) != 0;
     for (cualign_bp *s : S) CA_TRY(ensure_gh(s, (int64_t)s->p + n));
     for (int32_t k = 0; k < n; k++) {
         for (cualign_bp *s : S) CA_TRY(bp_front_top2(s));
         CA_TRY(X->top2(S));
         for (cualign_bp *s : S) CA_TRY(bp_front_edge(s));
         CA_TRY(X->allgather(S, &cualign_bp::u));
-        CA_TRY(X->allgather(S, &cualign_bp::yc));
-        CA_TRY(X->allgather(S, &cualign_bp::zc));
-        if (damped) {
-            CA_TRY(X->allgather(S, &cualign_bp::yp));
-            CA_TRY(X->allgather(S, &cualign_bp::zp));
-        }
         for (cualign_bp *s : S) CA_TRY(bp_iterate_back(s));
         CA_TRY(X->reduce_t(S));
         for (cualign_bp *s : S) s->p += 1;
@@ -225,8 +277,32 @@ cualign_status shard_iterate(cualign_bp *h, int32_t n)
 
 cualign_status shard_round(cualign_bp *h)
 {
-    if (h->vshards.empty()) return match_round(h);
-    for (cualign_bp *s : h->vshards) CA_TRY(match_round(s));
+    std::vector<cualign_bp *> S;
+    Exchange *X = exchange_for(h, S);
+    const int64_t n2B = 2 * (int64_t)S[0]->L.nB;
+    for (cualign_bp *s : S) CA_TRY(dist_match_begin(s));
+    int rounds = 0;
+    while (true) {
+        for (cualign_bp *s : S) CA_TRY(dist_match_local(s));
+        CA_TRY(X->allreduce(S, [](cualign_bp *q) -> void * { return q->dist_wxg; }, n2B, RED_MAX_U64));
+        for (cualign_bp *s : S) CA_TRY(dist_match_cand(s));
+        CA_TRY(X->allreduce(S, [](cualign_bp *q) -> void * { return q->dist_wid; }, n2B, RED_MIN_I32));
+        for (cualign_bp *s : S) CA_TRY(dist_match_update(s));
+        CA_TRY(X->allreduce(S, [](cualign_bp *q) -> void * { return q->dist_cnt; }, 1, RED_SUM_U64));
+        unsigned long long active = 0;
+        CA_CUDA(cudaMemcpyAsync(&active, S[0]->dist_cnt, sizeof(active), cudaMemcpyDeviceToHost, S[0]->stream));
+        CA_CUDA(cudaStreamSynchronize(S[0]->stream));
+        rounds++;
+        if (!active) break;
+        if (rounds > (1 << 24)) {
+            set_error("sharded rounding did not converge");
+            return CUALIGN_ECUDA;
+        }
+    }
+    for (cualign_bp *s : S) {
+        s->dist_rounds = rounds;
+        CA_TRY(dist_match_finish(s));
+    }
     return CUALIGN_OK;
 }
 
