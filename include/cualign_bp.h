@@ -284,6 +284,20 @@ cualign_status cualign_quality_eval(const cualign_graph *A, const cualign_graph 
                                     const int32_t *truth, const cualign_params *params,
                                     cualign_quality *out);
 
+/* NEXT-2: kNN sparsification -- L from given embeddings, Alg. 1 lines 7-14
+ * (PAPER.md:133-140, :121): s(u, v) = cosine similarity of Y_A(u) and Y_B(v)
+ * (l.9) for all pairs, and for every A vertex the k most similar B vertices
+ * (reading Z19; ties to the lower B index).  YA (n_a x d) and YB (n_b x d) are
+ * row-major fp32 (host, or device with CUDA_FLAG_DEVICE_PTRS), 1 <= d <= 256,
+ * 1 <= k <= min(32, n_b), all entries finite (EINVAL otherwise).  A zero row
+ * has similarity 0 with everything.  Writes m = n_a * k edges into the
+ * caller's L_a, L_b (int32) and L_w (double, the similarity) in canonical
+ * order (a ascending, then b ascending) -- ready for cualign_bp_init.
+ * Precision: tensor-core products of the unit rows rounded to bf16, fp32
+ * accumulation. */
+cualign_status cualign_knn(const float *YA, int32_t n_a, const float *YB, int32_t n_b, int32_t d, int32_t k,
+                           const cualign_params *params, int32_t *L_a, int32_t *L_b, double *L_w);
+
 /* NCCL unique id for a sharded init (write len >= 128 bytes into id). */
 cualign_status cualign_nccl_unique_id(void *id, int32_t len);
 

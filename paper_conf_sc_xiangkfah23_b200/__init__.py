@@ -6,7 +6,7 @@ the end-to-end `align` helper and the sharded (multi-GPU) driver.
 """
 import time
 
-from ._lib import (CuAlignBP, CuAlignError, match, quality, alignment_map, load_library, version, nccl_unique_id,
+from ._lib import (CuAlignBP, CuAlignError, match, quality, alignment_map, knn, KnnCandidates, load_library, version, nccl_unique_id,
                    FLAG_DEVICE_PTRS, FLAG_EXACT, FLAG_OTHERMAX_LITERAL, FLAG_ROUND_DAMPED,
                    FLAG_TIMING, FLAG_MATCH_ROUNDS, FLAG_FP32_S, EXPORTED, LIB_PATH, KERNEL_CLASS_NAMES)
 
@@ -25,6 +25,6 @@ def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=
     return mate, info, infos
 
 
-__all__ = ["CuAlignBP", "CuAlignError", "match", "quality", "alignment_map", "align", "load_library", "version", "nccl_unique_id",
+__all__ = ["CuAlignBP", "CuAlignError", "match", "quality", "alignment_map", "knn", "KnnCandidates", "align", "load_library", "version", "nccl_unique_id",
            "FLAG_DEVICE_PTRS", "FLAG_EXACT", "FLAG_OTHERMAX_LITERAL", "FLAG_ROUND_DAMPED",
            "FLAG_TIMING", "FLAG_MATCH_ROUNDS", "FLAG_FP32_S", "EXPORTED", "LIB_PATH", "KERNEL_CLASS_NAMES"]

@@ -33,7 +33,7 @@ EXPORTED = ["cualign_bp_init", "cualign_bp_iterate", "cualign_bp_round", "cualig
             "cualign_bp_set_timing", "cualign_bp_get_best",
             "cualign_bp_free", "cualign_bp_get_sizes", "cualign_bp_get_S", "cualign_bp_get_state",
             "cualign_bp_set_state", "cualign_bp_get_stats", "cualign_match", "cualign_last_error",
-            "cualign_version", "cualign_nccl_unique_id", "cualign_quality_eval"]
+            "cualign_version", "cualign_nccl_unique_id", "cualign_quality_eval", "cualign_knn"]
 
 
 class CuAlignError(RuntimeError):
@@ -134,6 +134,8 @@ def load_library():
     lib.cualign_bp_get_stats.argtypes = [P, P, I32]
     lib.cualign_match.restype = I32
     lib.cualign_match.argtypes = [P, I32, I32, P, P, P, P, P]
+    lib.cualign_knn.restype = I32
+    lib.cualign_knn.argtypes = [P, I32, P, I32, I32, I32, P, P, P, P]
     lib.cualign_quality_eval.restype = I32
     lib.cualign_quality_eval.argtypes = [P, P, P, P, P, P]
     lib.cualign_last_error.restype = ctypes.c_char_p
@@ -379,6 +381,57 @@ def quality(A, B, map_ab, truth=None, device=0, flags=0):
     _check(lib.cualign_quality_eval(ctypes.byref(ga), ctypes.byref(gb), _ptr(mp), _ptr(tr), ctypes.byref(prm),
                                     ctypes.byref(q)))
     return q.as_dict()
+
+
+class KnnCandidates:
+    """L built by knn(): m = n_a * k edges in canonical (a, b) order."""
+
+    def __init__(self, n_a, n_b, a, b, w):
+        self.n_a, self.n_b, self.a, self.b, self.w = int(n_a), int(n_b), a, b, w
+
+    @property
+    def m(self):
+        return int(self.a.shape[0])
+
+
+def knn(YA, YB, k, device=0, flags=0):
+    """NEXT-2: L from embeddings (cualign_knn): the k most cosine-similar B
+    vertices of every A vertex, on the tensor cores.  YA (n_a x d), YB
+    (n_b x d): float32 host arrays or CUDA tensors (then the result is CUDA
+    tensors too)."""
+    lib = load_library()
+    if _is_torch(YA) != _is_torch(YB):
+        raise ValueError("YA and YB must both be host arrays or both be tensors")
+    if _is_torch(YA):
+        import torch
+        ya, yb = YA.to(torch.float32).contiguous(), YB.to(torch.float32).contiguous()
+        n_a, d = ya.shape
+        n_b = yb.shape[0]
+        if ya.is_cuda != yb.is_cuda:
+            raise ValueError("YA and YB must be on the same side")
+        dev = ya.is_cuda
+    else:
+        ya, yb = _as_host(YA, np.float32), _as_host(YB, np.float32)
+        n_a, d = ya.shape
+        n_b = yb.shape[0]
+        dev = False
+    if yb.shape[1] != d:
+        raise ValueError("YA and YB need the same embedding dimension")
+    m = n_a * k
+    if dev:
+        import torch
+        flags |= FLAG_DEVICE_PTRS
+        a = torch.empty(max(m, 1), dtype=torch.int32, device=ya.device)
+        b = torch.empty(max(m, 1), dtype=torch.int32, device=ya.device)
+        w = torch.empty(max(m, 1), dtype=torch.float64, device=ya.device)
+    else:
+        a = np.empty(max(m, 1), dtype=np.int32)
+        b = np.empty(max(m, 1), dtype=np.int32)
+        w = np.empty(max(m, 1), dtype=np.float64)
+    prm = Params_t(1.0, 0.0, 1.0, int(flags), int(device), None, 0, 1, None)
+    _check(lib.cualign_knn(_ptr(ya), int(n_a), _ptr(yb), int(n_b), int(d), int(k), ctypes.byref(prm),
+                           _ptr(a), _ptr(b), _ptr(w)))
+    return KnnCandidates(n_a, n_b, a[:m], b[:m], w[:m])
 
 
 def version():

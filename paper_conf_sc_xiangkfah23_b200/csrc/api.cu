@@ -821,4 +821,33 @@ cualign_status cualign_quality_eval(const cualign_graph *A, const cualign_graph 
     return st;
 }
 
+cualign_status cualign_knn(const float *YA, int32_t n_a, const float *YB, int32_t n_b, int32_t d, int32_t k,
+                           const cualign_params *params, int32_t *L_a, int32_t *L_b, double *L_w)
+{
+    API_ENTER();
+    if (!params || n_a < 0 || n_b < 0 || (n_a > 0 && (!YA || !L_a || !L_b || !L_w)) || (n_b > 0 && !YB)) {
+        set_error("cualign_knn: NULL or negative-size input");
+        return CUALIGN_EINVAL;
+    }
+    if (d < 1 || d > 256 || k < 1 || k > 32 || (n_a > 0 && k > n_b)) {
+        set_error("cualign_knn: need 1 <= d <= 256, 1 <= k <= min(32, n_b) (d = %d, k = %d, n_b = %d)", d, k, n_b);
+        return CUALIGN_EINVAL;
+    }
+    cualign_params prm = *params;
+    prm.alpha = 1.0;
+    prm.beta = 0.0;
+    prm.gamma = 1.0;
+    prm.rank = 0;
+    prm.world = 1;
+    prm.nccl_unique_id = nullptr;
+    prm.flags &= (CUALIGN_FLAG_DEVICE_PTRS | CUALIGN_FLAG_TIMING);
+    cualign_bp *h = nullptr;
+    cualign_status st = open_handle(&prm, &h);
+    if (st == CUALIGN_OK) st = knn_build(h, YA, n_a, YB, n_b, d, k, L_a, L_b, L_w);
+    std::string msg = g_err;
+    close_handle(h);
+    if (st != CUALIGN_OK) set_error("%s", msg.c_str());
+    return st;
+}
+
 } // extern "C"

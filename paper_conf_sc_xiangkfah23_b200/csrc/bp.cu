@@ -28,6 +28,7 @@
 // integer sum (exact per term to 2^-fp_bits, deterministic, see DESIGN.md
 // "Row sums"); CUALIGN_FLAG_EXACT sums in the oracle's order instead.
 #include "internal.cuh"
+#include "ptx.cuh"
 
 #include <cooperative_groups.h>
 #include <cub/cub.cuh>
@@ -362,40 +363,7 @@ constexpr int SQT_STAGES = 4;
 constexpr int SQT_CWARPS = 8;             // consumer warps; + 1 producer warp
 constexpr int SQT_PER_THREAD = SQT_CHUNK / (SQT_CWARPS * 32);
 
-__device__ __forceinline__ uint32_t smem_addr(const void *p)
-{
-    return (uint32_t)__cvta_generic_to_shared(p);
-}
-__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count)
-{
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes)
-{
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes)
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t *bar)
-{
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
-{
-    asm volatile("{\n\t.reg .pred p;\n"
-                 "MBAR_WAIT_%=:\n\t"
-                 "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-                 "@!p bra MBAR_WAIT_%=;\n}\n" ::"r"(smem_addr(bar)),
-                 "r"(parity)
-                 : "memory");
-}
-__device__ __forceinline__ void bulk_load(void *dst, const void *src, uint32_t bytes, uint64_t *bar,
-                                          uint64_t policy)
-{
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
-                 " [%0], [%1], %2, [%3], %4;" ::"r"(smem_addr(dst)),
-                 "l"(src), "r"(bytes), "r"(smem_addr(bar)), "l"(policy)
-                 : "memory");
-}
+using namespace ptx;
 
 template <class V>
 __global__ void __launch_bounds__((SQT_CWARPS + 1) * 32)
@@ -416,14 +384,13 @@ k_square_tma(int64_t nsq, const int2 *__restrict__ sq_ef, V *__restrict__ sq_val
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], SQT_CWARPS);
         }
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        fence_mbar_init();
     }
     __syncthreads();
     if (warp == SQT_CWARPS) {
         // producer: one lane issues the bulk copies of this CTA's chunks
         if (lane == 0) {
-            uint64_t policy;
-            asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(policy));
+            const uint64_t policy = policy_evict_first();
             int i = 0;
             for (int64_t c = blockIdx.x; c < nchunks; c += gridDim.x, i++) {
                 const int s = i % SQT_STAGES;
@@ -462,7 +429,7 @@ k_square_tma(int64_t nsq, const int2 *__restrict__ sq_ef, V *__restrict__ sq_val
         // order this warp's generic-proxy reads of the stage before the
         // async-proxy (bulk copy) writes that refill it -- without the fence
         // a refill can land before the LDS has read the stage (measured)
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        fence_proxy_async_smem();
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[s]); // stage may be refilled
         double ue[SQT_PER_THREAD], uf[SQT_PER_THREAD];

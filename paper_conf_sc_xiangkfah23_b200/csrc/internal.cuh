@@ -230,6 +230,8 @@ cualign_status bp_gather_Sp(cualign_bp *h, const double *Sfull_dev);   // CSR ->
 // match.cu
 cualign_status quality_eval(cualign_bp *h, const cualign_graph *A, const cualign_graph *B, const int32_t *map_ab,
                             const int32_t *truth, cualign_quality *out); // NEXT-4 (quality.cu)
+cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const float *YB, int32_t n_b, int32_t d,
+                         int32_t k, int32_t *La, int32_t *Lb, double *Lw); // NEXT-2 (knn.cu)
 cualign_status match_setup(cualign_bp *h);
 cualign_status match_round(cualign_bp *h);  // a7 + a8 on the device
 cualign_status match_evaluate(cualign_bp *h); // a8 on mateA / mateB
