@@ -12,7 +12,8 @@ import os
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "lib", "libcualign_bp.so")
+# CUALIGN_LIB: load another build of the same library (A/B measurements only)
+LIB_PATH = os.environ.get("CUALIGN_LIB") or os.path.join(HERE, "lib", "libcualign_bp.so")
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ESTATE = 0, -1, -2, -3, -4, -5
 FLAG_DEVICE_PTRS = 0x01

@@ -205,25 +205,43 @@ k_sbuild(int64_t e_begin, int64_t e_end, const int32_t *__restrict__ La, const i
     }
 }
 
-// sq_pos[q] = (pos of (e,f) in row e, pos of (e) in row f)
+// sq_pos[q] = (pos of (e,f) in row e, pos of (e) in row f): both by binary
+// search in the sorted CSR rows, so it holds for any order of the squares
+__device__ __forceinline__ int64_t lower_bound_i32(const int32_t *__restrict__ x, int64_t lo, int64_t hi, int32_t v)
+{
+    while (lo < hi) {
+        const int64_t mid = lo + ((hi - lo) >> 1);
+        if (x[mid] < v) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
 __global__ void k_sq_pos(int64_t nsq, const int2 *__restrict__ sq_ef, const int64_t *__restrict__ Srp,
-                         const int64_t *__restrict__ sq_rp, const int32_t *__restrict__ Scol,
-                         longlong2 *__restrict__ sq_pos)
+                         const int32_t *__restrict__ Scol, longlong2 *__restrict__ sq_pos)
 {
     for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq;
          q += (int64_t)gridDim.x * blockDim.x) {
         const int2 ef = sq_ef[q];
         const int e = ef.x, f = ef.y;
-        const int64_t row_len = Srp[e + 1] - Srp[e];
-        const int64_t up_len = sq_rp[e + 1] - sq_rp[e];
-        const int64_t pef = Srp[e] + (row_len - up_len) + (q - sq_rp[e]);
-        int64_t lo = Srp[f], hi = Srp[f + 1];
-        while (lo < hi) {
-            int64_t mid = lo + ((hi - lo) >> 1);
-            if (Scol[mid] < e) lo = mid + 1;
-            else hi = mid;
-        }
-        sq_pos[q] = make_longlong2(pef, lo);
+        sq_pos[q] = make_longlong2(lower_bound_i32(Scol, Srp[e], Srp[e + 1], f),
+                                   lower_bound_i32(Scol, Srp[f], Srp[f + 1], e));
+    }
+}
+
+// Square tiles: the square pass gathers u[f] and
+// adds into tacc[f] for the scattered endpoint f of every square.  Once m x 16 B
+// exceeds L2 those become HBM sector misses, so the squares are ordered by
+// (e block, f block) with blocks of 2^log_b edges -- inside a tile the
+// scattered accesses stay in two blocks (2 x 2^log_b x 16 B, L2-resident) --
+// and by (e, f) inside a tile (a stable sort of the (e, f)-sorted build).
+__global__ void k_sq_tile_key(int64_t nsq, const int2 *__restrict__ sq_ef, int log_b, uint32_t nblocks,
+                              uint32_t *__restrict__ key)
+{
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq;
+         q += (int64_t)gridDim.x * blockDim.x) {
+        const int2 ef = sq_ef[q];
+        key[q] = ((uint32_t)ef.x >> log_b) * nblocks + ((uint32_t)ef.y >> log_b);
     }
 }
 
@@ -276,6 +294,24 @@ __global__ void k_upper_count(int64_t n, const int64_t *__restrict__ rp, const i
             else hi = mid;
         }
         cnt[i] = end - lo;
+    }
+}
+
+// insert every undirected B edge {u < v} into the membership set
+__global__ void k_bhash_insert(int64_t n, const int64_t *__restrict__ rp, const int32_t *__restrict__ col,
+                               unsigned long long *__restrict__ T, int log2n)
+{
+    const uint64_t mask = (1ull << log2n) - 1;
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
+        for (int64_t x = rp[u]; x < rp[u + 1]; x++) {
+            const int32_t v = col[x];
+            if (v <= (int32_t)u) continue;
+            const unsigned long long key = bhash_key((int32_t)u, v);
+            for (uint64_t i = bhash_slot(key, log2n);; i = (i + 1) & mask) {
+                const unsigned long long old = atomicCAS(T + i, BHASH_EMPTY, key);
+                if (old == BHASH_EMPTY || old == key) break;
+            }
+        }
     }
 }
 
@@ -532,6 +568,7 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
         if (fp32) CA_CUDA(cudaMemsetAsync(h->sq_val32, 0, sizeof(float2) * ((size_t)h->nsq + 2), h->stream));
         else CA_CUDA(cudaMemsetAsync(h->sq_val, 0, sizeof(double2) * ((size_t)h->nsq + 2), h->stream));
     }
+    CA_TRY(tile_squares(h));
     // the graphs are not needed after S is built
     CA_CUDA(cudaStreamSynchronize(h->stream));
     // Evaluate counts overlapped edges by the definition: it
@@ -568,6 +605,16 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
         if (tmp) cudaFree(tmp);
         CA_TRY(st);
         CA_CUDA(cudaGetLastError());
+        // E_B membership set for evaluate: >= 2 slots per undirected edge
+        int lg = 4;
+        while ((1ll << lg) < nnzB) lg++; // nnzB = 2 |E_B| directed entries
+        h->Bhash_log = lg;
+        CA_TRY(dalloc(h, &h->Bhash, (size_t)1 << lg));
+        CA_CUDA(cudaMemsetAsync(h->Bhash, 0xff, sizeof(unsigned long long) << lg, h->stream));
+        const int64_t nB = B->n;
+        if (nB > 0)
+            k_bhash_insert<<<grid_for(nB, 256, G), 256, 0, h->stream>>>(nB, Bp, Bj, h->Bhash, lg);
+        CA_CUDA(cudaGetLastError());
     }
     dfree(h, Ap);
     dfree(h, Aj);
@@ -588,13 +635,54 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
     return CUALIGN_OK;
 }
 
+// Reorder the squares into (e block, f block) tiles (see k_sq_tile_key).
+// S^p is still all zero, so only (e, f) moves.  CUALIGN_SQ_TILE_LOG overrides
+// the block size (0 = keep the (e, f) order; measurement knob).
+cualign_status tile_squares(cualign_bp *h)
+{
+    static const int log_env = getenv("CUALIGN_SQ_TILE_LOG") ? atoi(getenv("CUALIGN_SQ_TILE_LOG")) : -1;
+    const int log_b = log_env >= 0 ? log_env : SQ_TILE_LOG;
+    h->sq_tile_log = 0;
+    if (log_b <= 0 || h->nsq < 2 || h->nsq >= INT32_MAX) return CUALIGN_OK;
+    const uint32_t nblocks = (uint32_t)(((h->L.m - 1) >> log_b) + 1);
+    if (nblocks < 2 || (uint64_t)nblocks * nblocks >= (1ull << 32)) return CUALIGN_OK;
+    int end_bit = 1;
+    while ((1ull << end_bit) < (uint64_t)nblocks * nblocks) end_bit++;
+    const int n = (int)h->nsq;
+    TmpBuf keys, keys2, tmp;
+    int2 *sorted = nullptr;
+    CA_CUDA(cudaMalloc(&keys.p, sizeof(uint32_t) * (size_t)n));
+    CA_CUDA(cudaMalloc(&keys2.p, sizeof(uint32_t) * (size_t)n));
+    CA_TRY(dalloc(h, &sorted, (size_t)n + 2));
+    {
+        KScope ks(h, CUALIGN_K_INIT);
+        k_sq_tile_key<<<grid_for(n, 256, h->num_sms * 16), 256, 0, h->stream>>>(n, h->sq_ef, log_b, nblocks,
+                                                                                (uint32_t *)keys.p);
+        CA_CUDA(cudaGetLastError());
+        size_t tb = 0;
+        const unsigned long long *vin = reinterpret_cast<const unsigned long long *>(h->sq_ef);
+        unsigned long long *vout = reinterpret_cast<unsigned long long *>(sorted);
+        CA_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, (const uint32_t *)keys.p, (uint32_t *)keys2.p, vin,
+                                                vout, n, 0, end_bit, h->stream));
+        CA_CUDA(cudaMalloc(&tmp.p, tb ? tb : 1));
+        CA_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tb, (const uint32_t *)keys.p, (uint32_t *)keys2.p, vin, vout,
+                                                n, 0, end_bit, h->stream));
+        CA_CUDA(cudaMemsetAsync(sorted + n, 0, 2 * sizeof(int2), h->stream));
+    }
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    dfree(h, h->sq_ef);
+    h->sq_ef = sorted;
+    h->sq_tile_log = log_b;
+    return CUALIGN_OK;
+}
+
 cualign_status ensure_sq_pos(cualign_bp *h)
 {
     if (h->sq_pos || h->nsq == 0) return CUALIGN_OK;
     KScope ks(h, CUALIGN_K_INIT);
     CA_TRY(dalloc(h, &h->sq_pos, (size_t)h->nsq));
     k_sq_pos<<<grid_for(h->nsq, 256, h->num_sms * 16), 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->Srp,
-                                                                            h->sq_rp, h->Scol, h->sq_pos);
+                                                                            h->Scol, h->sq_pos);
     CA_CUDA(cudaGetLastError());
     return CUALIGN_OK;
 }

@@ -97,8 +97,9 @@ struct cualign_bp {
     int64_t s = 0, nsq = 0, max_row = 0;
     int64_t *Srp = nullptr;      // (e1-e0)+1, indexed e - e0
     int32_t *Scol = nullptr;     // s
-    int64_t *sq_rp = nullptr;    // (e1-e0)+1: squares {e<f} of row e are sq_rp[e-e0]..sq_rp[e-e0+1]-1
-    int2 *sq_ef = nullptr;       // nsq: (e, f), e < f, sorted by (e, f)
+    int64_t *sq_rp = nullptr;    // (e1-e0)+1: row e has sq_rp[e-e0+1]-sq_rp[e-e0] squares {e<f} (build offsets)
+    int2 *sq_ef = nullptr;       // nsq: (e, f), e < f, sorted by (e, f) inside (e block, f block) tiles
+    int sq_tile_log = 0;         // tile blocks of 2^sq_tile_log edges (0: plain (e, f) order)
     double2 *sq_val = nullptr;   // nsq: (S^p_ef, S^p_fe)
     float2 *sq_val32 = nullptr;  // same, CUALIGN_FLAG_FP32_S storage (sq_val unused then)
     longlong2 *sq_pos = nullptr; // nsq: (pos(e,f), pos(f,e)) in the CSR; built lazily
@@ -153,6 +154,8 @@ struct cualign_bp {
     int64_t *Bp = nullptr;
     int32_t *Bj = nullptr;
     int2 *Apairs = nullptr;  // undirected A edges (i, j), i < j
+    unsigned long long *Bhash = nullptr; // E_B membership: open-addressing set of (u << 32 | v), u < v
+    int Bhash_log = 0;                   // 2^Bhash_log slots (load <= 1/2)
     int64_t nApairs = 0;
     int64_t max_deg_a = 0, max_deg_b = 0;     // max degree of A / B vertices in L
     cualign::RoundDev *rd = nullptr;
@@ -183,6 +186,31 @@ inline cualign_status dalloc(cualign_bp *h, T **p, size_t n)
 void dfree(cualign_bp *h, void *p);
 void dfree_all(cualign_bp *h);
 
+// ------------------------------------------------- B-edge membership set
+// Evaluate asks "is (M(i), M(j)) an edge of B?" once per
+// undirected A edge and matching.  A sorted-row binary search is ~5 dependent
+// loads; this set answers in ~1: key (min << 32 | max), multiplicative hash,
+// linear probing, empty = ~0.
+constexpr unsigned long long BHASH_EMPTY = ~0ull;
+__host__ __device__ __forceinline__ unsigned long long bhash_key(int32_t u, int32_t v)
+{
+    const uint32_t lo = (uint32_t)(u < v ? u : v), hi = (uint32_t)(u < v ? v : u);
+    return ((unsigned long long)lo << 32) | hi;
+}
+__host__ __device__ __forceinline__ uint64_t bhash_slot(unsigned long long key, int log2n)
+{
+    return (key * 0x9E3779B97F4A7C15ull) >> (64 - log2n);
+}
+__device__ __forceinline__ bool bhash_has(const unsigned long long *__restrict__ T, int log2n, unsigned long long key)
+{
+    const uint64_t mask = (1ull << log2n) - 1;
+    for (uint64_t i = bhash_slot(key, log2n);; i = (i + 1) & mask) {
+        const unsigned long long x = __ldg(T + i);
+        if (x == key) return true;
+        if (x == BHASH_EMPTY) return false;
+    }
+}
+
 // ------------------------------------------------------- launch accounting
 struct KScope {
     cualign_bp *h;
@@ -201,6 +229,8 @@ cualign_status upload_graph(cualign_bp *h, const cualign_graph *g, const char *w
 cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualign_graph *B,
                              const cualign_edges *E);
 cualign_status ensure_sq_pos(cualign_bp *h);
+cualign_status tile_squares(cualign_bp *h);
+constexpr int SQ_TILE_LOG = 21; // square tiles: blocks of 2^21 edges (2 x 32 MB of u + tacc per tile)
 
 // api.cu
 void invalidate_graphs(cualign_bp *h);

@@ -12,7 +12,10 @@
 //                NS-stage mbarrier ring).  Warp 1: TMEM allocation and the
 //                single-thread tcgen05.mma issue (M=128, N=BN, K=16 per
 //                instruction, bf16 in / fp32 accumulate) into one of two TMEM
-//                accumulators.  Warps 2-5: epilogue, one A row per thread:
+//                accumulators.  Warps 2-9: epilogue, one A row per thread
+//                of each TMEM lane quarter, two warps per quarter on
+//                interleaved 32-column chunks; a chunk is tested against the
+//                row's running k-th best by its max (FMNMX3 tree) first:
 //                tcgen05.ld 32 columns at a time and a running top-k (values
 //                above the row's current k-th best are inserted) -- the
 //                n_A x n_B similarity matrix never leaves the SM.
@@ -38,7 +41,8 @@ using namespace ptx;
 
 constexpr int KNN_BM = 128;       // A rows per CTA (MMA M)
 constexpr int KNN_KMAX = 32;      // max neighbours per row
-constexpr int KNN_EPI_WARPS = 4;  // one A row per epilogue thread
+constexpr int KNN_EPI_H = 2;      // epilogue warps per TMEM lane quarter (column interleave)
+constexpr int KNN_EPI_WARPS = 4 * KNN_EPI_H; // one A row per thread of each quarter
 constexpr int KNN_THREADS = (2 + KNN_EPI_WARPS) * 32;
 
 // Unit rows -> bf16 -> swizzled tile image.  Tile t holds rows [t*R, t*R+R),
@@ -78,7 +82,7 @@ __global__ void k_knn_prep(const float *__restrict__ Y, int32_t n, int32_t d, in
 }
 
 // Partial top-k of one CTA: rows [rb*128, +128) x B tiles [t0, t1).
-// Output pv / pi: [row][split][k] (unsorted), idx INT_MAX = empty.
+// Output pv / pi: [row][split][half][k] (unsorted), idx INT_MAX = empty.
 template <int BN>
 __global__ void __launch_bounds__(KNN_THREADS, 1)
 k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32_t n_a, int32_t n_b, int32_t KB,
@@ -92,9 +96,9 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
     const uint32_t b_bytes = (uint32_t)KB * BN * 128;
     uint8_t *sA = smem;
     uint8_t *sB = smem + a_bytes;                         // nstages x b_bytes (multiples of 1024)
-    float *tv = reinterpret_cast<float *>(sB + (size_t)nstages * b_bytes);   // [k][128]
-    int32_t *ti = reinterpret_cast<int32_t *>(tv + KNN_KMAX * KNN_BM);       // [k][128]
-    uint64_t *bars = reinterpret_cast<uint64_t *>(ti + KNN_KMAX * KNN_BM);
+    float *tv_all = reinterpret_cast<float *>(sB + (size_t)nstages * b_bytes);          // [H][k][128]
+    int32_t *ti_all = reinterpret_cast<int32_t *>(tv_all + KNN_EPI_H * KNN_KMAX * KNN_BM); // [H][k][128]
+    uint64_t *bars = reinterpret_cast<uint64_t *>(ti_all + KNN_EPI_H * KNN_KMAX * KNN_BM);
     uint64_t *full = bars;                  // [nstages]
     uint64_t *empty = bars + nstages;       // [nstages]
     uint64_t *tfull = bars + 2 * nstages;   // [2]
@@ -166,8 +170,14 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
         }
     } else {
         // --------------------------------------------------- epilogue
+        // warp w may read TMEM lanes 32*(w%4)..+31 only; the KNN_EPI_H warps of
+        // one quarter take interleaved 32-column chunks of each tile and keep
+        // their own running top-k (merged by k_knn_merge)
         const int q = warp & 3;            // TMEM lane quarter this warp may access
+        const int half = (warp - 2) >> 2;  // which chunks of a tile
         const int row = q * 32 + lane;     // A row within the block = TMEM lane
+        float *tv = tv_all + half * KNN_KMAX * KNN_BM;
+        int32_t *ti = ti_all + half * KNN_KMAX * KNN_BM;
         for (int j = 0; j < k; j++) {
             tv[j * KNN_BM + row] = -INFINITY;
             ti[j * KNN_BM + row] = INT_MAX;
@@ -180,15 +190,34 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
             tc_fence_after();
             const int vbase = (t0 + i) * BN;
 #pragma unroll 1
-            for (int c = 0; c < BN / 32; c++) {
+            for (int c = half; c < BN / 32; c += KNN_EPI_H) {
                 uint32_t r[32];
                 tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN + c * 32), r);
                 tmem_ld_wait();
+                const int v0 = vbase + c * 32;
+                if (v0 + 32 > n_b) { // padding columns of the last tile never enter
+#pragma unroll
+                    for (int j = 0; j < 32; j++)
+                        if (v0 + j >= n_b) r[j] = __float_as_uint(-INFINITY);
+                }
+                // chunk max first (FMNMX3 tree): almost every chunk is rejected
+                // after the first tiles, so the per-element test runs rarely
+                float m4[4];
+#pragma unroll
+                for (int t = 0; t < 4; t++) {
+                    float x = __uint_as_float(r[8 * t]);
+#pragma unroll
+                    for (int j = 1; j < 8; j += 2)
+                        x = fmaxf(fmaxf(x, __uint_as_float(r[8 * t + j])),
+                                  __uint_as_float(r[8 * t + (j + 1 < 8 ? j + 1 : j)]));
+                    m4[t] = x;
+                }
+                if (!(fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) > thr)) continue;
 #pragma unroll
                 for (int j = 0; j < 32; j++) {
                     const float val = __uint_as_float(r[j]);
-                    const int v = vbase + c * 32 + j;
-                    if (val > thr && v < n_b) {
+                    const int v = v0 + j;
+                    if (val > thr) {
                         // replace the current worst, then find the new worst:
                         // (lowest value; among equal values the highest index)
                         tv[thr_pos * KNN_BM + row] = val;
@@ -215,7 +244,7 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
         }
         const int64_t u = (int64_t)rb * KNN_BM + row;
         if (u < n_a) {
-            const int64_t o = (u * nsplit + split) * k;
+            const int64_t o = ((u * nsplit + split) * KNN_EPI_H + half) * k;
             for (int j = 0; j < k; j++) {
                 pv[o + j] = tv[j * KNN_BM + row];
                 pi[o + j] = ti[j * KNN_BM + row];
@@ -338,7 +367,7 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
     nsplit = (ntilesB + tps - 1) / tps;
     // shared memory: A tile, B stages, top-k arrays, barriers
     const size_t a_bytes = (size_t)KB * KNN_BM * 128, b_bytes = (size_t)KB * BN * 128;
-    const size_t fixed = a_bytes + (size_t)KNN_KMAX * KNN_BM * 8 + 256;
+    const size_t fixed = a_bytes + (size_t)KNN_EPI_H * KNN_KMAX * KNN_BM * 8 + 256;
     int smem_optin = 0;
     int dev = 0;
     CA_CUDA(cudaGetDevice(&dev));
@@ -351,8 +380,8 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
     const size_t smem = fixed + (size_t)nstages * b_bytes + 1024; // +1024: alignment slack
     float *pv = nullptr;
     int32_t *pi = nullptr;
-    CA_TRY(dalloc(h, &pv, (size_t)n_a * nsplit * k));
-    CA_TRY(dalloc(h, &pi, (size_t)n_a * nsplit * k));
+    CA_TRY(dalloc(h, &pv, (size_t)n_a * nsplit * KNN_EPI_H * k));
+    CA_TRY(dalloc(h, &pi, (size_t)n_a * nsplit * KNN_EPI_H * k));
     int32_t *oa = La, *ob = Lb;
     double *ow = Lw;
     const int64_t m = (int64_t)n_a * k;
@@ -369,7 +398,7 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
         else
             CA_TRY(knn_launch<128>(h, (const uint8_t *)Asw, (const uint8_t *)Bsw, n_a, n_b, KB, k, pv, pi, nsplit, tps,
                                    nstages, smem));
-        k_knn_merge<<<grid_for(n_a, 128, G), 128, 0, h->stream>>>(n_a, k, nsplit, pv, pi, oa, ob, ow);
+        k_knn_merge<<<grid_for(n_a, 128, G), 128, 0, h->stream>>>(n_a, k, nsplit * KNN_EPI_H, pv, pi, oa, ob, ow);
         CA_CUDA(cudaGetLastError());
     }
     if (!devp) {
