@@ -41,7 +41,8 @@ using namespace ptx;
 
 constexpr int KNN_BM = 128;       // A rows per CTA (MMA M)
 constexpr int KNN_KMAX = 32;      // max neighbours per row
-constexpr int KNN_EPI_H = 2;      // epilogue warps per TMEM lane quarter (column interleave)
+constexpr int KNN_EPI_H = 1;      // epilogue warps per TMEM lane quarter (column interleave)
+constexpr int KNN_CB = 16;        // per-row candidate buffer (entries above the row's k-th best)
 constexpr int KNN_EPI_WARPS = 4 * KNN_EPI_H; // one A row per thread of each quarter
 constexpr int KNN_THREADS = (2 + KNN_EPI_WARPS) * 32;
 
@@ -98,7 +99,9 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
     uint8_t *sB = smem + a_bytes;                         // nstages x b_bytes (multiples of 1024)
     float *tv_all = reinterpret_cast<float *>(sB + (size_t)nstages * b_bytes);          // [H][k][128]
     int32_t *ti_all = reinterpret_cast<int32_t *>(tv_all + KNN_EPI_H * KNN_KMAX * KNN_BM); // [H][k][128]
-    uint64_t *bars = reinterpret_cast<uint64_t *>(ti_all + KNN_EPI_H * KNN_KMAX * KNN_BM);
+    float *cv_all = reinterpret_cast<float *>(ti_all + KNN_EPI_H * KNN_KMAX * KNN_BM);     // [H][CB][128]
+    int32_t *ci_all = reinterpret_cast<int32_t *>(cv_all + KNN_EPI_H * KNN_CB * KNN_BM);    // [H][CB][128]
+    uint64_t *bars = reinterpret_cast<uint64_t *>(ci_all + KNN_EPI_H * KNN_CB * KNN_BM);
     uint64_t *full = bars;                  // [nstages]
     uint64_t *empty = bars + nstages;       // [nstages]
     uint64_t *tfull = bars + 2 * nstages;   // [2]
@@ -178,12 +181,43 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
         const int row = q * 32 + lane;     // A row within the block = TMEM lane
         float *tv = tv_all + half * KNN_KMAX * KNN_BM;
         int32_t *ti = ti_all + half * KNN_KMAX * KNN_BM;
+        float *cv = cv_all + half * KNN_CB * KNN_BM;
+        int32_t *ci = ci_all + half * KNN_CB * KNN_BM;
         for (int j = 0; j < k; j++) {
             tv[j * KNN_BM + row] = -INFINITY;
             ti[j * KNN_BM + row] = INT_MAX;
         }
-        float thr = -INFINITY; // current k-th best of the row
-        int thr_pos = 0;
+        float thr = -INFINITY; // the row's k-th best (as of the last compaction)
+        int thr_pos = 0, cnt = 0;
+        // Entries above thr are appended to the row's candidate buffer (two
+        // shared-memory stores); the buffer is folded into the top-k by the
+        // whole warp at once when some lane could overflow it.  Folding takes
+        // the buffered entries in column order with the same strict test as a
+        // sequential scan, so the kept set (value desc, lowest index among
+        // equals) is the sequential one; only the per-insertion rescan of the
+        // k slots is batched instead of diverging the warp per element.
+        auto fold = [&]() {
+            for (int b = 0; b < cnt; b++) {
+                const float val = cv[b * KNN_BM + row];
+                if (!(val > thr)) continue;
+                tv[thr_pos * KNN_BM + row] = val;
+                ti[thr_pos * KNN_BM + row] = ci[b * KNN_BM + row];
+                float wv = INFINITY;
+                int wi = -1, wp = 0;
+                for (int jj = 0; jj < k; jj++) { // new worst: lowest value, then highest index
+                    const float x = tv[jj * KNN_BM + row];
+                    const int xi = ti[jj * KNN_BM + row];
+                    if (x < wv || (x == wv && xi > wi)) {
+                        wv = x;
+                        wi = xi;
+                        wp = jj;
+                    }
+                }
+                thr = wv;
+                thr_pos = wp;
+            }
+            cnt = 0;
+        };
         for (int i = 0; i < ntiles; i++) {
             const int buf = i & 1;
             mbar_wait(&tfull[buf], (uint32_t)(i >> 1) & 1u);
@@ -192,6 +226,7 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
 #pragma unroll 1
             for (int c = half; c < BN / 32; c += KNN_EPI_H) {
                 uint32_t r[32];
+                __syncwarp(); // .sync.aligned load: reconverge after a fold
                 tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN + c * 32), r);
                 tmem_ld_wait();
                 const int v0 = vbase + c * 32;
@@ -200,8 +235,8 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
                     for (int j = 0; j < 32; j++)
                         if (v0 + j >= n_b) r[j] = __float_as_uint(-INFINITY);
                 }
-                // chunk max first (FMNMX3 tree): almost every chunk is rejected
-                // after the first tiles, so the per-element test runs rarely
+                // chunk max first (FMNMX3 tree): after the first tiles almost
+                // every chunk of every row is below the row's k-th best
                 float m4[4];
 #pragma unroll
                 for (int t = 0; t < 4; t++) {
@@ -212,29 +247,20 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
                                   __uint_as_float(r[8 * t + (j + 1 < 8 ? j + 1 : j)]));
                     m4[t] = x;
                 }
-                if (!(fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) > thr)) continue;
+                const bool pass = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) > thr;
+                if (!__any_sync(0xffffffffu, pass)) continue; // warp-uniform
 #pragma unroll
-                for (int j = 0; j < 32; j++) {
-                    const float val = __uint_as_float(r[j]);
-                    const int v = v0 + j;
-                    if (val > thr) {
-                        // replace the current worst, then find the new worst:
-                        // (lowest value; among equal values the highest index)
-                        tv[thr_pos * KNN_BM + row] = val;
-                        ti[thr_pos * KNN_BM + row] = v;
-                        float wv = INFINITY;
-                        int wi = -1, wp = 0;
-                        for (int jj = 0; jj < k; jj++) {
-                            const float x = tv[jj * KNN_BM + row];
-                            const int xi = ti[jj * KNN_BM + row];
-                            if (x < wv || (x == wv && xi > wi)) {
-                                wv = x;
-                                wi = xi;
-                                wp = jj;
-                            }
+                for (int g = 0; g < 4; g++) {
+                    // room for 8 more in every lane's buffer (warp-uniform fold)
+                    if (__any_sync(0xffffffffu, cnt > KNN_CB - 8)) fold();
+#pragma unroll
+                    for (int jj = 0; jj < 8; jj++) {
+                        const float val = __uint_as_float(r[8 * g + jj]);
+                        if (val > thr) {
+                            cv[cnt * KNN_BM + row] = val;
+                            ci[cnt * KNN_BM + row] = v0 + 8 * g + jj;
+                            cnt++;
                         }
-                        thr = wv;
-                        thr_pos = wp;
                     }
                 }
             }
@@ -242,6 +268,7 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
             __syncwarp();
             if (lane == 0) mbar_arrive(&tempty[buf]);
         }
+        fold();
         const int64_t u = (int64_t)rb * KNN_BM + row;
         if (u < n_a) {
             const int64_t o = ((u * nsplit + split) * KNN_EPI_H + half) * k;
@@ -367,7 +394,7 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
     nsplit = (ntilesB + tps - 1) / tps;
     // shared memory: A tile, B stages, top-k arrays, barriers
     const size_t a_bytes = (size_t)KB * KNN_BM * 128, b_bytes = (size_t)KB * BN * 128;
-    const size_t fixed = a_bytes + (size_t)KNN_EPI_H * KNN_KMAX * KNN_BM * 8 + 256;
+    const size_t fixed = a_bytes + (size_t)KNN_EPI_H * (KNN_KMAX + KNN_CB) * KNN_BM * 8 + 256;
     int smem_optin = 0;
     int dev = 0;
     CA_CUDA(cudaGetDevice(&dev));

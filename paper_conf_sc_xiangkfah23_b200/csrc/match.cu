@@ -221,8 +221,8 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
     }
 }
 
-template <int G, int U, bool DIST = false>
-__global__ void __launch_bounds__(128) k_suitor(MatchParams P)
+template <int G, int U, bool DIST = false, int MINB = 1>
+__global__ void __launch_bounds__(128, MINB) k_suitor(MatchParams P)
 {
     auto tile = cg::tiled_partition<G>(cg::this_thread_block());
     const int lane = tile.thread_rank();
@@ -572,15 +572,41 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, con
             card[1]++;
         }
     }
-    for (int64_t q = tid; q < P.npairs; q += nthr) {
-        const int2 ij = __ldg(P.pairs + q);
+    // EVAL_U pairs per thread and pass, each level of the dependent chain
+    // (pair -> mates -> M(i), M(j) -> probe) issued for all of them together
+    constexpr int EVAL_U = 4;
+    for (int64_t base = tid; base < P.npairs; base += nthr * EVAL_U) {
+        int2 ij[EVAL_U];
+        int em[EVAL_U][4]; // mates of i and j in both instances (edge ids)
 #pragma unroll
-        for (int k = 0; k < 2; k++) {
-            const int ei = P.mateA[k * P.nA + ij.x];
-            const int ej = P.mateA[k * P.nA + ij.y];
-            if (ei < 0 || ej < 0) continue;
-            const int mi = __ldg(P.Lb + ei), mj = __ldg(P.Lb + ej); // M(i), M(j) in V_B
-            if (bhash_has(P.Bhash, P.Bhash_log, bhash_key(mi, mj))) ov[k]++;
+        for (int u = 0; u < EVAL_U; u++) {
+            const int64_t q = base + u * nthr;
+            ij[u] = q < P.npairs ? __ldg(P.pairs + q) : make_int2(-1, -1);
+        }
+#pragma unroll
+        for (int u = 0; u < EVAL_U; u++) {
+#pragma unroll
+            for (int k = 0; k < 2; k++) {
+                em[u][2 * k] = ij[u].x >= 0 ? P.mateA[k * P.nA + ij[u].x] : -1;
+                em[u][2 * k + 1] = ij[u].x >= 0 ? P.mateA[k * P.nA + ij[u].y] : -1;
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < EVAL_U; u++) {
+#pragma unroll
+            for (int k = 0; k < 2; k++) {
+                const bool both = em[u][2 * k] >= 0 && em[u][2 * k + 1] >= 0;
+                // M(i), M(j) in V_B (-1: not both matched)
+                em[u][2 * k] = both ? __ldg(P.Lb + em[u][2 * k]) : -1;
+                em[u][2 * k + 1] = both ? __ldg(P.Lb + em[u][2 * k + 1]) : -1;
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < EVAL_U; u++) {
+#pragma unroll
+            for (int k = 0; k < 2; k++)
+                if (em[u][2 * k] >= 0 && bhash_has(P.Bhash, P.Bhash_log, bhash_key(em[u][2 * k], em[u][2 * k + 1])))
+                    ov[k]++;
         }
     }
     for (int k = 0; k < 2; k++) {
@@ -707,7 +733,15 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
         else if (G == 8) k_suitor<8, 3><<<grid_for(slots * 8, 128, 1 << 30), 128, 0, h->stream>>>(P);
         else if (G == 2) k_suitor<2, 9><<<grid_for(slots * 2, 128, 1 << 30), 128, 0, h->stream>>>(P);
         else if (G == 1) k_suitor<1, 8><<<grid_for(slots, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else k_suitor<4, 5><<<grid_for(slots * 4, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else {
+            // resident blocks per SM (register cap): measurement knob
+            static const int minb = getenv("CUALIGN_SUITOR_MINB") ? atoi(getenv("CUALIGN_SUITOR_MINB")) : 0;
+            const int grid = grid_for(slots * 4, 128, 1 << 30);
+            if (minb >= 16) k_suitor<4, 5, false, 16><<<grid, 128, 0, h->stream>>>(P);
+            else if (minb >= 12) k_suitor<4, 5, false, 12><<<grid, 128, 0, h->stream>>>(P);
+            else if (minb >= 10) k_suitor<4, 5, false, 10><<<grid, 128, 0, h->stream>>>(P);
+            else k_suitor<4, 5><<<grid, 128, 0, h->stream>>>(P);
+        }
         CA_CUDA(cudaGetLastError());
     }
     if (dbg) {
@@ -763,7 +797,13 @@ cualign_status match_setup(cualign_bp *h)
     int64_t want = ((int64_t)2 * (nA + nB) + 255) / 256;
     int64_t cap = (int64_t)occ * h->num_sms;
     h->match_grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
-    h->eval_grid = grid_for(h->nApairs > (int64_t)nA ? h->nApairs : (int64_t)nA, 256, h->num_sms * 8);
+    {
+        // one wave of k_eval (every block resident at once)
+        int occ = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_eval, 256, 0) != cudaSuccess || occ < 1) occ = 1;
+        (void)cudaGetLastError();
+        h->eval_grid = grid_for(h->nApairs > (int64_t)nA ? h->nApairs : (int64_t)nA, 256, h->num_sms * occ);
+    }
     CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * h->eval_grid));
     return CUALIGN_OK;
 }
