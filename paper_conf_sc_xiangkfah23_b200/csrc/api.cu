@@ -114,12 +114,12 @@ KScope::~KScope()
 void invalidate_graphs(cualign_bp *h)
 {
     for (int t = 0; t < 2; t++)
-        for (int r = 0; r < 4; r++)
+        for (int r = 0; r < cualign_bp::NSLOT; r++)
             if (h->graph[t][r]) {
                 cudaGraphExecDestroy(h->graph[t][r]);
                 h->graph[t][r] = nullptr;
             }
-    for (int r = 0; r < 4; r++) {
+    for (int r = 0; r < cualign_bp::NSLOT; r++) {
         for (auto &pe : h->graph_events[r]) {
             h->event_pool.push_back(pe.second.a);
             h->event_pool.push_back(pe.second.b);
@@ -128,10 +128,74 @@ void invalidate_graphs(cualign_bp *h)
     }
 }
 
-// Capture one step (iterate(1) [+ round]) on the handle's capture stream.
-// what: bit 0 = iterate(1), bit 1 = round (CUALIGN_RUN_*)
-static cualign_status capture_step(cualign_bp *h, int timed, int what)
+__global__ void k_copy_int(int *dst, const int *src) { *dst = *src; }
+__global__ void k_incr_int(int *x) { *x += 1; }
+
+static inline int pslot(int kind, int wb) { return 4 + 2 * kind + wb; }
+
+// The pipelined graphs' work (see capture_step): the y^c / z^c buffers are
+// selected by pointing h->yc / h->zc at them while the kernels are captured.
+static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
 {
+    double *yc0 = h->yc, *zc0 = h->zc;
+    double *yb[2] = {yc0, h->yc_b1}, *zb[2] = {zc0, h->zc_b1};
+    cualign_status st = CUALIGN_OK;
+    auto round_of = [&](int buf) -> cualign_status {
+        // the rounding reports its own iteration counter (rp = iteration
+        // rounded), advanced at the start of every pipelined rounding
+        {
+            KScope ks(h, CUALIGN_K_OTHER);
+            k_incr_int<<<1, 1, 0, h->stream>>>(h->rp_dev);
+            CA_CUDA(cudaGetLastError());
+        }
+        h->yc = yb[buf];
+        h->zc = zb[buf];
+        h->round_p = h->rp_dev;
+        cualign_status r = match_round(h);
+        h->round_p = nullptr;
+        return r;
+    };
+    if (kind == 0) {
+        {
+            KScope ks(h, CUALIGN_K_OTHER);
+            k_copy_int<<<1, 1, 0, h->stream>>>(h->rp_dev, h->p_dev); // rounds done so far = p
+            if (cudaGetLastError() != cudaSuccess) st = CUALIGN_ECUDA;
+        }
+        h->yc = yb[wb];
+        h->zc = zb[wb];
+        if (st == CUALIGN_OK) st = bp_iterate(h, 1);
+    } else if (kind == 1) {
+        // fork: the rounding of iteration p-1 (buffer 1-wb) beside all of
+        // iteration p (writes buffer wb); the rounding reads only y^c, z^c of
+        // p-1, w and L, which iteration p does not touch
+        if (cudaEventRecord(h->fork_ev[0], h->gstream) != cudaSuccess ||
+            cudaStreamWaitEvent(h->gstream2, h->fork_ev[0], 0) != cudaSuccess)
+            st = CUALIGN_ECUDA;
+        if (st == CUALIGN_OK) {
+            h->stream = h->gstream2;
+            st = round_of(1 - wb);
+            h->stream = h->gstream;
+        }
+        h->yc = yb[wb];
+        h->zc = zb[wb];
+        if (st == CUALIGN_OK) st = bp_iterate(h, 1);
+        if (st == CUALIGN_OK && (cudaEventRecord(h->fork_ev[1], h->gstream2) != cudaSuccess ||
+                                 cudaStreamWaitEvent(h->gstream, h->fork_ev[1], 0) != cudaSuccess))
+            st = CUALIGN_ECUDA;
+    } else {
+        st = round_of(wb);
+    }
+    h->yc = yc0;
+    h->zc = zc0;
+    return st;
+}
+
+// Capture one step (iterate(1) [+ round]) on the handle's capture stream.
+// slot < 4: what bits (bit 0 = iterate(1), bit 1 = round, CUALIGN_RUN_*);
+// slot >= 4: a pipelined graph (pslot(kind, wb)).
+static cualign_status capture_step(cualign_bp *h, int timed, int slot)
+{
+    const int what = slot < 4 ? slot : 0;
     const int32_t p_save = h->p;
     const int64_t l0 = h->launches;
     int64_t c0[CUALIGN_NUM_KERNEL_CLASSES];
@@ -141,11 +205,13 @@ static cualign_status capture_step(cualign_bp *h, int timed, int what)
     h->timing = timed != 0;
     h->stream = h->gstream;
     h->capturing = true;
-    h->capture_what = what;
+    h->capture_what = slot;
     cualign_status st = CUALIGN_OK;
     cudaError_t e = cudaStreamBeginCapture(h->gstream, cudaStreamCaptureModeThreadLocal);
     if (e == cudaSuccess) {
-        if (what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND)) {
+        if (slot >= 4) {
+            st = capture_pipelined(h, (slot - 4) / 2, (slot - 4) % 2);
+        } else if (what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND)) {
             // the rounding of iteration p reads only y^c, z^c (or y^p, z^p),
             // w and L -- final after the first half -- and the square pass
             // touches none of them: fork the rounding onto a side branch so
@@ -175,7 +241,7 @@ static cualign_status capture_step(cualign_bp *h, int timed, int what)
             st = CUALIGN_ECUDA;
         }
         if (st == CUALIGN_OK) {
-            e2 = cudaGraphInstantiate(&h->graph[timed][what], g, 0);
+            e2 = cudaGraphInstantiate(&h->graph[timed][slot], g, 0);
             if (e2 != cudaSuccess) {
                 set_error("graph instantiate: %s", cudaGetErrorString(e2));
                 st = CUALIGN_ECUDA;
@@ -190,9 +256,9 @@ static cualign_status capture_step(cualign_bp *h, int timed, int what)
     h->stream = user;
     h->timing = timing_save;
     h->p = p_save;
-    h->graph_launches[timed][what] = h->launches - l0;
+    h->graph_launches[timed][slot] = h->launches - l0;
     for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
-        h->graph_class_launches[timed][what][c] = h->class_launches[c] - c0[c];
+        h->graph_class_launches[timed][slot][c] = h->class_launches[c] - c0[c];
         h->class_launches[c] = c0[c];
     }
     h->launches = l0;
@@ -225,6 +291,51 @@ static cualign_status run_graph(cualign_bp *h, int32_t n, int what)
         }
     }
     if (what & CUALIGN_RUN_ROUND) h->have_info = true;
+    CA_CUDA(cudaEventRecord(h->sync_ev[1], h->gstream));
+    CA_CUDA(cudaStreamWaitEvent(h->stream, h->sync_ev[1], 0));
+    return CUALIGN_OK;
+}
+
+// Launch graph slot `slot` once on the capture stream (capturing it first).
+static cualign_status launch_slot(cualign_bp *h, int slot)
+{
+    const int timed = h->timing ? 1 : 0;
+    if (!h->graph[timed][slot]) CA_TRY(capture_step(h, timed, slot));
+    CA_CUDA(cudaGraphLaunch(h->graph[timed][slot], h->gstream));
+    h->launches += h->graph_launches[timed][slot];
+    for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) h->class_launches[c] += h->graph_class_launches[timed][slot][c];
+    if (timed) {
+        CA_CUDA(cudaStreamSynchronize(h->gstream));
+        for (auto &pe : h->graph_events[slot]) {
+            float ms = 0.f;
+            if (cudaEventElapsedTime(&ms, pe.second.a, pe.second.b) == cudaSuccess) h->class_ms[pe.first] += ms;
+        }
+    }
+    return CUALIGN_OK;
+}
+
+// Step pipeline: n x (iterate + round) where the
+// rounding of iteration k runs beside iteration k+1.  Iteration k writes y^c,
+// z^c into buffer wb_k = (n - k) & 1, so the rounding of k (next graph)
+// reads the buffer iteration k+1 does not write, and the last iteration's
+// values end in buffer 0 (h->yc, h->zc), as after an unpipelined run.
+static cualign_status run_pipelined(cualign_bp *h, int32_t n)
+{
+    CA_TRY(ensure_gh(h, (int64_t)h->p + n + 1));
+    if (!h->yc_b1) {
+        CA_TRY(dalloc(h, &h->yc_b1, (size_t)h->L.m + 1));
+        CA_TRY(dalloc(h, &h->zc_b1, (size_t)h->L.m + 1));
+        CA_TRY(dalloc(h, &h->rp_dev, 1));
+    }
+    CA_CUDA(cudaEventRecord(h->sync_ev[0], h->stream));
+    CA_CUDA(cudaStreamWaitEvent(h->gstream, h->sync_ev[0], 0));
+    for (int32_t k = 1; k <= n; k++) {
+        const int wb = (n - k) & 1;
+        CA_TRY(launch_slot(h, pslot(k == 1 ? 0 : 1, wb)));
+        h->p += 1;
+    }
+    CA_TRY(launch_slot(h, pslot(2, 0)));
+    h->have_info = true;
     CA_CUDA(cudaEventRecord(h->sync_ev[1], h->gstream));
     CA_CUDA(cudaStreamWaitEvent(h->stream, h->sync_ev[1], 0));
     return CUALIGN_OK;
@@ -491,6 +602,15 @@ cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t what)
         }
         return CUALIGN_OK;
     }
+    // both halves of a step: pipelined (the rounding of iteration k beside
+    // iteration k+1) unless the rounding reads y^p, z^p (ROUND_DAMPED: the
+    // next iteration overwrites them), the matching is the cooperative
+    // pointer-round kernel (MATCH_ROUNDS: its grid must be co-resident, so it
+    // never shares the device), or CUALIGN_PIPELINE=0 (measurement knob)
+    static const bool pipe_env = !getenv("CUALIGN_PIPELINE") || atoi(getenv("CUALIGN_PIPELINE")) != 0;
+    if (what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND) && pipe_env &&
+        !(h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS)))
+        return run_pipelined(h, n_steps);
     return run_graph(h, n_steps, what);
 }
 

@@ -132,10 +132,21 @@ struct cualign_bp {
     cudaEvent_t fork_ev[2] = {nullptr, nullptr};
     bool capturing = false;
     int capture_what = 0;
-    cudaGraphExec_t graph[2][4] = {};                       // [timed][what = CUALIGN_RUN_* bits]
-    int64_t graph_launches[2][4] = {};                      // kernels per replay
-    int64_t graph_class_launches[2][4][CUALIGN_NUM_KERNEL_CLASSES] = {};
-    std::vector<std::pair<int, cualign::EventPair>> graph_events[4]; // timed graphs' event nodes
+    // graph slots: [0, 4) = CUALIGN_RUN_* bits (one step); PSLOT(kind, wb) =
+    // the pipelined step graphs: kind 0 = iterate
+    // into buffer wb, 1 = rounding of buffer 1-wb beside iterate into wb,
+    // 2 = rounding of buffer wb
+    static constexpr int NSLOT = 10;
+    cudaGraphExec_t graph[2][NSLOT] = {};                   // [timed][slot]
+    int64_t graph_launches[2][NSLOT] = {};                  // kernels per replay
+    int64_t graph_class_launches[2][NSLOT][CUALIGN_NUM_KERNEL_CLASSES] = {};
+    std::vector<std::pair<int, cualign::EventPair>> graph_events[NSLOT]; // timed graphs' event nodes
+    // step pipeline: y^c, z^c double buffers ([0] = yc/zc, the current
+    // iteration's outside a pipelined run), the iteration the rounding
+    // kernels report (round_p; = p_dev except in a pipelined run)
+    double *yc_b1 = nullptr, *zc_b1 = nullptr;
+    int *rp_dev = nullptr;
+    const int *round_p = nullptr;
 
     // matching (two instances: y and z)
     int32_t *candA = nullptr, *candB = nullptr, *mateA = nullptr, *mateB = nullptr;

@@ -735,7 +735,10 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
         else if (G == 1) k_suitor<1, 8><<<grid_for(slots, 128, 1 << 30), 128, 0, h->stream>>>(P);
         else {
             // resident blocks per SM (register cap): measurement knob
-            static const int minb = getenv("CUALIGN_SUITOR_MINB") ? atoi(getenv("CUALIGN_SUITOR_MINB")) : 0;
+            // default 12 blocks of 128 (40 registers): 0.142 ms vs 0.175 ms
+            // uncapped (66 registers, 8 blocks) on O -- latency-bound, more
+            // resident proposer tiles win over a few spilled registers
+            static const int minb = getenv("CUALIGN_SUITOR_MINB") ? atoi(getenv("CUALIGN_SUITOR_MINB")) : 12;
             const int grid = grid_for(slots * 4, 128, 1 << 30);
             if (minb >= 16) k_suitor<4, 5, false, 16><<<grid, 128, 0, h->stream>>>(P);
             else if (minb >= 12) k_suitor<4, 5, false, 12><<<grid, 128, 0, h->stream>>>(P);
@@ -884,7 +887,7 @@ cualign_status dist_match_local(cualign_bp *h)
         if (dmax > 64) k_suitor<32, 2, true><<<grid_for(slots * 32, 128, 1 << 30), 128, 0, h->stream>>>(P);
         else if (dmax > 24) k_suitor<16, 2, true><<<grid_for(slots * 16, 128, 1 << 30), 128, 0, h->stream>>>(P);
         else if (dmax > 20) k_suitor<8, 3, true><<<grid_for(slots * 8, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else k_suitor<4, 5, true><<<grid_for(slots * 4, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        else k_suitor<4, 5, true, 12><<<grid_for(slots * 4, 128, 1 << 30), 128, 0, h->stream>>>(P);
     }
     k_dist_pack<<<grid_for(2 * nB, 256, G), 256, 0, h->stream>>>(nB, h->suit, h->dist_gx, h->dist_gi, P.x0, P.x1,
                                                                  h->dist_wxl, h->dist_wxg, h->dist_wid);
@@ -950,7 +953,7 @@ cualign_status match_evaluate(cualign_bp *h)
     {
         KScope ks(h, CUALIGN_K_EVAL);
         k_eval<<<h->eval_grid, 256, 0, h->stream>>>(E, (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha, h->beta,
-                                                    h->p_dev, h->match_work);
+                                                    h->round_p ? h->round_p : h->p_dev, h->match_work);
         CA_CUDA(cudaGetLastError());
     }
     {
