@@ -209,6 +209,39 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def read_peaks_bf16():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as fh:
+            return float(json.load(fh)["bf16_tflops"]), "measured (MEASURED_PEAKS.json bf16_tflops)"
+    except Exception:
+        return 2250.0, "fallback (nominal dense bf16)"
+
+
+def knn_measure(ca, dev, peak, n=65536, d=128, k=20, reps=3):
+    """NEXT-2: L from embeddings by cualign_knn -- cosine
+    similarity tiles on the tcgen05 tensor cores (bf16 in, fp32 accumulate)
+    with the fused running top-k.  Device-resident N(0,1) embeddings; the
+    whole call (prep, similarity + top-k, merge) timed with CUDA events;
+    dense-equivalent 2 n^2 d flop per call against the measured bf16 peak."""
+    import torch
+    g = torch.Generator(device=f"cuda:{dev}").manual_seed(20231112)
+    YA = torch.randn(n, d, device=f"cuda:{dev}", generator=g)
+    YB = torch.randn(n, d, device=f"cuda:{dev}", generator=g)
+    ca.knn(YA, YB, k, device=dev)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(reps):
+        ca.knn(YA, YB, k, device=dev)
+    e1.record()
+    torch.cuda.synchronize()
+    sec = e0.elapsed_time(e1) / 1e3 / reps
+    tf = 2.0 * n * n * d / sec / 1e12
+    return {"workload": f"n_A = n_B = {n}, d = {d}, top-{k}, N(0,1) embeddings", "s_per_call": sec,
+            "roofline": {"bound": "tensor", "achieved": tf, "peak": peak[0], "unit": "TFLOP/s",
+                         "frac": tf / peak[0], "peak_source": peak[1]}}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -227,6 +260,7 @@ def main():
     ap.add_argument("--match-rounds", action="store_true", help="pointer-round matching schedule")
     ap.add_argument("--prof-steps", type=int, default=20, help="steps of the per-kernel timing pass")
     ap.add_argument("--strong", action="store_true", help="N > 1: shard the same instance (strong scaling)")
+    ap.add_argument("--no-knn", action="store_true", help="skip the NEXT-2 kNN measurement")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
@@ -404,6 +438,14 @@ def main():
         except Exception as e:  # pragma: no cover
             cpu = {"value": None, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": f"failed: {e}"}
 
+    # ------------------------------------------- NEXT-2: kNN on the tensor cores
+    knn = None
+    if rank == 0 and world == 1 and not args.no_knn:
+        try:
+            knn = knn_measure(ca, dev, read_peaks_bf16())
+        except Exception as e:  # pragma: no cover
+            knn = {"error": str(e)}
+
     if rank != 0:
         return
     line = {
@@ -439,6 +481,7 @@ def main():
         "last_round": {k: info[k] for k in ("iter", "card_y", "card_z", "overlap_y", "overlap_z",
                                             "rounds_y", "rounds_z", "score")},
         "match_schedule": "rounds" if args.match_rounds else "suitor",
+        "next2_knn": knn,
     }
     print(json.dumps(line), flush=True)
 

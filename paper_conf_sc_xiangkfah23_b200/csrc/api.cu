@@ -296,6 +296,17 @@ static cualign_status run_graph(cualign_bp *h, int32_t n, int what)
     return CUALIGN_OK;
 }
 
+// second y^c / z^c buffers and the rounding's iteration counter of the step
+// pipeline; allocated at init next to the first ones (a later allocation
+// fragments the stream-ordered pool the next handle reuses)
+static cualign_status alloc_pipeline(cualign_bp *h)
+{
+    CA_TRY(dalloc(h, &h->yc_b1, (size_t)h->L.m + 1));
+    CA_TRY(dalloc(h, &h->zc_b1, (size_t)h->L.m + 1));
+    CA_TRY(dalloc(h, &h->rp_dev, 1));
+    return CUALIGN_OK;
+}
+
 // Launch graph slot `slot` once on the capture stream (capturing it first).
 static cualign_status launch_slot(cualign_bp *h, int slot)
 {
@@ -322,11 +333,7 @@ static cualign_status launch_slot(cualign_bp *h, int slot)
 static cualign_status run_pipelined(cualign_bp *h, int32_t n)
 {
     CA_TRY(ensure_gh(h, (int64_t)h->p + n + 1));
-    if (!h->yc_b1) {
-        CA_TRY(dalloc(h, &h->yc_b1, (size_t)h->L.m + 1));
-        CA_TRY(dalloc(h, &h->zc_b1, (size_t)h->L.m + 1));
-        CA_TRY(dalloc(h, &h->rp_dev, 1));
-    }
+    if (!h->yc_b1) CA_TRY(alloc_pipeline(h));
     CA_CUDA(cudaEventRecord(h->sync_ev[0], h->stream));
     CA_CUDA(cudaStreamWaitEvent(h->gstream, h->sync_ev[0], 0));
     for (int32_t k = 1; k <= n; k++) {
@@ -466,6 +473,8 @@ static cualign_status alloc_state(cualign_bp *h)
         CA_TRY(dalloc(h, p, m));
         CA_CUDA(cudaMemsetAsync(*p, 0, sizeof(double) * (m ? m : 1), h->stream));
     }
+    if (h->world == 1 && !(h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS)))
+        CA_TRY(alloc_pipeline(h));
     CA_TRY(bp_setup(h));
     CA_TRY(dalloc(h, &h->p_dev, 1));
     CA_CUDA(cudaMemsetAsync(h->p_dev, 0, sizeof(int), h->stream));
@@ -714,6 +723,7 @@ cualign_status cualign_bp_get_S(cualign_bp *h, int64_t *rowptr, int32_t *col, in
         set_error("get_S: a process shard holds only its own rows; use virtual shards or world = 1");
         return CUALIGN_ESTATE;
     }
+    CA_TRY(ensure_csr(h));
     if (rowptr)
         CA_CUDA(cudaMemcpyAsync(rowptr, h->Srp, sizeof(int64_t) * ((size_t)h->L.m + 1), cudaMemcpyDeviceToHost,
                                 h->stream));

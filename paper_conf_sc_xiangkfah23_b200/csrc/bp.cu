@@ -231,19 +231,30 @@ __global__ void __launch_bounds__(256, MINB) k_edge(EdgeArgs R)
     }
 }
 
-// segmented (by sorted key) warp sum, then one atomic per segment
+// Warp sum per run of equal keys, then one atomic per run.  Runs are maximal
+// stretches of consecutive lanes with the same key; the same key may occur in
+// two runs (the squares are sorted by e only inside a tile, so a warp that
+// straddles a tile boundary can see e again) and each run is added on its own.
+// Run sum = inclusive prefix sum at the run's last lane minus the one before
+// its head (u64 arithmetic is exact mod 2^64; the sums stay below 2^62).
 __device__ __forceinline__ void seg_atomic_add(unsigned long long v, int key, int lane,
                                                unsigned long long *dst)
 {
+    unsigned long long incl = v;
 #pragma unroll
     for (int off = 1; off < 32; off <<= 1) {
-        const unsigned long long ov = __shfl_down_sync(FULL_MASK, v, off);
-        const int ok = __shfl_down_sync(FULL_MASK, key, off);
-        if (lane + off < 32 && ok == key) v += ov;
+        const unsigned long long o = __shfl_up_sync(FULL_MASK, incl, off);
+        if (lane >= off) incl += o;
     }
-    const int pk = __shfl_up_sync(FULL_MASK, key, 1);
-    const bool head = (lane == 0) || (pk != key);
-    if (head && key >= 0 && v) atomicAdd(dst + key, v);
+    const int kn = __shfl_down_sync(FULL_MASK, key, 1);
+    const int kp = __shfl_up_sync(FULL_MASK, key, 1);
+    const unsigned last = __ballot_sync(FULL_MASK, lane == 31 || kn != key); // run ends
+    const bool head = (lane == 0) || (kp != key);
+    const int end = __ffs(last >> lane) - 1 + lane;          // last lane of this lane's run
+    const unsigned long long at_end = __shfl_sync(FULL_MASK, incl, end);
+    const unsigned long long before = __shfl_sync(FULL_MASK, incl, lane > 0 ? lane - 1 : 0);
+    const unsigned long long sum = at_end - (lane > 0 ? before : 0ull);
+    if (head && key >= 0 && sum) atomicAdd(dst + key, sum);
 }
 
 // UPDATE = apply lines 9, 13, 16 to the pair; otherwise only (re)compute the

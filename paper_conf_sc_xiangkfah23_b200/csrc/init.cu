@@ -119,7 +119,11 @@ __global__ void k_iota(int64_t m, int32_t *x)
 // hit iff b in N_B(i').  Rows e in [e_begin, e_end); the count pass writes
 // cnt[e] (global index), the fill pass reads row pointers relative to e_begin
 // (a shard builds only its own rows).
-template <bool FILL>
+// UPPER: only the squares {e < f} (f > e <=> j > i: no self loops), i.e. the
+// A neighbours j > i -- half the candidates; the count pass writes ucnt only
+// and the fill pass writes sq_ef only (the CSR is built on demand from the
+// squares, see ensure_csr).
+template <bool FILL, bool UPPER = false>
 __global__ void __launch_bounds__(256)
 k_sbuild(int64_t e_begin, int64_t e_end, const int32_t *__restrict__ La, const int32_t *__restrict__ Lb,
          const int64_t *__restrict__ Arow, const int64_t *__restrict__ Ap,
@@ -135,17 +139,29 @@ k_sbuild(int64_t e_begin, int64_t e_end, const int32_t *__restrict__ La, const i
     for (int64_t e = e_begin + warp; e < e_end; e += nwarps) {
         const int32_t i = La[e], ip = Lb[e];
         const int64_t bs = Bp[ip], be = Bp[ip + 1];
-        const int64_t a_lo = Ap[i], a_hi = Ap[i + 1];
+        int64_t a_lo = Ap[i];
+        const int64_t a_hi = Ap[i + 1];
+        if (UPPER) { // first A neighbour j > i (rows sorted)
+            int64_t lo = a_lo, hi = a_hi;
+            while (lo < hi) {
+                const int64_t mid = lo + ((hi - lo) >> 1);
+                if (Aj[mid] <= i) lo = mid + 1;
+                else hi = mid;
+            }
+            a_lo = lo;
+        }
         int64_t total = 0, upper = 0, lower_cnt = 0, row0 = 0, sq0 = 0;
         if (FILL) {
             const int64_t r = e - e_begin;
-            row0 = Srp[r];
             sq0 = sq_rp[r];
-            lower_cnt = (Srp[r + 1] - row0) - (sq_rp[r + 1] - sq0);
+            if (!UPPER) {
+                row0 = Srp[r];
+                lower_cnt = (Srp[r + 1] - row0) - (sq_rp[r + 1] - sq0);
+            }
         }
         if (be == bs) {
             if (!FILL && lane == 0) {
-                cnt[e] = 0;
+                if (!UPPER) cnt[e] = 0;
                 ucnt[e] = 0;
             }
             continue;
@@ -185,12 +201,16 @@ k_sbuild(int64_t e_begin, int64_t e_end, const int32_t *__restrict__ La, const i
                     hit = bsearch_i32(Bj, bs, be, Lb[f]);
                 }
                 const unsigned mask = __ballot_sync(FULL_MASK, hit);
-                if (FILL) {
+                if (FILL && UPPER) {
+                    if (hit) sq_ef[sq0 + total + __popc(mask & lt_mask)] = make_int2((int)e, (int)f);
+                } else if (FILL) {
                     if (hit) {
                         const int64_t idx = total + __popc(mask & lt_mask);
                         Scol[row0 + idx] = (int32_t)f;
                         if (idx >= lower_cnt) sq_ef[sq0 + (idx - lower_cnt)] = make_int2((int)e, (int)f);
                     }
+                } else if (UPPER) {
+                    // every candidate is an upper one
                 } else {
                     const unsigned um = __ballot_sync(FULL_MASK, hit && f > e);
                     upper += __popc(um);
@@ -199,9 +219,40 @@ k_sbuild(int64_t e_begin, int64_t e_end, const int32_t *__restrict__ La, const i
             }
         }
         if (!FILL && lane == 0) {
-            cnt[e] = total;
-            ucnt[e] = upper;
+            if (!UPPER) cnt[e] = total;
+            ucnt[e] = UPPER ? total : upper;
         }
+    }
+}
+
+// lower-triangle row counts (row f gets one per square {e < f}); with the
+// upper counts they give the full row lengths (max row -> fixed-point scale)
+__global__ void k_lower_count(int64_t nsq, const int2 *__restrict__ sq_ef, unsigned int *__restrict__ lcnt)
+{
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq; q += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(lcnt + sq_ef[q].y, 1u);
+}
+__global__ void k_row_total(int64_t m, const int64_t *__restrict__ ucnt, const unsigned int *__restrict__ lcnt,
+                            int64_t *__restrict__ cnt)
+{
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x)
+        cnt[e] = ucnt[e] + (int64_t)lcnt[e];
+}
+// CSR keys: (e, f) and (f, e) for every square {e < f}
+__global__ void k_csr_keys(int64_t nsq, const int2 *__restrict__ sq_ef, unsigned long long *__restrict__ key)
+{
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq; q += (int64_t)gridDim.x * blockDim.x) {
+        const int2 ef = sq_ef[q];
+        key[q] = ((unsigned long long)(uint32_t)ef.x << 32) | (uint32_t)ef.y;
+        key[nsq + q] = ((unsigned long long)(uint32_t)ef.y << 32) | (uint32_t)ef.x;
+    }
+}
+__global__ void k_csr_cols(int64_t s, const unsigned long long *__restrict__ key, int32_t *__restrict__ col,
+                           int32_t *__restrict__ row)
+{
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < s; q += (int64_t)gridDim.x * blockDim.x) {
+        col[q] = (int32_t)(uint32_t)key[q];
+        row[q] = (int32_t)(key[q] >> 32);
     }
 }
 
@@ -442,6 +493,77 @@ cualign_status upload_graph(cualign_bp *h, const cualign_graph *g, const char *w
 }
 
 // ------------------------------------------------------------ problem build
+// S for an unsharded handle: only the squares {e < f}
+// are enumerated (half the candidates of the full rows), written straight
+// into the square layout; nnz(S) = 2 x squares, and the full row lengths (for
+// the fixed-point scale) come from a histogram of the squares' upper
+// endpoints.  The CSR (get_S, exact mode, state transfer) is built from the
+// squares only when one of those asks for it (ensure_csr).
+static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int32_t *Aj, const int64_t *Bp,
+                                    const int32_t *Bj)
+{
+    const int64_t m = h->L.m;
+    const int G = h->num_sms * 8;
+    h->bounds.assign(2, 0);
+    h->bounds[1] = m;
+    h->e0 = 0;
+    h->e1 = m;
+    h->a0 = 0;
+    h->a1 = h->L.nA;
+    KScope ks(h, CUALIGN_K_INIT);
+    TmpBuf ucnt, tmp, mx;
+    CA_CUDA(cudaMalloc(&ucnt.p, sizeof(int64_t) * (m ? m : 1)));
+    CA_TRY(dalloc(h, &h->sq_rp, (size_t)m + 1));
+    CA_CUDA(cudaMemsetAsync(h->sq_rp, 0, sizeof(int64_t), h->stream));
+    h->nsq = 0;
+    if (m) {
+        const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
+        k_sbuild<false, true><<<blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
+                                                             nullptr, (int64_t *)ucnt.p, nullptr, nullptr, nullptr,
+                                                             nullptr);
+        CA_CUDA(cudaGetLastError());
+        size_t tb = 0;
+        CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, (int64_t *)ucnt.p, h->sq_rp + 1, (int)m, h->stream));
+        CA_CUDA(cudaMalloc(&tmp.p, tb ? tb : 1));
+        CA_CUDA(cub::DeviceScan::InclusiveSum(tmp.p, tb, (int64_t *)ucnt.p, h->sq_rp + 1, (int)m, h->stream));
+        CA_CUDA(cudaMemcpyAsync(&h->nsq, h->sq_rp + m, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaStreamSynchronize(h->stream));
+    }
+    h->s = 2 * h->nsq;
+    h->s_total = h->s;
+    h->nsq_total = h->nsq;
+    CA_TRY(dalloc(h, &h->sq_ef, (size_t)h->nsq + 2)); // +2: 16-byte bulk-copy tails
+    const bool fp32 = (h->flags & CUALIGN_FLAG_FP32_S) != 0;
+    if (fp32) CA_TRY(dalloc(h, &h->sq_val32, (size_t)h->nsq + 2));
+    else CA_TRY(dalloc(h, &h->sq_val, (size_t)h->nsq + 2));
+    h->max_row = 0;
+    if (h->nsq) {
+        const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
+        k_sbuild<true, true><<<blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
+                                                            nullptr, nullptr, nullptr, h->sq_rp, nullptr, h->sq_ef);
+        CA_CUDA(cudaGetLastError());
+        // full row lengths: upper (ucnt) + lower (histogram of f) -> max row
+        TmpBuf lcnt, tot, tmp2;
+        CA_CUDA(cudaMalloc(&lcnt.p, sizeof(unsigned int) * (size_t)m));
+        CA_CUDA(cudaMalloc(&tot.p, sizeof(int64_t) * (size_t)m));
+        CA_CUDA(cudaMalloc(&mx.p, sizeof(int64_t)));
+        CA_CUDA(cudaMemsetAsync(lcnt.p, 0, sizeof(unsigned int) * (size_t)m, h->stream));
+        k_lower_count<<<grid_for(h->nsq, 256, G), 256, 0, h->stream>>>(h->nsq, h->sq_ef, (unsigned int *)lcnt.p);
+        k_row_total<<<grid_for(m, 256, G), 256, 0, h->stream>>>(m, (const int64_t *)ucnt.p,
+                                                                (const unsigned int *)lcnt.p, (int64_t *)tot.p);
+        CA_CUDA(cudaGetLastError());
+        size_t tb = 0;
+        CA_CUDA(cub::DeviceReduce::Max(nullptr, tb, (int64_t *)tot.p, (int64_t *)mx.p, (int)m, h->stream));
+        CA_CUDA(cudaMalloc(&tmp2.p, tb ? tb : 1));
+        CA_CUDA(cub::DeviceReduce::Max(tmp2.p, tb, (int64_t *)tot.p, (int64_t *)mx.p, (int)m, h->stream));
+        CA_CUDA(cudaMemcpyAsync(&h->max_row, mx.p, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+    }
+    if (fp32) CA_CUDA(cudaMemsetAsync(h->sq_val32, 0, sizeof(float2) * ((size_t)h->nsq + 2), h->stream));
+    else CA_CUDA(cudaMemsetAsync(h->sq_val, 0, sizeof(double2) * ((size_t)h->nsq + 2), h->stream));
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    return CUALIGN_OK;
+}
+
 cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualign_graph *B,
                              const cualign_edges *E)
 {
@@ -459,6 +581,9 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
         set_error("m = %lld exceeds int32 edge ids", (long long)m);
         return CUALIGN_EINVAL;
     }
+    if (h->world == 1) {
+        CA_TRY(build_S_upper(h, Ap, Aj, Bp, Bj));
+    } else {
     // S: count pass over all rows (a shard needs every row's count for the
     // partition and the global max row), then this handle's rows [e0, e1)
     {
@@ -568,6 +693,7 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
         if (fp32) CA_CUDA(cudaMemsetAsync(h->sq_val32, 0, sizeof(float2) * ((size_t)h->nsq + 2), h->stream));
         else CA_CUDA(cudaMemsetAsync(h->sq_val, 0, sizeof(double2) * ((size_t)h->nsq + 2), h->stream));
     }
+    }
     CA_TRY(tile_squares(h));
     // the graphs are not needed after S is built
     CA_CUDA(cudaStreamSynchronize(h->stream));
@@ -676,8 +802,51 @@ cualign_status tile_squares(cualign_bp *h)
     return CUALIGN_OK;
 }
 
+// The CSR of S (Srp, Scol; rows ascending) from the squares: the keys
+// (e, f) and (f, e) of every square {e < f}, radix-sorted, are exactly the
+// CSR order.  Built on demand for an unsharded handle (get_S, exact mode,
+// state transfer); a shard builds its rows' CSR at init.
+cualign_status ensure_csr(cualign_bp *h)
+{
+    if (h->Scol || h->world > 1) return CUALIGN_OK;
+    const int64_t m = h->L.m, s = h->s;
+    CA_TRY(dalloc(h, &h->Srp, (size_t)m + 1));
+    CA_TRY(dalloc(h, &h->Scol, (size_t)(s ? s : 1)));
+    CA_CUDA(cudaMemsetAsync(h->Srp, 0, sizeof(int64_t) * ((size_t)m + 1), h->stream));
+    if (s == 0) return CUALIGN_OK;
+    if (s >= INT32_MAX) {
+        set_error("CSR of S: nnz(S) = %lld too large for the on-demand build", (long long)s);
+        return CUALIGN_ENOMEM;
+    }
+    KScope ks(h, CUALIGN_K_INIT);
+    TmpBuf k1, k2, tmp, rows;
+    CA_CUDA(cudaMalloc(&k1.p, sizeof(unsigned long long) * (size_t)s));
+    CA_CUDA(cudaMalloc(&k2.p, sizeof(unsigned long long) * (size_t)s));
+    CA_CUDA(cudaMalloc(&rows.p, sizeof(int32_t) * (size_t)s));
+    const int G = h->num_sms * 16;
+    k_csr_keys<<<grid_for(h->nsq, 256, G), 256, 0, h->stream>>>(h->nsq, h->sq_ef, (unsigned long long *)k1.p);
+    CA_CUDA(cudaGetLastError());
+    int bits = 1;
+    while ((1ll << bits) < m) bits++;
+    size_t tb = 0;
+    CA_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, tb, (const unsigned long long *)k1.p,
+                                           (unsigned long long *)k2.p, (int)s, 0, 32 + bits, h->stream));
+    CA_CUDA(cudaMalloc(&tmp.p, tb ? tb : 1));
+    CA_CUDA(cub::DeviceRadixSort::SortKeys(tmp.p, tb, (const unsigned long long *)k1.p, (unsigned long long *)k2.p,
+                                           (int)s, 0, 32 + bits, h->stream));
+    k_csr_cols<<<grid_for(s, 256, G), 256, 0, h->stream>>>(s, (const unsigned long long *)k2.p, h->Scol,
+                                                          (int32_t *)rows.p);
+    // row pointers: rowptr[e] = first position with row >= e
+    k_rowptr_from_sorted<<<grid_for(m + 1, 256, G), 256, 0, h->stream>>>(s, (const int32_t *)rows.p, (int32_t)m,
+                                                                          h->Srp);
+    CA_CUDA(cudaGetLastError());
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    return CUALIGN_OK;
+}
+
 cualign_status ensure_sq_pos(cualign_bp *h)
 {
+    CA_TRY(ensure_csr(h));
     if (h->sq_pos || h->nsq == 0) return CUALIGN_OK;
     KScope ks(h, CUALIGN_K_INIT);
     CA_TRY(dalloc(h, &h->sq_pos, (size_t)h->nsq));

@@ -240,6 +240,7 @@ cualign_status upload_graph(cualign_bp *h, const cualign_graph *g, const char *w
 cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualign_graph *B,
                              const cualign_edges *E);
 cualign_status ensure_sq_pos(cualign_bp *h);
+cualign_status ensure_csr(cualign_bp *h);
 cualign_status tile_squares(cualign_bp *h);
 constexpr int SQ_TILE_LOG = 21; // square tiles: blocks of 2^21 edges (2 x 32 MB of u + tacc per tile)
 

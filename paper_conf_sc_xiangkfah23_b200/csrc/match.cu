@@ -233,6 +233,23 @@ __global__ void __launch_bounds__(128, MINB) k_suitor(MatchParams P)
     if (slot < P.ninst * nP) suitor_tile<G, U, DIST>(P, tile, lane, fromB, nP, nT, slot);
 }
 
+// Persistent form: one wave of tiles, tile t proposes for slots t, t + T,
+// t + 2T, ... -- a tile whose proposer runs a long displacement chain delays
+// only its own later slots, instead of holding its whole block (and the
+// block's SM slot) until its last tile finishes.
+template <int G, int U, int MINB>
+__global__ void __launch_bounds__(128, MINB) k_suitor_persistent(MatchParams P)
+{
+    auto tile = cg::tiled_partition<G>(cg::this_thread_block());
+    const int lane = tile.thread_rank();
+    const bool fromB = P.propose_from_b != 0;
+    const int64_t nP = fromB ? P.nB : P.nA;
+    const int64_t nT = fromB ? P.nA : P.nB;
+    const int64_t T = ((int64_t)gridDim.x * blockDim.x) / G;
+    for (int64_t slot = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G; slot < P.ninst * nP; slot += T)
+        suitor_tile<G, U, false>(P, tile, lane, fromB, nP, nT, slot);
+}
+
 // ------------------------------------------------- DIST round helper kernels
 // slots of a round start from the global suitors
 __global__ void k_dist_init_slots(int64_t n, const unsigned long long *__restrict__ gx, const int32_t *__restrict__ gi,
@@ -740,7 +757,16 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
             // resident proposer tiles win over a few spilled registers
             static const int minb = getenv("CUALIGN_SUITOR_MINB") ? atoi(getenv("CUALIGN_SUITOR_MINB")) : 12;
             const int grid = grid_for(slots * 4, 128, 1 << 30);
-            if (minb >= 16) k_suitor<4, 5, false, 16><<<grid, 128, 0, h->stream>>>(P);
+            static const int pers = getenv("CUALIGN_SUITOR_PERSIST") ? atoi(getenv("CUALIGN_SUITOR_PERSIST")) : 0;
+            if (pers) {
+                int occ = 0;
+                if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_suitor_persistent<4, 5, 12>, 128, 0) !=
+                        cudaSuccess || occ < 1)
+                    occ = 1;
+                (void)cudaGetLastError();
+                k_suitor_persistent<4, 5, 12><<<grid_for(slots * 4, 128, (int64_t)occ * h->num_sms), 128, 0,
+                                                h->stream>>>(P);
+            } else if (minb >= 16) k_suitor<4, 5, false, 16><<<grid, 128, 0, h->stream>>>(P);
             else if (minb >= 12) k_suitor<4, 5, false, 12><<<grid, 128, 0, h->stream>>>(P);
             else if (minb >= 10) k_suitor<4, 5, false, 10><<<grid, 128, 0, h->stream>>>(P);
             else k_suitor<4, 5><<<grid, 128, 0, h->stream>>>(P);

@@ -1,0 +1,116 @@
+"""Order-independence of the square layout and the step pipeline.
+
+* Square tiles: the squares are reordered into
+  (e block, f block) tiles at init.  Every result is order-independent
+  (integer fixed-point F sums, per-square arithmetic), so a run with tiny
+  blocks (many tiles, CUALIGN_SQ_TILE_LOG, read once per process -> a
+  subprocess) must equal the default run bit for bit.
+* Step pipeline: run(n) overlaps the rounding of
+  iteration k with iteration k+1 through double-buffered y^c, z^c; for every
+  n (1, even, odd) and interleaved with eager calls the state, the last round
+  and the best matching equal the eager sequence bit for bit.
+"""
+import json
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+from synth import make_config
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def ca():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_sc_xiangkfah23_b200 as ca
+    ca.load_library()
+    return ca
+
+
+_CHILD = r"""
+import json, sys, numpy as np
+sys.path.insert(0, sys.argv[1])
+import paper_conf_sc_xiangkfah23_b200 as ca
+from synth import make_config
+inst = make_config("P", scale=0.1)
+with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma) as h:
+    h.run(7)
+    st = h.get_state()
+    rp, col = h.get_S()
+    mate, info = h.get_best()
+    out = {k: np.asarray(st[k]).view(np.uint64).tolist() for k in ("yc", "zc", "yp", "zp", "d", "Sp")}
+    out["S"] = [int(x) for x in np.concatenate([rp, col]).tolist()]
+    out["mate"] = np.asarray(mate).tolist()
+    out["best"] = [info["best_score"], info["best_iter"]]
+print(json.dumps(out))
+"""
+
+
+def _child(tile_log):
+    env = dict(os.environ)
+    if tile_log is not None:
+        env["CUALIGN_SQ_TILE_LOG"] = str(tile_log)
+    r = subprocess.run([sys.executable, "-c", _CHILD, ROOT], capture_output=True, text=True, env=env,
+                       timeout=600)
+    assert r.returncode == 0, r.stderr[-2000:]
+    return json.loads(r.stdout.strip().splitlines()[-1])
+
+
+def test_square_tiles_bitwise_invariant(ca):
+    base = _child(0)          # plain (e, f) order
+    tiled = _child(6)         # blocks of 64 edges: hundreds of tiles on P10
+    default = _child(None)    # default block size
+    for k in base:
+        assert base[k] == tiled[k], k
+        assert base[k] == default[k], k
+
+
+def _eager(ca, inst, n):
+    h = ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma)
+    infos = []
+    for _ in range(n):
+        h.iterate(1)
+        infos.append(h.round())
+    return h, infos
+
+
+@pytest.mark.parametrize("n", [1, 2, 5, 6])
+def test_pipelined_run_equals_eager(ca, n):
+    inst = make_config("P", scale=0.1)
+    h1, infos = _eager(ca, inst, n)
+    with h1, ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma) as h2:
+        h2.run(n)
+        s1, s2 = h1.get_state(), h2.get_state()
+        for k in ("yc", "zc", "yp", "zp", "d", "Sp"):
+            assert np.array_equal(s1[k], s2[k]), k
+        m1, i1 = h1.get_best()
+        m2, i2 = h2.get_best()
+        assert np.array_equal(m1, m2)
+        for k in ("iter", "best_score", "best_iter", "score_y", "score_z", "overlap_y", "overlap_z", "card_y",
+                  "card_z", "source", "improved"):
+            assert i1[k] == i2[k], (k, i1[k], i2[k])
+        assert i2["iter"] == n
+
+
+def test_pipelined_runs_interleaved_with_eager_calls(ca):
+    inst = make_config("T")
+    h1, _ = _eager(ca, inst, 9)
+    with h1, ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma) as h2:
+        h2.run(3)
+        h2.iterate(1)
+        h2.round()
+        h2.run(1)
+        h2.run(4)
+        s1, s2 = h1.get_state(), h2.get_state()
+        for k in ("yc", "zc", "yp", "zp", "d", "Sp"):
+            assert np.array_equal(s1[k], s2[k]), k
+        m1, i1 = h1.get_best()
+        m2, i2 = h2.get_best()
+        assert np.array_equal(m1, m2) and i1["best_score"] == i2["best_score"] and i1["iter"] == i2["iter"] == 9
