@@ -3,6 +3,8 @@
 // match.cu.
 #include "internal.cuh"
 
+#include <chrono>
+
 #include <math.h>
 #include <string.h>
 
@@ -296,6 +298,18 @@ static cualign_status run_graph(cualign_bp *h, int32_t n, int what)
     return CUALIGN_OK;
 }
 
+void init_trace(cualign_bp *h, const char *what)
+{
+    static const bool on = getenv("CUALIGN_INIT_TRACE") != nullptr;
+    if (!on) return;
+    static thread_local std::chrono::steady_clock::time_point t0;
+    cudaStreamSynchronize(h->stream);
+    const auto now = std::chrono::steady_clock::now();
+    if (what[0] == '^') t0 = now;
+    fprintf(stderr, "[init] %-24s %9.3f ms\n", what,
+            std::chrono::duration<double, std::milli>(now - t0).count());
+}
+
 // second y^c / z^c buffers and the rounding's iteration counter of the step
 // pipeline; allocated at init next to the first ones (a later allocation
 // fragments the stream-ordered pool the next handle reuses)
@@ -557,10 +571,15 @@ cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B, c
         }
     } else {
         if (st == CUALIGN_OK && h->world > 1) st = nccl_init_comm(h, params->nccl_unique_id);
+        init_trace(h, "^start");
         if (st == CUALIGN_OK) st = build_problem(h, A, B, L);
+        init_trace(h, "build_problem");
         if (st == CUALIGN_OK) st = alloc_state(h);
+        init_trace(h, "alloc_state");
         if (st == CUALIGN_OK) st = match_setup(h);
+        init_trace(h, "match_setup");
         if (st == CUALIGN_OK) st = h->world > 1 ? shard_fsum(h) : bp_fsum(h); // F(S^p = 0) sums for iteration 1
+        init_trace(h, "fsum");
     }
     if (st == CUALIGN_OK) {
         cudaError_t e = cudaStreamSynchronize(h->stream);

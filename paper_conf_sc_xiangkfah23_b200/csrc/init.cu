@@ -574,7 +574,9 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
     int32_t *Aj = nullptr, *Bj = nullptr;
     CA_TRY(upload_graph(h, A, "graph A", &Ap, &Aj, &nnzA));
     CA_TRY(upload_graph(h, B, "graph B", &Bp, &Bj, &nnzB));
+    init_trace(h, "upload graphs");
     CA_TRY(build_L(h, h->L, E, devp, true, A->n, B->n));
+    init_trace(h, "build_L");
     const int64_t m = h->L.m;
 
     if (m >= ((int64_t)1 << 31) - 1) {
@@ -694,7 +696,9 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
         else CA_CUDA(cudaMemsetAsync(h->sq_val, 0, sizeof(double2) * ((size_t)h->nsq + 2), h->stream));
     }
     }
+    init_trace(h, "S build");
     CA_TRY(tile_squares(h));
+    init_trace(h, "tile squares");
     // the graphs are not needed after S is built
     CA_CUDA(cudaStreamSynchronize(h->stream));
     // Evaluate counts overlapped edges by the definition: it
@@ -742,6 +746,7 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
             k_bhash_insert<<<grid_for(nB, 256, G), 256, 0, h->stream>>>(nB, Bp, Bj, h->Bhash, lg);
         CA_CUDA(cudaGetLastError());
     }
+    init_trace(h, "pairs + E_B set");
     dfree(h, Ap);
     dfree(h, Aj);
     // fixed-point scale for the F row sums: beta * max_row * 2^bits < 2^62

@@ -222,6 +222,10 @@ __device__ __forceinline__ bool bhash_has(const unsigned long long *__restrict__
     }
 }
 
+// ------------------------------------------------------------ diagnostics
+// CUALIGN_INIT_TRACE=1: synchronise and print the time of each init phase
+void init_trace(cualign_bp *h, const char *what);
+
 // ------------------------------------------------------- launch accounting
 struct KScope {
     cualign_bp *h;
