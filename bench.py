@@ -122,6 +122,15 @@ def dist_setup(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1 and os.environ.get("CUALIGN_ONE_GPU") == "1":
+        # test mode: every rank on cuda:0 (the sandbox has one GPU); a distinct
+        # NCCL host id per rank stops NCCL rejecting the shared device, so the
+        # ranks connect over its socket transport (timings are not B200 numbers)
+        local = 0
+        os.environ["NCCL_HOSTID"] = f"cualign-one-gpu-{rank}"
+        os.environ.setdefault("NCCL_SOCKET_IFNAME", "lo")
+        os.environ.setdefault("NCCL_IB_DISABLE", "1")
+        os.environ.setdefault("NCCL_NVLS_ENABLE", "0")
     if world > 1:
         import torch.distributed as dist
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
