@@ -225,6 +225,191 @@ k_sbuild(int64_t e_begin, int64_t e_end, const int32_t *__restrict__ La, const i
     }
 }
 
+// Group-map S build of the squares {e < f} (unsharded init; DESIGN.md
+// "S build").  One warp per A vertex i.  Every e = (i, i') of L's row i has
+// the same candidates f = (j, j'), j in N_A(i), j > i (Alg. 3 :185-197, the
+// upper half of row e), and (e, f) is a square iff j' in N_B(i').  The warp
+// takes the edges of row i in groups of <= 32 whose B degrees sum to <= SBG_CAP
+// and builds, in shared memory, the map j' -> {t : j' in N_B(b_t)} (a 32-bit
+// lane mask) over the group; every candidate f is then ONE map lookup of its
+// j', and each set bit t of the result is the square (e_t, f).  Per A vertex
+// that is sum_t deg_B(b_t) inserts + (#candidates x #groups) lookups instead
+// of one binary search per (e, f) pair.  An edge whose own B degree exceeds
+// the map is a group of its own and tests its candidates by binary search in
+// N_B(i') (the warp-per-e method).  Candidates run in ascending f, and an e
+// gets at most one hit per f, so the hits of e arrive in ascending f: lane t
+// keeps e_t's running count and the fill pass writes the same (e, f)-sorted
+// layout as k_sbuild.  Counts are 32-bit scans: the caller checks n_B < 2^26.
+constexpr int SBG_WARPS = 8;
+constexpr int SBG_SLOTS = 512;   // hash slots per warp (key j', value lane mask)
+constexpr int SBG_CAP = 256;     // inserts per group (load factor <= 1/2)
+
+__device__ __forceinline__ int sbg_hash(int32_t b) { return (int)(((uint32_t)b * 2654435761u) >> 23); }
+
+// first lane k whose inclusive sum exceeds pos (incl nondecreasing)
+__device__ __forceinline__ int sbg_find(int32_t incl, int32_t pos)
+{
+    int k = 0;
+#pragma unroll
+    for (int step = 16; step >= 1; step >>= 1) {
+        const int32_t v = __shfl_sync(FULL_MASK, incl, k + step - 1);
+        if (v <= pos) k += step;
+    }
+    return k;
+}
+
+__device__ __forceinline__ int32_t sbg_scan(int32_t v, int lane)
+{
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        const int32_t o = __shfl_up_sync(FULL_MASK, v, off);
+        if (lane >= off) v += o;
+    }
+    return v;
+}
+
+template <bool FILL>
+__global__ void __launch_bounds__(SBG_WARPS * 32)
+k_sbuild_g(int32_t nA, const int64_t *__restrict__ Arow, const int32_t *__restrict__ Lb,
+           const int64_t *__restrict__ Ap, const int32_t *__restrict__ Aj, const int64_t *__restrict__ Bp,
+           const int32_t *__restrict__ Bj, int64_t *__restrict__ ucnt, const int64_t *__restrict__ sq_rp,
+           int2 *__restrict__ sq_ef, unsigned long long *__restrict__ next_i)
+{
+    __shared__ __align__(16) int32_t hkey_all[SBG_WARPS][SBG_SLOTS];
+    __shared__ __align__(16) uint32_t hmask_all[SBG_WARPS][SBG_SLOTS];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    int32_t *hkey = hkey_all[wib];
+    uint32_t *hmask = hmask_all[wib];
+    const unsigned lt_mask = (1u << lane) - 1u;
+    // dynamic A-vertex queue: a warp takes the next vertex when it finishes
+    // one (hub vertices have up to ~10^4x the candidates of the median)
+    while (true) {
+        int64_t i = 0;
+        if (lane == 0) i = (int64_t)atomicAdd(next_i, 1ull);
+        i = __shfl_sync(FULL_MASK, i, 0);
+        if (i >= nA) break;
+        const int64_t l0 = Arow[i];
+        const int ni = (int)(Arow[i + 1] - l0);
+        if (ni == 0) continue;
+        int64_t a_lo = Ap[i];
+        const int64_t a_hi = Ap[i + 1];
+        {
+            int64_t lo = a_lo, hi = a_hi;
+            while (lo < hi) {
+                const int64_t mid = lo + ((hi - lo) >> 1);
+                if (Aj[mid] <= (int32_t)i) lo = mid + 1;
+                else hi = mid;
+            }
+            a_lo = lo;
+        }
+        if (a_lo == a_hi) continue; // no candidates: ucnt stays 0
+        for (int t0 = 0; t0 < ni;) {
+            // ---- next group: t0 .. t0+ng-1 with sum of B degrees <= SBG_CAP
+            const int t = t0 + lane;
+            int32_t bt = 0, bdeg = 0;
+            if (t < ni) {
+                bt = Lb[l0 + t];
+                bdeg = (int32_t)(Bp[bt + 1] - Bp[bt]);
+            }
+            const int32_t dincl = sbg_scan(bdeg, lane);
+            int ng = __popc(__ballot_sync(FULL_MASK, t < ni && dincl <= SBG_CAP));
+            const bool single = ng == 0; // edge t0 alone exceeds the map
+            if (single) ng = 1;
+            const int64_t e_l = l0 + t;  // this lane's edge (valid for lane < ng)
+            int64_t obase = 0;
+            if (FILL && lane < ng) obase = sq_rp[e_l];
+            int32_t cnt = 0;             // lane t: hits of e_{t0+t} so far
+            if (!single) {
+                // ---- build the map j' -> lanes over the group's B rows
+                for (int q = lane; q < SBG_SLOTS / 4; q += 32) {
+                    reinterpret_cast<int4 *>(hkey)[q] = make_int4(-1, -1, -1, -1);
+                    reinterpret_cast<uint4 *>(hmask)[q] = make_uint4(0u, 0u, 0u, 0u);
+                }
+                __syncwarp();
+                const int32_t gin = __shfl_sync(FULL_MASK, dincl, ng - 1);
+                const int32_t dexcl = dincl - bdeg;
+                const int64_t brow = (lane < ng) ? Bp[bt] : 0;
+                for (int32_t c = 0; c < gin; c += 32) {
+                    const int32_t pos = c + lane;
+                    const int k = sbg_find(dincl, pos);
+                    const int32_t ek = __shfl_sync(FULL_MASK, dexcl, k);
+                    const int64_t rk = __shfl_sync(FULL_MASK, brow, k);
+                    if (pos < gin) {
+                        const int32_t jp = Bj[rk + (pos - ek)];
+                        int slot = sbg_hash(jp);
+                        while (true) {
+                            const int32_t old = atomicCAS(&hkey[slot], -1, jp);
+                            if (old == -1 || old == jp) break;
+                            slot = (slot + 1) & (SBG_SLOTS - 1);
+                        }
+                        atomicOr(&hmask[slot], 1u << k);
+                    }
+                }
+                __syncwarp();
+            }
+            const int32_t sb = __shfl_sync(FULL_MASK, bt, 0);
+            const int64_t sblo = single ? Bp[sb] : 0, sbhi = single ? Bp[sb + 1] : 0;
+            // ---- candidates f in ascending order: A neighbours j > i, L rows
+            for (int64_t xb = a_lo; xb < a_hi; xb += 32) {
+                const int64_t x = xb + lane;
+                int64_t flo = 0;
+                int32_t flen = 0;
+                if (x < a_hi) {
+                    const int32_t j = Aj[x];
+                    flo = Arow[j];
+                    flen = (int32_t)(Arow[j + 1] - flo);
+                }
+                const int32_t fincl = sbg_scan(flen, lane);
+                const int32_t fT = __shfl_sync(FULL_MASK, fincl, 31);
+                const int32_t fexcl = fincl - flen;
+                for (int32_t c = 0; c < fT; c += 32) {
+                    const int32_t pos = c + lane;
+                    const int k = sbg_find(fincl, pos);
+                    const int32_t ek = __shfl_sync(FULL_MASK, fexcl, k);
+                    const int64_t lk = __shfl_sync(FULL_MASK, flo, k);
+                    int64_t f = 0;
+                    uint32_t hits = 0u;
+                    if (pos < fT) {
+                        f = lk + (pos - ek);
+                        const int32_t jp = Lb[f];
+                        if (single) {
+                            hits = bsearch_i32(Bj, sblo, sbhi, jp) ? 1u : 0u;
+                        } else {
+                            int slot = sbg_hash(jp);
+                            while (true) {
+                                const int32_t key = hkey[slot];
+                                if (key == jp) {
+                                    hits = hmask[slot];
+                                    break;
+                                }
+                                if (key < 0) break;
+                                slot = (slot + 1) & (SBG_SLOTS - 1);
+                            }
+                        }
+                    }
+                    uint32_t any = __reduce_or_sync(FULL_MASK, hits);
+                    while (any) {
+                        const int tt = __ffs(any) - 1;
+                        any &= any - 1u;
+                        const bool mine = (hits >> tt) & 1u;
+                        const unsigned bal = __ballot_sync(FULL_MASK, mine);
+                        const int32_t run = __shfl_sync(FULL_MASK, cnt, tt);
+                        if (FILL) {
+                            const int64_t ob = __shfl_sync(FULL_MASK, obase, tt);
+                            if (mine)
+                                sq_ef[ob + run + __popc(bal & lt_mask)] = make_int2((int)(l0 + t0 + tt), (int)f);
+                        }
+                        if (lane == tt) cnt += __popc(bal);
+                    }
+                }
+            }
+            if (!FILL && lane < ng) ucnt[e_l] = cnt;
+            __syncwarp();
+            t0 += ng;
+        }
+    }
+}
+
 // lower-triangle row counts (row f gets one per square {e < f}); with the
 // upper counts they give the full row lengths (max row -> fixed-point scale)
 __global__ void k_lower_count(int64_t nsq, const int2 *__restrict__ sq_ef, unsigned int *__restrict__ lcnt)
@@ -516,11 +701,35 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
     CA_TRY(dalloc(h, &h->sq_rp, (size_t)m + 1));
     CA_CUDA(cudaMemsetAsync(h->sq_rp, 0, sizeof(int64_t), h->stream));
     h->nsq = 0;
+    // group-map build (default) unless the 32-bit candidate counts could overflow
+    static const int sb_env = getenv("CUALIGN_SBUILD_VAR") ? atoi(getenv("CUALIGN_SBUILD_VAR")) : 1;
+    const bool group_map = sb_env == 1 && h->L.nB < (1 << 26);
+    const int32_t nA = h->L.nA;
+    int sbg_blocks = 1;
+    TmpBuf qctr;
+    if (group_map) {
+        // one resident wave; the warps pull A vertices from a queue
+        int occ = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sbuild_g<true>, SBG_WARPS * 32, 0) != cudaSuccess ||
+            occ < 1)
+            occ = 1;
+        (void)cudaGetLastError();
+        sbg_blocks = grid_for((int64_t)nA * 32, SBG_WARPS * 32, (int64_t)occ * h->num_sms);
+        CA_CUDA(cudaMalloc(&qctr.p, 2 * sizeof(unsigned long long)));
+        CA_CUDA(cudaMemsetAsync(qctr.p, 0, 2 * sizeof(unsigned long long), h->stream));
+    }
     if (m) {
-        const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
-        k_sbuild<false, true><<<blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
-                                                             nullptr, (int64_t *)ucnt.p, nullptr, nullptr, nullptr,
-                                                             nullptr);
+        if (group_map) {
+            CA_CUDA(cudaMemsetAsync(ucnt.p, 0, sizeof(int64_t) * (size_t)m, h->stream));
+            k_sbuild_g<false><<<sbg_blocks, SBG_WARPS * 32, 0, h->stream>>>(nA, h->L.Arow, h->L.Lb, Ap, Aj, Bp, Bj,
+                                                                          (int64_t *)ucnt.p, nullptr, nullptr,
+                                                                          (unsigned long long *)qctr.p);
+        } else {
+            const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
+            k_sbuild<false, true><<<blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
+                                                                 nullptr, (int64_t *)ucnt.p, nullptr, nullptr,
+                                                                 nullptr, nullptr);
+        }
         CA_CUDA(cudaGetLastError());
         size_t tb = 0;
         CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, (int64_t *)ucnt.p, h->sq_rp + 1, (int)m, h->stream));
@@ -538,9 +747,16 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
     else CA_TRY(dalloc(h, &h->sq_val, (size_t)h->nsq + 2));
     h->max_row = 0;
     if (h->nsq) {
-        const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
-        k_sbuild<true, true><<<blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
-                                                            nullptr, nullptr, nullptr, h->sq_rp, nullptr, h->sq_ef);
+        if (group_map) {
+            k_sbuild_g<true><<<sbg_blocks, SBG_WARPS * 32, 0, h->stream>>>(nA, h->L.Arow, h->L.Lb, Ap, Aj, Bp, Bj,
+                                                                         nullptr, h->sq_rp, h->sq_ef,
+                                                                         (unsigned long long *)qctr.p + 1);
+        } else {
+            const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
+            k_sbuild<true, true><<<blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
+                                                                nullptr, nullptr, nullptr, h->sq_rp, nullptr,
+                                                                h->sq_ef);
+        }
         CA_CUDA(cudaGetLastError());
         // full row lengths: upper (ucnt) + lower (histogram of f) -> max row
         TmpBuf lcnt, tot, tmp2;

@@ -14,7 +14,7 @@ import pytest
 import oracle
 from oracle import Oracle, gamma_power
 from synth import make_config, random_candidates, complete_candidates
-from tests.util import tiny_instance, graph_from_edges, load_golden, golden_instance
+from tests.util import tiny_instance, graph_from_edges, load_golden, golden_instance, candidates_from_lists
 
 pytestmark = pytest.mark.gpu
 
@@ -94,6 +94,38 @@ def test_S_hub_rows_longer_than_a_warp(ca):
         orp, ocol, _ = o.get_S()
         assert np.array_equal(rp, orp) and np.array_equal(col, ocol)
         assert np.max(np.diff(rp)) > 64
+
+
+def test_S_long_candidate_rows(ca):
+    """The S build's group map: L rows longer than one
+    group (> 32 candidates), groups cut by the sum of B degrees, a B hub whose
+    degree alone exceeds the map (its edges take the binary-search path), hub
+    A vertices, A vertices without candidates."""
+    rng = np.random.default_rng(11)
+    n_a, n_b = 90, 400
+    ea = [(0, j) for j in range(1, 60)] + [(int(u), int(v)) for u, v in rng.integers(0, n_a, (300, 2)) if u != v]
+    eb = [(0, j) for j in range(1, 300)] + [(1, j) for j in range(2, 120)] + \
+        [(int(u), int(v)) for u, v in rng.integers(0, n_b, (900, 2)) if u != v]
+    A = graph_from_edges(n_a, sorted(set((min(u, v), max(u, v)) for u, v in ea)))
+    B = graph_from_edges(n_b, sorted(set((min(u, v), max(u, v)) for u, v in eb)))
+    a, b = [], []
+    for i in range(n_a):
+        if i % 11 == 5:
+            continue  # no candidates
+        k = 140 if i % 3 == 0 else (65 if i % 3 == 1 else 12)
+        cand = set(rng.choice(n_b, size=k, replace=False).tolist())
+        if i % 2 == 0:
+            cand.add(0)  # the B hub (degree 299 > the map's 256 inserts)
+        for j in sorted(cand):
+            a.append(i)
+            b.append(int(j))
+    L = candidates_from_lists(n_a, n_b, a, b, rng.uniform(0.1, 1.0, len(a)))
+    o = Oracle(A, B, L, 1.0, 2.0)
+    with ca.CuAlignBP(A, B, L, 1.0, 2.0, 0.9) as h:
+        rp, col = h.get_S()
+        orp, ocol, _ = o.get_S()
+        assert np.array_equal(rp, orp) and np.array_equal(col, ocol)
+        assert o.s > 1000
 
 
 # ------------------------------------------------------- a3-a6: BP iteration
