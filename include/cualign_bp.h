@@ -201,6 +201,16 @@ cualign_status cualign_bp_round(cualign_bp *h, cualign_round_info *info);
 #define CUALIGN_RUN_ROUND   2
 cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t what);
 
+/* End-to-end loop of Alg. 2: n_steps x (iterate(1) +
+ * round), as cualign_bp_run(h, n_steps, CUALIGN_RUN_ITERATE |
+ * CUALIGN_RUN_ROUND), and infos[k] (host array of n_steps, caller-owned)
+ * receives the round info of step k with best_score / best_iter as of that
+ * step.  Each step's info is copied to the host as soon as its rounding has
+ * finished (stream-ordered, into pinned staging), so the host never stalls the
+ * device between steps; synchronises once before returning.  Errors: EINVAL
+ * for n_steps < 0 or a NULL infos with n_steps > 0. */
+cualign_status cualign_bp_run_trace(cualign_bp *h, int32_t n_steps, cualign_round_info *infos);
+
 /* Diagnostics: enable (1) / disable (0) per-kernel event timing (as
  * CUALIGN_FLAG_TIMING).  Graph replays with timing on synchronise after each
  * step to read the per-kernel events; results via cualign_bp_get_stats. */

@@ -16,10 +16,7 @@ def align(A, B, L, alpha=1.0, beta=2.0, gamma=0.99, n_iter=100, flags=0, device=
     x (iterate + round), best.  Returns (mate_a, info, per-round infos).
     shard: world / rank / nccl_id of a sharded run (see CuAlignBP)."""
     with CuAlignBP(A, B, L, alpha, beta, gamma, flags, device, stream, **shard) as h:
-        infos = []
-        for _ in range(n_iter):
-            h.run(1)                                      # graph replay of iterate + round
-            infos.append(h.get_best(with_mate=False)[1])  # the step's result to the host
+        infos = h.run_trace(n_iter)  # graph replays; every step's round info to the host
         mate, info = h.get_best()
         info["t_result"] = time.perf_counter()            # result on the host (before teardown)
     return mate, info, infos

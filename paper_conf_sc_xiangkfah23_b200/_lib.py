@@ -30,7 +30,7 @@ KERNEL_CLASS_NAMES = ["top2", "edge", "square", "rowsum", "match", "init", "stat
 NUM_KERNEL_CLASSES = 10
 
 # every symbol include/cualign_bp.h declares
-EXPORTED = ["cualign_bp_init", "cualign_bp_iterate", "cualign_bp_round", "cualign_bp_run",
+EXPORTED = ["cualign_bp_init", "cualign_bp_iterate", "cualign_bp_round", "cualign_bp_run", "cualign_bp_run_trace",
             "cualign_bp_set_timing", "cualign_bp_get_best",
             "cualign_bp_free", "cualign_bp_get_sizes", "cualign_bp_get_S", "cualign_bp_get_state",
             "cualign_bp_set_state", "cualign_bp_get_stats", "cualign_match", "cualign_last_error",
@@ -117,6 +117,8 @@ def load_library():
     lib.cualign_bp_round.argtypes = [P, P]
     lib.cualign_bp_run.restype = I32
     lib.cualign_bp_run.argtypes = [P, I32, I32]
+    lib.cualign_bp_run_trace.restype = I32
+    lib.cualign_bp_run_trace.argtypes = [P, I32, P]
     lib.cualign_bp_set_timing.restype = I32
     lib.cualign_bp_set_timing.argtypes = [P, I32]
     lib.cualign_bp_get_best.restype = I32
@@ -265,6 +267,15 @@ class CuAlignBP:
         """n_steps x (iterate(1) [+ round]) replayed from a CUDA graph (async)."""
         what = (1 if iterate else 0) | (2 if with_round else 0)
         _check(load_library().cualign_bp_run(self._h, int(n_steps), what))
+
+    def run_trace(self, n_steps):
+        """n_steps x (iterate + round); returns every step's round info (list of
+        dicts, best_score / best_iter as of that step), copied to the host
+        step by step without stalling the device (cualign_bp_run_trace)."""
+        n = int(n_steps)
+        arr = (RoundInfo_t * max(n, 1))()
+        _check(load_library().cualign_bp_run_trace(self._h, n, ctypes.cast(arr, ctypes.c_void_p)))
+        return [arr[k].as_dict() for k in range(n)]
 
     def set_timing(self, on=True):
         _check(load_library().cualign_bp_set_timing(self._h, 1 if on else 0))

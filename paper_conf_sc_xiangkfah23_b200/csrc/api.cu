@@ -38,6 +38,32 @@ static void keep_pool(int dev)
     done[dev] = true;
 }
 
+// Init temporaries (sort buffers, counts) come from a second pool, also
+// cached: taken from the main pool they would leave holes between the
+// handle's persistent arrays, and the next handle's persistent allocations
+// would then grow the main pool (measured: alloc_state 1.5 -> 240 ms).
+cudaMemPool_t temp_pool(int dev)
+{
+    static cudaMemPool_t pools[64] = {};
+    static bool made[64] = {};
+    if (dev < 0 || dev >= 64) return nullptr;
+    if (!made[dev]) {
+        made[dev] = true;
+        cudaMemPoolProps props = {};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        if (cudaMemPoolCreate(&pools[dev], &props) == cudaSuccess) {
+            uint64_t thr = UINT64_MAX;
+            cudaMemPoolSetAttribute(pools[dev], cudaMemPoolAttrReleaseThreshold, &thr);
+        } else {
+            pools[dev] = nullptr;
+        }
+        (void)cudaGetLastError();
+    }
+    return pools[dev];
+}
+
 cualign_status dmalloc(cualign_bp *h, void **p, size_t bytes)
 {
     if (bytes == 0) bytes = 16;
@@ -344,7 +370,7 @@ static cualign_status launch_slot(cualign_bp *h, int slot)
 // z^c into buffer wb_k = (n - k) & 1, so the rounding of k (next graph)
 // reads the buffer iteration k+1 does not write, and the last iteration's
 // values end in buffer 0 (h->yc, h->zc), as after an unpipelined run.
-static cualign_status run_pipelined(cualign_bp *h, int32_t n)
+static cualign_status run_pipelined(cualign_bp *h, int32_t n, RoundDev *trace = nullptr)
 {
     CA_TRY(ensure_gh(h, (int64_t)h->p + n + 1));
     if (!h->yc_b1) CA_TRY(alloc_pipeline(h));
@@ -354,8 +380,13 @@ static cualign_status run_pipelined(cualign_bp *h, int32_t n)
         const int wb = (n - k) & 1;
         CA_TRY(launch_slot(h, pslot(k == 1 ? 0 : 1, wb)));
         h->p += 1;
+        // the rounding of iteration k-1 finished inside this graph: its
+        // result to the host, stream-ordered before the next graph rewrites it
+        if (trace && k >= 2)
+            CA_CUDA(cudaMemcpyAsync(trace + (k - 2), h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->gstream));
     }
     CA_TRY(launch_slot(h, pslot(2, 0)));
+    if (trace) CA_CUDA(cudaMemcpyAsync(trace + (n - 1), h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->gstream));
     h->have_info = true;
     CA_CUDA(cudaEventRecord(h->sync_ev[1], h->gstream));
     CA_CUDA(cudaStreamWaitEvent(h->stream, h->sync_ev[1], 0));
@@ -487,12 +518,16 @@ static cualign_status alloc_state(cualign_bp *h)
         CA_TRY(dalloc(h, p, m));
         CA_CUDA(cudaMemsetAsync(*p, 0, sizeof(double) * (m ? m : 1), h->stream));
     }
+    init_trace(h, "state vectors");
     if (h->world == 1 && !(h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS)))
         CA_TRY(alloc_pipeline(h));
+    init_trace(h, "pipeline buffers");
     CA_TRY(bp_setup(h));
+    init_trace(h, "bp_setup");
     CA_TRY(dalloc(h, &h->p_dev, 1));
     CA_CUDA(cudaMemsetAsync(h->p_dev, 0, sizeof(int), h->stream));
     CA_TRY(ensure_gh(h, 1));
+    init_trace(h, "gamma table");
     if (h->flags & CUALIGN_FLAG_EXACT) {
         CA_TRY(dalloc(h, &h->texact, m));
         CA_TRY(dalloc(h, &h->Ffull, (size_t)h->s));
@@ -515,6 +550,8 @@ static cualign_bp *primary(cualign_bp *h) { return h->vshards.empty() ? h : h->v
         }                                           \
         CA_CUDA(cudaSetDevice(h->dev));             \
     } while (0)
+
+static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, RoundDev *trace);
 
 } // namespace cualign
 
@@ -622,12 +659,64 @@ cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t what)
         set_error("run: what must be CUALIGN_RUN_ITERATE, CUALIGN_RUN_ROUND or both");
         return CUALIGN_EINVAL;
     }
+    return run_steps(h, n_steps, what, nullptr);
+}
+
+// thread-local pinned staging for run_trace (cached: pinned allocation is slow)
+struct PinnedTrace {
+    RoundDev *p = nullptr;
+    size_t n = 0;
+    ~PinnedTrace()
+    {
+        if (p) cudaFreeHost(p);
+    }
+};
+
+cualign_status cualign_bp_run_trace(cualign_bp *h, int32_t n_steps, cualign_round_info *infos)
+{
+    API_ENTER();
+    CHECK_H();
+    if (n_steps < 0 || (n_steps > 0 && !infos)) {
+        set_error("run_trace: n_steps < 0 or infos is NULL");
+        return CUALIGN_EINVAL;
+    }
+    if (n_steps == 0) return CUALIGN_OK;
+    static thread_local PinnedTrace pt;
+    if (pt.n < (size_t)n_steps) {
+        if (pt.p) cudaFreeHost(pt.p);
+        pt.p = nullptr;
+        pt.n = 0;
+        CA_CUDA(cudaHostAlloc((void **)&pt.p, sizeof(RoundDev) * (size_t)n_steps, cudaHostAllocDefault));
+        pt.n = (size_t)n_steps;
+    }
+    CA_TRY(run_steps(h, n_steps, CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND, pt.p));
+    cualign_bp *q = primary(h);
+    CA_CUDA(cudaStreamSynchronize(q->stream));
+    CA_CUDA(cudaStreamSynchronize(q->gstream));
+    for (int32_t k = 0; k < n_steps; k++) {
+        infos[k] = pt.p[k].info;
+        infos[k].best_score = pt.p[k].best_score;
+        infos[k].best_iter = pt.p[k].best_iter;
+    }
+    q->last_info = infos[n_steps - 1];
+    return CUALIGN_OK;
+}
+
+} // extern "C"
+
+namespace cualign {
+static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, RoundDev *trace)
+{
     if (h->world > 1) {
         // sharded: eager per-step launches (the exchanges sit between kernels)
+        cualign_bp *q = primary(h);
         for (int32_t k = 0; k < n_steps; k++) {
             if (what & CUALIGN_RUN_ITERATE) CA_TRY(shard_iterate(h, 1));
             if (what & CUALIGN_RUN_ROUND) CA_TRY(shard_round(h));
+            if (trace)
+                CA_CUDA(cudaMemcpyAsync(trace + k, q->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, q->stream));
         }
+        h->have_info = h->have_info || (what & CUALIGN_RUN_ROUND);
         return CUALIGN_OK;
     }
     // both halves of a step: pipelined (the rounding of iteration k beside
@@ -638,9 +727,17 @@ cualign_status cualign_bp_run(cualign_bp *h, int32_t n_steps, int32_t what)
     static const bool pipe_env = !getenv("CUALIGN_PIPELINE") || atoi(getenv("CUALIGN_PIPELINE")) != 0;
     if (what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND) && pipe_env &&
         !(h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS)))
-        return run_pipelined(h, n_steps);
-    return run_graph(h, n_steps, what);
+        return run_pipelined(h, n_steps, trace);
+    if (!trace) return run_graph(h, n_steps, what);
+    for (int32_t k = 0; k < n_steps; k++) {
+        CA_TRY(run_graph(h, 1, what));
+        CA_CUDA(cudaMemcpyAsync(trace + k, h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->stream));
+    }
+    return CUALIGN_OK;
 }
+} // namespace cualign
+
+extern "C" {
 
 cualign_status cualign_bp_set_timing(cualign_bp *h, int32_t on)
 {
@@ -789,8 +886,9 @@ cualign_status cualign_bp_get_state(cualign_bp *h, double *yc, double *zc, doubl
     for (auto &v : vec)
         if (v.dst && mb) CA_CUDA(cudaMemcpyAsync(v.dst, v.src, mb, cudaMemcpyDeviceToHost, h->stream));
     if (Sp && h->s) {
-        double *tmp = nullptr;
-        CA_CUDA(cudaMalloc(&tmp, sizeof(double) * (size_t)h->s));
+        TmpBuf tb;
+        CA_CUDA(tmalloc(h, tb, sizeof(double) * (size_t)h->s));
+        double *tmp = (double *)tb.p;
         cualign_status st = bp_scatter_Sp(h, tmp);
         if (st == CUALIGN_OK) {
             cudaError_t e = cudaMemcpyAsync(Sp, tmp, sizeof(double) * (size_t)h->s, cudaMemcpyDeviceToHost, h->stream);
@@ -800,7 +898,6 @@ cualign_status cualign_bp_get_state(cualign_bp *h, double *yc, double *zc, doubl
                 st = CUALIGN_ECUDA;
             }
         }
-        cudaFree(tmp);
         CA_TRY(st);
     }
     CA_CUDA(cudaStreamSynchronize(h->stream));
@@ -827,8 +924,9 @@ cualign_status cualign_bp_set_state(cualign_bp *h, const double *yp, const doubl
         CA_CUDA(cudaMemcpyAsync(h->zp, zp, mb, cudaMemcpyHostToDevice, h->stream));
     }
     if (h->s) {
-        double *tmp = nullptr;
-        CA_CUDA(cudaMalloc(&tmp, sizeof(double) * (size_t)h->s));
+        TmpBuf tb;
+        CA_CUDA(tmalloc(h, tb, sizeof(double) * (size_t)h->s));
+        double *tmp = (double *)tb.p;
         cudaError_t e = cudaMemcpyAsync(tmp, Sp, sizeof(double) * (size_t)h->s, cudaMemcpyHostToDevice, h->stream);
         cualign_status st = CUALIGN_OK;
         if (e != cudaSuccess) {
@@ -837,7 +935,6 @@ cualign_status cualign_bp_set_state(cualign_bp *h, const double *yp, const doubl
         }
         if (st == CUALIGN_OK) st = bp_gather_Sp(h, tmp);
         if (st == CUALIGN_OK && cudaStreamSynchronize(h->stream) != cudaSuccess) st = CUALIGN_ECUDA;
-        cudaFree(tmp);
         CA_TRY(st);
     }
     h->p = p;

@@ -634,7 +634,7 @@ cualign_status launch_square(cualign_bp *h, bool update)
 cualign_status ensure_gh(cualign_bp *h, int64_t pmax)
 {
     if (pmax < h->gh_cap) return CUALIGN_OK;
-    int64_t cap = h->gh_cap ? h->gh_cap : 65536;
+    int64_t cap = h->gh_cap ? h->gh_cap : 1024; // doubles on demand (captured graphs are re-captured)
     while (cap <= pmax) cap *= 2;
     std::vector<double2> tab((size_t)cap);
     for (int64_t p = 0; p < cap; p++) {
@@ -731,10 +731,11 @@ cualign_status build_local_incidence(cualign_bp *h)
     const int64_t nB = h->L.nB, ml = h->e1 - h->e0;
     CA_TRY(dalloc(h, &h->Bedge_loc, (size_t)(ml ? ml : 1)));
     CA_TRY(dalloc(h, &h->Bptr_loc, (size_t)nB + 1));
-    int32_t *keys = nullptr, *ids = nullptr;
+    TmpBuf kb, ib, tb_;
+    CA_CUDA(tmalloc(h, kb, sizeof(int32_t) * (size_t)(ml ? ml : 1)));
+    CA_CUDA(tmalloc(h, ib, sizeof(int32_t) * (size_t)(ml ? ml : 1)));
+    int32_t *keys = (int32_t *)kb.p, *ids = (int32_t *)ib.p;
     void *tmp = nullptr;
-    CA_CUDA(cudaMalloc(&keys, sizeof(int32_t) * (size_t)(ml ? ml : 1)));
-    CA_CUDA(cudaMalloc(&ids, sizeof(int32_t) * (size_t)(ml ? ml : 1)));
     cualign_status st = CUALIGN_OK;
     if (ml) {
         k_iota_from<<<grid_for(ml, 256, h->num_sms * 8), 256, 0, h->stream>>>(ml, h->e0, ids);
@@ -743,7 +744,8 @@ cualign_status build_local_incidence(cualign_bp *h)
         size_t tb = 0;
         cub::DeviceRadixSort::SortPairs(nullptr, tb, h->L.Lb + h->e0, keys, ids, h->Bedge_loc, (int)ml, 0, end_bit,
                                         h->stream);
-        if (cudaMalloc(&tmp, tb ? tb : 1) != cudaSuccess) st = CUALIGN_ENOMEM;
+        if (tmalloc(h, tb_, tb ? tb : 1) != cudaSuccess) st = CUALIGN_ENOMEM;
+        tmp = tb_.p;
         if (st == CUALIGN_OK)
             cub::DeviceRadixSort::SortPairs(tmp, tb, h->L.Lb + h->e0, keys, ids, h->Bedge_loc, (int)ml, 0, end_bit,
                                             h->stream);
@@ -751,10 +753,6 @@ cualign_status build_local_incidence(cualign_bp *h)
     if (st == CUALIGN_OK)
         k_rowptr_from_sorted64<<<grid_for(nB + 1, 256, h->num_sms * 8), 256, 0, h->stream>>>(ml, keys, nB,
                                                                                          h->Bptr_loc);
-    cudaStreamSynchronize(h->stream);
-    cudaFree(keys);
-    cudaFree(ids);
-    if (tmp) cudaFree(tmp);
     CA_TRY(st);
     CA_CUDA(cudaGetLastError());
     return CUALIGN_OK;
@@ -784,18 +782,16 @@ cualign_status bp_setup(cualign_bp *h)
     CA_TRY(dalloc(h, &h->Bcp, (size_t)nB + 1));
     CA_CUDA(cudaMemsetAsync(h->Bcp, 0, sizeof(int64_t), h->stream));
     if (nB > 0) {
-        int64_t *cnt = nullptr;
-        void *tmp = nullptr;
+        TmpBuf cb, tb_;
         size_t tb = 0;
-        CA_CUDA(cudaMalloc(&cnt, sizeof(int64_t) * (size_t)nB));
+        CA_CUDA(tmalloc(h, cb, sizeof(int64_t) * (size_t)nB));
+        int64_t *cnt = (int64_t *)cb.p;
         k_chunk_count<<<grid_for(nB, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB, Bptr, cnt);
         CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, cnt, h->Bcp + 1, (int)nB, h->stream));
-        CA_CUDA(cudaMalloc(&tmp, tb ? tb : 1));
-        CA_CUDA(cub::DeviceScan::InclusiveSum(tmp, tb, cnt, h->Bcp + 1, (int)nB, h->stream));
+        CA_CUDA(tmalloc(h, tb_, tb ? tb : 1));
+        CA_CUDA(cub::DeviceScan::InclusiveSum(tb_.p, tb, cnt, h->Bcp + 1, (int)nB, h->stream));
         CA_CUDA(cudaMemcpyAsync(&h->nchunks, h->Bcp + nB, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
         CA_CUDA(cudaStreamSynchronize(h->stream));
-        cudaFree(cnt);
-        cudaFree(tmp);
     }
     CA_TRY(dalloc(h, &h->chunk_b, (size_t)h->nchunks + 1));
     CA_TRY(dalloc(h, &h->Bct, (size_t)h->nchunks + 1));

@@ -21,13 +21,6 @@ namespace cualign {
 
 namespace {
 
-struct TmpBuf {
-    void *p = nullptr;
-    ~TmpBuf()
-    {
-        if (p) cudaFree(p);
-    }
-};
 
 #define FULL_MASK 0xffffffffu
 
@@ -244,6 +237,22 @@ constexpr int SBG_WARPS = 8;
 constexpr int SBG_SLOTS = 512;   // hash slots per warp (key j', value lane mask)
 constexpr int SBG_CAP = 256;     // inserts per group (load factor <= 1/2)
 
+// 32 x 32 bit-matrix transpose across a warp: lane L holds row L (bit t =
+// M[L][t]); afterwards lane t holds column t (bit L = M[L][t]).  Five
+// butterfly steps swap the off-diagonal blocks of size 16, 8, 4, 2, 1.
+__device__ __forceinline__ uint32_t warp_bit_transpose(uint32_t x, int lane)
+{
+    const uint32_t lowmask[5] = {0x0000ffffu, 0x00ff00ffu, 0x0f0f0f0fu, 0x33333333u, 0x55555555u};
+#pragma unroll
+    for (int s = 0; s < 5; s++) {
+        const int j = 16 >> s;
+        const uint32_t m = lowmask[s];
+        const uint32_t y = __shfl_xor_sync(FULL_MASK, x, j);
+        x = (lane & j) ? ((x & ~m) | ((y & ~m) >> j)) : ((x & m) | ((y & m) << j));
+    }
+    return x;
+}
+
 __device__ __forceinline__ int sbg_hash(int32_t b) { return (int)(((uint32_t)b * 2654435761u) >> 23); }
 
 // first lane k whose inclusive sum exceeds pos (incl nondecreasing)
@@ -387,20 +396,24 @@ k_sbuild_g(int32_t nA, const int64_t *__restrict__ Arow, const int32_t *__restri
                             }
                         }
                     }
-                    uint32_t any = __reduce_or_sync(FULL_MASK, hits);
-                    while (any) {
-                        const int tt = __ffs(any) - 1;
-                        any &= any - 1u;
-                        const bool mine = (hits >> tt) & 1u;
-                        const unsigned bal = __ballot_sync(FULL_MASK, mine);
-                        const int32_t run = __shfl_sync(FULL_MASK, cnt, tt);
-                        if (FILL) {
+                    // lane t gets the lanes whose candidate hit e_t (bit transpose
+                    // of the 32 hit masks): its count, and each hit's rank among
+                    // the lower lanes = its place in row e_t (ascending f)
+                    const uint32_t col = warp_bit_transpose(hits, lane);
+                    if (FILL) {
+                        const int R = __reduce_max_sync(FULL_MASK, (unsigned)__popc(hits));
+                        uint32_t rem = hits;
+                        for (int r = 0; r < R; r++) {
+                            const bool has = rem != 0u;
+                            const int tt = has ? __ffs(rem) - 1 : 0;
+                            rem &= rem - 1u;
+                            const uint32_t ct = __shfl_sync(FULL_MASK, col, tt);
+                            const int32_t run = __shfl_sync(FULL_MASK, cnt, tt);
                             const int64_t ob = __shfl_sync(FULL_MASK, obase, tt);
-                            if (mine)
-                                sq_ef[ob + run + __popc(bal & lt_mask)] = make_int2((int)(l0 + t0 + tt), (int)f);
+                            if (has) sq_ef[ob + run + __popc(ct & lt_mask)] = make_int2((int)(l0 + t0 + tt), (int)f);
                         }
-                        if (lane == tt) cnt += __popc(bal);
                     }
+                    cnt += __popc(col);
                 }
             }
             if (!FILL && lane < ng) ucnt[e_l] = cnt;
@@ -607,7 +620,7 @@ cualign_status build_L(cualign_bp *h, LDev &L, const cualign_edges *E, bool devi
     if (E->w) CA_TRY(upload(h, (void **)&L.w, E->w, sizeof(double) * m, device_ptrs));
     if (validate) {
         TmpBuf err;
-        CA_CUDA(cudaMalloc(&err.p, sizeof(int)));
+        CA_CUDA(tmalloc(h, err, sizeof(int)));
         CA_CUDA(cudaMemsetAsync(err.p, 0, sizeof(int), h->stream));
         if (m) k_check_edges<<<grid_for(m, 256, G), 256, 0, h->stream>>>(m, nA, nB, L.La, L.Lb, L.w,
                                                                           (int *)err.p);
@@ -623,8 +636,8 @@ cualign_status build_L(cualign_bp *h, LDev &L, const cualign_edges *E, bool devi
     CA_TRY(dalloc(h, &L.Bptr, (size_t)nB + 1));
     {
         TmpBuf keys_out, ids_in, tmp;
-        CA_CUDA(cudaMalloc(&keys_out.p, sizeof(int32_t) * (m ? m : 1)));
-        CA_CUDA(cudaMalloc(&ids_in.p, sizeof(int32_t) * (m ? m : 1)));
+        CA_CUDA(tmalloc(h, keys_out, sizeof(int32_t) * (m ? m : 1)));
+        CA_CUDA(tmalloc(h, ids_in, sizeof(int32_t) * (m ? m : 1)));
         if (m) {
             k_iota<<<grid_for(m, 256, G), 256, 0, h->stream>>>(m, (int32_t *)ids_in.p);
             int end_bit = 1;
@@ -633,7 +646,7 @@ cualign_status build_L(cualign_bp *h, LDev &L, const cualign_edges *E, bool devi
             CA_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tbytes, L.Lb, (int32_t *)keys_out.p,
                                                     (int32_t *)ids_in.p, L.Bedge, (int)m, 0, end_bit,
                                                     h->stream));
-            CA_CUDA(cudaMalloc(&tmp.p, tbytes ? tbytes : 1));
+            CA_CUDA(tmalloc(h, tmp, tbytes ? tbytes : 1));
             CA_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tbytes, L.Lb, (int32_t *)keys_out.p,
                                                     (int32_t *)ids_in.p, L.Bedge, (int)m, 0, end_bit,
                                                     h->stream));
@@ -666,7 +679,7 @@ cualign_status upload_graph(cualign_bp *h, const cualign_graph *g, const char *w
     CA_TRY(upload(h, (void **)rp, g->rowptr, sizeof(int64_t) * ((size_t)g->n + 1), devp));
     CA_TRY(upload(h, (void **)col, g->col, sizeof(int32_t) * (size_t)nnz, devp));
     TmpBuf err;
-    CA_CUDA(cudaMalloc(&err.p, sizeof(int)));
+    CA_CUDA(tmalloc(h, err, sizeof(int)));
     CA_CUDA(cudaMemsetAsync(err.p, 0, sizeof(int), h->stream));
     if (g->n)
         k_check_graph<<<grid_for(g->n, 256, h->num_sms * 8), 256, 0, h->stream>>>(g->n, nnz, *rp, *col,
@@ -697,7 +710,7 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
     h->a1 = h->L.nA;
     KScope ks(h, CUALIGN_K_INIT);
     TmpBuf ucnt, tmp, mx;
-    CA_CUDA(cudaMalloc(&ucnt.p, sizeof(int64_t) * (m ? m : 1)));
+    CA_CUDA(tmalloc(h, ucnt, sizeof(int64_t) * (m ? m : 1)));
     CA_TRY(dalloc(h, &h->sq_rp, (size_t)m + 1));
     CA_CUDA(cudaMemsetAsync(h->sq_rp, 0, sizeof(int64_t), h->stream));
     h->nsq = 0;
@@ -715,7 +728,7 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
             occ = 1;
         (void)cudaGetLastError();
         sbg_blocks = grid_for((int64_t)nA * 32, SBG_WARPS * 32, (int64_t)occ * h->num_sms);
-        CA_CUDA(cudaMalloc(&qctr.p, 2 * sizeof(unsigned long long)));
+        CA_CUDA(tmalloc(h, qctr, 2 * sizeof(unsigned long long)));
         CA_CUDA(cudaMemsetAsync(qctr.p, 0, 2 * sizeof(unsigned long long), h->stream));
     }
     if (m) {
@@ -733,7 +746,7 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
         CA_CUDA(cudaGetLastError());
         size_t tb = 0;
         CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, (int64_t *)ucnt.p, h->sq_rp + 1, (int)m, h->stream));
-        CA_CUDA(cudaMalloc(&tmp.p, tb ? tb : 1));
+        CA_CUDA(tmalloc(h, tmp, tb ? tb : 1));
         CA_CUDA(cub::DeviceScan::InclusiveSum(tmp.p, tb, (int64_t *)ucnt.p, h->sq_rp + 1, (int)m, h->stream));
         CA_CUDA(cudaMemcpyAsync(&h->nsq, h->sq_rp + m, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
         CA_CUDA(cudaStreamSynchronize(h->stream));
@@ -760,9 +773,9 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
         CA_CUDA(cudaGetLastError());
         // full row lengths: upper (ucnt) + lower (histogram of f) -> max row
         TmpBuf lcnt, tot, tmp2;
-        CA_CUDA(cudaMalloc(&lcnt.p, sizeof(unsigned int) * (size_t)m));
-        CA_CUDA(cudaMalloc(&tot.p, sizeof(int64_t) * (size_t)m));
-        CA_CUDA(cudaMalloc(&mx.p, sizeof(int64_t)));
+        CA_CUDA(tmalloc(h, lcnt, sizeof(unsigned int) * (size_t)m));
+        CA_CUDA(tmalloc(h, tot, sizeof(int64_t) * (size_t)m));
+        CA_CUDA(tmalloc(h, mx, sizeof(int64_t)));
         CA_CUDA(cudaMemsetAsync(lcnt.p, 0, sizeof(unsigned int) * (size_t)m, h->stream));
         k_lower_count<<<grid_for(h->nsq, 256, G), 256, 0, h->stream>>>(h->nsq, h->sq_ef, (unsigned int *)lcnt.p);
         k_row_total<<<grid_for(m, 256, G), 256, 0, h->stream>>>(m, (const int64_t *)ucnt.p,
@@ -770,7 +783,7 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
         CA_CUDA(cudaGetLastError());
         size_t tb = 0;
         CA_CUDA(cub::DeviceReduce::Max(nullptr, tb, (int64_t *)tot.p, (int64_t *)mx.p, (int)m, h->stream));
-        CA_CUDA(cudaMalloc(&tmp2.p, tb ? tb : 1));
+        CA_CUDA(tmalloc(h, tmp2, tb ? tb : 1));
         CA_CUDA(cub::DeviceReduce::Max(tmp2.p, tb, (int64_t *)tot.p, (int64_t *)mx.p, (int)m, h->stream));
         CA_CUDA(cudaMemcpyAsync(&h->max_row, mx.p, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
     }
@@ -807,9 +820,9 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
     {
         KScope ks(h, CUALIGN_K_INIT);
         TmpBuf cnt, ucnt, tmp, mx, tot, bnd;
-        CA_CUDA(cudaMalloc(&cnt.p, sizeof(int64_t) * (m ? m : 1)));
-        CA_CUDA(cudaMalloc(&ucnt.p, sizeof(int64_t) * (m ? m : 1)));
-        CA_CUDA(cudaMalloc(&mx.p, 3 * sizeof(int64_t)));
+        CA_CUDA(tmalloc(h, cnt, sizeof(int64_t) * (m ? m : 1)));
+        CA_CUDA(tmalloc(h, ucnt, sizeof(int64_t) * (m ? m : 1)));
+        CA_CUDA(tmalloc(h, mx, 3 * sizeof(int64_t)));
         CA_CUDA(cudaMemsetAsync(mx.p, 0, 3 * sizeof(int64_t), h->stream));
         int64_t host3[3] = {0, 0, 0}; // max row, s, squares (global)
         if (m) {
@@ -822,7 +835,7 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
             CA_CUDA(cub::DeviceReduce::Max(nullptr, t3, (int64_t *)cnt.p, (int64_t *)mx.p, (int)m, h->stream));
             CA_CUDA(cub::DeviceReduce::Sum(nullptr, t1, (int64_t *)cnt.p, (int64_t *)mx.p + 1, (int)m, h->stream));
             size_t t2 = t1 > t3 ? t1 : t3;
-            CA_CUDA(cudaMalloc(&tmp.p, t2 ? t2 : 1));
+            CA_CUDA(tmalloc(h, tmp, t2 ? t2 : 1));
             CA_CUDA(cub::DeviceReduce::Max(tmp.p, t3, (int64_t *)cnt.p, (int64_t *)mx.p, (int)m, h->stream));
             CA_CUDA(cub::DeviceReduce::Sum(tmp.p, t1, (int64_t *)cnt.p, (int64_t *)mx.p + 1, (int)m, h->stream));
             CA_CUDA(cub::DeviceReduce::Sum(tmp.p, t1, (int64_t *)ucnt.p, (int64_t *)mx.p + 2, (int)m, h->stream));
@@ -841,13 +854,13 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
         h->bounds.assign((size_t)h->world + 1, 0);
         h->bounds[(size_t)h->world] = m;
         if (h->world > 1 && m) {
-            CA_CUDA(cudaMalloc(&tot.p, sizeof(int64_t) * (size_t)m));
-            CA_CUDA(cudaMalloc(&bnd.p, sizeof(int64_t) * ((size_t)h->world + 1)));
+            CA_CUDA(tmalloc(h, tot, sizeof(int64_t) * (size_t)m));
+            CA_CUDA(tmalloc(h, bnd, sizeof(int64_t) * ((size_t)h->world + 1)));
             k_shard_cost<<<grid_for(m, 256, G), 256, 0, h->stream>>>(m, (const int64_t *)ucnt.p, (int64_t *)tot.p);
             size_t tb = 0;
             TmpBuf tmp2;
             CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, (int64_t *)tot.p, (int64_t *)tot.p, (int)m, h->stream));
-            CA_CUDA(cudaMalloc(&tmp2.p, tb ? tb : 1));
+            CA_CUDA(tmalloc(h, tmp2, tb ? tb : 1));
             CA_CUDA(cub::DeviceScan::InclusiveSum(tmp2.p, tb, (int64_t *)tot.p, (int64_t *)tot.p, (int)m, h->stream));
             k_shard_bounds<<<1, 32, 0, h->stream>>>(m, (const int64_t *)tot.p, h->L.La, h->L.Arow, h->world,
                                                     (int64_t *)bnd.p);
@@ -880,7 +893,7 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
             TmpBuf tmp3;
             CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, (int64_t *)cnt.p + h->e0, h->Srp + 1, (int)ml,
                                                   h->stream));
-            CA_CUDA(cudaMalloc(&tmp3.p, tb ? tb : 1));
+            CA_CUDA(tmalloc(h, tmp3, tb ? tb : 1));
             CA_CUDA(cub::DeviceScan::InclusiveSum(tmp3.p, tb, (int64_t *)cnt.p + h->e0, h->Srp + 1, (int)ml,
                                                   h->stream));
             CA_CUDA(cub::DeviceScan::InclusiveSum(tmp3.p, tb, (int64_t *)ucnt.p + h->e0, h->sq_rp + 1, (int)ml,
@@ -925,17 +938,19 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
     {
         KScope ks(h, CUALIGN_K_INIT);
         const int64_t nA = A->n;
+        TmpBuf cntb, startb, tmpb;
         int64_t *cnt = nullptr, *start = nullptr;
-        void *tmp = nullptr;
         size_t tb = 0;
         h->nApairs = 0;
         if (nA > 0) {
-            CA_CUDA(cudaMalloc(&cnt, sizeof(int64_t) * (size_t)nA));
-            CA_CUDA(cudaMalloc(&start, sizeof(int64_t) * (size_t)nA));
+            CA_CUDA(tmalloc(h, cntb, sizeof(int64_t) * (size_t)nA));
+            CA_CUDA(tmalloc(h, startb, sizeof(int64_t) * (size_t)nA));
+            cnt = (int64_t *)cntb.p;
+            start = (int64_t *)startb.p;
             k_upper_count<<<grid_for(nA, 256, G), 256, 0, h->stream>>>(nA, Ap, Aj, cnt);
             CA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, start, (int)nA, h->stream));
-            CA_CUDA(cudaMalloc(&tmp, tb ? tb : 1));
-            CA_CUDA(cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, start, (int)nA, h->stream));
+            CA_CUDA(tmalloc(h, tmpb, tb ? tb : 1));
+            CA_CUDA(cub::DeviceScan::ExclusiveSum(tmpb.p, tb, cnt, start, (int)nA, h->stream));
             int64_t last[2];
             CA_CUDA(cudaMemcpyAsync(&last[0], start + nA - 1, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
             CA_CUDA(cudaMemcpyAsync(&last[1], cnt + nA - 1, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
@@ -945,10 +960,6 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
         cualign_status st = dalloc(h, &h->Apairs, (size_t)h->nApairs + 1);
         if (st == CUALIGN_OK && h->nApairs)
             k_upper_fill<<<grid_for(nA, 256, G), 256, 0, h->stream>>>(nA, Ap, Aj, start, h->Apairs);
-        cudaStreamSynchronize(h->stream);
-        if (cnt) cudaFree(cnt);
-        if (start) cudaFree(start);
-        if (tmp) cudaFree(tmp);
         CA_TRY(st);
         CA_CUDA(cudaGetLastError());
         // E_B membership set for evaluate: >= 2 slots per undirected edge
@@ -998,8 +1009,8 @@ cualign_status tile_squares(cualign_bp *h)
     const int n = (int)h->nsq;
     TmpBuf keys, keys2, tmp;
     int2 *sorted = nullptr;
-    CA_CUDA(cudaMalloc(&keys.p, sizeof(uint32_t) * (size_t)n));
-    CA_CUDA(cudaMalloc(&keys2.p, sizeof(uint32_t) * (size_t)n));
+    CA_CUDA(tmalloc(h, keys, sizeof(uint32_t) * (size_t)n));
+    CA_CUDA(tmalloc(h, keys2, sizeof(uint32_t) * (size_t)n));
     CA_TRY(dalloc(h, &sorted, (size_t)n + 2));
     {
         KScope ks(h, CUALIGN_K_INIT);
@@ -1011,7 +1022,7 @@ cualign_status tile_squares(cualign_bp *h)
         unsigned long long *vout = reinterpret_cast<unsigned long long *>(sorted);
         CA_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, (const uint32_t *)keys.p, (uint32_t *)keys2.p, vin,
                                                 vout, n, 0, end_bit, h->stream));
-        CA_CUDA(cudaMalloc(&tmp.p, tb ? tb : 1));
+        CA_CUDA(tmalloc(h, tmp, tb ? tb : 1));
         CA_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tb, (const uint32_t *)keys.p, (uint32_t *)keys2.p, vin, vout,
                                                 n, 0, end_bit, h->stream));
         CA_CUDA(cudaMemsetAsync(sorted + n, 0, 2 * sizeof(int2), h->stream));
@@ -1041,9 +1052,9 @@ cualign_status ensure_csr(cualign_bp *h)
     }
     KScope ks(h, CUALIGN_K_INIT);
     TmpBuf k1, k2, tmp, rows;
-    CA_CUDA(cudaMalloc(&k1.p, sizeof(unsigned long long) * (size_t)s));
-    CA_CUDA(cudaMalloc(&k2.p, sizeof(unsigned long long) * (size_t)s));
-    CA_CUDA(cudaMalloc(&rows.p, sizeof(int32_t) * (size_t)s));
+    CA_CUDA(tmalloc(h, k1, sizeof(unsigned long long) * (size_t)s));
+    CA_CUDA(tmalloc(h, k2, sizeof(unsigned long long) * (size_t)s));
+    CA_CUDA(tmalloc(h, rows, sizeof(int32_t) * (size_t)s));
     const int G = h->num_sms * 16;
     k_csr_keys<<<grid_for(h->nsq, 256, G), 256, 0, h->stream>>>(h->nsq, h->sq_ef, (unsigned long long *)k1.p);
     CA_CUDA(cudaGetLastError());
@@ -1052,7 +1063,7 @@ cualign_status ensure_csr(cualign_bp *h)
     size_t tb = 0;
     CA_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, tb, (const unsigned long long *)k1.p,
                                            (unsigned long long *)k2.p, (int)s, 0, 32 + bits, h->stream));
-    CA_CUDA(cudaMalloc(&tmp.p, tb ? tb : 1));
+    CA_CUDA(tmalloc(h, tmp, tb ? tb : 1));
     CA_CUDA(cub::DeviceRadixSort::SortKeys(tmp.p, tb, (const unsigned long long *)k1.p, (unsigned long long *)k2.p,
                                            (int)s, 0, 32 + bits, h->stream));
     k_csr_cols<<<grid_for(s, 256, G), 256, 0, h->stream>>>(s, (const unsigned long long *)k2.p, h->Scol,

@@ -189,6 +189,25 @@ namespace cualign {
 
 // --------------------------------------------------------------- memory
 cualign_status dmalloc(cualign_bp *h, void **p, size_t bytes);
+cudaMemPool_t temp_pool(int dev); // cached pool for init temporaries (nullptr: use the default)
+
+// init temporaries: stream-ordered from a cached pool of their own (no
+// device-wide synchronisation in cudaFree, memory reused across handles)
+struct TmpBuf {
+    void *p = nullptr;
+    cudaStream_t s = nullptr;
+    ~TmpBuf()
+    {
+        if (p) cudaFreeAsync(p, s);
+    }
+};
+inline cudaError_t tmalloc(cualign_bp *h, TmpBuf &b, size_t bytes)
+{
+    b.s = h->stream;
+    cudaMemPool_t pool = temp_pool(h->dev);
+    if (pool) return cudaMallocFromPoolAsync(&b.p, bytes ? bytes : 1, pool, h->stream);
+    return cudaMallocAsync(&b.p, bytes ? bytes : 1, h->stream);
+}
 template <class T>
 inline cualign_status dalloc(cualign_bp *h, T **p, size_t n)
 {

@@ -114,3 +114,30 @@ def test_pipelined_runs_interleaved_with_eager_calls(ca):
         m1, i1 = h1.get_best()
         m2, i2 = h2.get_best()
         assert np.array_equal(m1, m2) and i1["best_score"] == i2["best_score"] and i1["iter"] == i2["iter"] == 9
+
+
+@pytest.mark.parametrize("mode", ["pipelined", "damped", "shards3"])
+def test_run_trace_infos_equal_step_by_step(ca, mode):
+    """cualign_bp_run_trace (the e2e loop): every step's round info, copied to
+    the host without a per-step synchronisation, equals the info of the
+    eager iterate(1) + round() sequence; the final state is identical."""
+    inst = make_config("P", scale=0.05)
+    flags = ca.FLAG_ROUND_DAMPED if mode == "damped" else 0
+    kw = {"world": 3} if mode == "shards3" else {}
+    n = 7
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags) as h1, \
+            ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags, **kw) as h2:
+        eager = []
+        for _ in range(n):
+            h1.iterate(1)
+            h1.round()
+            eager.append(h1.get_best(with_mate=False)[1])
+        traced = h2.run_trace(n)
+        assert len(traced) == n
+        for k in range(n):
+            for key in ("iter", "score", "score_y", "score_z", "overlap_y", "overlap_z", "card_y", "card_z",
+                        "source", "best_score", "best_iter"):
+                assert eager[k][key] == traced[k][key], (k, key, eager[k][key], traced[k][key])
+        m1, _ = h1.get_best()
+        m2, _ = h2.get_best()
+        assert np.array_equal(m1, m2)
