@@ -357,6 +357,21 @@ def main():
     torch.cuda.synchronize()
     pst = h.stats(reset=True)
 
+    # sharded: the exchanges of one step: bytes each rank
+    # receives (counted by the library per collective) against NVLink 5's
+    # 900 GB/s per direction, time from events around the exchanges
+    exchange = None
+    if world > 1:
+        x_bytes = max_over_ranks(st["comm_bytes_in"] / args.steps, world, device=f"cuda:{dev}")
+        x_ms = max_over_ranks(pst["comm_ms"] / prof_steps, world, device=f"cuda:{dev}")
+        x_gbs = x_bytes / (x_ms * 1e-3) / 1e9 if x_ms > 0 else None
+        exchange = {"bytes_in_per_iter_per_rank": x_bytes, "calls_per_iter": st["comm_calls"] / args.steps,
+                    "ms_per_iter": x_ms, "achieved": x_gbs, "peak": 900.0, "unit": "GB/s",
+                    "frac": (x_gbs / 900.0) if x_gbs else None,
+                    "transport": ("NCCL socket transport, all ranks on one GPU (CUALIGN_ONE_GPU=1): "
+                                  "not an NVLink number" if os.environ.get("CUALIGN_ONE_GPU") == "1"
+                                  else "NCCL (NVLink / NVSwitch)")}
+
     # value: iterations/s of config O; at N > 1 in O-equivalent iterations/s
     # (iterations/s x squares of the N-times-larger instance / squares of O),
     # i.e. the whole job's throughput in units of the N = 1 workload
@@ -480,6 +495,7 @@ def main():
         "iteration_roofline": {"achieved": it_gbs, "frac": it_gbs / peak, "alg_bytes": it_bytes,
                                "bp_ms": bp_ms},
         "kernel_ms_per_step": {k: v / prof_steps for k, v in cls_ms.items() if v},
+        "exchange": exchange,
         "kernel_timing": (f"CUDA event-record nodes around each kernel inside the captured step "
                           f"graph, {prof_steps} steps after the timed region"),
         "cpu_baseline": cpu,

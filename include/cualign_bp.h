@@ -158,6 +158,11 @@ typedef struct {
     int64_t launches;                              /* all kernels launched by the handle */
     int64_t class_launches[CUALIGN_NUM_KERNEL_CLASSES];
     double class_ms[CUALIGN_NUM_KERNEL_CLASSES];   /* summed event time */
+    /* sharded handles: exchanges since the last reset */
+    int64_t comm_calls;      /* exchange steps (a grouped set of collectives counts once) */
+    int64_t comm_bytes_in;   /* bytes this process's shard(s) received (all-gathered,
+                                reduced-to-owner or all-reduced data arriving from peers) */
+    double comm_ms;          /* summed event time of the exchanges (timing on) */
 } cualign_stats;
 /* kernel classes */
 #define CUALIGN_K_TOP2    0 /* a4: per-vertex top-2 of y^p (A rows) and z^p (B columns) */

@@ -87,10 +87,12 @@ class Sizes_t(ctypes.Structure):
 class Stats_t(ctypes.Structure):
     _fields_ = [("launches", ctypes.c_int64),
                 ("class_launches", ctypes.c_int64 * NUM_KERNEL_CLASSES),
-                ("class_ms", ctypes.c_double * NUM_KERNEL_CLASSES)]
+                ("class_ms", ctypes.c_double * NUM_KERNEL_CLASSES),
+                ("comm_calls", ctypes.c_int64), ("comm_bytes_in", ctypes.c_int64), ("comm_ms", ctypes.c_double)]
 
     def as_dict(self):
-        return {"launches": self.launches,
+        return {"launches": self.launches, "comm_calls": self.comm_calls, "comm_bytes_in": self.comm_bytes_in,
+                "comm_ms": self.comm_ms,
                 "class_launches": {KERNEL_CLASS_NAMES[i]: self.class_launches[i] for i in range(NUM_KERNEL_CLASSES)},
                 "class_ms": {KERNEL_CLASS_NAMES[i]: self.class_ms[i] for i in range(NUM_KERNEL_CLASSES)}}
 

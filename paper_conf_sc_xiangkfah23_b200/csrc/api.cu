@@ -139,6 +139,25 @@ KScope::~KScope()
     }
 }
 
+CommScope::CommScope(cualign_bp *h_, int64_t bytes_in) : h(h_)
+{
+    h->comm_calls++;
+    h->comm_bytes_in += bytes_in;
+    if (h->timing && !h->capturing) {
+        b = get_event(h);
+        cudaEventRecord(b, h->stream);
+    }
+}
+
+CommScope::~CommScope()
+{
+    if (b) {
+        cudaEvent_t e = get_event(h);
+        cudaEventRecord(e, h->stream);
+        h->comm_events.push_back({b, e});
+    }
+}
+
 void invalidate_graphs(cualign_bp *h)
 {
     for (int t = 0; t < 2; t++)
@@ -604,7 +623,8 @@ cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B, c
             h->max_row = s0->max_row;
             h->fp_bits = s0->fp_bits;
             h->bounds = s0->bounds;
-            st = shard_fsum(h); // F(S^p = 0) row sums for iteration 1
+            st = shard_setup(h);
+            if (st == CUALIGN_OK) st = shard_fsum(h); // F(S^p = 0) row sums for iteration 1
         }
     } else {
         if (st == CUALIGN_OK && h->world > 1) st = nccl_init_comm(h, params->nccl_unique_id);
@@ -615,6 +635,7 @@ cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B, c
         init_trace(h, "alloc_state");
         if (st == CUALIGN_OK) st = match_setup(h);
         init_trace(h, "match_setup");
+        if (st == CUALIGN_OK && h->world > 1) st = shard_setup(h);
         if (st == CUALIGN_OK) st = h->world > 1 ? shard_fsum(h) : bp_fsum(h); // F(S^p = 0) sums for iteration 1
         init_trace(h, "fsum");
     }
@@ -959,9 +980,26 @@ cualign_status cualign_bp_get_stats(cualign_bp *h, cualign_stats *stats, int32_t
             stats->class_ms[c] = 0.0;
         }
     }
+    if (stats) {
+        stats->comm_calls = 0;
+        stats->comm_bytes_in = 0;
+        stats->comm_ms = 0.0;
+    }
     for (cualign_bp *s : S) {
         resolve_events(s);
+        for (auto &ep : s->comm_events) {
+            float ms = 0.f;
+            if (cudaEventSynchronize(ep.b) == cudaSuccess && cudaEventElapsedTime(&ms, ep.a, ep.b) == cudaSuccess)
+                s->comm_ms += ms;
+            s->event_pool.push_back(ep.a);
+            s->event_pool.push_back(ep.b);
+        }
+        s->comm_events.clear();
+        (void)cudaGetLastError();
         if (stats) {
+            stats->comm_calls += s->comm_calls;
+            stats->comm_bytes_in += s->comm_bytes_in;
+            stats->comm_ms += s->comm_ms;
             stats->launches += s->launches;
             for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
                 stats->class_launches[c] += s->class_launches[c];
@@ -969,6 +1007,9 @@ cualign_status cualign_bp_get_stats(cualign_bp *h, cualign_stats *stats, int32_t
             }
         }
         if (reset) {
+            s->comm_calls = 0;
+            s->comm_bytes_in = 0;
+            s->comm_ms = 0.0;
             s->launches = 0;
             for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) {
                 s->class_launches[c] = 0;

@@ -92,6 +92,16 @@ struct cualign_bp {
     double2 *Btop_all = nullptr;         // world x nB gathered partials
     int64_t *Bptr_loc = nullptr;         // B incidence of the owned edges (top-2 partials)
     int32_t *Bedge_loc = nullptr;
+    // sharded square-pass halo (SURVEY §8(e) "S halo"): the squares {e < f}
+    // of the owned rows touch f > e, i.e. edges of this or HIGHER shards only.
+    // need: sorted remote f this shard reads u_f of and adds F_fe to, grouped
+    // by owner (need_off[q]..need_off[q+1]); give: owned ids the lower shards
+    // need, grouped by requester (give_off[r]..give_off[r+1])
+    int32_t *halo_need = nullptr, *halo_give = nullptr;
+    std::vector<int64_t> need_off, give_off;
+    int64_t n_need = 0, n_give = 0;
+    double *hu_out = nullptr, *hu_in = nullptr;                // packed u_f: give side -> need side
+    unsigned long long *ht_out = nullptr, *ht_in = nullptr;    // packed F sums: need side -> give side
 
     // S: CSR over edge ids (rows [e0, e1)), and the square layout
     int64_t s = 0, nsq = 0, max_row = 0;
@@ -120,6 +130,9 @@ struct cualign_bp {
     double2 *Bct = nullptr;             // nchunks: (max1, max2) of z^p over the chunk
     unsigned int *Bcnt = nullptr;       // nB: chunks finished (hub columns' last-arriver merge)
     double2 *Atop = nullptr, *Btop = nullptr; // per-vertex (max1, max2) of y^p / z^p
+    int64_t comm_calls = 0, comm_bytes_in = 0; // exchanges (sharded handles)
+    double comm_ms = 0.0;
+    std::vector<cualign::EventPair> comm_events;
     int32_t p = 0;                      // host mirror of the iteration count
     int *p_dev = nullptr;               // device iteration count (kernels read p_dev + 1)
     double2 *gh_dev = nullptr;          // gh[p] = (gamma^p, 1 - gamma^p)
@@ -246,6 +259,15 @@ __device__ __forceinline__ bool bhash_has(const unsigned long long *__restrict__
 void init_trace(cualign_bp *h, const char *what);
 
 // ------------------------------------------------------- launch accounting
+// an exchange between shards (NCCL or loopback copies): bytes received by
+// the shard and, with timing on, its event time (not counted as a launch)
+struct CommScope {
+    cualign_bp *h;
+    cudaEvent_t b = nullptr;
+    CommScope(cualign_bp *h_, int64_t bytes_in);
+    ~CommScope();
+};
+
 struct KScope {
     cualign_bp *h;
     int cls;
@@ -283,6 +305,7 @@ cualign_status bp_merge_top2(cualign_bp *h);           // gathered B partials ->
 cualign_status bp_add_u64(cualign_bp *h, unsigned long long *dst, const unsigned long long *src, int64_t n);
 
 // shard.cu
+cualign_status shard_setup(cualign_bp *h);  // square-pass halo lists (after the S build)
 cualign_status shard_fsum(cualign_bp *h);
 cualign_status shard_iterate(cualign_bp *h, int32_t n);
 cualign_status shard_round(cualign_bp *h);

@@ -7,11 +7,12 @@
 // entries of y^p, z^p, d.  Per iteration the exchanges are:
 //   1. B-side top-2: every shard reduces its owned edges per B vertex; the
 //      partials are all-gathered and merged (max is exact).
-//   2. u: each shard's owned slice is all-gathered (the square pass needs
-//      u_f of any f).
-//   3. F row sums: each shard accumulates fixed-point partial sums for every
-//      edge; the slices are reduce-scattered to their owners.  Integer sums
-//      are associative, so the result is bitwise the single-GPU one.
+//   2. u halo: a shard's squares {e < f} (e owned) touch f > e only, i.e.
+//      edges of the same or higher shards; the owners send exactly the u_f
+//      of those remote f (lists exchanged once at init, shard_setup).
+//   3. F halo: the F_fe the square pass adds for remote f go back to their
+//      owners (packed, scatter-added there).  Integer sums are associative,
+//      so the result is bitwise the single-GPU one.
 //   Rounding (a7) is sharded (NEXT-1, see match.cu dist_match_*): proposals
 //   from the owned A rows, per-round all-reduces of the B-side suitors; the
 //   final matching and its evaluation (a8) are then replicated.
@@ -22,7 +23,10 @@
 // against the unsharded one on a single GPU.
 #include "internal.cuh"
 
+#include <algorithm>
+#include <cub/cub.cuh>
 #include <dlfcn.h>
+#include <thrust/iterator/counting_iterator.h>
 #include <nccl.h>
 
 namespace cualign {
@@ -38,14 +42,13 @@ struct NcclApi {
     ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
     ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
     ncclResult_t (*AllGather)(const void *, void *, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
-    ncclResult_t (*Broadcast)(const void *, void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
-    ncclResult_t (*Reduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, int, ncclComm_t,
-                           cudaStream_t) = nullptr;
     ncclResult_t (*AllReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
                               cudaStream_t) = nullptr;
     ncclResult_t (*GroupStart)() = nullptr;
     ncclResult_t (*GroupEnd)() = nullptr;
     const char *(*GetErrorString)(ncclResult_t) = nullptr;
+    ncclResult_t (*Send)(const void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*Recv)(void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
 };
 
 NcclApi &nccl()
@@ -60,14 +63,15 @@ NcclApi &nccl()
             api.CommInitRank = (decltype(api.CommInitRank))dlsym(lib, "ncclCommInitRank");
             api.CommDestroy = (decltype(api.CommDestroy))dlsym(lib, "ncclCommDestroy");
             api.AllGather = (decltype(api.AllGather))dlsym(lib, "ncclAllGather");
-            api.Broadcast = (decltype(api.Broadcast))dlsym(lib, "ncclBroadcast");
-            api.Reduce = (decltype(api.Reduce))dlsym(lib, "ncclReduce");
             api.AllReduce = (decltype(api.AllReduce))dlsym(lib, "ncclAllReduce");
             api.GroupStart = (decltype(api.GroupStart))dlsym(lib, "ncclGroupStart");
             api.GroupEnd = (decltype(api.GroupEnd))dlsym(lib, "ncclGroupEnd");
             api.GetErrorString = (decltype(api.GetErrorString))dlsym(lib, "ncclGetErrorString");
-            api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.AllGather && api.Broadcast &&
-                     api.Reduce && api.AllReduce && api.GroupStart && api.GroupEnd && api.GetErrorString;
+            api.Send = (decltype(api.Send))dlsym(lib, "ncclSend");
+            api.Recv = (decltype(api.Recv))dlsym(lib, "ncclRecv");
+            api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.AllGather &&
+                     api.AllReduce && api.GroupStart && api.GroupEnd && api.GetErrorString &&
+                     api.Send && api.Recv;
         }
     }
     return api;
@@ -89,11 +93,85 @@ NcclApi &nccl()
 
 enum RedOp { RED_MAX_U64, RED_MIN_I32, RED_SUM_U64 };
 
+// halo helpers
+__global__ void k_gather_d(int64_t n, const int32_t *__restrict__ ids, const double *__restrict__ src,
+                           double *__restrict__ dst)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dst[i] = src[ids[i]];
+}
+__global__ void k_scatter_d(int64_t n, const int32_t *__restrict__ ids, const double *__restrict__ src,
+                            double *__restrict__ dst)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dst[ids[i]] = src[i];
+}
+__global__ void k_gather_u64(int64_t n, const int32_t *__restrict__ ids, const unsigned long long *__restrict__ src,
+                             unsigned long long *__restrict__ dst)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dst[i] = src[ids[i]];
+}
+// several requesters may send the same owned id: integer atomics (exact,
+// order-independent)
+__global__ void k_scatter_add_u64(int64_t n, const int32_t *__restrict__ ids,
+                                  const unsigned long long *__restrict__ src, unsigned long long *__restrict__ dst)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        if (src[i]) atomicAdd(dst + ids[i], src[i]);
+}
+__global__ void k_mark_remote(int64_t nsq, const int2 *__restrict__ sq_ef, int64_t e1, uint8_t *__restrict__ flag)
+{
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq; q += (int64_t)gridDim.x * blockDim.x) {
+        const int f = sq_ef[q].y;
+        if (f >= e1) flag[f] = 1;
+    }
+}
+
+cualign_status halo_pack_u(cualign_bp *q)
+{
+    KScope ks(q, CUALIGN_K_OTHER);
+    if (q->n_give)
+        k_gather_d<<<grid_for(q->n_give, 256, q->num_sms * 8), 256, 0, q->stream>>>(q->n_give, q->halo_give, q->u,
+                                                                                 q->hu_out);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+cualign_status halo_unpack_u(cualign_bp *r)
+{
+    KScope ks(r, CUALIGN_K_OTHER);
+    if (r->n_need)
+        k_scatter_d<<<grid_for(r->n_need, 256, r->num_sms * 8), 256, 0, r->stream>>>(r->n_need, r->halo_need, r->hu_in,
+                                                                                  r->u);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+cualign_status halo_pack_t(cualign_bp *r)
+{
+    KScope ks(r, CUALIGN_K_OTHER);
+    if (r->n_need)
+        k_gather_u64<<<grid_for(r->n_need, 256, r->num_sms * 8), 256, 0, r->stream>>>(r->n_need, r->halo_need,
+                                                                                   r->tacc, r->ht_out);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+cualign_status halo_unpack_t(cualign_bp *q)
+{
+    KScope ks(q, CUALIGN_K_OTHER);
+    if (q->n_give)
+        k_scatter_add_u64<<<grid_for(q->n_give, 256, q->num_sms * 8), 256, 0, q->stream>>>(q->n_give, q->halo_give,
+                                                                                        q->ht_in, q->tacc);
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
 struct Exchange {
     virtual ~Exchange() {}
+    // the square-pass halo: u_f to the shards that read it, F sums back
+    virtual cualign_status halo_lists(std::vector<cualign_bp *> &S) = 0;
+    virtual cualign_status halo_u(std::vector<cualign_bp *> &S) = 0;
+    virtual cualign_status halo_t(std::vector<cualign_bp *> &S) = 0;
     virtual cualign_status top2(std::vector<cualign_bp *> &S) = 0;
-    virtual cualign_status allgather(std::vector<cualign_bp *> &S, double *cualign_bp::*field) = 0;
-    virtual cualign_status reduce_t(std::vector<cualign_bp *> &S) = 0;
     // in-place all-reduce of an array of n entries held by every shard
     virtual cualign_status allreduce(std::vector<cualign_bp *> &S, void *(*field)(cualign_bp *), int64_t n,
                                      RedOp op) = 0;
@@ -117,6 +195,13 @@ __global__ void k_red_sum_u64(int64_t n, unsigned long long *dst, const unsigned
 
 size_t red_size(RedOp op) { return op == RED_MIN_I32 ? sizeof(int32_t) : sizeof(unsigned long long); }
 
+// bytes a shard receives (algorithmic, as a ring moves them) per exchange
+int64_t in_top2(const cualign_bp *q) { return (int64_t)(q->world - 1) * q->L.nB * (int64_t)sizeof(double2); }
+int64_t in_allreduce(const cualign_bp *q, int64_t n, RedOp op)
+{
+    return 2 * (int64_t)(q->world - 1) * n * (int64_t)red_size(op) / q->world;
+}
+
 cualign_status zero_unowned(cualign_bp *q)
 {
     const int64_t m = q->L.m;
@@ -128,10 +213,72 @@ cualign_status zero_unowned(cualign_bp *q)
 
 // ---------------------------------------------------------------- loopback
 struct Loopback : Exchange {
+    cualign_status halo_lists(std::vector<cualign_bp *> &S) override
+    {
+        const int w = (int)S.size();
+        for (int q = 0; q < w; q++) {
+            cualign_bp *o = S[(size_t)q];
+            o->give_off.assign((size_t)w + 1, 0);
+            for (int r = 0; r < w; r++)
+                o->give_off[(size_t)r + 1] = o->give_off[(size_t)r] + (S[(size_t)r]->need_off[(size_t)q + 1] -
+                                                                       S[(size_t)r]->need_off[(size_t)q]);
+            o->n_give = o->give_off[(size_t)w];
+            CA_TRY(dalloc(o, &o->halo_give, (size_t)o->n_give + 1));
+            for (int r = 0; r < w; r++) {
+                cualign_bp *n = S[(size_t)r];
+                const int64_t c = n->need_off[(size_t)q + 1] - n->need_off[(size_t)q];
+                if (c)
+                    CA_CUDA(cudaMemcpyAsync(o->halo_give + o->give_off[(size_t)r], n->halo_need + n->need_off[(size_t)q],
+                                            sizeof(int32_t) * (size_t)c, cudaMemcpyDeviceToDevice, o->stream));
+            }
+        }
+        return CUALIGN_OK;
+    }
+    cualign_status halo_u(std::vector<cualign_bp *> &S) override
+    {
+        const int w = (int)S.size();
+        for (cualign_bp *q : S) CA_TRY(halo_pack_u(q));
+        for (int r = 0; r < w; r++) {
+            cualign_bp *n = S[(size_t)r];
+            CommScope cs(n, n->n_need * (int64_t)sizeof(double));
+            for (int q = 0; q < w; q++) {
+                cualign_bp *o = S[(size_t)q];
+                const int64_t c = n->need_off[(size_t)q + 1] - n->need_off[(size_t)q];
+                if (c)
+                    CA_CUDA(cudaMemcpyAsync(n->hu_in + n->need_off[(size_t)q], o->hu_out + o->give_off[(size_t)r],
+                                            sizeof(double) * (size_t)c, cudaMemcpyDeviceToDevice, n->stream));
+            }
+        }
+        for (cualign_bp *r : S) CA_TRY(halo_unpack_u(r));
+        return CUALIGN_OK;
+    }
+    cualign_status halo_t(std::vector<cualign_bp *> &S) override
+    {
+        const int w = (int)S.size();
+        for (cualign_bp *r : S) CA_TRY(halo_pack_t(r));
+        for (int q = 0; q < w; q++) {
+            cualign_bp *o = S[(size_t)q];
+            CommScope cs(o, o->n_give * (int64_t)sizeof(unsigned long long));
+            for (int r = 0; r < w; r++) {
+                cualign_bp *n = S[(size_t)r];
+                const int64_t c = o->give_off[(size_t)r + 1] - o->give_off[(size_t)r];
+                if (c)
+                    CA_CUDA(cudaMemcpyAsync(o->ht_in + o->give_off[(size_t)r], n->ht_out + n->need_off[(size_t)q],
+                                            sizeof(unsigned long long) * (size_t)c, cudaMemcpyDeviceToDevice,
+                                            o->stream));
+            }
+        }
+        for (cualign_bp *q : S) {
+            CA_TRY(halo_unpack_t(q));
+            CA_TRY(zero_unowned(q));
+        }
+        return CUALIGN_OK;
+    }
     cualign_status top2(std::vector<cualign_bp *> &S) override
     {
         const int64_t nB = S[0]->L.nB;
         for (cualign_bp *q : S) {
+            CommScope cs(q, in_top2(q));
             for (cualign_bp *r : S)
                 CA_CUDA(cudaMemcpyAsync(q->Btop_all + (int64_t)r->rank * nB, r->Btop_part, sizeof(double2) * (size_t)nB,
                                         cudaMemcpyDeviceToDevice, q->stream));
@@ -139,34 +286,12 @@ struct Loopback : Exchange {
         }
         return CUALIGN_OK;
     }
-    cualign_status allgather(std::vector<cualign_bp *> &S, double *cualign_bp::*field) override
-    {
-        for (cualign_bp *r : S) {
-            const int64_t n = r->e1 - r->e0;
-            if (!n) continue;
-            for (cualign_bp *q : S)
-                if (q != r)
-                    CA_CUDA(cudaMemcpyAsync(q->*field + r->e0, r->*field + r->e0, sizeof(double) * (size_t)n,
-                                            cudaMemcpyDeviceToDevice, q->stream));
-        }
-        return CUALIGN_OK;
-    }
-    cualign_status reduce_t(std::vector<cualign_bp *> &S) override
-    {
-        for (cualign_bp *r : S) {
-            const int64_t n = r->e1 - r->e0;
-            if (!n) continue;
-            for (cualign_bp *q : S) // fixed order; integer sums are exact anyway
-                if (q != r) CA_TRY(bp_add_u64(r, r->tacc + r->e0, q->tacc + r->e0, n));
-        }
-        for (cualign_bp *q : S) CA_TRY(zero_unowned(q));
-        return CUALIGN_OK;
-    }
     cualign_status allreduce(std::vector<cualign_bp *> &S, void *(*field)(cualign_bp *), int64_t n,
                              RedOp op) override
     {
         // fold every shard into shard 0 (fixed order), then copy back
         cualign_bp *h = S[0];
+        for (cualign_bp *q : S) CommScope(q, in_allreduce(q, n, op)); // accounting only
         void *dst = field(h);
         const int grid = grid_for(n, 256, h->num_sms * 8);
         for (size_t r = 1; r < S.size() && n; r++) {
@@ -187,40 +312,98 @@ struct Loopback : Exchange {
 
 // -------------------------------------------------------------------- NCCL
 struct Nccl : Exchange {
-    cualign_status top2(std::vector<cualign_bp *> &S) override
+    cualign_status halo_lists(std::vector<cualign_bp *> &S) override
     {
         cualign_bp *h = S[0];
-        const int64_t nB = h->L.nB;
-        CA_NCCL(AllGather(h->Btop_part, h->Btop_all, (size_t)(2 * nB), ncclFloat64, (ncclComm_t)h->comm,
-                              h->stream));
-        return bp_merge_top2(h);
-    }
-    cualign_status allgather(std::vector<cualign_bp *> &S, double *cualign_bp::*field) override
-    {
-        // all-gather-v: one in-place broadcast per owner, grouped
-        cualign_bp *h = S[0];
-        double *buf = h->*field;
+        const int w = h->world, me = h->rank;
+        // need counts of every rank from every owner: all-gather of [w] int64
+        int64_t *cnt_d = nullptr;
+        CA_TRY(dalloc(h, &cnt_d, (size_t)w * (size_t)(w + 1)));
+        std::vector<int64_t> mine((size_t)w), all((size_t)w * w);
+        for (int q = 0; q < w; q++) mine[(size_t)q] = h->need_off[(size_t)q + 1] - h->need_off[(size_t)q];
+        CA_CUDA(cudaMemcpyAsync(cnt_d + (size_t)w * w, mine.data(), sizeof(int64_t) * (size_t)w,
+                                cudaMemcpyHostToDevice, h->stream));
+        CA_NCCL(AllGather(cnt_d + (size_t)w * w, cnt_d, (size_t)w, ncclInt64, (ncclComm_t)h->comm, h->stream));
+        CA_CUDA(cudaMemcpyAsync(all.data(), cnt_d, sizeof(int64_t) * (size_t)w * w, cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaStreamSynchronize(h->stream));
+        h->give_off.assign((size_t)w + 1, 0);
+        for (int r = 0; r < w; r++) h->give_off[(size_t)r + 1] = h->give_off[(size_t)r] + all[(size_t)r * w + me];
+        h->n_give = h->give_off[(size_t)w];
+        CA_TRY(dalloc(h, &h->halo_give, (size_t)h->n_give + 1));
+        // the id lists: every rank sends its need segment to each owner
         CA_NCCL(GroupStart());
-        for (int r = 0; r < h->world; r++) {
-            const int64_t off = h->bounds[(size_t)r], n = h->bounds[(size_t)r + 1] - off;
-            if (n) CA_NCCL(Broadcast(buf + off, buf + off, (size_t)n, ncclFloat64, r, (ncclComm_t)h->comm, h->stream));
+        for (int q = 0; q < w; q++) {
+            const int64_t c = h->need_off[(size_t)q + 1] - h->need_off[(size_t)q];
+            if (q != me && c)
+                CA_NCCL(Send(h->halo_need + h->need_off[(size_t)q], (size_t)c, ncclInt32, q, (ncclComm_t)h->comm,
+                             h->stream));
+        }
+        for (int r = 0; r < w; r++) {
+            const int64_t c = h->give_off[(size_t)r + 1] - h->give_off[(size_t)r];
+            if (r != me && c)
+                CA_NCCL(Recv(h->halo_give + h->give_off[(size_t)r], (size_t)c, ncclInt32, r, (ncclComm_t)h->comm,
+                             h->stream));
         }
         CA_NCCL(GroupEnd());
         return CUALIGN_OK;
     }
-    cualign_status reduce_t(std::vector<cualign_bp *> &S) override
+    cualign_status halo_u(std::vector<cualign_bp *> &S) override
     {
-        // reduce-scatter-v: one in-place reduce per owner, grouped
         cualign_bp *h = S[0];
-        CA_NCCL(GroupStart());
-        for (int r = 0; r < h->world; r++) {
-            const int64_t off = h->bounds[(size_t)r], n = h->bounds[(size_t)r + 1] - off;
-            if (n)
-                CA_NCCL(Reduce(h->tacc + off, h->tacc + off, (size_t)n, ncclUint64, ncclSum, r,
-                                   (ncclComm_t)h->comm, h->stream));
+        const int w = h->world, me = h->rank;
+        CA_TRY(halo_pack_u(h));
+        {
+            CommScope cs(h, h->n_need * (int64_t)sizeof(double));
+            CA_NCCL(GroupStart());
+            for (int r = 0; r < w; r++) {
+                const int64_t c = h->give_off[(size_t)r + 1] - h->give_off[(size_t)r];
+                if (r != me && c)
+                    CA_NCCL(Send(h->hu_out + h->give_off[(size_t)r], (size_t)c, ncclFloat64, r, (ncclComm_t)h->comm,
+                                 h->stream));
+            }
+            for (int q = 0; q < w; q++) {
+                const int64_t c = h->need_off[(size_t)q + 1] - h->need_off[(size_t)q];
+                if (q != me && c)
+                    CA_NCCL(Recv(h->hu_in + h->need_off[(size_t)q], (size_t)c, ncclFloat64, q, (ncclComm_t)h->comm,
+                                 h->stream));
+            }
+            CA_NCCL(GroupEnd());
         }
-        CA_NCCL(GroupEnd());
+        return halo_unpack_u(h);
+    }
+    cualign_status halo_t(std::vector<cualign_bp *> &S) override
+    {
+        cualign_bp *h = S[0];
+        const int w = h->world, me = h->rank;
+        CA_TRY(halo_pack_t(h));
+        {
+            CommScope cs(h, h->n_give * (int64_t)sizeof(unsigned long long));
+            CA_NCCL(GroupStart());
+            for (int q = 0; q < w; q++) {
+                const int64_t c = h->need_off[(size_t)q + 1] - h->need_off[(size_t)q];
+                if (q != me && c)
+                    CA_NCCL(Send(h->ht_out + h->need_off[(size_t)q], (size_t)c, ncclUint64, q, (ncclComm_t)h->comm,
+                                 h->stream));
+            }
+            for (int r = 0; r < w; r++) {
+                const int64_t c = h->give_off[(size_t)r + 1] - h->give_off[(size_t)r];
+                if (r != me && c)
+                    CA_NCCL(Recv(h->ht_in + h->give_off[(size_t)r], (size_t)c, ncclUint64, r, (ncclComm_t)h->comm,
+                                 h->stream));
+            }
+            CA_NCCL(GroupEnd());
+        }
+        CA_TRY(halo_unpack_t(h));
         return zero_unowned(h);
+    }
+    cualign_status top2(std::vector<cualign_bp *> &S) override
+    {
+        cualign_bp *h = S[0];
+        const int64_t nB = h->L.nB;
+        CommScope cs(h, in_top2(h));
+        CA_NCCL(AllGather(h->Btop_part, h->Btop_all, (size_t)(2 * nB), ncclFloat64, (ncclComm_t)h->comm,
+                              h->stream));
+        return bp_merge_top2(h);
     }
     cualign_status allreduce(std::vector<cualign_bp *> &S, void *(*field)(cualign_bp *), int64_t n,
                              RedOp op) override
@@ -230,6 +413,7 @@ struct Nccl : Exchange {
         if (!n) return CUALIGN_OK;
         const ncclDataType_t t = op == RED_MIN_I32 ? ncclInt32 : ncclUint64;
         const ncclRedOp_t o = op == RED_MAX_U64 ? ncclMax : (op == RED_MIN_I32 ? ncclMin : ncclSum);
+        CommScope cs(h, in_allreduce(h, n, op));
         CA_NCCL(AllReduce(buf, buf, (size_t)n, t, o, (ncclComm_t)h->comm, h->stream));
         return CUALIGN_OK;
     }
@@ -249,12 +433,60 @@ Exchange *exchange_for(cualign_bp *h, std::vector<cualign_bp *> &S)
 
 } // namespace
 
+// The square-pass halo of every shard: mark the remote f of the owned
+// squares, compact them (sorted), split by owner, exchange the lists.
+cualign_status shard_setup(cualign_bp *h)
+{
+    std::vector<cualign_bp *> S;
+    Exchange *X = exchange_for(h, S);
+    for (cualign_bp *s : S) {
+        KScope ks(s, CUALIGN_K_INIT);
+        const int64_t m = s->L.m;
+        TmpBuf flag, nsel, tmp;
+        CA_CUDA(tmalloc(s, flag, (size_t)m + 1));
+        CA_CUDA(tmalloc(s, nsel, sizeof(int64_t)));
+        CA_CUDA(cudaMemsetAsync(flag.p, 0, (size_t)m + 1, s->stream));
+        if (s->nsq)
+            k_mark_remote<<<grid_for(s->nsq, 256, s->num_sms * 8), 256, 0, s->stream>>>(s->nsq, s->sq_ef, s->e1,
+                                                                                     (uint8_t *)flag.p);
+        CA_CUDA(cudaGetLastError());
+        CA_TRY(dalloc(s, &s->halo_need, (size_t)m + 1)); // upper bound; the used prefix is n_need
+        size_t tb = 0;
+        thrust::counting_iterator<int32_t> iota(0);
+        CA_CUDA(cub::DeviceSelect::Flagged(nullptr, tb, iota, (const uint8_t *)flag.p, s->halo_need,
+                                           (int64_t *)nsel.p, (int)m, s->stream));
+        CA_CUDA(tmalloc(s, tmp, tb));
+        CA_CUDA(cub::DeviceSelect::Flagged(tmp.p, tb, iota, (const uint8_t *)flag.p, s->halo_need, (int64_t *)nsel.p,
+                                           (int)m, s->stream));
+        CA_CUDA(cudaMemcpyAsync(&s->n_need, nsel.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s->stream));
+        CA_CUDA(cudaStreamSynchronize(s->stream));
+        std::vector<int32_t> need((size_t)s->n_need);
+        if (s->n_need)
+            CA_CUDA(cudaMemcpy(need.data(), s->halo_need, sizeof(int32_t) * (size_t)s->n_need, cudaMemcpyDeviceToHost));
+        const int w = s->world;
+        s->need_off.assign((size_t)w + 1, 0);
+        for (int q = 0; q < w; q++)
+            s->need_off[(size_t)q + 1] =
+                std::lower_bound(need.begin(), need.end(), (int32_t)std::min<int64_t>(s->bounds[(size_t)q + 1], INT32_MAX)) -
+                need.begin();
+        s->need_off[(size_t)w] = s->n_need;
+        CA_TRY(dalloc(s, &s->hu_in, (size_t)s->n_need + 1));
+        CA_TRY(dalloc(s, &s->ht_out, (size_t)s->n_need + 1));
+    }
+    CA_TRY(X->halo_lists(S));
+    for (cualign_bp *s : S) {
+        CA_TRY(dalloc(s, &s->hu_out, (size_t)s->n_give + 1));
+        CA_TRY(dalloc(s, &s->ht_in, (size_t)s->n_give + 1));
+    }
+    return CUALIGN_OK;
+}
+
 cualign_status shard_fsum(cualign_bp *h)
 {
     std::vector<cualign_bp *> S;
     Exchange *X = exchange_for(h, S);
     for (cualign_bp *s : S) CA_TRY(bp_fsum(s));
-    return X->reduce_t(S);
+    return X->halo_t(S);
 }
 
 cualign_status shard_iterate(cualign_bp *h, int32_t n)
@@ -266,9 +498,9 @@ cualign_status shard_iterate(cualign_bp *h, int32_t n)
         for (cualign_bp *s : S) CA_TRY(bp_front_top2(s));
         CA_TRY(X->top2(S));
         for (cualign_bp *s : S) CA_TRY(bp_front_edge(s));
-        CA_TRY(X->allgather(S, &cualign_bp::u));
+        CA_TRY(X->halo_u(S));
         for (cualign_bp *s : S) CA_TRY(bp_iterate_back(s));
-        CA_TRY(X->reduce_t(S));
+        CA_TRY(X->halo_t(S));
         for (cualign_bp *s : S) s->p += 1;
     }
     h->p = S[0]->p;

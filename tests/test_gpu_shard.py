@@ -119,3 +119,23 @@ def test_sharded_rounding_merge_rounds(ca, world):
         got, _, _ = ca.match(inst.L, inst.L.n_a, inst.L.n_b, st["yc"])
         assert np.array_equal(got, want)
         assert np.array_equal(h1.get_best()[0], hs.get_best()[0])
+
+
+def test_exchange_accounting_virtual_shards(ca):
+    """Bytes the shards receive per iteration: the B-side
+    top-2 all-gather, (w-1)·n_B·16 per shard, plus the square-pass halo (u_f
+    of the remote f a shard's squares touch, and their F sums back to the
+    owners) -- strictly less than all-gathering u and reducing full F-sum
+    vectors, (w-1)·16·m summed over the shards."""
+    inst = make_config("O", scale=0.01)
+    w = 3
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, world=w) as h:
+        h.stats(reset=True)
+        h.iterate(2)
+        st = h.stats(reset=True)
+        m, nB = inst.L.m, inst.B.n
+        top2 = 2 * w * (w - 1) * nB * 16
+        halo = st["comm_bytes_in"] - top2
+        assert 0 < halo < 2 * (w - 1) * 16 * m
+        assert halo % 16 == 0  # every halo entry moves once each way (8 B u + 8 B F sum)
+        assert st["comm_calls"] > 0
