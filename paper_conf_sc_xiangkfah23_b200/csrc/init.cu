@@ -42,30 +42,35 @@ __device__ __forceinline__ bool bsearch_i32(const int32_t *x, int64_t lo, int64_
     return false;
 }
 
+// One warp per row (hub rows of ~10^3 entries would serialise one thread):
+// lanes take the row's entries; sortedness compares each entry with its left
+// neighbour, symmetry binary-searches i in row c.
 __global__ void k_check_graph(int32_t n, int64_t nnz, const int64_t *rp, const int32_t *col,
                               int *err)
 {
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
-         i += (int64_t)gridDim.x * blockDim.x) {
-        int64_t lo = rp[i], hi = rp[i + 1];
+    const int lane = threadIdx.x & 31;
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t i = warp; i < n; i += nwarps) {
+        const int64_t lo = rp[i], hi = rp[i + 1];
         if (lo < 0 || hi < lo || hi > nnz) {
-            atomicOr(err, E_ROWPTR);
+            if (lane == 0) atomicOr(err, E_ROWPTR);
             continue;
         }
-        int32_t prev = -1;
-        for (int64_t x = lo; x < hi; x++) {
-            int32_t c = col[x];
+        int bad = 0;
+        for (int64_t x = lo + lane; x < hi; x += 32) {
+            const int32_t c = col[x];
             if (c < 0 || c >= n) {
-                atomicOr(err, E_COLRANGE);
-                break;
+                bad |= E_COLRANGE;
+                continue;
             }
-            if (c == (int32_t)i) atomicOr(err, E_SELFLOOP);
-            if (c <= prev) atomicOr(err, E_UNSORTED);
-            prev = c;
-            int64_t clo = rp[c], chi = rp[c + 1];
-            if (clo < 0 || chi < clo || chi > nnz || !bsearch_i32(col, clo, chi, (int32_t)i))
-                atomicOr(err, E_ASYM);
+            if (c == (int32_t)i) bad |= E_SELFLOOP;
+            if (x > lo && c <= col[x - 1]) bad |= E_UNSORTED;
+            const int64_t clo = rp[c], chi = rp[c + 1];
+            if (clo < 0 || chi < clo || chi > nnz || !bsearch_i32(col, clo, chi, (int32_t)i)) bad |= E_ASYM;
         }
+        bad = __reduce_or_sync(FULL_MASK, bad);
+        if (lane == 0 && bad) atomicOr(err, bad);
     }
 }
 
@@ -547,12 +552,17 @@ __global__ void k_upper_count(int64_t n, const int64_t *__restrict__ rp, const i
 }
 
 // insert every undirected B edge {u < v} into the membership set
+// one warp per B vertex (lanes over the row: hub rows do not serialise)
 __global__ void k_bhash_insert(int64_t n, const int64_t *__restrict__ rp, const int32_t *__restrict__ col,
                                unsigned long long *__restrict__ T, int log2n)
 {
     const uint64_t mask = (1ull << log2n) - 1;
-    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n; u += (int64_t)gridDim.x * blockDim.x) {
-        for (int64_t x = rp[u]; x < rp[u + 1]; x++) {
+    const int lane = threadIdx.x & 31;
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u = warp; u < n; u += nwarps) {
+        const int64_t hi = rp[u + 1];
+        for (int64_t x = rp[u] + lane; x < hi; x += 32) {
             const int32_t v = col[x];
             if (v <= (int32_t)u) continue;
             const unsigned long long key = bhash_key((int32_t)u, v);
@@ -682,7 +692,7 @@ cualign_status upload_graph(cualign_bp *h, const cualign_graph *g, const char *w
     CA_CUDA(tmalloc(h, err, sizeof(int)));
     CA_CUDA(cudaMemsetAsync(err.p, 0, sizeof(int), h->stream));
     if (g->n)
-        k_check_graph<<<grid_for(g->n, 256, h->num_sms * 8), 256, 0, h->stream>>>(g->n, nnz, *rp, *col,
+        k_check_graph<<<grid_for((int64_t)g->n * 32, 256, h->num_sms * 16), 256, 0, h->stream>>>(g->n, nnz, *rp, *col,
                                                                                    (int *)err.p);
     CA_CUDA(cudaGetLastError());
     CA_TRY(check_flags(h, (int *)err.p, what));
@@ -970,7 +980,7 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
         CA_CUDA(cudaMemsetAsync(h->Bhash, 0xff, sizeof(unsigned long long) << lg, h->stream));
         const int64_t nB = B->n;
         if (nB > 0)
-            k_bhash_insert<<<grid_for(nB, 256, G), 256, 0, h->stream>>>(nB, Bp, Bj, h->Bhash, lg);
+            k_bhash_insert<<<grid_for(nB * 32, 256, h->num_sms * 16), 256, 0, h->stream>>>(nB, Bp, Bj, h->Bhash, lg);
         CA_CUDA(cudaGetLastError());
     }
     init_trace(h, "pairs + E_B set");
