@@ -41,10 +41,11 @@ using namespace ptx;
 
 constexpr int KNN_BM = 128;       // A rows per CTA (MMA M)
 constexpr int KNN_KMAX = 32;      // max neighbours per row
-constexpr int KNN_EPI_H = 1;      // epilogue warps per TMEM lane quarter (column interleave)
 constexpr int KNN_CB = 16;        // per-row candidate buffer (entries above the row's k-th best)
-constexpr int KNN_EPI_WARPS = 4 * KNN_EPI_H; // one A row per thread of each quarter
-constexpr int KNN_THREADS = (2 + KNN_EPI_WARPS) * 32;
+// EH epilogue warps per TMEM lane quarter (column interleave), 2 when the
+// per-row top-k arrays of both fit next to >= 2 B stages (k_knn_tc<BN, EH>)
+template <int EH>
+constexpr int knn_threads() { return (2 + 4 * EH) * 32; }
 
 // Unit rows -> bf16 -> swizzled tile image.  Tile t holds rows [t*R, t*R+R),
 // K-block kb (64 columns) of the tile at byte (t*KB + kb) * R*128, row rr at
@@ -84,11 +85,11 @@ __global__ void k_knn_prep(const float *__restrict__ Y, int32_t n, int32_t d, in
 
 // Partial top-k of one CTA: rows [rb*128, +128) x B tiles [t0, t1).
 // Output pv / pi: [row][split][half][k] (unsorted), idx INT_MAX = empty.
-template <int BN>
-__global__ void __launch_bounds__(KNN_THREADS, 1)
+template <int BN, int EH>
+__global__ void __launch_bounds__(knn_threads<EH>(), 1)
 k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32_t n_a, int32_t n_b, int32_t KB,
          int32_t k, int32_t ntilesB, int32_t tiles_per_split, int32_t nstages, float *__restrict__ pv,
-         int32_t *__restrict__ pi)
+         int32_t *__restrict__ pi, int probe)
 {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     // the swizzle atoms need 1024-byte aligned tiles: align the base explicitly
@@ -98,10 +99,10 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
     uint8_t *sA = smem;
     uint8_t *sB = smem + a_bytes;                         // nstages x b_bytes (multiples of 1024)
     float *tv_all = reinterpret_cast<float *>(sB + (size_t)nstages * b_bytes);          // [H][k][128]
-    int32_t *ti_all = reinterpret_cast<int32_t *>(tv_all + KNN_EPI_H * KNN_KMAX * KNN_BM); // [H][k][128]
-    float *cv_all = reinterpret_cast<float *>(ti_all + KNN_EPI_H * KNN_KMAX * KNN_BM);     // [H][CB][128]
-    int32_t *ci_all = reinterpret_cast<int32_t *>(cv_all + KNN_EPI_H * KNN_CB * KNN_BM);    // [H][CB][128]
-    uint64_t *bars = reinterpret_cast<uint64_t *>(ci_all + KNN_EPI_H * KNN_CB * KNN_BM);
+    int32_t *ti_all = reinterpret_cast<int32_t *>(tv_all + EH * k * KNN_BM);  // [H][k][128]
+    float *cv_all = reinterpret_cast<float *>(ti_all + EH * k * KNN_BM);      // [H][CB][128]
+    int32_t *ci_all = reinterpret_cast<int32_t *>(cv_all + EH * KNN_CB * KNN_BM); // [H][CB][128]
+    uint64_t *bars = reinterpret_cast<uint64_t *>(ci_all + EH * KNN_CB * KNN_BM);
     uint64_t *full = bars;                  // [nstages]
     uint64_t *empty = bars + nstages;       // [nstages]
     uint64_t *tfull = bars + 2 * nstages;   // [2]
@@ -122,7 +123,7 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
         }
         for (int b = 0; b < 2; b++) {
             mbar_init(&tfull[b], 1);
-            mbar_init(&tempty[b], KNN_EPI_WARPS);
+            mbar_init(&tempty[b], 4 * EH);
         }
         mbar_init(afull, 1);
         fence_mbar_init();
@@ -159,7 +160,7 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
                 if (i >= 2) mbar_wait(&tempty[buf], (uint32_t)((i >> 1) - 1) & 1u);
                 tc_fence_after();
                 const uint32_t b_base = smem_addr(sB + (size_t)s * b_bytes);
-                for (int kb = 0; kb < KB; kb++) {
+                for (int kb = 0; kb < (probe == 2 ? 0 : KB); kb++) { // probe 2: no MMA (timing only)
 #pragma unroll
                     for (int kk = 0; kk < 4; kk++) { // K = 16 bf16 = 32 bytes per instruction
                         const uint64_t ad = sw128_kmajor_desc(a_base + kb * (KNN_BM * 128) + kk * 32);
@@ -173,14 +174,14 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
         }
     } else {
         // --------------------------------------------------- epilogue
-        // warp w may read TMEM lanes 32*(w%4)..+31 only; the KNN_EPI_H warps of
+        // warp w may read TMEM lanes 32*(w%4)..+31 only; the EH warps of
         // one quarter take interleaved 32-column chunks of each tile and keep
         // their own running top-k (merged by k_knn_merge)
         const int q = warp & 3;            // TMEM lane quarter this warp may access
         const int half = (warp - 2) >> 2;  // which chunks of a tile
         const int row = q * 32 + lane;     // A row within the block = TMEM lane
-        float *tv = tv_all + half * KNN_KMAX * KNN_BM;
-        int32_t *ti = ti_all + half * KNN_KMAX * KNN_BM;
+        float *tv = tv_all + half * k * KNN_BM;
+        int32_t *ti = ti_all + half * k * KNN_BM;
         float *cv = cv_all + half * KNN_CB * KNN_BM;
         int32_t *ci = ci_all + half * KNN_CB * KNN_BM;
         for (int j = 0; j < k; j++) {
@@ -224,7 +225,7 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
             tc_fence_after();
             const int vbase = (t0 + i) * BN;
 #pragma unroll 1
-            for (int c = half; c < BN / 32; c += KNN_EPI_H) {
+            for (int c = half; c < (probe == 1 ? 0 : BN / 32); c += EH) { // probe 1: no epilogue (timing only)
                 uint32_t r[32];
                 __syncwarp(); // .sync.aligned load: reconverge after a fold
                 tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN + c * 32), r);
@@ -271,7 +272,7 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
         fold();
         const int64_t u = (int64_t)rb * KNN_BM + row;
         if (u < n_a) {
-            const int64_t o = ((u * nsplit + split) * KNN_EPI_H + half) * k;
+            const int64_t o = ((u * nsplit + split) * EH + half) * k;
             for (int j = 0; j < k; j++) {
                 pv[o + j] = tv[j * KNN_BM + row];
                 pi[o + j] = ti[j * KNN_BM + row];
@@ -334,16 +335,19 @@ __global__ void k_knn_merge(int32_t n_a, int32_t k, int32_t nsplit, const float 
     }
 }
 
-template <int BN>
+template <int BN, int EH>
 cualign_status knn_launch(cualign_bp *h, const uint8_t *Asw, const uint8_t *Bsw, int32_t n_a, int32_t n_b,
                           int32_t KB, int32_t k, float *pv, int32_t *pi, int32_t nsplit, int32_t tps,
                           int32_t nstages, size_t smem)
 {
-    auto fn = k_knn_tc<BN>;
+    auto fn = k_knn_tc<BN, EH>;
     CA_CUDA(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int32_t ntilesB = (n_b + BN - 1) / BN;
     dim3 grid((unsigned)((n_a + KNN_BM - 1) / KNN_BM), (unsigned)nsplit);
-    fn<<<grid, KNN_THREADS, smem, h->stream>>>(Asw, Bsw, n_a, n_b, KB, k, ntilesB, tps, nstages, pv, pi);
+    // CUALIGN_KNN_PROBE (timing probes, wrong results): 1 = no epilogue, 2 = no MMA
+    static const int probe = getenv("CUALIGN_KNN_PROBE") ? atoi(getenv("CUALIGN_KNN_PROBE")) : 0;
+    fn<<<grid, knn_threads<EH>(), smem, h->stream>>>(Asw, Bsw, n_a, n_b, KB, k, ntilesB, tps, nstages, pv, pi,
+                                                     probe);
     CA_CUDA(cudaGetLastError());
     return CUALIGN_OK;
 }
@@ -355,7 +359,32 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
 {
     const bool devp = (h->flags & CUALIGN_FLAG_DEVICE_PTRS) != 0;
     const int32_t KB = (d + 63) / 64;
-    const int BN = KB <= 2 ? 256 : 128;
+    // shared memory: A tile, B stages, per-row top-k arrays of EH epilogue
+    // warps per TMEM lane quarter, barriers.  Two warps per quarter (the
+    // epilogue is latency-bound with one warp per SMSP) when their arrays fit
+    // next to >= 2 B stages of 128 columns; else one warp, BN = 256 for d <= 128
+    const size_t a_bytes = (size_t)KB * KNN_BM * 128;
+    int smem_optin = 0;
+    {
+        int dev = 0;
+        CA_CUDA(cudaGetDevice(&dev));
+        CA_CUDA(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    }
+    auto fixed_for = [&](int eh) { return a_bytes + (size_t)eh * (k + KNN_CB) * KNN_BM * 8 + 256; };
+    auto stages_for = [&](int eh, int bn) -> int32_t {
+        const size_t f = fixed_for(eh) + 1024, bb = (size_t)KB * bn * 128;
+        return f >= (size_t)smem_optin ? 0 : (int32_t)std::min<size_t>(4, ((size_t)smem_optin - f) / bb);
+    };
+    static const int eh_env = getenv("CUALIGN_KNN_EH") ? atoi(getenv("CUALIGN_KNN_EH")) : 1;
+    const int EH = (eh_env >= 2 && stages_for(2, 128) >= 2) ? 2 : 1;
+    const int BN = (EH == 1 && KB <= 2) ? 256 : 128;
+    const int32_t nstages = stages_for(EH, BN);
+    if (nstages < 1) {
+        set_error("cualign_knn: d = %d needs more shared memory than available", d);
+        return CUALIGN_EINVAL;
+    }
+    const size_t b_bytes = (size_t)KB * BN * 128;
+    const size_t smem = fixed_for(EH) + (size_t)nstages * b_bytes + 1024; // +1024: alignment slack
     const int64_t rowsA = ((int64_t)n_a + KNN_BM - 1) / KNN_BM * KNN_BM;
     const int64_t rowsB = ((int64_t)n_b + BN - 1) / BN * BN;
     float *dA = nullptr, *dB = nullptr;
@@ -392,23 +421,10 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
     nsplit = std::max(1, std::min(nsplit, std::max(1, ntilesB / 4)));
     const int32_t tps = (ntilesB + nsplit - 1) / nsplit;
     nsplit = (ntilesB + tps - 1) / tps;
-    // shared memory: A tile, B stages, top-k arrays, barriers
-    const size_t a_bytes = (size_t)KB * KNN_BM * 128, b_bytes = (size_t)KB * BN * 128;
-    const size_t fixed = a_bytes + (size_t)KNN_EPI_H * (KNN_KMAX + KNN_CB) * KNN_BM * 8 + 256;
-    int smem_optin = 0;
-    int dev = 0;
-    CA_CUDA(cudaGetDevice(&dev));
-    CA_CUDA(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
-    int32_t nstages = (int32_t)std::min<size_t>(4, (smem_optin - fixed - 1024) / b_bytes);
-    if (nstages < 1) {
-        set_error("cualign_knn: d = %d needs more shared memory than available", d);
-        return CUALIGN_EINVAL;
-    }
-    const size_t smem = fixed + (size_t)nstages * b_bytes + 1024; // +1024: alignment slack
     float *pv = nullptr;
     int32_t *pi = nullptr;
-    CA_TRY(dalloc(h, &pv, (size_t)n_a * nsplit * KNN_EPI_H * k));
-    CA_TRY(dalloc(h, &pi, (size_t)n_a * nsplit * KNN_EPI_H * k));
+    CA_TRY(dalloc(h, &pv, (size_t)n_a * nsplit * EH * k));
+    CA_TRY(dalloc(h, &pi, (size_t)n_a * nsplit * EH * k));
     int32_t *oa = La, *ob = Lb;
     double *ow = Lw;
     const int64_t m = (int64_t)n_a * k;
@@ -419,13 +435,14 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
     }
     {
         KScope ks(h, CUALIGN_K_OTHER);
-        if (BN == 256)
-            CA_TRY(knn_launch<256>(h, (const uint8_t *)Asw, (const uint8_t *)Bsw, n_a, n_b, KB, k, pv, pi, nsplit, tps,
-                                   nstages, smem));
-        else
-            CA_TRY(knn_launch<128>(h, (const uint8_t *)Asw, (const uint8_t *)Bsw, n_a, n_b, KB, k, pv, pi, nsplit, tps,
-                                   nstages, smem));
-        k_knn_merge<<<grid_for(n_a, 128, G), 128, 0, h->stream>>>(n_a, k, nsplit * KNN_EPI_H, pv, pi, oa, ob, ow);
+        const uint8_t *a8 = (const uint8_t *)Asw, *b8 = (const uint8_t *)Bsw;
+        cualign_status lst;
+        if (BN == 256 && EH == 2) lst = knn_launch<256, 2>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
+        else if (BN == 256) lst = knn_launch<256, 1>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
+        else if (EH == 2) lst = knn_launch<128, 2>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
+        else lst = knn_launch<128, 1>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
+        CA_TRY(lst);
+        k_knn_merge<<<grid_for(n_a, 128, G), 128, 0, h->stream>>>(n_a, k, nsplit * EH, pv, pi, oa, ob, ow);
         CA_CUDA(cudaGetLastError());
     }
     if (!devp) {
