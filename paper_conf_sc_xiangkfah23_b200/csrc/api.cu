@@ -637,6 +637,7 @@ cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B, c
         init_trace(h, "match_setup");
         if (st == CUALIGN_OK && h->world > 1) st = shard_setup(h);
         if (st == CUALIGN_OK) st = h->world > 1 ? shard_fsum(h) : bp_fsum(h); // F(S^p = 0) sums for iteration 1
+        if (st == CUALIGN_OK && h->world == 1) st = bp_top2(h);                 // othermax inputs of iteration 1
         init_trace(h, "fsum");
     }
     if (st == CUALIGN_OK) {
@@ -962,6 +963,7 @@ cualign_status cualign_bp_set_state(cualign_bp *h, const double *yp, const doubl
     CA_TRY(ensure_gh(h, (int64_t)p + 1));
     CA_CUDA(cudaMemcpyAsync(h->p_dev, &h->p, sizeof(int), cudaMemcpyHostToDevice, h->stream));
     CA_TRY(bp_fsum(h));
+    CA_TRY(bp_top2(h)); // othermax inputs of the next iteration from the injected y^p, z^p
     CA_CUDA(cudaStreamSynchronize(h->stream));
     return CUALIGN_OK;
 }

@@ -810,13 +810,9 @@ cualign_status bp_fsum(cualign_bp *h)
 // Start of an iteration: the device counter advances to this iteration p
 // (kernels read gh[p]); per-vertex top-2 of y^p over the owned A rows and of
 // z^p over the B columns (partial over the owned edges when sharded).
-cualign_status bp_front_top2(cualign_bp *h)
+// per-vertex top-2 of the current y^p (A rows) and z^p (B columns)
+cualign_status bp_top2(cualign_bp *h)
 {
-    {
-        KScope ks(h, CUALIGN_K_OTHER);
-        k_advance<<<1, 1, 0, h->stream>>>(h->p_dev);
-        CA_CUDA(cudaGetLastError());
-    }
     if (h->L.m > 0) {
         KScope ks(h, CUALIGN_K_TOP2);
         const bool sh = h->world > 1;
@@ -827,6 +823,22 @@ cualign_status bp_front_top2(cualign_bp *h)
             k_top2<<<grid_for((T.nA + T.nchunks) * TG, 256, 1 << 30), 256, 0, h->stream>>>(T);
         CA_CUDA(cudaGetLastError());
     }
+    return CUALIGN_OK;
+}
+
+// Start of an iteration: the device counter advances to this iteration p.
+// Unsharded, the top-2 inputs of iteration p were computed right after the
+// k_edge of iteration p-1 (while y^p, z^p are still in L2 -- the square pass
+// streams ~2 GB through it before the next iteration starts) or at init /
+// set_state; sharded, the partial top-2 is computed here and then merged.
+cualign_status bp_front_top2(cualign_bp *h)
+{
+    {
+        KScope ks(h, CUALIGN_K_OTHER);
+        k_advance<<<1, 1, 0, h->stream>>>(h->p_dev);
+        CA_CUDA(cudaGetLastError());
+    }
+    if (h->world > 1) return bp_top2(h);
     return CUALIGN_OK;
 }
 
@@ -856,6 +868,7 @@ cualign_status bp_front_edge(cualign_bp *h)
         }
         CA_CUDA(cudaGetLastError());
     }
+    if (h->world == 1) CA_TRY(bp_top2(h)); // the next iteration's othermax inputs
     return CUALIGN_OK;
 }
 

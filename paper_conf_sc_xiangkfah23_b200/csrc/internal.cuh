@@ -299,6 +299,7 @@ cualign_status bp_fsum(cualign_bp *h);                 // t <- sum_f F(S^p) (ini
 cualign_status bp_iterate(cualign_bp *h, int32_t n);   // Alg. 2 l.9-16, n times
 cualign_status bp_iterate_front(cualign_bp *h);        // advance p, top-2, k_edge
 cualign_status bp_iterate_back(cualign_bp *h);         // square pass
+cualign_status bp_top2(cualign_bp *h);                 // per-vertex top-2 of the current y^p, z^p
 cualign_status bp_front_top2(cualign_bp *h);           // advance p, top-2 (partial B when sharded)
 cualign_status bp_front_edge(cualign_bp *h);           // k_edge on the owned edges
 cualign_status bp_merge_top2(cualign_bp *h);           // gathered B partials -> Btop
