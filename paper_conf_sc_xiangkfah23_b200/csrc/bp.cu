@@ -99,7 +99,7 @@ struct Top2Args {
     int64_t nA, nchunks;    // A rows to process (a0 .. a0+nA-1), B chunks
     int64_t a0;
     const int64_t *Arow;
-    const int32_t *chunk_b;
+    const int4 *cdesc;     // per B chunk: (start, end) in the incidence, b, first chunk of b (-1: b has one)
     const int64_t *Bcp, *Bptr;
     const int32_t *Bedge;
     const double *yp, *zp;
@@ -133,10 +133,9 @@ __global__ void __launch_bounds__(256) k_top2(Top2Args T)
         } else {
             // B chunk: gather z^p through the incidence
             const int64_t c = t - T.nA;
-            const int b = T.chunk_b[c];
-            const int64_t c0 = T.Bcp[b], c1 = T.Bcp[b + 1];
-            const int64_t start = T.Bptr[b] + (c - c0) * B_CHUNK;
-            const int64_t end = min(start + (int64_t)B_CHUNK, T.Bptr[b + 1]);
+            const int4 dsc = __ldg(T.cdesc + c); // one load instead of chunk_b -> Bcp, Bptr
+            const int b = dsc.z;
+            const int64_t start = dsc.x, end = dsc.y;
             int eidx[TB_U];
 #pragma unroll
             for (int j = 0; j < TB_U; j++) {
@@ -148,9 +147,10 @@ __global__ void __launch_bounds__(256) k_top2(Top2Args T)
                 if (eidx[j] >= 0) top2_push(m1, m2, T.zp[eidx[j]]);
             tile_top2<TG>(tile, m1, m2);
             if (lane == 0) {
-                if (c1 - c0 == 1) {
+                if (dsc.w < 0) {
                     T.Btop[b] = make_double2(m1, m2);
                 } else {
+                    const int64_t c0 = dsc.w, c1 = T.Bcp[b + 1];
                     // hub column: the last chunk to finish merges all chunks
                     T.Bct[c] = make_double2(m1, m2);
                     __threadfence();
@@ -527,10 +527,16 @@ __global__ void k_chunk_count(int64_t nB, const int64_t *__restrict__ Bptr, int6
         cnt[b] = (Bptr[b + 1] - Bptr[b] + B_CHUNK - 1) / B_CHUNK;
 }
 
-__global__ void k_chunk_fill(int64_t nB, const int64_t *__restrict__ Bcp, int32_t *__restrict__ chunk_b)
+__global__ void k_chunk_fill(int64_t nB, const int64_t *__restrict__ Bcp, const int64_t *__restrict__ Bptr,
+                             int4 *__restrict__ cdesc)
 {
-    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nB; b += (int64_t)gridDim.x * blockDim.x)
-        for (int64_t c = Bcp[b]; c < Bcp[b + 1]; c++) chunk_b[c] = (int32_t)b;
+    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nB; b += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t c0 = Bcp[b], c1 = Bcp[b + 1], e1 = Bptr[b + 1];
+        for (int64_t c = c0; c < c1; c++) {
+            const int64_t st = Bptr[b] + (c - c0) * B_CHUNK;
+            cdesc[c] = make_int4((int)st, (int)min(st + (int64_t)B_CHUNK, e1), (int)b, c1 - c0 > 1 ? (int)c0 : -1);
+        }
+    }
 }
 
 // Grid-stride kernels run as exactly one wave: (resident CTAs per SM) x SMs,
@@ -793,9 +799,10 @@ cualign_status bp_setup(cualign_bp *h)
         CA_CUDA(cudaMemcpyAsync(&h->nchunks, h->Bcp + nB, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
         CA_CUDA(cudaStreamSynchronize(h->stream));
     }
-    CA_TRY(dalloc(h, &h->chunk_b, (size_t)h->nchunks + 1));
+    CA_TRY(dalloc(h, &h->cdesc, (size_t)h->nchunks + 1));
     CA_TRY(dalloc(h, &h->Bct, (size_t)h->nchunks + 1));
-    if (nB > 0) k_chunk_fill<<<grid_for(nB, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB, h->Bcp, h->chunk_b);
+    if (nB > 0)
+        k_chunk_fill<<<grid_for(nB, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB, h->Bcp, Bptr, h->cdesc);
     CA_CUDA(cudaGetLastError());
     return CUALIGN_OK;
 }
@@ -816,7 +823,7 @@ cualign_status bp_top2(cualign_bp *h)
     if (h->L.m > 0) {
         KScope ks(h, CUALIGN_K_TOP2);
         const bool sh = h->world > 1;
-        Top2Args T{(int64_t)(h->a1 - h->a0), h->nchunks, (int64_t)h->a0, h->L.Arow, h->chunk_b, h->Bcp,
+        Top2Args T{(int64_t)(h->a1 - h->a0), h->nchunks, (int64_t)h->a0, h->L.Arow, h->cdesc, h->Bcp,
                    sh ? h->Bptr_loc : h->L.Bptr, sh ? h->Bedge_loc : h->L.Bedge, h->yp, h->zp, h->Atop,
                    sh ? h->Btop_part : h->Btop, h->Bct, h->Bcnt};
         if (T.nA + T.nchunks > 0)

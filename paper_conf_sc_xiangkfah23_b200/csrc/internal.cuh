@@ -126,7 +126,7 @@ struct cualign_bp {
     double *Ffull = nullptr;            // exact mode: F in CSR order
     int64_t nchunks = 0;                // B incidence chunks (k_top2B load balance)
     int64_t *Bcp = nullptr;             // nB+1: chunks of B vertex b are Bcp[b]..Bcp[b+1]-1
-    int32_t *chunk_b = nullptr;         // nchunks: owning B vertex
+    int4 *cdesc = nullptr;              // nchunks: (start, end, owning B vertex, first chunk of a hub or -1)
     double2 *Bct = nullptr;             // nchunks: (max1, max2) of z^p over the chunk
     unsigned int *Bcnt = nullptr;       // nB: chunks finished (hub columns' last-arriver merge)
     double2 *Atop = nullptr, *Btop = nullptr; // per-vertex (max1, max2) of y^p / z^p
