@@ -128,7 +128,7 @@ k_sbuild(int64_t e_begin, int64_t e_end, const int32_t *__restrict__ La, const i
          const int32_t *__restrict__ Aj, const int64_t *__restrict__ Bp,
          const int32_t *__restrict__ Bj, int64_t *__restrict__ cnt, int64_t *__restrict__ ucnt,
          const int64_t *__restrict__ Srp, const int64_t *__restrict__ sq_rp,
-         int32_t *__restrict__ Scol, int2 *__restrict__ sq_ef)
+         int32_t *__restrict__ Scol, int2 *__restrict__ sq_ef, const uint8_t *__restrict__ only = nullptr)
 {
     const int lane = threadIdx.x & 31;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -136,6 +136,7 @@ k_sbuild(int64_t e_begin, int64_t e_end, const int32_t *__restrict__ La, const i
     const unsigned lt_mask = (1u << lane) - 1u;
     for (int64_t e = e_begin + warp; e < e_end; e += nwarps) {
         const int32_t i = La[e], ip = Lb[e];
+        if (only && !only[i]) continue; // rows the group-map build leaves to this kernel
         const int64_t bs = Bp[ip], be = Bp[ip + 1];
         int64_t a_lo = Ap[i];
         const int64_t a_hi = Ap[i + 1];
@@ -241,6 +242,10 @@ k_sbuild(int64_t e_begin, int64_t e_end, const int32_t *__restrict__ La, const i
 constexpr int SBG_WARPS = 8;
 constexpr int SBG_SLOTS = 512;   // hash slots per warp (key j', value lane mask)
 constexpr int SBG_CAP = 256;     // inserts per group (load factor <= 1/2)
+// candidates x row length above which a vertex's rows go to k_sbuild (warp
+// per e): a bound on the lookups this one warp would make (one per candidate
+// and group, at most one group per edge of the row)
+constexpr int64_t SBG_HEAVY = (int64_t)1 << 22;
 
 // 32 x 32 bit-matrix transpose across a warp: lane L holds row L (bit t =
 // M[L][t]); afterwards lane t holds column t (bit L = M[L][t]).  Five
@@ -287,7 +292,7 @@ __global__ void __launch_bounds__(SBG_WARPS * 32)
 k_sbuild_g(int32_t nA, const int64_t *__restrict__ Arow, const int32_t *__restrict__ Lb,
            const int64_t *__restrict__ Ap, const int32_t *__restrict__ Aj, const int64_t *__restrict__ Bp,
            const int32_t *__restrict__ Bj, int64_t *__restrict__ ucnt, const int64_t *__restrict__ sq_rp,
-           int2 *__restrict__ sq_ef, unsigned long long *__restrict__ next_i)
+           int2 *__restrict__ sq_ef, unsigned long long *__restrict__ next_i, uint8_t *__restrict__ heavy)
 {
     __shared__ __align__(16) int32_t hkey_all[SBG_WARPS][SBG_SLOTS];
     __shared__ __align__(16) uint32_t hmask_all[SBG_WARPS][SBG_SLOTS];
@@ -317,6 +322,29 @@ k_sbuild_g(int32_t nA, const int64_t *__restrict__ Arow, const int32_t *__restri
             a_lo = lo;
         }
         if (a_lo == a_hi) continue; // no candidates: ucnt stays 0
+        // heavy vertex (hub of A in R-MAT graphs): its candidates would be
+        // walked once per group by this one warp; leave its rows to the
+        // warp-per-e kernel
+        // (one warp per L edge of the row).  The count pass decides, the
+        // fill pass follows the flag.
+        if (FILL) {
+            if (heavy[i]) continue;
+        } else {
+            int64_t tot = 0;
+            for (int64_t x = a_lo + lane; x < a_hi; x += 32) {
+                const int32_t j = Aj[x];
+                tot += Arow[j + 1] - Arow[j];
+            }
+#pragma unroll
+            for (int off = 16; off >= 1; off >>= 1) tot += __shfl_xor_sync(FULL_MASK, tot, off);
+            if (tot * ni > SBG_HEAVY) {
+                if (lane == 0) {
+                    heavy[i] = 1;
+                    heavy[nA] = 1; // any heavy vertex: the warp-per-e passes run
+                }
+                continue;
+            }
+        }
         for (int t0 = 0; t0 < ni;) {
             // ---- next group: t0 .. t0+ng-1 with sum of B degrees <= SBG_CAP
             const int t = t0 + lane;
@@ -729,7 +757,7 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
     const bool group_map = sb_env == 1 && h->L.nB < (1 << 26);
     const int32_t nA = h->L.nA;
     int sbg_blocks = 1;
-    TmpBuf qctr;
+    TmpBuf qctr, heavy;
     if (group_map) {
         // one resident wave; the warps pull A vertices from a queue
         int occ = 0;
@@ -740,13 +768,25 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
         sbg_blocks = grid_for((int64_t)nA * 32, SBG_WARPS * 32, (int64_t)occ * h->num_sms);
         CA_CUDA(tmalloc(h, qctr, 2 * sizeof(unsigned long long)));
         CA_CUDA(cudaMemsetAsync(qctr.p, 0, 2 * sizeof(unsigned long long), h->stream));
+        CA_CUDA(tmalloc(h, heavy, (size_t)nA + 1));
+        CA_CUDA(cudaMemsetAsync(heavy.p, 0, (size_t)nA + 1, h->stream));
     }
+    const int old_blocks = grid_for(m * 32, 256, h->num_sms * 16);
+    uint8_t any_heavy = 0;
     if (m) {
         if (group_map) {
             CA_CUDA(cudaMemsetAsync(ucnt.p, 0, sizeof(int64_t) * (size_t)m, h->stream));
             k_sbuild_g<false><<<sbg_blocks, SBG_WARPS * 32, 0, h->stream>>>(nA, h->L.Arow, h->L.Lb, Ap, Aj, Bp, Bj,
                                                                           (int64_t *)ucnt.p, nullptr, nullptr,
-                                                                          (unsigned long long *)qctr.p);
+                                                                          (unsigned long long *)qctr.p,
+                                                                          (uint8_t *)heavy.p);
+            CA_CUDA(cudaMemcpyAsync(&any_heavy, (uint8_t *)heavy.p + nA, 1, cudaMemcpyDeviceToHost, h->stream));
+            CA_CUDA(cudaStreamSynchronize(h->stream));
+            if (any_heavy)
+                k_sbuild<false, true><<<old_blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj,
+                                                                         Bp, Bj, nullptr, (int64_t *)ucnt.p, nullptr,
+                                                                         nullptr, nullptr, nullptr,
+                                                                         (const uint8_t *)heavy.p);
         } else {
             const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
             k_sbuild<false, true><<<blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,
@@ -773,7 +813,12 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
         if (group_map) {
             k_sbuild_g<true><<<sbg_blocks, SBG_WARPS * 32, 0, h->stream>>>(nA, h->L.Arow, h->L.Lb, Ap, Aj, Bp, Bj,
                                                                          nullptr, h->sq_rp, h->sq_ef,
-                                                                         (unsigned long long *)qctr.p + 1);
+                                                                         (unsigned long long *)qctr.p + 1,
+                                                                         (uint8_t *)heavy.p);
+            if (any_heavy)
+                k_sbuild<true, true><<<old_blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp,
+                                                                        Bj, nullptr, nullptr, nullptr, h->sq_rp,
+                                                                        nullptr, h->sq_ef, (const uint8_t *)heavy.p);
         } else {
             const int blocks = grid_for(m * 32, 256, h->num_sms * 16);
             k_sbuild<true, true><<<blocks, 256, 0, h->stream>>>(0, m, h->L.La, h->L.Lb, h->L.Arow, Ap, Aj, Bp, Bj,

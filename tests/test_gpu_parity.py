@@ -128,6 +128,25 @@ def test_S_long_candidate_rows(ca):
         assert o.s > 1000
 
 
+def test_S_heavy_vertex(ca):
+    """An A hub whose candidate list (sum of its neighbours' L rows) exceeds
+    the group-map build's limit: its rows go to the warp-per-e build, the
+    other rows to the group map, all in one S (complete L: S = A (x) B)."""
+    rng = np.random.default_rng(5)
+    n_a, n_b = 130, 200
+    ea = [(0, j) for j in range(1, n_a)] + [(int(u), int(v)) for u, v in rng.integers(1, n_a, (60, 2)) if u != v]
+    eb = [(0, j) for j in range(1, 40)] + [(int(u), int(v)) for u, v in rng.integers(0, n_b, (500, 2)) if u != v]
+    A = graph_from_edges(n_a, sorted(set((min(u, v), max(u, v)) for u, v in ea)))
+    B = graph_from_edges(n_b, sorted(set((min(u, v), max(u, v)) for u, v in eb)))
+    L = complete_candidates(n_a, n_b, rng.uniform(0.1, 1.0, n_a * n_b))
+    o = Oracle(A, B, L, 1.0, 2.0)
+    with ca.CuAlignBP(A, B, L, 1.0, 2.0, 0.9) as h:
+        rp, col = h.get_S()
+        orp, ocol, _ = o.get_S()
+        assert np.array_equal(rp, orp) and np.array_equal(col, ocol)
+        assert (n_a - 1) * n_b * n_b > 1 << 22  # vertex 0 is heavy: candidates x row length
+
+
 # ------------------------------------------------------- a3-a6: BP iteration
 def _run_both(ca, inst, n_iter, flags=0, gamma=None, alpha=None, beta=None, check=None):
     alpha = inst.alpha if alpha is None else alpha

@@ -1,6 +1,6 @@
 """Init (a1-a2) timing on a config: first and second handle (pool warm),
 with CUALIGN_INIT_TRACE phase lines on stderr.  Usage:
-    python tools/probe_init.py [config] [scale]"""
+    python tools/probe_init.py [config] [scale] [k]"""
 import os
 import sys
 import time
@@ -12,7 +12,8 @@ from synth import make_config  # noqa: E402
 
 cfg = sys.argv[1] if len(sys.argv) > 1 else "O"
 scale = float(sys.argv[2]) if len(sys.argv) > 2 else 1.0
-inst = make_config(cfg, scale=scale)
+k = int(sys.argv[3]) if len(sys.argv) > 3 else None
+inst = make_config(cfg, scale=scale, k=k) if k else make_config(cfg, scale=scale)
 torch.cuda.init()
 for rep in range(3):
     torch.cuda.synchronize()
