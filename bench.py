@@ -325,6 +325,9 @@ def main():
 
     # ------------------------------------------------------------- warmup
     # (each step = iterate(1) + round, replayed from the library's CUDA graph)
+    # The library picks the step schedule (pipelined or not) on its first run
+    # of >= 8 steps by timing both; do that here, untimed, before the warm-up.
+    h.run(8)
     h.run(args.warmup)
     torch.cuda.synchronize()
     h.stats(reset=True)

@@ -391,6 +391,7 @@ static cualign_status launch_slot(cualign_bp *h, int slot)
 // values end in buffer 0 (h->yc, h->zc), as after an unpipelined run.
 static cualign_status run_pipelined(cualign_bp *h, int32_t n, RoundDev *trace = nullptr)
 {
+    if (n <= 0) return CUALIGN_OK;
     CA_TRY(ensure_gh(h, (int64_t)h->p + n + 1));
     if (!h->yc_b1) CA_TRY(alloc_pipeline(h));
     CA_CUDA(cudaEventRecord(h->sync_ev[0], h->stream));
@@ -746,16 +747,46 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
     // next iteration overwrites them), the matching is the cooperative
     // pointer-round kernel (MATCH_ROUNDS: its grid must be co-resident, so it
     // never shares the device), or CUALIGN_PIPELINE=0 (measurement knob)
-    static const bool pipe_env = !getenv("CUALIGN_PIPELINE") || atoi(getenv("CUALIGN_PIPELINE")) != 0;
-    if (what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND) && pipe_env &&
-        !(h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS)))
-        return run_pipelined(h, n_steps, trace);
-    if (!trace) return run_graph(h, n_steps, what);
-    for (int32_t k = 0; k < n_steps; k++) {
-        CA_TRY(run_graph(h, 1, what));
-        CA_CUDA(cudaMemcpyAsync(trace + k, h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->stream));
-    }
-    return CUALIGN_OK;
+    // Whether the pipeline pays depends on the instance: the rounding branch
+    // takes SM slots from the one-wave square pass, whose static partition
+    // then waits for them (measured: O 1246 -> 1300 it/s pipelined, R-MAT
+    // k = 5 1.03 -> 1.62 ms per step).  The first run of >= 8 steps times 3
+    // steps of each schedule (after one capture step each) and keeps the
+    // faster; results are identical either way (tests compare both with the
+    // eager sequence bit for bit).  CUALIGN_PIPELINE=0/1 forces a schedule.
+    static const int pipe_env = getenv("CUALIGN_PIPELINE") ? atoi(getenv("CUALIGN_PIPELINE")) : -1;
+    const bool both = what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND) &&
+                      !(h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS));
+    auto run_plain = [&](int32_t n, RoundDev *tr) -> cualign_status {
+        if (!tr) return run_graph(h, n, what);
+        for (int32_t k = 0; k < n; k++) {
+            CA_TRY(run_graph(h, 1, what));
+            CA_CUDA(cudaMemcpyAsync(tr + k, h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->stream));
+        }
+        return CUALIGN_OK;
+    };
+    if (!both || pipe_env == 0) return run_plain(n_steps, trace);
+    if (pipe_env == 1 || h->pipe_mode == 1) return run_pipelined(h, n_steps, trace);
+    if (h->pipe_mode == 0) return run_plain(n_steps, trace);
+    if (n_steps < 8 || h->timing) return run_pipelined(h, n_steps, trace); // undecided: default
+    cudaEvent_t ev[4];
+    for (auto &e : ev) e = get_event(h);
+    auto tr = [&](int32_t off) { return trace ? trace + off : nullptr; };
+    CA_TRY(run_pipelined(h, 1, tr(0)));
+    CA_CUDA(cudaEventRecord(ev[0], h->stream));
+    CA_TRY(run_pipelined(h, 3, tr(1)));
+    CA_CUDA(cudaEventRecord(ev[1], h->stream));
+    CA_TRY(run_plain(1, tr(4)));
+    CA_CUDA(cudaEventRecord(ev[2], h->stream));
+    CA_TRY(run_plain(3, tr(5)));
+    CA_CUDA(cudaEventRecord(ev[3], h->stream));
+    CA_CUDA(cudaEventSynchronize(ev[3]));
+    float tp = 0.f, tg = 0.f;
+    CA_CUDA(cudaEventElapsedTime(&tp, ev[0], ev[1]));
+    CA_CUDA(cudaEventElapsedTime(&tg, ev[2], ev[3]));
+    for (auto &e : ev) h->event_pool.push_back(e);
+    h->pipe_mode = tp < tg ? 1 : 0;
+    return h->pipe_mode ? run_pipelined(h, n_steps - 8, tr(8)) : run_plain(n_steps - 8, tr(8));
 }
 } // namespace cualign
 
