@@ -325,9 +325,9 @@ def main():
 
     # ------------------------------------------------------------- warmup
     # (each step = iterate(1) + round, replayed from the library's CUDA graph)
-    # The library picks the step schedule (pipelined or not) on its first run
-    # of >= 8 steps by timing both; do that here, untimed, before the warm-up.
-    h.run(8)
+    # The library picks the step schedule on its first run of >= 21 steps by
+    # timing each; do that here, untimed, before the warm-up.
+    h.run(21)
     h.run(args.warmup)
     torch.cuda.synchronize()
     h.stats(reset=True)
@@ -350,6 +350,8 @@ def main():
     elapsed_ms = max_over_ranks(elapsed_ms, world, device=f"cuda:{dev}")
     st = h.stats(reset=True)
     _, info = h.get_best()
+    step_schedule = {-1: "undecided", 0: "rounding forked beside the square pass", 1: "pipelined",
+                     2: "serial"}.get(h.sizes()["schedule"], "?")
 
     # ----------------------------------------------- per-kernel timing pass
     # event-record nodes inside the captured step graph, read after each replay
@@ -542,6 +544,7 @@ def main():
         "last_round": {k: info[k] for k in ("iter", "card_y", "card_z", "overlap_y", "overlap_z",
                                             "rounds_y", "rounds_z", "score")},
         "match_schedule": "rounds" if args.match_rounds else "suitor",
+        "step_schedule": step_schedule,
         "next2_knn": knn,
     }
     print(json.dumps(line), flush=True)

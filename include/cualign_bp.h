@@ -148,7 +148,8 @@ typedef struct {
     int64_t edge_begin, edge_end; /* owned canonical edge ids [begin, end) */
     int64_t squares_local;    /* squares stored by this shard */
     int32_t merge_rounds;     /* sharded rounding (NEXT-1): merge rounds of the last round() (0 if unsharded) */
-    int32_t reserved;
+    int32_t schedule;         /* step schedule run() selected: -1 not yet, 0 rounding forked beside the
+                                 square pass, 1 pipelined (rounding of k beside iteration k+1), 2 serial */
 } cualign_sizes;
 
 /* Diagnostics: per-kernel-class event timing (needs CUALIGN_FLAG_TIMING) and

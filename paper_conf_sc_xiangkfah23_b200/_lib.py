@@ -78,7 +78,7 @@ class Sizes_t(ctypes.Structure):
                 ("p", ctypes.c_int32), ("fixed_point_bits", ctypes.c_int32),
                 ("device_bytes", ctypes.c_int64), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("edge_begin", ctypes.c_int64), ("edge_end", ctypes.c_int64),
-                ("squares_local", ctypes.c_int64), ("merge_rounds", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("squares_local", ctypes.c_int64), ("merge_rounds", ctypes.c_int32), ("schedule", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

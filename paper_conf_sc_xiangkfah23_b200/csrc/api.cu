@@ -747,13 +747,17 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
     // next iteration overwrites them), the matching is the cooperative
     // pointer-round kernel (MATCH_ROUNDS: its grid must be co-resident, so it
     // never shares the device), or CUALIGN_PIPELINE=0 (measurement knob)
-    // Whether the pipeline pays depends on the instance: the rounding branch
-    // takes SM slots from the one-wave square pass, whose static partition
-    // then waits for them (measured: O 1246 -> 1300 it/s pipelined, R-MAT
-    // k = 5 1.03 -> 1.62 ms per step).  The first run of >= 8 steps times 3
-    // steps of each schedule (after one capture step each) and keeps the
-    // faster; results are identical either way (tests compare both with the
-    // eager sequence bit for bit).  CUALIGN_PIPELINE=0/1 forces a schedule.
+    // Which step schedule is fastest depends on the instance: the rounding
+    // branch takes SM slots from the one-wave square pass, whose static
+    // partition then waits for them.  Schedules: 0 = one graph per step with
+    // the rounding forked beside the square pass, 1 = pipelined (rounding of
+    // k beside iteration k+1), 2 = serial (iterate graph, then round graph).
+    // Measured: O 1246 / 1300 / ~1300 it/s; R-MAT k = 5 1.03 / 1.62 / ~1.03
+    // ms per step; R k = 50 8.3 ms with a fork vs 7.7 serial.  The first run
+    // of >= 21 steps times 4 steps of each (after a capture and 2 warm steps)
+    // and keeps the fastest; results are identical whichever runs (tests compare
+    // them with the eager sequence bit for bit).  CUALIGN_PIPELINE=0/1/2
+    // forces one.
     static const int pipe_env = getenv("CUALIGN_PIPELINE") ? atoi(getenv("CUALIGN_PIPELINE")) : -1;
     const bool both = what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND) &&
                       !(h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS));
@@ -765,28 +769,43 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
         }
         return CUALIGN_OK;
     };
-    if (!both || pipe_env == 0) return run_plain(n_steps, trace);
-    if (pipe_env == 1 || h->pipe_mode == 1) return run_pipelined(h, n_steps, trace);
-    if (h->pipe_mode == 0) return run_plain(n_steps, trace);
-    if (n_steps < 8 || h->timing) return run_pipelined(h, n_steps, trace); // undecided: default
-    cudaEvent_t ev[4];
-    for (auto &e : ev) e = get_event(h);
+    auto run_serial = [&](int32_t n, RoundDev *tr) -> cualign_status {
+        for (int32_t k = 0; k < n; k++) {
+            CA_TRY(run_graph(h, 1, CUALIGN_RUN_ITERATE));
+            CA_TRY(run_graph(h, 1, CUALIGN_RUN_ROUND));
+            if (tr) CA_CUDA(cudaMemcpyAsync(tr + k, h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->stream));
+        }
+        return CUALIGN_OK;
+    };
+    auto run_mode = [&](int mode, int32_t n, RoundDev *tr) -> cualign_status {
+        if (mode == 1) return run_pipelined(h, n, tr);
+        if (mode == 2) return run_serial(n, tr);
+        return run_plain(n, tr);
+    };
+    if (!both) return run_plain(n_steps, trace);
+    if (pipe_env >= 0 && pipe_env <= 2) return run_mode(pipe_env, n_steps, trace);
+    if (h->pipe_mode >= 0) return run_mode(h->pipe_mode, n_steps, trace);
+    constexpr int32_t PRE = 3, TIMED = 4, PER = PRE + TIMED; // per schedule: capture + warm, timed
+    if (n_steps < 3 * PER || h->timing) return run_pipelined(h, n_steps, trace); // undecided: default
     auto tr = [&](int32_t off) { return trace ? trace + off : nullptr; };
-    CA_TRY(run_pipelined(h, 1, tr(0)));
-    CA_CUDA(cudaEventRecord(ev[0], h->stream));
-    CA_TRY(run_pipelined(h, 3, tr(1)));
-    CA_CUDA(cudaEventRecord(ev[1], h->stream));
-    CA_TRY(run_plain(1, tr(4)));
-    CA_CUDA(cudaEventRecord(ev[2], h->stream));
-    CA_TRY(run_plain(3, tr(5)));
-    CA_CUDA(cudaEventRecord(ev[3], h->stream));
-    CA_CUDA(cudaEventSynchronize(ev[3]));
-    float tp = 0.f, tg = 0.f;
-    CA_CUDA(cudaEventElapsedTime(&tp, ev[0], ev[1]));
-    CA_CUDA(cudaEventElapsedTime(&tg, ev[2], ev[3]));
-    for (auto &e : ev) h->event_pool.push_back(e);
-    h->pipe_mode = tp < tg ? 1 : 0;
-    return h->pipe_mode ? run_pipelined(h, n_steps - 8, tr(8)) : run_plain(n_steps - 8, tr(8));
+    float t[3] = {0.f, 0.f, 0.f};
+    for (int mode = 0; mode < 3; mode++) {
+        cudaEvent_t e0 = get_event(h), e1 = get_event(h);
+        CA_TRY(run_mode(mode, PRE, tr(PER * mode)));
+        CA_CUDA(cudaEventRecord(e0, h->stream));
+        CA_TRY(run_mode(mode, TIMED, tr(PER * mode + PRE)));
+        CA_CUDA(cudaEventRecord(e1, h->stream));
+        CA_CUDA(cudaEventSynchronize(e1));
+        CA_CUDA(cudaEventElapsedTime(&t[mode], e0, e1));
+        h->event_pool.push_back(e0);
+        h->event_pool.push_back(e1);
+    }
+    // the pipelined schedule unless another is clearly (> 2 %) faster
+    int best = 1;
+    for (int mode : {0, 2})
+        if (t[mode] < 0.98f * t[best]) best = mode;
+    h->pipe_mode = best;
+    return run_mode(h->pipe_mode, n_steps - 3 * PER, tr(3 * PER));
 }
 } // namespace cualign
 
@@ -864,6 +883,7 @@ cualign_status cualign_bp_get_sizes(cualign_bp *h, cualign_sizes *sz)
     sz->edge_end = h->vshards.empty() ? h->e1 : q->L.m;
     sz->squares_local = h->vshards.empty() ? h->nsq : q->nsq_total;
     sz->merge_rounds = q->dist_rounds;
+    sz->schedule = h->pipe_mode;
     return CUALIGN_OK;
 }
 

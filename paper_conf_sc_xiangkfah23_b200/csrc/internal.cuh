@@ -158,7 +158,7 @@ struct cualign_bp {
     // iteration's outside a pipelined run), the iteration the rounding
     // kernels report (round_p; = p_dev except in a pipelined run)
     double *yc_b1 = nullptr, *zc_b1 = nullptr;
-    int pipe_mode = -1;                 // step schedule: -1 undecided, 0 plain graph, 1 pipelined
+    int pipe_mode = -1;                 // step schedule: -1 undecided, 0 forked graph, 1 pipelined, 2 serial
     int *rp_dev = nullptr;
     const int *round_p = nullptr;
 

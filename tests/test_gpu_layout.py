@@ -81,7 +81,7 @@ def _eager(ca, inst, n):
     return h, infos
 
 
-@pytest.mark.parametrize("n", [1, 2, 5, 6, 8, 13])  # >= 8: the first run times both schedules
+@pytest.mark.parametrize("n", [1, 2, 5, 6, 21, 24])  # >= 21: the first run times the schedules
 def test_pipelined_run_equals_eager(ca, n):
     inst = make_config("P", scale=0.1)
     h1, infos = _eager(ca, inst, n)
@@ -124,7 +124,7 @@ def test_run_trace_infos_equal_step_by_step(ca, mode):
     inst = make_config("P", scale=0.05)
     flags = ca.FLAG_ROUND_DAMPED if mode == "damped" else 0
     kw = {"world": 3} if mode == "shards3" else {}
-    n = 11  # >= 8: includes the schedule selection steps
+    n = 23  # >= 21: includes the schedule selection steps
     with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags) as h1, \
             ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags, **kw) as h2:
         eager = []

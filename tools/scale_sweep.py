@@ -88,7 +88,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--points", default="S,R5,R10,R20,R35,R50")
     ap.add_argument("--n", type=int, default=20)
-    ap.add_argument("--warm", type=int, default=10)  # >= 8: the schedule selection runs here
+    ap.add_argument("--warm", type=int, default=21)  # >= 21: the schedule selection runs here
     ap.add_argument("--out", default="gpurun_out/scale_sweep.jsonl")
     args = ap.parse_args()
     import torch
