@@ -473,6 +473,7 @@ def main():
         e2e = {"value": args.e2e_iters * work_units / align_time_s, "unit": UNIT,
                "h2d_bytes_per_step": h2d / args.e2e_iters, "d2h_bytes_per_step": d2h / args.e2e_iters,
                "align_time_s": align_time_s, "teardown_s": teardown_s, "iters": args.e2e_iters,
+               "phases_s": binfo.get("phases_s"),
                "best_score": binfo["best_score"], "best_iter": binfo["best_iter"]}
         if rank == 0:
             # NEXT-4: quality of the best alignment against the generator's ground truth

@@ -179,6 +179,7 @@ __global__ void k_copy_int(int *dst, const int *src) { *dst = *src; }
 __global__ void k_incr_int(int *x) { *x += 1; }
 
 static inline int pslot(int kind, int wb) { return 4 + 2 * kind + wb; }
+static constexpr int SERIAL_SLOT = 10; // one step as ONE graph: iterate(1), then the rounding (no fork)
 
 // The pipelined graphs' work (see capture_step): the y^c / z^c buffers are
 // selected by pointing h->yc / h->zc at them while the kernels are captured.
@@ -256,7 +257,10 @@ static cualign_status capture_step(cualign_bp *h, int timed, int slot)
     cualign_status st = CUALIGN_OK;
     cudaError_t e = cudaStreamBeginCapture(h->gstream, cudaStreamCaptureModeThreadLocal);
     if (e == cudaSuccess) {
-        if (slot >= 4) {
+        if (slot == SERIAL_SLOT) {
+            st = bp_iterate(h, 1);
+            if (st == CUALIGN_OK) st = match_round(h);
+        } else if (slot >= 4) {
             st = capture_pipelined(h, (slot - 4) / 2, (slot - 4) % 2);
         } else if (what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND)) {
             // the rounding of iteration p reads only y^c, z^c (or y^p, z^p),
@@ -770,11 +774,18 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
         return CUALIGN_OK;
     };
     auto run_serial = [&](int32_t n, RoundDev *tr) -> cualign_status {
+        if (n <= 0) return CUALIGN_OK;
+        CA_TRY(ensure_gh(h, (int64_t)h->p + n + 1));
+        CA_CUDA(cudaEventRecord(h->sync_ev[0], h->stream));
+        CA_CUDA(cudaStreamWaitEvent(h->gstream, h->sync_ev[0], 0));
         for (int32_t k = 0; k < n; k++) {
-            CA_TRY(run_graph(h, 1, CUALIGN_RUN_ITERATE));
-            CA_TRY(run_graph(h, 1, CUALIGN_RUN_ROUND));
-            if (tr) CA_CUDA(cudaMemcpyAsync(tr + k, h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->stream));
+            CA_TRY(launch_slot(h, SERIAL_SLOT));
+            h->p += 1;
+            if (tr) CA_CUDA(cudaMemcpyAsync(tr + k, h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->gstream));
         }
+        h->have_info = true;
+        CA_CUDA(cudaEventRecord(h->sync_ev[1], h->gstream));
+        CA_CUDA(cudaStreamWaitEvent(h->stream, h->sync_ev[1], 0));
         return CUALIGN_OK;
     };
     auto run_mode = [&](int mode, int32_t n, RoundDev *tr) -> cualign_status {
@@ -783,7 +794,10 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
         return run_plain(n, tr);
     };
     if (!both) return run_plain(n_steps, trace);
-    if (pipe_env >= 0 && pipe_env <= 2) return run_mode(pipe_env, n_steps, trace);
+    if (pipe_env >= 0 && pipe_env <= 2) {
+        h->pipe_mode = pipe_env; // forced (reported as chosen)
+        return run_mode(pipe_env, n_steps, trace);
+    }
     if (h->pipe_mode >= 0) return run_mode(h->pipe_mode, n_steps, trace);
     constexpr int32_t PRE = 3, TIMED = 4, PER = PRE + TIMED; // per schedule: capture + warm, timed
     if (n_steps < 3 * PER || h->timing) return run_pipelined(h, n_steps, trace); // undecided: default

@@ -149,7 +149,7 @@ struct cualign_bp {
     // the pipelined step graphs: kind 0 = iterate
     // into buffer wb, 1 = rounding of buffer 1-wb beside iterate into wb,
     // 2 = rounding of buffer wb
-    static constexpr int NSLOT = 10;
+    static constexpr int NSLOT = 11;  // + SERIAL_SLOT: iterate(1) then round, no fork
     cudaGraphExec_t graph[2][NSLOT] = {};                   // [timed][slot]
     int64_t graph_launches[2][NSLOT] = {};                  // kernels per replay
     int64_t graph_class_launches[2][NSLOT][CUALIGN_NUM_KERNEL_CLASSES] = {};
