@@ -164,6 +164,7 @@ struct cualign_bp {
 
     // matching (two instances: y and z)
     int32_t *candA = nullptr, *candB = nullptr, *mateA = nullptr, *mateB = nullptr;
+    int32_t *mvA = nullptr; // 2 instances x n_A: M(i) as a B vertex (-1: unmatched), for evaluate
     unsigned long long *suit = nullptr; // Suitor slots, 2 instances x max(nA, nB)
     // sharded rounding (NEXT-1): replicated global suitors per (instance, B vertex)
     unsigned long long *dist_gx = nullptr, *dist_wxl = nullptr, *dist_wxg = nullptr, *dist_cnt = nullptr;

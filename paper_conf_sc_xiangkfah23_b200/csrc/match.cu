@@ -493,6 +493,7 @@ struct EvalParams {
     const int32_t *Lb;
     const double *w;
     const int32_t *mateA; // 2 instances, final
+    const int32_t *mvA;   // 2 instances: M(i) as a B vertex (-1: unmatched), k_mate_vertex
     const unsigned long long *Bhash; // E_B membership set
     int Bhash_log;
     const int2 *pairs;    // undirected A edges (i < j)
@@ -600,29 +601,21 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, con
             const int64_t q = base + u * nthr;
             ij[u] = q < P.npairs ? __ldg(P.pairs + q) : make_int2(-1, -1);
         }
+        // M(i), M(j) as B vertices (-1: unmatched), one gather each
 #pragma unroll
         for (int u = 0; u < EVAL_U; u++) {
 #pragma unroll
             for (int k = 0; k < 2; k++) {
-                em[u][2 * k] = ij[u].x >= 0 ? P.mateA[k * P.nA + ij[u].x] : -1;
-                em[u][2 * k + 1] = ij[u].x >= 0 ? P.mateA[k * P.nA + ij[u].y] : -1;
-            }
-        }
-#pragma unroll
-        for (int u = 0; u < EVAL_U; u++) {
-#pragma unroll
-            for (int k = 0; k < 2; k++) {
-                const bool both = em[u][2 * k] >= 0 && em[u][2 * k + 1] >= 0;
-                // M(i), M(j) in V_B (-1: not both matched)
-                em[u][2 * k] = both ? __ldg(P.Lb + em[u][2 * k]) : -1;
-                em[u][2 * k + 1] = both ? __ldg(P.Lb + em[u][2 * k + 1]) : -1;
+                em[u][2 * k] = ij[u].x >= 0 ? P.mvA[k * P.nA + ij[u].x] : -1;
+                em[u][2 * k + 1] = ij[u].x >= 0 ? P.mvA[k * P.nA + ij[u].y] : -1;
             }
         }
 #pragma unroll
         for (int u = 0; u < EVAL_U; u++) {
 #pragma unroll
             for (int k = 0; k < 2; k++)
-                if (em[u][2 * k] >= 0 && bhash_has(P.Bhash, P.Bhash_log, bhash_key(em[u][2 * k], em[u][2 * k + 1])))
+                if (em[u][2 * k] >= 0 && em[u][2 * k + 1] >= 0 &&
+                    bhash_has(P.Bhash, P.Bhash_log, bhash_key(em[u][2 * k], em[u][2 * k + 1])))
                     ov[k]++;
         }
     }
@@ -643,6 +636,19 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, con
     __threadfence();
     round_final_block(P, gridDim.x, exact, alpha, beta, p_dev, work, sd);
     if (threadIdx.x == 0) P.rd->done = 0u;
+}
+
+// M(i) as a B vertex for both instances (evaluate reads it per A edge
+// instead of mate -> L_b twice), and the round's overlap / cardinality
+// accumulators zeroed (this kernel precedes k_eval)
+__global__ void k_mate_vertex(int64_t n2, const int32_t *__restrict__ mateA, const int32_t *__restrict__ Lb,
+                              int32_t *__restrict__ mvA, RoundDev *rd)
+{
+    if (blockIdx.x == 0 && threadIdx.x < 4) (&rd->overlap[0])[threadIdx.x] = 0ull; // overlap[2], card[2]
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n2; i += (int64_t)gridDim.x * blockDim.x) {
+        const int e = mateA[i];
+        mvA[i] = e >= 0 ? __ldg(Lb + e) : -1;
+    }
 }
 
 __global__ void k_copy_best(int64_t nA, const int32_t *__restrict__ mateA, const RoundDev *__restrict__ rd,
@@ -799,6 +805,7 @@ cualign_status match_setup(cualign_bp *h)
     CA_TRY(dalloc(h, &h->candB, 2 * nB + 1));
     CA_TRY(dalloc(h, &h->suit, 2 * (nA > nB ? nA : nB) + 1));
     CA_TRY(dalloc(h, &h->mateA, 2 * nA + 1));
+    CA_TRY(dalloc(h, &h->mvA, 2 * nA + 1));
     CA_TRY(dalloc(h, &h->mateB, 2 * nB + 1));
     CA_TRY(dalloc(h, &h->best_mate, nA + 1));
     CA_TRY(dalloc(h, &h->rd, 1));
@@ -968,14 +975,21 @@ cualign_status match_evaluate(cualign_bp *h)
     E.Lb = h->L.Lb;
     E.w = h->L.w;
     E.mateA = h->mateA;
+    E.mvA = h->mvA;
     E.Bhash = h->Bhash;
     E.Bhash_log = h->Bhash_log;
     E.pairs = h->Apairs;
     E.npairs = h->nApairs;
     E.partial_w = h->partial_w;
     E.rd = h->rd;
-    // overlap / card accumulators (the rest of rd persists: best)
-    CA_CUDA(cudaMemsetAsync(&h->rd->overlap[0], 0, 4 * sizeof(unsigned long long), h->stream));
+    {
+        // M(i) as B vertices + zeroed overlap / card accumulators (the rest of rd persists: best)
+        KScope ks(h, CUALIGN_K_MATCHAUX);
+        const int64_t n2 = 2 * (int64_t)h->L.nA;
+        k_mate_vertex<<<grid_for(n2 > 0 ? n2 : 1, 256, h->num_sms * 4), 256, 0, h->stream>>>(n2, h->mateA, h->L.Lb,
+                                                                                            h->mvA, h->rd);
+        CA_CUDA(cudaGetLastError());
+    }
     {
         KScope ks(h, CUALIGN_K_EVAL);
         k_eval<<<h->eval_grid, 256, 0, h->stream>>>(E, (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha, h->beta,
