@@ -109,6 +109,7 @@ struct Top2Args {
 
 __global__ void __launch_bounds__(256) k_top2(Top2Args T)
 {
+    pdl_wait();
     auto tile = cg::tiled_partition<TG>(cg::this_thread_block());
     const int lane = tile.thread_rank();
     const int64_t t0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / TG;
@@ -187,6 +188,7 @@ struct EdgeArgs {
 template <int EPT, bool EXACT, bool LITERAL, int MINB = 1>
 __global__ void __launch_bounds__(256, MINB) k_edge(EdgeArgs R)
 {
+    pdl_wait();
     const int64_t base = R.e0 + (int64_t)blockIdx.x * blockDim.x * EPT + threadIdx.x;
     const double2 ghp = R.gh[*R.p_dev];
     const double g = ghp.x, hh = ghp.y;
@@ -406,6 +408,7 @@ k_square_tma(int64_t nsq, const int2 *__restrict__ sq_ef, V *__restrict__ sq_val
         fence_mbar_init();
     }
     __syncthreads();
+    pdl_wait(); // the barrier setup above overlaps the predecessor's tail
     if (warp == SQT_CWARPS) {
         // producer: one lane issues the bulk copies of this CTA's chunks
         if (lane == 0) {
@@ -549,7 +552,11 @@ int one_wave_grid(cualign_bp *h, const void *fn, int block, int64_t items, int64
     return grid_for((items + items_per_block - 1) / items_per_block, 1, occ * h->num_sms);
 }
 
-__global__ void k_advance(int *p_dev) { *p_dev += 1; }
+__global__ void k_advance(int *p_dev)
+{
+    pdl_wait();
+    *p_dev += 1;
+}
 
 template <bool UPDATE, bool EXACT, int SQ_U, bool HINTS, bool NOATOM, class V>
 void square_launch_v(cualign_bp *h, V *vals)
@@ -586,8 +593,8 @@ void square_tma_launch_v(cualign_bp *h, V *vals)
     (void)cudaGetLastError();
     const int64_t nchunks = (h->nsq + SQT_CHUNK - 1) / SQT_CHUNK;
     const int grid = grid_for(nchunks, 1, (int64_t)occ * h->num_sms);
-    fn<<<grid, block, smem, h->stream>>>(h->nsq, h->sq_ef, vals, h->u, h->beta, h->gh_dev, h->p_dev, h->fp_scale,
-                                         h->tacc);
+    (void)launch_pdl(fn, dim3(grid), dim3(block), smem, h->stream, h->nsq, h->sq_ef, vals, (const double *)h->u,
+                     h->beta, (const double2 *)h->gh_dev, (const int *)h->p_dev, h->fp_scale, h->tacc);
 }
 
 void square_tma_launch(cualign_bp *h)
@@ -827,7 +834,8 @@ cualign_status bp_top2(cualign_bp *h)
                    sh ? h->Bptr_loc : h->L.Bptr, sh ? h->Bedge_loc : h->L.Bedge, h->yp, h->zp, h->Atop,
                    sh ? h->Btop_part : h->Btop, h->Bct, h->Bcnt};
         if (T.nA + T.nchunks > 0)
-            k_top2<<<grid_for((T.nA + T.nchunks) * TG, 256, 1 << 30), 256, 0, h->stream>>>(T);
+            CA_CUDA(launch_pdl(k_top2, dim3(grid_for((T.nA + T.nchunks) * TG, 256, 1 << 30)), dim3(256), 0,
+                               h->stream, T));
         CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;
@@ -842,8 +850,7 @@ cualign_status bp_front_top2(cualign_bp *h)
 {
     {
         KScope ks(h, CUALIGN_K_OTHER);
-        k_advance<<<1, 1, 0, h->stream>>>(h->p_dev);
-        CA_CUDA(cudaGetLastError());
+        CA_CUDA(launch_pdl(k_advance, dim3(1), dim3(1), 0, h->stream, h->p_dev));
     }
     if (h->world > 1) return bp_top2(h);
     return CUALIGN_OK;
@@ -871,7 +878,7 @@ cualign_status bp_front_edge(cualign_bp *h)
             static const int var = getenv("CUALIGN_EDGE_VAR") ? atoi(getenv("CUALIGN_EDGE_VAR")) : 0;
             if (var == 1) k_edge<1, false, false><<<grid_for(ml, 256, 1 << 30), 256, 0, h->stream>>>(R);
             else if (var == 4) k_edge<4, false, false><<<grid_for((ml + 3) / 4, 256, 1 << 30), 256, 0, h->stream>>>(R);
-            else k_edge<EPT, false, false><<<grid, 256, 0, h->stream>>>(R);
+            else CA_CUDA(launch_pdl(k_edge<EPT, false, false>, dim3(grid), dim3(256), 0, h->stream, R));
         }
         CA_CUDA(cudaGetLastError());
     }

@@ -11,6 +11,8 @@
 
 #include "../../include/cualign_bp.h"
 
+#include <utility>
+
 namespace cualign {
 
 // ------------------------------------------------------------------ errors
@@ -201,6 +203,30 @@ struct cualign_bp {
 };
 
 namespace cualign {
+
+// ---------------------------------------------- programmatic dependent launch
+// Kernels of the step chain start with pdl_wait(): launched with
+// launch_pdl they are scheduled while their predecessor drains (its launch
+// latency hidden); the wait returns once the predecessor grid has completed
+// and its memory is visible.  Launched normally, the wait is a no-op.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                              Args &&...args)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
 
 // --------------------------------------------------------------- memory
 cualign_status dmalloc(cualign_bp *h, void **p, size_t bytes);

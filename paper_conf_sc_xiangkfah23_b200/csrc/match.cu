@@ -224,6 +224,7 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
 template <int G, int U, bool DIST = false, int MINB = 1>
 __global__ void __launch_bounds__(128, MINB) k_suitor(MatchParams P)
 {
+    pdl_wait();
     auto tile = cg::tiled_partition<G>(cg::this_thread_block());
     const int lane = tile.thread_rank();
     const bool fromB = !DIST && P.propose_from_b != 0;
@@ -347,6 +348,7 @@ __global__ void k_suitor_to_mates(int64_t nT, int ninst, const int32_t *__restri
                                   const unsigned long long *__restrict__ sT, int32_t *__restrict__ mateT,
                                   int32_t *__restrict__ mateP, int64_t nP)
 {
+    pdl_wait();
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * nT;
          v += (int64_t)gridDim.x * blockDim.x) {
         const int k = (int)(v / nT);
@@ -572,6 +574,7 @@ __device__ void round_final_block(const EvalParams &P, int nblocks, int exact, d
 __global__ void __launch_bounds__(256)
 k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, const unsigned long long *work)
 {
+    pdl_wait();
     __shared__ double sd[32];
     __shared__ unsigned long long su[32];
     __shared__ bool last;
@@ -644,6 +647,7 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, con
 __global__ void k_mate_vertex(int64_t n2, const int32_t *__restrict__ mateA, const int32_t *__restrict__ Lb,
                               int32_t *__restrict__ mvA, RoundDev *rd)
 {
+    pdl_wait();
     if (blockIdx.x == 0 && threadIdx.x < 4) (&rd->overlap[0])[threadIdx.x] = 0ull; // overlap[2], card[2]
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n2; i += (int64_t)gridDim.x * blockDim.x) {
         const int e = mateA[i];
@@ -651,9 +655,21 @@ __global__ void k_mate_vertex(int64_t n2, const int32_t *__restrict__ mateA, con
     }
 }
 
+__global__ void k_match_reset(int64_t ns, unsigned long long *__restrict__ suit, int64_t nm,
+                              int32_t *__restrict__ mate)
+{
+    pdl_wait();
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < (ns > nm ? ns : nm);
+         i += (int64_t)gridDim.x * blockDim.x) {
+        if (i < ns) suit[i] = 0ull;
+        if (i < nm) mate[i] = -1;
+    }
+}
+
 __global__ void k_copy_best(int64_t nA, const int32_t *__restrict__ mateA, const RoundDev *__restrict__ rd,
                             int32_t *__restrict__ best_mate)
 {
+    pdl_wait();
     if (!rd->improved) return;
     const int32_t *src = mateA + (int64_t)rd->source * nA;
     for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < nA; a += (int64_t)gridDim.x * blockDim.x)
@@ -733,9 +749,14 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     const bool fromB = h->propose_from_b;
     P.propose_from_b = fromB ? 1 : 0;
     const int64_t nP = fromB ? nB : nA, nT = fromB ? nA : nB;
-    CA_CUDA(cudaMemsetAsync(h->suit, 0, sizeof(unsigned long long) * (size_t)(2 * nT + 1), h->stream));
-    CA_CUDA(cudaMemsetAsync(fromB ? h->mateB : h->mateA, 0xff, sizeof(int32_t) * (size_t)(2 * nP + 1),
-                            h->stream));
+    {
+        // suitor slots to 0 and proposer mates to -1 (one kernel, not two
+        // memset nodes: keeps the step's kernel chain programmatic)
+        KScope ks(h, CUALIGN_K_MATCHAUX);
+        const int64_t nmax = (2 * nT + 1) > (2 * nP + 1) ? (2 * nT + 1) : (2 * nP + 1);
+        CA_CUDA(launch_pdl(k_match_reset, dim3(grid_for(nmax, 256, h->num_sms * 4)), dim3(256), 0, h->stream,
+                           2 * nT + 1, h->suit, 2 * nP + 1, fromB ? h->mateB : h->mateA));
+    }
     const int64_t slots = P.ninst * nP;
     static const bool dbg_env = getenv("CUALIGN_MATCH_DEBUG") != nullptr;
     const bool dbg = dbg_env && !h->capturing;
@@ -773,7 +794,7 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
                 k_suitor_persistent<4, 5, 12><<<grid_for(slots * 4, 128, (int64_t)occ * h->num_sms), 128, 0,
                                                 h->stream>>>(P);
             } else if (minb >= 16) k_suitor<4, 5, false, 16><<<grid, 128, 0, h->stream>>>(P);
-            else if (minb >= 12) k_suitor<4, 5, false, 12><<<grid, 128, 0, h->stream>>>(P);
+            else if (minb >= 12) CA_CUDA(launch_pdl(k_suitor<4, 5, false, 12>, dim3(grid), dim3(128), 0, h->stream, P));
             else if (minb >= 10) k_suitor<4, 5, false, 10><<<grid, 128, 0, h->stream>>>(P);
             else k_suitor<4, 5><<<grid, 128, 0, h->stream>>>(P);
         }
@@ -789,8 +810,9 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     }
     if (P.ninst * nT > 0) {
         KScope ks(h, CUALIGN_K_MATCHAUX);
-        k_suitor_to_mates<<<grid_for(P.ninst * nT, 256, h->num_sms * 8), 256, 0, h->stream>>>(
-            nT, P.ninst, fromB ? P.Lb : P.La, h->suit, fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP);
+        CA_CUDA(launch_pdl(k_suitor_to_mates, dim3(grid_for(P.ninst * nT, 256, h->num_sms * 8)), dim3(256), 0,
+                           h->stream, nT, P.ninst, fromB ? P.Lb : P.La, (const unsigned long long *)h->suit,
+                           fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP));
         CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;
@@ -986,20 +1008,22 @@ cualign_status match_evaluate(cualign_bp *h)
         // M(i) as B vertices + zeroed overlap / card accumulators (the rest of rd persists: best)
         KScope ks(h, CUALIGN_K_MATCHAUX);
         const int64_t n2 = 2 * (int64_t)h->L.nA;
-        k_mate_vertex<<<grid_for(n2 > 0 ? n2 : 1, 256, h->num_sms * 4), 256, 0, h->stream>>>(n2, h->mateA, h->L.Lb,
-                                                                                            h->mvA, h->rd);
+        CA_CUDA(launch_pdl(k_mate_vertex, dim3(grid_for(n2 > 0 ? n2 : 1, 256, h->num_sms * 4)), dim3(256), 0,
+                           h->stream, n2, (const int32_t *)h->mateA, (const int32_t *)h->L.Lb, h->mvA, h->rd));
         CA_CUDA(cudaGetLastError());
     }
     {
         KScope ks(h, CUALIGN_K_EVAL);
-        k_eval<<<h->eval_grid, 256, 0, h->stream>>>(E, (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha, h->beta,
-                                                    h->round_p ? h->round_p : h->p_dev, h->match_work);
+        CA_CUDA(launch_pdl(k_eval, dim3(h->eval_grid), dim3(256), 0, h->stream, E,
+                           (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha, h->beta,
+                           (const int *)(h->round_p ? h->round_p : h->p_dev),
+                           (const unsigned long long *)h->match_work));
         CA_CUDA(cudaGetLastError());
     }
     {
         KScope ks(h, CUALIGN_K_MATCHAUX);
-        k_copy_best<<<grid_for(h->L.nA, 256, h->num_sms * 4), 256, 0, h->stream>>>(h->L.nA, h->mateA, h->rd,
-                                                                                  h->best_mate);
+        CA_CUDA(launch_pdl(k_copy_best, dim3(grid_for(h->L.nA, 256, h->num_sms * 4)), dim3(256), 0, h->stream,
+                           (int64_t)h->L.nA, (const int32_t *)h->mateA, (const RoundDev *)h->rd, h->best_mate));
         CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;
