@@ -3,6 +3,8 @@
 // match.cu.
 #include "internal.cuh"
 
+#include <mutex>
+
 #include <chrono>
 
 #include <math.h>
@@ -46,7 +48,9 @@ cudaMemPool_t temp_pool(int dev)
 {
     static cudaMemPool_t pools[64] = {};
     static bool made[64] = {};
+    static std::mutex mu; // handles may be created from several host threads
     if (dev < 0 || dev >= 64) return nullptr;
+    std::lock_guard<std::mutex> lock(mu);
     if (!made[dev]) {
         made[dev] = true;
         cudaMemPoolProps props = {};
