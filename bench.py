@@ -562,3 +562,9 @@ def main():
 
 if __name__ == "__main__":
     main()
+    try:
+        import torch.distributed as dist
+        if dist.is_available() and dist.is_initialized():
+            dist.destroy_process_group()
+    except Exception:  # pragma: no cover
+        pass
