@@ -189,6 +189,14 @@ static constexpr int SERIAL_SLOT = 10; // one step as ONE graph: iterate(1), the
 // selected by pointing h->yc / h->zc at them while the kernels are captured.
 static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
 {
+    // k_top2 one lane per tile here: 4x fewer threads than the 4-lane form
+    // (0.089 vs 0.065 ms alone) leave SM slots to the rounding beside it --
+    // O: 1446 vs 1394 it/s pipelined (serial: 1352 vs 1389, so 2 lanes there)
+    struct TgScope {
+        cualign_bp *h;
+        ~TgScope() { h->top2_tg = 0; }
+    } tg_scope{h};
+    h->top2_tg = 1;
     double *yc0 = h->yc, *zc0 = h->zc;
     double *yb[2] = {yc0, h->yc_b1}, *zb[2] = {zc0, h->zc_b1};
     cualign_status st = CUALIGN_OK;
@@ -762,7 +770,7 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
     // k beside iteration k+1), 2 = serial (iterate graph, then round graph).
     // Measured: O 1246 / 1300 / ~1300 it/s; R-MAT k = 5 1.03 / 1.62 / ~1.03
     // ms per step; R k = 50 8.3 ms with a fork vs 7.7 serial.  The first run
-    // of >= 21 steps times 4 steps of each (after a capture and 2 warm steps)
+    // of >= 21 steps times 4 steps of each (16 if it has >= 57 steps; after a capture and 2 warm steps)
     // and keeps the fastest; results are identical whichever runs (tests compare
     // them with the eager sequence bit for bit).  CUALIGN_PIPELINE=0/1/2
     // forces one.
@@ -803,7 +811,10 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
         return run_mode(pipe_env, n_steps, trace);
     }
     if (h->pipe_mode >= 0) return run_mode(h->pipe_mode, n_steps, trace);
-    constexpr int32_t PRE = 3, TIMED = 4, PER = PRE + TIMED; // per schedule: capture + warm, timed
+    // per schedule: capture + warm, timed (16 timed steps when the run is
+    // long enough: 4 steps of ~0.7 ms left the O choice to noise)
+    constexpr int32_t PRE = 3;
+    const int32_t TIMED = n_steps >= 3 * (PRE + 16) ? 16 : 4, PER = PRE + TIMED;
     if (n_steps < 3 * PER || h->timing) return run_pipelined(h, n_steps, trace); // undecided: default
     auto tr = [&](int32_t off) { return trace ? trace + off : nullptr; };
     float t[3] = {0.f, 0.f, 0.f};

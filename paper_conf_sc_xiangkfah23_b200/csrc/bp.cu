@@ -92,8 +92,7 @@ __device__ __forceinline__ double clamp_beta(double x, double beta)
 }
 
 constexpr int B_CHUNK = 32;
-constexpr int TG = 8;                 // lanes per tile in k_top2
-constexpr int TB_U = B_CHUNK / TG;    // gathers per lane per chunk
+constexpr int TG_DEFAULT = 2;         // lanes per tile in k_top2 (CUALIGN_TOP2_TG: 1, 2, 4 or 8)
 
 struct Top2Args {
     int64_t nA, nchunks;    // A rows to process (a0 .. a0+nA-1), B chunks
@@ -107,8 +106,11 @@ struct Top2Args {
     unsigned int *Bcnt;
 };
 
+// TG lanes per tile; each lane keeps B_CHUNK / TG gathers in flight
+template <int TG>
 __global__ void __launch_bounds__(256) k_top2(Top2Args T)
 {
+    constexpr int TB_U = B_CHUNK / TG; // gathers per lane per chunk
     pdl_wait();
     auto tile = cg::tiled_partition<TG>(cg::this_thread_block());
     const int lane = tile.thread_rank();
@@ -121,7 +123,7 @@ __global__ void __launch_bounds__(256) k_top2(Top2Args T)
             const int64_t a = T.a0 + t;
             const int64_t lo = T.Arow[a], hi = T.Arow[a + 1];
             // TA_U loads per lane in flight before any use (rows are ~k long)
-            constexpr int TA_U = 4;
+            constexpr int TA_U = B_CHUNK / TG;
             for (int64_t e0 = lo + lane; e0 < hi; e0 += TG * TA_U) {
                 double v[TA_U];
 #pragma unroll
@@ -833,9 +835,25 @@ cualign_status bp_top2(cualign_bp *h)
         Top2Args T{(int64_t)(h->a1 - h->a0), h->nchunks, (int64_t)h->a0, h->L.Arow, h->cdesc, h->Bcp,
                    sh ? h->Bptr_loc : h->L.Bptr, sh ? h->Bedge_loc : h->L.Bedge, h->yp, h->zp, h->Atop,
                    sh ? h->Btop_part : h->Btop, h->Bct, h->Bcnt};
-        if (T.nA + T.nchunks > 0)
-            CA_CUDA(launch_pdl(k_top2, dim3(grid_for((T.nA + T.nchunks) * TG, 256, 1 << 30)), dim3(256), 0,
-                               h->stream, T));
+        // lanes per tile: CUALIGN_TOP2_TG (measurement knob), else the
+        // capturing graph's choice (h->top2_tg), else TG_DEFAULT
+        static const int tg_env = [] {
+            const char *v = getenv("CUALIGN_TOP2_TG");
+            const int x = v ? atoi(v) : 0;
+            return (x == 1 || x == 2 || x == 4 || x == 8) ? x : 0;
+        }();
+        const int tg = tg_env ? tg_env : (h->top2_tg ? h->top2_tg : TG_DEFAULT);
+        const int64_t nt = T.nA + T.nchunks;
+        if (nt > 0) {
+            if (tg == 1)
+                CA_CUDA(launch_pdl(k_top2<1>, dim3(grid_for(nt, 256, 1 << 30)), dim3(256), 0, h->stream, T));
+            else if (tg == 2)
+                CA_CUDA(launch_pdl(k_top2<2>, dim3(grid_for(nt * 2, 256, 1 << 30)), dim3(256), 0, h->stream, T));
+            else if (tg == 4)
+                CA_CUDA(launch_pdl(k_top2<4>, dim3(grid_for(nt * 4, 256, 1 << 30)), dim3(256), 0, h->stream, T));
+            else
+                CA_CUDA(launch_pdl(k_top2<8>, dim3(grid_for(nt * 8, 256, 1 << 30)), dim3(256), 0, h->stream, T));
+        }
         CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;

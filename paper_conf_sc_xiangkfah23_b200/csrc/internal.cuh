@@ -161,6 +161,7 @@ struct cualign_bp {
     // kernels report (round_p; = p_dev except in a pipelined run)
     double *yc_b1 = nullptr, *zc_b1 = nullptr;
     int pipe_mode = -1;                 // step schedule: -1 undecided, 0 forked graph, 1 pipelined, 2 serial
+    int top2_tg = 0;                    // k_top2 lanes per tile while capturing (0: default; pipelined graphs: 1)
     int *rp_dev = nullptr;
     const int *round_p = nullptr;
 
