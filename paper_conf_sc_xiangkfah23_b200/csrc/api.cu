@@ -514,7 +514,10 @@ static cualign_status open_handle(const cualign_params *params, cualign_bp **out
         // kernels are scheduled first when square-pass CTAs retire
         int lo = 0, hi = 0;
         CA_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-        CA_CUDA(cudaStreamCreateWithPriority(&h->gstream2, cudaStreamNonBlocking, hi));
+        // CUALIGN_ROUND_PRIO (measurement knob): 0 = hi (default), 1 = same as
+        // the iteration, 2 = lowest
+        static const int rp = getenv("CUALIGN_ROUND_PRIO") ? atoi(getenv("CUALIGN_ROUND_PRIO")) : 0;
+        CA_CUDA(cudaStreamCreateWithPriority(&h->gstream2, cudaStreamNonBlocking, rp == 1 ? 0 : rp == 2 ? lo : hi));
     }
     for (int i = 0; i < 2; i++) {
         CA_CUDA(cudaEventCreateWithFlags(&h->sync_ev[i], cudaEventDisableTiming));

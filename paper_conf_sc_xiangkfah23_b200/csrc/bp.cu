@@ -388,12 +388,20 @@ constexpr int SQT_PER_THREAD = SQT_CHUNK / (SQT_CWARPS * 32);
 
 using namespace ptx;
 
-template <class V, bool NOATOM = false>
+// DYN: chunks taken from a queue (ctr[0], one atomic per chunk by the
+// producer lane, STAGES chunks ahead of use) instead of the static stride
+// blockIdx + k*grid: a CTA that starts late -- its SM still running the
+// rounding branch of a pipelined step -- takes fewer chunks instead of
+// finishing last.  The last producer to finish resets the queue (ctr[1]
+// counts finished producers).  The chunk id travels with its stage in smem.
+template <class V, bool NOATOM = false, bool DYN = false>
 __global__ void __launch_bounds__((SQT_CWARPS + 1) * 32)
 k_square_tma(int64_t nsq, const int2 *__restrict__ sq_ef, V *__restrict__ sq_val,
              const double *__restrict__ u, double beta, const double2 *__restrict__ gh,
-             const int *__restrict__ p_dev, double fp_scale, unsigned long long *__restrict__ tacc)
+             const int *__restrict__ p_dev, double fp_scale, unsigned long long *__restrict__ tacc,
+             unsigned int *__restrict__ ctr)
 {
+    __shared__ int s_chunk[SQT_STAGES];
     // dynamic shared memory: [full | empty barriers (128 B)] [ef stages] [value stages]
     extern __shared__ __align__(128) unsigned char sq_smem[];
     uint64_t *full = reinterpret_cast<uint64_t *>(sq_smem);
@@ -416,9 +424,25 @@ k_square_tma(int64_t nsq, const int2 *__restrict__ sq_ef, V *__restrict__ sq_val
         if (lane == 0) {
             const uint64_t policy = policy_evict_first();
             int i = 0;
-            for (int64_t c = blockIdx.x; c < nchunks; c += gridDim.x, i++) {
+            for (int64_t c = blockIdx.x;; c += gridDim.x, i++) {
                 const int s = i % SQT_STAGES;
                 if (i >= SQT_STAGES) mbar_wait(&empty[s], (uint32_t)((i / SQT_STAGES) - 1) & 1u);
+                if (DYN) {
+                    c = atomicAdd(ctr, 1u);
+                    if (c >= nchunks) {
+                        s_chunk[s] = -1; // end of queue: released by the arrive
+                        mbar_arrive(&full[s]);
+                        __threadfence();
+                        if (atomicAdd(ctr + 1, 1u) == gridDim.x - 1) {
+                            ctr[0] = 0u; // every producer is past its last take
+                            ctr[1] = 0u;
+                        }
+                        break;
+                    }
+                    s_chunk[s] = (int)c;
+                } else if (c >= nchunks) {
+                    break;
+                }
                 const int64_t q0 = c * SQT_CHUNK;
                 const int n = (int)((nsq - q0) < SQT_CHUNK ? (nsq - q0) : SQT_CHUNK);
                 // 16-byte multiples (the arrays carry 2 elements of padding)
@@ -435,9 +459,14 @@ k_square_tma(int64_t nsq, const int2 *__restrict__ sq_ef, V *__restrict__ sq_val
     const double g = ghp.x, hh = ghp.y;
     const int tid = threadIdx.x; // consumer thread 0 .. SQT_CWARPS*32-1
     int i = 0;
-    for (int64_t c = blockIdx.x; c < nchunks; c += gridDim.x, i++) {
+    for (int64_t c = blockIdx.x;; c += gridDim.x, i++) {
         const int s = i % SQT_STAGES;
+        if (!DYN && c >= nchunks) break;
         mbar_wait(&full[s], (uint32_t)(i / SQT_STAGES) & 1u);
+        if (DYN) {
+            c = *(volatile int *)&s_chunk[s];
+            if (c < 0) break;
+        }
         const int64_t q0 = c * SQT_CHUNK;
         const int n = (int)((nsq - q0) < SQT_CHUNK ? (nsq - q0) : SQT_CHUNK);
         int2 ef[SQT_PER_THREAD];
@@ -579,10 +608,10 @@ constexpr size_t square_tma_smem()
     return 128 + (sizeof(int2) + sizeof(V)) * SQT_STAGES * SQT_CHUNK;
 }
 
-template <class V, bool NOATOM = false>
+template <class V, bool NOATOM = false, bool DYN = false>
 void square_tma_launch_v(cualign_bp *h, V *vals)
 {
-    auto fn = k_square_tma<V, NOATOM>;
+    auto fn = k_square_tma<V, NOATOM, DYN>;
     constexpr size_t smem = square_tma_smem<V>();
     static bool attr_set = false; // per process and V: the attribute is a property of the function
     if (!attr_set) {
@@ -596,13 +625,20 @@ void square_tma_launch_v(cualign_bp *h, V *vals)
     const int64_t nchunks = (h->nsq + SQT_CHUNK - 1) / SQT_CHUNK;
     const int grid = grid_for(nchunks, 1, (int64_t)occ * h->num_sms);
     (void)launch_pdl(fn, dim3(grid), dim3(block), smem, h->stream, h->nsq, h->sq_ef, vals, (const double *)h->u,
-                     h->beta, (const double2 *)h->gh_dev, (const int *)h->p_dev, h->fp_scale, h->tacc);
+                     h->beta, (const double2 *)h->gh_dev, (const int *)h->p_dev, h->fp_scale, h->tacc, h->sq_ctr);
 }
 
 void square_tma_launch(cualign_bp *h)
 {
-    if (h->sq_val32) square_tma_launch_v(h, h->sq_val32);
-    else square_tma_launch_v(h, h->sq_val);
+    // CUALIGN_SQ_DYN (measurement knob): 1 = chunk queue, 0 = static stride
+    static const int dyn = getenv("CUALIGN_SQ_DYN") ? atoi(getenv("CUALIGN_SQ_DYN")) : 0;
+    if (dyn) {
+        if (h->sq_val32) square_tma_launch_v<float2, false, true>(h, h->sq_val32);
+        else square_tma_launch_v<double2, false, true>(h, h->sq_val);
+    } else {
+        if (h->sq_val32) square_tma_launch_v(h, h->sq_val32);
+        else square_tma_launch_v(h, h->sq_val);
+    }
 }
 
 template <bool UPDATE, bool EXACT, int SQ_U, bool HINTS, bool NOATOM = false>
@@ -783,6 +819,10 @@ cualign_status bp_setup(cualign_bp *h)
     CA_TRY(dalloc(h, &h->Btop, (size_t)nB + 1));
     CA_TRY(dalloc(h, &h->Bcnt, (size_t)nB + 1));
     CA_CUDA(cudaMemsetAsync(h->Bcnt, 0, sizeof(unsigned int) * ((size_t)nB + 1), h->stream));
+    if (!h->sq_ctr) {
+        CA_TRY(dalloc(h, &h->sq_ctr, 2));
+        CA_CUDA(cudaMemsetAsync(h->sq_ctr, 0, 2 * sizeof(unsigned int), h->stream));
+    }
     const int64_t *Bptr = h->L.Bptr;
     if (h->world > 1) {
         // partial B-side top-2 over the owned edges, gathered and merged

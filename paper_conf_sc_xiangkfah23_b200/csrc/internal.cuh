@@ -131,6 +131,7 @@ struct cualign_bp {
     int4 *cdesc = nullptr;              // nchunks: (start, end, owning B vertex, first chunk of a hub or -1)
     double2 *Bct = nullptr;             // nchunks: (max1, max2) of z^p over the chunk
     unsigned int *Bcnt = nullptr;       // nB: chunks finished (hub columns' last-arriver merge)
+    unsigned int *sq_ctr = nullptr;     // 2: square-pass chunk queue head, CTAs done (self-resetting)
     double2 *Atop = nullptr, *Btop = nullptr; // per-vertex (max1, max2) of y^p / z^p
     int64_t comm_calls = 0, comm_bytes_in = 0; // exchanges (sharded handles)
     double comm_ms = 0.0;
