@@ -883,16 +883,20 @@ cualign_status bp_top2(cualign_bp *h)
             return (x == 1 || x == 2 || x == 4 || x == 8) ? x : 0;
         }();
         const int tg = tg_env ? tg_env : (h->top2_tg ? h->top2_tg : TG_DEFAULT);
+        // CUALIGN_TOP2_GRID (measurement knob): at most this many blocks per SM
+        // (grid-stride tiles), leaving SM slots to a concurrent rounding
+        static const int gcap_env = getenv("CUALIGN_TOP2_GRID") ? atoi(getenv("CUALIGN_TOP2_GRID")) : 0;
+        const int gcap = gcap_env > 0 ? gcap_env * h->num_sms : (1 << 30);
         const int64_t nt = T.nA + T.nchunks;
         if (nt > 0) {
             if (tg == 1)
-                CA_CUDA(launch_pdl(k_top2<1>, dim3(grid_for(nt, 256, 1 << 30)), dim3(256), 0, h->stream, T));
+                CA_CUDA(launch_pdl(k_top2<1>, dim3(grid_for(nt, 256, gcap)), dim3(256), 0, h->stream, T));
             else if (tg == 2)
-                CA_CUDA(launch_pdl(k_top2<2>, dim3(grid_for(nt * 2, 256, 1 << 30)), dim3(256), 0, h->stream, T));
+                CA_CUDA(launch_pdl(k_top2<2>, dim3(grid_for(nt * 2, 256, gcap)), dim3(256), 0, h->stream, T));
             else if (tg == 4)
-                CA_CUDA(launch_pdl(k_top2<4>, dim3(grid_for(nt * 4, 256, 1 << 30)), dim3(256), 0, h->stream, T));
+                CA_CUDA(launch_pdl(k_top2<4>, dim3(grid_for(nt * 4, 256, gcap)), dim3(256), 0, h->stream, T));
             else
-                CA_CUDA(launch_pdl(k_top2<8>, dim3(grid_for(nt * 8, 256, 1 << 30)), dim3(256), 0, h->stream, T));
+                CA_CUDA(launch_pdl(k_top2<8>, dim3(grid_for(nt * 8, 256, gcap)), dim3(256), 0, h->stream, T));
         }
         CA_CUDA(cudaGetLastError());
     }
