@@ -326,9 +326,9 @@ def main():
 
     # ------------------------------------------------------------- warmup
     # (each step = iterate(1) + round, replayed from the library's CUDA graph)
-    # The library picks the step schedule on its first run of >= 21 steps by
-    # timing each (16 timed steps per schedule from 57 steps on); do that
-    # here, untimed, before the warm-up.
+    # The library picks the step schedule on its first run of >= 14 steps by
+    # timing pipelined and serial (16 timed steps each from 38 steps on); do
+    # that here, untimed, before the warm-up.
     h.run(57)
     h.run(args.warmup)
     torch.cuda.synchronize()

@@ -773,7 +773,7 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
     // k beside iteration k+1), 2 = serial (iterate graph, then round graph).
     // Measured: O 1246 / 1300 / ~1300 it/s; R-MAT k = 5 1.03 / 1.62 / ~1.03
     // ms per step; R k = 50 8.3 ms with a fork vs 7.7 serial.  The first run
-    // of >= 21 steps times 4 steps of each (16 if it has >= 57 steps; after a capture and 2 warm steps)
+    // of >= 14 steps times 4 steps of pipelined and serial (16 if it has >= 38 steps; after a capture and 2 warm steps)
     // and keeps the fastest; results are identical whichever runs (tests compare
     // them with the eager sequence bit for bit).  CUALIGN_PIPELINE=0/1/2
     // forces one.
@@ -815,29 +815,33 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
     }
     if (h->pipe_mode >= 0) return run_mode(h->pipe_mode, n_steps, trace);
     // per schedule: capture + warm, timed (16 timed steps when the run is
-    // long enough: 4 steps of ~0.7 ms left the O choice to noise)
-    constexpr int32_t PRE = 3;
-    const int32_t TIMED = n_steps >= 3 * (PRE + 16) ? 16 : 4, PER = PRE + TIMED;
-    if (n_steps < 3 * PER || h->timing) return run_pipelined(h, n_steps, trace); // undecided: default
+    // long enough: 4 steps of ~0.7 ms left the O choice to noise).  Only
+    // pipelined and serial are timed: the forked graph was never ahead of
+    // the better of the two (O 1246 vs 1300+, R k = 5 1.03 vs 1.01-1.03 ms,
+    // R k = 50 8.3 vs 7.7 ms) and its timed steps are part of the run.
+    constexpr int32_t PRE = 3, NSEL = 2;
+    const int sel[NSEL] = {1, 2};
+    const int32_t TIMED = n_steps >= NSEL * (PRE + 16) ? 16 : 4, PER = PRE + TIMED;
+    if (n_steps < NSEL * PER || h->timing) return run_pipelined(h, n_steps, trace); // undecided: default
     auto tr = [&](int32_t off) { return trace ? trace + off : nullptr; };
     float t[3] = {0.f, 0.f, 0.f};
-    for (int mode = 0; mode < 3; mode++) {
+    for (int i = 0; i < NSEL; i++) {
+        const int mode = sel[i];
         cudaEvent_t e0 = get_event(h), e1 = get_event(h);
-        CA_TRY(run_mode(mode, PRE, tr(PER * mode)));
+        CA_TRY(run_mode(mode, PRE, tr(PER * i)));
         CA_CUDA(cudaEventRecord(e0, h->stream));
-        CA_TRY(run_mode(mode, TIMED, tr(PER * mode + PRE)));
+        CA_TRY(run_mode(mode, TIMED, tr(PER * i + PRE)));
         CA_CUDA(cudaEventRecord(e1, h->stream));
         CA_CUDA(cudaEventSynchronize(e1));
         CA_CUDA(cudaEventElapsedTime(&t[mode], e0, e1));
         h->event_pool.push_back(e0);
         h->event_pool.push_back(e1);
     }
-    // the pipelined schedule unless another is clearly (> 2 %) faster
+    // the pipelined schedule unless serial is clearly (> 2 %) faster
     int best = 1;
-    for (int mode : {0, 2})
-        if (t[mode] < 0.98f * t[best]) best = mode;
+    if (t[2] < 0.98f * t[1]) best = 2;
     h->pipe_mode = best;
-    return run_mode(h->pipe_mode, n_steps - 3 * PER, tr(3 * PER));
+    return run_mode(h->pipe_mode, n_steps - NSEL * PER, tr(NSEL * PER));
 }
 } // namespace cualign
 
