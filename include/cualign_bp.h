@@ -116,6 +116,17 @@ typedef struct {
     int32_t rank;
     int32_t world;
     const void *nccl_unique_id; /* 128-byte ncclUniqueId or NULL */
+    /* Result-neutral tuning (0 = automatic; every choice gives the same bits):
+     *   schedule: step schedule of cualign_bp_run / run_trace with both
+     *     halves of a step: 0 = chosen by the
+     *     library, 1 = pipelined (rounding of iteration k beside iteration
+     *     k+1), 2 = serial (iteration, then its rounding), 3 = forked (the
+     *     rounding beside the square pass of its own iteration);
+     *   square_tile_log: the squares are grouped into (e block, f block)
+     *     tiles of 2^k edges; -1 = no tiles,
+     *     1..30 = that block size. */
+    int32_t schedule;
+    int32_t square_tile_log;
 } cualign_params;
 
 /* Result of one rounding step (Alg. 2 l.17-24). */

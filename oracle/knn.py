@@ -6,13 +6,12 @@ V_B, s(u, v) = cosine_similarity(Y_A(u), Y_B(v)) (l.9), then keep the kNN
 edges (l.12-14).  Readings (DESIGN.md "kNN"):
   * Z19: "k least-weighted edges" of a *similarity* is read as the k MOST
     similar B vertices of each A vertex; ties go to the lower B index;
-  * a zero embedding has similarity 0 with everything;
-  * precision: the tensor-core path multiplies the unit vectors rounded to
-    bf16 (round to nearest even) and accumulates in fp32.  The oracle follows
-    the same definition with exact arithmetic: unit vectors in fp64 (sum of
-    squares in ascending coordinate order, sqrt, divide), rounded to bf16,
-    dot products of the bf16 values in fp64 (every product is exact).
-    `cosine_fp64` gives the unrounded cosine for comparison.
+  * a zero embedding has similarity 0 with everything.
+The reference is the paper's cosine in fp64 (`cosine_fp64`): unit vectors
+(sum of squares in ascending coordinate order, sqrt, divide) and their dot
+products.  An implementation that computes in lower precision is judged
+against it with the rigorous error bound `dot_error_bound` (below), not
+against a copy of its own rounding.
 Plain numpy, written for checking by eye, not speed.
 """
 from __future__ import annotations
@@ -20,51 +19,43 @@ from __future__ import annotations
 import numpy as np
 
 
-def round_bf16(x: np.ndarray) -> np.ndarray:
-    """fp64 -> nearest bf16 (ties to even), returned as fp64.  Done as
-    fp64 -> fp32 (nearest) -> bf16 (nearest even on the top 16 bits) only when
-    the fp32 step is exact for the final rounding; to avoid double rounding
-    the bf16 rounding is applied to the fp64 value directly."""
-    x = np.asarray(x, dtype=np.float64)
-    out = np.empty_like(x)
-    flat, res = x.ravel(), out.ravel()
-    for i in range(flat.shape[0]):
-        v = float(flat[i])
-        if v == 0.0 or not np.isfinite(v):
-            res[i] = v
-            continue
-        m, e = np.frexp(v)            # v = m * 2^e, 0.5 <= |m| < 1
-        # bf16 keeps 8 significant bits: |m| * 2^8 rounded to an integer, ties to even
-        scaled = m * 256.0
-        r = np.round(scaled)          # numpy rounds half to even
-        res[i] = np.ldexp(r / 256.0, e)
-    return out
-
-
 def unit_rows(Y: np.ndarray) -> np.ndarray:
-    """Rows divided by their Euclidean norm (fp64; zero rows stay zero)."""
+    """Rows divided by their Euclidean norm (fp64; zero rows stay zero).  The
+    sum of squares runs over the coordinates in ascending order (one column
+    at a time, all rows together)."""
     Y = np.asarray(Y, dtype=np.float64)
+    ss = np.zeros(Y.shape[0])
+    for j in range(Y.shape[1]):
+        ss = ss + Y[:, j] * Y[:, j]
     out = np.zeros_like(Y)
-    for i in range(Y.shape[0]):
-        ss = 0.0
-        for j in range(Y.shape[1]):       # ascending coordinate order
-            ss = ss + Y[i, j] * Y[i, j]
-        if ss > 0.0:
-            nrm = np.sqrt(ss)
-            out[i] = Y[i] / nrm
+    nz = ss > 0.0
+    out[nz] = Y[nz] / np.sqrt(ss[nz])[:, None]
     return out
-
-
-def similarity_bf16(YA: np.ndarray, YB: np.ndarray) -> np.ndarray:
-    """s(u, v) of the tensor-core definition: dot products of the bf16-rounded
-    unit vectors, exact products summed in fp64."""
-    ua = round_bf16(unit_rows(YA))
-    ub = round_bf16(unit_rows(YB))
-    return ua @ ub.T
 
 
 def cosine_fp64(YA: np.ndarray, YB: np.ndarray) -> np.ndarray:
+    """s(u, v) = cos(Y_A(u), Y_B(v)) (Alg. 1 l.9), all pairs, fp64."""
     return unit_rows(YA) @ unit_rows(YB).T
+
+
+def dot_error_bound(YA: np.ndarray, YB: np.ndarray, unit_roundoff: float, acc_roundoff: float) -> np.ndarray:
+    """Rigorous bound on |s~(u, v) - s(u, v)| for a dot product of the unit
+    vectors whose inputs are each rounded to a format with unit roundoff
+    `unit_roundoff` (bf16: 2^-8) and accumulated in a format with unit
+    roundoff `acc_roundoff` (fp32: 2^-24) over d terms.  With
+    u~_i = u_i (1 + a_i), v~_i = v_i (1 + b_i), |a_i|, |b_i| <= r:
+        |u~.v~ - u.v| <= (2 r + r^2) sum_i |u_i v_i|
+    and the accumulation of d products adds at most
+        gamma_d sum_i |u~_i v~_i| <= gamma_d (1 + r)^2 sum_i |u_i v_i|,
+    gamma_d = d q / (1 - d q) (standard recursive-summation bound, q = acc
+    roundoff; it also covers any summation order and fused products).
+    The extra 1e-15 absorbs the fp64 error of computing the reference itself."""
+    UA, UB = np.abs(unit_rows(YA)), np.abs(unit_rows(YB))
+    d = UA.shape[1]
+    r, q = float(unit_roundoff), float(acc_roundoff)
+    gamma_d = d * q / (1.0 - d * q)
+    absdot = UA @ UB.T
+    return (2 * r + r * r + gamma_d * (1 + r) ** 2) * absdot + 1e-15
 
 
 def knn_from_similarity(S: np.ndarray, k: int):
@@ -84,5 +75,5 @@ def knn_from_similarity(S: np.ndarray, k: int):
 
 
 def knn(YA: np.ndarray, YB: np.ndarray, k: int):
-    """Alg. 1 l.7-14 under the readings above."""
-    return knn_from_similarity(similarity_bf16(YA, YB), k)
+    """Alg. 1 l.7-14 under the readings above (fp64 cosine)."""
+    return knn_from_similarity(cosine_fp64(YA, YB), k)

@@ -56,7 +56,8 @@ class Params_t(ctypes.Structure):
     _fields_ = [("alpha", ctypes.c_double), ("beta", ctypes.c_double), ("gamma", ctypes.c_double),
                 ("flags", ctypes.c_uint32), ("device", ctypes.c_int32), ("stream", ctypes.c_void_p),
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
-                ("nccl_unique_id", ctypes.c_void_p)]
+                ("nccl_unique_id", ctypes.c_void_p), ("schedule", ctypes.c_int32),
+                ("square_tile_log", ctypes.c_int32)]
 
 
 class RoundInfo_t(ctypes.Structure):
@@ -203,9 +204,10 @@ class CuAlignBP:
     """One alignment problem resident on a GPU (Alg. 2 state + S)."""
 
     def __init__(self, A, B, L, alpha=1.0, beta=2.0, gamma=0.99, flags=0, device=0, stream=None,
-                 world=1, rank=0, nccl_id=None):
+                 world=1, rank=0, nccl_id=None, schedule=0, square_tile_log=0):
         """world > 1 with nccl_id (bytes): this process is shard `rank`;
-        world > 1 without nccl_id: `world` virtual shards in one handle."""
+        world > 1 without nccl_id: `world` virtual shards in one handle.
+        schedule / square_tile_log: result-neutral tuning (cualign_params)."""
         lib = load_library()
         Ap, dA = _prep(A.rowptr, np.int64, "int64")
         Aj, _ = _prep(A.col, np.int32, "int32")
@@ -233,7 +235,8 @@ class CuAlignBP:
         self._nccl_id = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
         prm = Params_t(float(alpha), float(beta), float(gamma), int(flags), int(device),
                        _stream_ptr(stream), int(rank), self.world,
-                       ctypes.cast(self._nccl_id, ctypes.c_void_p) if self._nccl_id is not None else None)
+                       ctypes.cast(self._nccl_id, ctypes.c_void_p) if self._nccl_id is not None else None,
+                       int(schedule), int(square_tile_log))
         h = ctypes.c_void_p()
         _check(lib.cualign_bp_init(ctypes.byref(ga), ctypes.byref(gb), ctypes.byref(el),
                                    ctypes.byref(prm), ctypes.byref(h)))

@@ -14,6 +14,14 @@ namespace cualign {
 
 static thread_local char g_err[1024] = "";
 
+#ifdef CUALIGN_PROBES
+int probe_knob(const char *name, int dflt)
+{
+    const char *v = getenv(name);
+    return v ? atoi(v) : dflt;
+}
+#endif
+
 void set_error(const char *fmt, ...)
 {
     va_list ap;
@@ -361,7 +369,7 @@ static cualign_status run_graph(cualign_bp *h, int32_t n, int what)
 
 void init_trace(cualign_bp *h, const char *what)
 {
-    static const bool on = getenv("CUALIGN_INIT_TRACE") != nullptr;
+    static const bool on = probe_knob("CUALIGN_INIT_TRACE", 0) != 0;
     if (!on) return;
     static thread_local std::chrono::steady_clock::time_point t0;
     cudaStreamSynchronize(h->stream);
@@ -462,6 +470,14 @@ static cualign_status check_params(const cualign_params *p)
         set_error("gamma must be in (0, 1], got %g", p->gamma);
         return CUALIGN_EINVAL;
     }
+    if (p->schedule < 0 || p->schedule > 3) {
+        set_error("schedule must be 0 (automatic), 1 (pipelined), 2 (serial) or 3 (forked), got %d", p->schedule);
+        return CUALIGN_EINVAL;
+    }
+    if (p->square_tile_log < -1 || p->square_tile_log > 30) {
+        set_error("square_tile_log must be -1 (no tiles), 0 (automatic) or 1..30, got %d", p->square_tile_log);
+        return CUALIGN_EINVAL;
+    }
     if ((p->flags & CUALIGN_FLAG_FP32_S) && (p->flags & CUALIGN_FLAG_EXACT)) {
         set_error("CUALIGN_FLAG_FP32_S and CUALIGN_FLAG_EXACT are exclusive");
         return CUALIGN_EINVAL;
@@ -499,6 +515,8 @@ static cualign_status open_handle(const cualign_params *params, cualign_bp **out
     h->timing = (params->flags & CUALIGN_FLAG_TIMING) != 0;
     h->world = params->world <= 0 ? 1 : params->world;
     h->rank = params->rank < 0 ? 0 : params->rank;
+    h->sched_param = params->schedule;
+    h->tile_log_param = params->square_tile_log;
     *out = h;
     CA_CUDA(cudaSetDevice(h->dev));
     CA_CUDA(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->dev));
@@ -514,9 +532,9 @@ static cualign_status open_handle(const cualign_params *params, cualign_bp **out
         // kernels are scheduled first when square-pass CTAs retire
         int lo = 0, hi = 0;
         CA_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-        // CUALIGN_ROUND_PRIO (measurement knob): 0 = hi (default), 1 = same as
+        // CUALIGN_ROUND_PRIO (probe build): 0 = hi (default), 1 = same as
         // the iteration, 2 = lowest
-        static const int rp = getenv("CUALIGN_ROUND_PRIO") ? atoi(getenv("CUALIGN_ROUND_PRIO")) : 0;
+        static const int rp = probe_knob("CUALIGN_ROUND_PRIO", 0);
         CA_CUDA(cudaStreamCreateWithPriority(&h->gstream2, cudaStreamNonBlocking, rp == 1 ? 0 : rp == 2 ? lo : hi));
     }
     for (int i = 0; i < 2; i++) {
@@ -777,7 +795,8 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
     // and keeps the fastest; results are identical whichever runs (tests compare
     // them with the eager sequence bit for bit).  CUALIGN_PIPELINE=0/1/2
     // forces one.
-    static const int pipe_env = getenv("CUALIGN_PIPELINE") ? atoi(getenv("CUALIGN_PIPELINE")) : -1;
+    // cualign_params.schedule: 1 pipelined, 2 serial, 3 forked (pipe_mode 0)
+    const int pipe_env = h->sched_param == 3 ? 0 : (h->sched_param > 0 ? h->sched_param : -1);
     const bool both = what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND) &&
                       !(h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS));
     auto run_plain = [&](int32_t n, RoundDev *tr) -> cualign_status {
@@ -810,7 +829,7 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
     };
     if (!both) return run_plain(n_steps, trace);
     if (pipe_env >= 0 && pipe_env <= 2) {
-        h->pipe_mode = pipe_env; // forced (reported as chosen)
+        h->pipe_mode = pipe_env; // given by the caller (reported as chosen)
         return run_mode(pipe_env, n_steps, trace);
     }
     if (h->pipe_mode >= 0) return run_mode(h->pipe_mode, n_steps, trace);
@@ -819,7 +838,7 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
     // pipelined and serial are timed: the forked graph was never ahead of
     // the better of the two (O 1246 vs 1300+, R k = 5 1.03 vs 1.01-1.03 ms,
     // R k = 50 8.3 vs 7.7 ms) and its timed steps are part of the run.
-    constexpr int32_t PRE = 3, NSEL = 2;
+    constexpr int32_t PRE = 4, NSEL = 2; // PRE even: warm-up and timed windows use the same buffer parity
     const int sel[NSEL] = {1, 2};
     const int32_t TIMED = n_steps >= NSEL * (PRE + 16) ? 16 : 4, PER = PRE + TIMED;
     if (n_steps < NSEL * PER || h->timing) return run_pipelined(h, n_steps, trace); // undecided: default

@@ -596,7 +596,7 @@ void square_launch_v(cualign_bp *h, V *vals)
     int grid = one_wave_grid(h, (const void *)fn, 256, h->nsq, 256 * SQ_U);
     // leave room for the concurrent rounding branch (graph step): a fraction
     // of the resident CTAs still saturates HBM
-    static const double frac = getenv("CUALIGN_SQ_FRAC") ? atof(getenv("CUALIGN_SQ_FRAC")) : 1.0;
+    static const double frac = probe_knob("CUALIGN_SQ_FRAC_PCT", 100) / 100.0;
     if (frac > 0.0 && frac < 1.0) grid = (int)(grid * frac) > 0 ? (int)(grid * frac) : 1;
     fn<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, vals, h->u, h->beta, h->gh_dev, h->p_dev, h->fp_scale, h->tacc,
                                     h->sq_pos, h->Ffull);
@@ -609,36 +609,35 @@ constexpr size_t square_tma_smem()
 }
 
 template <class V, bool NOATOM = false, bool DYN = false>
-void square_tma_launch_v(cualign_bp *h, V *vals)
+cualign_status square_tma_launch_v(cualign_bp *h, V *vals)
 {
     auto fn = k_square_tma<V, NOATOM, DYN>;
     constexpr size_t smem = square_tma_smem<V>();
-    static bool attr_set = false; // per process and V: the attribute is a property of the function
-    if (!attr_set) {
-        cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        attr_set = true;
-    }
+    // > 48 KB of dynamic shared memory needs the opt-in attribute, which
+    // belongs to the function in the CURRENT device's context: set it on
+    // every launch (cheap), so handles on several devices each get it
+    CA_CUDA(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int block = (SQT_CWARPS + 1) * 32;
     int occ = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, block, smem) != cudaSuccess || occ < 1) occ = 1;
     (void)cudaGetLastError();
     const int64_t nchunks = (h->nsq + SQT_CHUNK - 1) / SQT_CHUNK;
     const int grid = grid_for(nchunks, 1, (int64_t)occ * h->num_sms);
-    (void)launch_pdl(fn, dim3(grid), dim3(block), smem, h->stream, h->nsq, h->sq_ef, vals, (const double *)h->u,
-                     h->beta, (const double2 *)h->gh_dev, (const int *)h->p_dev, h->fp_scale, h->tacc, h->sq_ctr);
+    CA_CUDA(launch_pdl(fn, dim3(grid), dim3(block), smem, h->stream, h->nsq, h->sq_ef, vals, (const double *)h->u,
+                       h->beta, (const double2 *)h->gh_dev, (const int *)h->p_dev, h->fp_scale, h->tacc, h->sq_ctr));
+    return CUALIGN_OK;
 }
 
-void square_tma_launch(cualign_bp *h)
+cualign_status square_tma_launch(cualign_bp *h)
 {
-    // CUALIGN_SQ_DYN (measurement knob): 1 = chunk queue, 0 = static stride
-    static const int dyn = getenv("CUALIGN_SQ_DYN") ? atoi(getenv("CUALIGN_SQ_DYN")) : 0;
+    // CUALIGN_SQ_DYN (probe build): 1 = chunk queue, 0 = static stride
+    static const int dyn = probe_knob("CUALIGN_SQ_DYN", 0);
     if (dyn) {
-        if (h->sq_val32) square_tma_launch_v<float2, false, true>(h, h->sq_val32);
-        else square_tma_launch_v<double2, false, true>(h, h->sq_val);
-    } else {
-        if (h->sq_val32) square_tma_launch_v(h, h->sq_val32);
-        else square_tma_launch_v(h, h->sq_val);
+        if (h->sq_val32) return square_tma_launch_v<float2, false, true>(h, h->sq_val32);
+        return square_tma_launch_v<double2, false, true>(h, h->sq_val);
     }
+    if (h->sq_val32) return square_tma_launch_v(h, h->sq_val32);
+    return square_tma_launch_v(h, h->sq_val);
 }
 
 template <bool UPDATE, bool EXACT, int SQ_U, bool HINTS, bool NOATOM = false>
@@ -655,9 +654,9 @@ cualign_status launch_square(cualign_bp *h, bool update)
         KScope ks(h, CUALIGN_K_SQUARE);
         if (update && exact) square_launch<true, true, 2, true>(h);
         else if (update) {
-            static const int var = getenv("CUALIGN_SQ_VARIANT") ? atoi(getenv("CUALIGN_SQ_VARIANT")) : 6;
-            if (var == 6) square_tma_launch(h);
-            else if (var == 8) square_tma_launch_v<double2, true>(h, h->sq_val); // timing probe only: no F sums
+            static const int var = probe_knob("CUALIGN_SQ_VARIANT", 6); // probe build only (5, 8: timing probes)
+            if (var == 6) CA_TRY(square_tma_launch(h));
+            else if (var == 8) CA_TRY((square_tma_launch_v<double2, true>(h, h->sq_val))); // timing probe: no F sums
             else if (var == 0) square_launch<true, false, 1, false>(h);
             else if (var == 1) square_launch<true, false, 1, true>(h);
             else if (var == 2) square_launch<true, false, 2, false>(h);
@@ -878,14 +877,13 @@ cualign_status bp_top2(cualign_bp *h)
         // lanes per tile: CUALIGN_TOP2_TG (measurement knob), else the
         // capturing graph's choice (h->top2_tg), else TG_DEFAULT
         static const int tg_env = [] {
-            const char *v = getenv("CUALIGN_TOP2_TG");
-            const int x = v ? atoi(v) : 0;
+            const int x = probe_knob("CUALIGN_TOP2_TG", 0);
             return (x == 1 || x == 2 || x == 4 || x == 8) ? x : 0;
         }();
         const int tg = tg_env ? tg_env : (h->top2_tg ? h->top2_tg : TG_DEFAULT);
         // CUALIGN_TOP2_GRID (measurement knob): at most this many blocks per SM
         // (grid-stride tiles), leaving SM slots to a concurrent rounding
-        static const int gcap_env = getenv("CUALIGN_TOP2_GRID") ? atoi(getenv("CUALIGN_TOP2_GRID")) : 0;
+        static const int gcap_env = probe_knob("CUALIGN_TOP2_GRID", 0);
         const int gcap = gcap_env > 0 ? gcap_env * h->num_sms : (1 << 30);
         const int64_t nt = T.nA + T.nchunks;
         if (nt > 0) {
@@ -937,7 +935,7 @@ cualign_status bp_front_edge(cualign_bp *h)
         else if (literal) k_edge<EPT, false, true><<<grid, 256, 0, h->stream>>>(R);
         else {
             // measurement knob: 1 = 1 edge per thread, 4 = 4 edges per thread
-            static const int var = getenv("CUALIGN_EDGE_VAR") ? atoi(getenv("CUALIGN_EDGE_VAR")) : 0;
+            static const int var = probe_knob("CUALIGN_EDGE_VAR", 0);
             if (var == 1) k_edge<1, false, false><<<grid_for(ml, 256, 1 << 30), 256, 0, h->stream>>>(R);
             else if (var == 4) k_edge<4, false, false><<<grid_for((ml + 3) / 4, 256, 1 << 30), 256, 0, h->stream>>>(R);
             else CA_CUDA(launch_pdl(k_edge<EPT, false, false>, dim3(grid), dim3(256), 0, h->stream, R));

@@ -648,6 +648,12 @@ cualign_status build_L(cualign_bp *h, LDev &L, const cualign_edges *E, bool devi
                        bool validate, int32_t nA, int32_t nB)
 {
     KScope ks(h, CUALIGN_K_INIT);
+    // edge ids are int32 and the sorts below take an int count: reject an
+    // oversized m before any upload or launch
+    if (E->m >= ((int64_t)1 << 31) - 1) {
+        set_error("m = %lld exceeds int32 edge ids", (long long)E->m);
+        return CUALIGN_EINVAL;
+    }
     L.nA = nA;
     L.nB = nB;
     L.m = E->m;
@@ -753,7 +759,7 @@ static cualign_status build_S_upper(cualign_bp *h, const int64_t *Ap, const int3
     CA_CUDA(cudaMemsetAsync(h->sq_rp, 0, sizeof(int64_t), h->stream));
     h->nsq = 0;
     // group-map build (default) unless the 32-bit candidate counts could overflow
-    static const int sb_env = getenv("CUALIGN_SBUILD_VAR") ? atoi(getenv("CUALIGN_SBUILD_VAR")) : 1;
+    static const int sb_env = probe_knob("CUALIGN_SBUILD_VAR", 1);
     const bool group_map = sb_env == 1 && h->L.nB < (1 << 26);
     const int32_t nA = h->L.nA;
     int sbg_blocks = 1;
@@ -862,11 +868,6 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
     CA_TRY(build_L(h, h->L, E, devp, true, A->n, B->n));
     init_trace(h, "build_L");
     const int64_t m = h->L.m;
-
-    if (m >= ((int64_t)1 << 31) - 1) {
-        set_error("m = %lld exceeds int32 edge ids", (long long)m);
-        return CUALIGN_EINVAL;
-    }
     if (h->world == 1) {
         CA_TRY(build_S_upper(h, Ap, Aj, Bp, Bj));
     } else {
@@ -1049,12 +1050,11 @@ cualign_status build_problem(cualign_bp *h, const cualign_graph *A, const cualig
 }
 
 // Reorder the squares into (e block, f block) tiles (see k_sq_tile_key).
-// S^p is still all zero, so only (e, f) moves.  CUALIGN_SQ_TILE_LOG overrides
-// the block size (0 = keep the (e, f) order; measurement knob).
+// S^p is still all zero, so only (e, f) moves.  cualign_params.square_tile_log
+// overrides the block size (-1 = keep the (e, f) order; result-neutral).
 cualign_status tile_squares(cualign_bp *h)
 {
-    static const int log_env = getenv("CUALIGN_SQ_TILE_LOG") ? atoi(getenv("CUALIGN_SQ_TILE_LOG")) : -1;
-    const int log_b = log_env >= 0 ? log_env : SQ_TILE_LOG;
+    const int log_b = h->tile_log_param < 0 ? 0 : (h->tile_log_param > 0 ? h->tile_log_param : SQ_TILE_LOG);
     h->sq_tile_log = 0;
     if (log_b <= 0 || h->nsq < 2 || h->nsq >= INT32_MAX) return CUALIGN_OK;
     const uint32_t nblocks = (uint32_t)(((h->L.m - 1) >> log_b) + 1);

@@ -15,6 +15,17 @@
 
 namespace cualign {
 
+// ------------------------------------------------------------ probe knobs
+// Measurement variants (timing probes, alternative launch shapes) are read
+// from the environment ONLY in a probe build (-DCUALIGN_PROBES, see
+// build.py --probes; never the product library): some of them skip work and
+// give wrong results.  In the product build probe_knob() is the default.
+#ifdef CUALIGN_PROBES
+int probe_knob(const char *name, int dflt);
+#else
+inline int probe_knob(const char *, int dflt) { return dflt; }
+#endif
+
 // ------------------------------------------------------------------ errors
 void set_error(const char *fmt, ...);
 void clear_error();
@@ -162,6 +173,8 @@ struct cualign_bp {
     // kernels report (round_p; = p_dev except in a pipelined run)
     double *yc_b1 = nullptr, *zc_b1 = nullptr;
     int pipe_mode = -1;                 // step schedule: -1 undecided, 0 forked graph, 1 pipelined, 2 serial
+    int sched_param = 0;                // cualign_params.schedule (0 = library's choice)
+    int tile_log_param = 0;             // cualign_params.square_tile_log (0 = SQ_TILE_LOG, -1 = none)
     int top2_tg = 0;                    // k_top2 lanes per tile while capturing (0: default; pipelined graphs: 1)
     int *rp_dev = nullptr;
     const int *round_p = nullptr;

@@ -345,7 +345,7 @@ cualign_status knn_launch(cualign_bp *h, const uint8_t *Asw, const uint8_t *Bsw,
     const int32_t ntilesB = (n_b + BN - 1) / BN;
     dim3 grid((unsigned)((n_a + KNN_BM - 1) / KNN_BM), (unsigned)nsplit);
     // CUALIGN_KNN_PROBE (timing probes, wrong results): 1 = no epilogue, 2 = no MMA
-    static const int probe = getenv("CUALIGN_KNN_PROBE") ? atoi(getenv("CUALIGN_KNN_PROBE")) : 0;
+    static const int probe = probe_knob("CUALIGN_KNN_PROBE", 0); // probe build only
     fn<<<grid, knn_threads<EH>(), smem, h->stream>>>(Asw, Bsw, n_a, n_b, KB, k, ntilesB, tps, nstages, pv, pi,
                                                      probe);
     CA_CUDA(cudaGetLastError());
@@ -375,7 +375,7 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
         const size_t f = fixed_for(eh) + 1024, bb = (size_t)KB * bn * 128;
         return f >= (size_t)smem_optin ? 0 : (int32_t)std::min<size_t>(4, ((size_t)smem_optin - f) / bb);
     };
-    static const int eh_env = getenv("CUALIGN_KNN_EH") ? atoi(getenv("CUALIGN_KNN_EH")) : 1;
+    static const int eh_env = probe_knob("CUALIGN_KNN_EH", 1);
     const int EH = (eh_env >= 2 && stages_for(2, 128) >= 2) ? 2 : 1;
     const int BN = (EH == 1 && KB <= 2) ? 256 : 128;
     const int32_t nstages = stages_for(EH, BN);

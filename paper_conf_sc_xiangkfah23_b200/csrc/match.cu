@@ -758,7 +758,7 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
                            2 * nT + 1, h->suit, 2 * nP + 1, fromB ? h->mateB : h->mateA));
     }
     const int64_t slots = P.ninst * nP;
-    static const bool dbg_env = getenv("CUALIGN_MATCH_DEBUG") != nullptr;
+    static const bool dbg_env = probe_knob("CUALIGN_MATCH_DEBUG", 0) != 0;
     const bool dbg = dbg_env && !h->capturing;
     unsigned long long *dbuf = nullptr;
     if (dbg) {
@@ -769,7 +769,7 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     if (slots > 0) {
         KScope ks(h, CUALIGN_K_MATCH);
         const int64_t dmax = fromB ? h->max_deg_b : h->max_deg_a;
-        static const int genv = getenv("CUALIGN_SUITOR_G") ? atoi(getenv("CUALIGN_SUITOR_G")) : 0;
+        static const int genv = probe_knob("CUALIGN_SUITOR_G", 0);
         // tile width: G lanes x U edges cover a typical proposer list in one pass
         const int G = genv ? genv : (dmax > 64 ? 32 : (dmax > 24 ? 16 : (dmax > 20 ? 8 : 4)));
         if (G == 32) k_suitor<32, 2><<<grid_for(slots * 32, 128, 1 << 30), 128, 0, h->stream>>>(P);
@@ -782,9 +782,9 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
             // default 12 blocks of 128 (40 registers): 0.142 ms vs 0.175 ms
             // uncapped (66 registers, 8 blocks) on O -- latency-bound, more
             // resident proposer tiles win over a few spilled registers
-            static const int minb = getenv("CUALIGN_SUITOR_MINB") ? atoi(getenv("CUALIGN_SUITOR_MINB")) : 12;
+            static const int minb = probe_knob("CUALIGN_SUITOR_MINB", 12);
             const int grid = grid_for(slots * 4, 128, 1 << 30);
-            static const int pers = getenv("CUALIGN_SUITOR_PERSIST") ? atoi(getenv("CUALIGN_SUITOR_PERSIST")) : 0;
+            static const int pers = probe_knob("CUALIGN_SUITOR_PERSIST", 0);
             if (pers) {
                 int occ = 0;
                 if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_suitor_persistent<4, 5, 12>, 128, 0) !=

@@ -49,3 +49,16 @@ def test_header_documents_every_entry_point():
         idx = re.search(r"(cualign_status|void|const char \*)\s*" + sym + r"\(", text).start()
         assert "*/" in text[max(0, idx - 1500):idx], sym
     assert "PAPER.md" in text
+
+
+def test_product_library_reads_no_environment_knobs():
+    """Measurement knobs (some skip work and give wrong results) exist only in
+    the probe build (-DCUALIGN_PROBES); the product library holds no knob
+    name, so a stray CUALIGN_* variable in a user's shell cannot change a
+    result.  (getenv itself is imported by the static CUDA runtime and NVTX.)"""
+    from paper_conf_sc_xiangkfah23_b200 import build
+    path = build.build()
+    data = open(path, "rb").read()
+    knobs = set(re.findall(rb"CUALIGN_[A-Z0-9_]+", data))
+    # only the flag names quoted in error messages remain
+    assert knobs <= {b"CUALIGN_FLAG_EXACT", b"CUALIGN_FLAG_FP32_S", b"CUALIGN_RUN_ITERATE", b"CUALIGN_RUN_ROUND"}, knobs

@@ -3,17 +3,14 @@
 * Square tiles: the squares are reordered into
   (e block, f block) tiles at init.  Every result is order-independent
   (integer fixed-point F sums, per-square arithmetic), so a run with tiny
-  blocks (many tiles, CUALIGN_SQ_TILE_LOG, read once per process -> a
-  subprocess) must equal the default run bit for bit.
+  blocks (many tiles, cualign_params.square_tile_log) must equal the
+  default run bit for bit.
 * Step pipeline: run(n) overlaps the rounding of
   iteration k with iteration k+1 through double-buffered y^c, z^c; for every
   n (1, even, odd) and interleaved with eager calls the state, the last round
   and the best matching equal the eager sequence bit for bit.
 """
-import json
 import os
-import subprocess
-import sys
 
 import numpy as np
 import pytest
@@ -34,42 +31,28 @@ def ca():
     return ca
 
 
-_CHILD = r"""
-import json, sys, numpy as np
-sys.path.insert(0, sys.argv[1])
-import paper_conf_sc_xiangkfah23_b200 as ca
-from synth import make_config
-inst = make_config("P", scale=0.1)
-with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma) as h:
-    h.run(7)
-    st = h.get_state()
-    rp, col = h.get_S()
-    mate, info = h.get_best()
-    out = {k: np.asarray(st[k]).view(np.uint64).tolist() for k in ("yc", "zc", "yp", "zp", "d", "Sp")}
-    out["S"] = [int(x) for x in np.concatenate([rp, col]).tolist()]
-    out["mate"] = np.asarray(mate).tolist()
-    out["best"] = [info["best_score"], info["best_iter"]]
-print(json.dumps(out))
-"""
-
-
-def _child(tile_log):
-    env = dict(os.environ)
-    if tile_log is not None:
-        env["CUALIGN_SQ_TILE_LOG"] = str(tile_log)
-    r = subprocess.run([sys.executable, "-c", _CHILD, ROOT], capture_output=True, text=True, env=env,
-                       timeout=600)
-    assert r.returncode == 0, r.stderr[-2000:]
-    return json.loads(r.stdout.strip().splitlines()[-1])
+def _run_tiles(ca, tile_log):
+    inst = make_config("P", scale=0.1)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma,
+                      square_tile_log=tile_log) as h:
+        h.run(7)
+        st = h.get_state()
+        rp, col = h.get_S()
+        mate, info = h.get_best()
+        out = {k: np.asarray(st[k]).view(np.uint64) for k in ("yc", "zc", "yp", "zp", "d", "Sp")}
+        out["S"] = np.concatenate([rp, col])
+        out["mate"] = np.asarray(mate)
+        out["best"] = np.asarray([info["best_score"], info["best_iter"]])
+    return out
 
 
 def test_square_tiles_bitwise_invariant(ca):
-    base = _child(0)          # plain (e, f) order
-    tiled = _child(6)         # blocks of 64 edges: hundreds of tiles on P10
-    default = _child(None)    # default block size
+    base = _run_tiles(ca, -1)      # plain (e, f) order
+    tiled = _run_tiles(ca, 6)      # blocks of 64 edges: hundreds of tiles on P10
+    default = _run_tiles(ca, 0)    # default block size
     for k in base:
-        assert base[k] == tiled[k], k
-        assert base[k] == default[k], k
+        assert np.array_equal(base[k], tiled[k]), k
+        assert np.array_equal(base[k], default[k]), k
 
 
 def _eager(ca, inst, n):
@@ -81,11 +64,14 @@ def _eager(ca, inst, n):
     return h, infos
 
 
-@pytest.mark.parametrize("n", [1, 2, 5, 6, 21, 24])  # >= 21: the first run times the schedules
-def test_pipelined_run_equals_eager(ca, n):
+@pytest.mark.parametrize("n,schedule", [(1, 0), (2, 0), (5, 0), (6, 0), (21, 0), (24, 0), (40, 0),
+                                        (7, 1), (7, 2), (7, 3), (40, 1), (40, 2), (40, 3)])
+def test_pipelined_run_equals_eager(ca, n, schedule):
+    """Every step schedule (cualign_params.schedule: 0 = the library's
+    choice, 1 pipelined, 2 serial, 3 forked) for short and long runs."""
     inst = make_config("P", scale=0.1)
     h1, infos = _eager(ca, inst, n)
-    with h1, ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma) as h2:
+    with h1, ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, schedule=schedule) as h2:
         h2.run(n)
         s1, s2 = h1.get_state(), h2.get_state()
         for k in ("yc", "zc", "yp", "zp", "d", "Sp"):
@@ -124,7 +110,7 @@ def test_run_trace_infos_equal_step_by_step(ca, mode):
     inst = make_config("P", scale=0.05)
     flags = ca.FLAG_ROUND_DAMPED if mode == "damped" else 0
     kw = {"world": 3} if mode == "shards3" else {}
-    n = 23  # >= 21: includes the schedule selection steps
+    n = 23
     with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags) as h1, \
             ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags, **kw) as h2:
         eager = []

@@ -165,3 +165,42 @@ def test_Z8_selection_and_best_semantics():
     assert info["source"] == 0 and info["improved"] == 0
     mate, best, it = o.get_best()
     assert best == 0.0 and it == 0 and np.all(mate == -1)
+
+
+@pytest.mark.parametrize("reading", ["undamped", "damped"])
+def test_P16_worked_example_W3_round_source(reading):
+    """Worked example W3 (tests/golden/W3.json, reading Z5): the oracle's
+    rounding uses y^c, z^c (Alg. 2 l.17/19) or, with
+    ROUND_DAMPED, y^p, z^p (text :201).  At p = 2 the four greedy matchings
+    differ and the two readings pick different sources, so swapping y and z
+    or c and p fails here."""
+    import oracle
+    from fractions import Fraction
+    from tests.util import load_golden, golden_instance
+    g = load_golden("W3.json")
+    A, B, L = golden_instance(g)
+    gamma = float(Fraction(g["gamma"]))
+    p2 = g["iterations"][1]
+    assert len({tuple(p2["undamped"]["My"]), tuple(p2["undamped"]["Mz"]),
+                tuple(p2["damped"]["My"]), tuple(p2["damped"]["Mz"])}) == 4
+    assert p2["undamped"]["source"] != p2["damped"]["source"]
+    o = Oracle(A, B, L, g["alpha"], g["beta"], oracle.ROUND_DAMPED if reading == "damped" else 0)
+    for it in g["iterations"]:
+        o.step_gamma(gamma)
+        st = o.get_state()
+        for key in ("d", "yc", "zc", "yp", "zp"):
+            assert list(st[key]) == [float(Fraction(x)) for x in it[key]], (it["p"], key)
+        info = o.round()
+        want = it[reading]
+        assert sorted(e for e in info["mate_y"] if e >= 0) == want["My"], it["p"]
+        assert sorted(e for e in info["mate_z"] if e >= 0) == want["Mz"], it["p"]
+        for k in ("score_y", "score_z", "weight_y", "weight_z", "best_score"):
+            assert info[k] == float(Fraction(want[k])), (it["p"], k)
+        for k in ("overlap_y", "overlap_z", "source", "best_iter"):
+            assert info[k] == want[k], (it["p"], k)
+    mate, best, best_it = o.get_best()
+    last = g["iterations"][-1][reading]
+    assert best == float(Fraction(last["best_score"])) and best_it == last["best_iter"]
+    src = g["iterations"][best_it - 1][reading]
+    want_best = src["My"] if src["source"] == 0 else src["Mz"]
+    assert sorted(e for e in mate if e >= 0) == want_best
