@@ -262,6 +262,27 @@ cualign_status cualign_bp_get_state(cualign_bp *h, double *yc, double *zc, doubl
 cualign_status cualign_bp_set_state(cualign_bp *h, const double *yp, const double *zp,
                                     const double *Sp, int32_t p);
 
+/* The two matchings of the last rounding (Alg. 2 l.17-20):
+ * mate_y[a] / mate_z[a] = canonical id of the L edge matched at A vertex a in
+ * M_y (rounding of y^c, or y^p with CUALIGN_FLAG_ROUND_DAMPED) / M_z, or -1
+ * (host buffers of n_A int32; either may be NULL).  Sharded handles: the
+ * replicated final matchings.  ESTATE before the first rounding.
+ * Synchronises. */
+cualign_status cualign_bp_get_round_mates(cualign_bp *h, int32_t *mate_y, int32_t *mate_z);
+
+/* Sampled S^p (test / diagnostic hook for one-step parity at sizes where the
+ * full S^p does not fit the host): every square {e, f} (e < f, S_ef = S_fe =
+ * 1) with e or f in edges[0..n) (host array of canonical ids),
+ * as e_out[i] = e, f_out[i] = f, v_ef[i] = S^p_ef, v_fe[i] = S^p_fe (host
+ * buffers of cap entries; any may be NULL), in unspecified order.  At most cap
+ * are written; *n_out receives the number of such squares (call again with a
+ * larger cap if it exceeds cap).  Single-GPU and virtual-shard handles (a
+ * process shard holds only its own squares: ESTATE).  EINVAL on an id
+ * outside [0, m).  Synchronises. */
+cualign_status cualign_bp_sample_squares(cualign_bp *h, const int32_t *edges, int64_t n, int64_t cap,
+                                         int32_t *e_out, int32_t *f_out, double *v_ef, double *v_fe,
+                                         int64_t *n_out);
+
 /* Diagnostics; reset = 1 clears counters after reading. Synchronises. */
 cualign_status cualign_bp_get_stats(cualign_bp *h, cualign_stats *stats, int32_t reset);
 

@@ -46,6 +46,24 @@ class SampledProblem:
                     out.append(f)
         return out
 
+    def S_row_vec(self, e):
+        """Row e of S by the same definition, vectorised over the candidate
+        pairs (for hub rows with 10^5-10^8 pairs): f = (j, j') in L with
+        j in N_A(i) and j' in N_B(i'), ascending f (= ascending (j, j'), the
+        canonical order).  Pinned against S_row (tests/test_oracle_sample.py)."""
+        i, ip = int(self.L.a[e]), int(self.L.b[e])
+        A, B = self.A, self.B
+        J = A.col[A.rowptr[i]:A.rowptr[i + 1]].astype(np.int64)
+        NB = B.col[B.rowptr[ip]:B.rowptr[ip + 1]].astype(np.int64)
+        if J.shape[0] == 0 or NB.shape[0] == 0:
+            return []
+        lo, hi = self.arow[J], self.arow[J + 1]
+        cnt = hi - lo
+        f = np.repeat(lo - np.concatenate([[0], np.cumsum(cnt)[:-1]]), cnt) + np.arange(int(cnt.sum()))
+        bf = self.L.b[f].astype(np.int64)
+        hit = np.isin(bf, NB)
+        return sorted(int(x) for x in f[hit])
+
     def othermax(self, edges, e, v, literal):
         others = [float(v[f]) for f in edges if f != e]
         if literal:
@@ -60,10 +78,11 @@ class SampledProblem:
                 om = x
         return om
 
-    def step(self, e, alpha, beta, g, h, yp, zp, sp, literal=False):
-        """Iteration outputs at edge e.  sp(e, f) -> S^p value of nonzero (e, f)."""
+    def step(self, e, alpha, beta, g, h, yp, zp, sp, literal=False, vec=False):
+        """Iteration outputs at edge e.  sp(e, f) -> S^p value of nonzero (e, f).
+        vec: build the S row with S_row_vec (hub rows)."""
         L = self.L
-        row = self.S_row(e)
+        row = self.S_row_vec(e) if vec else self.S_row(e)
         F = []
         t = 0.0
         for f in row:

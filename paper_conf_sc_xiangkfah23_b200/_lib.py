@@ -33,7 +33,8 @@ NUM_KERNEL_CLASSES = 10
 EXPORTED = ["cualign_bp_init", "cualign_bp_iterate", "cualign_bp_round", "cualign_bp_run", "cualign_bp_run_trace",
             "cualign_bp_set_timing", "cualign_bp_get_best",
             "cualign_bp_free", "cualign_bp_get_sizes", "cualign_bp_get_S", "cualign_bp_get_state",
-            "cualign_bp_set_state", "cualign_bp_get_stats", "cualign_match", "cualign_last_error",
+            "cualign_bp_set_state", "cualign_bp_get_stats", "cualign_bp_get_round_mates",
+            "cualign_bp_sample_squares", "cualign_match", "cualign_last_error",
             "cualign_version", "cualign_nccl_unique_id", "cualign_quality_eval", "cualign_knn"]
 
 
@@ -136,6 +137,10 @@ def load_library():
     lib.cualign_bp_get_state.argtypes = [P, P, P, P, P, P, P, P]
     lib.cualign_bp_set_state.restype = I32
     lib.cualign_bp_set_state.argtypes = [P, P, P, P, I32]
+    lib.cualign_bp_get_round_mates.restype = I32
+    lib.cualign_bp_get_round_mates.argtypes = [P, P, P]
+    lib.cualign_bp_sample_squares.restype = I32
+    lib.cualign_bp_sample_squares.argtypes = [P, P, I64, I64, P, P, P, P, P]
     lib.cualign_bp_get_stats.restype = I32
     lib.cualign_bp_get_stats.argtypes = [P, P, I32]
     lib.cualign_match.restype = I32
@@ -332,6 +337,29 @@ class CuAlignBP:
         zp = _as_host(zp, np.float64)
         Sp = _as_host(Sp, np.float64)
         _check(load_library().cualign_bp_set_state(self._h, _ptr(yp), _ptr(zp), _ptr(Sp), int(p)))
+
+    def round_mates(self):
+        """(M_y, M_z) of the last rounding as L edge ids per A vertex (-1 = none)."""
+        my = np.zeros(max(self.n_a, 1), dtype=np.int32)
+        mz = np.zeros(max(self.n_a, 1), dtype=np.int32)
+        _check(load_library().cualign_bp_get_round_mates(self._h, _ptr(my), _ptr(mz)))
+        return my[:self.n_a], mz[:self.n_a]
+
+    def sample_squares(self, edges):
+        """Every square {e < f} touching the given edge ids: dict with arrays
+        e, f, v_ef = S^p_ef, v_fe = S^p_fe (cualign_bp_sample_squares)."""
+        ed = _as_host(edges, np.int32)
+        cnt = ctypes.c_int64()
+        cap = 0
+        while True:
+            out = {"e": np.zeros(max(cap, 1), np.int32), "f": np.zeros(max(cap, 1), np.int32),
+                   "v_ef": np.zeros(max(cap, 1)), "v_fe": np.zeros(max(cap, 1))}
+            _check(load_library().cualign_bp_sample_squares(self._h, _ptr(ed), int(ed.shape[0]), int(cap),
+                                                            _ptr(out["e"]), _ptr(out["f"]), _ptr(out["v_ef"]),
+                                                            _ptr(out["v_fe"]), ctypes.byref(cnt)))
+            if cnt.value <= cap:
+                return {k: v[:cnt.value] for k, v in out.items()}
+            cap = int(cnt.value)
 
     def stats(self, reset=False):
         st = Stats_t()

@@ -598,6 +598,9 @@ static cualign_status alloc_state(cualign_bp *h)
 // the handle that holds the replicated rounding state (shard 0 of a group)
 static cualign_bp *primary(cualign_bp *h) { return h->vshards.empty() ? h : h->vshards[0]; }
 
+// device array [2][n_A] of the last rounding's M_y, M_z
+static const int32_t *round_mates(cualign_bp *h) { return h->mateA; }
+
 #define API_ENTER() clear_error()
 #define CHECK_H()                                   \
     do {                                            \
@@ -1071,6 +1074,52 @@ cualign_status cualign_bp_set_state(cualign_bp *h, const double *yp, const doubl
     CA_TRY(bp_fsum(h));
     CA_TRY(bp_top2(h)); // othermax inputs of the next iteration from the injected y^p, z^p
     CA_CUDA(cudaStreamSynchronize(h->stream));
+    return CUALIGN_OK;
+}
+
+cualign_status cualign_bp_get_round_mates(cualign_bp *h, int32_t *mate_y, int32_t *mate_z)
+{
+    API_ENTER();
+    CHECK_H();
+    cualign_bp *q = primary(h);
+    if (!h->have_info && !q->have_info) {
+        set_error("get_round_mates: no rounding has run on this handle");
+        return CUALIGN_ESTATE;
+    }
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    CA_CUDA(cudaStreamSynchronize(q->stream));
+    const size_t nb = sizeof(int32_t) * (size_t)q->L.nA;
+    const int32_t *src = round_mates(q);
+    if (nb && mate_y) CA_CUDA(cudaMemcpy(mate_y, src, nb, cudaMemcpyDeviceToHost));
+    if (nb && mate_z) CA_CUDA(cudaMemcpy(mate_z, src + q->L.nA, nb, cudaMemcpyDeviceToHost));
+    return CUALIGN_OK;
+}
+
+cualign_status cualign_bp_sample_squares(cualign_bp *h, const int32_t *edges, int64_t n, int64_t cap,
+                                         int32_t *e_out, int32_t *f_out, double *v_ef, double *v_fe,
+                                         int64_t *n_out)
+{
+    API_ENTER();
+    CHECK_H();
+    if (!n_out || n < 0 || (n > 0 && !edges)) {
+        set_error("sample_squares: NULL n_out / edges or n < 0");
+        return CUALIGN_EINVAL;
+    }
+    if (h->world > 1 && h->vshards.empty()) {
+        set_error("sample_squares: a process shard holds only its own squares");
+        return CUALIGN_ESTATE;
+    }
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    std::vector<cualign_bp *> S = h->vshards.empty() ? std::vector<cualign_bp *>{h} : h->vshards;
+    int64_t total = 0;
+    for (cualign_bp *s : S) {
+        int64_t k = 0;
+        const int64_t off = total < cap ? total : cap;
+        CA_TRY(bp_sample_squares(s, edges, n, cap - off, e_out ? e_out + off : nullptr, f_out ? f_out + off : nullptr,
+                                 v_ef ? v_ef + off : nullptr, v_fe ? v_fe + off : nullptr, &k));
+        total += k;
+    }
+    *n_out = total;
     return CUALIGN_OK;
 }
 

@@ -970,6 +970,81 @@ cualign_status bp_iterate(cualign_bp *h, int32_t n)
     return CUALIGN_OK;
 }
 
+namespace {
+// every square {e < f} with e or f marked: (e, f, S^p_ef, S^p_fe), appended
+// at an atomic cursor (order unspecified; at most cap written, all counted)
+template <class V>
+__global__ void k_sample_squares(int64_t nsq, const int2 *__restrict__ sq_ef, const V *__restrict__ sq_val,
+                                 const unsigned char *__restrict__ mark, int64_t cap,
+                                 unsigned long long *__restrict__ cnt, int2 *__restrict__ out_ef,
+                                 double2 *__restrict__ out_v)
+{
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq;
+         q += (int64_t)gridDim.x * blockDim.x) {
+        const int2 ef = sq_ef[q];
+        if (!(mark[ef.x] | mark[ef.y])) continue;
+        const unsigned long long k = atomicAdd(cnt, 1ull);
+        if ((int64_t)k < cap) {
+            out_ef[k] = ef;
+            out_v[k] = load_pair<false>(sq_val + q);
+        }
+    }
+}
+} // namespace
+
+cualign_status bp_sample_squares(cualign_bp *h, const int32_t *edges, int64_t n, int64_t cap, int32_t *e_out,
+                                 int32_t *f_out, double *v_ef, double *v_fe, int64_t *n_out)
+{
+    const int64_t m = h->L.m;
+    std::vector<unsigned char> mk((size_t)(m ? m : 1), 0);
+    for (int64_t i = 0; i < n; i++) {
+        if (edges[i] < 0 || edges[i] >= m) {
+            set_error("sample_squares: edge id %d outside [0, %lld)", edges[i], (long long)m);
+            return CUALIGN_EINVAL;
+        }
+        mk[(size_t)edges[i]] = 1;
+    }
+    TmpBuf mb, cb, eb, vb;
+    const int64_t c = cap > 0 ? cap : 0;
+    CA_CUDA(tmalloc(h, mb, mk.size()));
+    CA_CUDA(tmalloc(h, cb, sizeof(unsigned long long)));
+    CA_CUDA(tmalloc(h, eb, sizeof(int2) * (size_t)(c ? c : 1)));
+    CA_CUDA(tmalloc(h, vb, sizeof(double2) * (size_t)(c ? c : 1)));
+    CA_CUDA(cudaMemcpyAsync(mb.p, mk.data(), mk.size(), cudaMemcpyHostToDevice, h->stream));
+    CA_CUDA(cudaMemsetAsync(cb.p, 0, sizeof(unsigned long long), h->stream));
+    if (h->nsq > 0) {
+        KScope ks(h, CUALIGN_K_STATE);
+        const int grid = grid_for(h->nsq, 256, h->num_sms * 8);
+        if (h->sq_val32)
+            k_sample_squares<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->sq_val32, (const unsigned char *)mb.p,
+                                                          c, (unsigned long long *)cb.p, (int2 *)eb.p,
+                                                          (double2 *)vb.p);
+        else
+            k_sample_squares<<<grid, 256, 0, h->stream>>>(h->nsq, h->sq_ef, h->sq_val, (const unsigned char *)mb.p,
+                                                          c, (unsigned long long *)cb.p, (int2 *)eb.p,
+                                                          (double2 *)vb.p);
+        CA_CUDA(cudaGetLastError());
+    }
+    unsigned long long total = 0;
+    CA_CUDA(cudaMemcpyAsync(&total, cb.p, sizeof(total), cudaMemcpyDeviceToHost, h->stream));
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    const int64_t k = (int64_t)total < c ? (int64_t)total : c;
+    if (k > 0) {
+        std::vector<int2> ef((size_t)k);
+        std::vector<double2> v((size_t)k);
+        CA_CUDA(cudaMemcpy(ef.data(), eb.p, sizeof(int2) * (size_t)k, cudaMemcpyDeviceToHost));
+        CA_CUDA(cudaMemcpy(v.data(), vb.p, sizeof(double2) * (size_t)k, cudaMemcpyDeviceToHost));
+        for (int64_t i = 0; i < k; i++) {
+            if (e_out) e_out[i] = ef[(size_t)i].x;
+            if (f_out) f_out[i] = ef[(size_t)i].y;
+            if (v_ef) v_ef[i] = v[(size_t)i].x;
+            if (v_fe) v_fe[i] = v[(size_t)i].y;
+        }
+    }
+    *n_out = (int64_t)total;
+    return CUALIGN_OK;
+}
+
 cualign_status bp_scatter_Sp(cualign_bp *h, double *Sfull_dev)
 {
     CA_TRY(ensure_sq_pos(h));

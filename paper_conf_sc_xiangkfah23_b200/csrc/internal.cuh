@@ -356,6 +356,8 @@ cualign_status shard_round(cualign_bp *h);
 cualign_status nccl_init_comm(cualign_bp *h, const void *unique_id);
 void nccl_free_comm(cualign_bp *h);
 cualign_status nccl_unique_id(void *out, int32_t len);
+cualign_status bp_sample_squares(cualign_bp *h, const int32_t *edges, int64_t n, int64_t cap, int32_t *e_out,
+                                 int32_t *f_out, double *v_ef, double *v_fe, int64_t *n_out);
 cualign_status bp_scatter_Sp(cualign_bp *h, double *Sfull_dev);        // squares -> CSR
 cualign_status bp_gather_Sp(cualign_bp *h, const double *Sfull_dev);   // CSR -> squares
 

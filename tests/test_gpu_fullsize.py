@@ -106,3 +106,87 @@ def test_full_O_matching_and_round(full_O):
     assert r["overlap_y"] == overlap
     weight = float(np.sum(inst.L.w[want[sel]]))
     assert abs(r["weight_y"] - weight) <= 1e-12 * weight
+
+
+# ------------------------------------------------ configs S and R, one step
+# SURVEY §8(c) parity contract: one-step parity (bound 1e-12 of the vector's
+# max norm) on O, S and R.  S^p of these instances (10^9 nonzeros) does not
+# fit a host round trip, so the GPU's OWN state after 5 graph steps is the
+# input: y^p, z^p in full (get_state) and S^p on the squares touching a
+# sample of edges (cualign_bp_sample_squares); one more iteration of the
+# bench's graph step; every output at the sampled edges (d, y^c, z^c, y^p,
+# z^p and the whole new S^p row) against oracle/sample.py.  The sample holds
+# random edges, the edges with the largest deg_A(a) deg_B(b) (longest rows),
+# and edges of the highest-degree A and B vertices (R-MAT hub rows / columns).
+ONE_STEP_TOL = 1e-12
+
+
+def _sample_edges(inst, n_rand=150, seed=21):
+    L, A, B = inst.L, inst.A, inst.B
+    rng = np.random.default_rng(seed)
+    dA, dB = np.diff(A.rowptr), np.diff(B.rowptr)
+    prod = dA[L.a].astype(np.float64) * dB[L.b]
+    long_rows = np.argsort(prod)[-20:]
+    a_hub = int(np.argmax(np.bincount(L.a, minlength=L.n_a) * (dA > 0) + dA))  # A hub with candidates
+    arow = np.searchsorted(L.a, [a_hub, a_hub + 1])
+    hub_row = np.arange(arow[0], min(arow[1], arow[0] + 10))
+    b_hub = int(np.argmax(dB))
+    hub_col = np.nonzero(L.b == b_hub)[0][:10]
+    s = np.concatenate([rng.choice(L.m, n_rand, replace=False), long_rows, hub_row, hub_col, [0, L.m - 1]])
+    return np.unique(s.astype(np.int64))
+
+
+def _one_step_large(name, **kw):
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_sc_xiangkfah23_b200 as ca
+    ca.load_library()
+    inst = make_config(name, **kw)
+    stream = torch.cuda.Stream()
+    sample = _sample_edges(inst)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, stream=stream) as h:
+        h.run(5)
+        pre = h.get_state(with_S=False)
+        sq0 = h.sample_squares(sample)
+        h.run(1, with_round=False)
+        post = h.get_state(with_S=False)
+        sq1 = h.sample_squares(sample)
+    assert (pre["p"], post["p"]) == (5, 6)
+    val0, val1 = {}, {}
+    for sq, val in ((sq0, val0), (sq1, val1)):
+        for e, f, vef, vfe in zip(sq["e"], sq["f"], sq["v_ef"], sq["v_fe"]):
+            val[(int(e), int(f))] = float(vef)
+            val[(int(f), int(e))] = float(vfe)
+    g = gamma_power(inst.gamma, 6)
+    sp = SampledProblem(inst.A, inst.B, inst.L)
+    scale = {k: max(float(np.max(np.abs(post[k]))), 1.0) for k in ("d", "yc", "zc", "yp", "zp")}
+    sp_scale = max(max((abs(v) for v in val1.values()), default=0.0), 1.0)
+    worst = 0.0
+    for e in sample:
+        e = int(e)
+        r = sp.step(e, inst.alpha, inst.beta, g, 1.0 - g, pre["yp"], pre["zp"], lambda a, b: val0[(a, b)], vec=True)
+        # structure: the squares touching e are exactly the S row by definition
+        assert sorted(f for (a, f) in val1 if a == e) == r["row"], e
+        for k in ("d", "yc", "zc", "yp", "zp"):
+            err = abs(post[k][e] - r[k]) / scale[k]
+            worst = max(worst, err)
+            assert err <= ONE_STEP_TOL, (name, e, k, post[k][e], r[k])
+        for f, want in zip(r["row"], r["Sp"]):
+            err = abs(val1[(e, f)] - want) / sp_scale
+            worst = max(worst, err)
+            assert err <= ONE_STEP_TOL, (name, e, f, val1[(e, f)], want)
+    return worst, len(sample)
+
+
+@pytest.mark.slow
+def test_config_S_one_step_sampled():
+    worst, n = _one_step_large("S")
+    assert n >= 150
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("k", [5, 50])
+def test_config_R_one_step_sampled(k):
+    worst, n = _one_step_large("R", k=k)
+    assert n >= 150

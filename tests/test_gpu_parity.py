@@ -50,6 +50,7 @@ def assert_state_equal(g, o, keys=("d", "yc", "zc", "yp", "zp", "Sp"), where="")
 
 INSTANCES = {
     "T": lambda: make_config("T"),
+    "P": lambda: make_config("P"),
     "P10": lambda: make_config("P", scale=0.1),
     "O005": lambda: make_config("O", scale=0.005),
 }
@@ -163,8 +164,10 @@ def _run_both(ca, inst, n_iter, flags=0, gamma=None, alpha=None, beta=None, chec
     return o, h
 
 
-@pytest.mark.parametrize("name,n_iter", [("T", 20), ("P10", 30), ("O005", 10)])
+@pytest.mark.parametrize("name,n_iter", [("T", 20), ("P10", 30), ("O005", 10), ("P", 100)])
 def test_fast_mode_trajectory_within_1e9(ca, name, n_iter):
+    """Every iteration within 1e-9 of the oracle (SURVEY §8(c) parity
+    contract), T and P at BASELINE.json's full size and iteration count."""
     inst = INSTANCES[name]()
 
     def check(p, g, o, *_):
@@ -332,11 +335,64 @@ def test_round_matches_oracle(ca, name, n_iter):
             my, cy = o.greedy(g["yc"])
             mz, cz = o.greedy(g["zc"])
             ey, ez = o.evaluate(my), o.evaluate(mz)
+            gy, gz = h.round_mates()
+            assert np.array_equal(gy, my) and np.array_equal(gz, mz), p
             assert r["card_y"] == cy and r["card_z"] == cz
             assert r["overlap_y"] == ey["overlap"] and r["overlap_z"] == ez["overlap"]
             assert abs(r["weight_y"] - ey["weight"]) <= 1e-12 * max(1, ey["weight"])
             assert abs(r["score_z"] - ez["score"]) <= 1e-12 * max(1, ez["score"])
             assert r["iter"] == p
+
+
+@pytest.mark.parametrize("name,n_iter", [("T", 20), ("P10", 20)])
+def test_round_damped_matches_oracle(ca, name, n_iter):
+    """Reading Z5 variant (CUALIGN_FLAG_ROUND_DAMPED): the
+    rounding takes y^p, z^p.  On the GPU's own messages, every round's M_y,
+    M_z equal the oracle's greedy matchings of y^p, z^p bit for bit, and the
+    round info equals the oracle's evaluation of them."""
+    inst = INSTANCES[name]()
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta, oracle.ROUND_DAMPED)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, ca.FLAG_ROUND_DAMPED) as h:
+        for p in range(1, n_iter + 1):
+            h.iterate(1)
+            r = h.round()
+            g = h.get_state(with_S=False)
+            my, cy = o.greedy(g["yp"])
+            mz, cz = o.greedy(g["zp"])
+            gy, gz = h.round_mates()
+            assert np.array_equal(gy, my) and np.array_equal(gz, mz), p
+            ey, ez = o.evaluate(my), o.evaluate(mz)
+            assert r["card_y"] == cy and r["card_z"] == cz
+            assert r["overlap_y"] == ey["overlap"] and r["overlap_z"] == ez["overlap"]
+            assert abs(r["score_y"] - ey["score"]) <= 1e-12 * max(1, ey["score"])
+            assert abs(r["score_z"] - ez["score"]) <= 1e-12 * max(1, ez["score"])
+            assert r["source"] == (0 if r["score_y"] >= r["score_z"] else 1)
+
+
+@pytest.mark.parametrize("reading", ["undamped", "damped"])
+def test_W3_on_gpu(ca, reading):
+    """Worked example W3 (tests/golden/W3.json): exact dyadic values, so the
+    GPU's messages, matchings, scores and best equal the golden bit for bit
+    under both readings of Z5."""
+    from fractions import Fraction
+    g = load_golden("W3.json")
+    A, B, L = golden_instance(g)
+    flags = ca.FLAG_ROUND_DAMPED if reading == "damped" else 0
+    with ca.CuAlignBP(A, B, L, g["alpha"], g["beta"], float(Fraction(g["gamma"])), flags) as h:
+        for it in g["iterations"]:
+            h.iterate(1)
+            st = h.get_state()
+            for key in ("d", "yc", "zc", "yp", "zp"):
+                assert list(st[key]) == [float(Fraction(x)) for x in it[key]], (it["p"], key)
+            r = h.round()
+            want = it[reading]
+            gy, gz = h.round_mates()
+            assert sorted(e for e in gy if e >= 0) == want["My"], it["p"]
+            assert sorted(e for e in gz if e >= 0) == want["Mz"], it["p"]
+            for k in ("score_y", "score_z", "weight_y", "weight_z", "best_score"):
+                assert r[k] == float(Fraction(want[k])), (it["p"], k)
+            for k in ("overlap_y", "overlap_z", "source", "best_iter"):
+                assert r[k] == want[k], (it["p"], k)
 
 
 @pytest.mark.parametrize("name", ["T", "P10"])

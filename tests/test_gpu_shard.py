@@ -121,6 +121,34 @@ def test_sharded_rounding_merge_rounds(ca, world):
         assert np.array_equal(h1.get_best()[0], hs.get_best()[0])
 
 
+@pytest.mark.parametrize("world", [2, 5])
+@pytest.mark.parametrize("damped", [False, True])
+def test_sharded_round_mates_equal_oracle_greedy(ca, world, damped):
+    """NEXT-1 against the oracle directly: every round's sharded M_y and M_z
+    (the replicated result of the merge rounds) equal the oracle's greedy
+    matching (readings Z6/Z7) of the y^c, z^c (y^p, z^p
+    under ROUND_DAMPED, reading Z5) gathered from the shards, and the round's
+    cardinalities / overlaps equal the oracle's evaluation of them."""
+    from oracle import LightOracle
+    inst = make_config("O", scale=0.02)
+    flags = ca.FLAG_ROUND_DAMPED if damped else 0
+    lo = LightOracle(inst.L)
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags, world=world) as hs:
+        for p in range(1, 6):
+            hs.iterate(1)
+            r = hs.round()
+            st = hs.get_state(with_S=False)
+            my, mz = hs.round_mates()
+            wy, cy = lo.greedy(st["yp" if damped else "yc"])
+            wz, cz = lo.greedy(st["zp" if damped else "zc"])
+            assert np.array_equal(my, wy), (p, "M_y")
+            assert np.array_equal(mz, wz), (p, "M_z")
+            assert r["card_y"] == cy and r["card_z"] == cz
+            ey, ez = o.evaluate(wy), o.evaluate(wz)
+            assert r["overlap_y"] == ey["overlap"] and r["overlap_z"] == ez["overlap"], p
+
+
 def test_exchange_accounting_virtual_shards(ca):
     """Bytes the shards receive per iteration: the B-side
     top-2 all-gather, (w-1)·n_B·16 per shard, plus the square-pass halo (u_f

@@ -48,3 +48,17 @@ def test_sp_value_is_a_function_of_the_pair():
     assert v[0] == v[2] and v[0] != v[1]
     assert np.all(v >= -4.0) and np.all(v < 2.0)
     assert sp_value(e, f, seed=4)[0] != v[0]
+
+
+@pytest.mark.parametrize("name,scale", [("T", 1.0), ("O", 0.002), ("R", 1 / 256)])
+def test_vectorised_S_row_equals_definition_loops(name, scale):
+    inst = make_config(name, scale=scale, **({"k": 20} if name == "R" else {}))
+    sp = SampledProblem(inst.A, inst.B, inst.L)
+    o = Oracle(inst.A, inst.B, inst.L, 1.0, 2.0)
+    rowptr, col, _ = o.get_S()
+    rng = np.random.default_rng(3)
+    deg = np.diff(inst.A.rowptr)[inst.L.a] * np.diff(inst.B.rowptr)[inst.L.b]
+    sample = np.concatenate([rng.choice(inst.L.m, 80, replace=False), np.argsort(deg)[-10:]])
+    for e in sample:
+        want = list(col[rowptr[e]:rowptr[e + 1]])
+        assert sp.S_row_vec(int(e)) == want == sp.S_row(int(e)), e

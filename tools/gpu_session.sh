@@ -1,0 +1,31 @@
+#!/bin/bash
+# One gpurun session: GPU test suite, probe-build diagnostics, bench.
+#   gpurun --timeout 2400 -- 'bash tools/gpu_session.sh <tag> [what...]'
+# what: tests | suitor | parts | bench | ncu_<kernel-regex>   (default: tests parts bench)
+TAG=${1:-run}; shift
+WHAT=${@:-tests parts bench}
+OUT=gpurun_out/$TAG
+mkdir -p $OUT
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > $OUT/gpu.txt 2>&1
+lscpu | grep -E "Model name|^CPU\(s\)" > $OUT/host.txt 2>&1; free -g >> $OUT/host.txt 2>&1
+PROBES=$PWD/paper_conf_sc_xiangkfah23_b200/lib/libcualign_bp_probes.so
+for w in $WHAT; do
+  case $w in
+    tests)
+      timeout 1500 python -m pytest tests -m gpu -q -p no:cacheprovider --durations=15 > $OUT/pytest.txt 2>&1
+      echo "pytest rc=$?"; tail -25 $OUT/pytest.txt ;;
+    suitor)
+      CUALIGN_LIB=$PROBES CUALIGN_MATCH_DEBUG=1 timeout 300 python tools/probe_suitor.py > $OUT/suitor.txt 2>&1
+      echo "suitor rc=$?"; tail -20 $OUT/suitor.txt ;;
+    parts)
+      timeout 300 python tools/bench_parts.py --pre 80 --n 50 > $OUT/parts.json 2> $OUT/parts.err
+      echo "parts rc=$?"; cat $OUT/parts.json ;;
+    bench)
+      timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err
+      echo "bench rc=$?"; cut -c1-1500 $OUT/bench.json ;;
+    ncu_*)
+      K=${w#ncu_}
+      timeout 900 ncu --set full --import-source on --clock-control none -k regex:$K -s 40 -c 1 -o $OUT/ncu_$K -f python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn > $OUT/ncu_$K.log 2>&1
+      echo "ncu $K rc=$?"; tail -3 $OUT/ncu_$K.log ;;
+  esac
+done
