@@ -598,8 +598,15 @@ static cualign_status alloc_state(cualign_bp *h)
 // the handle that holds the replicated rounding state (shard 0 of a group)
 static cualign_bp *primary(cualign_bp *h) { return h->vshards.empty() ? h : h->vshards[0]; }
 
-// device array [2][n_A] of the last rounding's M_y, M_z
-static const int32_t *round_mates(cualign_bp *h) { return h->mateA; }
+// device array [2][n_A] of the last rounding's M_y, M_z (its RoundDev slot)
+static cualign_status round_mates(cualign_bp *h, const int32_t **out)
+{
+    int slot = 0;
+    CA_CUDA(cudaMemcpyAsync(&slot, &h->rd->last_slot, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    *out = h->mates + (int64_t)slot * 2 * h->L.nA;
+    return CUALIGN_OK;
+}
 
 #define API_ENTER() clear_error()
 #define CHECK_H()                                   \
@@ -899,12 +906,17 @@ cualign_status cualign_bp_get_best(cualign_bp *h, int32_t *mate_a, cualign_round
     API_ENTER();
     CHECK_H();
     h = primary(h); // rounding is replicated on every shard
-    if (mate_a && h->L.nA)
-        CA_CUDA(cudaMemcpyAsync(mate_a, h->best_mate, sizeof(int32_t) * (size_t)h->L.nA, cudaMemcpyDeviceToHost,
-                                h->stream));
     RoundDev r;
     CA_CUDA(cudaMemcpyAsync(&r, h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->stream));
     CA_CUDA(cudaStreamSynchronize(h->stream));
+    if (mate_a && h->L.nA) {
+        // bestM lives in its round's mate slot (RoundDev); empty until a score > 0
+        if (r.best_iter > 0)
+            CA_CUDA(cudaMemcpy(mate_a, h->mates + ((int64_t)r.best_slot * 2 + r.best_source) * h->L.nA,
+                               sizeof(int32_t) * (size_t)h->L.nA, cudaMemcpyDeviceToHost));
+        else
+            for (int32_t a = 0; a < h->L.nA; a++) mate_a[a] = -1;
+    }
     if (info) {
         *info = r.info;
         info->best_score = r.best_score;
@@ -1089,7 +1101,8 @@ cualign_status cualign_bp_get_round_mates(cualign_bp *h, int32_t *mate_y, int32_
     CA_CUDA(cudaStreamSynchronize(h->stream));
     CA_CUDA(cudaStreamSynchronize(q->stream));
     const size_t nb = sizeof(int32_t) * (size_t)q->L.nA;
-    const int32_t *src = round_mates(q);
+    const int32_t *src = nullptr;
+    CA_TRY(round_mates(q, &src));
     if (nb && mate_y) CA_CUDA(cudaMemcpy(mate_y, src, nb, cudaMemcpyDeviceToHost));
     if (nb && mate_z) CA_CUDA(cudaMemcpy(mate_z, src + q->L.nA, nb, cudaMemcpyDeviceToHost));
     return CUALIGN_OK;
@@ -1219,9 +1232,14 @@ cualign_status cualign_match(const cualign_edges *L, int32_t n_a, int32_t n_b, c
         }
     }
     if (st == CUALIGN_OK) st = match_standalone(h, xd, rounds_out);
+    int ws = 0;
+    if (st == CUALIGN_OK && (cudaMemcpyAsync(&ws, &h->rd->wslot, sizeof(int), cudaMemcpyDeviceToHost, h->stream) !=
+                                 cudaSuccess ||
+                             cudaStreamSynchronize(h->stream) != cudaSuccess))
+        st = CUALIGN_ECUDA;
     if (st == CUALIGN_OK && mate_a && n_a)
-        if (cudaMemcpyAsync(mate_a, h->mateA, sizeof(int32_t) * (size_t)n_a, cudaMemcpyDeviceToHost, h->stream) !=
-            cudaSuccess)
+        if (cudaMemcpyAsync(mate_a, h->mates + (int64_t)ws * 2 * n_a, sizeof(int32_t) * (size_t)n_a,
+                            cudaMemcpyDeviceToHost, h->stream) != cudaSuccess)
             st = CUALIGN_ECUDA;
     if (st == CUALIGN_OK && mate_b && n_b)
         if (cudaMemcpyAsync(mate_b, h->mateB, sizeof(int32_t) * (size_t)n_b, cudaMemcpyDeviceToHost, h->stream) !=

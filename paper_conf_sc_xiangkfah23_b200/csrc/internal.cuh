@@ -62,6 +62,10 @@ struct LDev {
 };
 
 // Device-side round bookkeeping (persistent across rounds: best).
+// Mate arrays live in two slots of [2 instances][n_A] (cualign_bp::mates):
+// a rounding writes slot wslot; if it improves the best, that slot becomes
+// best_slot and the next rounding writes the other one -- the best matching is
+// never copied (Alg. 2 l.22-24 keep bestM by reference).
 struct RoundDev {
     unsigned int flag[2][2];      // [round parity][instance]: a match happened
     int rounds[2];
@@ -73,6 +77,9 @@ struct RoundDev {
     int improved;
     int source;
     unsigned int done;            // k_eval blocks finished (last-block final reduction)
+    int best_slot, best_source;   // where bestM lives: mates[best_slot][best_source] (valid if best_iter > 0)
+    int wslot;                    // slot the next rounding writes (= 1 - best_slot)
+    int last_slot;                // slot the last rounding wrote
     cualign_round_info info;
 };
 
@@ -180,14 +187,14 @@ struct cualign_bp {
     const int *round_p = nullptr;
 
     // matching (two instances: y and z)
-    int32_t *candA = nullptr, *candB = nullptr, *mateA = nullptr, *mateB = nullptr;
-    int32_t *mvA = nullptr; // 2 instances x n_A: M(i) as a B vertex (-1: unmatched), for evaluate
+    int32_t *candA = nullptr, *candB = nullptr, *mateB = nullptr;
+    int32_t *mates = nullptr; // [2 slots][2 instances][n_A]: matched edge per A vertex (RoundDev slots)
+    int2 *mvA = nullptr;      // n_A: (M_y(i), M_z(i)) as B vertices (-1: unmatched), for evaluate
     unsigned long long *suit = nullptr; // Suitor slots, 2 instances x max(nA, nB)
     // sharded rounding (NEXT-1): replicated global suitors per (instance, B vertex)
     unsigned long long *dist_gx = nullptr, *dist_wxl = nullptr, *dist_wxg = nullptr, *dist_cnt = nullptr;
     int32_t *dist_gi = nullptr, *dist_wid = nullptr, *dist_hold = nullptr, *dist_act = nullptr;
     int dist_rounds = 0; // merge rounds of the last sharded rounding
-    int32_t *best_mate = nullptr;
     double *partial_w = nullptr;
     int match_grid = 0, match_block = 256, eval_grid = 1;
     unsigned long long *match_work = nullptr; // proposals (suitor) or rounds, per instance

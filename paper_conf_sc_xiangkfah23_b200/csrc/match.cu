@@ -47,7 +47,11 @@ struct MatchParams {
     int32_t *candA, *candB; // POINTER ROUNDS: candidate pointers
     unsigned long long *suit; // SUITOR: suitor slots of the targets (packed, see suitor_key)
     int propose_from_b;     // SUITOR: proposing side
-    int32_t *mateA, *mateB;
+    int32_t *mates;         // [2 slots][2 instances][nA]; the round writes slot *wslot (RoundDev)
+    const int *wslot;
+    int32_t *mateA;         // device-side: mates + *wslot * 2 nA (set in the kernels)
+    int32_t *mateB;         // [ninst][nB] (transient)
+    int2 *mvA;              // (M_y(i), M_z(i)) as B vertices, for evaluate
     RoundDev *rd;
     unsigned long long *work; // proposals (suitor) / rounds, spread counters
     unsigned long long *dbg;  // optional diagnostics (CUALIGN_MATCH_DEBUG)
@@ -68,6 +72,18 @@ __device__ __forceinline__ bool better(double xa, int ea, double xb, int eb)
 }
 
 __device__ __forceinline__ const double *xk(const MatchParams &P, int k) { return k ? P.x1 : P.x0; }
+
+// this round's mate slot (RoundDev: never the slot that holds bestM)
+__device__ __forceinline__ int32_t *slot_mates(const MatchParams &P)
+{
+    return P.mates + (int64_t)(*(volatile const int *)P.wslot) * 2 * P.nA;
+}
+
+__device__ __forceinline__ void set_mv(int2 *mvA, int64_t a, int k, int b)
+{
+    int *p = reinterpret_cast<int *>(mvA + a);
+    p[k] = b;
+}
 
 // ------------------------------------------------------------------ Suitor
 // One-sided proposals.  In a bipartite graph whose preferences come from ONE
@@ -135,9 +151,12 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
     bool filter = false;
     while (true) {
         scans++;
-        // heaviest eligible neighbour of `cur` whose suitor is lighter
-        int best = -1;
+        // heaviest eligible neighbour of `cur` whose suitor is lighter; its
+        // target and the slot value seen (the CAS's expected value: 0 on the
+        // unfiltered first scan -- optimistic, a free slot takes one atomic)
+        int best = -1, bt = -1;
         double bx = 0.0;
+        unsigned long long bs = 0ull;
         const int hi = (int)rp[cur + 1]; // positions < m < 2^31: 32-bit index math
         for (int j0 = (int)rp[cur] + lane; j0 < hi; j0 += G * U) {
             int ee[U], tt[U];
@@ -165,6 +184,8 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
                 if (better(xx[u], ee[u], bx, best)) {
                     best = ee[u];
                     bx = xx[u];
+                    bt = tt[u];
+                    bs = filter ? ss[u] : 0ull;
                 }
             }
         }
@@ -173,20 +194,37 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
         for (int off = G / 2; off >= 1; off >>= 1) {
             const double ox = tile.shfl_xor(bx, off);
             const int oe = tile.shfl_xor(best, off);
+            const int ot = tile.shfl_xor(bt, off);
+            const unsigned long long os = tile.shfl_xor(bs, off);
             if (oe >= 0 && better(ox, oe, bx, best)) {
                 bx = ox;
                 best = oe;
+                bt = ot;
+                bs = os;
             }
         }
-        if (best < 0) break; // tile-uniform after the all-reduce
+        if (best < 0) {      // tile-uniform after the all-reduce
+            // exhausted: `cur` stays unmatched (nobody proposes to a
+            // proposer), so this is its only mate write this round -- the
+            // matched ones are written from the target slots by k_collect
+            if (!DIST && lane == 0) {
+                if (fromB) {
+                    P.mateB[k * nP + cur] = -1;
+                } else {
+                    slot_mates(P)[k * nP + cur] = -1;
+                    set_mv(P.mvA, cur, k, -1);
+                }
+            }
+            break;
+        }
         int code = 0;        // 0 rescan, 1 done, 2 displaced
         int next = cur;
         if (lane == 0) {
-            const int tb = __ldg(tgt + best);
+            const int tb = bt;
             unsigned long long *slotp = sT + tb;
             const uint32_t kb = suitor_key(bx);
             const unsigned long long mine = ((unsigned long long)kb << 32) | (uint32_t)best;
-            unsigned long long s = *(volatile unsigned long long *)slotp;
+            unsigned long long s = bs;
             // CAS loop: retry directly while our edge still beats the occupant,
             // rescan the list only when it does not
             while (beats<DIST>(P, x, k, nT, tb, bx, best, kb, s)) {
@@ -329,8 +367,9 @@ __global__ void k_dist_active(int32_t nPl, int64_t nB, const int32_t *__restrict
 }
 
 __global__ void k_dist_mates(int64_t nB, int64_t nA, const int32_t *__restrict__ gi, const int32_t *__restrict__ La,
-                             int32_t *__restrict__ mateA, int32_t *__restrict__ mateB)
+                             MatchParams P, int32_t *__restrict__ mateB)
 {
+    int32_t *mateA = slot_mates(P);
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < 2 * nB; v += (int64_t)gridDim.x * blockDim.x) {
         const int e = gi[v];
         mateB[v] = e;
@@ -343,20 +382,43 @@ __global__ void k_fill_i32(int64_t n, int32_t *__restrict__ x, int32_t v)
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) x[i] = v;
 }
 
-// the final suitor of each target is its mate (mate arrays pre-set to -1)
-__global__ void k_suitor_to_mates(int64_t nT, int ninst, const int32_t *__restrict__ own,
-                                  const unsigned long long *__restrict__ sT, int32_t *__restrict__ mateT,
-                                  int32_t *__restrict__ mateP, int64_t nP)
+// The final suitor of each target is its mate: mates of both sides and the
+// B vertex of each matched A vertex (evaluate's input) from the target slots;
+// proposers left unmatched were written by k_suitor.  Every slot is reset to
+// empty for the next rounding (no separate reset pass), and the round's
+// overlap / cardinality accumulators are zeroed (k_eval follows).
+__global__ void k_collect(MatchParams P, int64_t nT, int64_t nP, int fromB)
 {
     pdl_wait();
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < ninst * nT;
+    if (blockIdx.x == 0 && threadIdx.x < 4) (&P.rd->overlap[0])[threadIdx.x] = 0ull; // overlap[2], card[2]
+    int32_t *mateA = slot_mates(P);
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < P.ninst * nT;
          v += (int64_t)gridDim.x * blockDim.x) {
         const int k = (int)(v / nT);
-        const unsigned long long s = sT[v];
+        const int64_t t = v - k * nT;
+        const unsigned long long s = P.suit[v];
+        if (s) P.suit[v] = 0ull;
         const int e = s ? (int)(uint32_t)s : -1;
-        mateT[v] = e;
-        if (e >= 0) mateP[k * nP + own[e]] = e;
+        if (!fromB) {             // targets are B vertices
+            P.mateB[v] = e;
+            if (e >= 0) {
+                const int a = __ldg(P.La + e);
+                mateA[k * nP + a] = e;
+                set_mv(P.mvA, a, k, (int)t);
+            }
+        } else {                  // targets are A vertices
+            mateA[v] = e;
+            set_mv(P.mvA, t, k, e >= 0 ? __ldg(P.Lb + e) : -1);
+            if (e >= 0) P.mateB[k * nP + __ldg(P.Lb + e)] = e;
+        }
     }
+}
+
+__global__ void k_fill_slot(MatchParams P, int64_t n)
+{
+    int32_t *mateA = slot_mates(P);
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        mateA[i] = -1;
 }
 
 // ---------------------------------------------------------- pointer rounds
@@ -401,6 +463,7 @@ __device__ int cand_B(const MatchParams &P, int k, int b)
 
 __global__ void __launch_bounds__(256) k_pointer_rounds(MatchParams P)
 {
+    P.mateA = slot_mates(P);
     cg::grid_group grid = cg::this_grid();
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
@@ -494,8 +557,9 @@ struct EvalParams {
     int64_t nA;
     const int32_t *Lb;
     const double *w;
-    const int32_t *mateA; // 2 instances, final
-    const int32_t *mvA;   // 2 instances: M(i) as a B vertex (-1: unmatched), k_mate_vertex
+    const int32_t *mates; // [2 slots][2 instances][nA]; this round's slot is *wslot
+    const int *wslot;
+    const int2 *mvA;      // (M_y(i), M_z(i)) as B vertices (-1: unmatched)
     const unsigned long long *Bhash; // E_B membership set
     int Bhash_log;
     const int2 *pairs;    // undirected A edges (i < j)
@@ -506,8 +570,8 @@ struct EvalParams {
 
 // One block (the last one of k_eval to finish): finish the sums, score, select,
 // best (Alg. 2 l.21-24).
-__device__ void round_final_block(const EvalParams &P, int nblocks, int exact, double alpha, double beta,
-                                  const int *p_dev, const unsigned long long *work, double *sd)
+__device__ void round_final_block(const EvalParams &P, const int32_t *mateA, int nblocks, int exact, double alpha,
+                                  double beta, const int *p_dev, unsigned long long *work, double *sd)
 {
     double wk[2] = {0.0, 0.0};
     for (int k = 0; k < 2; k++) {
@@ -515,7 +579,7 @@ __device__ void round_final_block(const EvalParams &P, int nblocks, int exact, d
             // oracle order: ascending edge id == ascending A vertex
             if (threadIdx.x == 0) {
                 double s = 0.0;
-                const int32_t *mA = P.mateA + (int64_t)k * P.nA;
+                const int32_t *mA = mateA + (int64_t)k * P.nA;
                 for (int64_t a = 0; a < P.nA; a++)
                     if (mA[a] >= 0) s = s + P.w[mA[a]];
                 wk[k] = s;
@@ -546,6 +610,8 @@ __device__ void round_final_block(const EvalParams &P, int nblocks, int exact, d
     for (int i = 0; i < WORK_SPREAD; i++) {
         w0 += work[i * WORK_STRIDE];
         w1 += work[i * WORK_STRIDE + 1];
+        work[i * WORK_STRIDE] = 0ull; // ready for the next rounding
+        work[i * WORK_STRIDE + 1] = 0ull;
     }
     I.rounds_y = (int32_t)w0;
     I.rounds_z = (int32_t)w1;
@@ -553,15 +619,20 @@ __device__ void round_final_block(const EvalParams &P, int nblocks, int exact, d
     I.source = src;
     I.score = src ? I.score_z : I.score_y;
     I.improved = 0;
+    const int ws = rd->wslot;
     if (I.score > rd->best_score) {
         rd->best_score = I.score;
         rd->best_iter = p;
+        rd->best_slot = ws; // bestM = this round's M_src, kept in place
+        rd->best_source = src;
         I.improved = 1;
     }
     I.best_score = rd->best_score;
     I.best_iter = rd->best_iter;
     rd->improved = I.improved;
     rd->source = src;
+    rd->last_slot = ws;
+    rd->wslot = 1 - rd->best_slot;
 }
 
 // Evaluate M_y and M_z.  weight: partial sums per block over a fixed
@@ -572,7 +643,7 @@ __device__ void round_final_block(const EvalParams &P, int nblocks, int exact, d
 // a ~5-load binary search in B's row of M(i)) -- balanced whatever the degree
 // of i.  The last block to finish runs the final reduction.
 __global__ void __launch_bounds__(256)
-k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, const unsigned long long *work)
+k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, unsigned long long *work)
 {
     pdl_wait();
     __shared__ double sd[32];
@@ -580,10 +651,11 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, con
     __shared__ bool last;
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+    const int32_t *mateA = P.mates + (int64_t)(*(volatile const int *)P.wslot) * 2 * P.nA;
     double wsum[2] = {0.0, 0.0};
     unsigned long long ov[2] = {0, 0}, card[2] = {0, 0};
     for (int64_t i = tid; i < P.nA; i += nthr) {
-        const int e0 = P.mateA[i], e1 = P.mateA[P.nA + i];
+        const int e0 = mateA[i], e1 = mateA[P.nA + i];
         if (e0 >= 0) {
             wsum[0] += P.w[e0];
             card[0]++;
@@ -598,28 +670,22 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, con
     constexpr int EVAL_U = 4;
     for (int64_t base = tid; base < P.npairs; base += nthr * EVAL_U) {
         int2 ij[EVAL_U];
-        int em[EVAL_U][4]; // mates of i and j in both instances (edge ids)
+        int2 mi[EVAL_U], mj[EVAL_U]; // (M_y, M_z) of i and of j as B vertices
 #pragma unroll
         for (int u = 0; u < EVAL_U; u++) {
             const int64_t q = base + u * nthr;
             ij[u] = q < P.npairs ? __ldg(P.pairs + q) : make_int2(-1, -1);
         }
-        // M(i), M(j) as B vertices (-1: unmatched), one gather each
+        // both instances' images of i and j: one 8-byte gather each
 #pragma unroll
         for (int u = 0; u < EVAL_U; u++) {
-#pragma unroll
-            for (int k = 0; k < 2; k++) {
-                em[u][2 * k] = ij[u].x >= 0 ? P.mvA[k * P.nA + ij[u].x] : -1;
-                em[u][2 * k + 1] = ij[u].x >= 0 ? P.mvA[k * P.nA + ij[u].y] : -1;
-            }
+            mi[u] = ij[u].x >= 0 ? P.mvA[ij[u].x] : make_int2(-1, -1);
+            mj[u] = ij[u].x >= 0 ? P.mvA[ij[u].y] : make_int2(-1, -1);
         }
 #pragma unroll
         for (int u = 0; u < EVAL_U; u++) {
-#pragma unroll
-            for (int k = 0; k < 2; k++)
-                if (em[u][2 * k] >= 0 && em[u][2 * k + 1] >= 0 &&
-                    bhash_has(P.Bhash, P.Bhash_log, bhash_key(em[u][2 * k], em[u][2 * k + 1])))
-                    ov[k]++;
+            if (mi[u].x >= 0 && mj[u].x >= 0 && bhash_has(P.Bhash, P.Bhash_log, bhash_key(mi[u].x, mj[u].x))) ov[0]++;
+            if (mi[u].y >= 0 && mj[u].y >= 0 && bhash_has(P.Bhash, P.Bhash_log, bhash_key(mi[u].y, mj[u].y))) ov[1]++;
         }
     }
     for (int k = 0; k < 2; k++) {
@@ -637,43 +703,23 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, con
     __syncthreads();
     if (!last) return;
     __threadfence();
-    round_final_block(P, gridDim.x, exact, alpha, beta, p_dev, work, sd);
+    round_final_block(P, mateA, gridDim.x, exact, alpha, beta, p_dev, work, sd);
     if (threadIdx.x == 0) P.rd->done = 0u;
 }
 
-// M(i) as a B vertex for both instances (evaluate reads it per A edge
-// instead of mate -> L_b twice), and the round's overlap / cardinality
-// accumulators zeroed (this kernel precedes k_eval)
-__global__ void k_mate_vertex(int64_t n2, const int32_t *__restrict__ mateA, const int32_t *__restrict__ Lb,
-                              int32_t *__restrict__ mvA, RoundDev *rd)
+// Schedules whose kernels leave complete mate arrays (pointer rounds, the
+// sharded merge): (M_y(i), M_z(i)) as B vertices from this round's slot, and
+// the round's overlap / cardinality accumulators zeroed (k_eval follows).
+__global__ void k_mate_vertex(int64_t nA, const int32_t *__restrict__ mates, const int *__restrict__ wslot,
+                              const int32_t *__restrict__ Lb, int2 *__restrict__ mvA, RoundDev *rd)
 {
     pdl_wait();
     if (blockIdx.x == 0 && threadIdx.x < 4) (&rd->overlap[0])[threadIdx.x] = 0ull; // overlap[2], card[2]
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n2; i += (int64_t)gridDim.x * blockDim.x) {
-        const int e = mateA[i];
-        mvA[i] = e >= 0 ? __ldg(Lb + e) : -1;
+    const int32_t *mA = mates + (int64_t)(*(volatile const int *)wslot) * 2 * nA;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nA; i += (int64_t)gridDim.x * blockDim.x) {
+        const int e0 = mA[i], e1 = mA[nA + i];
+        mvA[i] = make_int2(e0 >= 0 ? __ldg(Lb + e0) : -1, e1 >= 0 ? __ldg(Lb + e1) : -1);
     }
-}
-
-__global__ void k_match_reset(int64_t ns, unsigned long long *__restrict__ suit, int64_t nm,
-                              int32_t *__restrict__ mate)
-{
-    pdl_wait();
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < (ns > nm ? ns : nm);
-         i += (int64_t)gridDim.x * blockDim.x) {
-        if (i < ns) suit[i] = 0ull;
-        if (i < nm) mate[i] = -1;
-    }
-}
-
-__global__ void k_copy_best(int64_t nA, const int32_t *__restrict__ mateA, const RoundDev *__restrict__ rd,
-                            int32_t *__restrict__ best_mate)
-{
-    pdl_wait();
-    if (!rd->improved) return;
-    const int32_t *src = mateA + (int64_t)rd->source * nA;
-    for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < nA; a += (int64_t)gridDim.x * blockDim.x)
-        best_mate[a] = src[a];
 }
 
 __global__ void k_maxdeg(int64_t nA, const int64_t *__restrict__ Arow, int64_t nB,
@@ -719,18 +765,23 @@ MatchParams base_params(cualign_bp *h)
     P.candA = h->candA;
     P.candB = h->candB;
     P.suit = h->suit;
-    P.mateA = h->mateA;
+    P.mates = h->mates;
+    P.wslot = &h->rd->wslot;
     P.mateB = h->mateB;
+    P.mvA = h->mvA;
     P.rd = h->rd;
     P.work = h->match_work;
     return P;
 }
 
-// run the matching of ninst instances; leaves mateA / mateB final
+// Run the matching of P.ninst instances into this round's mate slot.
+// Suitor: k_suitor (exhausted proposers) + k_collect (everything held in a
+// target slot; resets the slots) leave the mates of both sides, mvA and zeroed
+// round accumulators -- ready for k_eval.  Pointer rounds leave complete mate
+// arrays (k_mate_vertex prepares evaluate).
 cualign_status run_matching(cualign_bp *h, MatchParams &P)
 {
     const int64_t nA = h->L.nA, nB = h->L.nB;
-    CA_CUDA(cudaMemsetAsync(h->match_work, 0, WORK_SPREAD * WORK_STRIDE * sizeof(unsigned long long), h->stream));
     if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) {
         KScope ks(h, CUALIGN_K_MATCH);
         // cooperative launch through cudaLaunchKernelEx: capturable into a graph
@@ -749,14 +800,6 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
     const bool fromB = h->propose_from_b;
     P.propose_from_b = fromB ? 1 : 0;
     const int64_t nP = fromB ? nB : nA, nT = fromB ? nA : nB;
-    {
-        // suitor slots to 0 and proposer mates to -1 (one kernel, not two
-        // memset nodes: keeps the step's kernel chain programmatic)
-        KScope ks(h, CUALIGN_K_MATCHAUX);
-        const int64_t nmax = (2 * nT + 1) > (2 * nP + 1) ? (2 * nT + 1) : (2 * nP + 1);
-        CA_CUDA(launch_pdl(k_match_reset, dim3(grid_for(nmax, 256, h->num_sms * 4)), dim3(256), 0, h->stream,
-                           2 * nT + 1, h->suit, 2 * nP + 1, fromB ? h->mateB : h->mateA));
-    }
     const int64_t slots = P.ninst * nP;
     static const bool dbg_env = probe_knob("CUALIGN_MATCH_DEBUG", 0) != 0;
     const bool dbg = dbg_env && !h->capturing;
@@ -772,13 +815,13 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
         static const int genv = probe_knob("CUALIGN_SUITOR_G", 0);
         // tile width: G lanes x U edges cover a typical proposer list in one pass
         const int G = genv ? genv : (dmax > 64 ? 32 : (dmax > 24 ? 16 : (dmax > 20 ? 8 : 4)));
-        if (G == 32) k_suitor<32, 2><<<grid_for(slots * 32, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else if (G == 16) k_suitor<16, 2><<<grid_for(slots * 16, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else if (G == 8) k_suitor<8, 3><<<grid_for(slots * 8, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else if (G == 2) k_suitor<2, 9><<<grid_for(slots * 2, 128, 1 << 30), 128, 0, h->stream>>>(P);
-        else if (G == 1) k_suitor<1, 8><<<grid_for(slots, 128, 1 << 30), 128, 0, h->stream>>>(P);
+        if (G == 32) CA_CUDA(launch_pdl(k_suitor<32, 2>, dim3(grid_for(slots * 32, 128, 1 << 30)), dim3(128), 0, h->stream, P));
+        else if (G == 16) CA_CUDA(launch_pdl(k_suitor<16, 2>, dim3(grid_for(slots * 16, 128, 1 << 30)), dim3(128), 0, h->stream, P));
+        else if (G == 8) CA_CUDA(launch_pdl(k_suitor<8, 3>, dim3(grid_for(slots * 8, 128, 1 << 30)), dim3(128), 0, h->stream, P));
+        else if (G == 2) CA_CUDA(launch_pdl(k_suitor<2, 9>, dim3(grid_for(slots * 2, 128, 1 << 30)), dim3(128), 0, h->stream, P));
+        else if (G == 1) CA_CUDA(launch_pdl(k_suitor<1, 8>, dim3(grid_for(slots, 128, 1 << 30)), dim3(128), 0, h->stream, P));
         else {
-            // resident blocks per SM (register cap): measurement knob
+            // resident blocks per SM (register cap), probe build knob:
             // default 12 blocks of 128 (40 registers): 0.142 ms vs 0.175 ms
             // uncapped (66 registers, 8 blocks) on O -- latency-bound, more
             // resident proposer tiles win over a few spilled registers
@@ -793,10 +836,10 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
                 (void)cudaGetLastError();
                 k_suitor_persistent<4, 5, 12><<<grid_for(slots * 4, 128, (int64_t)occ * h->num_sms), 128, 0,
                                                 h->stream>>>(P);
-            } else if (minb >= 16) k_suitor<4, 5, false, 16><<<grid, 128, 0, h->stream>>>(P);
+            } else if (minb >= 16) CA_CUDA(launch_pdl(k_suitor<4, 5, false, 16>, dim3(grid), dim3(128), 0, h->stream, P));
             else if (minb >= 12) CA_CUDA(launch_pdl(k_suitor<4, 5, false, 12>, dim3(grid), dim3(128), 0, h->stream, P));
-            else if (minb >= 10) k_suitor<4, 5, false, 10><<<grid, 128, 0, h->stream>>>(P);
-            else k_suitor<4, 5><<<grid, 128, 0, h->stream>>>(P);
+            else if (minb >= 10) CA_CUDA(launch_pdl(k_suitor<4, 5, false, 10>, dim3(grid), dim3(128), 0, h->stream, P));
+            else CA_CUDA(launch_pdl(k_suitor<4, 5>, dim3(grid), dim3(128), 0, h->stream, P));
         }
         CA_CUDA(cudaGetLastError());
     }
@@ -808,13 +851,25 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
                 (long long)slots, d[0], d[1], d[2], d[3], d[4]);
         cudaFree(dbuf);
     }
-    if (P.ninst * nT > 0) {
+    {
         KScope ks(h, CUALIGN_K_MATCHAUX);
-        CA_CUDA(launch_pdl(k_suitor_to_mates, dim3(grid_for(P.ninst * nT, 256, h->num_sms * 8)), dim3(256), 0,
-                           h->stream, nT, P.ninst, fromB ? P.Lb : P.La, (const unsigned long long *)h->suit,
-                           fromB ? P.mateA : P.mateB, fromB ? P.mateB : P.mateA, nP));
+        CA_CUDA(launch_pdl(k_collect, dim3(grid_for(P.ninst * nT > 0 ? P.ninst * nT : 1, 256, h->num_sms * 8)),
+                           dim3(256), 0, h->stream, P, nT, nP, fromB ? 1 : 0));
         CA_CUDA(cudaGetLastError());
     }
+    return CUALIGN_OK;
+}
+
+// (M_y(i), M_z(i)) for evaluate from complete mate arrays (pointer rounds,
+// sharded merge)
+cualign_status prep_eval_from_mates(cualign_bp *h)
+{
+    KScope ks(h, CUALIGN_K_MATCHAUX);
+    const int64_t nA = h->L.nA;
+    CA_CUDA(launch_pdl(k_mate_vertex, dim3(grid_for(nA > 0 ? nA : 1, 256, h->num_sms * 4)), dim3(256), 0, h->stream,
+                       nA, (const int32_t *)h->mates, (const int *)&h->rd->wslot, (const int32_t *)h->L.Lb, h->mvA,
+                       h->rd));
+    CA_CUDA(cudaGetLastError());
     return CUALIGN_OK;
 }
 
@@ -823,27 +878,34 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
 cualign_status match_setup(cualign_bp *h)
 {
     const size_t nA = (size_t)h->L.nA, nB = (size_t)h->L.nB;
+    const size_t nmax = nA > nB ? nA : nB;
     CA_TRY(dalloc(h, &h->candA, 2 * nA + 1));
     CA_TRY(dalloc(h, &h->candB, 2 * nB + 1));
-    CA_TRY(dalloc(h, &h->suit, 2 * (nA > nB ? nA : nB) + 1));
-    CA_TRY(dalloc(h, &h->mateA, 2 * nA + 1));
-    CA_TRY(dalloc(h, &h->mvA, 2 * nA + 1));
+    CA_TRY(dalloc(h, &h->suit, 2 * nmax + 1));
+    CA_TRY(dalloc(h, &h->mates, 4 * nA + 1));
+    CA_TRY(dalloc(h, &h->mvA, nA + 1));
     CA_TRY(dalloc(h, &h->mateB, 2 * nB + 1));
-    CA_TRY(dalloc(h, &h->best_mate, nA + 1));
     CA_TRY(dalloc(h, &h->rd, 1));
     CA_TRY(dalloc(h, &h->match_work, WORK_SPREAD * WORK_STRIDE));
-    CA_CUDA(cudaMemsetAsync(h->rd, 0, sizeof(RoundDev), h->stream));
-    CA_CUDA(cudaMemsetAsync(h->mateA, 0xff, sizeof(int32_t) * (2 * nA + 1), h->stream));
+    {
+        RoundDev r0;
+        memset(&r0, 0, sizeof(r0));
+        r0.wslot = 1; // slot 0 "holds" the empty bestM (best_iter = 0)
+        CA_CUDA(cudaMemcpyAsync(h->rd, &r0, sizeof(RoundDev), cudaMemcpyHostToDevice, h->stream));
+        CA_CUDA(cudaStreamSynchronize(h->stream)); // r0 is a stack object
+    }
+    CA_CUDA(cudaMemsetAsync(h->suit, 0, sizeof(unsigned long long) * (2 * nmax + 1), h->stream));
+    CA_CUDA(cudaMemsetAsync(h->mates, 0xff, sizeof(int32_t) * (4 * nA + 1), h->stream));
     CA_CUDA(cudaMemsetAsync(h->mateB, 0xff, sizeof(int32_t) * (2 * nB + 1), h->stream));
-    CA_CUDA(cudaMemsetAsync(h->best_mate, 0xff, sizeof(int32_t) * (nA + 1), h->stream));
+    CA_CUDA(cudaMemsetAsync(h->match_work, 0, sizeof(unsigned long long) * WORK_SPREAD * WORK_STRIDE, h->stream));
     {
         KScope ks(h, CUALIGN_K_INIT);
         unsigned long long md[2] = {0, 0};
-        CA_CUDA(cudaMemsetAsync(h->match_work, 0, 2 * sizeof(unsigned long long), h->stream));
         k_maxdeg<<<grid_for((int64_t)(nA + nB), 256, h->num_sms * 8), 256, 0, h->stream>>>(
             (int64_t)nA, h->L.Arow, (int64_t)nB, h->L.Bptr, h->match_work);
         CA_CUDA(cudaGetLastError());
         CA_CUDA(cudaMemcpyAsync(md, h->match_work, sizeof(md), cudaMemcpyDeviceToHost, h->stream));
+        CA_CUDA(cudaMemsetAsync(h->match_work, 0, 2 * sizeof(unsigned long long), h->stream));
         CA_CUDA(cudaStreamSynchronize(h->stream));
         h->max_deg_a = (int64_t)md[0];
         h->max_deg_b = (int64_t)md[1];
@@ -874,6 +936,7 @@ cualign_status match_round(cualign_bp *h)
     P.x0 = damped ? h->yp : h->yc;
     P.x1 = damped ? h->zp : h->zc;
     CA_TRY(run_matching(h, P));
+    if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) CA_TRY(prep_eval_from_mates(h));
     return match_evaluate(h);
 }
 
@@ -978,25 +1041,29 @@ cualign_status dist_match_update(cualign_bp *h)
 cualign_status dist_match_finish(cualign_bp *h)
 {
     const int64_t nA = h->L.nA, nB = h->L.nB;
-    CA_CUDA(cudaMemsetAsync(h->mateA, 0xff, sizeof(int32_t) * (size_t)(2 * nA + 1), h->stream));
     {
         KScope ks(h, CUALIGN_K_MATCHAUX);
+        MatchParams P = base_params(h);
+        k_fill_slot<<<grid_for(2 * nA + 1, 256, h->num_sms * 8), 256, 0, h->stream>>>(P, 2 * nA);
         if (nB)
             k_dist_mates<<<grid_for(2 * nB, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB, nA, h->dist_gi, h->L.La,
-                                                                                       h->mateA, h->mateB);
+                                                                                       P, h->mateB);
         CA_CUDA(cudaGetLastError());
     }
+    CA_TRY(prep_eval_from_mates(h));
     return match_evaluate(h);
 }
 
-// a8 (evaluate + best) of the matchings in mateA / mateB
+// a8 (evaluate + best) of this round's mates (slot rd->wslot) and mvA; the
+// final block records bestM by slot (no copy)
 cualign_status match_evaluate(cualign_bp *h)
 {
     EvalParams E{};
     E.nA = h->L.nA;
     E.Lb = h->L.Lb;
     E.w = h->L.w;
-    E.mateA = h->mateA;
+    E.mates = h->mates;
+    E.wslot = &h->rd->wslot;
     E.mvA = h->mvA;
     E.Bhash = h->Bhash;
     E.Bhash_log = h->Bhash_log;
@@ -1005,25 +1072,10 @@ cualign_status match_evaluate(cualign_bp *h)
     E.partial_w = h->partial_w;
     E.rd = h->rd;
     {
-        // M(i) as B vertices + zeroed overlap / card accumulators (the rest of rd persists: best)
-        KScope ks(h, CUALIGN_K_MATCHAUX);
-        const int64_t n2 = 2 * (int64_t)h->L.nA;
-        CA_CUDA(launch_pdl(k_mate_vertex, dim3(grid_for(n2 > 0 ? n2 : 1, 256, h->num_sms * 4)), dim3(256), 0,
-                           h->stream, n2, (const int32_t *)h->mateA, (const int32_t *)h->L.Lb, h->mvA, h->rd));
-        CA_CUDA(cudaGetLastError());
-    }
-    {
         KScope ks(h, CUALIGN_K_EVAL);
         CA_CUDA(launch_pdl(k_eval, dim3(h->eval_grid), dim3(256), 0, h->stream, E,
                            (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha, h->beta,
-                           (const int *)(h->round_p ? h->round_p : h->p_dev),
-                           (const unsigned long long *)h->match_work));
-        CA_CUDA(cudaGetLastError());
-    }
-    {
-        KScope ks(h, CUALIGN_K_MATCHAUX);
-        CA_CUDA(launch_pdl(k_copy_best, dim3(grid_for(h->L.nA, 256, h->num_sms * 4)), dim3(256), 0, h->stream,
-                           (int64_t)h->L.nA, (const int32_t *)h->mateA, (const RoundDev *)h->rd, h->best_mate));
+                           (const int *)(h->round_p ? h->round_p : h->p_dev), h->match_work));
         CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;
@@ -1035,6 +1087,7 @@ cualign_status match_standalone(cualign_bp *h, const double *x_dev, int32_t *rou
     P.ninst = 1;
     P.x0 = x_dev;
     P.x1 = x_dev;
+    CA_CUDA(cudaMemsetAsync(h->match_work, 0, WORK_SPREAD * WORK_STRIDE * sizeof(unsigned long long), h->stream));
     CA_TRY(run_matching(h, P));
     if (rounds) {
         std::vector<unsigned long long> w(WORK_SPREAD * WORK_STRIDE);
