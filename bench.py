@@ -20,6 +20,7 @@ import json
 import os
 import platform
 import statistics
+import subprocess
 import sys
 import threading
 import time
@@ -31,6 +32,8 @@ if ROOT not in sys.path:
 import numpy as np
 
 METRIC = "BP iterations/sec and squares/sec; end-to-end align time at 1/2/4/8 B200"
+CONFIGS_DESC_O = ("ontology-shaped: clustered power-law n_A=3e5 (avg deg 18), B=P(A[V']) |V'|=2e5 +5%; "
+                  "proxy k=16.67 -> m~5e6; s~1e8")
 UNIT = "iterations/s"
 # algorithmic bytes: (2*sigma + 4) per nonzero of S, (9*sigma + 8) per L edge
 SIGMA = 8
@@ -158,62 +161,105 @@ def max_over_ranks(x, world, device=None):
     return float(t.item())
 
 
-def oracle_rate(scale, n_iter, full_work):
-    """Oracle (single thread, fp64) on config O generated at `scale`: create +
-    n_iter x (step + round).  Returns (iterations/s extrapolated to the full
-    workload linearly in s + m, detail dict)."""
-    import oracle
+def host_info():
+    """The host the oracle runs on: cores, CPU model, memory."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as fh:
+            for line in fh:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    try:
+        mem_gb = os.sysconf("SC_PAGE_SIZE") * os.sysconf("SC_PHYS_PAGES") / 2 ** 30
+    except (ValueError, OSError, AttributeError):
+        mem_gb = None
+    return {"nproc": os.cpu_count(), "cpu_model": model or platform.processor() or platform.machine(),
+            "mem_gib": round(mem_gb, 1) if mem_gb else None}
+
+
+def oracle_on_O(n_warm, n_steps, pin_core=0):
+    """The oracle (oracle/, single-threaded fp64 C, as it stands) on the FULL
+    config O instance, pinned to one core: create (S by its definition), then
+    n_warm untimed and n_steps timed steps, a step = Alg. 2 l.9-16 + l.17-24
+    (step_gamma + round).  Returns a dict of timings."""
+    try:
+        os.sched_setaffinity(0, {pin_core})
+    except (AttributeError, OSError):
+        pass
+    os.environ["OMP_NUM_THREADS"] = "1"
     from oracle import Oracle
     from synth import make_config
-    inst = make_config("O", scale=scale)
     t0 = time.perf_counter()
-    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    inst = make_config("O")
     t1 = time.perf_counter()
-    for _ in range(n_iter):
+    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
+    t2 = time.perf_counter()
+    for _ in range(n_warm):
         o.step_gamma(inst.gamma)
         o.round()
-    t2 = time.perf_counter()
-    per_iter = (t2 - t1) / n_iter
-    work = o.s + o.m
-    rate_sample = 1.0 / per_iter
-    rate_full = rate_sample * work / full_work
-    return rate_full, dict(scale=scale, m=o.m, s=o.s, iters=n_iter, create_s=t1 - t0,
-                           per_iter_s=per_iter, rate_sample=rate_sample)
+    step_s = []
+    for _ in range(n_steps):
+        ts = time.perf_counter()
+        o.step_gamma(inst.gamma)
+        o.round()
+        step_s.append(time.perf_counter() - ts)
+    try:
+        cores = len(os.sched_getaffinity(0))
+    except (AttributeError, OSError):
+        cores = None
+    return {"gen_s": t1 - t0, "create_s": t2 - t1, "step_s": step_s, "m": o.m, "s": o.s, "cores": cores,
+            "pinned_core": pin_core, "n_warm": n_warm, "n_steps": n_steps}
+
+
+def start_oracle_child(n_steps):
+    """cpu_baseline leg: the oracle on full O in a child process pinned to core
+    0 (OMP_NUM_THREADS=1), running while the GPU is measured (the bench process
+    moves to the other cores); collected at the end."""
+    env = dict(os.environ, OMP_NUM_THREADS="1")
+    env.pop("RANK", None)
+    env.pop("WORLD_SIZE", None)
+    return subprocess.Popen([sys.executable, os.path.abspath(__file__), "--oracle-child", str(n_steps)],
+                            stdout=subprocess.PIPE, stderr=subprocess.PIPE, text=True, env=env, cwd=ROOT)
+
+
+def finish_oracle_child(proc):
+    out, err = proc.communicate()
+    if proc.returncode != 0:
+        return {"value": None, "unit": UNIT, "cores": 1, "kind": "oracle",
+                "sample": "failed: " + (err or "")[-300:]}
+    d = json.loads(out.strip().splitlines()[-1])
+    per = statistics.mean(d["step_s"])
+    return {"value": 1.0 / per, "unit": UNIT, "cores": d["cores"], "kind": "oracle",
+            "sample": (f"full config O (m={d['m']}, s={d['s']}): oracle create {d['create_s']:.1f} s (untimed), "
+                       f"then {d['n_steps']} timed steps of Alg. 2 step + round, single thread pinned to core "
+                       f"{d['pinned_core']} (taskset-equivalent sched_setaffinity, OMP_NUM_THREADS=1); "
+                       f"value = 1 / mean step time ({per:.3f} s)"),
+            "step_s": d["step_s"], "create_s": d["create_s"], "host": host_info()}
 
 
 def run_reference(args, rank, world):
-    """--impl reference: the oracle as it stands on the host cores (no
-    reference implementation exists)."""
+    """--impl reference: the oracle as it stands on one host core, on the SAME
+    workload as our arm (full config O), W warm-up and K timed steps, a step =
+    one Alg. 2 iteration + its rounding (no reference implementation exists:
+    the reference is a paper).  Rank 0 only; other ranks exit without work."""
     if rank != 0:
         return
-    from synth import O_full_work
-    full_m, full_s = O_full_work()
-    full_work = full_m + full_s
-    import oracle
-    from oracle import Oracle
-    from synth import make_config
-    scale = args.ref_scale
-    inst = make_config("O", scale=scale)
-    o = Oracle(inst.A, inst.B, inst.L, inst.alpha, inst.beta)
-    for _ in range(args.warmup):
-        o.step_gamma(inst.gamma)
-        o.round()
-    t0 = time.perf_counter()
-    for _ in range(args.steps):
-        o.step_gamma(inst.gamma)
-        o.round()
-    dt = time.perf_counter() - t0
-    rate_sample = args.steps / dt
-    value = rate_sample * (o.s + o.m) / full_work
-    sample = (f"config O generator at scale {scale} (m={o.m}, s={o.s}); {args.steps} steps of "
-              f"oracle step+round, single thread; rate extrapolated linearly in (s+m) to full O "
-              f"(m={full_m}, s={full_s})")
+    d = oracle_on_O(args.warmup, args.steps)
+    total = sum(d["step_s"])
+    value = args.steps / total
+    sample = (f"full config O (m={d['m']}, s={d['s']}); oracle create {d['create_s']:.1f} s untimed, "
+              f"{args.warmup} warm-up + {args.steps} timed steps (Alg. 2 step + round each), single thread "
+              f"pinned to core {d['pinned_core']}")
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000.0 / value,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000.0 * total / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
-            "config": {"workload": "O: ontology-shaped pair (BASELINE.json configs[2])", "sample": sample},
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "config": {"workload": "O: " + CONFIGS_DESC_O, "m": d["m"], "s": d["s"], "sample": sample},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": d["cores"], "kind": "oracle", "sample": sample,
+                             "host": host_info()},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -251,20 +297,108 @@ def knn_measure(ca, dev, peak, n=65536, d=128, k=20, reps=3):
                          "frac": tf / peak[0], "peak_source": peak[1]}}
 
 
+def launch_floor_ms(n_kernels, reps=200):
+    """Graph-replay floor of a step of n_kernels tiny kernels: a CUDA graph of
+    n_kernels one-element torch kernels, replayed, CUDA-event timed."""
+    import torch
+    x = torch.zeros(1, device="cuda")
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(s):
+        for _ in range(3):
+            x.add_(1.0)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(n_kernels):
+                x.add_(1.0)
+        for _ in range(10):
+            g.replay()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        for _ in range(reps):
+            g.replay()
+        e1.record(s)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps
+
+
+def config_point(ca, name, k, steps, stream, dev):
+    """One BASELINE.json config on one GPU: generate (seeded),
+    init through the C ABI, the library's schedule selection + warm-up, then
+    `steps` device-timed steps (iteration + rounding) on the launching stream;
+    iterate-only and round-only graph replays with per-kernel event nodes for
+    the split and the square pass's HBM fraction (20 B per nonzero of S)."""
+    import torch
+    from synth import make_config
+    t0 = time.perf_counter()
+    inst = make_config(name, k=k)
+    row = {"n_a": inst.A.n, "n_b": inst.B.n, "m": int(inst.L.m), "gen_s": round(time.perf_counter() - t0, 1),
+           "desc": inst.meta["desc"] + (f" (k = {k})" if k else "")}
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    h = ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, device=dev, stream=stream)
+    torch.cuda.synchronize()
+    row["init_s"] = time.perf_counter() - t0
+    peak, _ = read_peaks()
+    with h:
+        sz = h.sizes()
+        s_nz = int(sz["s"])
+        row.update(s=s_nz, squares=s_nz // 2, device_gb=round(sz["device_bytes"] / 1e9, 2))
+        h.run(57)       # the library's schedule selection (timed pipelined vs serial), untimed here
+        h.run(5)
+        torch.cuda.synchronize()
+        h.stats(reset=True)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        h.run(steps)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1) / steps
+        st = h.stats(reset=True)
+        kernels = st["launches"] / steps
+        row.update(steps=steps, ms_per_step=ms, iters_per_s=1e3 / ms, squares_per_s=(s_nz / 2) * 1e3 / ms,
+                   kernels_per_step=kernels,
+                   schedule={1: "pipelined", 2: "serial", 0: "forked"}.get(h.sizes()["schedule"], "?"))
+        h.set_timing(True)
+        h.run(steps, with_round=False)
+        torch.cuda.synchronize()
+        it = {c: v / steps for c, v in h.stats(reset=True)["class_ms"].items() if v}
+        h.run(steps, with_round=True, iterate=False)
+        torch.cuda.synchronize()
+        rd = {c: v / steps for c, v in h.stats(reset=True)["class_ms"].items() if v}
+        h.set_timing(False)
+        bp_ms = sum(it.values())
+        alg = BYTES_PER_NZ * s_nz + BYTES_PER_EDGE * row["m"]
+        row.update(bp_ms=bp_ms, round_ms=sum(rd.values()), iterate_kernel_ms=it, round_kernel_ms=rd,
+                   iteration_hbm_frac=alg / (bp_ms * 1e-3) / 1e9 / peak)
+        if it.get("square"):
+            row["square_hbm_frac"] = BYTES_PER_NZ * s_nz / (it["square"] * 1e-3) / 1e9 / peak
+    if name in ("T", "P"):
+        # latency-bound working sets (SURVEY §8(d)): against the graph-replay floor
+        fl = launch_floor_ms(int(round(kernels)))
+        row["graph_replay_floor_ms"] = fl
+        row["floor_frac"] = fl / ms
+    return row
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=300)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--config", default="O")
+    ap.add_argument("--config", default=None,
+                    help="workload: O at N = 1 (BASELINE.json configs[2]); S sharded at N > 1 (configs[3])")
     ap.add_argument("--scale", type=float, default=1.0)
     ap.add_argument("--e2e-iters", type=int, default=100)
     ap.add_argument("--e2e-reps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-scale", type=float, default=0.2)
-    ap.add_argument("--ref-scale", type=float, default=0.05)
+    ap.add_argument("--oracle-steps", type=int, default=3, help="timed oracle steps of the cpu_baseline leg")
+    ap.add_argument("--oracle-child", type=int, default=None, help=argparse.SUPPRESS)
+    ap.add_argument("--no-configs", action="store_true", help="skip the T/P/S/R sub-measurements")
+    ap.add_argument("--config-points", default="T,P,S,R5,R50")
+    ap.add_argument("--config-steps", type=int, default=20)
     ap.add_argument("--exact", action="store_true", help="CUALIGN_FLAG_EXACT (oracle-order sums)")
     ap.add_argument("--fp32", action="store_true", help="CUALIGN_FLAG_FP32_S (S^p stored in fp32, NEXT-3)")
     ap.add_argument("--match-rounds", action="store_true", help="pointer-round matching schedule")
@@ -272,12 +406,30 @@ def main():
     ap.add_argument("--strong", action="store_true", help="N > 1: shard the same instance (strong scaling)")
     ap.add_argument("--no-knn", action="store_true", help="skip the NEXT-2 kNN measurement")
     args = ap.parse_args()
+    if args.oracle_child is not None:
+        print(json.dumps(oracle_on_O(0, args.oracle_child)), flush=True)
+        return
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
     rank, world, local = dist_setup(args)
     if args.impl == "reference":
         run_reference(args, rank, world)
         return
+    if args.config is None:
+        args.config = "O" if world == 1 else "S"
+    if world > 1 and args.config == "S":
+        args.strong = True  # configs[3]: one instance sharded over the N GPUs
+    # cpu_baseline: the oracle on full O in a child pinned to core 0, running
+    # while the GPU is measured; this process keeps off that core
+    oracle_proc = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and args.config == "O" and args.scale == 1.0:
+        oracle_proc = start_oracle_child(args.oracle_steps)
+        try:
+            others = set(range(os.cpu_count() or 1)) - {0}
+            if others:
+                os.sched_setaffinity(0, others)
+        except (AttributeError, OSError):
+            pass
 
     import torch
     import paper_conf_sc_xiangkfah23_b200 as ca
@@ -285,9 +437,10 @@ def main():
 
     dev = local
     torch.cuda.set_device(dev)
-    # N > 1: weak scaling -- the same generator at N x the size, sharded by
-    # A-vertex blocks over the N ranks; every rank generates the
-    # identical seeded instance
+    # N > 1: config S (BASELINE.json configs[3], "sharded across 2/4/8 B200")
+    # split by A-vertex blocks over the N ranks, strong scaling;
+    # --config O at N > 1: weak scaling, the O generator at N x the size.
+    # Every rank generates the identical seeded instance.
     scale = args.scale * (world if (world > 1 and not args.strong) else 1)
     t_gen = time.perf_counter()
     inst = make_config(args.config, scale=scale, seed=None)
@@ -411,12 +564,13 @@ def main():
                                   "not an NVLink number" if os.environ.get("CUALIGN_ONE_GPU") == "1"
                                   else "NCCL (NVLink / NVSwitch)")}
 
-    # value: iterations/s of config O; at N > 1 in O-equivalent iterations/s
-    # (iterations/s x squares of the N-times-larger instance / squares of O),
+    # value: iterations/s of the instance; weak scaling (O x N) in
+    # O-equivalent iterations/s (iterations/s x squares / squares of one O),
     # i.e. the whole job's throughput in units of the N = 1 workload
     from synth import O_full_work
+    weak = world > 1 and not args.strong
     unit_squares = O_full_work()[1] / 2 if (args.config == "O" and args.scale == 1.0) else squares / max(world, 1)
-    work_units = squares / unit_squares if world > 1 else 1.0
+    work_units = squares / unit_squares if weak else 1.0
     value = args.steps * work_units / (elapsed_ms / 1e3)
     ms_per_step = elapsed_ms / args.steps
     cls_ms = pst["class_ms"]
@@ -429,16 +583,9 @@ def main():
     sq_gbs = sq_bytes / (sq_ms * 1e-3) / 1e9 if sq_ms > 0 else 0.0
     it_bytes = bytes_per_nz * s_local + BYTES_PER_EDGE * (sz["edge_end"] - sz["edge_begin"])
     it_gbs = it_bytes / (bp_ms * 1e-3) / 1e9 if bp_ms > 0 else 0.0
+    # DRAM traffic needs a profiler pass (ncu dram__bytes), which this timed
+    # run cannot take: null here; the ncu --set full captures are in profiles/
     traffic = None
-    tpath = os.path.join(ROOT, "profiles", "square_traffic.json")
-    if os.path.exists(tpath):
-        try:
-            with open(tpath) as fh:
-                tj = json.load(fh)
-            if tj.get("s") == s and bool(tj.get("fp32", False)) == bool(args.fp32):
-                traffic = tj.get("dram_bytes_per_launch")
-        except Exception:
-            pass
 
     # ------------------------------------------------------------------ e2e
     e2e = None
@@ -497,18 +644,20 @@ def main():
         del h
 
     # --------------------------------------------------------- cpu baseline
-    cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline and args.config == "O":
-        try:
-            rate, det = oracle_rate(args.cpu_scale, 3, m + s)
-            cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
-                   "sample": (f"config O generator at scale {det['scale']} (m={det['m']}, s={det['s']}), "
-                              f"oracle create + {det['iters']} x (step + round) single-threaded fp64 "
-                              f"({det['per_iter_s']:.3f} s/iteration); extrapolated linearly in s+m to "
-                              f"full O (m={m}, s={s})"),
-                   "host": platform.processor() or platform.machine(), "nproc": os.cpu_count()}
-        except Exception as e:  # pragma: no cover
-            cpu = {"value": None, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": f"failed: {e}"}
+    # ------------------------------------------------ other configs (T/P/S/R)
+    configs = None
+    if rank == 0 and world == 1 and not args.no_configs:
+        configs = {}
+        for pt in [x for x in args.config_points.split(",") if x]:
+            name, k = pt[0], (int(pt[1:]) if len(pt) > 1 else None)
+            try:
+                configs[pt] = config_point(ca, name, k, args.config_steps, stream, dev)
+            except Exception as ex:  # pragma: no cover
+                configs[pt] = {"error": str(ex)[:300]}
+            log(f"[config {pt}] {json.dumps(configs[pt])[:300]}")
+            torch.cuda.empty_cache()
+
+    cpu = finish_oracle_child(oracle_proc) if oracle_proc is not None else None
 
     # ------------------------------------------- NEXT-2: kNN on the tensor cores
     knn = None
@@ -530,7 +679,7 @@ def main():
                    "alpha": inst.alpha, "beta": inst.beta, "gamma": inst.gamma,
                    "parallelism": (f"A-vertex-block shards x{world} (NCCL)" if world > 1 else "single"),
                    "value_unit_note": ("O-equivalent iterations/s: iterations/s x squares / squares(O)"
-                                       if world > 1 else "iterations/s of this instance"),
+                                       if weak else "iterations/s of this instance"),
                    "l2": "inputs larger than L2 (square layout %.2f GB vs 126 MB L2)" % (24 * squares / 1e9),
                    "mode": ("exact" if args.exact else "fast") + ("+fp32S" if args.fp32 else "")},
         "squares_per_s": squares * args.steps / (elapsed_ms / 1e3),
@@ -557,6 +706,7 @@ def main():
         "match_schedule": "rounds" if args.match_rounds else "suitor",
         "step_schedule": step_schedule,
         "next2_knn": knn,
+        "configs": configs,
     }
     print(json.dumps(line), flush=True)
 

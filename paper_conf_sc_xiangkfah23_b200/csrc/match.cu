@@ -152,8 +152,9 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
     while (true) {
         scans++;
         // heaviest eligible neighbour of `cur` whose suitor is lighter; its
-        // target and the slot value seen (the CAS's expected value: 0 on the
-        // unfiltered first scan -- optimistic, a free slot takes one atomic)
+        // target and, on a filtered scan, the slot value seen (the CAS's
+        // expected value; the unfiltered first scan reads the slot first --
+        // an optimistic CAS on an unread slot serialises on popular targets)
         int best = -1, bt = -1;
         double bx = 0.0;
         unsigned long long bs = 0ull;
@@ -189,6 +190,7 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
                 }
             }
         }
+        const bool filtered = filter;
         filter = true;
 #pragma unroll
         for (int off = G / 2; off >= 1; off >>= 1) {
@@ -224,7 +226,7 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
             unsigned long long *slotp = sT + tb;
             const uint32_t kb = suitor_key(bx);
             const unsigned long long mine = ((unsigned long long)kb << 32) | (uint32_t)best;
-            unsigned long long s = bs;
+            unsigned long long s = filtered ? bs : *(volatile unsigned long long *)slotp;
             // CAS loop: retry directly while our edge still beats the occupant,
             // rescan the list only when it does not
             while (beats<DIST>(P, x, k, nT, tb, bx, best, kb, s)) {

@@ -23,9 +23,14 @@ for w in $WHAT; do
     bench)
       timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err
       echo "bench rc=$?"; cut -c1-1500 $OUT/bench.json ;;
+    sanitize)
+      for tool in memcheck racecheck synccheck initcheck; do
+        timeout 1200 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_workload.py > $OUT/sanitize_$tool.txt 2>&1
+        echo "sanitize $tool rc=$?"; tail -4 $OUT/sanitize_$tool.txt
+      done ;;
     ncu_*)
       K=${w#ncu_}
-      timeout 900 ncu --set full --import-source on --clock-control none -k regex:$K -s 40 -c 1 -o $OUT/ncu_$K -f python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn > $OUT/ncu_$K.log 2>&1
+      timeout 900 ncu --set full --import-source on --clock-control none -k regex:$K -s 40 -c 1 -o $OUT/ncu_$K -f python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/ncu_$K.log 2>&1
       echo "ncu $K rc=$?"; tail -3 $OUT/ncu_$K.log ;;
   esac
 done
