@@ -52,6 +52,7 @@ struct MatchParams {
     int32_t *mateA;         // device-side: mates + *wslot * 2 nA (set in the kernels)
     int32_t *mateB;         // [ninst][nB] (transient)
     int2 *mvA;              // (M_y(i), M_z(i)) as B vertices, for evaluate
+    int *qcnt;              // two-phase Suitor: sub-queue counters (reset by k_collect), or null
     RoundDev *rd;
     unsigned long long *work; // proposals (suitor) / rounds, spread counters
     unsigned long long *dbg;  // optional diagnostics (CUALIGN_MATCH_DEBUG)
@@ -65,6 +66,8 @@ struct MatchParams {
 };
 
 constexpr int WORK_SPREAD = 64, WORK_STRIDE = 16; // counter slots, 128 B apart
+constexpr int NQ = 64;          // two-phase Suitor sub-queues (one atomic counter each, 32 B apart)
+constexpr int QSTRIDE = 8;
 
 __device__ __forceinline__ bool better(double xa, int ea, double xb, int eb)
 {
@@ -130,16 +133,14 @@ __device__ __forceinline__ bool beats(const MatchParams &P, const double *__rest
     return better(xe, e, xs, es);
 }
 
+// The proposal chain of one tile: proposer `cur` of instance k proposes
+// (filter0: starting with a filtered scan -- it lost a proposal or was
+// displaced before), and every proposer it displaces continues in the same
+// tile, until a proposal lands in a free slot or a proposer is exhausted.
 template <int G, int U, bool DIST, class Tile>
-__device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
-                                            int64_t nT, int64_t slot)
+__device__ __forceinline__ void suitor_chain(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
+                                             int64_t nT, int k, int cur, bool filter0, int64_t wslot_id)
 {
-    const int k = (int)(slot / nP);
-    int cur = (int)(slot - k * nP);
-    if (DIST) {
-        if (!P.act[slot]) return; // settled (or exhausted) in an earlier round
-        cur += P.p0;
-    }
     const double *__restrict__ x = xk(P, k);
     unsigned long long *sT = P.suit + k * nT;
     const int64_t *__restrict__ rp = fromB ? P.Bptr : P.Arow;
@@ -148,7 +149,7 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
     unsigned long long proposals = 0, scans = 0;
     // the first scan of a proposer skips the suitor filter (its best target
     // is tried directly; a better occupant sends it back to a filtered scan)
-    bool filter = false;
+    bool filter = filter0;
     while (true) {
         scans++;
         // heaviest eligible neighbour of `cur` whose suitor is lighter; its
@@ -251,13 +252,148 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
     }
     // proposal counters spread over WORK_SPREAD slots (one global address
     // would serialise ~10^5 atomics in one L2 slice)
-    if (lane == 0 && proposals) atomicAdd(P.work + (slot % WORK_SPREAD) * WORK_STRIDE + k, proposals);
+    if (lane == 0 && proposals) atomicAdd(P.work + (wslot_id % WORK_SPREAD) * WORK_STRIDE + k, proposals);
     if (P.dbg && lane == 0) {
         atomicMax(P.dbg + 0, scans);
         atomicAdd(P.dbg + 1, scans);
         if (scans > 8) atomicAdd(P.dbg + 2, 1ull);
         if (scans > 64) atomicAdd(P.dbg + 3, 1ull);
         atomicMax(P.dbg + 4, proposals);
+    }
+}
+
+template <int G, int U, bool DIST, class Tile>
+__device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, int lane, bool fromB, int64_t nP,
+                                            int64_t nT, int64_t slot)
+{
+    const int k = (int)(slot / nP);
+    int cur = (int)(slot - k * nP);
+    if (DIST) {
+        if (!P.act[slot]) return; // settled (or exhausted) in an earlier round
+        cur += P.p0;
+    }
+    suitor_chain<G, U, DIST>(P, tile, lane, fromB, nP, nT, k, cur, false, slot);
+}
+
+// ---------------------------------------------- two-phase Suitor (A proposers)
+// Phase 1 (k_propose1): every proposer's FIRST proposal, one thread per
+// (instance, A row): the row (contiguous, ~k entries, L1-reused) is scanned
+// for its best eligible edge and one CAS is tried on that target -- no
+// chains, no tile shuffles, every proposer in flight at once.  A proposer
+// that lost (a better suitor holds the slot) and every proposer displaced by
+// a phase-1 proposal go to a queue; phase 2 (k_suitor_q) runs the ordinary
+// Suitor chains (filtered scans) from the queue.  Any order of proposals
+// reaches the same stable matching (= greedy, pin P9), so the split changes
+// no result.  On config O at p = 80 phase 1 settles 88 % (M_y) / 61 % (M_z)
+// of the proposers (bulk-synchronous count, tools/ analysis in DESIGN.md).
+
+template <int U>
+__global__ void __launch_bounds__(256) k_propose1(MatchParams P, int32_t *__restrict__ queue, int *__restrict__ qcnt,
+                                                  int64_t qcap)
+{
+    pdl_wait();
+    const int64_t nP = P.nA, nT = P.nB;
+    const int64_t slot = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    int push = -1;
+    if (slot < P.ninst * nP) {
+        const int k = (int)(slot / nP);
+        const int cur = (int)(slot - k * nP);
+        const double *__restrict__ x = xk(P, k);
+        unsigned long long *sT = P.suit + k * nT;
+        const int lo = (int)__ldg(P.Arow + cur), hi = (int)__ldg(P.Arow + cur + 1);
+        int best = -1, bt = -1;
+        double bx = 0.0;
+        for (int j0 = lo; j0 < hi; j0 += U) {
+            double xx[U];
+            int tt[U];
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                if (j0 + u < hi) {
+                    xx[u] = __ldg(x + j0 + u);
+                    tt[u] = __ldg(P.Lb + j0 + u);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                const int j = j0 + u;
+                if (j < hi && xx[u] > 0.0 && better(xx[u], j, bx, best)) { // only x > 0 (Z6)
+                    best = j;
+                    bx = xx[u];
+                    bt = tt[u];
+                }
+            }
+        }
+        if (best < 0) {
+            slot_mates(P)[k * nP + cur] = -1; // exhausted (see suitor_chain)
+            set_mv(P.mvA, cur, k, -1);
+        } else {
+            unsigned long long *sp = sT + bt;
+            const uint32_t kb = suitor_key(bx);
+            const unsigned long long mine = ((unsigned long long)kb << 32) | (uint32_t)best;
+            unsigned long long s = *(volatile unsigned long long *)sp;
+            push = (int)(k * nP + cur); // lost: a filtered rescan in phase 2
+            while (beats<false>(P, x, k, nT, bt, bx, best, kb, s)) {
+                const unsigned long long old = atomicCAS(sp, s, mine);
+                if (old == s) {
+                    push = s ? (int)(k * nP + __ldg(P.La + (int)(uint32_t)s)) : -1; // the displaced one
+                    atomicAdd(P.work + (slot % WORK_SPREAD) * WORK_STRIDE + k, 1ull);
+                    break;
+                }
+                s = old;
+            }
+        }
+    }
+    // warp-aggregated push into sub-queue (warp id mod NQ): <= 1 entry per
+    // lane, so sub-queue q holds at most 32 x (warps mapped to it) = qcap
+    const unsigned mask = __ballot_sync(0xffffffffu, push >= 0);
+    if (mask) {
+        const int lane = threadIdx.x & 31;
+        const int leader = __ffs(mask) - 1;
+        const int q = (int)((slot >> 5) % NQ);
+        int base = 0;
+        if (lane == leader) base = atomicAdd(qcnt + q * QSTRIDE, __popc(mask));
+        base = __shfl_sync(0xffffffffu, base, leader);
+        if (push >= 0) queue[q * qcap + base + __popc(mask & ((1u << lane) - 1u))] = push;
+    }
+}
+
+// Phase 2: one wave of G-lane tiles over the queued proposers (static stride
+// over the concatenated sub-queues), each running the Suitor chain.
+template <int G, int U, int MINB>
+__global__ void __launch_bounds__(128, MINB) k_suitor_q(MatchParams P, const int32_t *__restrict__ queue,
+                                                        const int *__restrict__ qcnt, int64_t qcap)
+{
+    __shared__ int s_off[NQ + 1];
+    pdl_wait();
+    if (threadIdx.x < 32) {
+        // exclusive prefix of the NQ counts (one warp, two per lane)
+        const int c0 = qcnt[(2 * threadIdx.x) * QSTRIDE], c1 = qcnt[(2 * threadIdx.x + 1) * QSTRIDE];
+        int v = c0 + c1;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const int o = __shfl_up_sync(0xffffffffu, v, off);
+            if ((int)threadIdx.x >= off) v += o;
+        }
+        s_off[2 * threadIdx.x + 1] = v - c1;
+        s_off[2 * threadIdx.x + 2] = v;
+        if (threadIdx.x == 0) s_off[0] = 0;
+    }
+    __syncthreads();
+    auto tile = cg::tiled_partition<G>(cg::this_thread_block());
+    const int lane = tile.thread_rank();
+    const int64_t nP = P.nA, nT = P.nB;
+    const int total = s_off[NQ];
+    const int T = (int)(((int64_t)gridDim.x * blockDim.x) / G);
+    for (int idx = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G); idx < total; idx += T) {
+        int lo = 0, hi = NQ; // sub-queue q with s_off[q] <= idx < s_off[q + 1]
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (s_off[mid] <= idx) lo = mid;
+            else hi = mid;
+        }
+        const int v = __ldg(queue + lo * qcap + (idx - s_off[lo]));
+        const int k = (int)(v / nP);
+        suitor_chain<G, U, false>(P, tile, lane, false, nP, nT, k, (int)(v - k * nP), true, idx);
     }
 }
 
@@ -393,6 +529,7 @@ __global__ void k_collect(MatchParams P, int64_t nT, int64_t nP, int fromB)
 {
     pdl_wait();
     if (blockIdx.x == 0 && threadIdx.x < 4) (&P.rd->overlap[0])[threadIdx.x] = 0ull; // overlap[2], card[2]
+    if (P.qcnt && blockIdx.x == 0 && threadIdx.x < NQ) P.qcnt[threadIdx.x * QSTRIDE] = 0; // queues: next round
     int32_t *mateA = slot_mates(P);
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < P.ninst * nT;
          v += (int64_t)gridDim.x * blockDim.x) {
@@ -811,7 +948,24 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
         CA_CUDA(cudaMemsetAsync(dbuf, 0, 8 * sizeof(unsigned long long), h->stream));
         P.dbg = dbuf;
     }
-    if (slots > 0) {
+    static const int two_env = probe_knob("CUALIGN_SUITOR_TWOPHASE", 1);
+    const bool two = two_env && !fromB && h->max_deg_a <= 64 && h->squeue && !dbg;
+    if (two && slots > 0) {
+        // two-phase Suitor (see k_propose1): first proposals thread per row,
+        // then the queued proposers' chains in one wave of 4-lane tiles
+        P.qcnt = h->qcnt;
+        KScope ks(h, CUALIGN_K_MATCH);
+        CA_CUDA(launch_pdl(k_propose1<6>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P, h->squeue,
+                           h->qcnt, h->qcap));
+        static const int q2_minb = probe_knob("CUALIGN_SUITOR_Q_MINB", 8);
+        if (q2_minb == 12)
+            CA_CUDA(launch_pdl(k_suitor_q<4, 5, 12>, dim3(h->q2_grid * 12 / 8), dim3(128), 0, h->stream, P,
+                               (const int32_t *)h->squeue, (const int *)h->qcnt, h->qcap));
+        else
+            CA_CUDA(launch_pdl(k_suitor_q<4, 5, 8>, dim3(h->q2_grid), dim3(128), 0, h->stream, P,
+                               (const int32_t *)h->squeue, (const int *)h->qcnt, h->qcap));
+        CA_CUDA(cudaGetLastError());
+    } else if (slots > 0) {
         KScope ks(h, CUALIGN_K_MATCH);
         const int64_t dmax = fromB ? h->max_deg_b : h->max_deg_a;
         static const int genv = probe_knob("CUALIGN_SUITOR_G", 0);
@@ -927,6 +1081,21 @@ cualign_status match_setup(cualign_bp *h)
         h->eval_grid = grid_for(h->nApairs > (int64_t)nA ? h->nApairs : (int64_t)nA, 256, h->num_sms * occ);
     }
     CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * h->eval_grid));
+    {
+        // two-phase Suitor queues: sub-queue q collects the pushes of the
+        // phase-1 warps w with w mod NQ = q, <= 32 per warp
+        const int64_t nwarps = ((int64_t)2 * nA + 31) / 32;
+        h->qcap = 32 * ((nwarps + NQ - 1) / NQ);
+        CA_TRY(dalloc(h, &h->squeue, (size_t)(NQ * h->qcap)));
+        CA_TRY(dalloc(h, &h->qcnt, (size_t)NQ * QSTRIDE));
+        CA_CUDA(cudaMemsetAsync(h->qcnt, 0, sizeof(int) * NQ * QSTRIDE, h->stream));
+        int occ2 = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_suitor_q<4, 5, 8>, 128, 0) != cudaSuccess ||
+            occ2 < 1)
+            occ2 = 1;
+        (void)cudaGetLastError();
+        h->q2_grid = occ2 * h->num_sms;
+    }
     return CUALIGN_OK;
 }
 

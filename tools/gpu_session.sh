@@ -20,6 +20,11 @@ for w in $WHAT; do
     parts)
       timeout 300 python tools/bench_parts.py --pre 80 --n 50 > $OUT/parts.json 2> $OUT/parts.err
       echo "parts rc=$?"; cat $OUT/parts.json ;;
+    pp_*)
+      # parts with the probe build and env assignments: pp_NAME=VAL,NAME2=VAL2
+      ENVS=$(echo ${w#pp_} | tr ',' ' ')
+      env CUALIGN_LIB=$PROBES $ENVS timeout 300 python tools/bench_parts.py --pre 80 --n 50 > $OUT/parts_${w}.json 2> $OUT/parts_${w}.err
+      echo "$w rc=$?"; cat $OUT/parts_${w}.json ;;
     bench)
       timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err
       echo "bench rc=$?"; cut -c1-1500 $OUT/bench.json ;;
