@@ -33,6 +33,14 @@ for w in $WHAT; do
         timeout 1200 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_workload.py > $OUT/sanitize_$tool.txt 2>&1
         echo "sanitize $tool rc=$?"; tail -4 $OUT/sanitize_$tool.txt
       done ;;
+    nculist)
+      # launch list (cold-cache, serialised) of a round-only replay at a fixed state
+      timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"k_propose1|k_suitor|k_collect|k_eval|k_mate" -s 300 -c 60 --csv --log-file $OUT/launches_round.csv python tools/bench_parts.py --pre 80 --n 20 > $OUT/nculist.log 2>&1
+      echo "nculist rc=$?"; python tools/launches.py $OUT/launches_round.csv 2>/dev/null | head -20 ;;
+    ncuparts_*)
+      K=${w#ncuparts_}
+      timeout 900 ncu --set full --import-source on --clock-control none -k regex:$K -s 100 -c 1 -o $OUT/ncu_$K -f python tools/bench_parts.py --pre 80 --n 10 > $OUT/ncu_$K.log 2>&1
+      echo "ncu $K rc=$?"; tail -2 $OUT/ncu_$K.log ;;
     ncu_*)
       K=${w#ncu_}
       timeout 900 ncu --set full --import-source on --clock-control none -k regex:$K -s 40 -c 1 -o $OUT/ncu_$K -f python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/ncu_$K.log 2>&1
