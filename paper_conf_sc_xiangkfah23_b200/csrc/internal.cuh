@@ -198,10 +198,11 @@ struct cualign_bp {
     double *partial_w = nullptr;
     int match_grid = 0, match_block = 256, eval_grid = 1;
     unsigned long long *match_work = nullptr; // proposals (suitor) or rounds, per instance
-    int32_t *squeue = nullptr;                // two-phase Suitor: queued proposers (NQ sub-queues of qcap)
+    int32_t *squeue = nullptr;                // Suitor rounds: queued proposers (3 buffers x NQ sub-queues of qcap)
     int *qcnt = nullptr;                      // sub-queue counters
     int64_t qcap = 0;
-    int q2_grid = 1;                          // phase-2 grid (one wave)
+    int q2_grid = 1;                          // chain-form grid (one wave)
+    int qr_grid = 1;                          // proposal-round grid (one wave)
     bool propose_from_b = false;              // suitor: proposing side (smaller max degree)
     // graphs A and B (CSR), kept for evaluate: overlap = #A edges {i,j} with
     // (M(i), M(j)) in E_B

@@ -52,7 +52,7 @@ struct MatchParams {
     int32_t *mateA;         // device-side: mates + *wslot * 2 nA (set in the kernels)
     int32_t *mateB;         // [ninst][nB] (transient)
     int2 *mvA;              // (M_y(i), M_z(i)) as B vertices, for evaluate
-    int *qcnt;              // two-phase Suitor: sub-queue counters (reset by k_collect), or null
+    int *qcnt;              // Suitor rounds: sub-queue counters (reset by k_collect), or null
     RoundDev *rd;
     unsigned long long *work; // proposals (suitor) / rounds, spread counters
     unsigned long long *dbg;  // optional diagnostics (CUALIGN_MATCH_DEBUG)
@@ -66,7 +66,7 @@ struct MatchParams {
 };
 
 constexpr int WORK_SPREAD = 64, WORK_STRIDE = 16; // counter slots, 128 B apart
-constexpr int NQ = 64;          // two-phase Suitor sub-queues (one atomic counter each, 32 B apart)
+constexpr int NQ = 64;          // Suitor-round sub-queues (one atomic counter each, 32 B apart)
 constexpr int QSTRIDE = 8;
 
 __device__ __forceinline__ bool better(double xa, int ea, double xb, int eb)
@@ -275,98 +275,44 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
     suitor_chain<G, U, DIST>(P, tile, lane, fromB, nP, nT, k, cur, false, slot);
 }
 
-// ---------------------------------------------- two-phase Suitor (A proposers)
-// Phase 1 (k_propose1): every proposer's FIRST proposal, one thread per
-// (instance, A row): the row (contiguous, ~k entries, L1-reused) is scanned
-// for its best eligible edge and one CAS is tried on that target -- no
-// chains, no tile shuffles, every proposer in flight at once.  A proposer
-// that lost (a better suitor holds the slot) and every proposer displaced by
-// a phase-1 proposal go to a queue; phase 2 (k_suitor_q) runs the ordinary
-// Suitor chains (filtered scans) from the queue.  Any order of proposals
-// reaches the same stable matching (= greedy, pin P9), so the split changes
-// no result.  On config O at p = 80 phase 1 settles 88 % (M_y) / 61 % (M_z)
-// of the proposers (bulk-synchronous count, tools/ analysis in DESIGN.md).
+// ------------------------------------- Suitor in proposal rounds (A proposers)
+// Round 0 (k_propose_round<FIRST>): every proposer's FIRST proposal, one
+// thread per (instance, A row): the row (contiguous, ~k entries, L1-reused)
+// is scanned for its best eligible edge and a CAS tries that target.
+// Rounds 1..R: one thread per queued proposer -- those that lost a CAS to a
+// better suitor and those a proposal displaced -- scanning its row for the
+// best target whose CURRENT suitor it beats (filtered scan) and proposing.
+// A thread never follows a displacement chain: the displaced proposer goes to
+// the next round's queue, so every round is a flat pass with all its
+// proposers in flight at once (no tile divergence, no chain tails).  Whatever
+// is still queued after round R runs the chain form (k_suitor_q).  Any order
+// of proposals reaches the same stable matching (= greedy, pin P9), so the
+// schedule changes no result.  Config O, p = 80 (bulk-synchronous count):
+// round 0 settles 87 % (M_y) / 61 % (M_z) of the proposers, 10 rounds settle
+// all.  Queues: 3 buffers of NQ sub-queues (sub-queue = 32-entry chunk index
+// mod NQ, one warp-aggregated atomic per chunk); round r reads buffer r % 3,
+// writes (r + 1) % 3 and clears the counters of (r + 2) % 3, which round
+// r + 1 writes (k_collect clears all of them for the next rounding).
+constexpr int QBUF = 3;
 
-template <int U>
-__global__ void __launch_bounds__(256) k_propose1(MatchParams P, int32_t *__restrict__ queue, int *__restrict__ qcnt,
-                                                  int64_t qcap)
+__device__ __forceinline__ void queue_push(int push, int64_t chunk, int32_t *__restrict__ queue,
+                                           int *__restrict__ qcnt, int64_t qcap)
 {
-    pdl_wait();
-    const int64_t nP = P.nA, nT = P.nB;
-    const int64_t slot = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    int push = -1;
-    if (slot < P.ninst * nP) {
-        const int k = (int)(slot / nP);
-        const int cur = (int)(slot - k * nP);
-        const double *__restrict__ x = xk(P, k);
-        unsigned long long *sT = P.suit + k * nT;
-        const int lo = (int)__ldg(P.Arow + cur), hi = (int)__ldg(P.Arow + cur + 1);
-        int best = -1, bt = -1;
-        double bx = 0.0;
-        for (int j0 = lo; j0 < hi; j0 += U) {
-            double xx[U];
-            int tt[U];
-#pragma unroll
-            for (int u = 0; u < U; u++) {
-                if (j0 + u < hi) {
-                    xx[u] = __ldg(x + j0 + u);
-                    tt[u] = __ldg(P.Lb + j0 + u);
-                }
-            }
-#pragma unroll
-            for (int u = 0; u < U; u++) {
-                const int j = j0 + u;
-                if (j < hi && xx[u] > 0.0 && better(xx[u], j, bx, best)) { // only x > 0 (Z6)
-                    best = j;
-                    bx = xx[u];
-                    bt = tt[u];
-                }
-            }
-        }
-        if (best < 0) {
-            slot_mates(P)[k * nP + cur] = -1; // exhausted (see suitor_chain)
-            set_mv(P.mvA, cur, k, -1);
-        } else {
-            unsigned long long *sp = sT + bt;
-            const uint32_t kb = suitor_key(bx);
-            const unsigned long long mine = ((unsigned long long)kb << 32) | (uint32_t)best;
-            unsigned long long s = *(volatile unsigned long long *)sp;
-            push = (int)(k * nP + cur); // lost: a filtered rescan in phase 2
-            while (beats<false>(P, x, k, nT, bt, bx, best, kb, s)) {
-                const unsigned long long old = atomicCAS(sp, s, mine);
-                if (old == s) {
-                    push = s ? (int)(k * nP + __ldg(P.La + (int)(uint32_t)s)) : -1; // the displaced one
-                    atomicAdd(P.work + (slot % WORK_SPREAD) * WORK_STRIDE + k, 1ull);
-                    break;
-                }
-                s = old;
-            }
-        }
-    }
-    // warp-aggregated push into sub-queue (warp id mod NQ): <= 1 entry per
-    // lane, so sub-queue q holds at most 32 x (warps mapped to it) = qcap
     const unsigned mask = __ballot_sync(0xffffffffu, push >= 0);
-    if (mask) {
-        const int lane = threadIdx.x & 31;
-        const int leader = __ffs(mask) - 1;
-        const int q = (int)((slot >> 5) % NQ);
-        int base = 0;
-        if (lane == leader) base = atomicAdd(qcnt + q * QSTRIDE, __popc(mask));
-        base = __shfl_sync(0xffffffffu, base, leader);
-        if (push >= 0) queue[q * qcap + base + __popc(mask & ((1u << lane) - 1u))] = push;
-    }
+    if (!mask) return;
+    const int lane = threadIdx.x & 31;
+    const int leader = __ffs(mask) - 1;
+    const int q = (int)(chunk % NQ);
+    int base = 0;
+    if (lane == leader) base = atomicAdd(qcnt + q * QSTRIDE, __popc(mask));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    if (push >= 0) queue[q * qcap + base + __popc(mask & ((1u << lane) - 1u))] = push;
 }
 
-// Phase 2: one wave of G-lane tiles over the queued proposers (static stride
-// over the concatenated sub-queues), each running the Suitor chain.
-template <int G, int U, int MINB>
-__global__ void __launch_bounds__(128, MINB) k_suitor_q(MatchParams P, const int32_t *__restrict__ queue,
-                                                        const int *__restrict__ qcnt, int64_t qcap)
+// exclusive prefix of the NQ sub-queue counts into s_off[0..NQ] (one warp)
+__device__ __forceinline__ void queue_offsets(const int *__restrict__ qcnt, int *s_off)
 {
-    __shared__ int s_off[NQ + 1];
-    pdl_wait();
     if (threadIdx.x < 32) {
-        // exclusive prefix of the NQ counts (one warp, two per lane)
         const int c0 = qcnt[(2 * threadIdx.x) * QSTRIDE], c1 = qcnt[(2 * threadIdx.x + 1) * QSTRIDE];
         int v = c0 + c1;
 #pragma unroll
@@ -379,19 +325,138 @@ __global__ void __launch_bounds__(128, MINB) k_suitor_q(MatchParams P, const int
         if (threadIdx.x == 0) s_off[0] = 0;
     }
     __syncthreads();
+}
+
+__device__ __forceinline__ int queue_at(const int32_t *__restrict__ queue, const int *s_off, int64_t qcap, int idx)
+{
+    int lo = 0, hi = NQ; // sub-queue q with s_off[q] <= idx < s_off[q + 1]
+    while (hi - lo > 1) {
+        const int mid = (lo + hi) >> 1;
+        if (s_off[mid] <= idx) lo = mid;
+        else hi = mid;
+    }
+    return __ldg(queue + lo * qcap + (idx - s_off[lo]));
+}
+
+// One proposal of proposer `cur` of instance k (row scan, filtered unless
+// FIRST, CAS); returns the proposer to queue for the next round (itself if it
+// lost, the displaced one if it displaced a suitor) or -1.
+template <int U, bool FIRST>
+__device__ __forceinline__ int propose_once(const MatchParams &P, int64_t nP, int64_t nT, int k, int cur,
+                                            int64_t work_id)
+{
+    const double *__restrict__ x = xk(P, k);
+    unsigned long long *sT = P.suit + k * nT;
+    const int lo = (int)__ldg(P.Arow + cur), hi = (int)__ldg(P.Arow + cur + 1);
+    int best = -1, bt = -1;
+    double bx = 0.0;
+    unsigned long long bs = 0ull;
+    for (int j0 = lo; j0 < hi; j0 += U) {
+        double xx[U];
+        int tt[U];
+        unsigned long long ss[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            if (j0 + u < hi) {
+                xx[u] = __ldg(x + j0 + u);
+                tt[u] = __ldg(P.Lb + j0 + u);
+            }
+        }
+        if (!FIRST) {
+#pragma unroll
+            for (int u = 0; u < U; u++)
+                ss[u] = (j0 + u < hi && xx[u] > 0.0) ? *(volatile unsigned long long *)(sT + tt[u]) : 0ull;
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const int j = j0 + u;
+            if (j >= hi || !(xx[u] > 0.0)) continue; // only x > 0 is eligible (Z6)
+            if (!FIRST && !beats<false>(P, x, k, nT, tt[u], xx[u], j, suitor_key(xx[u]), ss[u])) continue;
+            if (better(xx[u], j, bx, best)) {
+                best = j;
+                bx = xx[u];
+                bt = tt[u];
+                bs = FIRST ? 0ull : ss[u];
+            }
+        }
+    }
+    if (best < 0) {
+        slot_mates(P)[k * nP + cur] = -1; // exhausted (see suitor_chain)
+        set_mv(P.mvA, cur, k, -1);
+        return -1;
+    }
+    unsigned long long *sp = sT + bt;
+    const uint32_t kb = suitor_key(bx);
+    const unsigned long long mine = ((unsigned long long)kb << 32) | (uint32_t)best;
+    unsigned long long s = FIRST ? *(volatile unsigned long long *)sp : bs;
+    while (beats<false>(P, x, k, nT, bt, bx, best, kb, s)) {
+        const unsigned long long old = atomicCAS(sp, s, mine);
+        if (old == s) {
+            atomicAdd(P.work + (work_id % WORK_SPREAD) * WORK_STRIDE + k, 1ull);
+            return s ? (int)(k * nP + __ldg(P.La + (int)(uint32_t)s)) : -1; // the displaced one
+        }
+        s = old;
+    }
+    return (int)(k * nP + cur); // lost: next round
+}
+
+template <int U>
+__global__ void __launch_bounds__(256) k_propose_first(MatchParams P, int32_t *__restrict__ qout,
+                                                       int *__restrict__ cout, int64_t qcap)
+{
+    pdl_wait();
+    const int64_t nP = P.nA, nT = P.nB;
+    const int64_t slot = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    int push = -1;
+    if (slot < P.ninst * nP) {
+        const int k = (int)(slot / nP);
+        push = propose_once<U, true>(P, nP, nT, k, (int)(slot - k * nP), slot);
+    }
+    queue_push(push, slot >> 5, qout, cout, qcap);
+}
+
+template <int U>
+__global__ void __launch_bounds__(256) k_propose_round(MatchParams P, const int32_t *__restrict__ qin,
+                                                       const int *__restrict__ cin, int32_t *__restrict__ qout,
+                                                       int *__restrict__ cout, int *__restrict__ cclr, int64_t qcap)
+{
+    __shared__ int s_off[NQ + 1];
+    pdl_wait();
+    if (blockIdx.x == 0 && threadIdx.x < NQ) cclr[threadIdx.x * QSTRIDE] = 0;
+    queue_offsets(cin, s_off);
+    const int total = s_off[NQ];
+    const int64_t nP = P.nA, nT = P.nB;
+    const int64_t gwarp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t base = gwarp * 32; base < total; base += nwarps * 32) {
+        const int idx = (int)(base + (threadIdx.x & 31));
+        int push = -1;
+        if (idx < total) {
+            const int v = queue_at(qin, s_off, qcap, idx);
+            const int k = (int)(v / nP);
+            push = propose_once<U, false>(P, nP, nT, k, (int)(v - k * nP), idx);
+        }
+        queue_push(push, base >> 5, qout, cout, qcap);
+    }
+}
+
+// After the last round: one wave of G-lane tiles over what is still queued,
+// each running the Suitor chain (displaced proposers continue in the tile)
+// until the matching is complete.
+template <int G, int U, int MINB>
+__global__ void __launch_bounds__(128, MINB) k_suitor_q(MatchParams P, const int32_t *__restrict__ queue,
+                                                        const int *__restrict__ qcnt, int64_t qcap)
+{
+    __shared__ int s_off[NQ + 1];
+    pdl_wait();
+    queue_offsets(qcnt, s_off);
     auto tile = cg::tiled_partition<G>(cg::this_thread_block());
     const int lane = tile.thread_rank();
     const int64_t nP = P.nA, nT = P.nB;
     const int total = s_off[NQ];
     const int T = (int)(((int64_t)gridDim.x * blockDim.x) / G);
     for (int idx = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G); idx < total; idx += T) {
-        int lo = 0, hi = NQ; // sub-queue q with s_off[q] <= idx < s_off[q + 1]
-        while (hi - lo > 1) {
-            const int mid = (lo + hi) >> 1;
-            if (s_off[mid] <= idx) lo = mid;
-            else hi = mid;
-        }
-        const int v = __ldg(queue + lo * qcap + (idx - s_off[lo]));
+        const int v = queue_at(queue, s_off, qcap, idx);
         const int k = (int)(v / nP);
         suitor_chain<G, U, false>(P, tile, lane, false, nP, nT, k, (int)(v - k * nP), true, idx);
     }
@@ -529,7 +594,7 @@ __global__ void k_collect(MatchParams P, int64_t nT, int64_t nP, int fromB)
 {
     pdl_wait();
     if (blockIdx.x == 0 && threadIdx.x < 4) (&P.rd->overlap[0])[threadIdx.x] = 0ull; // overlap[2], card[2]
-    if (P.qcnt && blockIdx.x == 0 && threadIdx.x < NQ) P.qcnt[threadIdx.x * QSTRIDE] = 0; // queues: next round
+    if (P.qcnt && blockIdx.x == 0 && threadIdx.x < QBUF * NQ) P.qcnt[threadIdx.x * QSTRIDE] = 0; // next rounding
     int32_t *mateA = slot_mates(P);
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < P.ninst * nT;
          v += (int64_t)gridDim.x * blockDim.x) {
@@ -948,22 +1013,26 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
         CA_CUDA(cudaMemsetAsync(dbuf, 0, 8 * sizeof(unsigned long long), h->stream));
         P.dbg = dbuf;
     }
-    static const int two_env = probe_knob("CUALIGN_SUITOR_TWOPHASE", 1);
+    static const int two_env = probe_knob("CUALIGN_SUITOR_QROUNDS", 1);
     const bool two = two_env && !fromB && h->max_deg_a <= 64 && h->squeue && !dbg;
     if (two && slots > 0) {
-        // two-phase Suitor (see k_propose1): first proposals thread per row,
-        // then the queued proposers' chains in one wave of 4-lane tiles
+        // proposal rounds (see k_propose_round), then the chain form for
+        // whatever is still queued
         P.qcnt = h->qcnt;
         KScope ks(h, CUALIGN_K_MATCH);
-        CA_CUDA(launch_pdl(k_propose1<6>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P, h->squeue,
-                           h->qcnt, h->qcap));
-        static const int q2_minb = probe_knob("CUALIGN_SUITOR_Q_MINB", 8);
-        if (q2_minb == 12)
-            CA_CUDA(launch_pdl(k_suitor_q<4, 5, 12>, dim3(h->q2_grid * 12 / 8), dim3(128), 0, h->stream, P,
-                               (const int32_t *)h->squeue, (const int *)h->qcnt, h->qcap));
-        else
-            CA_CUDA(launch_pdl(k_suitor_q<4, 5, 8>, dim3(h->q2_grid), dim3(128), 0, h->stream, P,
-                               (const int32_t *)h->squeue, (const int *)h->qcnt, h->qcap));
+        const int64_t qc = h->qcap, cs = (int64_t)NQ * QSTRIDE;
+        static const int nrounds = probe_knob("CUALIGN_SUITOR_ROUNDS", 6);
+        CA_CUDA(launch_pdl(k_propose_first<6>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P,
+                           h->squeue + 1 * NQ * qc, h->qcnt + 1 * cs, qc));
+        for (int r = 1; r <= nrounds; r++) {
+            const int bi = r % QBUF, bo = (r + 1) % QBUF, bc = (r + 2) % QBUF;
+            CA_CUDA(launch_pdl(k_propose_round<6>, dim3(h->qr_grid), dim3(256), 0, h->stream, P,
+                               (const int32_t *)(h->squeue + bi * NQ * qc), (const int *)(h->qcnt + bi * cs),
+                               h->squeue + bo * NQ * qc, h->qcnt + bo * cs, h->qcnt + bc * cs, qc));
+        }
+        const int bl = (nrounds + 1) % QBUF;
+        CA_CUDA(launch_pdl(k_suitor_q<4, 5, 8>, dim3(h->q2_grid), dim3(128), 0, h->stream, P,
+                           (const int32_t *)(h->squeue + bl * NQ * qc), (const int *)(h->qcnt + bl * cs), qc));
         CA_CUDA(cudaGetLastError());
     } else if (slots > 0) {
         KScope ks(h, CUALIGN_K_MATCH);
@@ -1082,13 +1151,19 @@ cualign_status match_setup(cualign_bp *h)
     }
     CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * h->eval_grid));
     {
-        // two-phase Suitor queues: sub-queue q collects the pushes of the
+        // Suitor-round queues: sub-queue q collects the pushes of the
         // phase-1 warps w with w mod NQ = q, <= 32 per warp
         const int64_t nwarps = ((int64_t)2 * nA + 31) / 32;
         h->qcap = 32 * ((nwarps + NQ - 1) / NQ);
-        CA_TRY(dalloc(h, &h->squeue, (size_t)(NQ * h->qcap)));
-        CA_TRY(dalloc(h, &h->qcnt, (size_t)NQ * QSTRIDE));
-        CA_CUDA(cudaMemsetAsync(h->qcnt, 0, sizeof(int) * NQ * QSTRIDE, h->stream));
+        CA_TRY(dalloc(h, &h->squeue, (size_t)(QBUF * NQ * h->qcap)));
+        CA_TRY(dalloc(h, &h->qcnt, (size_t)QBUF * NQ * QSTRIDE));
+        CA_CUDA(cudaMemsetAsync(h->qcnt, 0, sizeof(int) * QBUF * NQ * QSTRIDE, h->stream));
+        int occr = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occr, k_propose_round<6>, 256, 0) != cudaSuccess ||
+            occr < 1)
+            occr = 1;
+        (void)cudaGetLastError();
+        h->qr_grid = occr * h->num_sms;
         int occ2 = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_suitor_q<4, 5, 8>, 128, 0) != cudaSuccess ||
             occ2 < 1)
