@@ -33,9 +33,15 @@ for w in $WHAT; do
         timeout 1200 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_workload.py > $OUT/sanitize_$tool.txt 2>&1
         echo "sanitize $tool rc=$?"; tail -4 $OUT/sanitize_$tool.txt
       done ;;
+    kern*)
+      # in-situ per-kernel durations (CUPTI via torch.profiler); kern or kern_ENV=V,ENV2=V
+      ENVS=""; LIBENV=""
+      if [ "$w" != "kern" ]; then ENVS=$(echo ${w#kern_} | tr ',' ' '); LIBENV="CUALIGN_LIB=$PROBES"; fi
+      env $LIBENV $ENVS timeout 300 python tools/probe_kernels.py --pre 80 --n 20 > $OUT/$w.json 2> $OUT/$w.err
+      echo "$w rc=$?"; python -c "import json,sys; d=json.load(open('$OUT/$w.json')); [print(p, {k: round(v['us_per_step'],1) for k,v in d[p].items()}) for p in d]" ;;
     nculist)
       # launch list (cold-cache, serialised) of a round-only replay at a fixed state
-      timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"k_propose1|k_suitor|k_collect|k_eval|k_mate" -s 300 -c 60 --csv --log-file $OUT/launches_round.csv python tools/bench_parts.py --pre 80 --n 20 > $OUT/nculist.log 2>&1
+      timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"k_propose|k_suitor|k_collect|k_eval|k_mate" -s 100 -c 60 --csv --log-file $OUT/launches_round.csv python tools/bench_parts.py --pre 80 --n 20 > $OUT/nculist.log 2>&1
       echo "nculist rc=$?"; python tools/launches.py $OUT/launches_round.csv 2>/dev/null | head -20 ;;
     ncuparts_*)
       K=${w#ncuparts_}
