@@ -41,8 +41,8 @@ def main():
         for ev in prof.events():
             if ev.device_type.name != "CUDA":
                 continue
-            nm = ev.name.split("(")[0].replace("cualign::", "").replace("(anonymous namespace)::", "")
-            nm = nm.replace("void ", "")[:60]
+            nm = ev.name.replace("(anonymous namespace)::", "").replace("cualign::", "").replace("void ", "")
+            nm = nm.split("(")[0][:60]
             agg[nm][0] += 1
             agg[nm][1] += ev.device_time_total if hasattr(ev, "device_time_total") else ev.cuda_time_total
         out[name] = {k: {"n_per_step": v[0] / args.n, "us_per_step": v[1] / args.n} for k, v in
