@@ -207,8 +207,6 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
     h->top2_tg = 1;
     double *yc0 = h->yc, *zc0 = h->zc;
     double *yb[2] = {yc0, h->yc_b1}, *zb[2] = {zc0, h->zc_b1};
-    int32_t *pr0 = h->prop;
-    int32_t *pb[2] = {pr0, h->prop_b1}; // the rounding head start travels with y^c, z^c
     cualign_status st = CUALIGN_OK;
     auto round_of = [&](int buf) -> cualign_status {
         // the rounding reports its own iteration counter (rp = iteration
@@ -220,7 +218,6 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
         }
         h->yc = yb[buf];
         h->zc = zb[buf];
-        h->prop = pb[buf];
         h->round_p = h->rp_dev;
         cualign_status r = match_round(h);
         h->round_p = nullptr;
@@ -234,7 +231,6 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
         }
         h->yc = yb[wb];
         h->zc = zb[wb];
-        h->prop = pb[wb];
         if (st == CUALIGN_OK) st = bp_iterate(h, 1);
     } else if (kind == 1) {
         // fork: the rounding of iteration p-1 (buffer 1-wb) beside all of
@@ -250,7 +246,6 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
         }
         h->yc = yb[wb];
         h->zc = zb[wb];
-        h->prop = pb[wb];
         if (st == CUALIGN_OK) st = bp_iterate(h, 1);
         if (st == CUALIGN_OK && (cudaEventRecord(h->fork_ev[1], h->gstream2) != cudaSuccess ||
                                  cudaStreamWaitEvent(h->gstream, h->fork_ev[1], 0) != cudaSuccess))
@@ -260,7 +255,6 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
     }
     h->yc = yc0;
     h->zc = zc0;
-    h->prop = pr0;
     return st;
 }
 
@@ -392,10 +386,6 @@ static cualign_status alloc_pipeline(cualign_bp *h)
 {
     CA_TRY(dalloc(h, &h->yc_b1, (size_t)h->L.m + 1));
     CA_TRY(dalloc(h, &h->zc_b1, (size_t)h->L.m + 1));
-    if (h->prop) {
-        CA_TRY(dalloc(h, &h->prop_b1, 2 * (size_t)h->L.nA + 1));
-        CA_CUDA(cudaMemsetAsync(h->prop_b1, 0xFE, sizeof(int32_t) * (2 * (size_t)h->L.nA + 1), h->stream));
-    }
     CA_TRY(dalloc(h, &h->rp_dev, 1));
     return CUALIGN_OK;
 }
@@ -586,12 +576,6 @@ static cualign_status alloc_state(cualign_bp *h)
         CA_CUDA(cudaMemsetAsync(*p, 0, sizeof(double) * (m ? m : 1), h->stream));
     }
     init_trace(h, "state vectors");
-    // the rounding's head start (k_edge's per-row best edges); dropped again
-    // by match_setup when the Suitor rounds do not apply (B-side proposers)
-    if (h->world == 1 && !(h->flags & (CUALIGN_FLAG_MATCH_ROUNDS | CUALIGN_FLAG_EXACT))) {
-        CA_TRY(dalloc(h, &h->prop, 2 * (size_t)h->L.nA + 1));
-        CA_CUDA(cudaMemsetAsync(h->prop, 0xFE, sizeof(int32_t) * (2 * (size_t)h->L.nA + 1), h->stream)); // PROP_SCAN
-    }
     if (h->world == 1 && !(h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS)))
         CA_TRY(alloc_pipeline(h));
     init_trace(h, "pipeline buffers");
@@ -1097,9 +1081,6 @@ cualign_status cualign_bp_set_state(cualign_bp *h, const double *yp, const doubl
         CA_TRY(st);
     }
     h->p = p;
-    // the rounding's head start no longer describes the messages: scan rows
-    for (int32_t *pr : {h->prop, h->prop_b1})
-        if (pr) CA_CUDA(cudaMemsetAsync(pr, 0xFE, sizeof(int32_t) * (2 * (size_t)h->L.nA + 1), h->stream));
     CA_TRY(ensure_gh(h, (int64_t)p + 1));
     CA_CUDA(cudaMemcpyAsync(h->p_dev, &h->p, sizeof(int), cudaMemcpyHostToDevice, h->stream));
     CA_TRY(bp_fsum(h));

@@ -185,24 +185,11 @@ struct EdgeArgs {
     const double *texact;
     const double2 *Atop, *Btop;
     double *yp, *zp, *yc, *zc, *d, *u;
-    // a7 head start: per A row, the best edge of the
-    // vectors the rounding takes (y^c, z^c; y^p, z^p with ROUND_DAMPED) by
-    // (x desc, id asc) among x > 0: prop[k * nA + a] = edge, -1 none,
-    // PROP_SCAN the row crosses this block's edge range (the rounding scans it)
-    int32_t *prop;
-    const int64_t *Arow;
-    int64_t nA;
-    int damped;
 };
 
-constexpr int EDGE_BLOCK = 256;
-
-template <int EPT, bool EXACT, bool LITERAL, int MINB = 1, bool PROP = false>
+template <int EPT, bool EXACT, bool LITERAL, int MINB = 1>
 __global__ void __launch_bounds__(256, MINB) k_edge(EdgeArgs R)
 {
-    // PROP: the block's rounding values and A vertices staged for the row argmax
-    __shared__ double s_xy[PROP ? EPT * EDGE_BLOCK : 1], s_xz[PROP ? EPT * EDGE_BLOCK : 1];
-    __shared__ int s_a[PROP ? EPT * EDGE_BLOCK : 1];
     pdl_wait();
     const int64_t base = R.e0 + (int64_t)blockIdx.x * blockDim.x * EPT + threadIdx.x;
     const double2 ghp = R.gh[*R.p_dev];
@@ -245,39 +232,6 @@ __global__ void __launch_bounds__(256, MINB) k_edge(EdgeArgs R)
         R.d[e[j]] = de;
         R.u[e[j]] = ue;
         if (!EXACT) R.tacc[e[j]] = 0ull; // ready for this iteration's k_square
-        if (PROP) {
-            const int li = threadIdx.x + j * EDGE_BLOCK;
-            s_xy[li] = R.damped ? g * yce + hh * ype[j] : yce;
-            s_xz[li] = R.damped ? g * zce + hh * zpe[j] : zce;
-        }
-    }
-    if (PROP) {
-#pragma unroll
-        for (int j = 0; j < EPT; j++) s_a[threadIdx.x + j * EDGE_BLOCK] = e[j] < R.e1 ? a[j] : -1;
-        __syncthreads();
-        const int64_t b0 = R.e0 + (int64_t)blockIdx.x * EDGE_BLOCK * EPT;
-#pragma unroll
-        for (int j = 0; j < EPT; j++) {
-            const int li = threadIdx.x + j * EDGE_BLOCK;
-            if (e[j] >= R.e1) continue;
-            const int av = s_a[li];
-            // row start: the first edge of its A row
-            const bool start = li > 0 ? s_a[li - 1] != av : (e[j] == R.e0 || __ldg(R.La + e[j] - 1) != av);
-            if (!start) continue;
-            int be[2] = {-1, -1};
-            double bv[2] = {0.0, 0.0};
-            int lj = li;
-            for (; lj < EPT * EDGE_BLOCK && s_a[lj] == av; lj++) {
-                const int ee = (int)(b0 + lj);
-                const double vy = s_xy[lj], vz = s_xz[lj];
-                // strict order (x desc, id asc), only x > 0 (readings Z6, Z7)
-                if (vy > 0.0 && (be[0] < 0 || vy > bv[0])) { be[0] = ee; bv[0] = vy; }
-                if (vz > 0.0 && (be[1] < 0 || vz > bv[1])) { be[1] = ee; bv[1] = vz; }
-            }
-            if (lj == EPT * EDGE_BLOCK && b0 + lj < R.e1 && __ldg(R.La + b0 + lj) == av) be[0] = be[1] = PROP_SCAN;
-            R.prop[av] = be[0];
-            R.prop[R.nA + av] = be[1];
-        }
     }
 }
 
@@ -973,16 +927,12 @@ cualign_status bp_front_edge(cualign_bp *h)
     if (ml > 0) {
         KScope ks(h, CUALIGN_K_EDGE);
         EdgeArgs R{h->e0, h->e1, h->L.La, h->L.Lb, h->L.w, h->alpha, h->fp_inv, h->gh_dev, h->p_dev, h->tacc,
-                   h->texact, h->Atop, h->Btop, h->yp, h->zp, h->yc, h->zc, h->d, h->u,
-                   h->prop, h->L.Arow, (int64_t)h->L.nA, (h->flags & CUALIGN_FLAG_ROUND_DAMPED) ? 1 : 0};
-        const bool prop = h->prop != nullptr && !exact;
+                   h->texact, h->Atop, h->Btop, h->yp, h->zp, h->yc, h->zc, h->d, h->u};
         constexpr int EPT = 2; // measured: EPT 2 (48 regs) 0.085 ms vs EPT 4 (66 regs) 0.098 ms on O
         const int grid = grid_for((ml + EPT - 1) / EPT, 256, 1 << 30);
         if (exact && literal) k_edge<EPT, true, true><<<grid, 256, 0, h->stream>>>(R);
         else if (exact) k_edge<EPT, true, false><<<grid, 256, 0, h->stream>>>(R);
-        else if (literal && prop) CA_CUDA(launch_pdl(k_edge<EPT, false, true, 1, true>, dim3(grid), dim3(256), 0, h->stream, R));
         else if (literal) k_edge<EPT, false, true><<<grid, 256, 0, h->stream>>>(R);
-        else if (prop) CA_CUDA(launch_pdl(k_edge<EPT, false, false, 1, true>, dim3(grid), dim3(256), 0, h->stream, R));
         else {
             // measurement knob: 1 = 1 edge per thread, 4 = 4 edges per thread
             static const int var = probe_knob("CUALIGN_EDGE_VAR", 0);

@@ -179,7 +179,6 @@ struct cualign_bp {
     // iteration's outside a pipelined run), the iteration the rounding
     // kernels report (round_p; = p_dev except in a pipelined run)
     double *yc_b1 = nullptr, *zc_b1 = nullptr;
-    int32_t *prop = nullptr, *prop_b1 = nullptr; // per A row and instance: best edge for the rounding (k_edge)
     int pipe_mode = -1;                 // step schedule: -1 undecided, 0 forked graph, 1 pipelined, 2 serial
     int sched_param = 0;                // cualign_params.schedule (0 = library's choice)
     int tile_log_param = 0;             // cualign_params.square_tile_log (0 = SQ_TILE_LOG, -1 = none)
@@ -255,10 +254,6 @@ inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, siz
     cfg.numAttrs = 1;
     return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
-
-// k_edge's per-row head start for the rounding (prop): "scan the row
-// yourself" -- a byte pattern, so cudaMemset can write it (0xFE bytes)
-constexpr int32_t PROP_SCAN = (int32_t)0xFEFEFEFE;
 
 // --------------------------------------------------------------- memory
 cualign_status dmalloc(cualign_bp *h, void **p, size_t bytes);

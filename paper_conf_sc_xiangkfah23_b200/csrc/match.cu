@@ -53,7 +53,6 @@ struct MatchParams {
     int32_t *mateB;         // [ninst][nB] (transient)
     int2 *mvA;              // (M_y(i), M_z(i)) as B vertices, for evaluate
     int *qcnt;              // Suitor rounds: sub-queue counters (reset by k_collect), or null
-    const int32_t *prop;    // k_edge's best edge per (instance, A row): -1 none, PROP_SCAN scan (or null)
     RoundDev *rd;
     unsigned long long *work; // proposals (suitor) / rounds, spread counters
     unsigned long long *dbg;  // optional diagnostics (CUALIGN_MATCH_DEBUG)
@@ -296,7 +295,6 @@ __device__ __forceinline__ void suitor_tile(const MatchParams &P, Tile &tile, in
 // writes (r + 1) % 3 and clears the counters of (r + 2) % 3, which round
 // r + 1 writes (k_collect clears all of them for the next rounding).
 constexpr int QBUF = 3;
-constexpr int ROUND_U = 18; // a filtered round loads a whole row (<= 18 entries) in one batch
 
 __device__ __forceinline__ void queue_push(int push, int64_t chunk, int32_t *__restrict__ queue,
                                            int *__restrict__ qcnt, int64_t qcap)
@@ -350,20 +348,10 @@ __device__ __forceinline__ int propose_once(const MatchParams &P, int64_t nP, in
 {
     const double *__restrict__ x = xk(P, k);
     unsigned long long *sT = P.suit + k * nT;
+    const int lo = (int)__ldg(P.Arow + cur), hi = (int)__ldg(P.Arow + cur + 1);
     int best = -1, bt = -1;
     double bx = 0.0;
     unsigned long long bs = 0ull;
-    int lo = 0, hi = 0;
-    const int pr = (FIRST && P.prop) ? __ldg(P.prop + k * nP + cur) : PROP_SCAN;
-    if (pr >= 0) {
-        // k_edge found the row's best edge: no scan
-        best = pr;
-        bx = __ldg(x + pr);
-        bt = __ldg(P.Lb + pr);
-    } else if (pr == PROP_SCAN) {
-        lo = (int)__ldg(P.Arow + cur);
-        hi = (int)__ldg(P.Arow + cur + 1);
-    }
     for (int j0 = lo; j0 < hi; j0 += U) {
         double xx[U];
         int tt[U];
@@ -986,7 +974,6 @@ MatchParams base_params(cualign_bp *h)
     P.wslot = &h->rd->wslot;
     P.mateB = h->mateB;
     P.mvA = h->mvA;
-    P.prop = nullptr;
     P.rd = h->rd;
     P.work = h->match_work;
     return P;
@@ -1035,12 +1022,14 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
         P.qcnt = h->qcnt;
         KScope ks(h, CUALIGN_K_MATCH);
         const int64_t qc = h->qcap, cs = (int64_t)NQ * QSTRIDE;
-        static const int nrounds = probe_knob("CUALIGN_SUITOR_ROUNDS", 6);
+        // 3 rounds: 0.127 ms for both matchings on O vs 0.150 / 0.165 with 6 / 9
+        // (each round costs ~9 dependent memory round trips, even nearly empty)
+        static const int nrounds = probe_knob("CUALIGN_SUITOR_ROUNDS", 3);
         CA_CUDA(launch_pdl(k_propose_first<6>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P,
                            h->squeue + 1 * NQ * qc, h->qcnt + 1 * cs, qc));
         for (int r = 1; r <= nrounds; r++) {
             const int bi = r % QBUF, bo = (r + 1) % QBUF, bc = (r + 2) % QBUF;
-            CA_CUDA(launch_pdl(k_propose_round<ROUND_U>, dim3(h->qr_grid), dim3(256), 0, h->stream, P,
+            CA_CUDA(launch_pdl(k_propose_round<6>, dim3(h->qr_grid), dim3(256), 0, h->stream, P,
                                (const int32_t *)(h->squeue + bi * NQ * qc), (const int *)(h->qcnt + bi * cs),
                                h->squeue + bo * NQ * qc, h->qcnt + bo * cs, h->qcnt + bc * cs, qc));
         }
@@ -1149,7 +1138,6 @@ cualign_status match_setup(cualign_bp *h)
         h->max_deg_a = (int64_t)md[0];
         h->max_deg_b = (int64_t)md[1];
         h->propose_from_b = h->max_deg_b < h->max_deg_a;
-        if (h->propose_from_b || h->max_deg_a > SUITOR_ROUNDS_MAXDEG) h->prop = h->prop_b1 = nullptr;
     }
     int occ = 0;
     CA_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_pointer_rounds, 256, 0));
@@ -1174,7 +1162,7 @@ cualign_status match_setup(cualign_bp *h)
         CA_TRY(dalloc(h, &h->qcnt, (size_t)QBUF * NQ * QSTRIDE));
         CA_CUDA(cudaMemsetAsync(h->qcnt, 0, sizeof(int) * QBUF * NQ * QSTRIDE, h->stream));
         int occr = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occr, k_propose_round<ROUND_U>, 256, 0) != cudaSuccess ||
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occr, k_propose_round<6>, 256, 0) != cudaSuccess ||
             occr < 1)
             occr = 1;
         (void)cudaGetLastError();
@@ -1196,7 +1184,6 @@ cualign_status match_round(cualign_bp *h)
     P.ninst = 2;
     P.x0 = damped ? h->yp : h->yc;
     P.x1 = damped ? h->zp : h->zc;
-    P.prop = h->prop; // written by this iteration's k_edge
     CA_TRY(run_matching(h, P));
     if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) CA_TRY(prep_eval_from_mates(h));
     return match_evaluate(h);

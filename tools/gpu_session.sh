@@ -45,7 +45,7 @@ for w in $WHAT; do
       echo "nculist rc=$?"; python tools/launches.py $OUT/launches_round.csv 2>/dev/null | head -20 ;;
     ncuparts_*)
       K=${w#ncuparts_}
-      timeout 900 ncu --set full --import-source on --clock-control none -k regex:$K -s 100 -c 1 -o $OUT/ncu_$K -f python tools/bench_parts.py --pre 80 --n 10 > $OUT/ncu_$K.log 2>&1
+      timeout 900 ncu --set full --import-source on --clock-control none -k regex:$K -s 20 -c 1 -o $OUT/ncu_$K -f python tools/bench_parts.py --pre 80 --n 10 > $OUT/ncu_$K.log 2>&1
       echo "ncu $K rc=$?"; tail -2 $OUT/ncu_$K.log ;;
     ncu_*)
       K=${w#ncu_}
