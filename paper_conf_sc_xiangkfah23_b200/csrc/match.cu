@@ -310,6 +310,19 @@ __device__ __forceinline__ void queue_push(int push, int64_t chunk, int32_t *__r
     if (push >= 0) queue[q * qcap + base + __popc(mask & ((1u << lane) - 1u))] = push;
 }
 
+// successful proposals (round info rounds_y / rounds_z): one atomic per
+// warp and instance, spread over WORK_SPREAD counters
+__device__ __forceinline__ void count_proposals(const MatchParams &P, bool proposed, int k, int64_t chunk)
+{
+    const unsigned b0 = __ballot_sync(0xffffffffu, proposed && k == 0);
+    const unsigned b1 = __ballot_sync(0xffffffffu, proposed && k == 1);
+    if ((threadIdx.x & 31) == 0) {
+        unsigned long long *w = P.work + (chunk % WORK_SPREAD) * WORK_STRIDE;
+        if (b0) atomicAdd(w, (unsigned long long)__popc(b0));
+        if (b1) atomicAdd(w + 1, (unsigned long long)__popc(b1));
+    }
+}
+
 // exclusive prefix of the NQ sub-queue counts into s_off[0..NQ] (one warp)
 __device__ __forceinline__ void queue_offsets(const int *__restrict__ qcnt, int *s_off)
 {
@@ -344,7 +357,7 @@ __device__ __forceinline__ int queue_at(const int32_t *__restrict__ queue, const
 // lost, the displaced one if it displaced a suitor) or -1.
 template <int U, bool FIRST>
 __device__ __forceinline__ int propose_once(const MatchParams &P, int64_t nP, int64_t nT, int k, int cur,
-                                            int64_t work_id)
+                                            bool &proposed)
 {
     const double *__restrict__ x = xk(P, k);
     unsigned long long *sT = P.suit + k * nT;
@@ -393,7 +406,7 @@ __device__ __forceinline__ int propose_once(const MatchParams &P, int64_t nP, in
     while (beats<false>(P, x, k, nT, bt, bx, best, kb, s)) {
         const unsigned long long old = atomicCAS(sp, s, mine);
         if (old == s) {
-            atomicAdd(P.work + (work_id % WORK_SPREAD) * WORK_STRIDE + k, 1ull);
+            proposed = true;
             return s ? (int)(k * nP + __ldg(P.La + (int)(uint32_t)s)) : -1; // the displaced one
         }
         s = old;
@@ -408,11 +421,13 @@ __global__ void __launch_bounds__(256) k_propose_first(MatchParams P, int32_t *_
     pdl_wait();
     const int64_t nP = P.nA, nT = P.nB;
     const int64_t slot = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    int push = -1;
+    int push = -1, k = 0;
+    bool proposed = false;
     if (slot < P.ninst * nP) {
-        const int k = (int)(slot / nP);
-        push = propose_once<U, true>(P, nP, nT, k, (int)(slot - k * nP), slot);
+        k = (int)(slot / nP);
+        push = propose_once<U, true>(P, nP, nT, k, (int)(slot - k * nP), proposed);
     }
+    count_proposals(P, proposed, k, slot >> 5);
     queue_push(push, slot >> 5, qout, cout, qcap);
 }
 
@@ -431,12 +446,14 @@ __global__ void __launch_bounds__(256) k_propose_round(MatchParams P, const int3
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t base = gwarp * 32; base < total; base += nwarps * 32) {
         const int idx = (int)(base + (threadIdx.x & 31));
-        int push = -1;
+        int push = -1, k = 0;
+        bool proposed = false;
         if (idx < total) {
             const int v = queue_at(qin, s_off, qcap, idx);
-            const int k = (int)(v / nP);
-            push = propose_once<U, false>(P, nP, nT, k, (int)(v - k * nP), idx);
+            k = (int)(v / nP);
+            push = propose_once<U, false>(P, nP, nT, k, (int)(v - k * nP), proposed);
         }
+        count_proposals(P, proposed, k, base >> 5);
         queue_push(push, base >> 5, qout, cout, qcap);
     }
 }

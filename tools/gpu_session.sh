@@ -25,6 +25,9 @@ for w in $WHAT; do
       ENVS=$(echo ${w#pp_} | tr ',' ' ')
       env CUALIGN_LIB=$PROBES $ENVS timeout 300 python tools/bench_parts.py --pre 80 --n 50 > $OUT/parts_${w}.json 2> $OUT/parts_${w}.err
       echo "$w rc=$?"; cat $OUT/parts_${w}.json ;;
+    sched)
+      timeout 1200 python tools/probe_schedules.py > $OUT/sched.jsonl 2> $OUT/sched.err
+      echo "sched rc=$?"; cat $OUT/sched.jsonl ;;
     bench)
       timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err
       echo "bench rc=$?"; cut -c1-1500 $OUT/bench.json ;;
