@@ -202,9 +202,12 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
     // O: 1446 vs 1394 it/s pipelined (serial: 1352 vs 1389, so 2 lanes there)
     struct TgScope {
         cualign_bp *h;
-        ~TgScope() { h->top2_tg = 0; }
+        ~TgScope() { h->top2_tg = 0; h->sq_ctas = 0; }
     } tg_scope{h};
     h->top2_tg = 1;
+    // the square pass leaves SM room to the rounding running beside it
+    static const int pipe_sq = probe_knob("CUALIGN_PIPE_SQ_CTAS", 0);
+    h->sq_ctas = pipe_sq;
     double *yc0 = h->yc, *zc0 = h->zc;
     double *yb[2] = {yc0, h->yc_b1}, *zb[2] = {zc0, h->zc_b1};
     cualign_status st = CUALIGN_OK;

@@ -621,6 +621,7 @@ cualign_status square_tma_launch_v(cualign_bp *h, V *vals)
     int occ = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, block, smem) != cudaSuccess || occ < 1) occ = 1;
     (void)cudaGetLastError();
+    if (h->sq_ctas > 0 && h->sq_ctas < occ) occ = h->sq_ctas;
     const int64_t nchunks = (h->nsq + SQT_CHUNK - 1) / SQT_CHUNK;
     const int grid = grid_for(nchunks, 1, (int64_t)occ * h->num_sms);
     CA_CUDA(launch_pdl(fn, dim3(grid), dim3(block), smem, h->stream, h->nsq, h->sq_ef, vals, (const double *)h->u,

@@ -183,6 +183,7 @@ struct cualign_bp {
     int sched_param = 0;                // cualign_params.schedule (0 = library's choice)
     int tile_log_param = 0;             // cualign_params.square_tile_log (0 = SQ_TILE_LOG, -1 = none)
     int top2_tg = 0;                    // k_top2 lanes per tile while capturing (0: default; pipelined graphs: 1)
+    int sq_ctas = 0;                    // square-pass CTAs per SM while capturing (0: as many as fit)
     int *rp_dev = nullptr;
     const int *round_p = nullptr;
 

@@ -28,6 +28,11 @@ for w in $WHAT; do
     sched)
       timeout 1200 python tools/probe_schedules.py > $OUT/sched.jsonl 2> $OUT/sched.err
       echo "sched rc=$?"; cat $OUT/sched.jsonl ;;
+    sched_*)
+      # schedule probe on O with the probe build and env: sched_NAME=V,NAME2=V
+      ENVS=$(echo ${w#sched_} | tr ',' ' ')
+      env CUALIGN_LIB=$PROBES $ENVS timeout 600 python tools/probe_schedules.py --points O > $OUT/$w.jsonl 2> $OUT/$w.err
+      echo "$w rc=$?"; cat $OUT/$w.jsonl ;;
     bench)
       timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err
       echo "bench rc=$?"; cut -c1-1500 $OUT/bench.json ;;
