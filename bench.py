@@ -324,7 +324,7 @@ def launch_floor_ms(n_kernels, reps=200):
 
 def config_point(ca, name, k, steps, stream, dev):
     """One BASELINE.json config on one GPU: generate (seeded),
-    init through the C ABI, the library's schedule selection + warm-up, then
+    init through the C ABI, warm-up steps, then
     `steps` device-timed steps (iteration + rounding) on the launching stream;
     iterate-only and round-only graph replays with per-kernel event nodes for
     the split and the square pass's HBM fraction (20 B per nonzero of S)."""
@@ -344,8 +344,7 @@ def config_point(ca, name, k, steps, stream, dev):
         sz = h.sizes()
         s_nz = int(sz["s"])
         row.update(s=s_nz, squares=s_nz // 2, device_gb=round(sz["device_bytes"] / 1e9, 2))
-        h.run(57)       # the library's schedule selection (timed pipelined vs serial), untimed here
-        h.run(5)
+        h.run(10)
         torch.cuda.synchronize()
         h.stats(reset=True)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -478,11 +477,8 @@ def main():
         f"fp_bits={sz['fixed_point_bits']} device_bytes={sz['device_bytes']/1e9:.2f}GB")
 
     # ------------------------------------------------------------- warmup
-    # (each step = iterate(1) + round, replayed from the library's CUDA graph)
-    # The library picks the step schedule on its first run of >= 14 steps by
-    # timing pipelined and serial (16 timed steps each from 38 steps on); do
-    # that here, untimed, before the warm-up.
-    h.run(57)
+    # (each step = iterate(1) + round, replayed from the library's CUDA graph;
+    # the library's step schedule comes from its size rule, no timed selection)
     h.run(args.warmup)
     torch.cuda.synchronize()
     h.stats(reset=True)

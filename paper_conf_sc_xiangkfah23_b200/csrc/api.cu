@@ -778,6 +778,20 @@ cualign_status cualign_bp_run_trace(cualign_bp *h, int32_t n_steps, cualign_roun
 } // extern "C"
 
 namespace cualign {
+// Step schedule of run() when the caller leaves it to the library (no timed
+// selection on the critical path).  Measured (tools/probe_schedules.py,
+// profiles/r02_schedules.jsonl, ms per step pipelined / serial): T 0.043 /
+// 0.051, P 0.118 / 0.131 -- launch- and latency-bound steps gain from
+// overlapping the rounding with the next iteration; O 0.704 / 0.693, S 5.91 /
+// 5.64, R k = 5 1.14 / 0.81, R k = 50 7.50 / 6.97 -- once the square pass
+// (which needs every SM's registers at full speed) dominates, any overlap
+// only delays it.  Serial from 10^7 nonzeros of S on.
+static int default_schedule(cualign_bp *h)
+{
+    const int64_t s = h->s_total ? h->s_total : h->s;
+    return s >= 10000000 ? 2 : 1;
+}
+
 static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, RoundDev *trace)
 {
     if (h->world > 1) {
@@ -792,22 +806,15 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
         h->have_info = h->have_info || (what & CUALIGN_RUN_ROUND);
         return CUALIGN_OK;
     }
-    // both halves of a step: pipelined (the rounding of iteration k beside
-    // iteration k+1) unless the rounding reads y^p, z^p (ROUND_DAMPED: the
-    // next iteration overwrites them), the matching is the cooperative
-    // pointer-round kernel (MATCH_ROUNDS: its grid must be co-resident, so it
-    // never shares the device), or CUALIGN_PIPELINE=0 (measurement knob)
-    // Which step schedule is fastest depends on the instance: the rounding
-    // branch takes SM slots from the one-wave square pass, whose static
-    // partition then waits for them.  Schedules: 0 = one graph per step with
-    // the rounding forked beside the square pass, 1 = pipelined (rounding of
-    // k beside iteration k+1), 2 = serial (iterate graph, then round graph).
-    // Measured: O 1246 / 1300 / ~1300 it/s; R-MAT k = 5 1.03 / 1.62 / ~1.03
-    // ms per step; R k = 50 8.3 ms with a fork vs 7.7 serial.  The first run
-    // of >= 14 steps times 4 steps of pipelined and serial (16 if it has >= 38 steps; after a capture and 2 warm steps)
-    // and keeps the fastest; results are identical whichever runs (tests compare
-    // them with the eager sequence bit for bit).  CUALIGN_PIPELINE=0/1/2
-    // forces one.
+    // both halves of a step: schedules 0 = one graph per step with the
+    // rounding forked beside the square pass, 1 = pipelined (rounding of k
+    // beside iteration k+1), 2 = serial (one graph: iteration, then its
+    // rounding); results are identical whichever runs (tests compare them
+    // with the eager sequence bit for bit).  Not pipelined when the rounding
+    // reads y^p, z^p (ROUND_DAMPED: the next iteration overwrites them) or
+    // the matching is the cooperative pointer-round kernel (MATCH_ROUNDS: its
+    // grid must be co-resident).  The caller picks one with
+    // cualign_params.schedule, else default_schedule().
     // cualign_params.schedule: 1 pipelined, 2 serial, 3 forked (pipe_mode 0)
     const int pipe_env = h->sched_param == 3 ? 0 : (h->sched_param > 0 ? h->sched_param : -1);
     const bool both = what == (CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND) &&
@@ -845,35 +852,8 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
         h->pipe_mode = pipe_env; // given by the caller (reported as chosen)
         return run_mode(pipe_env, n_steps, trace);
     }
-    if (h->pipe_mode >= 0) return run_mode(h->pipe_mode, n_steps, trace);
-    // per schedule: capture + warm, timed (16 timed steps when the run is
-    // long enough: 4 steps of ~0.7 ms left the O choice to noise).  Only
-    // pipelined and serial are timed: the forked graph was never ahead of
-    // the better of the two (O 1246 vs 1300+, R k = 5 1.03 vs 1.01-1.03 ms,
-    // R k = 50 8.3 vs 7.7 ms) and its timed steps are part of the run.
-    constexpr int32_t PRE = 4, NSEL = 2; // PRE even: warm-up and timed windows use the same buffer parity
-    const int sel[NSEL] = {1, 2};
-    const int32_t TIMED = n_steps >= NSEL * (PRE + 16) ? 16 : 4, PER = PRE + TIMED;
-    if (n_steps < NSEL * PER || h->timing) return run_pipelined(h, n_steps, trace); // undecided: default
-    auto tr = [&](int32_t off) { return trace ? trace + off : nullptr; };
-    float t[3] = {0.f, 0.f, 0.f};
-    for (int i = 0; i < NSEL; i++) {
-        const int mode = sel[i];
-        cudaEvent_t e0 = get_event(h), e1 = get_event(h);
-        CA_TRY(run_mode(mode, PRE, tr(PER * i)));
-        CA_CUDA(cudaEventRecord(e0, h->stream));
-        CA_TRY(run_mode(mode, TIMED, tr(PER * i + PRE)));
-        CA_CUDA(cudaEventRecord(e1, h->stream));
-        CA_CUDA(cudaEventSynchronize(e1));
-        CA_CUDA(cudaEventElapsedTime(&t[mode], e0, e1));
-        h->event_pool.push_back(e0);
-        h->event_pool.push_back(e1);
-    }
-    // the pipelined schedule unless serial is clearly (> 2 %) faster
-    int best = 1;
-    if (t[2] < 0.98f * t[1]) best = 2;
-    h->pipe_mode = best;
-    return run_mode(h->pipe_mode, n_steps - NSEL * PER, tr(NSEL * PER));
+    if (h->pipe_mode < 0) h->pipe_mode = default_schedule(h);
+    return run_mode(h->pipe_mode, n_steps, trace);
 }
 } // namespace cualign
 

@@ -25,7 +25,7 @@ def main():
             h.run(6)
             h.get_best()
     with ca.CuAlignBP(A, B, L, **kw) as h:
-        h.run_trace(40)          # library's own schedule selection
+        h.run_trace(40)          # library's own schedule
         h.iterate(2)
         h.round()
         h.round_mates()
