@@ -204,10 +204,11 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
         cualign_bp *h;
         ~TgScope() { h->top2_tg = 0; h->sq_ctas = 0; }
     } tg_scope{h};
-    h->top2_tg = 1;
+    h->top2_tg = probe_knob("CUALIGN_PIPE_TOP2_TG", 1);
     // the square pass leaves SM room to the rounding running beside it
     static const int pipe_sq = probe_knob("CUALIGN_PIPE_SQ_CTAS", 0);
     h->sq_ctas = pipe_sq;
+    h->pipe_join_front = probe_knob("CUALIGN_PIPE_JOIN_FRONT", 0) != 0;
     double *yc0 = h->yc, *zc0 = h->zc;
     double *yb[2] = {yc0, h->yc_b1}, *zb[2] = {zc0, h->zc_b1};
     cualign_status st = CUALIGN_OK;
@@ -249,10 +250,22 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
         }
         h->yc = yb[wb];
         h->zc = zb[wb];
-        if (st == CUALIGN_OK) st = bp_iterate(h, 1);
-        if (st == CUALIGN_OK && (cudaEventRecord(h->fork_ev[1], h->gstream2) != cudaSuccess ||
-                                 cudaStreamWaitEvent(h->gstream, h->fork_ev[1], 0) != cudaSuccess))
-            st = CUALIGN_ECUDA;
+        // the join before the square pass (h->pipe_join_front): the rounding
+        // overlaps only the latency-bound front (k_edge, k_top2) of iteration
+        // p; the square pass, which needs every SM at full occupancy, runs alone
+        if (h->pipe_join_front) {
+            if (st == CUALIGN_OK) st = bp_iterate_front(h);
+            if (st == CUALIGN_OK && (cudaEventRecord(h->fork_ev[1], h->gstream2) != cudaSuccess ||
+                                     cudaStreamWaitEvent(h->gstream, h->fork_ev[1], 0) != cudaSuccess))
+                st = CUALIGN_ECUDA;
+            if (st == CUALIGN_OK) st = bp_iterate_back(h);
+            if (st == CUALIGN_OK) h->p += 1;
+        } else {
+            if (st == CUALIGN_OK) st = bp_iterate(h, 1);
+            if (st == CUALIGN_OK && (cudaEventRecord(h->fork_ev[1], h->gstream2) != cudaSuccess ||
+                                     cudaStreamWaitEvent(h->gstream, h->fork_ev[1], 0) != cudaSuccess))
+                st = CUALIGN_ECUDA;
+        }
     } else {
         st = round_of(wb);
     }
@@ -622,6 +635,26 @@ static cualign_status round_mates(cualign_bp *h, const int32_t **out)
     } while (0)
 
 static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, RoundDev *trace);
+static int default_schedule(cualign_bp *h);
+
+// Capture (and upload) the step graphs run() will replay for the handle's
+// schedule at init, so the first steps of an alignment do not pay graph
+// capture / instantiation / upload.
+static cualign_status precapture_step_graphs(cualign_bp *h)
+{
+    if (h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS)) return CUALIGN_OK;
+    const int mode = h->sched_param == 3 ? 0 : (h->sched_param > 0 ? h->sched_param : default_schedule(h));
+    CA_TRY(ensure_gh(h, (int64_t)h->p + 2));
+    std::vector<int> slots;
+    if (mode == 2) slots = {SERIAL_SLOT};
+    else if (mode == 1) slots = {pslot(0, 0), pslot(0, 1), pslot(1, 0), pslot(1, 1), pslot(2, 0)};
+    else slots = {CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND};
+    for (int sl : slots) {
+        if (!h->graph[0][sl]) CA_TRY(capture_step(h, 0, sl));
+        CA_CUDA(cudaGraphUpload(h->graph[0][sl], h->gstream));
+    }
+    return CUALIGN_OK;
+}
 
 } // namespace cualign
 
@@ -690,6 +723,8 @@ cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B, c
         if (st == CUALIGN_OK) st = h->world > 1 ? shard_fsum(h) : bp_fsum(h); // F(S^p = 0) sums for iteration 1
         if (st == CUALIGN_OK && h->world == 1) st = bp_top2(h);                 // othermax inputs of iteration 1
         init_trace(h, "fsum");
+        if (st == CUALIGN_OK && h->world == 1) st = precapture_step_graphs(h);
+        init_trace(h, "step graphs");
     }
     if (st == CUALIGN_OK) {
         cudaError_t e = cudaStreamSynchronize(h->stream);

@@ -184,6 +184,7 @@ struct cualign_bp {
     int tile_log_param = 0;             // cualign_params.square_tile_log (0 = SQ_TILE_LOG, -1 = none)
     int top2_tg = 0;                    // k_top2 lanes per tile while capturing (0: default; pipelined graphs: 1)
     int sq_ctas = 0;                    // square-pass CTAs per SM while capturing (0: as many as fit)
+    bool pipe_join_front = false;       // pipelined graphs: rounding joins before the square pass
     int *rp_dev = nullptr;
     const int *round_p = nullptr;
 
