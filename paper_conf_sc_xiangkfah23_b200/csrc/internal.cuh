@@ -77,6 +77,7 @@ struct RoundDev {
     int improved;
     int source;
     unsigned int done;            // k_eval blocks finished (last-block final reduction)
+    unsigned int gbar;            // k_eval<COLLECT>: blocks past the collect pass (grid barrier)
     int best_slot, best_source;   // where bestM lives: mates[best_slot][best_source] (valid if best_iter > 0)
     int wslot;                    // slot the next rounding writes (= 1 - best_slot)
     int last_slot;                // slot the last rounding wrote
@@ -198,7 +199,7 @@ struct cualign_bp {
     int32_t *dist_gi = nullptr, *dist_wid = nullptr, *dist_hold = nullptr, *dist_act = nullptr;
     int dist_rounds = 0; // merge rounds of the last sharded rounding
     double *partial_w = nullptr;
-    int match_grid = 0, match_block = 256, eval_grid = 1;
+    int match_grid = 0, match_block = 256, eval_grid = 1, evalc_grid = 1;
     unsigned long long *match_work = nullptr; // proposals (suitor) or rounds, per instance
     int32_t *squeue = nullptr;                // Suitor rounds: queued proposers (3 buffers x NQ sub-queues of qcap)
     int *qcnt = nullptr;                      // sub-queue counters
@@ -382,7 +383,7 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
                          int32_t k, int32_t *La, int32_t *Lb, double *Lw); // NEXT-2 (knn.cu)
 cualign_status match_setup(cualign_bp *h);
 cualign_status match_round(cualign_bp *h);  // a7 + a8 on the device
-cualign_status match_evaluate(cualign_bp *h); // a8 on mateA / mateB
+cualign_status match_evaluate(cualign_bp *h); // a8 on the round's mate slot (collect done)
 // sharded rounding (NEXT-1), driven by shard_round: begin, then rounds of
 // local -> all-reduce MAX(dist_wxg) -> cand -> all-reduce MIN(dist_wid) ->
 // update -> all-reduce SUM(dist_cnt) until the count is 0, then finish

@@ -608,9 +608,8 @@ __global__ void k_fill_i32(int64_t n, int32_t *__restrict__ x, int32_t v)
 // proposers left unmatched were written by k_suitor.  Every slot is reset to
 // empty for the next rounding (no separate reset pass), and the round's
 // overlap / cardinality accumulators are zeroed (k_eval follows).
-__global__ void k_collect(MatchParams P, int64_t nT, int64_t nP, int fromB)
+__device__ __forceinline__ void collect_body(const MatchParams &P, int64_t nT, int64_t nP, int fromB)
 {
-    pdl_wait();
     if (blockIdx.x == 0 && threadIdx.x < 4) (&P.rd->overlap[0])[threadIdx.x] = 0ull; // overlap[2], card[2]
     if (P.qcnt && blockIdx.x == 0 && threadIdx.x < QBUF * NQ) P.qcnt[threadIdx.x * QSTRIDE] = 0; // next rounding
     int32_t *mateA = slot_mates(P);
@@ -634,6 +633,12 @@ __global__ void k_collect(MatchParams P, int64_t nT, int64_t nP, int fromB)
             if (e >= 0) P.mateB[k * nP + __ldg(P.Lb + e)] = e;
         }
     }
+}
+
+__global__ void k_collect(MatchParams P, int64_t nT, int64_t nP, int fromB)
+{
+    pdl_wait();
+    collect_body(P, nT, nP, fromB);
 }
 
 __global__ void k_fill_slot(MatchParams P, int64_t n)
@@ -864,13 +869,31 @@ __device__ void round_final_block(const EvalParams &P, const int32_t *mateA, int
 // edge of B (one probe of the E_B membership set, ~1 dependent load instead of
 // a ~5-load binary search in B's row of M(i)) -- balanced whatever the degree
 // of i.  The last block to finish runs the final reduction.
+//
+// COLLECT: the Suitor's collect pass (k_collect) runs first inside this kernel
+// -- the grid is one wave (every block resident), so a grid-wide barrier
+// (arrival counter in RoundDev, reset by the final block after every block
+// has left it) separates the two instead of a kernel boundary.
+template <bool COLLECT>
 __global__ void __launch_bounds__(256)
-k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, unsigned long long *work)
+k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, unsigned long long *work,
+       MatchParams M, int64_t nT, int64_t nP, int fromB)
 {
     pdl_wait();
     __shared__ double sd[32];
     __shared__ unsigned long long su[32];
     __shared__ bool last;
+    if (COLLECT) {
+        collect_body(M, nT, nP, fromB);
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            __threadfence();
+            atomicAdd(&P.rd->gbar, 1u);
+            while (*(volatile unsigned int *)&P.rd->gbar < gridDim.x) __nanosleep(64);
+            __threadfence();
+        }
+        __syncthreads();
+    }
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
     const int32_t *mateA = P.mates + (int64_t)(*(volatile const int *)P.wslot) * 2 * P.nA;
@@ -934,7 +957,10 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, uns
     if (!last) return;
     __threadfence();
     round_final_block(P, mateA, gridDim.x, exact, alpha, beta, p_dev, work, sd);
-    if (threadIdx.x == 0) P.rd->done = 0u;
+    if (threadIdx.x == 0) {
+        P.rd->done = 0u;
+        if (COLLECT) P.rd->gbar = 0u; // every block is past the barrier (it counted in `done`)
+    }
 }
 
 // Schedules whose kernels leave complete mate arrays (pointer rounds, the
@@ -1009,7 +1035,7 @@ MatchParams base_params(cualign_bp *h)
 // target slot; resets the slots) leave the mates of both sides, mvA and zeroed
 // round accumulators -- ready for k_eval.  Pointer rounds leave complete mate
 // arrays (k_mate_vertex prepares evaluate).
-cualign_status run_matching(cualign_bp *h, MatchParams &P)
+cualign_status run_matching(cualign_bp *h, MatchParams &P, bool collect_in_eval = false)
 {
     const int64_t nA = h->L.nA, nB = h->L.nB;
     if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) {
@@ -1104,7 +1130,7 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P)
                 (long long)slots, d[0], d[1], d[2], d[3], d[4]);
         cudaFree(dbuf);
     }
-    {
+    if (!collect_in_eval) { // else the collect pass opens k_eval<true> (match_evaluate)
         KScope ks(h, CUALIGN_K_MATCHAUX);
         CA_CUDA(launch_pdl(k_collect, dim3(grid_for(P.ninst * nT > 0 ? P.ninst * nT : 1, 256, h->num_sms * 8)),
                            dim3(256), 0, h->stream, P, nT, nP, fromB ? 1 : 0));
@@ -1173,11 +1199,19 @@ cualign_status match_setup(cualign_bp *h)
     {
         // one wave of k_eval (every block resident at once)
         int occ = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_eval, 256, 0) != cudaSuccess || occ < 1) occ = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_eval<false>, 256, 0) != cudaSuccess || occ < 1)
+            occ = 1;
         (void)cudaGetLastError();
         h->eval_grid = grid_for(h->nApairs > (int64_t)nA ? h->nApairs : (int64_t)nA, 256, h->num_sms * occ);
+        // k_eval<true> holds a grid barrier: exactly one wave of its own occupancy
+        int occc = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occc, k_eval<true>, 256, 0) != cudaSuccess || occc < 1)
+            occc = 1;
+        (void)cudaGetLastError();
+        h->evalc_grid = grid_for(std::max<int64_t>(std::max<int64_t>(h->nApairs, (int64_t)nA), 2 * (int64_t)nmax), 256,
+                                 h->num_sms * occc);
     }
-    CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * h->eval_grid));
+    CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * std::max(h->eval_grid, h->evalc_grid)));
     {
         // Suitor-round queues: sub-queue q collects the pushes of the
         // phase-1 warps w with w mod NQ = q, <= 32 per warp
@@ -1202,6 +1236,10 @@ cualign_status match_setup(cualign_bp *h)
     return CUALIGN_OK;
 }
 
+static cualign_status evaluate_impl(cualign_bp *h, const MatchParams *Pc);
+
+cualign_status match_evaluate(cualign_bp *h) { return evaluate_impl(h, nullptr); }
+
 cualign_status match_round(cualign_bp *h)
 {
     MatchParams P = base_params(h);
@@ -1209,9 +1247,13 @@ cualign_status match_round(cualign_bp *h)
     P.ninst = 2;
     P.x0 = damped ? h->yp : h->yc;
     P.x1 = damped ? h->zp : h->zc;
-    CA_TRY(run_matching(h, P));
-    if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) CA_TRY(prep_eval_from_mates(h));
-    return match_evaluate(h);
+    if (h->flags & CUALIGN_FLAG_MATCH_ROUNDS) {
+        CA_TRY(run_matching(h, P));
+        CA_TRY(prep_eval_from_mates(h));
+        return match_evaluate(h);
+    }
+    CA_TRY(run_matching(h, P, true));
+    return evaluate_impl(h, &P);
 }
 
 // ------------------------------------------------ sharded rounding (NEXT-1)
@@ -1329,8 +1371,9 @@ cualign_status dist_match_finish(cualign_bp *h)
 }
 
 // a8 (evaluate + best) of this round's mates (slot rd->wslot) and mvA; the
-// final block records bestM by slot (no copy)
-cualign_status match_evaluate(cualign_bp *h)
+// final block records bestM by slot (no copy).  Pc: the Suitor's collect
+// pass runs at the start of the same kernel (k_eval<true>).
+static cualign_status evaluate_impl(cualign_bp *h, const MatchParams *Pc)
 {
     EvalParams E{};
     E.nA = h->L.nA;
@@ -1347,9 +1390,17 @@ cualign_status match_evaluate(cualign_bp *h)
     E.rd = h->rd;
     {
         KScope ks(h, CUALIGN_K_EVAL);
-        CA_CUDA(launch_pdl(k_eval, dim3(h->eval_grid), dim3(256), 0, h->stream, E,
-                           (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0, h->alpha, h->beta,
-                           (const int *)(h->round_p ? h->round_p : h->p_dev), h->match_work));
+        const int exact = (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0;
+        const int *pd = (const int *)(h->round_p ? h->round_p : h->p_dev);
+        if (Pc) {
+            const bool fromB = Pc->propose_from_b != 0;
+            const int64_t nT = fromB ? h->L.nA : h->L.nB, nP = fromB ? h->L.nB : h->L.nA;
+            CA_CUDA(launch_pdl(k_eval<true>, dim3(h->evalc_grid), dim3(256), 0, h->stream, E, exact, h->alpha,
+                               h->beta, pd, h->match_work, *Pc, nT, nP, fromB ? 1 : 0));
+        } else {
+            CA_CUDA(launch_pdl(k_eval<false>, dim3(h->eval_grid), dim3(256), 0, h->stream, E, exact, h->alpha,
+                               h->beta, pd, h->match_work, MatchParams{}, (int64_t)0, (int64_t)0, 0));
+        }
         CA_CUDA(cudaGetLastError());
     }
     return CUALIGN_OK;
