@@ -621,13 +621,28 @@ def main():
                          t_done - binfo["t_result"], binfo))
         runs.sort(key=lambda r: r[0])
         align_time_s, teardown_s, binfo = runs[len(runs) // 2]
+        # device time of the same e2e_iters steps from p = 0 on a fresh handle
+        # (CUDA events, no host copies): the iterations phase's floor -- early
+        # iterations differ from the steady state the timed region measures
+        dev_iter_s = None
+        if world == 1:
+            with ca.CuAlignBP(GA, GB, GL, inst.alpha, inst.beta, inst.gamma, flags=flags, device=dev,
+                              stream=stream) as hf:
+                torch.cuda.synchronize()
+                f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                f0.record(stream)
+                hf.run(args.e2e_iters)
+                f1.record(stream)
+                torch.cuda.synchronize()
+                dev_iter_s = f0.elapsed_time(f1) / 1e3
         d2h = args.e2e_iters * 112 + 4 * inst.A.n
         e2e = {"value": args.e2e_iters * work_units / align_time_s, "unit": UNIT,
                "h2d_bytes_per_step": h2d / args.e2e_iters, "d2h_bytes_per_step": d2h / args.e2e_iters,
                "align_time_s": align_time_s, "teardown_s": teardown_s, "iters": args.e2e_iters,
                "phases_s": binfo.get("phases_s"), "schedule": binfo.get("schedule"),
                "align_times_s": [r[0] for r in runs], "timing": f"median of {len(runs)} alignments",
-               "best_score": binfo["best_score"], "best_iter": binfo["best_iter"]}
+               "best_score": binfo["best_score"], "best_iter": binfo["best_iter"],
+               "iterations_device_s": dev_iter_s}
         if rank == 0:
             # NEXT-4: quality of the best alignment against the generator's ground truth
             try:
