@@ -577,6 +577,7 @@ static void close_handle(cualign_bp *h)
     for (auto e : h->fork_ev)
         if (e) cudaEventDestroy(e);
     dfree_all(h);
+    if (h->dist_cnt_host) cudaFreeHost(h->dist_cnt_host);
     if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
     if (h->gstream) cudaStreamDestroy(h->gstream);
     if (h->gstream2) cudaStreamDestroy(h->gstream2);
@@ -700,6 +701,9 @@ cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B, c
             if (st == CUALIGN_OK) st = match_setup(s);
         }
         if (st == CUALIGN_OK) {
+            // one exchange stream for the group: the loopback's copies read
+            // one shard's packed halo and write another's
+            for (cualign_bp *s : h->vshards) s->cstream = h->gstream2;
             cualign_bp *s0 = h->vshards[0];
             h->L = s0->L; // sizes only (the group owns no arrays itself)
             h->s_total = s0->s_total;
@@ -712,6 +716,7 @@ cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B, c
         }
     } else {
         if (st == CUALIGN_OK && h->world > 1) st = nccl_init_comm(h, params->nccl_unique_id);
+        if (h && h->world > 1) h->cstream = h->gstream2; // the shard's exchange stream
         init_trace(h, "^start");
         if (st == CUALIGN_OK) st = build_problem(h, A, B, L);
         init_trace(h, "build_problem");

@@ -608,9 +608,13 @@ constexpr size_t square_tma_smem()
     return 128 + (sizeof(int2) + sizeof(V)) * SQT_STAGES * SQT_CHUNK;
 }
 
+// squares [q0, q1) (q1 < 0: all); q0 even (16-byte aligned bulk copies)
 template <class V, bool NOATOM = false, bool DYN = false>
-cualign_status square_tma_launch_v(cualign_bp *h, V *vals)
+cualign_status square_tma_launch_v(cualign_bp *h, V *vals, int64_t q0 = 0, int64_t q1 = -1)
 {
+    if (q1 < 0) q1 = h->nsq;
+    const int64_t nq = q1 - q0;
+    if (nq <= 0) return CUALIGN_OK;
     auto fn = k_square_tma<V, NOATOM, DYN>;
     constexpr size_t smem = square_tma_smem<V>();
     // > 48 KB of dynamic shared memory needs the opt-in attribute, which
@@ -622,15 +626,20 @@ cualign_status square_tma_launch_v(cualign_bp *h, V *vals)
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, block, smem) != cudaSuccess || occ < 1) occ = 1;
     (void)cudaGetLastError();
     if (h->sq_ctas > 0 && h->sq_ctas < occ) occ = h->sq_ctas;
-    const int64_t nchunks = (h->nsq + SQT_CHUNK - 1) / SQT_CHUNK;
+    const int64_t nchunks = (nq + SQT_CHUNK - 1) / SQT_CHUNK;
     const int grid = grid_for(nchunks, 1, (int64_t)occ * h->num_sms);
-    CA_CUDA(launch_pdl(fn, dim3(grid), dim3(block), smem, h->stream, h->nsq, h->sq_ef, vals, (const double *)h->u,
-                       h->beta, (const double2 *)h->gh_dev, (const int *)h->p_dev, h->fp_scale, h->tacc, h->sq_ctr));
+    CA_CUDA(launch_pdl(fn, dim3(grid), dim3(block), smem, h->stream, nq, (const int2 *)(h->sq_ef + q0), vals + q0,
+                       (const double *)h->u, h->beta, (const double2 *)h->gh_dev, (const int *)h->p_dev, h->fp_scale,
+                       h->tacc, h->sq_ctr));
     return CUALIGN_OK;
 }
 
-cualign_status square_tma_launch(cualign_bp *h)
+cualign_status square_tma_launch(cualign_bp *h, int64_t q0 = 0, int64_t q1 = -1)
 {
+    if (q0 != 0 || q1 >= 0) {
+        if (h->sq_val32) return square_tma_launch_v(h, h->sq_val32, q0, q1);
+        return square_tma_launch_v(h, h->sq_val, q0, q1);
+    }
     // CUALIGN_SQ_DYN (probe build): 1 = chunk queue, 0 = static stride
     static const int dyn = probe_knob("CUALIGN_SQ_DYN", 0);
     if (dyn) {
@@ -648,9 +657,16 @@ void square_launch(cualign_bp *h)
     else square_launch_v<UPDATE, EXACT, SQ_U, HINTS, NOATOM>(h, h->sq_val);
 }
 
-cualign_status launch_square(cualign_bp *h, bool update)
+cualign_status launch_square(cualign_bp *h, bool update, int64_t q0 = 0, int64_t q1 = -1)
 {
     const bool exact = (h->flags & CUALIGN_FLAG_EXACT) != 0;
+    if (update && !exact && (q0 != 0 || q1 >= 0)) {
+        // a range of the squares (sharded: local-f / remote-f parts)
+        KScope ks(h, CUALIGN_K_SQUARE);
+        CA_TRY(square_tma_launch(h, q0, q1));
+        CA_CUDA(cudaGetLastError());
+        return CUALIGN_OK;
+    }
     if (h->nsq > 0) {
         KScope ks(h, CUALIGN_K_SQUARE);
         if (update && exact) square_launch<true, true, 2, true>(h);
@@ -957,6 +973,13 @@ cualign_status bp_iterate_front(cualign_bp *h)
 cualign_status bp_iterate_back(cualign_bp *h)
 {
     if (h->L.m > 0) CA_TRY(launch_square(h, true));
+    return CUALIGN_OK;
+}
+
+// the square pass over squares [q0, q1) only (sharded overlap, shard.cu)
+cualign_status bp_iterate_back_range(cualign_bp *h, int64_t q0, int64_t q1)
+{
+    if (h->L.m > 0 && q1 > q0) CA_TRY(launch_square(h, true, q0, q1));
     return CUALIGN_OK;
 }
 

@@ -121,6 +121,9 @@ struct cualign_bp {
     int32_t *halo_need = nullptr, *halo_give = nullptr;
     std::vector<int64_t> need_off, give_off;
     int64_t n_need = 0, n_give = 0;
+    int64_t nsq_split = -1;            // sharded: squares [0, nsq_split) read owned f only (no halo);
+                                       // [nsq_split, nsq) need the u halo (-1: no split)
+    cudaStream_t cstream = nullptr;    // sharded: exchange stream (halo overlapped with the local squares)
     double *hu_out = nullptr, *hu_in = nullptr;                // packed u_f: give side -> need side
     unsigned long long *ht_out = nullptr, *ht_in = nullptr;    // packed F sums: need side -> give side
 
@@ -198,6 +201,7 @@ struct cualign_bp {
     unsigned long long *dist_gx = nullptr, *dist_wxl = nullptr, *dist_wxg = nullptr, *dist_cnt = nullptr;
     int32_t *dist_gi = nullptr, *dist_wid = nullptr, *dist_hold = nullptr, *dist_act = nullptr;
     int dist_rounds = 0; // merge rounds of the last sharded rounding
+    unsigned long long *dist_cnt_host = nullptr; // pinned: active count after each round of a batch
     double *partial_w = nullptr;
     int match_grid = 0, match_block = 256, eval_grid = 1, evalc_grid = 1;
     unsigned long long *match_work = nullptr; // proposals (suitor) or rounds, per instance
@@ -357,6 +361,7 @@ cualign_status bp_fsum(cualign_bp *h);                 // t <- sum_f F(S^p) (ini
 cualign_status bp_iterate(cualign_bp *h, int32_t n);   // Alg. 2 l.9-16, n times
 cualign_status bp_iterate_front(cualign_bp *h);        // advance p, top-2, k_edge
 cualign_status bp_iterate_back(cualign_bp *h);         // square pass
+cualign_status bp_iterate_back_range(cualign_bp *h, int64_t q0, int64_t q1); // square pass over [q0, q1)
 cualign_status bp_top2(cualign_bp *h);                 // per-vertex top-2 of the current y^p, z^p
 cualign_status bp_front_top2(cualign_bp *h);           // advance p, top-2 (partial B when sharded)
 cualign_status bp_front_edge(cualign_bp *h);           // k_edge on the owned edges

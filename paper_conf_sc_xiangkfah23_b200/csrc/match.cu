@@ -1299,6 +1299,7 @@ cualign_status dist_match_begin(cualign_bp *h)
         CA_TRY(dalloc(h, &h->dist_hold, 2 * nPl + 1));
         CA_TRY(dalloc(h, &h->dist_act, 2 * nPl + 1));
         CA_TRY(dalloc(h, &h->dist_cnt, 1));
+        CA_CUDA(cudaHostAlloc((void **)&h->dist_cnt_host, sizeof(unsigned long long) * 16, cudaHostAllocDefault));
     }
     const int G = h->num_sms * 8;
     CA_CUDA(cudaMemsetAsync(h->match_work, 0, WORK_SPREAD * WORK_STRIDE * sizeof(unsigned long long), h->stream));

@@ -92,6 +92,7 @@ NcclApi &nccl()
     } while (0)
 
 enum RedOp { RED_MAX_U64, RED_MIN_I32, RED_SUM_U64 };
+constexpr int DIST_MAX_BATCH = 16; // merge rounds enqueued per host check (sharded rounding)
 
 // halo helpers
 __global__ void k_gather_d(int64_t n, const int32_t *__restrict__ ids, const double *__restrict__ src,
@@ -120,6 +121,13 @@ __global__ void k_scatter_add_u64(int64_t n, const int32_t *__restrict__ ids,
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         if (src[i]) atomicAdd(dst + ids[i], src[i]);
 }
+// 1 = the square reads a remote f (needs the u halo), 0 = owned f only
+__global__ void k_remote_key(int64_t nsq, const int2 *__restrict__ sq_ef, int64_t e1, uint8_t *__restrict__ key)
+{
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq; q += (int64_t)gridDim.x * blockDim.x)
+        key[q] = sq_ef[q].y >= e1 ? 1 : 0;
+}
+
 __global__ void k_mark_remote(int64_t nsq, const int2 *__restrict__ sq_ef, int64_t e1, uint8_t *__restrict__ flag)
 {
     for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nsq; q += (int64_t)gridDim.x * blockDim.x) {
@@ -433,6 +441,46 @@ Exchange *exchange_for(cualign_bp *h, std::vector<cualign_bp *> &S)
 
 } // namespace
 
+// Stable partition of a shard's squares: those whose f is owned first (the
+// square pass over them needs no halo and runs while the u halo is in
+// flight), then those with a remote f.  Every result is order-independent
+// (integer F sums, per-square arithmetic), so the order changes no bit.  The
+// split is rounded down to an even index: the second part's bulk copies need
+// 16-byte aligned starts (a local square in the second part only waits).
+// S^p is still zero here, so only (e, f) moves.
+cualign_status split_squares(cualign_bp *s)
+{
+    s->nsq_split = -1;
+    const int64_t n = s->nsq;
+    if (n < 2 || n >= INT32_MAX) return CUALIGN_OK;
+    TmpBuf kin, kout, vout, tmp, cnt;
+    CA_CUDA(tmalloc(s, kin, (size_t)n));
+    CA_CUDA(tmalloc(s, kout, (size_t)n));
+    CA_CUDA(tmalloc(s, vout, sizeof(int2) * (size_t)n));
+    k_remote_key<<<grid_for(n, 256, s->num_sms * 8), 256, 0, s->stream>>>(n, s->sq_ef, s->e1, (uint8_t *)kin.p);
+    CA_CUDA(cudaGetLastError());
+    size_t tb = 0;
+    const long long *vin = reinterpret_cast<const long long *>(s->sq_ef);
+    CA_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, (const uint8_t *)kin.p, (uint8_t *)kout.p, vin,
+                                            (long long *)vout.p, (int)n, 0, 1, s->stream));
+    CA_CUDA(tmalloc(s, tmp, tb ? tb : 1));
+    CA_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tb, (const uint8_t *)kin.p, (uint8_t *)kout.p, vin,
+                                            (long long *)vout.p, (int)n, 0, 1, s->stream));
+    CA_CUDA(cudaMemcpyAsync(s->sq_ef, vout.p, sizeof(int2) * (size_t)n, cudaMemcpyDeviceToDevice, s->stream));
+    // number of local squares = number of zero keys (sum of the keys = remote ones)
+    CA_CUDA(tmalloc(s, cnt, sizeof(int64_t)));
+    TmpBuf tmp2;
+    size_t tb2 = 0;
+    CA_CUDA(cub::DeviceReduce::Sum(nullptr, tb2, (const uint8_t *)kin.p, (int64_t *)cnt.p, (int)n, s->stream));
+    CA_CUDA(tmalloc(s, tmp2, tb2 ? tb2 : 1));
+    CA_CUDA(cub::DeviceReduce::Sum(tmp2.p, tb2, (const uint8_t *)kin.p, (int64_t *)cnt.p, (int)n, s->stream));
+    int64_t remote = 0;
+    CA_CUDA(cudaMemcpyAsync(&remote, cnt.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s->stream));
+    CA_CUDA(cudaStreamSynchronize(s->stream));
+    s->nsq_split = ((n - remote) / 2) * 2;
+    return CUALIGN_OK;
+}
+
 // The square-pass halo of every shard: mark the remote f of the owned
 // squares, compact them (sorted), split by owner, exchange the lists.
 cualign_status shard_setup(cualign_bp *h)
@@ -472,6 +520,7 @@ cualign_status shard_setup(cualign_bp *h)
         s->need_off[(size_t)w] = s->n_need;
         CA_TRY(dalloc(s, &s->hu_in, (size_t)s->n_need + 1));
         CA_TRY(dalloc(s, &s->ht_out, (size_t)s->n_need + 1));
+        CA_TRY(split_squares(s));
     }
     CA_TRY(X->halo_lists(S));
     for (cualign_bp *s : S) {
@@ -498,8 +547,30 @@ cualign_status shard_iterate(cualign_bp *h, int32_t n)
         for (cualign_bp *s : S) CA_TRY(bp_front_top2(s));
         CA_TRY(X->top2(S));
         for (cualign_bp *s : S) CA_TRY(bp_front_edge(s));
-        CA_TRY(X->halo_u(S));
-        for (cualign_bp *s : S) CA_TRY(bp_iterate_back(s));
+        // the u halo travels on the exchange stream while the squares whose
+        // f is owned run (they read no halo value); the remote-f squares
+        // wait for it (SURVEY §8(e) "overlap the exchange with interior rows")
+        for (cualign_bp *s : S) {
+            CA_CUDA(cudaEventRecord(s->fork_ev[0], s->stream));
+            CA_CUDA(cudaStreamWaitEvent(s->cstream, s->fork_ev[0], 0));
+        }
+        std::vector<cudaStream_t> main_streams;
+        for (cualign_bp *s : S) {
+            main_streams.push_back(s->stream);
+            s->stream = s->cstream;
+        }
+        const cualign_status hs = X->halo_u(S);
+        for (size_t i = 0; i < S.size(); i++) S[i]->stream = main_streams[i];
+        CA_TRY(hs);
+        for (cualign_bp *s : S) CA_CUDA(cudaEventRecord(s->fork_ev[1], s->cstream));
+        for (cualign_bp *s : S) {
+            const int64_t split = s->nsq_split >= 0 ? s->nsq_split : 0;
+            CA_TRY(bp_iterate_back_range(s, 0, split));
+        }
+        for (cualign_bp *s : S) {
+            CA_CUDA(cudaStreamWaitEvent(s->stream, s->fork_ev[1], 0));
+            CA_TRY(bp_iterate_back_range(s, s->nsq_split >= 0 ? s->nsq_split : 0, s->nsq));
+        }
         CA_TRY(X->halo_t(S));
         for (cualign_bp *s : S) s->p += 1;
     }
@@ -513,23 +584,38 @@ cualign_status shard_round(cualign_bp *h)
     Exchange *X = exchange_for(h, S);
     const int64_t n2B = 2 * (int64_t)S[0]->L.nB;
     for (cualign_bp *s : S) CA_TRY(dist_match_begin(s));
-    int rounds = 0;
+    // Merge rounds are enqueued in batches; the host reads the all-reduced
+    // active count once per batch (a round after convergence changes
+    // nothing: no proposer is active, the merges reproduce the global
+    // suitors).  The batch grows (2, 4, 8, ...) so that a rounding needing r
+    // rounds costs ~log2(r) host round trips and < 2r rounds.  Each shard's
+    // count is read into pinned memory on its own stream.
+    int rounds = 0, batch = 2;
     while (true) {
-        for (cualign_bp *s : S) CA_TRY(dist_match_local(s));
-        CA_TRY(X->allreduce(S, [](cualign_bp *q) -> void * { return q->dist_wxg; }, n2B, RED_MAX_U64));
-        for (cualign_bp *s : S) CA_TRY(dist_match_cand(s));
-        CA_TRY(X->allreduce(S, [](cualign_bp *q) -> void * { return q->dist_wid; }, n2B, RED_MIN_I32));
-        for (cualign_bp *s : S) CA_TRY(dist_match_update(s));
-        CA_TRY(X->allreduce(S, [](cualign_bp *q) -> void * { return q->dist_cnt; }, 1, RED_SUM_U64));
-        unsigned long long active = 0;
-        CA_CUDA(cudaMemcpyAsync(&active, S[0]->dist_cnt, sizeof(active), cudaMemcpyDeviceToHost, S[0]->stream));
-        CA_CUDA(cudaStreamSynchronize(S[0]->stream));
-        rounds++;
-        if (!active) break;
-        if (rounds > (1 << 24)) {
-            set_error("sharded rounding did not converge");
-            return CUALIGN_ECUDA;
+        for (int b = 0; b < batch; b++) {
+            for (cualign_bp *s : S) CA_TRY(dist_match_local(s));
+            CA_TRY(X->allreduce(S, [](cualign_bp *q) -> void * { return q->dist_wxg; }, n2B, RED_MAX_U64));
+            for (cualign_bp *s : S) CA_TRY(dist_match_cand(s));
+            CA_TRY(X->allreduce(S, [](cualign_bp *q) -> void * { return q->dist_wid; }, n2B, RED_MIN_I32));
+            for (cualign_bp *s : S) CA_TRY(dist_match_update(s));
+            CA_TRY(X->allreduce(S, [](cualign_bp *q) -> void * { return q->dist_cnt; }, 1, RED_SUM_U64));
+            CA_CUDA(cudaMemcpyAsync(S[0]->dist_cnt_host + b, S[0]->dist_cnt, sizeof(unsigned long long),
+                                    cudaMemcpyDeviceToHost, S[0]->stream));
         }
+        CA_CUDA(cudaStreamSynchronize(S[0]->stream));
+        int converged_at = -1;
+        for (int b = 0; b < batch && converged_at < 0; b++)
+            if (S[0]->dist_cnt_host[b] == 0ull) converged_at = b;
+        if (converged_at >= 0) {
+            rounds += converged_at + 1; // rounds that did work (the rest were no-ops)
+            break;
+        }
+        rounds += batch;
+        if (rounds > (1 << 20)) {
+            set_error("sharded rounding: no convergence after %d merge rounds", rounds);
+            return CUALIGN_ESTATE;
+        }
+        batch = std::min(2 * batch, DIST_MAX_BATCH);
     }
     for (cualign_bp *s : S) {
         s->dist_rounds = rounds;

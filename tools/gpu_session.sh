@@ -25,6 +25,11 @@ for w in $WHAT; do
       ENVS=$(echo ${w#pp_} | tr ',' ' ')
       env CUALIGN_LIB=$PROBES $ENVS timeout 300 python tools/bench_parts.py --pre 80 --n 50 > $OUT/parts_${w}.json 2> $OUT/parts_${w}.err
       echo "$w rc=$?"; cat $OUT/parts_${w}.json ;;
+    shardtests)
+      timeout 900 python -m pytest tests/test_gpu_shard.py tests/test_gpu_nccl.py tests/test_gpu_layout.py -q -p no:cacheprovider > $OUT/shardtests.txt 2>&1
+      echo "shardtests rc=$?"; tail -5 $OUT/shardtests.txt ;;
+    n2)
+      bash tools/run_bench_n2_onegpu.sh $TAG ;;
     sched)
       timeout 1200 python tools/probe_schedules.py > $OUT/sched.jsonl 2> $OUT/sched.err
       echo "sched rc=$?"; cat $OUT/sched.jsonl ;;
