@@ -571,7 +571,7 @@ def main():
     ms_per_step = elapsed_ms / args.steps
     cls_ms = pst["class_ms"]
     cls_n = pst["class_launches"]
-    sq_ms = cls_ms["square"] / max(cls_n["square"], 1)
+    sq_ms = cls_ms["square"] / prof_steps  # per step (a sharded step runs it in two ranges)
     bp_ms = (cls_ms["top2"] + cls_ms["edge"] + cls_ms["square"] + cls_ms["rowsum"] + cls_ms["other"]) / prof_steps
     round_ms = (cls_ms["match"] + cls_ms["eval"] + cls_ms["matchaux"]) / prof_steps
     peak, peak_src = read_peaks()

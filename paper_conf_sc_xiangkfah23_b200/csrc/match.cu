@@ -431,6 +431,38 @@ __global__ void __launch_bounds__(256) k_propose_first(MatchParams P, int32_t *_
     queue_push(push, slot >> 5, qout, cout, qcap);
 }
 
+// Thread-level Suitor chains (no queues): the first proposal of every
+// proposer, then the thread follows its chain -- the proposer it displaced,
+// or itself after a lost CAS -- with filtered proposals until one lands in a
+// free slot or a proposer is exhausted.
+template <int U>
+__global__ void __launch_bounds__(256) k_propose_chain(MatchParams P)
+{
+    pdl_wait();
+    const int64_t nP = P.nA, nT = P.nB;
+    const int64_t slot = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    bool proposed = false;
+    int k = 0;
+    unsigned long long nprop[2] = {0ull, 0ull};
+    if (slot < P.ninst * nP) {
+        k = (int)(slot / nP);
+        int v = propose_once<U, true>(P, nP, nT, k, (int)(slot - k * nP), proposed);
+        nprop[k] += proposed;
+        while (v >= 0) {
+            const int kk = (int)(v / nP);
+            proposed = false;
+            v = propose_once<U, false>(P, nP, nT, kk, (int)(v - kk * nP), proposed);
+            nprop[kk] += proposed;
+        }
+    }
+    for (int kk = 0; kk < 2; kk++) {
+        unsigned long long c = nprop[kk];
+#pragma unroll
+        for (int off = 16; off >= 1; off >>= 1) c += __shfl_down_sync(0xffffffffu, c, off);
+        if ((threadIdx.x & 31) == 0 && c) atomicAdd(P.work + ((slot >> 5) % WORK_SPREAD) * WORK_STRIDE + kk, c);
+    }
+}
+
 template <int U>
 __global__ void __launch_bounds__(256) k_propose_round(MatchParams P, const int32_t *__restrict__ qin,
                                                        const int *__restrict__ cin, int32_t *__restrict__ qout,
@@ -1067,7 +1099,13 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P, bool collect_in_eval 
     }
     static const int two_env = probe_knob("CUALIGN_SUITOR_QROUNDS", 1);
     const bool two = two_env && !fromB && h->max_deg_a <= SUITOR_ROUNDS_MAXDEG && h->squeue && !dbg;
-    if (two && slots > 0) {
+    static const int chain_mode = probe_knob("CUALIGN_SUITOR_CHAIN", 0);
+    if (two && slots > 0 && chain_mode) {
+        P.qcnt = h->qcnt;
+        KScope ks(h, CUALIGN_K_MATCH);
+        CA_CUDA(launch_pdl(k_propose_chain<6>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P));
+        CA_CUDA(cudaGetLastError());
+    } else if (two && slots > 0) {
         // proposal rounds (see k_propose_round), then the chain form for
         // whatever is still queued
         P.qcnt = h->qcnt;
