@@ -52,6 +52,13 @@ for w in $WHAT; do
       if [ "$w" != "kern" ]; then ENVS=$(echo ${w#kern_} | tr ',' ' '); LIBENV="CUALIGN_LIB=$PROBES"; fi
       env $LIBENV $ENVS timeout 300 python tools/probe_kernels.py --pre 80 --n 20 > $OUT/$w.json 2> $OUT/$w.err
       echo "$w rc=$?"; python -c "import json,sys; d=json.load(open('$OUT/$w.json')); [print(p, {k: round(v['us_per_step'],1) for k,v in d[p].items()}) for p in d]" ;;
+    launchlist)
+      # the bench command's launch list (cold-cache, serialised: compare shares)
+      timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $OUT/launches_bench.csv python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/launchlist.log 2>&1
+      echo "launchlist rc=$?"; python tools/launches.py $OUT/launches_bench.csv | head -25 ;;
+    ncufp32)
+      timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_square_tma -s 40 -c 1 -o $OUT/ncu_sq32 -f python bench.py --fp32 --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/ncu_sq32.log 2>&1
+      echo "ncufp32 rc=$?"; tail -2 $OUT/ncu_sq32.log ;;
     nculist)
       # launch list (cold-cache, serialised) of a round-only replay at a fixed state
       timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"k_propose|k_suitor|k_collect|k_eval|k_mate" -s 100 -c 60 --csv --log-file $OUT/launches_round.csv python tools/bench_parts.py --pre 80 --n 20 > $OUT/nculist.log 2>&1
