@@ -38,6 +38,11 @@ for w in $WHAT; do
       ENVS=$(echo ${w#sched_} | tr ',' ' ')
       env CUALIGN_LIB=$PROBES $ENVS timeout 600 python tools/probe_schedules.py --points O > $OUT/$w.jsonl 2> $OUT/$w.err
       echo "$w rc=$?"; cat $OUT/$w.jsonl ;;
+    driver)
+      # what the driver runs at round end (1 GPU): smoke, bench (20/5), reference arm
+      ( time python -c "import __graft_entry__ as g; g.smoke()" ) > $OUT/smoke.txt 2>&1; echo "smoke rc=$?"; tail -4 $OUT/smoke.txt
+      ( time timeout 1700 python bench.py --gpus 1 --steps 20 --warmup 5 ) > $OUT/bench_driver.json 2> $OUT/bench_driver.err; echo "bench rc=$?"; tail -4 $OUT/bench_driver.err; head -c 600 $OUT/bench_driver.json
+      ( time timeout 1700 python bench.py --impl reference --gpus 1 --steps 20 --warmup 5 ) > $OUT/ref_driver.json 2> $OUT/ref_driver.err; echo "ref rc=$?"; tail -4 $OUT/ref_driver.err; head -c 400 $OUT/ref_driver.json ;;
     bench)
       timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err
       echo "bench rc=$?"; cut -c1-1500 $OUT/bench.json ;;
@@ -57,7 +62,7 @@ for w in $WHAT; do
       timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $OUT/launches_bench.csv python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/launchlist.log 2>&1
       echo "launchlist rc=$?"; python tools/launches.py $OUT/launches_bench.csv | head -25 ;;
     ncufp32)
-      timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_square_tma -s 40 -c 1 -o $OUT/ncu_sq32 -f python bench.py --fp32 --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/ncu_sq32.log 2>&1
+      timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_square_tma -s 10 -c 1 -o $OUT/ncu_sq32 -f python bench.py --fp32 --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/ncu_sq32.log 2>&1
       echo "ncufp32 rc=$?"; tail -2 $OUT/ncu_sq32.log ;;
     nculist)
       # launch list (cold-cache, serialised) of a round-only replay at a fixed state
@@ -69,7 +74,7 @@ for w in $WHAT; do
       echo "ncu $K rc=$?"; tail -2 $OUT/ncu_$K.log ;;
     ncu_*)
       K=${w#ncu_}
-      timeout 900 ncu --set full --import-source on --clock-control none -k regex:$K -s 40 -c 1 -o $OUT/ncu_$K -f python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/ncu_$K.log 2>&1
+      timeout 900 ncu --set full --import-source on --clock-control none -k regex:$K -s 10 -c 1 -o $OUT/ncu_$K -f python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/ncu_$K.log 2>&1
       echo "ncu $K rc=$?"; tail -3 $OUT/ncu_$K.log ;;
   esac
 done
