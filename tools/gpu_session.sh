@@ -38,6 +38,12 @@ for w in $WHAT; do
       ENVS=$(echo ${w#sched_} | tr ',' ' ')
       env CUALIGN_LIB=$PROBES $ENVS timeout 600 python tools/probe_schedules.py --points O > $OUT/$w.jsonl 2> $OUT/$w.err
       echo "$w rc=$?"; cat $OUT/$w.jsonl ;;
+    steps)
+      timeout 600 python tools/probe_steps.py > $OUT/steps.json 2> $OUT/steps.err
+      echo "steps rc=$?"; python -c "
+import json; d=json.load(open('$OUT/steps.json')); ms=d['ms_per_step']
+print('ms per step, first 40:', ms[:40]); print('mean 6-25', sum(ms[5:25])/20, 'mean 60-120', sum(ms[60:])/len(ms[60:]))
+[print(x) for x in d['split']]" ;;
     driver)
       # what the driver runs at round end (1 GPU): smoke, bench (20/5), reference arm
       ( time python -c "import __graft_entry__ as g; g.smoke()" ) > $OUT/smoke.txt 2>&1; echo "smoke rc=$?"; tail -4 $OUT/smoke.txt
