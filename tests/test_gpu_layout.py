@@ -127,3 +127,56 @@ def test_run_trace_infos_equal_step_by_step(ca, mode):
         m1, _ = h1.get_best()
         m2, _ = h2.get_best()
         assert np.array_equal(m1, m2)
+
+
+def test_default_schedule_rule(ca):
+    """cualign_params.schedule = 0: the library's size rule (DESIGN.md §6
+    "Step graph and schedule"): pipelined below 10^7 nonzeros of S, serial
+    from there on; reported by cualign_sizes.schedule after a run."""
+    small = make_config("T")
+    with ca.CuAlignBP(small.A, small.B, small.L, small.alpha, small.beta, small.gamma) as h:
+        h.run(3)
+        assert h.sizes()["schedule"] == 1
+    big = make_config("O", scale=0.2)
+    with ca.CuAlignBP(big.A, big.B, big.L, big.alpha, big.beta, big.gamma) as h:
+        assert h.sizes()["s"] >= 10_000_000
+        h.run(3)
+        assert h.sizes()["schedule"] == 2
+
+
+@pytest.mark.parametrize("field,value", [("schedule", 4), ("schedule", -1), ("square_tile_log", 31),
+                                         ("square_tile_log", -2)])
+def test_tuning_params_validated(ca, field, value):
+    inst = make_config("T", scale=0.2)
+    with pytest.raises(ca.CuAlignError) as ei:
+        ca.CuAlignBP(inst.A, inst.B, inst.L, **{field: value})
+    assert ei.value.status == -1
+
+
+def test_round_mates_and_sample_squares_contracts(ca):
+    """get_round_mates before any rounding is ESTATE; sample_squares returns
+    exactly the squares touching the sampled edges (S by its definition) on
+    single and virtual-shard handles, and EINVAL on an id out of range."""
+    from oracle.sample import SampledProblem
+    inst = make_config("P", scale=0.05)
+    sp = SampledProblem(inst.A, inst.B, inst.L)
+    rng = np.random.default_rng(3)
+    sample = rng.choice(inst.L.m, 40, replace=False).astype(np.int32)
+    for kw in ({}, {"world": 3}):
+        with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, **kw) as h:
+            with pytest.raises(ca.CuAlignError) as ei:
+                h.round_mates()
+            assert ei.value.status == -5
+            h.iterate(2)
+            h.round()
+            my, mz = h.round_mates()
+            assert my.shape == (inst.A.n,) and mz.shape == (inst.A.n,)
+            sq = h.sample_squares(sample)
+            assert np.all(sq["e"] < sq["f"])
+            for e in sample:
+                got = sorted([int(f) for a, f in zip(sq["e"], sq["f"]) if a == e] +
+                             [int(a) for a, f in zip(sq["e"], sq["f"]) if f == e])
+                assert got == sp.S_row(int(e)), (kw, e)
+            with pytest.raises(ca.CuAlignError) as ei:
+                h.sample_squares(np.array([inst.L.m], np.int32))
+            assert ei.value.status == -1
