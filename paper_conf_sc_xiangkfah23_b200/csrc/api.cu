@@ -172,6 +172,10 @@ CommScope::~CommScope()
 
 void invalidate_graphs(cualign_bp *h)
 {
+    if (h->shard_graph) {
+        cudaGraphExecDestroy(h->shard_graph);
+        h->shard_graph = nullptr;
+    }
     for (int t = 0; t < 2; t++)
         for (int r = 0; r < cualign_bp::NSLOT; r++)
             if (h->graph[t][r]) {
@@ -832,13 +836,104 @@ static int default_schedule(cualign_bp *h)
     return s >= 10000000 ? 2 : 1;
 }
 
+// The sharded iteration (k_edge, top-2 all-gather, u halo on the exchange
+// stream beside the owned-f squares, remote-f squares, F halo; NCCL calls
+// are capturable) as ONE graph, replayed by run(): no host work per kernel or
+// exchange.  Captured on the group's capture stream with every shard's main
+// stream pointed at it; re-captured when a shard's gamma table moves.
+static cualign_status shard_iterate_graph(cualign_bp *h)
+{
+    std::vector<cualign_bp *> S = h->vshards.empty() ? std::vector<cualign_bp *>{h} : h->vshards;
+    for (cualign_bp *s : S) CA_TRY(ensure_gh(s, (int64_t)s->p + 2));
+    std::vector<const void *> gh;
+    for (cualign_bp *s : S) gh.push_back(s->gh_dev);
+    if (h->shard_graph && gh != h->shard_graph_gh) {
+        cudaGraphExecDestroy(h->shard_graph);
+        h->shard_graph = nullptr;
+    }
+    if (!h->shard_graph) {
+        struct Saved {
+            cudaStream_t stream;
+            int32_t p;
+            int64_t launches, class_launches[CUALIGN_NUM_KERNEL_CLASSES], comm_calls, comm_bytes_in;
+        };
+        std::vector<Saved> saved;
+        for (cualign_bp *s : S) {
+            Saved v{s->stream, s->p, s->launches, {}, s->comm_calls, s->comm_bytes_in};
+            for (int c = 0; c < CUALIGN_NUM_KERNEL_CLASSES; c++) v.class_launches[c] = s->class_launches[c];
+            saved.push_back(v);
+            s->stream = h->gstream;
+            s->capturing = true;
+        }
+        const int32_t hp = h->p;
+        cualign_status st = CUALIGN_OK;
+        cudaGraph_t g = nullptr;
+        if (cudaStreamBeginCapture(h->gstream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+            set_error("sharded step: graph capture could not start");
+            st = CUALIGN_ECUDA;
+        } else {
+            st = shard_iterate(h, 1);
+            const cudaError_t e2 = cudaStreamEndCapture(h->gstream, &g);
+            if (st == CUALIGN_OK && e2 != cudaSuccess) {
+                set_error("sharded step capture: %s", cudaGetErrorString(e2));
+                st = CUALIGN_ECUDA;
+            }
+            if (st == CUALIGN_OK && cudaGraphInstantiate(&h->shard_graph, g, 0) != cudaSuccess) {
+                set_error("sharded step: graph instantiate failed");
+                st = CUALIGN_ECUDA;
+            }
+            if (g) cudaGraphDestroy(g);
+        }
+        // what one replay launches / exchanges (per shard), then the counters
+        // as they were: the capture ran nothing
+        h->shard_step_counts.assign(S.size(), {});
+        for (size_t i = 0; i < S.size(); i++) {
+            cualign_bp *s = S[i];
+            auto &c = h->shard_step_counts[i];
+            c.launches = s->launches - saved[i].launches;
+            for (int k = 0; k < CUALIGN_NUM_KERNEL_CLASSES; k++)
+                c.class_launches[k] = s->class_launches[k] - saved[i].class_launches[k];
+            c.comm_calls = s->comm_calls - saved[i].comm_calls;
+            c.comm_bytes_in = s->comm_bytes_in - saved[i].comm_bytes_in;
+            s->stream = saved[i].stream;
+            s->p = saved[i].p;
+            s->launches = saved[i].launches;
+            for (int k = 0; k < CUALIGN_NUM_KERNEL_CLASSES; k++) s->class_launches[k] = saved[i].class_launches[k];
+            s->comm_calls = saved[i].comm_calls;
+            s->comm_bytes_in = saved[i].comm_bytes_in;
+            s->capturing = false;
+        }
+        h->p = hp;
+        (void)cudaGetLastError();
+        CA_TRY(st);
+        h->shard_graph_gh = gh;
+    }
+    CA_CUDA(cudaEventRecord(h->sync_ev[0], h->stream));
+    CA_CUDA(cudaStreamWaitEvent(h->gstream, h->sync_ev[0], 0));
+    CA_CUDA(cudaGraphLaunch(h->shard_graph, h->gstream));
+    CA_CUDA(cudaEventRecord(h->sync_ev[1], h->gstream));
+    CA_CUDA(cudaStreamWaitEvent(h->stream, h->sync_ev[1], 0));
+    for (size_t i = 0; i < S.size(); i++) {
+        cualign_bp *s = S[i];
+        const auto &c = h->shard_step_counts[i];
+        s->p += 1;
+        s->launches += c.launches;
+        for (int k = 0; k < CUALIGN_NUM_KERNEL_CLASSES; k++) s->class_launches[k] += c.class_launches[k];
+        s->comm_calls += c.comm_calls;
+        s->comm_bytes_in += c.comm_bytes_in;
+    }
+    if (!h->vshards.empty()) h->p += 1;
+    return CUALIGN_OK;
+}
+
 static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, RoundDev *trace)
 {
     if (h->world > 1) {
-        // sharded: eager per-step launches (the exchanges sit between kernels)
+        // sharded: the iteration replayed from its graph (eager with timing
+        // on: per-exchange events), the rounding's merge batches on the host
         cualign_bp *q = primary(h);
         for (int32_t k = 0; k < n_steps; k++) {
-            if (what & CUALIGN_RUN_ITERATE) CA_TRY(shard_iterate(h, 1));
+            if (what & CUALIGN_RUN_ITERATE) CA_TRY(h->timing ? shard_iterate(h, 1) : shard_iterate_graph(h));
             if (what & CUALIGN_RUN_ROUND) CA_TRY(shard_round(h));
             if (trace)
                 CA_CUDA(cudaMemcpyAsync(trace + k, q->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, q->stream));

@@ -176,6 +176,12 @@ struct cualign_bp {
     // 2 = rounding of buffer wb
     static constexpr int NSLOT = 11;  // + SERIAL_SLOT: iterate(1) then round, no fork
     cudaGraphExec_t graph[2][NSLOT] = {};                   // [timed][slot]
+    cudaGraphExec_t shard_graph = nullptr;                  // sharded: one iteration (all exchanges) as a graph
+    struct StepCounts {
+        int64_t launches = 0, class_launches[CUALIGN_NUM_KERNEL_CLASSES] = {}, comm_calls = 0, comm_bytes_in = 0;
+    };
+    std::vector<StepCounts> shard_step_counts;              // per shard: what one replay launches / exchanges
+    std::vector<const void *> shard_graph_gh;               // the shards' gamma tables the graph reads
     int64_t graph_launches[2][NSLOT] = {};                  // kernels per replay
     int64_t graph_class_launches[2][NSLOT][CUALIGN_NUM_KERNEL_CLASSES] = {};
     std::vector<std::pair<int, cualign::EventPair>> graph_events[NSLOT]; // timed graphs' event nodes
