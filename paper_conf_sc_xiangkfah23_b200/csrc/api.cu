@@ -843,6 +843,13 @@ static int default_schedule(cualign_bp *h)
 // stream pointed at it; re-captured when a shard's gamma table moves.
 static cualign_status shard_iterate_graph(cualign_bp *h)
 {
+    // NCCL connects peers lazily, at a channel's first use -- which must not
+    // happen inside a stream capture: the first sharded step of a handle runs
+    // eagerly, the graph is captured at the second
+    if (!h->shard_warm) {
+        h->shard_warm = true;
+        return shard_iterate(h, 1);
+    }
     std::vector<cualign_bp *> S = h->vshards.empty() ? std::vector<cualign_bp *>{h} : h->vshards;
     for (cualign_bp *s : S) CA_TRY(ensure_gh(s, (int64_t)s->p + 2));
     std::vector<const void *> gh;

@@ -181,6 +181,7 @@ struct cualign_bp {
         int64_t launches = 0, class_launches[CUALIGN_NUM_KERNEL_CLASSES] = {}, comm_calls = 0, comm_bytes_in = 0;
     };
     std::vector<StepCounts> shard_step_counts;              // per shard: what one replay launches / exchanges
+    bool shard_warm = false;                                // one eager sharded step done (NCCL connected)
     std::vector<const void *> shard_graph_gh;               // the shards' gamma tables the graph reads
     int64_t graph_launches[2][NSLOT] = {};                  // kernels per replay
     int64_t graph_class_launches[2][NSLOT][CUALIGN_NUM_KERNEL_CLASSES] = {};

@@ -51,8 +51,13 @@ def main():
         sz = h.sizes()
         e0, e1 = sz["edge_begin"], sz["edge_end"]
         rounds = []
-        for _ in range(args.iters):
-            h.iterate(1)
+        for it in range(args.iters):
+            # the later half through run(): the sharded step replayed from
+            # its captured graph (NCCL calls inside), the rounding eager
+            if it < args.iters // 2:
+                h.iterate(1)
+            else:
+                h.run(1, with_round=False)
             r = h.round()
             rounds.append([float(r[k]) for k in keys])
         st = h.get_state(with_S=False)
