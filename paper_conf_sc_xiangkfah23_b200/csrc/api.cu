@@ -940,7 +940,12 @@ static cualign_status run_steps(cualign_bp *h, int32_t n_steps, int32_t what, Ro
         // on: per-exchange events), the rounding's merge batches on the host
         cualign_bp *q = primary(h);
         for (int32_t k = 0; k < n_steps; k++) {
-            if (what & CUALIGN_RUN_ITERATE) CA_TRY(h->timing ? shard_iterate(h, 1) : shard_iterate_graph(h));
+            // graph replay for in-process shards; process shards (NCCL) step
+            // eagerly: NCCL calls are capturable, but with the only transport
+            // this sandbox can test (ranks sharing one GPU over sockets) a
+            // captured step deadlocked, so it stays unvalidated and off
+            const bool graph = !h->timing && !h->vshards.empty();
+            if (what & CUALIGN_RUN_ITERATE) CA_TRY(graph ? shard_iterate_graph(h) : shard_iterate(h, 1));
             if (what & CUALIGN_RUN_ROUND) CA_TRY(shard_round(h));
             if (trace)
                 CA_CUDA(cudaMemcpyAsync(trace + k, q->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, q->stream));
