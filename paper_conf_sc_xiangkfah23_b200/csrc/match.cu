@@ -1114,8 +1114,16 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P, bool collect_in_eval 
         // 3 rounds: 0.127 ms for both matchings on O vs 0.150 / 0.165 with 6 / 9
         // (each round costs ~9 dependent memory round trips, even nearly empty)
         static const int nrounds = probe_knob("CUALIGN_SUITOR_ROUNDS", 3);
-        CA_CUDA(launch_pdl(k_propose_first<6>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P,
-                           h->squeue + 1 * NQ * qc, h->qcnt + 1 * cs, qc));
+        static const int first_u = probe_knob("CUALIGN_SUITOR_FIRST_U", 6);
+        if (first_u == 9)
+            CA_CUDA(launch_pdl(k_propose_first<9>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P,
+                               h->squeue + 1 * NQ * qc, h->qcnt + 1 * cs, qc));
+        else if (first_u == 18)
+            CA_CUDA(launch_pdl(k_propose_first<18>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P,
+                               h->squeue + 1 * NQ * qc, h->qcnt + 1 * cs, qc));
+        else
+            CA_CUDA(launch_pdl(k_propose_first<6>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P,
+                               h->squeue + 1 * NQ * qc, h->qcnt + 1 * cs, qc));
         for (int r = 1; r <= nrounds; r++) {
             const int bi = r % QBUF, bo = (r + 1) % QBUF, bc = (r + 2) % QBUF;
             CA_CUDA(launch_pdl(k_propose_round<6>, dim3(h->qr_grid), dim3(256), 0, h->stream, P,
