@@ -1111,9 +1111,10 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P, bool collect_in_eval 
         P.qcnt = h->qcnt;
         KScope ks(h, CUALIGN_K_MATCH);
         const int64_t qc = h->qcap, cs = (int64_t)NQ * QSTRIDE;
-        // 3 rounds: 0.127 ms for both matchings on O vs 0.150 / 0.165 with 6 / 9
-        // (each round costs ~9 dependent memory round trips, even nearly empty)
-        static const int nrounds = probe_knob("CUALIGN_SUITOR_ROUNDS", 3);
+        // 2 rounds: 0.112 ms for both matchings on O (p = 80) vs 0.184 / 0.129
+        // / 0.121 / 0.130 with 0 / 1 / 3 / 4 (each round costs ~9 dependent
+        // memory round trips even nearly empty; the chain form takes the rest)
+        static const int nrounds = probe_knob("CUALIGN_SUITOR_ROUNDS", 2);
         static const int first_u = probe_knob("CUALIGN_SUITOR_FIRST_U", 6);
         if (first_u == 9)
             CA_CUDA(launch_pdl(k_propose_first<9>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P,
