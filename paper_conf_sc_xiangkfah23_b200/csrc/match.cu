@@ -953,12 +953,14 @@ k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, uns
             const int64_t q = base + u * nthr;
             ij[u] = q < P.npairs ? __ldg(P.pairs + q) : make_int2(-1, -1);
         }
-        // both instances' images of i and j: one 8-byte gather each
+        // both instances' images of i and j: one 8-byte gather each (pairs
+        // are sorted by i, so the i gathers mostly hit the same line; j is
+        // gathered only when i is matched in some instance)
 #pragma unroll
-        for (int u = 0; u < EVAL_U; u++) {
-            mi[u] = ij[u].x >= 0 ? P.mvA[ij[u].x] : make_int2(-1, -1);
-            mj[u] = ij[u].x >= 0 ? P.mvA[ij[u].y] : make_int2(-1, -1);
-        }
+        for (int u = 0; u < EVAL_U; u++) mi[u] = ij[u].x >= 0 ? P.mvA[ij[u].x] : make_int2(-1, -1);
+#pragma unroll
+        for (int u = 0; u < EVAL_U; u++)
+            mj[u] = (mi[u].x >= 0 || mi[u].y >= 0) ? P.mvA[ij[u].y] : make_int2(-1, -1);
 #pragma unroll
         for (int u = 0; u < EVAL_U; u++) {
             // M_y and M_z agree on most vertices (94 % on O): when both
