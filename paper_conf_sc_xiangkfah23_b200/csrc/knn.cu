@@ -85,7 +85,7 @@ __global__ void k_knn_prep(const float *__restrict__ Y, int32_t n, int32_t d, in
 
 // Partial top-k of one CTA: rows [rb*128, +128) x B tiles [t0, t1).
 // Output pv / pi: [row][split][half][k] (unsorted), idx INT_MAX = empty.
-template <int BN, int EH>
+template <int BN, int EH, int CPL>
 __global__ void __launch_bounds__(knn_threads<EH>(), 1)
 k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32_t n_a, int32_t n_b, int32_t KB,
          int32_t k, int32_t ntilesB, int32_t tiles_per_split, int32_t nstages, float *__restrict__ pv,
@@ -224,43 +224,56 @@ k_knn_tc(const uint8_t *__restrict__ Asw, const uint8_t *__restrict__ Bsw, int32
             mbar_wait(&tfull[buf], (uint32_t)(i >> 1) & 1u);
             tc_fence_after();
             const int vbase = (t0 + i) * BN;
+            // CPL chunks of 32 columns per TMEM wait: their loads are issued
+            // back to back, so the tcgen05.ld latency is paid once per CPL
+            // chunks (the epilogue, not the MMA, bounds this kernel)
+            const int nch = probe == 1 ? 0 : BN / 32; // probe 1: no epilogue (timing only)
 #pragma unroll 1
-            for (int c = half; c < (probe == 1 ? 0 : BN / 32); c += EH) { // probe 1: no epilogue (timing only)
-                uint32_t r[32];
+            for (int c0 = half; c0 < nch; c0 += EH * CPL) {
+                uint32_t r[CPL][32];
                 __syncwarp(); // .sync.aligned load: reconverge after a fold
-                tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN + c * 32), r);
+#pragma unroll
+                for (int cc = 0; cc < CPL; cc++) {
+                    const int c = c0 + cc * EH;
+                    if (c < nch) tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(buf * BN + c * 32), r[cc]);
+                }
                 tmem_ld_wait();
-                const int v0 = vbase + c * 32;
-                if (v0 + 32 > n_b) { // padding columns of the last tile never enter
 #pragma unroll
-                    for (int j = 0; j < 32; j++)
-                        if (v0 + j >= n_b) r[j] = __float_as_uint(-INFINITY);
-                }
-                // chunk max first (FMNMX3 tree): after the first tiles almost
-                // every chunk of every row is below the row's k-th best
-                float m4[4];
+                for (int cc = 0; cc < CPL; cc++) {
+                    const int c = c0 + cc * EH;
+                    if (c >= nch) break;
+                    const int v0 = vbase + c * 32;
+                    if (v0 + 32 > n_b) { // padding columns of the last tile never enter
 #pragma unroll
-                for (int t = 0; t < 4; t++) {
-                    float x = __uint_as_float(r[8 * t]);
+                        for (int j = 0; j < 32; j++)
+                            if (v0 + j >= n_b) r[cc][j] = __float_as_uint(-INFINITY);
+                    }
+                    // chunk max first (FMNMX3 tree): after the first tiles almost
+                    // every chunk of every row is below the row's k-th best
+                    float m4[4];
 #pragma unroll
-                    for (int j = 1; j < 8; j += 2)
-                        x = fmaxf(fmaxf(x, __uint_as_float(r[8 * t + j])),
-                                  __uint_as_float(r[8 * t + (j + 1 < 8 ? j + 1 : j)]));
-                    m4[t] = x;
-                }
-                const bool pass = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) > thr;
-                if (!__any_sync(0xffffffffu, pass)) continue; // warp-uniform
+                    for (int t = 0; t < 4; t++) {
+                        float x = __uint_as_float(r[cc][8 * t]);
 #pragma unroll
-                for (int g = 0; g < 4; g++) {
-                    // room for 8 more in every lane's buffer (warp-uniform fold)
-                    if (__any_sync(0xffffffffu, cnt > KNN_CB - 8)) fold();
+                        for (int j = 1; j < 8; j += 2)
+                            x = fmaxf(fmaxf(x, __uint_as_float(r[cc][8 * t + j])),
+                                      __uint_as_float(r[cc][8 * t + (j + 1 < 8 ? j + 1 : j)]));
+                        m4[t] = x;
+                    }
+                    const bool pass = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) > thr;
+                    if (!__any_sync(0xffffffffu, pass)) continue; // warp-uniform
 #pragma unroll
-                    for (int jj = 0; jj < 8; jj++) {
-                        const float val = __uint_as_float(r[8 * g + jj]);
-                        if (val > thr) {
-                            cv[cnt * KNN_BM + row] = val;
-                            ci[cnt * KNN_BM + row] = v0 + 8 * g + jj;
-                            cnt++;
+                    for (int g = 0; g < 4; g++) {
+                        // room for 8 more in every lane's buffer (warp-uniform fold)
+                        if (__any_sync(0xffffffffu, cnt > KNN_CB - 8)) fold();
+#pragma unroll
+                        for (int jj = 0; jj < 8; jj++) {
+                            const float val = __uint_as_float(r[cc][8 * g + jj]);
+                            if (val > thr) {
+                                cv[cnt * KNN_BM + row] = val;
+                                ci[cnt * KNN_BM + row] = v0 + 8 * g + jj;
+                                cnt++;
+                            }
                         }
                     }
                 }
@@ -335,12 +348,12 @@ __global__ void k_knn_merge(int32_t n_a, int32_t k, int32_t nsplit, const float 
     }
 }
 
-template <int BN, int EH>
+template <int BN, int EH, int CPL = 1>
 cualign_status knn_launch(cualign_bp *h, const uint8_t *Asw, const uint8_t *Bsw, int32_t n_a, int32_t n_b,
                           int32_t KB, int32_t k, float *pv, int32_t *pi, int32_t nsplit, int32_t tps,
                           int32_t nstages, size_t smem)
 {
-    auto fn = k_knn_tc<BN, EH>;
+    auto fn = k_knn_tc<BN, EH, CPL>;
     CA_CUDA(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int32_t ntilesB = (n_b + BN - 1) / BN;
     dim3 grid((unsigned)((n_a + KNN_BM - 1) / KNN_BM), (unsigned)nsplit);
@@ -437,7 +450,10 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
         KScope ks(h, CUALIGN_K_OTHER);
         const uint8_t *a8 = (const uint8_t *)Asw, *b8 = (const uint8_t *)Bsw;
         cualign_status lst;
+        static const int cpl = probe_knob("CUALIGN_KNN_CPL", 2);
         if (BN == 256 && EH == 2) lst = knn_launch<256, 2>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
+        else if (BN == 256 && cpl == 4) lst = knn_launch<256, 1, 4>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
+        else if (BN == 256 && cpl == 2) lst = knn_launch<256, 1, 2>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
         else if (BN == 256) lst = knn_launch<256, 1>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
         else if (EH == 2) lst = knn_launch<128, 2>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
         else lst = knn_launch<128, 1>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);

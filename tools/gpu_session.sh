@@ -30,6 +30,13 @@ for w in $WHAT; do
       echo "shardtests rc=$?"; tail -5 $OUT/shardtests.txt ;;
     n2)
       bash tools/run_bench_n2_onegpu.sh $TAG ;;
+    knntests)
+      timeout 600 python -m pytest tests/test_gpu_knn.py -q -p no:cacheprovider > $OUT/knntests.txt 2>&1
+      echo "knntests rc=$?"; tail -3 $OUT/knntests.txt ;;
+    knn_*)
+      ENVS=$(echo ${w#knn_} | tr ',' ' ')
+      env CUALIGN_LIB=$PROBES $ENVS timeout 600 python tools/bench_knn.py > $OUT/$w.jsonl 2> $OUT/$w.err
+      echo "$w rc=$?"; cat $OUT/$w.jsonl ;;
     sched)
       timeout 1200 python tools/probe_schedules.py > $OUT/sched.jsonl 2> $OUT/sched.err
       echo "sched rc=$?"; cat $OUT/sched.jsonl ;;
