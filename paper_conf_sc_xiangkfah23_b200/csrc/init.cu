@@ -678,25 +678,25 @@ cualign_status build_L(cualign_bp *h, LDev &L, const cualign_edges *E, bool devi
     // B-side incidence: stable radix sort of edge ids by b (ids stay ascending)
     CA_TRY(dalloc(h, &L.Bedge, (size_t)(m ? m : 1)));
     CA_TRY(dalloc(h, &L.Bptr, (size_t)nB + 1));
+    CA_TRY(dalloc(h, &L.Bcol, (size_t)m + 8)); // the sorted keys: b of every incidence entry (k_top2)
     {
-        TmpBuf keys_out, ids_in, tmp;
-        CA_CUDA(tmalloc(h, keys_out, sizeof(int32_t) * (m ? m : 1)));
+        TmpBuf ids_in, tmp;
         CA_CUDA(tmalloc(h, ids_in, sizeof(int32_t) * (m ? m : 1)));
         if (m) {
             k_iota<<<grid_for(m, 256, G), 256, 0, h->stream>>>(m, (int32_t *)ids_in.p);
             int end_bit = 1;
             while (end_bit < 31 && ((int64_t)1 << end_bit) < (int64_t)nB) end_bit++;
             size_t tbytes = 0;
-            CA_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tbytes, L.Lb, (int32_t *)keys_out.p,
+            CA_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tbytes, L.Lb, L.Bcol,
                                                     (int32_t *)ids_in.p, L.Bedge, (int)m, 0, end_bit,
                                                     h->stream));
             CA_CUDA(tmalloc(h, tmp, tbytes ? tbytes : 1));
-            CA_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tbytes, L.Lb, (int32_t *)keys_out.p,
+            CA_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tbytes, L.Lb, L.Bcol,
                                                     (int32_t *)ids_in.p, L.Bedge, (int)m, 0, end_bit,
                                                     h->stream));
         }
         k_rowptr_from_sorted<<<grid_for((int64_t)nB + 1, 256, G), 256, 0, h->stream>>>(
-            m, (int32_t *)keys_out.p, nB, L.Bptr);
+            m, L.Bcol, nB, L.Bptr);
         CA_CUDA(cudaGetLastError());
         CA_CUDA(cudaStreamSynchronize(h->stream)); // TmpBufs die here
     }
@@ -1056,9 +1056,9 @@ cualign_status tile_squares(cualign_bp *h)
 {
     const int log_b = h->tile_log_param < 0 ? 0 : (h->tile_log_param > 0 ? h->tile_log_param : SQ_TILE_LOG);
     h->sq_tile_log = 0;
-    if (log_b <= 0 || h->nsq < 2 || h->nsq >= INT32_MAX) return CUALIGN_OK;
+    if (log_b <= 0 || h->nsq < 2 || h->nsq >= INT32_MAX) return pack_squares(h);
     const uint32_t nblocks = (uint32_t)(((h->L.m - 1) >> log_b) + 1);
-    if (nblocks < 2 || (uint64_t)nblocks * nblocks >= (1ull << 32)) return CUALIGN_OK;
+    if (nblocks < 2 || (uint64_t)nblocks * nblocks >= (1ull << 32)) return pack_squares(h);
     int end_bit = 1;
     while ((1ull << end_bit) < (uint64_t)nblocks * nblocks) end_bit++;
     const int n = (int)h->nsq;
@@ -1086,6 +1086,101 @@ cualign_status tile_squares(cualign_bp *h)
     dfree(h, h->sq_ef);
     h->sq_ef = sorted;
     h->sq_tile_log = log_b;
+    return pack_squares(h);
+}
+
+// Packed square indices.  The squares
+// are cut into chunks of <= SQP_CHUNK consecutive squares inside which every
+// f lies in one 2^SQP_FBITS block (fb = its start) and every e in
+// [eb, eb + 2^SQP_EBITS) with eb = the chunk's first e; square q then packs
+// into one 32-bit word (e - eb) << SQP_FBITS | (f - fb), half of the int2.
+// Windows of SQP_CHUNK squares (also cut at nsq_split) are split greedily by
+// one thread each: pass 1 counts the chunks per window, pass 2 writes them.
+template <bool FILL>
+__global__ void k_sqp_pack(int64_t nsq, int64_t split, const int2 *__restrict__ sq_ef,
+                           int64_t *__restrict__ wcnt, int4 *__restrict__ desc, uint32_t *__restrict__ words)
+{
+    const int64_t nwin = (nsq + SQP_CHUNK - 1) / SQP_CHUNK;
+    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nwin;
+         w += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t q0 = w * SQP_CHUNK, q1 = (q0 + SQP_CHUNK < nsq) ? q0 + SQP_CHUNK : nsq;
+        int64_t c = FILL ? (w ? wcnt[w - 1] : 0) : 0; // wcnt: inclusive prefix after pass 1
+        int64_t cs = q0;
+        int eb = 0, fb = 0;
+        for (int64_t q = q0; q < q1; q++) {
+            const int2 ef = sq_ef[q];
+            const int fblk = (int)(((uint32_t)ef.y >> SQP_FBITS) << SQP_FBITS);
+            const bool cut = q == q0 || q == split || fblk != fb || ef.x < eb ||
+                             (int64_t)ef.x - eb >= (1ll << SQP_EBITS);
+            if (cut) {
+                if (FILL && q > q0) desc[c] = make_int4((int)cs, (int)(q - cs), eb, fb);
+                if (q > q0) c++;
+                cs = q;
+                eb = ef.x;
+                fb = fblk;
+            }
+            if (FILL) words[q] = ((uint32_t)(ef.x - eb) << SQP_FBITS) | (uint32_t)(ef.y - fb);
+        }
+        if (FILL) desc[c] = make_int4((int)cs, (int)(q1 - cs), eb, fb);
+        else wcnt[w] = c + 1;
+    }
+}
+
+// first chunk starting at or after q (chunk starts ascend)
+__global__ void k_sqp_find(int64_t n, const int4 *__restrict__ desc, int64_t q, int64_t *__restrict__ out)
+{
+    int64_t lo = 0, hi = n;
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (desc[mid].x < q) lo = mid + 1;
+        else hi = mid;
+    }
+    *out = lo;
+}
+
+cualign_status pack_squares(cualign_bp *h)
+{
+    if (h->sqp_w) dfree(h, h->sqp_w);
+    if (h->sqp_desc) dfree(h, h->sqp_desc);
+    h->sqp_w = nullptr;
+    h->sqp_desc = nullptr;
+    h->sqp_nchunks = 0;
+    h->sqp_split_chunk = 0;
+    const int64_t n = h->nsq;
+    if (n < 1 || n >= INT32_MAX) return CUALIGN_OK;
+    const int64_t nwin = (n + SQP_CHUNK - 1) / SQP_CHUNK;
+    TmpBuf cnt, tmp, res;
+    CA_CUDA(tmalloc(h, cnt, sizeof(int64_t) * (size_t)nwin));
+    CA_CUDA(tmalloc(h, res, sizeof(int64_t)));
+    int64_t *wc = (int64_t *)cnt.p;
+    KScope ks(h, CUALIGN_K_INIT);
+    const int grid = grid_for(nwin, 128, h->num_sms * 16);
+    k_sqp_pack<false><<<grid, 128, 0, h->stream>>>(n, h->nsq_split, h->sq_ef, wc, nullptr, nullptr);
+    CA_CUDA(cudaGetLastError());
+    size_t tb = 0;
+    CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, wc, wc, (int)nwin, h->stream));
+    CA_CUDA(tmalloc(h, tmp, tb ? tb : 1));
+    CA_CUDA(cub::DeviceScan::InclusiveSum(tmp.p, tb, wc, wc, (int)nwin, h->stream));
+    int64_t nch = 0;
+    CA_CUDA(cudaMemcpyAsync(&nch, wc + nwin - 1, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    // chunks far below SQP_CHUNK (an untiled order over m > 2^SQP_FBITS
+    // edges) would starve the bulk copies: keep the int2 stream then
+    if (nch > 2 * nwin) return CUALIGN_OK;
+    CA_TRY(dalloc(h, &h->sqp_w, (size_t)n + 8)); // +8: 16-byte bulk-copy tails
+    CA_TRY(dalloc(h, &h->sqp_desc, (size_t)nch));
+    CA_CUDA(cudaMemsetAsync(h->sqp_w + n, 0, 8 * sizeof(uint32_t), h->stream));
+    k_sqp_pack<true><<<grid, 128, 0, h->stream>>>(n, h->nsq_split, h->sq_ef, wc, h->sqp_desc, h->sqp_w);
+    CA_CUDA(cudaGetLastError());
+    int64_t sc = 0;
+    if (h->nsq_split > 0) {
+        k_sqp_find<<<1, 1, 0, h->stream>>>(nch, h->sqp_desc, h->nsq_split, (int64_t *)res.p);
+        CA_CUDA(cudaGetLastError());
+        CA_CUDA(cudaMemcpyAsync(&sc, res.p, sizeof(int64_t), cudaMemcpyDeviceToHost, h->stream));
+    }
+    CA_CUDA(cudaStreamSynchronize(h->stream));
+    h->sqp_nchunks = nch;
+    h->sqp_split_chunk = sc;
     return CUALIGN_OK;
 }
 

@@ -59,6 +59,7 @@ struct LDev {
     double *w = nullptr;
     int64_t *Arow = nullptr, *Bptr = nullptr;
     int32_t *Bedge = nullptr;
+    int32_t *Bcol = nullptr; // m (+8): b of every B-incidence entry (Lb in Bedge order)
 };
 
 // Device-side round bookkeeping (persistent across rounds: best).
@@ -113,6 +114,7 @@ struct cualign_bp {
     double2 *Btop_all = nullptr;         // world x nB gathered partials
     int64_t *Bptr_loc = nullptr;         // B incidence of the owned edges (top-2 partials)
     int32_t *Bedge_loc = nullptr;
+    int32_t *Bcol_loc = nullptr;         // b of every local incidence entry (k_top2)
     // sharded square-pass halo (SURVEY §8(e) "S halo"): the squares {e < f}
     // of the owned rows touch f > e, i.e. edges of this or HIGHER shards only.
     // need: sorted remote f this shard reads u_f of and adds F_fe to, grouped
@@ -137,6 +139,13 @@ struct cualign_bp {
     double2 *sq_val = nullptr;   // nsq: (S^p_ef, S^p_fe)
     float2 *sq_val32 = nullptr;  // same, CUALIGN_FLAG_FP32_S storage (sq_val unused then)
     longlong2 *sq_pos = nullptr; // nsq: (pos(e,f), pos(f,e)) in the CSR; built lazily
+    // packed square stream of the fast square pass (DESIGN.md "Packed square
+    // indices"): word q = (e - eb) << SQP_FBITS | (f - fb) for the chunk's
+    // (eb, fb); chunks of <= SQP_CHUNK consecutive squares, int4 (q0, n, eb, fb)
+    uint32_t *sqp_w = nullptr;   // nsq (+4 padding)
+    int4 *sqp_desc = nullptr;    // sqp_nchunks
+    int64_t sqp_nchunks = 0;     // 0: packed stream not built (the int2 stream is used)
+    int64_t sqp_split_chunk = 0; // first chunk at or after nsq_split (sharded square parts)
 
     // fixed-point accumulator of the F row sums (fast mode)
     int fp_bits = 0;
@@ -151,6 +160,8 @@ struct cualign_bp {
     int64_t nchunks = 0;                // B incidence chunks (k_top2B load balance)
     int64_t *Bcp = nullptr;             // nB+1: chunks of B vertex b are Bcp[b]..Bcp[b+1]-1
     int4 *cdesc = nullptr;              // nchunks: (start, end, owning B vertex, first chunk of a hub or -1)
+    double2 *t2part = nullptr;          // k_top2: 2 partial (max1, max2) per window (A windows, then B windows)
+    unsigned int *Acnt = nullptr;       // nA: windows finished (A rows spanning windows; last-arriver merge)
     double2 *Bct = nullptr;             // nchunks: (max1, max2) of z^p over the chunk
     unsigned int *Bcnt = nullptr;       // nB: chunks finished (hub columns' last-arriver merge)
     unsigned int *sq_ctr = nullptr;     // 2: square-pass chunk queue head, CTAs done (self-resetting)
@@ -357,6 +368,10 @@ cualign_status ensure_sq_pos(cualign_bp *h);
 cualign_status ensure_csr(cualign_bp *h);
 cualign_status tile_squares(cualign_bp *h);
 constexpr int SQ_TILE_LOG = 21; // square tiles: blocks of 2^21 edges (2 x 32 MB of u + tacc per tile)
+cualign_status pack_squares(cualign_bp *h); // packed square stream from sq_ef (after every reorder)
+constexpr int SQP_CHUNK = 512;              // squares per packed chunk (= square-pass stage)
+constexpr int SQP_FBITS = 21;               // f - fb in the low bits (f blocks of 2^21 = the tile blocks)
+constexpr int SQP_EBITS = 32 - SQP_FBITS;   // e - eb in the high bits
 
 // api.cu
 void invalidate_graphs(cualign_bp *h);

@@ -478,7 +478,7 @@ cualign_status split_squares(cualign_bp *s)
     CA_CUDA(cudaMemcpyAsync(&remote, cnt.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s->stream));
     CA_CUDA(cudaStreamSynchronize(s->stream));
     s->nsq_split = ((n - remote) / 2) * 2;
-    return CUALIGN_OK;
+    return pack_squares(s); // the order changed; chunks are also cut at nsq_split
 }
 
 // The square-pass halo of every shard: mark the remote f of the owned
