@@ -33,7 +33,6 @@
 #include <cooperative_groups.h>
 #include <cub/cub.cuh>
 #include <math.h>
-#include <climits>
 
 namespace cg = cooperative_groups;
 
@@ -173,196 +172,6 @@ __global__ void __launch_bounds__(256) k_top2(Top2Args T)
             }
         }
     }
-}
-
-// ---------------------------------------------- flat segmented top-2 (default)
-// The same per-vertex (max1, max2) as k_top2, over flat windows instead of
-// per-vertex tiles: a side is a sequence of entries [base, end) whose ids
-// (A row / B column) ascend -- A: the edges, id La[e], value y^p[e]; B: the
-// B incidence, id Bcol[i], value z^p[Bedge[i]] -- cut into windows of
-// T2W = 256 entries (aligned to multiples of T2W), one warp per window, 8
-// consecutive entries per lane.  Every load is independent of the others
-// (two int4 id loads, B: two int4 edge loads, then 8 value loads per lane),
-// where the tile form chained chunk descriptor -> edge -> value.  A lane
-// reduces its own runs sequentially; a segmented warp scan (key = the id of
-// the lane's last run) joins runs across lanes.  A run that is a whole id
-// writes top[id]; the id that starts before the window or continues after it
-// writes a partial to part[2 w] (the window's first id) or part[2 w + 1] (its
-// last id), and the last of its windows to finish merges them (counter per id).
-constexpr int T2W = 256;
-
-struct T2Side {
-    int64_t base, end;      // entries [base, end)
-    int64_t w0, nwin;       // first window (absolute, base / T2W), windows
-    const int32_t *id;      // id per entry (ascending over [base, end))
-    const int32_t *gidx;    // B: edge per entry (value = val[gidx[i]]); A: null (value = val[i])
-    const double *val;
-    const int64_t *ptr;     // entries of id c: ptr[c] .. ptr[c+1]-1
-    double2 *top;
-    double2 *part;          // 2 per window
-    unsigned int *cnt;      // per id
-};
-struct Top2FArgs {
-    T2Side s[2];
-};
-
-__device__ __forceinline__ void t2_load_ids(const int32_t *__restrict__ p, int64_t i0, int64_t base, int64_t end,
-                                            int (&c)[8])
-{
-    if (i0 >= base && i0 + 8 <= end) {
-        const int4 a = __ldg(reinterpret_cast<const int4 *>(p + i0));
-        const int4 b = __ldg(reinterpret_cast<const int4 *>(p + i0 + 4));
-        c[0] = a.x; c[1] = a.y; c[2] = a.z; c[3] = a.w;
-        c[4] = b.x; c[5] = b.y; c[6] = b.z; c[7] = b.w;
-    } else {
-#pragma unroll
-        for (int j = 0; j < 8; j++) {
-            const int64_t i = i0 + j;
-            c[j] = i < base ? -1 : (i >= end ? INT_MAX : __ldg(p + i));
-        }
-    }
-}
-
-__global__ void __launch_bounds__(256) k_top2f(Top2FArgs T)
-{
-    pdl_wait();
-    const int lane = threadIdx.x & 31;
-    const int64_t wv = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int sd = wv >= T.s[0].nwin;
-    if (wv >= T.s[0].nwin + T.s[1].nwin) return;
-    const int64_t w = wv - (sd ? T.s[0].nwin : 0);
-    const int64_t base = sd ? T.s[1].base : T.s[0].base, end = sd ? T.s[1].end : T.s[0].end;
-    const int64_t w0 = sd ? T.s[1].w0 : T.s[0].w0;
-    const int32_t *__restrict__ idp = sd ? T.s[1].id : T.s[0].id;
-    const int32_t *__restrict__ gidx = sd ? T.s[1].gidx : T.s[0].gidx;
-    const double *__restrict__ val = sd ? T.s[1].val : T.s[0].val;
-    const int64_t *__restrict__ ptr = sd ? T.s[1].ptr : T.s[0].ptr;
-    double2 *__restrict__ top = sd ? T.s[1].top : T.s[0].top;
-    double2 *__restrict__ part = sd ? T.s[1].part : T.s[0].part;
-    unsigned int *__restrict__ cnt = sd ? T.s[1].cnt : T.s[0].cnt;
-
-    const int64_t ws = (w0 + w) * T2W;
-    const int64_t vlo = ws > base ? ws : base;                          // first valid entry
-    const int64_t vhi = ws + T2W < end ? ws + T2W : end;                // one past the last
-    const int64_t i0 = ws + lane * 8;
-    int c[8];
-    double v[8];
-    t2_load_ids(idp, i0, base, end, c);
-    if (gidx) {
-        int g[8];
-        t2_load_ids(gidx, i0, base, end, g);
-#pragma unroll
-        for (int j = 0; j < 8; j++) v[j] = (c[j] >= 0 && c[j] != INT_MAX) ? __ldg(val + g[j]) : -INFINITY;
-    } else {
-#pragma unroll
-        for (int j = 0; j < 8; j++) v[j] = (c[j] >= 0 && c[j] != INT_MAX) ? __ldg(val + i0 + j) : -INFINITY;
-    }
-    // the window's first and last id, and whether they extend past the window
-    const int bfirst = __ldg(idp + vlo), blast = __ldg(idp + vhi - 1);
-    const bool cont_before = __ldg(ptr + bfirst) < vlo;
-    const bool cont_after = __ldg(ptr + blast + 1) > vhi;
-
-    auto emit = [&](int id, double m1, double m2) {
-        if (id < 0 || id == INT_MAX) return;
-        const bool first = id == bfirst;
-        if (!((first && cont_before) || (id == blast && cont_after))) {
-            top[id] = make_double2(m1, m2);
-            return;
-        }
-        // partial: this window's share of an id that spans windows
-        part[2 * w + (first ? 0 : 1)] = make_double2(m1, m2);
-        const int64_t lo = __ldg(ptr + id), hi = __ldg(ptr + id + 1);
-        const int64_t wa = (lo > base ? lo : base) / T2W - w0;
-        const int64_t wb = ((hi < end ? hi : end) - 1) / T2W - w0;
-        __threadfence();
-        const unsigned int prev = atomicAdd(cnt + id, 1u);
-        if (prev == (unsigned int)(wb - wa)) {
-            __threadfence();
-            double r1 = -INFINITY, r2 = -INFINITY;
-            for (int64_t x = wa; x <= wb; x++) {
-                const int64_t xs = (w0 + x) * T2W;
-                const bool idfirst = lo <= (xs > base ? xs : base); // id is window x's first id
-                const double2 o = __ldcg(part + 2 * x + (idfirst ? 0 : 1));
-                top2_merge(r1, r2, o.x, o.y);
-            }
-            top[id] = make_double2(r1, r2);
-            cnt[id] = 0u; // ready for the next iteration
-        }
-    };
-
-    // lane-local runs: the first (id c[0]) and last (id c[7]) are joined
-    // with the neighbouring lanes; inner runs are whole ids
-    double p1 = -INFINITY, p2 = -INFINITY; // run of c[0], if it is not also the last run
-    int cur = c[0];
-    double r1 = v[0], r2 = -INFINITY;
-#pragma unroll
-    for (int j = 1; j < 8; j++) {
-        if (c[j] == cur) {
-            top2_push(r1, r2, v[j]);
-        } else {
-            if (cur == c[0]) {
-                p1 = r1;
-                p2 = r2;
-            } else {
-                emit(cur, r1, r2);
-            }
-            cur = c[j];
-            r1 = v[j];
-            r2 = -INFINITY;
-        }
-    }
-    // segmented inclusive scan of the last runs over the lanes (ids ascend,
-    // so equal keys are one contiguous run of lanes)
-    const int key = c[7];
-    double s1 = r1, s2 = r2;
-#pragma unroll
-    for (int off = 1; off < 32; off <<= 1) {
-        const double o1 = __shfl_up_sync(FULL_MASK, s1, off);
-        const double o2 = __shfl_up_sync(FULL_MASK, s2, off);
-        const int ok = __shfl_up_sync(FULL_MASK, key, off);
-        if (lane >= off && ok == key) top2_merge(s1, s2, o1, o2);
-    }
-    const int prev_key = __shfl_up_sync(FULL_MASK, key, 1);
-    const double q1 = __shfl_up_sync(FULL_MASK, s1, 1);
-    const double q2 = __shfl_up_sync(FULL_MASK, s2, 1);
-    const int next_c0 = __shfl_down_sync(FULL_MASK, c[0], 1);
-    if (c[0] != key) {
-        // the first run ends in this lane: joined with the previous lanes' run
-        if (lane > 0 && prev_key == c[0]) top2_merge(p1, p2, q1, q2);
-        emit(c[0], p1, p2);
-    }
-    if (lane == 31 || next_c0 != key) emit(key, s1, s2);
-}
-
-// the two sides of k_top2f for this handle (A: owned edges; B: the owned
-// edges' incidence when sharded, else all of it)
-Top2FArgs top2f_args(const cualign_bp *h)
-{
-    const bool sh = h->world > 1;
-    Top2FArgs T;
-    auto side = [](T2Side &S, int64_t base, int64_t end) {
-        S.base = base;
-        S.end = end;
-        S.w0 = base / T2W;
-        S.nwin = end > base ? (end - 1) / T2W - S.w0 + 1 : 0;
-    };
-    side(T.s[0], h->e0, h->e1);
-    T.s[0].id = h->L.La;
-    T.s[0].gidx = nullptr;
-    T.s[0].val = h->yp;
-    T.s[0].ptr = h->L.Arow;
-    T.s[0].top = h->Atop;
-    T.s[0].part = h->t2part;
-    T.s[0].cnt = h->Acnt;
-    side(T.s[1], 0, sh ? h->e1 - h->e0 : h->L.m);
-    T.s[1].id = sh ? h->Bcol_loc : h->L.Bcol;
-    T.s[1].gidx = sh ? h->Bedge_loc : h->L.Bedge;
-    T.s[1].val = h->zp;
-    T.s[1].ptr = sh ? h->Bptr_loc : h->L.Bptr;
-    T.s[1].top = sh ? h->Btop_part : h->Btop;
-    T.s[1].part = h->t2part ? h->t2part + 2 * T.s[0].nwin : nullptr;
-    T.s[1].cnt = h->Bcnt;
-    return T;
 }
 
 struct EdgeArgs {
@@ -1155,10 +964,10 @@ cualign_status build_local_incidence(cualign_bp *h)
     const int64_t nB = h->L.nB, ml = h->e1 - h->e0;
     CA_TRY(dalloc(h, &h->Bedge_loc, (size_t)(ml ? ml : 1)));
     CA_TRY(dalloc(h, &h->Bptr_loc, (size_t)nB + 1));
-    CA_TRY(dalloc(h, &h->Bcol_loc, (size_t)ml + 8));
-    TmpBuf ib, tb_;
+    TmpBuf kb, ib, tb_;
+    CA_CUDA(tmalloc(h, kb, sizeof(int32_t) * (size_t)(ml ? ml : 1)));
     CA_CUDA(tmalloc(h, ib, sizeof(int32_t) * (size_t)(ml ? ml : 1)));
-    int32_t *keys = h->Bcol_loc, *ids = (int32_t *)ib.p;
+    int32_t *keys = (int32_t *)kb.p, *ids = (int32_t *)ib.p;
     void *tmp = nullptr;
     cualign_status st = CUALIGN_OK;
     if (ml) {
@@ -1206,14 +1015,7 @@ cualign_status bp_setup(cualign_bp *h)
         k_fill_neg_inf<<<grid_for(nB + 1, 256, h->num_sms * 8), 256, 0, h->stream>>>(nB + 1, h->Btop_part);
         CA_CUDA(cudaGetLastError());
     }
-    // k_top2f: window partials, per-A-row counters
-    {
-        const Top2FArgs T = top2f_args(h);
-        CA_TRY(dalloc(h, &h->t2part, (size_t)(2 * (T.s[0].nwin + T.s[1].nwin) + 2)));
-        CA_TRY(dalloc(h, &h->Acnt, (size_t)nA + 1));
-        CA_CUDA(cudaMemsetAsync(h->Acnt, 0, sizeof(unsigned int) * ((size_t)nA + 1), h->stream));
-    }
-    // B-side chunks for k_top2 (per-vertex tile form, probe build)
+    // B-side chunks for k_top2
     CA_TRY(dalloc(h, &h->Bcp, (size_t)nB + 1));
     CA_CUDA(cudaMemsetAsync(h->Bcp, 0, sizeof(int64_t), h->stream));
     if (nB > 0) {
@@ -1249,15 +1051,7 @@ cualign_status bp_fsum(cualign_bp *h)
 // per-vertex top-2 of the current y^p (A rows) and z^p (B columns)
 cualign_status bp_top2(cualign_bp *h)
 {
-    static const int flat = probe_knob("CUALIGN_TOP2_FLAT", 0); // probe build: 1 = flat windows (k_top2f)
-    if (h->L.m > 0 && flat) {
-        KScope ks(h, CUALIGN_K_TOP2);
-        const Top2FArgs T = top2f_args(h);
-        const int64_t nw = T.s[0].nwin + T.s[1].nwin;
-        if (nw > 0)
-            CA_CUDA(launch_pdl(k_top2f, dim3(grid_for(nw * 32, 256, 1 << 30)), dim3(256), 0, h->stream, T));
-        CA_CUDA(cudaGetLastError());
-    } else if (h->L.m > 0) {
+    if (h->L.m > 0) {
         KScope ks(h, CUALIGN_K_TOP2);
         const bool sh = h->world > 1;
         Top2Args T{(int64_t)(h->a1 - h->a0), h->nchunks, (int64_t)h->a0, h->L.Arow, h->cdesc, h->Bcp,

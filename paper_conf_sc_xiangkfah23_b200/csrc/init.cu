@@ -678,25 +678,25 @@ cualign_status build_L(cualign_bp *h, LDev &L, const cualign_edges *E, bool devi
     // B-side incidence: stable radix sort of edge ids by b (ids stay ascending)
     CA_TRY(dalloc(h, &L.Bedge, (size_t)(m ? m : 1)));
     CA_TRY(dalloc(h, &L.Bptr, (size_t)nB + 1));
-    CA_TRY(dalloc(h, &L.Bcol, (size_t)m + 8)); // the sorted keys: b of every incidence entry (k_top2)
     {
-        TmpBuf ids_in, tmp;
+        TmpBuf keys_out, ids_in, tmp;
+        CA_CUDA(tmalloc(h, keys_out, sizeof(int32_t) * (m ? m : 1)));
         CA_CUDA(tmalloc(h, ids_in, sizeof(int32_t) * (m ? m : 1)));
         if (m) {
             k_iota<<<grid_for(m, 256, G), 256, 0, h->stream>>>(m, (int32_t *)ids_in.p);
             int end_bit = 1;
             while (end_bit < 31 && ((int64_t)1 << end_bit) < (int64_t)nB) end_bit++;
             size_t tbytes = 0;
-            CA_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tbytes, L.Lb, L.Bcol,
+            CA_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tbytes, L.Lb, (int32_t *)keys_out.p,
                                                     (int32_t *)ids_in.p, L.Bedge, (int)m, 0, end_bit,
                                                     h->stream));
             CA_CUDA(tmalloc(h, tmp, tbytes ? tbytes : 1));
-            CA_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tbytes, L.Lb, L.Bcol,
+            CA_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tbytes, L.Lb, (int32_t *)keys_out.p,
                                                     (int32_t *)ids_in.p, L.Bedge, (int)m, 0, end_bit,
                                                     h->stream));
         }
         k_rowptr_from_sorted<<<grid_for((int64_t)nB + 1, 256, G), 256, 0, h->stream>>>(
-            m, L.Bcol, nB, L.Bptr);
+            m, (int32_t *)keys_out.p, nB, L.Bptr);
         CA_CUDA(cudaGetLastError());
         CA_CUDA(cudaStreamSynchronize(h->stream)); // TmpBufs die here
     }

@@ -59,7 +59,6 @@ struct LDev {
     double *w = nullptr;
     int64_t *Arow = nullptr, *Bptr = nullptr;
     int32_t *Bedge = nullptr;
-    int32_t *Bcol = nullptr; // m (+8): b of every B-incidence entry (Lb in Bedge order)
 };
 
 // Device-side round bookkeeping (persistent across rounds: best).
@@ -114,7 +113,6 @@ struct cualign_bp {
     double2 *Btop_all = nullptr;         // world x nB gathered partials
     int64_t *Bptr_loc = nullptr;         // B incidence of the owned edges (top-2 partials)
     int32_t *Bedge_loc = nullptr;
-    int32_t *Bcol_loc = nullptr;         // b of every local incidence entry (k_top2)
     // sharded square-pass halo (SURVEY §8(e) "S halo"): the squares {e < f}
     // of the owned rows touch f > e, i.e. edges of this or HIGHER shards only.
     // need: sorted remote f this shard reads u_f of and adds F_fe to, grouped
@@ -160,8 +158,6 @@ struct cualign_bp {
     int64_t nchunks = 0;                // B incidence chunks (k_top2B load balance)
     int64_t *Bcp = nullptr;             // nB+1: chunks of B vertex b are Bcp[b]..Bcp[b+1]-1
     int4 *cdesc = nullptr;              // nchunks: (start, end, owning B vertex, first chunk of a hub or -1)
-    double2 *t2part = nullptr;          // k_top2: 2 partial (max1, max2) per window (A windows, then B windows)
-    unsigned int *Acnt = nullptr;       // nA: windows finished (A rows spanning windows; last-arriver merge)
     double2 *Bct = nullptr;             // nchunks: (max1, max2) of z^p over the chunk
     unsigned int *Bcnt = nullptr;       // nB: chunks finished (hub columns' last-arriver merge)
     unsigned int *sq_ctr = nullptr;     // 2: square-pass chunk queue head, CTAs done (self-resetting)
