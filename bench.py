@@ -32,8 +32,6 @@ if ROOT not in sys.path:
 import numpy as np
 
 METRIC = "BP iterations/sec and squares/sec; end-to-end align time at 1/2/4/8 B200"
-CONFIGS_DESC_O = ("ontology-shaped: clustered power-law n_A=3e5 (avg deg 18), B=P(A[V']) |V'|=2e5 +5%; "
-                  "proxy k=16.67 -> m~5e6; s~1e8")
 UNIT = "iterations/s"
 # algorithmic bytes: (2*sigma + 4) per nonzero of S, (9*sigma + 8) per L edge
 SIGMA = 8
@@ -211,7 +209,7 @@ def oracle_on_O(n_warm, n_steps, pin_core=0):
     except (AttributeError, OSError):
         cores = None
     return {"gen_s": t1 - t0, "create_s": t2 - t1, "step_s": step_s, "m": o.m, "s": o.s, "cores": cores,
-            "pinned_core": pin_core, "n_warm": n_warm, "n_steps": n_steps}
+            "pinned_core": pin_core, "n_warm": n_warm, "n_steps": n_steps, "inst": inst}
 
 
 def start_oracle_child(n_steps):
@@ -240,6 +238,20 @@ def finish_oracle_child(proc):
             "step_s": d["step_s"], "create_s": d["create_s"], "host": host_info()}
 
 
+def workload_config(name, scale, inst, m, s, world, weak, exact=False, fp32=False):
+    """The bench line's `config` (both arms print the same one for the same
+    workload)."""
+    squares = s // 2
+    return {"workload": f"{name}: " + inst.meta["desc"], "scale": scale,
+            "n_a": inst.A.n, "n_b": inst.B.n, "m": m, "s": s, "squares": squares,
+            "alpha": inst.alpha, "beta": inst.beta, "gamma": inst.gamma,
+            "parallelism": (f"A-vertex-block shards x{world} (NCCL)" if world > 1 else "single"),
+            "value_unit_note": ("O-equivalent iterations/s: iterations/s x squares / squares(O)"
+                                if weak else "iterations/s of this instance"),
+            "l2": "inputs larger than L2 (square layout %.2f GB vs 126 MB L2)" % (24 * squares / 1e9),
+            "mode": ("exact" if exact else "fast") + ("+fp32S" if fp32 else "")}
+
+
 def run_reference(args, rank, world):
     """--impl reference: the oracle as it stands on one host core, on the SAME
     workload as our arm (full config O), W warm-up and K timed steps, a step =
@@ -257,7 +269,7 @@ def run_reference(args, rank, world):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000.0 * total / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
-            "config": {"workload": "O: " + CONFIGS_DESC_O, "m": d["m"], "s": d["s"], "sample": sample},
+            "config": workload_config("O", 1.0, d["inst"], d["m"], d["s"], 1, False),
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": d["cores"], "kind": "oracle", "sample": sample,
                              "host": host_info()},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -406,7 +418,9 @@ def main():
     ap.add_argument("--no-knn", action="store_true", help="skip the NEXT-2 kNN measurement")
     args = ap.parse_args()
     if args.oracle_child is not None:
-        print(json.dumps(oracle_on_O(0, args.oracle_child)), flush=True)
+        d = oracle_on_O(0, args.oracle_child)
+        d.pop("inst")
+        print(json.dumps(d), flush=True)
         return
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
@@ -685,14 +699,7 @@ def main():
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
         "scaling": "strong" if (world > 1 and args.strong) else "weak", "vs_baseline": None,
         "dtype": "f64", "data": "synthetic",
-        "config": {"workload": f"{args.config}: " + inst.meta["desc"], "scale": args.scale,
-                   "n_a": inst.A.n, "n_b": inst.B.n, "m": m, "s": s, "squares": squares,
-                   "alpha": inst.alpha, "beta": inst.beta, "gamma": inst.gamma,
-                   "parallelism": (f"A-vertex-block shards x{world} (NCCL)" if world > 1 else "single"),
-                   "value_unit_note": ("O-equivalent iterations/s: iterations/s x squares / squares(O)"
-                                       if weak else "iterations/s of this instance"),
-                   "l2": "inputs larger than L2 (square layout %.2f GB vs 126 MB L2)" % (24 * squares / 1e9),
-                   "mode": ("exact" if args.exact else "fast") + ("+fp32S" if args.fp32 else "")},
+        "config": workload_config(args.config, args.scale, inst, m, s, world, weak, args.exact, args.fp32),
         "squares_per_s": squares * args.steps / (elapsed_ms / 1e3),
         "bp_iters_per_s": 1e3 / bp_ms if bp_ms > 0 else None,
         "round_ms": round_ms, "bp_ms": bp_ms, "init_s": init_s,

@@ -64,6 +64,15 @@ print('ms per step, first 40:', ms[:40]); print('mean 6-25', sum(ms[5:25])/20, '
         timeout 1200 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_workload.py > $OUT/sanitize_$tool.txt 2>&1
         echo "sanitize $tool rc=$?"; tail -4 $OUT/sanitize_$tool.txt
       done ;;
+    bw_*)
+      # the driver's bench window (20 steps after 5) with the probe build and env: bw_NAME=V,NAME2=V
+      ENVS=$(echo ${w#bw_} | tr ',' ' ')
+      env CUALIGN_LIB=$PROBES $ENVS timeout 600 python bench.py --steps 20 --warmup 5 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/$w.json 2> $OUT/$w.err
+      echo "$w rc=$?"; python -c "import json; d=json.load(open('$OUT/$w.json')); print(round(d['value'],1), {k: round(v,4) for k,v in d['kernel_ms_per_step'].items()})" ;;
+    kernw)
+      # in-situ per-kernel durations inside the driver's window (p = 6 .. 25)
+      timeout 300 python tools/probe_kernels.py --pre 5 --n 20 > $OUT/kernw.json 2> $OUT/kernw.err
+      echo "kernw rc=$?"; python -c "import json,sys; d=json.load(open('$OUT/kernw.json')); [print(p, {k: round(v['us_per_step'],1) for k,v in d[p].items()}) for p in d]" ;;
     kern*)
       # in-situ per-kernel durations (CUPTI via torch.profiler); kern or kern_ENV=V,ENV2=V
       ENVS=""; LIBENV=""
