@@ -538,7 +538,9 @@ constexpr size_t square_pk_smem()
                                        sizeof(V) * (SQP_CHUNK + sqp_val_slack<V>() + 1));
 }
 
-template <class V>
+// PROBE (timing probes of the probe build only, wrong results): bit 0 = no
+// F-sum atomics, bit 1 = no u_f gathers (u_e used instead)
+template <class V, int PROBE = 0>
 __global__ void __launch_bounds__((SQT_CWARPS + 1) * 32)
 k_square_pk(int64_t c0, int64_t c1, const int4 *__restrict__ desc, const uint32_t *__restrict__ words,
             V *__restrict__ sq_val, const double *__restrict__ u, double beta, const double2 *__restrict__ gh,
@@ -615,7 +617,7 @@ k_square_pk(int64_t c0, int64_t c1, const int4 *__restrict__ desc, const uint32_
             const int r = j * (SQT_CWARPS * 32) + tid;
             if (r < n) {
                 ue[j] = __ldg(u + ef[j].x);
-                uf[j] = __ldg(u + ef[j].y);
+                uf[j] = (PROBE & 2) ? ue[j] : __ldg(u + ef[j].y);
             }
         }
 #pragma unroll
@@ -634,11 +636,11 @@ k_square_pk(int64_t c0, int64_t c1, const int4 *__restrict__ desc, const uint32_
                 const double Nef = clamp_beta(beta + v[j].y, beta);   // line 9 at p+1
                 const double Nfe = clamp_beta(beta + v[j].x, beta);
                 const unsigned long long Tfe = __double2ull_rn(Nfe * fp_scale);
-                if (Tfe) atomicAdd(tacc + ef[j].y, Tfe);
+                if (Tfe && !(PROBE & 1)) atomicAdd(tacc + ef[j].y, Tfe);
                 Tef = __double2ull_rn(Nef * fp_scale);
                 key = ef[j].x;
             }
-            seg_atomic_add(Tef, key, lane, tacc);
+            if (!(PROBE & 1)) seg_atomic_add(Tef, key, lane, tacc);
         }
     }
 }
@@ -763,7 +765,12 @@ template <class V>
 cualign_status square_pk_launch_v(cualign_bp *h, V *vals, int64_t c0, int64_t c1)
 {
     if (c1 <= c0) return CUALIGN_OK;
+#ifdef CUALIGN_PROBES
+    static const int probe = probe_knob("CUALIGN_SQ_PK_PROBE", 0); // timing probes (wrong results)
+    auto fn = probe == 1 ? k_square_pk<V, 1> : (probe == 2 ? k_square_pk<V, 2> : (probe == 3 ? k_square_pk<V, 3> : k_square_pk<V>));
+#else
     auto fn = k_square_pk<V>;
+#endif
     constexpr size_t smem = square_pk_smem<V>();
     CA_CUDA(cudaFuncSetAttribute((const void *)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int block = (SQT_CWARPS + 1) * 32;

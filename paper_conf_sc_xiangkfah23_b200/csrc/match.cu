@@ -1113,10 +1113,15 @@ cualign_status run_matching(cualign_bp *h, MatchParams &P, bool collect_in_eval 
         P.qcnt = h->qcnt;
         KScope ks(h, CUALIGN_K_MATCH);
         const int64_t qc = h->qcap, cs = (int64_t)NQ * QSTRIDE;
-        // 2 rounds: 0.112 ms for both matchings on O (p = 80) vs 0.184 / 0.129
-        // / 0.121 / 0.130 with 0 / 1 / 3 / 4 (each round costs ~9 dependent
-        // memory round trips even nearly empty; the chain form takes the rest)
-        static const int nrounds = probe_knob("CUALIGN_SUITOR_ROUNDS", 2);
+        // 3 rounds, measured in the bench's window (p = 6-25 on O): matching
+        // 0.206 / 0.165 / 0.148 / 0.158 / 0.176 ms with 1 / 2 / 3 / 4 / 6
+        // rounds (at p = 80 alone 2 rounds were best: 0.112 vs 0.121 ms; early
+        // BP iterations displace far more proposers).  Each round costs ~9
+        // dependent memory round trips even nearly empty; the chain form takes
+        // the rest.  Rejected: a persistent kernel looping over rounds with
+        // grid barriers until the queue is short (0.162 / 0.143 ms), rounds
+        // that skip once the queue is short (0.158 / 0.126 ms).
+        static const int nrounds = probe_knob("CUALIGN_SUITOR_ROUNDS", 3);
         static const int first_u = probe_knob("CUALIGN_SUITOR_FIRST_U", 6);
         if (first_u == 9)
             CA_CUDA(launch_pdl(k_propose_first<9>, dim3(grid_for(slots, 256, 1 << 30)), dim3(256), 0, h->stream, P,
