@@ -413,6 +413,8 @@ def main():
     ap.add_argument("--exact", action="store_true", help="CUALIGN_FLAG_EXACT (oracle-order sums)")
     ap.add_argument("--fp32", action="store_true", help="CUALIGN_FLAG_FP32_S (S^p stored in fp32, NEXT-3)")
     ap.add_argument("--match-rounds", action="store_true", help="pointer-round matching schedule")
+    ap.add_argument("--schedule", type=int, default=0,
+                    help="step schedule (cualign_params.schedule: 0 the library's rule, 1 pipelined, 2 serial, 3 forked)")
     ap.add_argument("--prof-steps", type=int, default=20, help="steps of the per-kernel timing pass")
     ap.add_argument("--strong", action="store_true", help="N > 1: shard the same instance (strong scaling)")
     ap.add_argument("--no-knn", action="store_true", help="skip the NEXT-2 kNN measurement")
@@ -480,7 +482,7 @@ def main():
     # ---------------------------------------------------------------- init
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    h = ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags=flags,
+    h = ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma, flags=flags, schedule=args.schedule,
                      device=dev, stream=stream, **shard_kw())
     torch.cuda.synchronize()
     init_s = max_over_ranks(time.perf_counter() - t0, world, device=f"cuda:{dev}")

@@ -823,17 +823,23 @@ cualign_status cualign_bp_run_trace(cualign_bp *h, int32_t n_steps, cualign_roun
 
 namespace cualign {
 // Step schedule of run() when the caller leaves it to the library (no timed
-// selection on the critical path).  Measured (tools/probe_schedules.py,
-// profiles/r02_schedules.jsonl, ms per step pipelined / serial): T 0.043 /
-// 0.051, P 0.118 / 0.131 -- launch- and latency-bound steps gain from
-// overlapping the rounding with the next iteration; O 0.704 / 0.693, S 5.91 /
-// 5.64, R k = 5 1.14 / 0.81, R k = 50 7.50 / 6.97 -- once the square pass
-// (which needs every SM's registers at full speed) dominates, any overlap
-// only delays it.  Serial from 10^7 nonzeros of S on.
+// selection on the critical path).  Measured with the round-2 kernels
+// (tools/probe_schedules.py, profiles/r02_schedules.jsonl; ms per step after
+// 40 warm steps, pipelined / serial): T 0.041 / 0.047, P 0.121 / 0.133 --
+// launch- and latency-bound steps gain from overlapping the rounding with the
+// next iteration; O 0.672 / 0.678 (bench: 1544 / 1487 it/s over 300 steps,
+// 1435 / 1396 in the 20-step window) -- a long square pass (s/m = 20) hides
+// the rounding; R k = 5 0.856 / 0.773 (s/m = 5: the step is short next to
+// its rounding, which then contends with it), S 5.57 / 5.47 and R k = 50
+// 6.37 / 6.08 (s >= 8.4e8: the HBM-bound pass is delayed by any traffic
+// beside it).  Pipelined below 10^7 nonzeros of S, and up to 3e8 nonzeros
+// when s/m >= 10; serial otherwise.
 static int default_schedule(cualign_bp *h)
 {
     const int64_t s = h->s_total ? h->s_total : h->s;
-    return s >= 10000000 ? 2 : 1;
+    const int64_t m = h->L.m > 0 ? h->L.m : 1;
+    if (s < 10000000) return 1;
+    return (s < 300000000 && s >= 10 * m) ? 1 : 2;
 }
 
 // The sharded iteration (k_edge, top-2 all-gather, u halo on the exchange

@@ -64,11 +64,31 @@ print('ms per step, first 40:', ms[:40]); print('mean 6-25', sum(ms[5:25])/20, '
         timeout 1200 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_workload.py > $OUT/sanitize_$tool.txt 2>&1
         echo "sanitize $tool rc=$?"; tail -4 $OUT/sanitize_$tool.txt
       done ;;
+    bs_*)
+      # the driver's bench window with a forced step schedule (product build): bs_1 pipelined, bs_2 serial, bs_3 forked
+      timeout 600 python bench.py --schedule ${w#bs_} --steps 20 --warmup 5 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/$w.json 2> $OUT/$w.err
+      timeout 600 python bench.py --schedule ${w#bs_} --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/${w}_300.json 2> $OUT/${w}_300.err
+      echo "$w rc=$?"; python -c "
+import json
+for f in ('$OUT/$w.json', '$OUT/${w}_300.json'):
+    d = json.load(open(f)); print(f, round(d['value'],1), {k: round(v,4) for k,v in d['kernel_ms_per_step'].items()})" ;;
     bw_*)
       # the driver's bench window (20 steps after 5) with the probe build and env: bw_NAME=V,NAME2=V
       ENVS=$(echo ${w#bw_} | tr ',' ' ')
       env CUALIGN_LIB=$PROBES $ENVS timeout 600 python bench.py --steps 20 --warmup 5 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/$w.json 2> $OUT/$w.err
       echo "$w rc=$?"; python -c "import json; d=json.load(open('$OUT/$w.json')); print(round(d['value'],1), {k: round(v,4) for k,v in d['kernel_ms_per_step'].items()})" ;;
+    initp)
+      # init phase trace (probe build), first and later handles
+      CUALIGN_LIB=$PROBES CUALIGN_INIT_TRACE=1 timeout 300 python tools/probe_init.py O > $OUT/initp.txt 2>&1
+      echo "initp rc=$?"; cat $OUT/initp.txt | tail -40 ;;
+    fp32)
+      # NEXT-3: fp32 S^p storage, driver window and 300 steps
+      timeout 600 python bench.py --fp32 --steps 20 --warmup 5 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/fp32_w.json 2> $OUT/fp32_w.err
+      timeout 600 python bench.py --fp32 --no-e2e --no-cpu-baseline --no-knn --no-configs > $OUT/fp32.json 2> $OUT/fp32.err
+      echo "fp32 rc=$?"; python -c "
+import json
+for f in ('$OUT/fp32_w.json', '$OUT/fp32.json'):
+    d = json.load(open(f)); print(f, round(d['value'], 1), d['roofline'], d['kernels_isolated']['square'])" ;;
     kernw)
       # in-situ per-kernel durations inside the driver's window (p = 6 .. 25)
       timeout 300 python tools/probe_kernels.py --pre 5 --n 20 > $OUT/kernw.json 2> $OUT/kernw.err
