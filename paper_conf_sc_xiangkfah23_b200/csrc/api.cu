@@ -201,14 +201,16 @@ static constexpr int SERIAL_SLOT = 10; // one step as ONE graph: iterate(1), the
 // selected by pointing h->yc / h->zc at them while the kernels are captured.
 static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
 {
-    // k_top2 one lane per tile here: 4x fewer threads than the 4-lane form
-    // (0.089 vs 0.065 ms alone) leave SM slots to the rounding beside it --
-    // O: 1446 vs 1394 it/s pipelined (serial: 1352 vs 1389, so 2 lanes there)
+    // k_top2 lanes per tile in the pipelined graphs.  Round 1 (the rounding
+    // then ran ~0.23 ms beside it) took 1 lane: 4x fewer threads left SM
+    // slots to the rounding.  Round 2 (packed square stream, 3 proposal
+    // rounds) measured the bench window on O: 1 lane 1421-1440 it/s, 2 lanes
+    // 1449-1469, 4 lanes 1465 -- 2 lanes, as in the serial graph.
     struct TgScope {
         cualign_bp *h;
         ~TgScope() { h->top2_tg = 0; h->sq_ctas = 0; }
     } tg_scope{h};
-    h->top2_tg = probe_knob("CUALIGN_PIPE_TOP2_TG", 1);
+    h->top2_tg = probe_knob("CUALIGN_PIPE_TOP2_TG", 2);
     // the square pass leaves SM room to the rounding running beside it
     static const int pipe_sq = probe_knob("CUALIGN_PIPE_SQ_CTAS", 0);
     h->sq_ctas = pipe_sq;
