@@ -1094,35 +1094,101 @@ cualign_status tile_squares(cualign_bp *h)
 // f lies in one 2^SQP_FBITS block (fb = its start) and every e in
 // [eb, eb + 2^SQP_EBITS) with eb = the chunk's first e; square q then packs
 // into one 32-bit word (e - eb) << SQP_FBITS | (f - fb), half of the int2.
-// Windows of SQP_CHUNK squares (also cut at nsq_split) are split greedily by
-// one thread each: pass 1 counts the chunks per window, pass 2 writes them.
+// Windows of SQP_CHUNK squares are split by one warp each: "hard" cuts (window
+// start, nsq_split, a new f block, e decreasing -- a new tile) come from
+// ballots over the window, and inside each hard segment (e non-decreasing)
+// the greedy e-range cuts are found by binary search on e from each chunk
+// start.  Pass 1 counts the chunks per window, pass 2 writes descriptors and
+// words.
+constexpr int SQP_PACK_WARPS = 4;
 template <bool FILL>
-__global__ void k_sqp_pack(int64_t nsq, int64_t split, const int2 *__restrict__ sq_ef,
-                           int64_t *__restrict__ wcnt, int4 *__restrict__ desc, uint32_t *__restrict__ words)
+__global__ void __launch_bounds__(SQP_PACK_WARPS * 32)
+k_sqp_pack(int64_t nsq, int64_t split, const int2 *__restrict__ sq_ef, int64_t *__restrict__ wcnt,
+           int4 *__restrict__ desc, uint32_t *__restrict__ words)
 {
+    constexpr int NB = SQP_CHUNK / 32;
+    constexpr int64_t ELIM = 1ll << SQP_EBITS;
+    __shared__ int s_start[SQP_PACK_WARPS][SQP_CHUNK + 1];
+    const int lane = threadIdx.x & 31;
+    int *starts = s_start[threadIdx.x >> 5];
     const int64_t nwin = (nsq + SQP_CHUNK - 1) / SQP_CHUNK;
-    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nwin;
-         w += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t q0 = w * SQP_CHUNK, q1 = (q0 + SQP_CHUNK < nsq) ? q0 + SQP_CHUNK : nsq;
-        int64_t c = FILL ? (w ? wcnt[w - 1] : 0) : 0; // wcnt: inclusive prefix after pass 1
-        int64_t cs = q0;
-        int eb = 0, fb = 0;
-        for (int64_t q = q0; q < q1; q++) {
-            const int2 ef = sq_ef[q];
-            const int fblk = (int)(((uint32_t)ef.y >> SQP_FBITS) << SQP_FBITS);
-            const bool cut = q == q0 || q == split || fblk != fb || ef.x < eb ||
-                             (int64_t)ef.x - eb >= (1ll << SQP_EBITS);
-            if (cut) {
-                if (FILL && q > q0) desc[c] = make_int4((int)cs, (int)(q - cs), eb, fb);
-                if (q > q0) c++;
-                cs = q;
-                eb = ef.x;
-                fb = fblk;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < nwin; w += nwarps) {
+        const int64_t q0 = w * SQP_CHUNK;
+        const int len = (int)((q0 + SQP_CHUNK < nsq) ? SQP_CHUNK : nsq - q0);
+        const int2 *__restrict__ W = sq_ef + q0;
+        unsigned hm[NB];
+#pragma unroll
+        for (int k = 0; k < NB; k++) {
+            const int r = lane + 32 * k;
+            bool cut = false;
+            if (r < len) {
+                if (r == 0 || q0 + r == split) {
+                    cut = true;
+                } else {
+                    const int2 ef = W[r], pv = W[r - 1];
+                    cut = ((uint32_t)ef.y >> SQP_FBITS) != ((uint32_t)pv.y >> SQP_FBITS) || ef.x < pv.x;
+                }
             }
-            if (FILL) words[q] = ((uint32_t)(ef.x - eb) << SQP_FBITS) | (uint32_t)(ef.y - fb);
+            hm[k] = __ballot_sync(FULL_MASK, cut);
         }
-        if (FILL) desc[c] = make_int4((int)cs, (int)(q1 - cs), eb, fb);
-        else wcnt[w] = c + 1;
+        int nc = 0;
+        if (lane == 0) {
+            int r = 0;
+            while (r < len) {
+                // next hard cut after r
+                int nh = len;
+                for (int x = r + 1; x < len;) {
+                    const unsigned m = hm[x >> 5] >> (x & 31);
+                    if (m) {
+                        nh = x + __ffs(m) - 1;
+                        break;
+                    }
+                    x = (x | 31) + 1;
+                }
+                for (int c = r; c < nh;) {
+                    starts[nc++] = c;
+                    const int eb = W[c].x;
+                    int lo = c + 1, hi = nh; // first index with e - eb >= ELIM
+                    while (lo < hi) {
+                        const int mid = (lo + hi) >> 1;
+                        if ((int64_t)W[mid].x - eb >= ELIM) hi = mid;
+                        else lo = mid + 1;
+                    }
+                    c = lo;
+                }
+                r = nh;
+            }
+            starts[nc] = len;
+        }
+        nc = __shfl_sync(FULL_MASK, nc, 0);
+        __syncwarp();
+        if (!FILL) {
+            if (lane == 0) wcnt[w] = nc;
+            __syncwarp();
+            continue;
+        }
+        const int64_t cbase = w ? wcnt[w - 1] : 0; // wcnt: inclusive prefix after pass 1
+        for (int c = lane; c < nc; c += 32) {
+            const int2 e0 = W[starts[c]];
+            desc[cbase + c] = make_int4((int)(q0 + starts[c]), starts[c + 1] - starts[c], e0.x,
+                                        (int)(((uint32_t)e0.y >> SQP_FBITS) << SQP_FBITS));
+        }
+#pragma unroll 4
+        for (int k = 0; k < NB; k++) {
+            const int r = lane + 32 * k;
+            if (r >= len) break;
+            int lo = 0, hi = nc - 1; // chunk c with starts[c] <= r < starts[c + 1]
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (starts[mid] <= r) lo = mid;
+                else hi = mid - 1;
+            }
+            const int2 e0 = W[starts[lo]], ef = W[r];
+            const int fb = (int)(((uint32_t)e0.y >> SQP_FBITS) << SQP_FBITS);
+            words[q0 + r] = ((uint32_t)(ef.x - e0.x) << SQP_FBITS) | (uint32_t)(ef.y - fb);
+        }
+        __syncwarp();
     }
 }
 
@@ -1154,8 +1220,8 @@ cualign_status pack_squares(cualign_bp *h)
     CA_CUDA(tmalloc(h, res, sizeof(int64_t)));
     int64_t *wc = (int64_t *)cnt.p;
     KScope ks(h, CUALIGN_K_INIT);
-    const int grid = grid_for(nwin, 128, h->num_sms * 16);
-    k_sqp_pack<false><<<grid, 128, 0, h->stream>>>(n, h->nsq_split, h->sq_ef, wc, nullptr, nullptr);
+    const int grid = grid_for(nwin * 32, SQP_PACK_WARPS * 32, h->num_sms * 16);
+    k_sqp_pack<false><<<grid, SQP_PACK_WARPS * 32, 0, h->stream>>>(n, h->nsq_split, h->sq_ef, wc, nullptr, nullptr);
     CA_CUDA(cudaGetLastError());
     size_t tb = 0;
     CA_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, wc, wc, (int)nwin, h->stream));
@@ -1170,7 +1236,7 @@ cualign_status pack_squares(cualign_bp *h)
     CA_TRY(dalloc(h, &h->sqp_w, (size_t)n + 8)); // +8: 16-byte bulk-copy tails
     CA_TRY(dalloc(h, &h->sqp_desc, (size_t)nch));
     CA_CUDA(cudaMemsetAsync(h->sqp_w + n, 0, 8 * sizeof(uint32_t), h->stream));
-    k_sqp_pack<true><<<grid, 128, 0, h->stream>>>(n, h->nsq_split, h->sq_ef, wc, h->sqp_desc, h->sqp_w);
+    k_sqp_pack<true><<<grid, SQP_PACK_WARPS * 32, 0, h->stream>>>(n, h->nsq_split, h->sq_ef, wc, h->sqp_desc, h->sqp_w);
     CA_CUDA(cudaGetLastError());
     int64_t sc = 0;
     if (h->nsq_split > 0) {
