@@ -450,7 +450,7 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
         KScope ks(h, CUALIGN_K_OTHER);
         const uint8_t *a8 = (const uint8_t *)Asw, *b8 = (const uint8_t *)Bsw;
         cualign_status lst;
-        static const int cpl = probe_knob("CUALIGN_KNN_CPL", 2);
+        static const int cpl = probe_knob("CUALIGN_KNN_CPL", 1); // measured: CPL 1 / 2 / 4 = 4.15 / 4.44 / 6.41 ms at 65536^2
         if (BN == 256 && EH == 2) lst = knn_launch<256, 2>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
         else if (BN == 256 && cpl == 4) lst = knn_launch<256, 1, 4>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);
         else if (BN == 256 && cpl == 2) lst = knn_launch<256, 1, 2>(h, a8, b8, n_a, n_b, KB, k, pv, pi, nsplit, tps, nstages, smem);

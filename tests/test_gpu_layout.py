@@ -55,6 +55,26 @@ def test_square_tiles_bitwise_invariant(ca):
         assert np.array_equal(base[k], default[k]), k
 
 
+def test_packed_square_chunks_across_f_blocks(ca):
+    """m > 2^21 edges: the packed square stream cuts its chunks at 2^21-edge
+    f blocks (and falls back to the int2 stream when an untiled order would
+    make them tiny); every layout gives the same bits (DESIGN.md §5 "Packed
+    square indices")."""
+    inst = make_config("R", scale=0.5, k=5)
+    assert inst.L.m > (1 << 21)
+    outs = []
+    for tile_log in (-1, 0, 12):
+        with ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma,
+                          square_tile_log=tile_log) as h:
+            h.run(4)
+            st = h.get_state(with_S=False)
+            outs.append({k: np.asarray(st[k]).view(np.uint64) for k in ("yc", "zc", "yp", "zp", "d")})
+            outs[-1]["best"] = np.asarray([h.get_best()[1]["best_score"]])
+    for o in outs[1:]:
+        for k in outs[0]:
+            assert np.array_equal(outs[0][k], o[k]), k
+
+
 def _eager(ca, inst, n):
     h = ca.CuAlignBP(inst.A, inst.B, inst.L, inst.alpha, inst.beta, inst.gamma)
     infos = []
