@@ -89,6 +89,11 @@ for f in ('$OUT/$w.json', '$OUT/${w}_300.json'):
 import json
 for f in ('$OUT/fp32_w.json', '$OUT/fp32.json'):
     d = json.load(open(f)); print(f, round(d['value'], 1), d['roofline'], d['kernels_isolated']['square'])" ;;
+    timeline)
+      timeout 300 python tools/probe_timeline.py --pre 10 --n 3 > $OUT/timeline.json 2> $OUT/timeline.err
+      echo "timeline rc=$?"; python -c "
+import json; d=json.load(open('$OUT/timeline.json'))
+for k in d['kernels']: print(k['t0_us'], k['t1_us'], k['dur_us'], k['stream'], k['kernel'])" ;;
     kernw)
       # in-situ per-kernel durations inside the driver's window (p = 6 .. 25)
       timeout 300 python tools/probe_kernels.py --pre 5 --n 20 > $OUT/kernw.json 2> $OUT/kernw.err
