@@ -195,7 +195,7 @@ __global__ void k_copy_int(int *dst, const int *src) { *dst = *src; }
 __global__ void k_incr_int(int *x) { *x += 1; }
 
 static inline int pslot(int kind, int wb) { return 4 + 2 * kind + wb; }
-static constexpr int SERIAL_SLOT = 10; // one step as ONE graph: iterate(1), then the rounding (no fork)
+static constexpr int SERIAL_SLOT = 14; // one step as ONE graph: iterate(1), then the rounding (no fork)
 
 // The pipelined graphs' work (see capture_step): the y^c / z^c buffers are
 // selected by pointing h->yc / h->zc at them while the kernels are captured.
@@ -208,13 +208,14 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
     // 1449-1469, 4 lanes 1465 -- 2 lanes, as in the serial graph.
     struct TgScope {
         cualign_bp *h;
-        ~TgScope() { h->top2_tg = 0; h->sq_ctas = 0; }
+        ~TgScope() { h->top2_tg = 0; h->sq_ctas = 0; h->probe_no_eval = false; }
     } tg_scope{h};
     h->top2_tg = probe_knob("CUALIGN_PIPE_TOP2_TG", 2);
     // the square pass leaves SM room to the rounding running beside it
     static const int pipe_sq = probe_knob("CUALIGN_PIPE_SQ_CTAS", 0);
     h->sq_ctas = pipe_sq;
     h->pipe_join_front = probe_knob("CUALIGN_PIPE_JOIN_FRONT", 0) != 0;
+    h->probe_no_eval = probe_knob("CUALIGN_PIPE_NO_EVAL", 0) != 0;
     double *yc0 = h->yc, *zc0 = h->zc;
     double *yb[2] = {yc0, h->yc_b1}, *zb[2] = {zc0, h->zc_b1};
     cualign_status st = CUALIGN_OK;
@@ -242,6 +243,72 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
         h->yc = yb[wb];
         h->zc = zb[wb];
         if (st == CUALIGN_OK) st = bp_iterate(h, 1);
+    } else if (h->defer_eval && kind != 0) {
+        // deferred evaluate: a round's
+        // matching beside the next iteration, its evaluate one graph later
+        // beside the iteration after that; the matching's collect pass waits
+        // for the previous round's evaluate.  The proposal counters and y^c /
+        // z^c of a round use set = buffer = wb of the iteration it rounds.
+        //   kind 1: iteration p || match(p-1)                     (p = 2)
+        //   kind 3: iteration p || match(p-1) || eval(p-2)        (p >= 3)
+        //   kind 4: eval(n-1)                                     (drain, n >= 2)
+        //   kind 2: match(n), eval(n)                             (drain)
+        auto eval_of = [&](int set) -> cualign_status {
+            {
+                KScope ks(h, CUALIGN_K_OTHER);
+                k_incr_int<<<1, 1, 0, h->stream>>>(h->rp_dev);
+                CA_CUDA(cudaGetLastError());
+            }
+            h->round_p = h->rp_dev;
+            cualign_status r = eval_round_deferred(h, set);
+            h->round_p = nullptr;
+            return r;
+        };
+        auto match_of = [&](int buf, cudaEvent_t ev) -> cualign_status {
+            h->yc = yb[buf];
+            h->zc = zb[buf];
+            return match_round_deferred(h, buf, ev);
+        };
+        if (kind == 2) {
+            st = match_of(wb, nullptr);
+            if (st == CUALIGN_OK) st = eval_of(wb);
+        } else if (kind == 4) {
+            st = eval_of(wb);
+        } else {
+            const bool with_eval = kind == 3;
+            // the evaluate runs on the iteration's stream ahead of its k_edge,
+            // beside the matching's first proposals (bench window on O: 1506-
+            // 1511 it/s; on a third stream beside k_edge: 1492-1494; evaluate
+            // in the round's own graph: 1469).  Probe build:
+            // CUALIGN_PIPE_EVAL_MAIN=0 takes the third stream.
+            static const bool eval_main = probe_knob("CUALIGN_PIPE_EVAL_MAIN", 1) != 0;
+            cudaStream_t es = eval_main ? h->gstream : h->gstream3;
+            if (cudaEventRecord(h->fork_ev[0], h->gstream) != cudaSuccess ||
+                cudaStreamWaitEvent(h->gstream2, h->fork_ev[0], 0) != cudaSuccess ||
+                (with_eval && !eval_main && cudaStreamWaitEvent(h->gstream3, h->fork_ev[0], 0) != cudaSuccess))
+                st = CUALIGN_ECUDA;
+            if (st == CUALIGN_OK && with_eval) {
+                h->stream = es;
+                st = eval_of(wb); // round p-2 read buffer wb
+                if (st == CUALIGN_OK && cudaEventRecord(h->eval_ev, es) != cudaSuccess) st = CUALIGN_ECUDA;
+                h->stream = h->gstream;
+            }
+            if (st == CUALIGN_OK) {
+                h->stream = h->gstream2;
+                st = match_of(1 - wb, with_eval ? h->eval_ev : nullptr);
+                h->stream = h->gstream;
+            }
+            h->yc = yb[wb];
+            h->zc = zb[wb];
+            if (st == CUALIGN_OK) st = bp_iterate(h, 1);
+            if (st == CUALIGN_OK && (cudaEventRecord(h->fork_ev[1], h->gstream2) != cudaSuccess ||
+                                     cudaStreamWaitEvent(h->gstream, h->fork_ev[1], 0) != cudaSuccess))
+                st = CUALIGN_ECUDA;
+            if (st == CUALIGN_OK && with_eval && !eval_main &&
+                (cudaEventRecord(h->join3_ev, h->gstream3) != cudaSuccess ||
+                 cudaStreamWaitEvent(h->gstream, h->join3_ev, 0) != cudaSuccess))
+                st = CUALIGN_ECUDA;
+        }
     } else if (kind == 1) {
         // fork: the rounding of iteration p-1 (buffer 1-wb) beside all of
         // iteration p (writes buffer wb); the rounding reads only y^c, z^c of
@@ -442,14 +509,21 @@ static cualign_status run_pipelined(cualign_bp *h, int32_t n, RoundDev *trace = 
     if (!h->yc_b1) CA_TRY(alloc_pipeline(h));
     CA_CUDA(cudaEventRecord(h->sync_ev[0], h->stream));
     CA_CUDA(cudaStreamWaitEvent(h->gstream, h->sync_ev[0], 0));
+    const bool dfr = h->defer_eval;
     for (int32_t k = 1; k <= n; k++) {
         const int wb = (n - k) & 1;
-        CA_TRY(launch_slot(h, pslot(k == 1 ? 0 : 1, wb)));
+        CA_TRY(launch_slot(h, pslot(k == 1 ? 0 : ((dfr && k >= 3) ? 3 : 1), wb)));
         h->p += 1;
-        // the rounding of iteration k-1 finished inside this graph: its
-        // result to the host, stream-ordered before the next graph rewrites it
-        if (trace && k >= 2)
-            CA_CUDA(cudaMemcpyAsync(trace + (k - 2), h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->gstream));
+        // the rounding (deferred: the evaluate) of iteration k-1 (k-2)
+        // finished inside this graph: its result to the host, stream-ordered
+        // before the next graph rewrites it
+        const int r = dfr ? k - 3 : k - 2;
+        if (trace && r >= 0)
+            CA_CUDA(cudaMemcpyAsync(trace + r, h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->gstream));
+    }
+    if (dfr && n >= 2) {
+        CA_TRY(launch_slot(h, pslot(4, 1))); // evaluate of round n-1 (it read buffer 1)
+        if (trace) CA_CUDA(cudaMemcpyAsync(trace + (n - 2), h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->gstream));
     }
     CA_TRY(launch_slot(h, pslot(2, 0)));
     if (trace) CA_CUDA(cudaMemcpyAsync(trace + (n - 1), h->rd, sizeof(RoundDev), cudaMemcpyDeviceToHost, h->gstream));
@@ -558,6 +632,9 @@ static cualign_status open_handle(const cualign_params *params, cualign_bp **out
         // the iteration, 2 = lowest
         static const int rp = probe_knob("CUALIGN_ROUND_PRIO", 0);
         CA_CUDA(cudaStreamCreateWithPriority(&h->gstream2, cudaStreamNonBlocking, rp == 1 ? 0 : rp == 2 ? lo : hi));
+        CA_CUDA(cudaStreamCreateWithPriority(&h->gstream3, cudaStreamNonBlocking, rp == 1 ? 0 : rp == 2 ? lo : hi));
+        CA_CUDA(cudaEventCreateWithFlags(&h->eval_ev, cudaEventDisableTiming));
+        CA_CUDA(cudaEventCreateWithFlags(&h->join3_ev, cudaEventDisableTiming));
     }
     for (int i = 0; i < 2; i++) {
         CA_CUDA(cudaEventCreateWithFlags(&h->sync_ev[i], cudaEventDisableTiming));
@@ -587,6 +664,9 @@ static void close_handle(cualign_bp *h)
     if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
     if (h->gstream) cudaStreamDestroy(h->gstream);
     if (h->gstream2) cudaStreamDestroy(h->gstream2);
+    if (h->gstream3) cudaStreamDestroy(h->gstream3);
+    if (h->eval_ev) cudaEventDestroy(h->eval_ev);
+    if (h->join3_ev) cudaEventDestroy(h->join3_ev);
     (void)cudaGetLastError();
     delete h;
 }
@@ -654,7 +734,10 @@ static cualign_status precapture_step_graphs(cualign_bp *h)
     CA_TRY(ensure_gh(h, (int64_t)h->p + 2));
     std::vector<int> slots;
     if (mode == 2) slots = {SERIAL_SLOT};
-    else if (mode == 1) slots = {pslot(0, 0), pslot(0, 1), pslot(1, 0), pslot(1, 1), pslot(2, 0)};
+    else if (mode == 1) {
+        slots = {pslot(0, 0), pslot(0, 1), pslot(1, 0), pslot(1, 1), pslot(2, 0)};
+        if (h->defer_eval) slots.insert(slots.end(), {pslot(3, 0), pslot(3, 1), pslot(4, 1)});
+    }
     else slots = {CUALIGN_RUN_ITERATE | CUALIGN_RUN_ROUND};
     for (int sl : slots) {
         if (!h->graph[0][sl]) CA_TRY(capture_step(h, 0, sl));
@@ -734,6 +817,9 @@ cualign_status cualign_bp_init(const cualign_graph *A, const cualign_graph *B, c
         if (st == CUALIGN_OK) st = h->world > 1 ? shard_fsum(h) : bp_fsum(h); // F(S^p = 0) sums for iteration 1
         if (st == CUALIGN_OK && h->world == 1) st = bp_top2(h);                 // othermax inputs of iteration 1
         init_trace(h, "fsum");
+        // pipelined graphs evaluate each round one step later (probe build:
+        // CUALIGN_PIPE_DEFER_EVAL=0 keeps evaluate in the round's own graph)
+        if (st == CUALIGN_OK) h->defer_eval = can_defer_eval(h) && probe_knob("CUALIGN_PIPE_DEFER_EVAL", 1) != 0;
         if (st == CUALIGN_OK && h->world == 1) st = precapture_step_graphs(h);
         init_trace(h, "step graphs");
     }

@@ -173,6 +173,10 @@ struct cualign_bp {
     // CUDA graphs of one step (iterate(1) [+ round]); [0] = no round, [1] = with round
     cudaStream_t gstream = nullptr;     // capture / replay stream (never the legacy stream)
     cudaStream_t gstream2 = nullptr;    // capture side branch: rounding overlapped with the square pass
+    cudaStream_t gstream3 = nullptr;    // capture side branch: deferred evaluate
+    cudaEvent_t eval_ev = nullptr;      // deferred evaluate done (the next collect waits for it)
+    cudaEvent_t join3_ev = nullptr;     // gstream3 joins the graph's main stream
+    bool defer_eval = false;            // pipelined graphs evaluate round k one step later
     cudaEvent_t sync_ev[2] = {nullptr, nullptr};
     cudaEvent_t fork_ev[2] = {nullptr, nullptr};
     bool capturing = false;
@@ -181,7 +185,7 @@ struct cualign_bp {
     // the pipelined step graphs: kind 0 = iterate
     // into buffer wb, 1 = rounding of buffer 1-wb beside iterate into wb,
     // 2 = rounding of buffer wb
-    static constexpr int NSLOT = 11;  // + SERIAL_SLOT: iterate(1) then round, no fork
+    static constexpr int NSLOT = 15;  // pipelined kinds 0-4 x 2 buffers (4..13) + SERIAL_SLOT (14)
     cudaGraphExec_t graph[2][NSLOT] = {};                   // [timed][slot]
     cudaGraphExec_t shard_graph = nullptr;                  // sharded: one iteration (all exchanges) as a graph
     struct StepCounts {
@@ -203,6 +207,7 @@ struct cualign_bp {
     int top2_tg = 0;                    // k_top2 lanes per tile while capturing (0: default; pipelined graphs: 1)
     int sq_ctas = 0;                    // square-pass CTAs per SM while capturing (0: as many as fit)
     bool pipe_join_front = false;       // pipelined graphs: rounding joins before the square pass
+    bool probe_no_eval = false;         // probe build timing probe: pipelined rounding without evaluate
     int *rp_dev = nullptr;
     const int *round_p = nullptr;
 
@@ -406,6 +411,9 @@ cualign_status knn_build(cualign_bp *h, const float *YA, int32_t n_a, const floa
                          int32_t k, int32_t *La, int32_t *Lb, double *Lw); // NEXT-2 (knn.cu)
 cualign_status match_setup(cualign_bp *h);
 cualign_status match_round(cualign_bp *h);  // a7 + a8 on the device
+cualign_status match_round_deferred(cualign_bp *h, int set, cudaEvent_t before_collect); // a7 (pipelined)
+cualign_status eval_round_deferred(cualign_bp *h, int set);                              // a8, one step later
+bool can_defer_eval(const cualign_bp *h);
 cualign_status match_evaluate(cualign_bp *h); // a8 on the round's mate slot (collect done)
 // sharded rounding (NEXT-1), driven by shard_round: begin, then rounds of
 // local -> all-reduce MAX(dist_wxg) -> cand -> all-reduce MIN(dist_wid) ->

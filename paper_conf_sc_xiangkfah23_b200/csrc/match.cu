@@ -63,6 +63,10 @@ struct MatchParams {
     const unsigned long long *gx;
     const int32_t *gi;
     const int32_t *act; // active flag per (instance, local proposer)
+    // deferred evaluate (pipelined graphs): exhausted proposers write nothing;
+    // k_defer_fill presets this round's mate slot and mvA to -1 just before
+    // k_collect, after the previous round's evaluate chose the slot
+    int defer;
 };
 
 constexpr int WORK_SPREAD = 64, WORK_STRIDE = 16; // counter slots, 128 B apart
@@ -211,7 +215,7 @@ __device__ __forceinline__ void suitor_chain(const MatchParams &P, Tile &tile, i
             // exhausted: `cur` stays unmatched (nobody proposes to a
             // proposer), so this is its only mate write this round -- the
             // matched ones are written from the target slots by k_collect
-            if (!DIST && lane == 0) {
+            if (!DIST && lane == 0 && !P.defer) {
                 if (fromB) {
                     P.mateB[k * nP + cur] = -1;
                 } else {
@@ -395,8 +399,10 @@ __device__ __forceinline__ int propose_once(const MatchParams &P, int64_t nP, in
         }
     }
     if (best < 0) {
-        slot_mates(P)[k * nP + cur] = -1; // exhausted (see suitor_chain)
-        set_mv(P.mvA, cur, k, -1);
+        if (!P.defer) {
+            slot_mates(P)[k * nP + cur] = -1; // exhausted (see suitor_chain)
+            set_mv(P.mvA, cur, k, -1);
+        }
         return -1;
     }
     unsigned long long *sp = sT + bt;
@@ -664,6 +670,19 @@ __device__ __forceinline__ void collect_body(const MatchParams &P, int64_t nT, i
             set_mv(P.mvA, t, k, e >= 0 ? __ldg(P.Lb + e) : -1);
             if (e >= 0) P.mateB[k * nP + __ldg(P.Lb + e)] = e;
         }
+    }
+}
+
+// deferred evaluate: this round's mate slot (both instances) and mvA to -1
+// (the collect pass then writes the matched entries)
+__global__ void k_defer_fill(MatchParams P)
+{
+    pdl_wait();
+    int32_t *mateA = slot_mates(P);
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.nA; i += (int64_t)gridDim.x * blockDim.x) {
+        mateA[i] = -1;
+        mateA[P.nA + i] = -1;
+        P.mvA[i] = make_int2(-1, -1);
     }
 }
 
@@ -1219,7 +1238,7 @@ cualign_status match_setup(cualign_bp *h)
     CA_TRY(dalloc(h, &h->mvA, nA + 1));
     CA_TRY(dalloc(h, &h->mateB, 2 * nB + 1));
     CA_TRY(dalloc(h, &h->rd, 1));
-    CA_TRY(dalloc(h, &h->match_work, WORK_SPREAD * WORK_STRIDE));
+    CA_TRY(dalloc(h, &h->match_work, 2 * WORK_SPREAD * WORK_STRIDE)); // 2 sets: deferred evaluate
     {
         RoundDev r0;
         memset(&r0, 0, sizeof(r0));
@@ -1230,7 +1249,7 @@ cualign_status match_setup(cualign_bp *h)
     CA_CUDA(cudaMemsetAsync(h->suit, 0, sizeof(unsigned long long) * (2 * nmax + 1), h->stream));
     CA_CUDA(cudaMemsetAsync(h->mates, 0xff, sizeof(int32_t) * (4 * nA + 1), h->stream));
     CA_CUDA(cudaMemsetAsync(h->mateB, 0xff, sizeof(int32_t) * (2 * nB + 1), h->stream));
-    CA_CUDA(cudaMemsetAsync(h->match_work, 0, sizeof(unsigned long long) * WORK_SPREAD * WORK_STRIDE, h->stream));
+    CA_CUDA(cudaMemsetAsync(h->match_work, 0, sizeof(unsigned long long) * 2 * WORK_SPREAD * WORK_STRIDE, h->stream));
     {
         KScope ks(h, CUALIGN_K_INIT);
         unsigned long long md[2] = {0, 0};
@@ -1294,6 +1313,67 @@ static cualign_status evaluate_impl(cualign_bp *h, const MatchParams *Pc);
 
 cualign_status match_evaluate(cualign_bp *h) { return evaluate_impl(h, nullptr); }
 
+// Deferred-evaluate rounding (pipelined graphs, DESIGN.md "Step graph and
+// schedule"): the matching of this round with proposal counters in `set`;
+// the collect pass waits for `before_collect` (the previous round's
+// evaluate, which picks this round's mate slot and reads mvA), presets the
+// slot and mvA, then writes the matched entries and resets the target slots.
+cualign_status match_round_deferred(cualign_bp *h, int set, cudaEvent_t before_collect)
+{
+    MatchParams P = base_params(h);
+    P.ninst = 2;
+    P.x0 = h->yc;
+    P.x1 = h->zc;
+    P.defer = 1;
+    P.work = h->match_work + (int64_t)set * WORK_SPREAD * WORK_STRIDE;
+    CA_TRY(run_matching(h, P, true)); // proposals only: the collect pass follows here
+    if (before_collect) CA_CUDA(cudaStreamWaitEvent(h->stream, before_collect, 0));
+    KScope ks(h, CUALIGN_K_MATCHAUX);
+    const bool fromB = P.propose_from_b != 0;
+    const int64_t nT = fromB ? h->L.nA : h->L.nB, nP = fromB ? h->L.nB : h->L.nA;
+    k_defer_fill<<<grid_for(h->L.nA > 0 ? h->L.nA : 1, 256, h->num_sms * 8), 256, 0, h->stream>>>(P);
+    CA_CUDA(cudaGetLastError());
+    CA_CUDA(launch_pdl(k_collect, dim3(grid_for(P.ninst * nT > 0 ? P.ninst * nT : 1, 256, h->num_sms * 8)),
+                       dim3(256), 0, h->stream, P, nT, nP, fromB ? 1 : 0));
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
+// Its evaluate (one step later): k_eval without the collect pass, over the
+// same block partition as k_eval<true> (evalc_grid), so the weights carry the
+// same bits as in the other schedules; proposal counters of `set`.
+cualign_status eval_round_deferred(cualign_bp *h, int set)
+{
+    EvalParams E{};
+    E.nA = h->L.nA;
+    E.Lb = h->L.Lb;
+    E.w = h->L.w;
+    E.mates = h->mates;
+    E.wslot = &h->rd->wslot;
+    E.mvA = h->mvA;
+    E.Bhash = h->Bhash;
+    E.Bhash_log = h->Bhash_log;
+    E.pairs = h->Apairs;
+    E.npairs = h->nApairs;
+    E.partial_w = h->partial_w;
+    E.rd = h->rd;
+    KScope ks(h, CUALIGN_K_EVAL);
+    const int exact = (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0;
+    const int *pd = (const int *)(h->round_p ? h->round_p : h->p_dev);
+    CA_CUDA(launch_pdl(k_eval<false>, dim3(h->evalc_grid), dim3(256), 0, h->stream, E, exact, h->alpha, h->beta, pd,
+                       h->match_work + (int64_t)set * WORK_SPREAD * WORK_STRIDE, MatchParams{}, (int64_t)0,
+                       (int64_t)0, 0));
+    CA_CUDA(cudaGetLastError());
+    return CUALIGN_OK;
+}
+
+// whether this handle's rounding can run deferred (Suitor proposal rounds)
+bool can_defer_eval(const cualign_bp *h)
+{
+    return !h->propose_from_b && h->max_deg_a <= SUITOR_ROUNDS_MAXDEG && h->squeue &&
+           !(h->flags & (CUALIGN_FLAG_ROUND_DAMPED | CUALIGN_FLAG_MATCH_ROUNDS)) && h->world == 1;
+}
+
 cualign_status match_round(cualign_bp *h)
 {
     MatchParams P = base_params(h);
@@ -1305,6 +1385,10 @@ cualign_status match_round(cualign_bp *h)
         CA_TRY(run_matching(h, P));
         CA_TRY(prep_eval_from_mates(h));
         return match_evaluate(h);
+    }
+    if (h->probe_no_eval) { // timing probe (probe build): collect only, no evaluate (wrong round info)
+        CA_TRY(run_matching(h, P, false));
+        return CUALIGN_OK;
     }
     CA_TRY(run_matching(h, P, true));
     return evaluate_impl(h, &P);
