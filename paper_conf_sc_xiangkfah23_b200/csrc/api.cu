@@ -922,8 +922,17 @@ namespace cualign {
 // 6.37 / 6.08 (s >= 8.4e8: the HBM-bound pass is delayed by any traffic
 // beside it).  Pipelined below 10^7 nonzeros of S, and up to 3e8 nonzeros
 // when s/m >= 10; serial otherwise.
+// With the deferred evaluate (the pipelined graphs evaluate each round one
+// step later, can_defer_eval) pipelined wins or ties on every config
+// (profiles/r02_schedules_deferred.jsonl, pipelined / serial ms per step):
+// T 0.036 / 0.052, P 0.107 / 0.132, O 0.633 / 0.677, R k = 5 0.696 / 0.768,
+// S 5.49 / 5.54, R k = 50 6.149 / 6.139; the size rule (measured before it,
+// comment above) stays for handles
+// whose rounding cannot be deferred (damped rounding, pointer rounds, B-side
+// proposers).
 static int default_schedule(cualign_bp *h)
 {
+    if (can_defer_eval(h)) return 1;
     const int64_t s = h->s_total ? h->s_total : h->s;
     const int64_t m = h->L.m > 0 ? h->L.m : 1;
     if (s < 10000000) return 1;
