@@ -539,9 +539,13 @@ constexpr size_t square_pk_smem()
 }
 
 // PROBE (timing probes of the probe build only, wrong results): bit 0 = no
-// F-sum atomics, bit 1 = no u_f gathers (u_e used instead)
+// F-sum atomics, bit 1 = no u_f gathers (u_e used instead).
+// 48 registers (was 51): 4 CTAs per SM then leave 10 K registers, room for
+// one 128-thread block of the rounding's chain form (k_suitor_q) beside the
+// square pass in the pipelined step instead of after it (bench window on O:
+// 1504-1509 -> 1520-1521 it/s; no spills).
 template <class V, int PROBE = 0>
-__global__ void __launch_bounds__((SQT_CWARPS + 1) * 32)
+__global__ void __maxnreg__(48)
 k_square_pk(int64_t c0, int64_t c1, const int4 *__restrict__ desc, const uint32_t *__restrict__ words,
             V *__restrict__ sq_val, const double *__restrict__ u, double beta, const double2 *__restrict__ gh,
             const int *__restrict__ p_dev, double fp_scale, unsigned long long *__restrict__ tacc)
