@@ -282,11 +282,24 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
             // in the round's own graph: 1469).  Probe build:
             // CUALIGN_PIPE_EVAL_MAIN=0 takes the third stream.
             static const bool eval_main = probe_knob("CUALIGN_PIPE_EVAL_MAIN", 1) != 0;
-            cudaStream_t es = eval_main ? h->gstream : h->gstream3;
+            // probe build: CUALIGN_PIPE_EVAL_LATE=1 starts the evaluate on the
+            // third stream after k_top2, beside the square pass
+            static const bool eval_late = probe_knob("CUALIGN_PIPE_EVAL_LATE", 0) != 0;
+            cudaStream_t es = (eval_main && !eval_late) ? h->gstream : h->gstream3;
             if (cudaEventRecord(h->fork_ev[0], h->gstream) != cudaSuccess ||
                 cudaStreamWaitEvent(h->gstream2, h->fork_ev[0], 0) != cudaSuccess ||
-                (with_eval && !eval_main && cudaStreamWaitEvent(h->gstream3, h->fork_ev[0], 0) != cudaSuccess))
+                (with_eval && !eval_main && !eval_late &&
+                 cudaStreamWaitEvent(h->gstream3, h->fork_ev[0], 0) != cudaSuccess))
                 st = CUALIGN_ECUDA;
+            if (st == CUALIGN_OK && with_eval && eval_late) {
+                // iteration front first; the evaluate forks after k_top2
+                h->yc = yb[wb];
+                h->zc = zb[wb];
+                st = bp_iterate_front(h);
+                if (st == CUALIGN_OK && (cudaEventRecord(h->join3_ev, h->gstream) != cudaSuccess ||
+                                         cudaStreamWaitEvent(h->gstream3, h->join3_ev, 0) != cudaSuccess))
+                    st = CUALIGN_ECUDA;
+            }
             if (st == CUALIGN_OK && with_eval) {
                 h->stream = es;
                 st = eval_of(wb); // round p-2 read buffer wb
@@ -300,11 +313,16 @@ static cualign_status capture_pipelined(cualign_bp *h, int kind, int wb)
             }
             h->yc = yb[wb];
             h->zc = zb[wb];
-            if (st == CUALIGN_OK) st = bp_iterate(h, 1);
+            if (st == CUALIGN_OK && with_eval && eval_late) {
+                st = bp_iterate_back(h);
+                if (st == CUALIGN_OK) h->p += 1;
+            } else if (st == CUALIGN_OK) {
+                st = bp_iterate(h, 1);
+            }
             if (st == CUALIGN_OK && (cudaEventRecord(h->fork_ev[1], h->gstream2) != cudaSuccess ||
                                      cudaStreamWaitEvent(h->gstream, h->fork_ev[1], 0) != cudaSuccess))
                 st = CUALIGN_ECUDA;
-            if (st == CUALIGN_OK && with_eval && !eval_main &&
+            if (st == CUALIGN_OK && with_eval && (!eval_main || eval_late) &&
                 (cudaEventRecord(h->join3_ev, h->gstream3) != cudaSuccess ||
                  cudaStreamWaitEvent(h->gstream, h->join3_ev, 0) != cudaSuccess))
                 st = CUALIGN_ECUDA;

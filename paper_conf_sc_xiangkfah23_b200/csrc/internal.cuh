@@ -370,6 +370,7 @@ cualign_status ensure_csr(cualign_bp *h);
 cualign_status tile_squares(cualign_bp *h);
 constexpr int SQ_TILE_LOG = 21; // square tiles: blocks of 2^21 edges (2 x 32 MB of u + tacc per tile)
 cualign_status pack_squares(cualign_bp *h); // packed square stream from sq_ef (after every reorder)
+constexpr int EVAL_BS = 128;                // k_eval block size (match.cu)
 constexpr int SQP_CHUNK = 512;              // squares per packed chunk (= square-pass stage)
 constexpr int SQP_FBITS = 21;               // f - fb in the low bits (f blocks of 2^21 = the tile blocks)
 constexpr int SQP_EBITS = 32 - SQP_FBITS;   // e - eb in the high bits

@@ -70,6 +70,9 @@ struct MatchParams {
 };
 
 constexpr int WORK_SPREAD = 64, WORK_STRIDE = 16; // counter slots, 128 B apart
+// evaluate blocks of 128 threads in every schedule (the weight sums' block
+// partition must not depend on the schedule): small enough for a block to
+// fit beside the 48-register square pass's 4 CTAs per SM
 constexpr int NQ = 64;          // Suitor-round sub-queues (one atomic counter each, 32 B apart)
 constexpr int QSTRIDE = 8;
 constexpr int SUITOR_ROUNDS_MAXDEG = 64; // proposal rounds scan a proposer's row in one thread
@@ -926,7 +929,7 @@ __device__ void round_final_block(const EvalParams &P, const int32_t *mateA, int
 // (arrival counter in RoundDev, reset by the final block after every block
 // has left it) separates the two instead of a kernel boundary.
 template <bool COLLECT>
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(EVAL_BS)
 k_eval(EvalParams P, int exact, double alpha, double beta, const int *p_dev, unsigned long long *work,
        MatchParams M, int64_t nT, int64_t nP, int fromB)
 {
@@ -1272,16 +1275,16 @@ cualign_status match_setup(cualign_bp *h)
     {
         // one wave of k_eval (every block resident at once)
         int occ = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_eval<false>, 256, 0) != cudaSuccess || occ < 1)
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_eval<false>, EVAL_BS, 0) != cudaSuccess || occ < 1)
             occ = 1;
         (void)cudaGetLastError();
-        h->eval_grid = grid_for(h->nApairs > (int64_t)nA ? h->nApairs : (int64_t)nA, 256, h->num_sms * occ);
+        h->eval_grid = grid_for(h->nApairs > (int64_t)nA ? h->nApairs : (int64_t)nA, EVAL_BS, h->num_sms * occ);
         // k_eval<true> holds a grid barrier: exactly one wave of its own occupancy
         int occc = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occc, k_eval<true>, 256, 0) != cudaSuccess || occc < 1)
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occc, k_eval<true>, EVAL_BS, 0) != cudaSuccess || occc < 1)
             occc = 1;
         (void)cudaGetLastError();
-        h->evalc_grid = grid_for(std::max<int64_t>(std::max<int64_t>(h->nApairs, (int64_t)nA), 2 * (int64_t)nmax), 256,
+        h->evalc_grid = grid_for(std::max<int64_t>(std::max<int64_t>(h->nApairs, (int64_t)nA), 2 * (int64_t)nmax), EVAL_BS,
                                  h->num_sms * occc);
     }
     CA_TRY(dalloc(h, &h->partial_w, (size_t)2 * std::max(h->eval_grid, h->evalc_grid)));
@@ -1360,7 +1363,7 @@ cualign_status eval_round_deferred(cualign_bp *h, int set)
     KScope ks(h, CUALIGN_K_EVAL);
     const int exact = (h->flags & CUALIGN_FLAG_EXACT) ? 1 : 0;
     const int *pd = (const int *)(h->round_p ? h->round_p : h->p_dev);
-    CA_CUDA(launch_pdl(k_eval<false>, dim3(h->evalc_grid), dim3(256), 0, h->stream, E, exact, h->alpha, h->beta, pd,
+    CA_CUDA(launch_pdl(k_eval<false>, dim3(h->evalc_grid), dim3(EVAL_BS), 0, h->stream, E, exact, h->alpha, h->beta, pd,
                        h->match_work + (int64_t)set * WORK_SPREAD * WORK_STRIDE, MatchParams{}, (int64_t)0,
                        (int64_t)0, 0));
     CA_CUDA(cudaGetLastError());
@@ -1534,10 +1537,10 @@ static cualign_status evaluate_impl(cualign_bp *h, const MatchParams *Pc)
         if (Pc) {
             const bool fromB = Pc->propose_from_b != 0;
             const int64_t nT = fromB ? h->L.nA : h->L.nB, nP = fromB ? h->L.nB : h->L.nA;
-            CA_CUDA(launch_pdl(k_eval<true>, dim3(h->evalc_grid), dim3(256), 0, h->stream, E, exact, h->alpha,
+            CA_CUDA(launch_pdl(k_eval<true>, dim3(h->evalc_grid), dim3(EVAL_BS), 0, h->stream, E, exact, h->alpha,
                                h->beta, pd, h->match_work, *Pc, nT, nP, fromB ? 1 : 0));
         } else {
-            CA_CUDA(launch_pdl(k_eval<false>, dim3(h->eval_grid), dim3(256), 0, h->stream, E, exact, h->alpha,
+            CA_CUDA(launch_pdl(k_eval<false>, dim3(h->eval_grid), dim3(EVAL_BS), 0, h->stream, E, exact, h->alpha,
                                h->beta, pd, h->match_work, MatchParams{}, (int64_t)0, (int64_t)0, 0));
         }
         CA_CUDA(cudaGetLastError());
